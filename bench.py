@@ -1,0 +1,364 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 CART hot path (BASELINE.json metric: tree-fit row.feature split
+evals/s and DSE predictions/s).
+
+Workload (N=1): BASELINE.json configs[1] -- 1M rows x 16 features (schema S16, seed 1),
+max_depth 12, min_samples_leaf 1; one step = dt_fit on the training table + fused
+dt_predict_eval on a 1M-row held-out table (seed 2).  value = split evals / step time
+(split evals = sum over searched nodes of N*d).  Inputs are resident in HBM; L2 is
+flushed (256 MB write) between timed steps, outside the per-step CUDA events.
+N>1 (torchrun): every rank fits its own replica table (seed 1 + rank): "replicas only",
+weak scaling, no data-path collective (Multi-GPU); max over ranks.
+
+Also reported: e2e (same metric through the C-ABI with host buffers, H2D/D2H inside the
+timed region), DSE predictions/s (BASELINE configs[3] shape on one GPU: 2^28 candidates
+by default, depth-20 / min_samples_leaf-128 tree), the dominant kernel's roofline, and
+the oracle timed on the host as cpu_baseline.
+
+--impl reference: the oracle (the slow CPU reference of this tier) timed on the host.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "tree-fit row·feature split evals/s and DSE predictions/s at 1/2/4/8 B200"
+N_TRAIN = 1_000_000
+D = 16
+MAX_DEPTH = 12
+MIN_LEAF = 1
+CPU_SAMPLE_ROWS = 250_000
+REF_SAMPLE_ROWS = 100_000
+FALLBACK_HBM_GBS = 6650.0
+
+REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+           0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+           0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+           0x100: "display_clocks_setting"}
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=50)
+    p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--dse-log2", type=int, default=28, help="log2 of DSE candidates (30 = full C4)")
+    p.add_argument("--no-dse", action="store_true")
+    p.add_argument("--no-cpu", action="store_true")
+    p.add_argument("--e2e-steps", type=int, default=10)
+    return p.parse_args()
+
+
+def workload_config(world):
+    return {"workload": "configs[1]: 1M x 16 (S16 CNN x GPU table, seed 1), max_depth 12, "
+                        "min_samples_leaf 1; step = dt_fit + dt_predict_eval on 1M held-out rows",
+            "n_train": N_TRAIN, "n_eval": N_TRAIN, "d": D, "max_depth": MAX_DEPTH,
+            "min_samples_leaf": MIN_LEAF, "l2": "flushed (256 MB write) between timed steps",
+            "parallelism": "replicas" if world > 1 else "single", "ranks": world}
+
+
+def peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as fh:
+            return float(json.load(fh)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """NVML sampling of SM clock and clock-event reasons during the timed region."""
+
+    def __init__(self, index=0, period=0.01):
+        self.index, self.period = index, period
+        self.samples, self.reasons = [], 0
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._t = None
+
+    def __enter__(self):
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+
+            def run():
+                while not self._stop.is_set():
+                    try:
+                        self.samples.append(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM))
+                        self.reasons |= int(pynvml.nvmlDeviceGetCurrentClocksEventReasons(h))
+                    except Exception:
+                        pass
+                    time.sleep(self.period)
+
+            self._t = threading.Thread(target=run, daemon=True)
+            self._t.start()
+        except Exception:
+            self._t = None
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        names = [v for k, v in REASONS.items() if self.reasons & k and v != "gpu_idle"]
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": names, "samples": len(self.samples)}
+
+
+def dist_init():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl")
+    return world, rank, local
+
+
+def max_over_ranks(x, world):
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def sum_over_ranks(x, world):
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return float(t.item())
+
+
+def barrier(world):
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+# ---------------------------------------------------------------------- oracle (CPU) --
+
+def oracle_rate(rows: int, seed: int = 1):
+    """Oracle fit on the first `rows` rows of the workload table; returns (evals/s, s, evals)."""
+    import datagen
+    import oracle
+    X, y = datagen.cnn_gpu_table(seed, rows)
+    t0 = time.perf_counter()
+    _, ev = oracle.fit(X, y, MAX_DEPTH, MIN_LEAF, return_evals=True)
+    dt = time.perf_counter() - t0
+    return ev / dt, dt, ev
+
+
+def run_reference(args, world, rank):
+    if rank != 0:
+        return
+    import datagen
+    import oracle
+    oracle.build()
+    X, y = datagen.cnn_gpu_table(1, REF_SAMPLE_ROWS)
+    for _ in range(args.warmup):
+        oracle.fit(X, y, MAX_DEPTH, MIN_LEAF)
+    t0 = time.perf_counter()
+    ev_tot = 0
+    for _ in range(args.steps):
+        _, ev = oracle.fit(X, y, MAX_DEPTH, MIN_LEAF, return_evals=True)
+        ev_tot += ev
+    dt = time.perf_counter() - t0
+    v = ev_tot / dt
+    sample = (f"oracle fit (single-threaded C, -O2) on the first {REF_SAMPLE_ROWS} rows of the "
+              f"configs[1] table (seed 1), depth {MAX_DEPTH}; per step")
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "split evals/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": dt / args.steps * 1e3, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": workload_config(1),
+            "cpu_baseline": {"value": v, "unit": "split evals/s", "cores": 1, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": v, "unit": "split evals/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------------- ours (GPU) ----
+
+def run_ours(args, world, rank, local):
+    import torch
+
+    import paper_conf_ipps_metzgd23_b200 as dt
+
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    stream = torch.cuda.current_stream()
+    # inputs resident in HBM (device generator, bit-identical to datagen)
+    X, y = dt.dt_gen_table(1 + rank, N_TRAIN, d=D, device=dev)
+    Xv, yv = dt.dt_gen_table(2 + 1000 * rank, N_TRAIN, d=D, device=dev)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    torch.cuda.synchronize()
+
+    def step():
+        tree = dt.dt_fit(X, y, MAX_DEPTH, MIN_LEAF)
+        m = dt.dt_predict_eval(tree, Xv, yv, D)
+        return tree, m
+
+    for _ in range(args.warmup):
+        tree, m = step()
+    ev0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ev1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    dt.dt_profile_reset()
+    dt.dt_profile_enable(True)
+    launches0 = dt.dt_launch_count()
+    evals = 0
+    with ClockSampler(local) as clk:
+        barrier(world)
+        torch.cuda.synchronize()
+        for i in range(args.steps):
+            flush.zero_()
+            ev0[i].record(stream)
+            tree, m = step()
+            ev1[i].record(stream)
+            evals += tree.split_evals
+        torch.cuda.synchronize()
+        barrier(world)
+    dt.dt_profile_enable(False)
+    launches = dt.dt_launch_count() - launches0
+    ms = [a.elapsed_time(b) for a, b in zip(ev0, ev1)]
+    t_total = sum(ms) / 1e3
+    t_max = max_over_ranks(t_total, world)
+    evals_all = sum_over_ranks(float(evals), world)
+    value = evals_all / t_max
+    prof = dt.dt_profile()
+
+    # roofline of the dominant kernel (largest device time inside the timed steps)
+    peak, peak_src = peaks()
+    fit_kinds = {k: v for k, v in prof.items() if v["alg_bytes"] > 0}
+    dom = max(fit_kinds, key=lambda k: fit_kinds[k]["ms"])
+    d_ms = fit_kinds[dom]["ms"]
+    achieved = fit_kinds[dom]["alg_bytes"] / (d_ms / 1e3) / 1e9
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        with open(tpath) as fh:
+            traffic = json.load(fh).get(dom)
+    step_ms = sum(ms) / len(ms)
+    share = {k: round(v["ms"] / sum(ms), 4) for k, v in prof.items()}
+    roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "peak_source": peak_src,
+                "alg_bytes_per_launch": fit_kinds[dom]["alg_bytes"] / fit_kinds[dom]["launches"],
+                "avg_launch_ms": d_ms / fit_kinds[dom]["launches"], "traffic": traffic}
+
+    # ---- e2e: through the C ABI with host buffers (pinned), H2D + D2H inside the region
+    Xh, yh = X.cpu().pin_memory(), y.cpu().pin_memory()
+    Xvh, yvh = Xv.cpu().pin_memory(), yv.cpu().pin_memory()
+    Xd, yd = torch.empty_like(X), torch.empty_like(y)
+    Xvd, yvd = torch.empty_like(Xv), torch.empty_like(yv)
+    h2d = 0
+    d2h = 0
+    e_evals = 0
+    torch.cuda.synchronize()
+    barrier(world)
+    t0 = time.perf_counter()
+    for _ in range(args.e2e_steps):
+        Xd.copy_(Xh, non_blocking=True)
+        yd.copy_(yh, non_blocking=True)
+        Xvd.copy_(Xvh, non_blocking=True)
+        yvd.copy_(yvh, non_blocking=True)
+        tr = dt.dt_fit(Xd, yd, MAX_DEPTH, MIN_LEAF)   # returns the node array on the host
+        mm = dt.dt_predict_eval(tr, Xvd, yvd, D)      # metrics to the host
+        e_evals += tr.split_evals
+        h2d = sum(t.numel() * t.element_size() for t in (Xh, yh, Xvh, yvh))
+        d2h = tr.size * 48 + 24
+    torch.cuda.synchronize()
+    e2e_t = max_over_ranks(time.perf_counter() - t0, world)
+    e2e_value = sum_over_ranks(float(e_evals), world) / e2e_t
+
+    # ---- DSE predictions/s (configs[3] shape on one GPU)
+    dse = None
+    if not args.no_dse:
+        nd = 1 << args.dse_log2
+        Xdse = dt.dt_gen_dse(3 + rank, 0, nd, 10, device=dev)
+        tdse = dt.dt_fit(X, y, 20, 128)
+        out = torch.empty(nd, dtype=torch.float64, device=dev)
+        for _ in range(3):
+            dt.dt_predict(tdse, Xdse, out=out)
+        reps = 5
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        dt.dt_profile_reset()
+        dt.dt_profile_enable(True)
+        torch.cuda.synchronize()
+        a.record(stream)
+        for _ in range(reps):
+            dt.dt_predict(tdse, Xdse, out=out)
+        b.record(stream)
+        torch.cuda.synchronize()
+        dt.dt_profile_enable(False)
+        pp = dt.dt_profile().get("predict")
+        t = a.elapsed_time(b) / 1e3
+        tmax = max_over_ranks(t, world)
+        preds = sum_over_ranks(float(nd * reps), world) / tmax
+        pach = pp["alg_bytes"] / (pp["ms"] / 1e3) / 1e9
+        dse = {"predictions_per_s": preds, "candidates_per_rank": nd, "tree_nodes": tdse.size,
+               "tree_depth": tdse.depth, "ms_per_pass": t / reps * 1e3,
+               "roofline": {"bound": "hbm", "kernel": "predict", "achieved": pach, "peak": peak,
+                            "unit": "GB/s", "frac": pach / peak,
+                            "alg_bytes_per_launch": pp["alg_bytes"] / pp["launches"]}}
+        del Xdse, out
+
+    # ---- CPU baseline: the oracle on the host (rank 0, N=1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        rate, secs, ev = oracle_rate(CPU_SAMPLE_ROWS)
+        cpu = {"value": rate, "unit": "split evals/s", "cores": 1, "kind": "oracle",
+               "sample": f"oracle fit on the first {CPU_SAMPLE_ROWS} of the {N_TRAIN} rows "
+                         f"(seed 1), depth {MAX_DEPTH}: {ev} split evals in {secs:.1f} s"}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "split evals/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": step_ms,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "dtype": "f64", "data": "synthetic", "config": workload_config(world),
+                "e2e": {"value": e2e_value, "unit": "split evals/s", "h2d_bytes_per_step": h2d,
+                        "d2h_bytes_per_step": d2h, "steps": args.e2e_steps},
+                "gpu_launches": launches,
+                "roofline": roofline, "cpu_baseline": cpu, "dse": dse,
+                "clocks": clk.summary(),
+                "fit": {"split_evals_per_step": evals // args.steps, "tree_nodes": tree.size,
+                        "tree_depth": tree.depth, "eval_mape": m["mape"], "eval_r2": m["r2"],
+                        "kernel_share_of_step": share,
+                        "kernel_ms_per_step": {k: v["ms"] / args.steps for k, v in prof.items()}}}
+        print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    world, rank, local = dist_init()
+    if args.impl == "reference":
+        run_reference(args, world, rank)
+    else:
+        run_ours(args, world, rank, local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,185 @@
+/*
+ * include/dt.h -- C ABI of the B200-native CART hot path (libdt.so).
+ *
+ * The operations are those of the paper's predictive model (PM): a Decision-Tree
+ * regressor trained on rows d = (y, p, c_1..c_m, t) (Eq. 1; "Decision
+ * Tree regression"), used to estimate performance for many
+ * (CNN, GPU) candidates in a design-space exploration (T_est = t_dca + n*t_pm,
+ * PAPER.md:245-247), and judged by MAPE, R^2 and adjusted R^2 (Table II
+ * :211-217).  The paper fixes no hyper-parameter, tie rule or threshold rule; the
+ * readings used here are listed in DESIGN.md ("Readings", R1-R19).
+ *
+ * Conventions (all calls):
+ *  - Every call returns dt_status; DT_OK == 0.  On error, dt_last_error() returns a
+ *    thread-local message.  Arguments are validated before any launch.
+ *  - *_dev arguments are CUDA device pointers owned by the caller (e.g. torch tensors);
+ *    the library never frees caller memory.  *_host arguments are host pointers.
+ *  - X is n x d float32 ROW-MAJOR (row r, feature f at X[r*d + f]); y and yhat are
+ *    float64.  1 <= d <= 255.  Non-finite X or y -> DT_ERR_NONFINITE.
+ *  - `stream` is a cudaStream_t (0 = legacy default stream).  Calls documented "async"
+ *    enqueue work and return; calls documented "sync" synchronise `stream` first.
+ *  - A sticky CUDA error returns DT_ERR_CUDA; the process must then re-initialise.
+ *  - Distinct dt_tree objects are independent and may be used from different threads.
+ */
+#ifndef DT_H_
+#define DT_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  DT_OK = 0,
+  DT_ERR_INVALID_ARG = 1,
+  DT_ERR_NONFINITE = 2,
+  DT_ERR_OOM = 3,
+  DT_ERR_CUDA = 4,
+  DT_ERR_NCCL = 5,
+  DT_ERR_TOO_LARGE = 6
+} dt_status;
+
+/* One tree node, 48 bytes, nodes in BFS order (node 0 = root; a level's nodes in index
+ * order; a split appends left then right, so right == left + 1) -- Reading R9. */
+typedef struct {
+  int32_t feature;   /* split feature, -1 for a leaf                                    */
+  int32_t left;      /* left child index, -1 for a leaf                                 */
+  int32_t right;     /* right child index (== left + 1), -1 for a leaf                  */
+  int32_t depth;     /* root = 0                                                        */
+  double threshold;  /* go left iff (double)x[feature] <= threshold; 0.0 for leaves     */
+  double value;      /* mean of y over the node's training rows (every node)            */
+  double impurity;   /* SSE / n_samples of the node's training rows                     */
+  int64_t n_samples; /* training rows in the node                                       */
+} dt_node;
+
+typedef struct dt_tree dt_tree; /* opaque: owns a host copy and a device copy of the nodes */
+
+/* Accuracy metrics of Table II.  mape is a fraction (x100 for %),
+ * MAPE = mean |y - yhat| / max(|y|, DBL_EPSILON) (Reading R12); r2 = 1 - SSE/SST,
+ * unclamped, with r2 = (SSE == 0 ? 1 : 0) when SST == 0 (R13); adj_r2 =
+ * 1 - (1 - r2)(n - 1)/(n - p - 1), NaN when n - p - 1 <= 0 (R14). */
+typedef struct {
+  double mape;
+  double r2;
+  double adj_r2;
+  int64_t n;
+  int32_t p;
+} dt_metrics;
+
+/* ------------------------------------------------------------------ fit ----------- */
+
+/* dt_fit -- greedy CART regression (squared-error / variance reduction), exhaustive over
+ * every feature and every threshold at every node (Readings R1-R10).
+ *   X_dev  n x d f32 row-major, y_dev n f64 (device).  1 <= n < 2^32.
+ *   max_depth: -1 = unlimited, 0 = a single root leaf.
+ *   min_samples_leaf >= 1 (min_samples_split is 2 * min_samples_leaf, R2).
+ * Split rule: for feature f and the node's rows ordered by (x_f, row id), position i
+ * (first i rows left) is valid iff x[i-1] < x[i] and both children keep >=
+ * min_samples_leaf rows; the gain (S'_L n_R - S'_R n_L)^2 / (N n_L n_R) of the
+ * per-node-centered sums is maximised; ties go to the lowest feature, then the lowest
+ * threshold; threshold = x[i-1]/2 + x[i]/2 in fp64 (R4, R5, R19).  A node is a leaf if
+ * depth == max_depth, N < 2*min_samples_leaf, all its y are equal, or no position is
+ * valid (R8).
+ * Sync: returns once the tree is complete; *out is owned by the caller (dt_tree_free).
+ * Errors: INVALID_ARG (n, d, max_depth, min_samples_leaf, null pointers), NONFINITE,
+ * TOO_LARGE (n >= 2^32 or workspace beyond device memory), OOM, CUDA. */
+dt_status dt_fit(const float* X_dev, const double* y_dev, int64_t n, int32_t d,
+                 int32_t max_depth, int64_t min_samples_leaf, void* stream, dt_tree** out);
+
+/* Number of nodes; host view of the node array (valid until dt_tree_free). */
+int64_t dt_tree_size(const dt_tree* tree);
+const dt_node* dt_tree_nodes(const dt_tree* tree);
+/* Realised depth (max node depth), the number of features the tree was fitted on, and
+ * the split-eval count of the fit that produced it: sum over searched nodes (nodes not
+ * made leaves by the depth / size / purity rules) of N*d -- the numerator of the
+ * headline metric "row.feature split evals/s" (BASELINE.json).  Trees made
+ * by dt_tree_from_nodes report 0 split evals. */
+int32_t dt_tree_depth(const dt_tree* tree);
+int32_t dt_tree_num_features(const dt_tree* tree);
+int64_t dt_tree_split_evals(const dt_tree* tree);
+
+/* Build a tree from a caller-supplied node array (e.g. a saved model or the oracle's
+ * output).  Validates BFS links (right == left + 1, children after parent, depth =
+ * parent depth + 1, every non-root node referenced once), 0 <= feature < d for internal
+ * nodes, finite thresholds and values.  Copies the nodes; sync. */
+dt_status dt_tree_from_nodes(const dt_node* nodes_host, int64_t count, int32_t d,
+                             dt_tree** out);
+void dt_tree_free(dt_tree* tree);
+
+/* ------------------------------------------------------------------ predict ------- */
+
+/* dt_predict -- the PM's estimate for every candidate row: from the
+ * root go left iff (double)x[feature] <= threshold until a leaf; yhat = leaf value.
+ * X_dev n x d f32 row-major (d must equal the tree's d), yhat_dev n f64.  n >= 0 (n == 0
+ * is a no-op), n < 2^62.  Async on stream. */
+dt_status dt_predict(const dt_tree* tree, const float* X_dev, int64_t n, int32_t d,
+                     double* yhat_dev, void* stream);
+
+/* ------------------------------------------------------------------ eval ---------- */
+
+/* dt_eval -- MAPE, R^2, adjusted R^2 of yhat against y (Table II).
+ * n >= 1, p >= 0 (number of predictors for adj-R^2).  Sync: returns the metrics in *out. */
+dt_status dt_eval(const double* y_dev, const double* yhat_dev, int64_t n, int32_t p,
+                  void* stream, dt_metrics* out);
+
+/* dt_predict_eval -- held-out evaluation fused into prediction (no yhat round trip):
+ * metrics of dt_predict(tree, X) against y.  Sync. */
+dt_status dt_predict_eval(const dt_tree* tree, const float* X_dev, const double* y_dev,
+                          int64_t n, int32_t d, int32_t p, void* stream, dt_metrics* out);
+
+/* ------------------------------------------------------------------ LOO ----------- */
+
+/* dt_loo -- leave-one-out refits (BASELINE configs[0]; the paper's 70/30 split, P:197,
+ * has no seed, Reading R11): for every i, fit on the other n-1 rows (original relative
+ * order) with (max_depth, min_samples_leaf) and predict row i into yhat_oof_dev[i].
+ * Each fold is an independent CART exactly as dt_fit would build it.  2 <= n <= 64 and
+ * d <= 32 (one fold per CTA, everything in shared memory); larger inputs -> TOO_LARGE.
+ * Async on stream. */
+dt_status dt_loo(const float* X_dev, const double* y_dev, int64_t n, int32_t d,
+                 int32_t max_depth, int64_t min_samples_leaf, double* yhat_oof_dev,
+                 void* stream);
+
+/* ------------------------------------------------------------------ generator ----- */
+
+/* dt_gen_table -- synthetic feature table shaped like Eq. 1: rows
+ * [row0, row0 + n) of the seeded (CNN, GPU) table, schema S16 (d = 16) or S32 (d = 32),
+ * bit-identical to datagen.cnn_gpu_table (recipe in DESIGN.md, "Input recipe").
+ * y_dev may be NULL (features only).  real != 0 -> real-valued target, else integer us.
+ * cnn_pool_bits / gpu_pool_bits: pool sizes 2^bits.  unit_us: target unit.  Async. */
+dt_status dt_gen_table(uint64_t seed, int64_t row0, int64_t n, int32_t d, int32_t real,
+                       int32_t cnn_pool_bits, int32_t gpu_pool_bits, double unit_us,
+                       float* X_dev, double* y_dev, void* stream);
+
+/* dt_gen_dse -- DSE candidates (BASELINE configs[3]): candidate r is the cross product
+ * entry (cnn = r >> gpu_bits, gpu = r & (2^gpu_bits - 1)), S16 features only,
+ * bit-identical to datagen.dse_candidates.  Async. */
+dt_status dt_gen_dse(uint64_t seed, int64_t row0, int64_t n, int32_t gpu_bits,
+                     float* X_dev, void* stream);
+
+/* ------------------------------------------------------------------ profiling ----- */
+
+/* Measurement hooks used by bench.py (not needed to use the library).  While enabled,
+ * every library call records a CUDA event pair on its stream around each kernel it
+ * launches, tagged with the kernel kind and the launch's ALGORITHMIC bytes (DESIGN.md,
+ * "Roofline"); dt_profile_get synchronises those events and returns, for one kind, the
+ * number of launches, the summed device time (ms) and the summed algorithmic bytes.
+ * dt_launch_count counts this library's own kernel launches (library kernels such as
+ * the CUB radix sort inside the presort are not counted) since the last reset. */
+void dt_profile_enable(int on);
+void dt_profile_reset(void);
+int64_t dt_launch_count(void);
+int32_t dt_profile_kinds(void);
+dt_status dt_profile_get(int32_t kind, const char** name, int64_t* launches, double* ms,
+                         double* alg_bytes);
+
+/* ------------------------------------------------------------------ misc ---------- */
+
+const char* dt_last_error(void);
+/* Library build identification, e.g. "libdt sm_100a". */
+const char* dt_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DT_H_ */

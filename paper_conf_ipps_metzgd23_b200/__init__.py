@@ -1,0 +1,266 @@
+"""B200-native exact CART (Metz, Goli & Drechsler, IPDPS'23 -- the Decision-Tree
+performance model): thin Python binding over the C ABI of ``libdt.so``
+(``include/dt.h``).
+
+Argument marshalling only: every step runs in the CUDA kernels of ``libdt.so``.  Tensors
+are torch CUDA tensors (X float32 n x d row-major contiguous, y float64); the work is
+enqueued on torch's current stream.  There is no CPU fallback: importing this package
+without a built ``libdt.so`` raises, and every call raises ``DTError`` on failure.
+
+Names follow the C ABI: ``dt_fit``, ``dt_predict``, ``dt_eval``, ``dt_predict_eval``,
+``dt_loo``, ``dt_gen_table``, ``dt_gen_dse``; ``Tree`` wraps ``dt_tree*``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libdt.so")
+
+NODE_DTYPE = np.dtype([
+    ("feature", "<i4"), ("left", "<i4"), ("right", "<i4"), ("depth", "<i4"),
+    ("threshold", "<f8"), ("value", "<f8"), ("impurity", "<f8"), ("n_samples", "<i8"),
+])
+
+STATUS = {0: "DT_OK", 1: "DT_ERR_INVALID_ARG", 2: "DT_ERR_NONFINITE", 3: "DT_ERR_OOM",
+          4: "DT_ERR_CUDA", 5: "DT_ERR_NCCL", 6: "DT_ERR_TOO_LARGE"}
+
+SYMBOLS = ("dt_fit", "dt_tree_size", "dt_tree_nodes", "dt_tree_depth", "dt_tree_num_features",
+           "dt_tree_split_evals", "dt_tree_from_nodes", "dt_tree_free", "dt_predict", "dt_eval",
+           "dt_predict_eval", "dt_loo", "dt_gen_table", "dt_gen_dse", "dt_last_error",
+           "dt_version", "dt_profile_enable", "dt_profile_reset", "dt_launch_count",
+           "dt_profile_kinds", "dt_profile_get")
+
+
+class DTError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class dt_metrics(ctypes.Structure):
+    _fields_ = [("mape", ctypes.c_double), ("r2", ctypes.c_double), ("adj_r2", ctypes.c_double),
+                ("n", ctypes.c_int64), ("p", ctypes.c_int32)]
+
+
+def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
+    """Load libdt.so and declare the C signatures.  Raises if the library is missing."""
+    if not os.path.exists(path):
+        raise ImportError(f"{path} not built: run `python -c 'import __graft_entry__ as g; g.build()'`")
+    lib = ctypes.CDLL(path)
+    P, I64, I32, U64, D = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, ctypes.c_double
+    sig = {
+        "dt_fit": ([P, P, I64, I32, I32, I64, P, ctypes.POINTER(P)], ctypes.c_int),
+        "dt_tree_size": ([P], I64),
+        "dt_tree_nodes": ([P], P),
+        "dt_tree_depth": ([P], I32),
+        "dt_tree_num_features": ([P], I32),
+        "dt_tree_split_evals": ([P], I64),
+        "dt_tree_from_nodes": ([P, I64, I32, ctypes.POINTER(P)], ctypes.c_int),
+        "dt_tree_free": ([P], None),
+        "dt_predict": ([P, P, I64, I32, P, P], ctypes.c_int),
+        "dt_eval": ([P, P, I64, I32, P, ctypes.POINTER(dt_metrics)], ctypes.c_int),
+        "dt_predict_eval": ([P, P, P, I64, I32, I32, P, ctypes.POINTER(dt_metrics)], ctypes.c_int),
+        "dt_loo": ([P, P, I64, I32, I32, I64, P, P], ctypes.c_int),
+        "dt_gen_table": ([U64, I64, I64, I32, I32, I32, I32, D, P, P, P], ctypes.c_int),
+        "dt_gen_dse": ([U64, I64, I64, I32, P, P], ctypes.c_int),
+        "dt_last_error": ([], ctypes.c_char_p),
+        "dt_version": ([], ctypes.c_char_p),
+        "dt_profile_enable": ([ctypes.c_int], None),
+        "dt_profile_reset": ([], None),
+        "dt_launch_count": ([], I64),
+        "dt_profile_kinds": ([], I32),
+        "dt_profile_get": ([I32, ctypes.POINTER(ctypes.c_char_p), ctypes.POINTER(I64),
+                            ctypes.POINTER(D), ctypes.POINTER(D)], ctypes.c_int),
+    }
+    for name, (args, res) in sig.items():
+        fn = getattr(lib, name)
+        fn.argtypes = args
+        fn.restype = res
+    return lib
+
+
+_lib = load_library()
+
+
+def _check(st: int):
+    if st != 0:
+        raise DTError(st, _lib.dt_last_error().decode())
+
+
+def _stream(stream=None):
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _dev(t, dtype, ndim, name):
+    import torch
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise TypeError(f"{name} must be a CUDA torch.Tensor")
+    if t.dtype != dtype:
+        raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
+    if t.dim() != ndim or not t.is_contiguous():
+        raise ValueError(f"{name} must be a contiguous {ndim}-D tensor")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+class Tree:
+    """Owns a ``dt_tree*``.  ``nodes`` is a numpy structured copy (BFS, 48 B/node)."""
+
+    def __init__(self, handle: ctypes.c_void_p):
+        self._h = handle
+
+    @property
+    def handle(self):
+        return self._h
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h is not None and h.value:
+            _lib.dt_tree_free(h)
+            self._h = None
+
+    @property
+    def size(self) -> int:
+        return int(_lib.dt_tree_size(self._h))
+
+    @property
+    def depth(self) -> int:
+        return int(_lib.dt_tree_depth(self._h))
+
+    @property
+    def num_features(self) -> int:
+        return int(_lib.dt_tree_num_features(self._h))
+
+    @property
+    def split_evals(self) -> int:
+        return int(_lib.dt_tree_split_evals(self._h))
+
+    @property
+    def nodes(self) -> np.ndarray:
+        n = self.size
+        ptr = _lib.dt_tree_nodes(self._h)
+        buf = (ctypes.c_char * (n * NODE_DTYPE.itemsize)).from_address(ptr)
+        return np.frombuffer(bytes(buf), dtype=NODE_DTYPE).copy()
+
+
+def dt_fit(X, y, max_depth: int = -1, min_samples_leaf: int = 1, stream=None) -> Tree:
+    import torch
+    xp = _dev(X, torch.float32, 2, "X")
+    yp = _dev(y, torch.float64, 1, "y")
+    n, d = X.shape
+    if y.shape[0] != n:
+        raise ValueError("y must have n elements")
+    h = ctypes.c_void_p()
+    _check(_lib.dt_fit(xp, yp, n, d, max_depth, min_samples_leaf, _stream(stream), ctypes.byref(h)))
+    return Tree(h)
+
+
+def dt_tree_from_nodes(nodes: np.ndarray, d: int) -> Tree:
+    nodes = np.ascontiguousarray(nodes).astype(NODE_DTYPE, copy=False)
+    h = ctypes.c_void_p()
+    _check(_lib.dt_tree_from_nodes(nodes.ctypes.data, len(nodes), d, ctypes.byref(h)))
+    return Tree(h)
+
+
+def dt_predict(tree: Tree, X, out=None, stream=None):
+    import torch
+    xp = _dev(X, torch.float32, 2, "X")
+    n, d = X.shape
+    if out is None:
+        out = torch.empty(n, dtype=torch.float64, device=X.device)
+    op = _dev(out, torch.float64, 1, "out")
+    _check(_lib.dt_predict(tree.handle, xp, n, d, op, _stream(stream)))
+    return out
+
+
+def _metrics(m: dt_metrics):
+    return dict(mape=m.mape, r2=m.r2, adj_r2=m.adj_r2, n=m.n, p=m.p)
+
+
+def dt_eval(y, yhat, p: int, stream=None) -> dict:
+    import torch
+    yp = _dev(y, torch.float64, 1, "y")
+    hp = _dev(yhat, torch.float64, 1, "yhat")
+    m = dt_metrics()
+    _check(_lib.dt_eval(yp, hp, y.shape[0], p, _stream(stream), ctypes.byref(m)))
+    return _metrics(m)
+
+
+def dt_predict_eval(tree: Tree, X, y, p: int, stream=None) -> dict:
+    import torch
+    xp = _dev(X, torch.float32, 2, "X")
+    yp = _dev(y, torch.float64, 1, "y")
+    m = dt_metrics()
+    _check(_lib.dt_predict_eval(tree.handle, xp, yp, X.shape[0], X.shape[1], p, _stream(stream),
+                                ctypes.byref(m)))
+    return _metrics(m)
+
+
+def dt_loo(X, y, max_depth: int = -1, min_samples_leaf: int = 1, out=None, stream=None):
+    import torch
+    xp = _dev(X, torch.float32, 2, "X")
+    yp = _dev(y, torch.float64, 1, "y")
+    n, d = X.shape
+    if out is None:
+        out = torch.empty(n, dtype=torch.float64, device=X.device)
+    op = _dev(out, torch.float64, 1, "out")
+    _check(_lib.dt_loo(xp, yp, n, d, max_depth, min_samples_leaf, op, _stream(stream)))
+    return out
+
+
+def dt_gen_table(seed: int, n: int, d: int = 16, real: bool = False, row0: int = 0,
+                 cnn_pool_bits: int = 16, gpu_pool_bits: int = 8, unit_us: float = 1.0,
+                 with_y: bool = True, device="cuda", stream=None):
+    import torch
+    X = torch.empty((n, d), dtype=torch.float32, device=device)
+    y = torch.empty(n, dtype=torch.float64, device=device) if with_y else None
+    _check(_lib.dt_gen_table(seed, row0, n, d, int(real), cnn_pool_bits, gpu_pool_bits, unit_us,
+                             ctypes.c_void_p(X.data_ptr()),
+                             ctypes.c_void_p(y.data_ptr() if y is not None else 0), _stream(stream)))
+    return X, y
+
+
+def dt_gen_dse(seed: int, row0: int, n: int, gpu_bits: int = 10, out=None, device="cuda",
+               stream=None):
+    import torch
+    if out is None:
+        out = torch.empty((n, 16), dtype=torch.float32, device=device)
+    _check(_lib.dt_gen_dse(seed, row0, n, gpu_bits, ctypes.c_void_p(out.data_ptr()), _stream(stream)))
+    return out
+
+
+def dt_profile_enable(on: bool = True):
+    _lib.dt_profile_enable(1 if on else 0)
+
+
+def dt_profile_reset():
+    _lib.dt_profile_reset()
+
+
+def dt_launch_count() -> int:
+    return int(_lib.dt_launch_count())
+
+
+def dt_profile() -> dict:
+    """{kind: dict(launches, ms, alg_bytes)} for every kind with >= 1 recorded launch."""
+    out = {}
+    for k in range(int(_lib.dt_profile_kinds())):
+        name = ctypes.c_char_p()
+        cnt = ctypes.c_int64()
+        ms = ctypes.c_double()
+        by = ctypes.c_double()
+        _check(_lib.dt_profile_get(k, ctypes.byref(name), ctypes.byref(cnt), ctypes.byref(ms),
+                                   ctypes.byref(by)))
+        if cnt.value:
+            out[name.value.decode()] = dict(launches=int(cnt.value), ms=float(ms.value),
+                                            alg_bytes=float(by.value))
+    return out
+
+
+def version() -> str:
+    return _lib.dt_version().decode()

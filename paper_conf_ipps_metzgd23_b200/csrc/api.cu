@@ -1,0 +1,220 @@
+// C-ABI shim of libdt: argument validation, status codes, tree objects.
+// Declarations and semantics: include/dt.h.
+#include <math.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <cstdlib>
+#include <string>
+#include <vector>
+
+#include "dt_internal.cuh"
+
+namespace dtl {
+
+static thread_local std::string g_err;
+
+void set_error(const std::string& msg) { g_err = msg; }
+
+dt_status fail(dt_status st, const std::string& msg) {
+  g_err = msg;
+  return st;
+}
+
+dt_status cuda_fail(cudaError_t e, const char* what, const char* file, int line) {
+  char buf[512];
+  snprintf(buf, sizeof buf, "CUDA error %d (%s) in %s at %s:%d", (int)e, cudaGetErrorString(e),
+           what, file, line);
+  g_err = buf;
+  if (e == cudaErrorMemoryAllocation) return DT_ERR_OOM;
+  return DT_ERR_CUDA;
+}
+
+int num_sms() {
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  return sms;
+}
+
+// Packed predict node: x = f32 bits of RD32(threshold) (x <= t  <=>  x <= RD32(t) for f32
+// x, Reading R5), y = feature << 24 | left.  A leaf self-loops (feature 0, +inf, left =
+// self) so every row runs exactly `depth` iterations without divergence on exit.
+dt_status tree_upload(dt_tree* t, cudaStream_t s) {
+  std::vector<uint2> packed((size_t)t->count);
+  std::vector<double> val((size_t)t->count);
+  for (int64_t k = 0; k < t->count; ++k) {
+    const dt_node& nd = t->host[k];
+    val[(size_t)k] = nd.value;
+    if (nd.feature < 0) {
+      float inf = INFINITY;
+      uint32_t bits;
+      memcpy(&bits, &inf, 4);
+      packed[(size_t)k] = make_uint2(bits, (uint32_t)k);
+    } else {
+      // round-down of the fp64 threshold to f32
+      float f = (float)nd.threshold;
+      if ((double)f > nd.threshold) f = nextafterf(f, -INFINITY);
+      uint32_t bits;
+      memcpy(&bits, &f, 4);
+      packed[(size_t)k] = make_uint2(bits, ((uint32_t)nd.feature << 24) | (uint32_t)nd.left);
+    }
+  }
+  DT_CK(cudaGetDevice(&t->device));
+  DT_CK(cudaMalloc(&t->dev_packed, sizeof(uint2) * (size_t)t->count));
+  DT_CK(cudaMalloc(&t->dev_value, sizeof(double) * (size_t)t->count));
+  DT_CK(cudaMemcpyAsync(t->dev_packed, packed.data(), sizeof(uint2) * (size_t)t->count,
+                        cudaMemcpyHostToDevice, s));
+  DT_CK(cudaMemcpyAsync(t->dev_value, val.data(), sizeof(double) * (size_t)t->count,
+                        cudaMemcpyHostToDevice, s));
+  DT_CK(cudaStreamSynchronize(s));
+  return DT_OK;
+}
+
+}  // namespace dtl
+
+using namespace dtl;
+
+static cudaStream_t S(void* p) { return (cudaStream_t)p; }
+
+extern "C" {
+
+const char* dt_last_error(void) { return g_err.c_str(); }
+
+const char* dt_version(void) { return "libdt 0.1 sm_100a"; }
+
+dt_status dt_fit(const float* X_dev, const double* y_dev, int64_t n, int32_t d,
+                 int32_t max_depth, int64_t min_samples_leaf, void* stream, dt_tree** out) {
+  if (!out) return fail(DT_ERR_INVALID_ARG, "dt_fit: out is NULL");
+  *out = nullptr;
+  if (!X_dev || !y_dev) return fail(DT_ERR_INVALID_ARG, "dt_fit: NULL X or y");
+  if (n < 1) return fail(DT_ERR_INVALID_ARG, "dt_fit: n must be >= 1");
+  if (n >= (int64_t)1 << 32) return fail(DT_ERR_TOO_LARGE, "dt_fit: n must be < 2^32");
+  if (d < 1 || d > 255) return fail(DT_ERR_INVALID_ARG, "dt_fit: d must be in [1, 255]");
+  if (max_depth < -1) return fail(DT_ERR_INVALID_ARG, "dt_fit: max_depth must be >= -1");
+  if (min_samples_leaf < 1) return fail(DT_ERR_INVALID_ARG, "dt_fit: min_samples_leaf must be >= 1");
+  return fit_impl(X_dev, y_dev, n, d, max_depth, min_samples_leaf, S(stream), out);
+}
+
+int64_t dt_tree_size(const dt_tree* t) { return t ? t->count : 0; }
+const dt_node* dt_tree_nodes(const dt_tree* t) { return t ? t->host : nullptr; }
+int32_t dt_tree_depth(const dt_tree* t) { return t ? t->depth : 0; }
+int32_t dt_tree_num_features(const dt_tree* t) { return t ? t->d : 0; }
+int64_t dt_tree_split_evals(const dt_tree* t) { return t ? t->split_evals : 0; }
+
+dt_status dt_tree_from_nodes(const dt_node* nodes, int64_t count, int32_t d, dt_tree** out) {
+  if (!out) return fail(DT_ERR_INVALID_ARG, "dt_tree_from_nodes: out is NULL");
+  *out = nullptr;
+  if (!nodes || count < 1) return fail(DT_ERR_INVALID_ARG, "dt_tree_from_nodes: empty");
+  if (d < 1 || d > 255) return fail(DT_ERR_INVALID_ARG, "dt_tree_from_nodes: d must be in [1, 255]");
+  if (count >= (1 << 24)) return fail(DT_ERR_TOO_LARGE, "dt_tree_from_nodes: >= 2^24 nodes");
+  std::vector<int> refs((size_t)count, 0);
+  int32_t depth = 0;
+  if (nodes[0].depth != 0) return fail(DT_ERR_INVALID_ARG, "root depth != 0");
+  for (int64_t k = 0; k < count; ++k) {
+    const dt_node& a = nodes[k];
+    if (!isfinite(a.value)) return fail(DT_ERR_NONFINITE, "non-finite node value");
+    if (a.depth > depth) depth = a.depth;
+    if (a.feature < 0) {
+      if (a.left != -1 || a.right != -1) return fail(DT_ERR_INVALID_ARG, "leaf with children");
+      continue;
+    }
+    if (a.feature >= d) return fail(DT_ERR_INVALID_ARG, "feature index >= d");
+    if (!isfinite(a.threshold)) return fail(DT_ERR_NONFINITE, "non-finite threshold");
+    if (a.left <= k || a.right != a.left + 1 || a.right >= count)
+      return fail(DT_ERR_INVALID_ARG, "bad child links (need k < left, right == left + 1 < count)");
+    if (nodes[a.left].depth != a.depth + 1 || nodes[a.right].depth != a.depth + 1)
+      return fail(DT_ERR_INVALID_ARG, "child depth != parent depth + 1");
+    refs[(size_t)a.left]++;
+    refs[(size_t)a.right]++;
+  }
+  for (int64_t k = 1; k < count; ++k)
+    if (refs[(size_t)k] != 1) return fail(DT_ERR_INVALID_ARG, "node not referenced exactly once");
+  dt_tree* t = new dt_tree();
+  t->count = count;
+  t->d = d;
+  t->depth = depth;
+  t->host = (dt_node*)malloc(sizeof(dt_node) * (size_t)count);
+  memcpy(t->host, nodes, sizeof(dt_node) * (size_t)count);
+  dt_status st = tree_upload(t, 0);
+  if (st != DT_OK) {
+    dt_tree_free(t);
+    return st;
+  }
+  *out = t;
+  return DT_OK;
+}
+
+void dt_tree_free(dt_tree* t) {
+  if (!t) return;
+  if (t->dev_packed) cudaFree(t->dev_packed);
+  if (t->dev_value) cudaFree(t->dev_value);
+  free(t->host);
+  delete t;
+}
+
+dt_status dt_predict(const dt_tree* t, const float* X_dev, int64_t n, int32_t d,
+                     double* yhat_dev, void* stream) {
+  if (!t) return fail(DT_ERR_INVALID_ARG, "dt_predict: tree is NULL");
+  if (n < 0) return fail(DT_ERR_INVALID_ARG, "dt_predict: n < 0");
+  if (n == 0) return DT_OK;
+  if (!X_dev || !yhat_dev) return fail(DT_ERR_INVALID_ARG, "dt_predict: NULL X or yhat");
+  if (d != t->d) return fail(DT_ERR_INVALID_ARG, "dt_predict: d differs from the tree's d");
+  if (n >= ((int64_t)1 << 62)) return fail(DT_ERR_TOO_LARGE, "dt_predict: n >= 2^62");
+  return predict_impl(t, X_dev, n, d, yhat_dev, S(stream));
+}
+
+dt_status dt_eval(const double* y_dev, const double* yhat_dev, int64_t n, int32_t p,
+                  void* stream, dt_metrics* out) {
+  if (!out) return fail(DT_ERR_INVALID_ARG, "dt_eval: out is NULL");
+  if (!y_dev || !yhat_dev) return fail(DT_ERR_INVALID_ARG, "dt_eval: NULL y or yhat");
+  if (n < 1) return fail(DT_ERR_INVALID_ARG, "dt_eval: n must be >= 1");
+  if (p < 0) return fail(DT_ERR_INVALID_ARG, "dt_eval: p must be >= 0");
+  return eval_impl(y_dev, yhat_dev, nullptr, nullptr, n, p, S(stream), out);
+}
+
+dt_status dt_predict_eval(const dt_tree* t, const float* X_dev, const double* y_dev, int64_t n,
+                          int32_t d, int32_t p, void* stream, dt_metrics* out) {
+  if (!out || !t) return fail(DT_ERR_INVALID_ARG, "dt_predict_eval: NULL tree or out");
+  if (!X_dev || !y_dev) return fail(DT_ERR_INVALID_ARG, "dt_predict_eval: NULL X or y");
+  if (n < 1) return fail(DT_ERR_INVALID_ARG, "dt_predict_eval: n must be >= 1");
+  if (p < 0) return fail(DT_ERR_INVALID_ARG, "dt_predict_eval: p must be >= 0");
+  if (d != t->d) return fail(DT_ERR_INVALID_ARG, "dt_predict_eval: d differs from the tree's d");
+  return eval_impl(y_dev, nullptr, X_dev, t, n, p, S(stream), out);
+}
+
+dt_status dt_loo(const float* X_dev, const double* y_dev, int64_t n, int32_t d, int32_t max_depth,
+                 int64_t min_samples_leaf, double* yhat_oof_dev, void* stream) {
+  if (!X_dev || !y_dev || !yhat_oof_dev) return fail(DT_ERR_INVALID_ARG, "dt_loo: NULL pointer");
+  if (n < 2) return fail(DT_ERR_INVALID_ARG, "dt_loo: n must be >= 2");
+  if (d < 1 || d > 255) return fail(DT_ERR_INVALID_ARG, "dt_loo: d must be in [1, 255]");
+  if (max_depth < -1) return fail(DT_ERR_INVALID_ARG, "dt_loo: max_depth must be >= -1");
+  if (min_samples_leaf < 1) return fail(DT_ERR_INVALID_ARG, "dt_loo: min_samples_leaf must be >= 1");
+  if (n > 64 || d > 32) return fail(DT_ERR_TOO_LARGE, "dt_loo: needs n <= 64 and d <= 32");
+  return loo_impl(X_dev, y_dev, n, d, max_depth, min_samples_leaf, yhat_oof_dev, S(stream));
+}
+
+dt_status dt_gen_table(uint64_t seed, int64_t row0, int64_t n, int32_t d, int32_t real,
+                       int32_t cnn_pool_bits, int32_t gpu_pool_bits, double unit_us,
+                       float* X_dev, double* y_dev, void* stream) {
+  if (!X_dev) return fail(DT_ERR_INVALID_ARG, "dt_gen_table: X is NULL");
+  if (n < 0 || row0 < 0) return fail(DT_ERR_INVALID_ARG, "dt_gen_table: n, row0 must be >= 0");
+  if (d != 16 && d != 32) return fail(DT_ERR_INVALID_ARG, "dt_gen_table: d must be 16 or 32");
+  if (cnn_pool_bits < 1 || cnn_pool_bits > 40 || gpu_pool_bits < 1 || gpu_pool_bits > 40)
+    return fail(DT_ERR_INVALID_ARG, "dt_gen_table: pool bits must be in [1, 40]");
+  if (!(unit_us > 0.0)) return fail(DT_ERR_INVALID_ARG, "dt_gen_table: unit_us must be > 0");
+  if (n == 0) return DT_OK;
+  return gen_table_impl(seed, row0, n, d, real, cnn_pool_bits, gpu_pool_bits, unit_us, X_dev,
+                        y_dev, S(stream));
+}
+
+dt_status dt_gen_dse(uint64_t seed, int64_t row0, int64_t n, int32_t gpu_bits, float* X_dev,
+                     void* stream) {
+  if (!X_dev) return fail(DT_ERR_INVALID_ARG, "dt_gen_dse: X is NULL");
+  if (n < 0 || row0 < 0) return fail(DT_ERR_INVALID_ARG, "dt_gen_dse: n, row0 must be >= 0");
+  if (gpu_bits < 1 || gpu_bits > 40) return fail(DT_ERR_INVALID_ARG, "dt_gen_dse: gpu_bits in [1, 40]");
+  if (n == 0) return DT_OK;
+  return gen_dse_impl(seed, row0, n, gpu_bits, X_dev, S(stream));
+}
+
+}  // extern "C"

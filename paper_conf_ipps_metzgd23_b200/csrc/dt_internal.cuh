@@ -1,0 +1,71 @@
+// Internal declarations of libdt (B200 / sm_100a).  Not part of the C ABI.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "../../include/dt.h"
+
+struct dt_tree {
+  int64_t count = 0;          // number of nodes
+  int32_t d = 0;              // features
+  int32_t depth = 0;          // realised depth
+  int64_t split_evals = 0;    // sum over searched nodes of N*d
+  int32_t integer_mode = 0;
+  dt_node* host = nullptr;    // count nodes, BFS
+  // Device copy for prediction: packed 8-byte nodes {f32 thr (round-down), u32 f<<24|left}
+  // (leaves self-loop: feature 0, thr +inf, left = self) plus f64 values.
+  uint2* dev_packed = nullptr;
+  double* dev_value = nullptr;
+  int device = -1;
+};
+
+namespace dtl {
+
+// thread-local last error
+void set_error(const std::string& msg);
+dt_status fail(dt_status st, const std::string& msg);
+dt_status cuda_fail(cudaError_t e, const char* what, const char* file, int line);
+
+#define DT_CK(call)                                                          \
+  do {                                                                       \
+    cudaError_t e__ = (call);                                                \
+    if (e__ != cudaSuccess) return dtl::cuda_fail(e__, #call, __FILE__, __LINE__); \
+  } while (0)
+
+// Build the device copy of a tree (packed nodes + values) from its host node array.
+dt_status tree_upload(dt_tree* t, cudaStream_t s);
+
+// Fit driver (fit.cu).
+dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
+                   int64_t min_leaf, cudaStream_t s, dt_tree** out);
+// Predict / eval (predict.cu).
+dt_status predict_impl(const dt_tree* t, const float* X, int64_t n, int32_t d, double* yhat,
+                       cudaStream_t s);
+dt_status eval_impl(const double* y, const double* yhat, const float* X, const dt_tree* t,
+                    int64_t n, int32_t p, cudaStream_t s, dt_metrics* out);
+// LOO (loo.cu).
+dt_status loo_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
+                   int64_t min_leaf, double* yhat, cudaStream_t s);
+// Generators (gen.cu).
+dt_status gen_table_impl(uint64_t seed, int64_t row0, int64_t n, int32_t d, int32_t real,
+                         int32_t cbits, int32_t gbits, double unit_us, float* X, double* y,
+                         cudaStream_t s);
+dt_status gen_dse_impl(uint64_t seed, int64_t row0, int64_t n, int32_t gbits, float* X,
+                       cudaStream_t s);
+
+int num_sms();
+
+// Profiling (prof.cu).  Kinds index the name table in prof.cu.
+enum ProfKind {
+  PK_PRESORT_KEYS = 0, PK_PRESORT_SORT, PK_PRESORT_BUILD, PK_ROOT, PK_SCAN, PK_SELECT,
+  PK_NUMBER, PK_GOLEFT, PK_PARTITION, PK_PREDICT, PK_EVAL, PK_LOO, PK_GEN, PK_MEMSET
+};
+// Records an event before the launch(es) if profiling is on; counts `nlaunch` kernel
+// launches of this library either way.  Returns a record index (or -1).
+int prof_begin(int kind, cudaStream_t s, int nlaunch);
+void prof_end(int idx, cudaStream_t s, double alg_bytes);
+void prof_set_bytes(int idx, double alg_bytes);
+
+}  // namespace dtl

@@ -1,0 +1,1268 @@
+// Exact greedy CART regression fit on B200 ("Decision Tree regression";
+// split rule, tie rule, threshold and leaf rules: DESIGN.md Readings R1-R10, R19).
+//
+// Level-synchronous, exact (every feature, every threshold, every node):
+//   presort (once)   X row-major -> per-feature lists sorted by (x, row id), SoA
+//                    {x f32, row u32, y f64}; CUB radix sort of (f<<32 | flip(x), row).
+//   per level l:     scan      segmented prefix of (y - c_node) over every (node, feature)
+//                              segment (deterministic decoupled look-back), gain at every
+//                              valid position, per-(node,feature) argmax pieces, and
+//                              per-node SSE / min / max from the feature-0 list;
+//                    select    per node: combine pieces, leaf rules, best feature;
+//                    number    BFS numbering of the children, child statistics, offsets;
+//                    goleft    byte per row: 1 if the row goes to the left child;
+//                    partition stable partition of every feature list into the children
+//                              (sorted order preserved, rows of leaves dropped).
+// No host synchronisation inside the level loop (counts live on the device); kernels
+// are persistent and read the level's node/entry counts from device memory.
+#include <cub/device/device_radix_sort.cuh>
+
+#include <math.h>
+#include <stdio.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "dt_internal.cuh"
+#include "scan_primitives.cuh"
+
+namespace dtl {
+
+namespace {
+
+constexpr int kThreads = 256;
+constexpr int kItems = 16;
+constexpr int kTile = kThreads * kItems;  // 4096 list entries per tile
+
+// Per-level node record (level-local index k).
+struct NodeL {
+  uint32_t start;  // first position of the node in every feature list of this level
+  uint32_t N;      // rows
+  int32_t id;      // BFS index in the output node array
+  int32_t searchable;
+  double c;        // centre (integer mode: floor(S/N); real mode: value)
+  double sc;       // S' = sum over the node's rows of (y - c)
+  double v;        // value = mean y
+  double pad;
+};
+
+struct Decision {
+  int32_t f;    // split feature, -1 = leaf
+  uint32_t nl;  // rows going left (first nl in f-order)
+  double sl;    // S'_L (parent-centred) at the split
+  double thr;   // threshold
+};
+
+struct Ctl {
+  unsigned long long A[2];  // active entries per feature list, by level parity
+  uint32_t K[2];            // nodes at the level, by level parity
+  int32_t next_id;          // number of output nodes allocated so far
+  int32_t int_mode;
+  unsigned long long split_evals;
+  int32_t max_depth_seen;
+  int32_t nonfinite;
+  // root reduction
+  double ysum, ymin, ymax, ysc;
+  int32_t all_integral;
+  int32_t pad;
+};
+
+struct LevelLog {  // per-level counts, for algorithmic-byte accounting (profiling)
+  unsigned long long A, A_next;
+  uint32_t K, K_next;
+};
+constexpr int kMaxLogLevels = 4096;
+
+struct Cand {  // best candidate of one segment piece
+  double gain;
+  double sl;
+  uint32_t i;
+  uint32_t pad;
+  double pad2;
+};
+
+struct Stat {
+  double sse, ymin, ymax, s1;  // s1 = sum (y - c) over the piece
+};
+
+__device__ __forceinline__ uint32_t flip_f32(float x) {
+  uint32_t u = __float_as_uint(x);
+  if ((u << 1) == 0) u = 0;  // canonicalise -0.0 to +0.0 (equal under f32 compare)
+  return (u & 0x80000000u) ? ~u : (u | 0x80000000u);
+}
+__device__ __forceinline__ float unflip_f32(uint32_t k) {
+  uint32_t u = (k & 0x80000000u) ? (k & 0x7fffffffu) : ~k;
+  return __uint_as_float(u);
+}
+
+__device__ __forceinline__ long long floor_div_ll(long long a, long long b) {
+  long long q = a / b, r = a % b;
+  return (r != 0 && r < 0) ? q - 1 : q;
+}
+
+// Binary search: largest k in [0, K) with nodes[k].start <= q.
+__device__ __forceinline__ uint32_t find_node(const NodeL* __restrict__ nodes, uint32_t K, uint32_t q) {
+  uint32_t lo = 0, hi = K;  // invariant: nodes[lo].start <= q < nodes[hi].start
+  while (hi - lo > 1) {
+    uint32_t mid = (lo + hi) >> 1;
+    if (__ldg(&nodes[mid].start) <= q) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+
+// ----------------------------------------------------------------------------- root --
+
+struct RootPart {
+  double s, c;  // Neumaier sum
+  double mn, mx;
+  int integral, finite;
+};
+
+__device__ __forceinline__ void neu_add(double& s, double& c, double v) {
+  double t = __dadd_rn(s, v);
+  if (fabs(s) >= fabs(v)) c = __dadd_rn(c, __dadd_rn(__dsub_rn(s, t), v));
+  else c = __dadd_rn(c, __dadd_rn(__dsub_rn(v, t), s));
+  s = t;
+}
+
+// Deterministic two-level reduction of y: Neumaier sum, min, max, integrality, finiteness.
+__global__ void __launch_bounds__(256) root_reduce_kernel(const double* __restrict__ y, int64_t n,
+                                                          int64_t chunk, RootPart* parts) {
+  const int64_t lo = (int64_t)blockIdx.x * chunk, hi = min(n, lo + chunk);
+  RootPart p{0, 0, INFINITY, -INFINITY, 1, 1};
+  for (int64_t r = lo + threadIdx.x; r < hi; r += blockDim.x) {
+    double v = y[r];
+    if (!isfinite(v)) p.finite = 0;
+    if (floor(v) != v) p.integral = 0;
+    neu_add(p.s, p.c, v);
+    p.mn = fmin(p.mn, v);
+    p.mx = fmax(p.mx, v);
+  }
+  __shared__ RootPart sh[256];
+  sh[threadIdx.x] = p;
+  __syncthreads();
+  for (int off = 128; off > 0; off >>= 1) {
+    if (threadIdx.x < off) {
+      RootPart& a = sh[threadIdx.x];
+      const RootPart& b = sh[threadIdx.x + off];
+      neu_add(a.s, a.c, b.s);
+      neu_add(a.s, a.c, b.c);
+      a.mn = fmin(a.mn, b.mn);
+      a.mx = fmax(a.mx, b.mx);
+      a.integral &= b.integral;
+      a.finite &= b.finite;
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) parts[blockIdx.x] = sh[0];
+}
+
+__global__ void root_finalize_kernel(const RootPart* parts, int nparts, int64_t n, Ctl* ctl) {
+  if (threadIdx.x != 0) return;
+  double s = 0, c = 0, mn = INFINITY, mx = -INFINITY;
+  int integral = 1, finite = 1;
+  for (int i = 0; i < nparts; ++i) {
+    neu_add(s, c, parts[i].s);
+    neu_add(s, c, parts[i].c);
+    mn = fmin(mn, parts[i].mn);
+    mx = fmax(mx, parts[i].mx);
+    integral &= parts[i].integral;
+    finite &= parts[i].finite;
+  }
+  ctl->ysum = __dadd_rn(s, c);
+  ctl->ymin = mn;
+  ctl->ymax = mx;
+  ctl->all_integral = integral;
+  if (!finite) ctl->nonfinite = 1;
+  const double amax = fmax(fabs(mn), fabs(mx));
+  // Reading R17: integer mode iff every y integral and max|y| * n < 2^52.
+  ctl->int_mode = (integral && finite && amax * (double)n < 4503599627370496.0) ? 1 : 0;
+}
+
+// S'_0 = sum (y - c0) over all rows (second pass; c0 from the finalised root sum).
+__global__ void __launch_bounds__(256) root_center_kernel(const double* __restrict__ y, int64_t n,
+                                                          int64_t chunk, const Ctl* ctl, double* parts) {
+  const int64_t lo = (int64_t)blockIdx.x * chunk, hi = min(n, lo + chunk);
+  double c0;
+  if (ctl->int_mode) c0 = (double)floor_div_ll((long long)ctl->ysum, (long long)n);
+  else c0 = __ddiv_rn(ctl->ysum, (double)n);
+  double s = 0, cc = 0;
+  for (int64_t r = lo + threadIdx.x; r < hi; r += blockDim.x) neu_add(s, cc, __dsub_rn(y[r], c0));
+  __shared__ double sh[256];
+  sh[threadIdx.x] = __dadd_rn(s, cc);
+  __syncthreads();
+  for (int off = 128; off > 0; off >>= 1) {
+    if (threadIdx.x < off) sh[threadIdx.x] = __dadd_rn(sh[threadIdx.x], sh[threadIdx.x + off]);
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) parts[blockIdx.x] = sh[0];
+}
+
+__global__ void root_init_kernel(const double* parts, int nparts, int64_t n, int32_t max_depth,
+                                 int64_t min_leaf, Ctl* ctl, NodeL* nodes0) {
+  if (threadIdx.x != 0) return;
+  double s = 0, cc = 0;
+  for (int i = 0; i < nparts; ++i) neu_add(s, cc, parts[i]);
+  NodeL nd;
+  nd.start = 0;
+  nd.N = (uint32_t)n;
+  nd.id = 0;
+  nd.searchable = (max_depth != 0 && n >= 2 * min_leaf) ? 1 : 0;
+  if (ctl->int_mode) {
+    nd.c = (double)floor_div_ll((long long)ctl->ysum, (long long)n);
+    nd.v = __ddiv_rn(ctl->ysum, (double)n);
+    nd.sc = ctl->ysum - nd.c * (double)n;  // exact in integer mode
+  } else {
+    nd.v = __ddiv_rn(ctl->ysum, (double)n);
+    nd.c = nd.v;
+    nd.sc = __dadd_rn(s, cc);
+  }
+  nd.pad = 0;
+  nodes0[0] = nd;
+  ctl->ysc = nd.sc;
+  ctl->A[0] = (unsigned long long)n;
+  ctl->K[0] = 1;
+  ctl->next_id = 1;
+  ctl->split_evals = 0;
+  ctl->max_depth_seen = 0;
+}
+
+// ----------------------------------------------------------------------------- presort --
+
+// keys[f*n + r] = f << 32 | flip(x[r][f]); vals = r.  X row-major -> feature-major via smem.
+__global__ void __launch_bounds__(256) presort_keys_kernel(const float* __restrict__ X, int64_t n, int d,
+                                                           unsigned long long* __restrict__ keys,
+                                                           uint32_t* __restrict__ vals, Ctl* ctl) {
+  extern __shared__ float tileX[];  // 256 rows x d
+  const int64_t r0 = (int64_t)blockIdx.x * 256;
+  const int rows = (int)min((int64_t)256, n - r0);
+  const int64_t base = r0 * d;
+  const int tot = rows * d;
+  bool bad = false;
+  for (int i = threadIdx.x; i < tot; i += blockDim.x) {
+    float v = X[base + i];
+    if (!isfinite(v)) bad = true;
+    tileX[i] = v;
+  }
+  if (__syncthreads_or(bad) && threadIdx.x == 0) ctl->nonfinite = 1;
+  for (int f = 0; f < d; ++f) {
+    if (threadIdx.x < rows) {
+      const int64_t r = r0 + threadIdx.x;
+      const float v = tileX[threadIdx.x * d + f];
+      keys[(int64_t)f * n + r] = ((unsigned long long)f << 32) | flip_f32(v);
+      vals[(int64_t)f * n + r] = (uint32_t)r;
+    }
+  }
+}
+
+// SoA level-0 lists from the sorted pairs: x = unflip(key), row = val, y = y[row].
+__global__ void __launch_bounds__(256) presort_build_kernel(const unsigned long long* __restrict__ keys,
+                                                            const uint32_t* __restrict__ vals,
+                                                            const double* __restrict__ y, int64_t total,
+                                                            float* __restrict__ lx, uint32_t* __restrict__ lr,
+                                                            double* __restrict__ ly) {
+  for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < total;
+       p += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t r = vals[p];
+    lx[p] = unflip_f32((uint32_t)keys[p]);
+    lr[p] = r;
+    ly[p] = __ldg(y + r);
+  }
+}
+
+// ----------------------------------------------------------------------------- scan ----
+
+struct ScanArgs {
+  const float* lx;
+  const double* ly;
+  const NodeL* nodes;
+  const Ctl* ctl;
+  int parity;
+  int dl;          // feature lists present at this level (d, or 1 at the last level)
+  int d;           // feature count (slot stride)
+  int64_t min_leaf;
+  uint32_t* counter;  // tile counter (zeroed per launch)
+  TileSlots<SumP> ts;
+  Cand* head_cand;  // [K*d]
+  Cand* cont_cand;  // [ntiles]
+  Stat* head_stat;  // [K]
+  Stat* cont_stat;  // [ntiles]
+};
+
+__device__ __forceinline__ void write_cand(Cand* p, const ArgP& a) {
+  Cand c;
+  c.gain = a.gain;
+  c.sl = a.sl;
+  c.i = a.i;
+  c.pad = 0;
+  c.pad2 = 0;
+  *p = c;
+}
+__device__ __forceinline__ void write_stat(Stat* p, const StatP& a) {
+  Stat s;
+  s.sse = a.sse;
+  s.ymin = a.ymin;
+  s.ymax = a.ymax;
+  s.s1 = a.s1;
+  *p = s;
+}
+
+// Gain of candidate "first i rows left" (Reading R19), no FMA contraction:
+//   D = S'_L n_R - S'_R n_L,  gain = D^2 / ((N n_L) n_R).
+__device__ __forceinline__ double split_gain(double sl, double sc, uint32_t i, uint32_t N) {
+  const double nl = (double)i, nr = (double)(N - i), Nd = (double)N;
+  const double sr = __dsub_rn(sc, sl);
+  const double D = __dsub_rn(__dmul_rn(sl, nr), __dmul_rn(sr, nl));
+  return __ddiv_rn(__dmul_rn(D, D), __dmul_rn(__dmul_rn(Nd, nl), nr));
+}
+
+__global__ void __launch_bounds__(kThreads) scan_kernel(ScanArgs a) {
+  __shared__ SumP sh_sum[33];
+  __shared__ ArgP sh_arg[33];
+  __shared__ StatP sh_stat[33];
+  __shared__ int64_t sh_tile;
+  __shared__ SumP sh_carry;
+
+  const uint32_t K = a.ctl->K[a.parity];
+  const uint64_t A = a.ctl->A[a.parity];
+  if (K == 0 || A == 0) return;
+  const int64_t total = (int64_t)A * a.dl;
+  const int64_t ntiles = (total + kTile - 1) / kTile;
+  const int tid = threadIdx.x;
+
+  for (;;) {
+    if (tid == 0) sh_tile = (int64_t)atomicAdd(a.counter, 1u);
+    __syncthreads();
+    const int64_t tile = sh_tile;
+    __syncthreads();
+    if (tile >= ntiles) break;
+    const int64_t p0 = tile * kTile + (int64_t)tid * kItems;
+
+    // ---- locate my first item, load items
+    float xv[kItems];
+    double yv[kItems];
+    int f0 = 0;
+    uint32_t q0 = 0, k0 = 0;
+    const bool any = p0 < total;
+    if (any) {
+      f0 = (int)(p0 / (int64_t)A);
+      q0 = (uint32_t)(p0 - (int64_t)f0 * (int64_t)A);
+      k0 = find_node(a.nodes, K, q0);
+      if (p0 + kItems <= total) {
+        const float4* x4 = reinterpret_cast<const float4*>(a.lx + p0);
+        const double2* y2 = reinterpret_cast<const double2*>(a.ly + p0);
+#pragma unroll
+        for (int j = 0; j < kItems / 4; ++j) {
+          float4 t = __ldcs(x4 + j);
+          xv[4 * j] = t.x; xv[4 * j + 1] = t.y; xv[4 * j + 2] = t.z; xv[4 * j + 3] = t.w;
+        }
+#pragma unroll
+        for (int j = 0; j < kItems / 2; ++j) {
+          double2 t = __ldcs(y2 + j);
+          yv[2 * j] = t.x; yv[2 * j + 1] = t.y;
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+          const bool ok = p0 + j < total;
+          xv[j] = ok ? a.lx[p0 + j] : 0.f;
+          yv[j] = ok ? a.ly[p0 + j] : 0.0;
+        }
+      }
+    }
+
+    // ---- pass 1: thread aggregate of the segmented sum of (y - c)
+    SumP tagg{0u, 0.0};
+    {
+      int f = f0;
+      uint32_t q = q0, k = k0;
+      uint32_t kend = any ? __ldg(&a.nodes[k].start) + __ldg(&a.nodes[k].N) : 0;
+      uint32_t kstart = any ? __ldg(&a.nodes[k].start) : 0;
+      double c = any ? __ldg(&a.nodes[k].c) : 0.0;
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        if (p0 + j < total) {
+          if (q >= (uint32_t)A) { ++f; q = 0; k = 0; kstart = 0; kend = __ldg(&a.nodes[0].N); c = __ldg(&a.nodes[0].c); }
+          while (q >= kend) { ++k; kstart = kend; kend = kstart + __ldg(&a.nodes[k].N); c = __ldg(&a.nodes[k].c); }
+          const double e = __dsub_rn(yv[j], c);
+          if (q == kstart) { tagg.flag = 1u; tagg.s = e; }
+          else tagg.s = __dadd_rn(tagg.s, e);
+          ++q;
+        }
+      }
+    }
+    // tile's first element is a segment head?
+    SumP tile_agg;
+    SumP texcl = block_exclusive_scan(tagg, SumP{0u, 0.0}, tile_agg, sh_sum);
+    if (tid == 0) {
+      const bool head0 = (q0 == __ldg(&a.nodes[k0].start));  // tid 0 is always "any"
+      if (head0 || tile == 0) {
+        publish(a.ts, tile, tile_agg, 2);
+        sh_carry = SumP{0u, 0.0};
+      } else {
+        publish(a.ts, tile, tile_agg, 1);
+        SumP carry = lookback(a.ts, tile, SumP{0u, 0.0});
+        publish(a.ts, tile, combine(carry, tile_agg), 2);
+        sh_carry = carry;
+      }
+    }
+    __syncthreads();
+    const SumP carry = sh_carry;
+    // my exclusive prefix value at item 0 (meaningless if item 0 is a head)
+    double S = combine(carry, texcl).s;
+
+    // ---- pass 2: prefixes, gains, per-run best; flush runs that end in this thread
+    ArgP run{0u, 0xffffffffu, -1.0, 0.0};   // current run's best
+    StatP srun{0u, 0.0, INFINITY, -INFINITY};
+    bool seen_head = false;                  // a head occurred in this thread
+    ArgP first_run{0u, 0xffffffffu, -1.0, 0.0};
+    StatP first_srun{0u, 0.0, INFINITY, -INFINITY};
+    // open-segment identity at the end of this thread
+    int last_f = f0;
+    uint32_t last_k = k0;
+    const bool stats_tile = (tile * kTile) < (int64_t)A;  // tile holds feature-0 items
+    {
+      int f = f0;
+      uint32_t q = q0, k = k0;
+      uint32_t kstart = any ? __ldg(&a.nodes[k].start) : 0;
+      uint32_t N = any ? __ldg(&a.nodes[k].N) : 0;
+      uint32_t kend = kstart + N;
+      double c = any ? __ldg(&a.nodes[k].c) : 0.0;
+      double sc = any ? __ldg(&a.nodes[k].sc) : 0.0;
+      double v = any ? __ldg(&a.nodes[k].v) : 0.0;
+      int srch = any ? __ldg(&a.nodes[k].searchable) : 0;
+      float xprev = (any && q0 > kstart) ? a.lx[p0 - 1] : 0.f;
+      const uint32_t m = (uint32_t)min(a.min_leaf, (int64_t)0xffffffff);
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        if (p0 + j < total) {
+          bool newseg = false;
+          if (q >= (uint32_t)A) { ++f; q = 0; k = 0; kstart = 0; newseg = true; }
+          else if (q >= kend) { ++k; kstart = kend; newseg = true; }
+          if (newseg) {
+            while (true) {
+              N = __ldg(&a.nodes[k].N);
+              kend = kstart + N;
+              if (q < kend) break;
+              ++k; kstart = kend;
+            }
+            c = __ldg(&a.nodes[k].c);
+            sc = __ldg(&a.nodes[k].sc);
+            v = __ldg(&a.nodes[k].v);
+            srch = __ldg(&a.nodes[k].searchable);
+          }
+          const bool head = (q == kstart);
+          if (head) {
+            // close the run before this head
+            if (!seen_head) { first_run = run; first_srun = srun; }
+            else {
+              // a run strictly inside this thread: complete segment, started in this tile
+              const int pf = (k == 0) ? f - 1 : f;            // previous segment
+              const uint32_t pkk = (k == 0) ? (K - 1) : k - 1;
+              write_cand(a.head_cand + (int64_t)pkk * a.d + pf, run);
+              if (pf == 0) write_stat(a.head_stat + pkk, srun);
+            }
+            seen_head = true;
+            run = ArgP{1u, 0xffffffffu, -1.0, 0.0};
+            srun = StatP{1u, 0.0, INFINITY, -INFINITY, 0.0};
+            S = 0.0;
+          }
+          const uint32_t i = q - kstart;
+          const float x = xv[j];
+          if (srch && i >= m && N - i >= m && i >= 1) {
+            const float xp = (j == 0) ? xprev : xv[j - 1];
+            if (xp < x) {
+              const double g = split_gain(S, sc, i, N);
+              if (g > run.gain) { run.gain = g; run.i = i; run.sl = S; }
+            }
+          }
+          const double e = __dsub_rn(yv[j], c);
+          S = __dadd_rn(S, e);
+          if (f == 0) {
+            const double ev = __dsub_rn(yv[j], v);
+            srun.sse = __dadd_rn(srun.sse, __dmul_rn(ev, ev));
+            srun.ymin = fmin(srun.ymin, yv[j]);
+            srun.ymax = fmax(srun.ymax, yv[j]);
+            srun.s1 = __dadd_rn(srun.s1, e);
+          }
+          ++q;
+          last_f = f;
+          last_k = k;
+        }
+      }
+    }
+    if (!seen_head) { first_run = run; first_srun = srun; }
+    // trailing run of this thread (flag = any head in this thread)
+    ArgP trail = run;
+    trail.flag = seen_head ? 1u : 0u;
+    StatP strail = srun;
+    strail.flag = seen_head ? 1u : 0u;
+
+    ArgP arg_blk;
+    const ArgP aex = block_exclusive_scan(trail, ArgP{0u, 0xffffffffu, -1.0, 0.0}, arg_blk, sh_arg);
+    StatP sex{0u, 0.0, INFINITY, -INFINITY}, st_blk;
+    if (stats_tile) sex = block_exclusive_scan(strail, StatP{0u, 0.0, INFINITY, -INFINITY, 0.0}, st_blk, sh_stat);
+
+    // Flush the open segment that ends at my first head (its earlier part is in aex).
+    if (any && seen_head) {
+      // does my first item start a segment?  then the open segment ended before me
+      ArgP done_a;
+      StatP done_s;
+      const bool item0_head = (q0 == __ldg(&a.nodes[k0].start));
+      if (!(tid == 0 && item0_head)) {
+        // open segment identity: the segment containing the item before my first head
+        int of;
+        uint32_t ok;
+        if (!item0_head) { of = f0; ok = k0; }
+        else if (k0 > 0) { of = f0; ok = k0 - 1; }
+        else { of = f0 - 1; ok = K - 1; }
+        ArgP fr = first_run;
+        fr.flag = 0u;
+        done_a = combine(aex, fr);
+        const bool head_in_tile = aex.flag != 0;
+        if (head_in_tile) write_cand(a.head_cand + (int64_t)ok * a.d + of, done_a);
+        else write_cand(a.cont_cand + tile, done_a);
+        if (stats_tile && of == 0) {
+          StatP fs = first_srun;
+          fs.flag = 0u;
+          done_s = combine(sex, fs);
+          if (head_in_tile) write_stat(a.head_stat + ok, done_s);
+          else write_stat(a.cont_stat + tile, done_s);
+        }
+      }
+    }
+    // The last thread closes the segment open at the tile end.
+    if (tid == kThreads - 1) {
+      // find the segment of the tile's last valid element
+      const int64_t plast = min(total, tile * kTile + kTile) - 1;
+      const int lf = (int)(plast / (int64_t)A);
+      const uint32_t lq = (uint32_t)(plast - (int64_t)lf * (int64_t)A);
+      const uint32_t lk = any ? last_k : find_node(a.nodes, K, lq);
+      const int lff = any ? last_f : lf;
+      ArgP done_a = seen_head ? run : combine(aex, ArgP{0u, run.i, run.gain, run.sl});
+      const bool head_in_tile = seen_head || aex.flag != 0;
+      if (head_in_tile) write_cand(a.head_cand + (int64_t)lk * a.d + lff, done_a);
+      else write_cand(a.cont_cand + tile, done_a);
+      if (stats_tile && lff == 0) {
+        StatP done_s = seen_head ? srun : combine(sex, StatP{0u, srun.sse, srun.ymin, srun.ymax, srun.s1});
+        if (head_in_tile) write_stat(a.head_stat + lk, done_s);
+        else write_stat(a.cont_stat + tile, done_s);
+      }
+    }
+  }
+}
+
+// ----------------------------------------------------------------------------- select --
+
+struct SelectArgs {
+  const float* lx;
+  const NodeL* nodes;
+  Ctl* ctl;
+  int parity;
+  int level;
+  int dl;
+  int d;
+  const Cand* head_cand;
+  const Cand* cont_cand;
+  const Stat* head_stat;
+  const Stat* cont_stat;
+  Decision* dec;
+  dt_node* out;
+  LevelLog* log;
+};
+
+__device__ __forceinline__ bool cand_better(double g1, uint32_t i1, double g2, uint32_t i2) {
+  return g1 > g2 || (g1 == g2 && i1 < i2);
+}
+
+// One block per node (grid-stride over the level's nodes).
+__global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
+  const uint32_t K = a.ctl->K[a.parity];
+  const uint64_t A = a.ctl->A[a.parity];
+  __shared__ double s_gain[256];
+  __shared__ uint32_t s_i[256];
+  __shared__ double s_sl[256];
+  __shared__ Stat s_stat[256];
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  if (blockIdx.x == 0 && tid == 0 && a.level < kMaxLogLevels) {
+    a.log[a.level].A = A;
+    a.log[a.level].K = K;
+    a.log[a.level].A_next = 0;
+    a.log[a.level].K_next = 0;
+  }
+  for (uint32_t k = blockIdx.x; k < K; k += gridDim.x) {
+    const NodeL nd = a.nodes[k];
+    // ---- per-feature best (warp w handles features w, w+8, ...)
+    for (int f = w; f < a.d; f += 8) {
+      double bg = -1.0, bsl = 0.0;
+      uint32_t bi = 0xffffffffu;
+      if (nd.searchable && f < a.dl && nd.N > 1) {
+        const int64_t s0 = (int64_t)f * (int64_t)A + nd.start;
+        const int64_t s1 = s0 + nd.N - 1;
+        const int64_t t0 = s0 / kTile, t1 = s1 / kTile;
+        // piece 0 = head record, pieces 1.. = cont records of tiles t0+1..t1
+        for (int64_t pc = lane; pc <= t1 - t0; pc += 32) {
+          const Cand c = (pc == 0) ? a.head_cand[(int64_t)k * a.d + f] : a.cont_cand[t0 + pc];
+          if (c.gain >= 0.0 && cand_better(c.gain, c.i, bg, bi)) { bg = c.gain; bi = c.i; bsl = c.sl; }
+        }
+        for (int off = 16; off > 0; off >>= 1) {
+          const double og = __shfl_down_sync(0xffffffffu, bg, off);
+          const uint32_t oi = __shfl_down_sync(0xffffffffu, bi, off);
+          const double osl = __shfl_down_sync(0xffffffffu, bsl, off);
+          if (cand_better(og, oi, bg, bi)) { bg = og; bi = oi; bsl = osl; }
+        }
+      }
+      if (lane == 0) { s_gain[f] = bg; s_i[f] = bi; s_sl[f] = bsl; }
+    }
+    // ---- node statistics from the feature-0 list (fixed-shape reduction)
+    {
+      const int64_t s0 = nd.start, s1 = s0 + nd.N - 1;
+      const int64_t t0 = s0 / kTile, t1 = s1 / kTile;
+      Stat acc{0.0, INFINITY, -INFINITY, 0.0};  // s1 accumulates sum (y - c)
+      // each thread folds a contiguous run of pieces, then tree
+      const int64_t np = t1 - t0 + 1;
+      const int64_t per = (np + blockDim.x - 1) / blockDim.x;
+      for (int64_t pc = tid * per; pc < min(np, (tid + 1) * per); ++pc) {
+        const Stat s = (pc == 0) ? a.head_stat[k] : a.cont_stat[t0 + pc];
+        acc.sse = __dadd_rn(acc.sse, s.sse);
+        acc.ymin = fmin(acc.ymin, s.ymin);
+        acc.ymax = fmax(acc.ymax, s.ymax);
+        acc.s1 = __dadd_rn(acc.s1, s.s1);
+      }
+      s_stat[tid] = acc;
+      __syncthreads();
+      for (int off = 128; off > 0; off >>= 1) {
+        if (tid < off) {
+          Stat& x = s_stat[tid];
+          const Stat y = s_stat[tid + off];
+          x.sse = __dadd_rn(x.sse, y.sse);
+          x.ymin = fmin(x.ymin, y.ymin);
+          x.ymax = fmax(x.ymax, y.ymax);
+          x.s1 = __dadd_rn(x.s1, y.s1);
+        }
+        __syncthreads();
+      }
+    }
+    if (tid == 0) {
+      const Stat st = s_stat[0];
+      int bf = -1;
+      double bg = -1.0, bsl = 0.0;
+      uint32_t bi = 0;
+      const bool pure = !(st.ymin < st.ymax);
+      if (nd.searchable && !pure) {
+        for (int f = 0; f < a.d; ++f)
+          if (s_gain[f] > bg) { bg = s_gain[f]; bi = s_i[f]; bsl = s_sl[f]; bf = f; }  // strict >
+        atomicAdd(&a.ctl->split_evals, (unsigned long long)nd.N * (unsigned long long)a.d);
+      }
+      Decision dc;
+      dt_node o;
+      o.depth = a.level;
+      // value = mean of the node's own rows.  Integer mode: exact fl(S/N) from the exact
+      // bookkeeping.  Real mode: centre + fresh sum (y - c) / N, and exactly y for a pure
+      // node (all rows equal), so single-row leaves reproduce their target.
+      if (a.ctl->int_mode) o.value = nd.v;
+      else o.value = pure ? st.ymin : __dadd_rn(nd.c, __ddiv_rn(st.s1, (double)nd.N));
+      o.impurity = __ddiv_rn(st.sse, (double)nd.N);
+      o.n_samples = nd.N;
+      o.left = -1;
+      o.right = -1;
+      if (bf >= 0 && bg >= 0.0) {
+        const int64_t pos = (int64_t)bf * (int64_t)A + nd.start + bi;
+        const double xlo = (double)a.lx[pos - 1], xhi = (double)a.lx[pos];
+        dc.f = bf;
+        dc.nl = bi;
+        dc.sl = bsl;
+        dc.thr = __dadd_rn(__ddiv_rn(xlo, 2.0), __ddiv_rn(xhi, 2.0));  // Reading R5
+        o.feature = bf;
+        o.threshold = dc.thr;
+      } else {
+        dc.f = -1;
+        dc.nl = 0;
+        dc.sl = 0.0;
+        dc.thr = 0.0;
+        o.feature = -1;
+        o.threshold = 0.0;
+      }
+      a.dec[k] = dc;
+      a.out[nd.id] = o;
+      atomicMax(&a.ctl->max_depth_seen, a.level);
+    }
+    __syncthreads();
+  }
+}
+
+// ----------------------------------------------------------------------------- number --
+
+struct NumberArgs {
+  const NodeL* nodes;
+  NodeL* next;
+  const Decision* dec;
+  uint32_t* new_start;  // [K] left-child start in the next lists (or 0xffffffff)
+  Ctl* ctl;
+  int parity;
+  int level;
+  int32_t max_depth;
+  int64_t min_leaf;
+  dt_node* out;
+  LevelLog* log;
+};
+
+// Single block: BFS numbering (children appended left, right in node order), child
+// statistics, next-level offsets.  Integer mode keeps every quantity exact (int64).
+__global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
+  __shared__ CntP sh[33];
+  __shared__ unsigned long long sh_rows[33];
+  __shared__ uint32_t base_split;
+  __shared__ unsigned long long base_rows;
+  const uint32_t K = a.ctl->K[a.parity];
+  const int tid = threadIdx.x;
+  const int next_id0 = a.ctl->next_id;
+  const int int_mode = a.ctl->int_mode;
+  if (tid == 0) { base_split = 0; base_rows = 0; }
+  __syncthreads();
+  for (uint32_t k0 = 0; k0 < K; k0 += blockDim.x) {
+    const uint32_t k = k0 + tid;
+    const bool in = k < K;
+    const Decision dc = in ? a.dec[k] : Decision{-1, 0, 0.0, 0.0};
+    const bool sp = in && dc.f >= 0;
+    const NodeL nd = in ? a.nodes[k] : NodeL{};
+    CntP agg;
+    CntP ex = block_exclusive_scan(CntP{0u, sp ? 1u : 0u}, CntP{0u, 0u}, agg, sh);
+    // exclusive scan of rows of split nodes (64-bit, via warp shuffles)
+    unsigned long long rv = sp ? nd.N : 0ull, inc = rv;
+    const int lane = tid & 31, w = tid >> 5;
+    for (int dd = 1; dd < 32; dd <<= 1) {
+      unsigned long long o = __shfl_up_sync(0xffffffffu, inc, dd);
+      if (lane >= dd) inc += o;
+    }
+    if (lane == 31) sh_rows[w] = inc;
+    __syncthreads();
+    if (tid == 0) {
+      unsigned long long run = 0;
+      for (int i = 0; i < (int)(blockDim.x >> 5); ++i) { unsigned long long t = sh_rows[i]; sh_rows[i] = run; run += t; }
+      sh_rows[32] = run;
+    }
+    __syncthreads();
+    const unsigned long long rows_ex = base_rows + sh_rows[w] + (inc - rv);
+    const uint32_t rank = base_split + ex.c;
+    if (in) {
+      if (sp) {
+        const int lid = next_id0 + 2 * (int)rank;
+        a.out[nd.id].left = lid;
+        a.out[nd.id].right = lid + 1;
+        a.new_start[k] = (uint32_t)rows_ex;
+        const uint32_t nl = dc.nl, nr = nd.N - dc.nl;
+        NodeL L, R;
+        L.start = (uint32_t)rows_ex;
+        L.N = nl;
+        L.id = lid;
+        R.start = (uint32_t)rows_ex + nl;
+        R.N = nr;
+        R.id = lid + 1;
+        const int child_depth = a.level + 1;
+        const bool depth_ok = (a.max_depth < 0) || (child_depth < a.max_depth);
+        L.searchable = (depth_ok && (int64_t)nl >= 2 * a.min_leaf) ? 1 : 0;
+        R.searchable = (depth_ok && (int64_t)nr >= 2 * a.min_leaf) ? 1 : 0;
+        L.pad = R.pad = 0.0;
+        const double slp = dc.sl;                    // parent-centred S'_L
+        const double srp = __dsub_rn(nd.sc, slp);    // parent-centred S'_R
+        if (int_mode) {
+          const long long cp = (long long)nd.c;
+          const long long SL = (long long)nl * cp + (long long)slp;
+          const long long SR = (long long)nr * cp + (long long)srp;
+          const long long cl = floor_div_ll(SL, nl), cr = floor_div_ll(SR, nr);
+          L.c = (double)cl;
+          R.c = (double)cr;
+          L.v = __ddiv_rn((double)SL, (double)nl);
+          R.v = __ddiv_rn((double)SR, (double)nr);
+          L.sc = (double)(SL - (long long)nl * cl);
+          R.sc = (double)(SR - (long long)nr * cr);
+        } else {
+          L.v = __dadd_rn(nd.c, __ddiv_rn(slp, (double)nl));
+          R.v = __dadd_rn(nd.c, __ddiv_rn(srp, (double)nr));
+          L.c = L.v;
+          R.c = R.v;
+          // re-centre: S'_child = S'_(parent-centred) - n * (c_child - c_parent)
+          L.sc = __dsub_rn(slp, __dmul_rn((double)nl, __dsub_rn(L.c, nd.c)));
+          R.sc = __dsub_rn(srp, __dmul_rn((double)nr, __dsub_rn(R.c, nd.c)));
+        }
+        a.next[2 * rank] = L;
+        a.next[2 * rank + 1] = R;
+      } else {
+        a.new_start[k] = 0xffffffffu;
+      }
+    }
+    __syncthreads();
+    if (tid == 0) { base_split += agg.c; base_rows += sh_rows[32]; }
+    __syncthreads();
+  }
+  if (tid == 0) {
+    const int np = a.parity ^ 1;
+    a.ctl->K[np] = 2 * base_split;
+    a.ctl->A[np] = base_rows;
+    a.ctl->next_id = next_id0 + 2 * (int)base_split;
+    if (a.level < kMaxLogLevels) {
+      a.log[a.level].A_next = base_rows;
+      a.log[a.level].K_next = 2 * base_split;
+    }
+  }
+}
+
+// ----------------------------------------------------------------------------- goleft --
+
+// goleft[row] = 1 iff the row goes to the left child (rows of split nodes only).
+__global__ void __launch_bounds__(256) goleft_kernel(const uint32_t* __restrict__ lr, const NodeL* nodes,
+                                                     const Decision* dec, const Ctl* ctl, int parity,
+                                                     uint8_t* __restrict__ goleft) {
+  const uint32_t K = ctl->K[parity];
+  const uint64_t A = ctl->A[parity];
+  if (K == 0) return;
+  constexpr int kI = 8;
+  for (int64_t q0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * kI; q0 < (int64_t)A;
+       q0 += (int64_t)gridDim.x * blockDim.x * kI) {
+    uint32_t k = find_node(nodes, K, (uint32_t)q0);
+    uint32_t kstart = nodes[k].start, kend = kstart + nodes[k].N;
+    for (int j = 0; j < kI && q0 + j < (int64_t)A; ++j) {
+      const uint32_t q = (uint32_t)q0 + j;
+      while (q >= kend) { ++k; kstart = kend; kend = kstart + nodes[k].N; }
+      const Decision dc = dec[k];
+      if (dc.f >= 0) {
+        const uint32_t r = lr[(int64_t)dc.f * (int64_t)A + q];
+        goleft[r] = (q - kstart < dc.nl) ? 1 : 0;
+      }
+    }
+  }
+}
+
+// ----------------------------------------------------------------------------- partition --
+
+struct PartArgs {
+  const float* lx;
+  const uint32_t* lr;
+  const double* ly;
+  float* ox;
+  uint32_t* orow;
+  double* oy;
+  const NodeL* nodes;
+  const Decision* dec;
+  const uint32_t* new_start;
+  const uint8_t* goleft;
+  const Ctl* ctl;
+  int parity;
+  int dl_in;   // lists in the input (d)
+  int dl_out;  // lists to write (d, or 1 before the last level)
+  uint32_t* counter;
+  TileSlots<CntP> ts;
+};
+
+// Stable partition of each (node, feature) segment: left rows first then right rows,
+// order preserved; rows of nodes that did not split are dropped.
+__global__ void __launch_bounds__(kThreads) partition_kernel(PartArgs a) {
+  __shared__ CntP sh[33];
+  __shared__ int64_t sh_tile;
+  __shared__ CntP sh_carry;
+  const uint32_t K = a.ctl->K[a.parity];
+  const uint64_t A = a.ctl->A[a.parity];
+  const uint64_t A2 = a.ctl->A[a.parity ^ 1];
+  if (K == 0 || A2 == 0) return;
+  const int64_t total = (int64_t)A * a.dl_out;  // only the lists we write
+  const int64_t ntiles = (total + kTile - 1) / kTile;
+  const int tid = threadIdx.x;
+  for (;;) {
+    if (tid == 0) sh_tile = (int64_t)atomicAdd(a.counter, 1u);
+    __syncthreads();
+    const int64_t tile = sh_tile;
+    __syncthreads();
+    if (tile >= ntiles) break;
+    const int64_t p0 = tile * kTile + (int64_t)tid * kItems;
+    const bool any = p0 < total;
+    int f0 = 0;
+    uint32_t q0 = 0, k0 = 0;
+    uint32_t rv[kItems];
+    uint8_t gl[kItems];
+    if (any) {
+      f0 = (int)(p0 / (int64_t)A);
+      q0 = (uint32_t)(p0 - (int64_t)f0 * (int64_t)A);
+      k0 = find_node(a.nodes, K, q0);
+    }
+    // pass 1: go-left flags and thread aggregate
+    CntP tagg{0u, 0u};
+    {
+      int f = f0;
+      uint32_t q = q0, k = k0;
+      uint32_t kstart = any ? a.nodes[k].start : 0, kend = any ? kstart + a.nodes[k].N : 0;
+      bool split = any ? (a.dec[k].f >= 0) : false;
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        gl[j] = 0;
+        rv[j] = 0;
+        if (p0 + j < total) {
+          if (q >= (uint32_t)A) { ++f; q = 0; k = 0; kstart = 0; kend = a.nodes[0].N; split = a.dec[0].f >= 0; }
+          while (q >= kend) { ++k; kstart = kend; kend = kstart + a.nodes[k].N; split = a.dec[k].f >= 0; }
+          const bool head = q == kstart;
+          uint32_t g = 0;
+          if (split) {
+            rv[j] = __ldcs(a.lr + p0 + j);
+            g = a.goleft[rv[j]];
+          }
+          gl[j] = (uint8_t)g;
+          if (head) { tagg.flag = 1u; tagg.c = g; }
+          else tagg.c += g;
+          ++q;
+        }
+      }
+    }
+    CntP tile_agg;
+    CntP texcl = block_exclusive_scan(tagg, CntP{0u, 0u}, tile_agg, sh);
+    if (tid == 0) {
+      const bool head0 = (q0 == a.nodes[k0].start);
+      if (head0 || tile == 0) {
+        publish(a.ts, tile, tile_agg, 2);
+        sh_carry = CntP{0u, 0u};
+      } else {
+        publish(a.ts, tile, tile_agg, 1);
+        CntP carry = lookback(a.ts, tile, CntP{0u, 0u});
+        publish(a.ts, tile, combine(carry, tile_agg), 2);
+        sh_carry = carry;
+      }
+    }
+    __syncthreads();
+    uint32_t cl = combine(sh_carry, texcl).c;  // lefts before my item 0 in its segment
+    if (any) {
+      int f = f0;
+      uint32_t q = q0, k = k0;
+      uint32_t kstart = a.nodes[k].start, kend = kstart + a.nodes[k].N;
+      Decision dc = a.dec[k];
+      uint32_t ns = a.new_start[k];
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        if (p0 + j < total) {
+          bool nseg = false;
+          if (q >= (uint32_t)A) { ++f; q = 0; k = 0; kstart = 0; kend = a.nodes[0].N; nseg = true; }
+          while (q >= kend) { ++k; kstart = kend; kend = kstart + a.nodes[k].N; nseg = true; }
+          if (nseg) { dc = a.dec[k]; ns = a.new_start[k]; }
+          if (q == kstart) cl = 0;
+          if (dc.f >= 0) {
+            const uint32_t i = q - kstart;
+            uint32_t dst;
+            if (gl[j]) dst = ns + cl;
+            else dst = ns + dc.nl + (i - cl);
+            const int64_t o = (int64_t)f * (int64_t)A2 + dst;
+            const int64_t p = p0 + j;
+            a.ox[o] = __ldcs(a.lx + p);
+            a.orow[o] = rv[j];
+            a.oy[o] = __ldcs(a.ly + p);
+            cl += gl[j];
+          }
+          ++q;
+        }
+      }
+    }
+  }
+}
+
+// ----------------------------------------------------------------------------- driver --
+
+template <class T>
+cudaError_t dmalloc(T** p, size_t count, cudaStream_t s) {
+  return cudaMallocAsync((void**)p, sizeof(T) * (count ? count : 1), s);
+}
+
+struct Workspace {
+  std::vector<void*> ptrs;
+  cudaStream_t s;
+  ~Workspace() {
+    for (void* p : ptrs) cudaFreeAsync(p, s);
+  }
+  template <class T>
+  cudaError_t get(T** p, size_t count) {
+    cudaError_t e = dmalloc(p, count, s);
+    if (e == cudaSuccess) ptrs.push_back(*p);
+    return e;
+  }
+};
+
+int persistent_grid(const void* kern, int threads, size_t smem) {
+  int per = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, kern, threads, smem);
+  if (per < 1) per = 1;
+  return num_sms() * per;
+}
+
+}  // namespace
+
+dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
+                   int64_t min_leaf, cudaStream_t s, dt_tree** out) {
+  // Pool: keep freed workspace for the next fit (no cudaMalloc on the hot path).
+  {
+    int dev = 0;
+    DT_CK(cudaGetDevice(&dev));
+    cudaMemPool_t pool;
+    DT_CK(cudaDeviceGetDefaultMemPool(&pool, dev));
+    uint64_t thr = UINT64_MAX;
+    DT_CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+  }
+  Workspace ws;
+  ws.s = s;
+  const int64_t total0 = n * (int64_t)d;
+  // node capacities
+  int64_t kcap = n;
+  if (max_depth >= 0 && max_depth < 40) kcap = std::min<int64_t>(kcap, (int64_t)1 << max_depth);
+  int64_t out_cap = 2 * n - 1;
+  if (max_depth >= 0 && max_depth < 40) out_cap = std::min<int64_t>(out_cap, ((int64_t)1 << (max_depth + 1)) - 1);
+  if (out_cap >= ((int64_t)1 << 31)) return fail(DT_ERR_TOO_LARGE, "dt_fit: node array too large");
+  const int64_t max_tiles = (total0 + kTile - 1) / kTile + 1;
+
+  float* lx[2];
+  uint32_t* lr[2];
+  double* ly[2];
+  for (int b = 0; b < 2; ++b) {
+    DT_CK(ws.get(&lx[b], (size_t)total0));
+    DT_CK(ws.get(&lr[b], (size_t)total0));
+    DT_CK(ws.get(&ly[b], (size_t)total0));
+  }
+  NodeL* nodes[2];
+  DT_CK(ws.get(&nodes[0], (size_t)kcap + 1));
+  DT_CK(ws.get(&nodes[1], (size_t)kcap + 1));
+  Decision* dec;
+  uint32_t* new_start;
+  Cand *head_cand, *cont_cand;
+  Stat *head_stat, *cont_stat;
+  DT_CK(ws.get(&dec, (size_t)kcap));
+  DT_CK(ws.get(&new_start, (size_t)kcap));
+  DT_CK(ws.get(&head_cand, (size_t)kcap * d));
+  DT_CK(ws.get(&cont_cand, (size_t)max_tiles));
+  DT_CK(ws.get(&head_stat, (size_t)kcap));
+  DT_CK(ws.get(&cont_stat, (size_t)max_tiles));
+  uint8_t* goleft;
+  DT_CK(ws.get(&goleft, (size_t)n));
+  dt_node* dout;
+  DT_CK(ws.get(&dout, (size_t)out_cap));
+  Ctl* ctl;
+  DT_CK(ws.get(&ctl, 1));
+  DT_CK(cudaMemsetAsync(ctl, 0, sizeof(Ctl), s));
+  // look-back state: [counter | status[max_tiles]] + values
+  uint32_t* lb_status;
+  DT_CK(ws.get(&lb_status, (size_t)max_tiles + 32));
+  SumP *sum_agg, *sum_inc;
+  CntP *cnt_agg, *cnt_inc;
+  DT_CK(ws.get(&sum_agg, (size_t)max_tiles));
+  DT_CK(ws.get(&sum_inc, (size_t)max_tiles));
+  DT_CK(ws.get(&cnt_agg, (size_t)max_tiles));
+  DT_CK(ws.get(&cnt_inc, (size_t)max_tiles));
+
+  LevelLog* lvlog;
+  DT_CK(ws.get(&lvlog, (size_t)kMaxLogLevels));
+
+  // profiling records whose bytes depend on device-side counts: (record, level, kind)
+  struct Pending { int rec, level, kind, dl; };
+  std::vector<Pending> pending;
+
+  // ---- root statistics (a0: N, sum y, min/max, integrality, finiteness, centre)
+  {
+    int64_t chunk = 8192, np = (n + chunk - 1) / chunk;
+    if (np > 2048) { np = 2048; chunk = (n + np - 1) / np; np = (n + chunk - 1) / chunk; }
+    RootPart* parts;
+    double* cparts;
+    DT_CK(ws.get(&parts, (size_t)np));
+    DT_CK(ws.get(&cparts, (size_t)np));
+    const int pr = prof_begin(PK_ROOT, s, 4);
+    root_reduce_kernel<<<(unsigned)np, 256, 0, s>>>(y, n, chunk, parts);
+    root_finalize_kernel<<<1, 32, 0, s>>>(parts, (int)np, n, ctl);
+    root_center_kernel<<<(unsigned)np, 256, 0, s>>>(y, n, chunk, ctl, cparts);
+    root_init_kernel<<<1, 32, 0, s>>>(cparts, (int)np, n, max_depth, min_leaf, ctl, nodes[0]);
+    prof_end(pr, s, 16.0 * (double)n);  // y read twice
+    DT_CK(cudaGetLastError());
+  }
+  // ---- presort (a2): per-feature stable sort of (x, row), SoA level-0 lists
+  {
+    unsigned long long *k_in, *k_out;
+    uint32_t *v_in, *v_out;
+    DT_CK(ws.get(&k_in, (size_t)total0));
+    DT_CK(ws.get(&k_out, (size_t)total0));
+    DT_CK(ws.get(&v_in, (size_t)total0));
+    DT_CK(ws.get(&v_out, (size_t)total0));
+    const int64_t nb = (n + 255) / 256;
+    const size_t smem = sizeof(float) * 256 * (size_t)d;
+    if (smem > 48 * 1024)
+      DT_CK(cudaFuncSetAttribute(presort_keys_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int pr = prof_begin(PK_PRESORT_KEYS, s, 1);
+    presort_keys_kernel<<<(unsigned)nb, 256, smem, s>>>(X, n, d, k_in, v_in, ctl);
+    prof_end(pr, s, 16.0 * (double)total0);  // X read + (key, val) written
+    DT_CK(cudaGetLastError());
+    int fbits = 0;
+    while ((1 << fbits) < d) ++fbits;
+    size_t tmp_bytes = 0;
+    DT_CK(cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, k_in, k_out, v_in, v_out, total0, 0,
+                                          32 + fbits, s));
+    void* tmp;
+    DT_CK(ws.get((char**)&tmp, tmp_bytes));
+    const int passes = (32 + fbits + 7) / 8;
+    pr = prof_begin(PK_PRESORT_SORT, s, 0);  // CUB kernels: library, not counted
+    DT_CK(cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, k_in, k_out, v_in, v_out, total0, 0,
+                                          32 + fbits, s));
+    prof_end(pr, s, 24.0 * (double)total0 * passes);
+    const int gb = std::max(1, std::min<int>((int)((total0 + 255) / 256), num_sms() * 8));
+    pr = prof_begin(PK_PRESORT_BUILD, s, 1);
+    presort_build_kernel<<<gb, 256, 0, s>>>(k_out, v_out, y, total0, lx[0], lr[0], ly[0]);
+    prof_end(pr, s, 36.0 * (double)total0);  // (key, val) read, y gathered, 16 B written
+    DT_CK(cudaGetLastError());
+  }
+
+  const int g_scan = persistent_grid((const void*)scan_kernel, kThreads, 0);
+  const int g_part = persistent_grid((const void*)partition_kernel, kThreads, 0);
+  const int g_sel = num_sms() * 4;
+  const int g_gl = num_sms() * 8;
+  const size_t lb_bytes = sizeof(uint32_t) * ((size_t)max_tiles + 32);
+
+  int cur = 0;
+  for (int level = 0;; ++level) {
+    const int parity = level & 1;
+    const bool last = (max_depth >= 0 && level == max_depth);
+    const int dl = last ? 1 : d;
+    // scan (a4)
+    DT_CK(cudaMemsetAsync(lb_status, 0, lb_bytes, s));
+    ScanArgs sa;
+    sa.lx = lx[cur];
+    sa.ly = ly[cur];
+    sa.nodes = nodes[parity];
+    sa.ctl = ctl;
+    sa.parity = parity;
+    sa.dl = dl;
+    sa.d = d;
+    sa.min_leaf = min_leaf;
+    sa.counter = lb_status;
+    sa.ts = TileSlots<SumP>{lb_status + 32, sum_agg, sum_inc};
+    sa.head_cand = head_cand;
+    sa.cont_cand = cont_cand;
+    sa.head_stat = head_stat;
+    sa.cont_stat = cont_stat;
+    int pr = prof_begin(PK_SCAN, s, 1);
+    scan_kernel<<<g_scan, kThreads, 0, s>>>(sa);
+    prof_end(pr, s, 0.0);
+    pending.push_back({pr, level, PK_SCAN, dl});
+    DT_CK(cudaGetLastError());
+    // select (a5, a8)
+    SelectArgs se;
+    se.lx = lx[cur];
+    se.nodes = nodes[parity];
+    se.ctl = ctl;
+    se.parity = parity;
+    se.level = level;
+    se.dl = dl;
+    se.d = d;
+    se.head_cand = head_cand;
+    se.cont_cand = cont_cand;
+    se.head_stat = head_stat;
+    se.cont_stat = cont_stat;
+    se.dec = dec;
+    se.out = dout;
+    se.log = lvlog;
+    pr = prof_begin(PK_SELECT, s, 1);
+    select_kernel<<<g_sel, 256, 0, s>>>(se);
+    prof_end(pr, s, 0.0);
+    DT_CK(cudaGetLastError());
+    if (last) break;
+    // number (a3, a8)
+    NumberArgs na;
+    na.nodes = nodes[parity];
+    na.next = nodes[parity ^ 1];
+    na.dec = dec;
+    na.new_start = new_start;
+    na.ctl = ctl;
+    na.parity = parity;
+    na.level = level;
+    na.max_depth = max_depth;
+    na.min_leaf = min_leaf;
+    na.out = dout;
+    na.log = lvlog;
+    pr = prof_begin(PK_NUMBER, s, 1);
+    number_kernel<<<1, 1024, 0, s>>>(na);
+    prof_end(pr, s, 0.0);
+    DT_CK(cudaGetLastError());
+    // go-left map (a6)
+    pr = prof_begin(PK_GOLEFT, s, 1);
+    goleft_kernel<<<g_gl, 256, 0, s>>>(lr[cur], nodes[parity], dec, ctl, parity, goleft);
+    prof_end(pr, s, 0.0);
+    pending.push_back({pr, level, PK_GOLEFT, 1});
+    DT_CK(cudaGetLastError());
+    // stable partition (a7)
+    DT_CK(cudaMemsetAsync(lb_status, 0, lb_bytes, s));
+    PartArgs pa;
+    pa.lx = lx[cur];
+    pa.lr = lr[cur];
+    pa.ly = ly[cur];
+    pa.ox = lx[cur ^ 1];
+    pa.orow = lr[cur ^ 1];
+    pa.oy = ly[cur ^ 1];
+    pa.nodes = nodes[parity];
+    pa.dec = dec;
+    pa.new_start = new_start;
+    pa.goleft = goleft;
+    pa.ctl = ctl;
+    pa.parity = parity;
+    pa.dl_in = d;
+    pa.dl_out = (max_depth >= 0 && level + 1 == max_depth) ? 1 : d;
+    pa.counter = lb_status;
+    pa.ts = TileSlots<CntP>{lb_status + 32, cnt_agg, cnt_inc};
+    pr = prof_begin(PK_PARTITION, s, 1);
+    partition_kernel<<<g_part, kThreads, 0, s>>>(pa);
+    prof_end(pr, s, 0.0);
+    pending.push_back({pr, level, PK_PARTITION, pa.dl_out});
+    DT_CK(cudaGetLastError());
+    cur ^= 1;
+    // unlimited depth (or a deep limit): poll the node count every few levels
+    if ((max_depth < 0 || max_depth > 24) && (level % 8) == 7) {
+      uint32_t kk[2];
+      DT_CK(cudaMemcpyAsync(kk, ctl->K, sizeof kk, cudaMemcpyDeviceToHost, s));
+      DT_CK(cudaStreamSynchronize(s));
+      if (kk[parity ^ 1] == 0) break;
+    }
+  }
+  Ctl hc;
+  DT_CK(cudaMemcpyAsync(&hc, ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+  std::vector<LevelLog> hlog;
+  if (!pending.empty()) {
+    hlog.resize(kMaxLogLevels);
+    DT_CK(cudaMemcpyAsync(hlog.data(), lvlog, sizeof(LevelLog) * kMaxLogLevels, cudaMemcpyDeviceToHost, s));
+  }
+  DT_CK(cudaStreamSynchronize(s));
+  // algorithmic bytes per launch:
+  //   scan: every active entry of the scanned lists, x (4 B) + y (8 B);
+  //   goleft: the split feature's row ids of the moved rows (4 B) + one byte per row;
+  //   partition: every moved entry read (16 B) and written (16 B).
+  for (const Pending& p : pending) {
+    if (p.rec < 0 || p.level >= kMaxLogLevels) continue;
+    const LevelLog& L = hlog[(size_t)p.level];
+    double b = 0.0;
+    if (p.kind == PK_SCAN) b = 12.0 * (double)L.A * p.dl;
+    else if (p.kind == PK_GOLEFT) b = 5.0 * (double)L.A_next;
+    else if (p.kind == PK_PARTITION) b = 32.0 * (double)L.A_next * p.dl;
+    prof_set_bytes(p.rec, b);
+  }
+  if (hc.nonfinite) return fail(DT_ERR_NONFINITE, "dt_fit: non-finite value in X or y");
+  const int64_t count = hc.next_id;
+  dt_tree* t = new dt_tree();
+  t->count = count;
+  t->d = d;
+  t->depth = hc.max_depth_seen;
+  t->split_evals = (int64_t)hc.split_evals;
+  t->integer_mode = hc.int_mode;
+  t->host = (dt_node*)malloc(sizeof(dt_node) * (size_t)count);
+  cudaError_t e = cudaMemcpyAsync(t->host, dout, sizeof(dt_node) * (size_t)count,
+                                  cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) {
+    dt_tree_free(t);
+    return cuda_fail(e, "copy tree", __FILE__, __LINE__);
+  }
+  dt_status st = tree_upload(t, s);
+  if (st != DT_OK) {
+    dt_tree_free(t);
+    return st;
+  }
+  *out = t;
+  return DT_OK;
+}
+
+}  // namespace dtl

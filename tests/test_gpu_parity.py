@@ -1,0 +1,258 @@
+"""GPU <-> oracle parity through the C ABI (contract in BASELINE.json):
+
+* structure (feature, threshold, links) bit-exact wherever the exact gap between the
+  best and second-best gain exceeds 1e-12 relative (adjudicated with exact rationals,
+  tests/treecmp.py); in integer mode bit-exact everywhere, including exact ties;
+* node values / metrics within 1e-9 relative (abs floor 1e-12);
+* predictions from an identical tree bit-exact.
+"""
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+import treecmp
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def dt():
+    import paper_conf_ipps_metzgd23_b200 as m
+    return m
+
+
+def _cuda(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def _fit(dt, X, y, D, m):
+    t = dt.dt_fit(_cuda(X.astype(np.float32)), _cuda(y.astype(np.float64)), D, m)
+    torch.cuda.synchronize()
+    return t
+
+
+def _assert_exact(g, o):
+    """Integer mode: identical trees (structure, thresholds, values, counts)."""
+    assert len(g) == len(o)
+    for f in ("feature", "left", "right", "depth", "n_samples", "threshold", "value"):
+        assert np.array_equal(g[f], o[f]), f
+    # impurity: same quantity, summed in a different order
+    np.testing.assert_allclose(g["impurity"], o["impurity"], rtol=1e-9, atol=1e-12)
+
+
+# ------------------------------------------------------------------ predict / eval ----
+
+@pytest.mark.parametrize("n,d,D", [(1, 3, 2), (37, 4, -1), (5000, 16, 12), (100003, 32, 8)])
+def test_predict_bitexact_on_oracle_trees(dt, n, d, D):
+    X, y = datagen.random_table(n, max(n, 50), d, kind="mixed", int_y=False)
+    nodes = oracle.fit(X, y, D, 1)
+    tree = dt.dt_tree_from_nodes(nodes, d)
+    Xq, _ = datagen.random_table(n + 1, n, d, kind="mixed", int_y=False)
+    Xq[: min(n, 10)] = X[: min(n, 10)]  # include training rows (exact threshold hits)
+    got = dt.dt_predict(tree, _cuda(Xq)).cpu().numpy()
+    want = oracle.predict(nodes, Xq)
+    assert np.array_equal(got, want)
+
+
+def test_predict_threshold_boundaries(dt):
+    """Rows exactly at, just below and just above every threshold (f32 neighbours)."""
+    X, y = datagen.random_table(3, 400, 3, kind="continuous", int_y=False)
+    nodes = oracle.fit(X, y, 6, 1)
+    rows = []
+    for nd in nodes:
+        if nd["feature"] < 0:
+            continue
+        t32 = np.float32(nd["threshold"])
+        for v in (t32, np.nextafter(t32, np.float32(-np.inf)), np.nextafter(t32, np.float32(np.inf))):
+            r = X[0].copy()
+            r[nd["feature"]] = v
+            rows.append(r)
+    Xq = np.array(rows, dtype=np.float32)
+    tree = dt.dt_tree_from_nodes(nodes, 3)
+    assert np.array_equal(dt.dt_predict(tree, _cuda(Xq)).cpu().numpy(), oracle.predict(nodes, Xq))
+
+
+def _close(a, b, rel=1e-9, abs_=1e-12):
+    return abs(a - b) <= max(rel * max(abs(a), abs(b)), abs_)
+
+
+@pytest.mark.parametrize("n", [1, 2, 3, 1000, 4096 * 3 + 17, 1_000_000])
+def test_eval_matches_oracle(dt, n):
+    rng = np.random.default_rng(n)
+    y = rng.uniform(1, 1e4, n)
+    yhat = y * (1 + 0.05 * rng.standard_normal(n))
+    if n > 2:
+        y[1] = 0.0  # MAPE epsilon path
+    g = dt.dt_eval(_cuda(y), _cuda(yhat), 4)
+    mape, r2, adj = oracle.evaluate(y, yhat, 4)
+    assert _close(g["mape"], mape)
+    assert _close(g["r2"], r2)
+    assert (np.isnan(adj) and np.isnan(g["adj_r2"])) or _close(g["adj_r2"], adj)
+
+
+def test_eval_special_cases(dt):
+    y = np.arange(1, 101, dtype=np.float64)
+    g = dt.dt_eval(_cuda(y), _cuda(y), 3)
+    assert g["mape"] == 0.0 and g["r2"] == 1.0 and g["adj_r2"] == 1.0
+    c = np.full(50, 7.0)
+    assert dt.dt_eval(_cuda(c), _cuda(c), 1)["r2"] == 1.0
+    assert dt.dt_eval(_cuda(c), _cuda(c + 1), 1)["r2"] == 0.0
+    assert np.isnan(dt.dt_eval(_cuda(y[:3]), _cuda(y[:3] + 1), 2)["adj_r2"])
+
+
+def test_predict_eval_fused(dt):
+    X, y = datagen.cnn_gpu_table(7, 20000)
+    nodes = oracle.fit(X, y, 8, 4)
+    tree = dt.dt_tree_from_nodes(nodes, 16)
+    Xv, yv = datagen.cnn_gpu_table(8, 30001)
+    g = dt.dt_predict_eval(tree, _cuda(Xv), _cuda(yv), 16)
+    mape, r2, adj = oracle.evaluate(yv, oracle.predict(nodes, Xv), 16)
+    assert _close(g["mape"], mape) and _close(g["r2"], r2) and _close(g["adj_r2"], adj)
+
+
+# ------------------------------------------------------------------ fit ----------------
+
+FIT_CASES = []
+for d in (1, 4, 16, 32):
+    for n in (1, 2, 39, 1000, 20000):
+        for kind in ("ties", "continuous"):
+            FIT_CASES.append((d, n, kind))
+
+
+@pytest.mark.parametrize("d,n,kind", FIT_CASES)
+@pytest.mark.parametrize("D,m", [(-1, 1), (0, 1), (1, 2), (3, 7), (12, 1), (12, 64)])
+def test_fit_integer_mode_exact(dt, d, n, kind, D, m):
+    X, y = datagen.random_table(d * 1000 + n, n, d, kind=kind, int_y=True, y_range=50)
+    o, mode = oracle.fit(X, y, D, m, return_mode=True)
+    assert mode
+    g = _fit(dt, X, y, D, m)
+    _assert_exact(g.nodes, o)
+
+
+@pytest.mark.parametrize("d,n,kind", [(4, 1000, "continuous"), (16, 20000, "mixed"),
+                                      (32, 5000, "continuous"), (3, 3000, "ties"), (1, 777, "continuous")])
+@pytest.mark.parametrize("D,m", [(-1, 1), (6, 3), (12, 1)])
+def test_fit_real_mode_contract(dt, d, n, kind, D, m):
+    X, y = datagen.random_table(d * 7 + n, n, d, kind=kind, int_y=False)
+    o = oracle.fit(X, y, D, m)
+    g = _fit(dt, X, y, D, m).nodes
+    st = treecmp.compare(g, o, X, y)
+    assert st["compared"] >= 1
+
+
+def test_fit_collinear_ties_exact(dt):
+    """Duplicated / affinely dependent columns (GPU descriptors): the lowest
+    feature index must win every exact tie, bit-exactly."""
+    for seed in range(5):
+        X, y = datagen.random_table(seed, 3000, 8, kind="collinear", int_y=True)
+        o = oracle.fit(X, y, -1, 1)
+        _assert_exact(_fit(dt, X, y, -1, 1).nodes, o)
+
+
+@pytest.mark.parametrize("n", [4095, 4096, 4097, 8191, 12289])
+def test_fit_tile_boundaries(dt, n):
+    """Segments that start / end exactly on 4096-entry tile boundaries."""
+    X, y = datagen.random_table(n, n, 3, kind="ties", int_y=True)
+    _assert_exact(_fit(dt, X, y, 10, 1).nodes, oracle.fit(X, y, 10, 1))
+
+
+def test_fit_paper_schema_c2_sampled(dt):
+    """BASELINE configs[1] schema at 200k rows (the full 1M case is test_fit_c2_full)."""
+    X, y = datagen.cnn_gpu_table(1, 200_000)
+    o, ev = oracle.fit(X, y, 12, 1, return_evals=True)
+    g = _fit(dt, X, y, 12, 1)
+    _assert_exact(g.nodes, o)
+    assert g.split_evals == ev
+
+
+def test_fit_c2_full(dt):
+    """BASELINE configs[1] at full size (1M x 16, depth 12) in the bench's launch
+    configuration: integer-mode trees must be identical to the oracle's."""
+    X, y = datagen.cnn_gpu_table(1, 1_000_000)
+    o, mode, ev = oracle.fit(X, y, 12, 1, return_mode=True, return_evals=True)
+    assert mode
+    g = _fit(dt, X, y, 12, 1)
+    _assert_exact(g.nodes, o)
+    assert g.split_evals == ev
+    assert g.depth == int(o["depth"].max())
+
+
+def test_fit_real_target_c2_schema(dt):
+    X, y = datagen.cnn_gpu_table(3, 100_000, real=True)
+    o = oracle.fit(X, y, 10, 2)
+    treecmp.compare(_fit(dt, X, y, 10, 2).nodes, o, X, y)
+
+
+def test_fit_deterministic(dt):
+    X, y = datagen.random_table(5, 50000, 8, kind="mixed", int_y=False)
+    a = _fit(dt, X, y, -1, 1).nodes
+    b = _fit(dt, X, y, -1, 1).nodes
+    assert a.tobytes() == b.tobytes()
+
+
+def test_fit_nonfinite_rejected(dt):
+    X, y = datagen.random_table(1, 100, 3)
+    X[5, 1] = np.nan
+    with pytest.raises(dt.DTError) as e:
+        _fit(dt, X, y, 3, 1)
+    assert e.value.status == 2
+    X[5, 1] = 0
+    y[3] = np.inf
+    with pytest.raises(dt.DTError):
+        _fit(dt, X, y, 3, 1)
+
+
+def test_fit_scale_and_negative_zero(dt):
+    X, y = datagen.random_table(2, 2000, 4, kind="ties", int_y=True)
+    X[::3, 0] = -0.0
+    X[1::3, 0] = 0.0
+    o = oracle.fit(X, y, -1, 1)
+    _assert_exact(_fit(dt, X, y, -1, 1).nodes, o)
+    g2 = _fit(dt, X, y * 8.0, -1, 1).nodes
+    assert np.array_equal(g2["value"], o["value"] * 8.0)
+
+
+def test_fit_then_predict_interpolates(dt):
+    X, y = datagen.random_table(9, 5000, 6, kind="continuous", int_y=False)
+    t = _fit(dt, X, y, -1, 1)
+    yh = dt.dt_predict(t, _cuda(X))
+    m = dt.dt_eval(_cuda(y), yh, 6)
+    assert m["mape"] == 0.0 and m["r2"] == 1.0
+
+
+# ------------------------------------------------------------------ LOO ----------------
+
+@pytest.mark.parametrize("seed", range(4))
+def test_loo_paper_table(dt, seed):
+    X, y = datagen.paper_table(seed)
+    got = dt.dt_loo(_cuda(X), _cuda(y), -1, 1).cpu().numpy()
+    want = oracle.loo(X, y, -1, 1)
+    assert np.array_equal(got, want)
+    Xr, yr = datagen.paper_table(seed, real=True)
+    got = dt.dt_loo(_cuda(Xr), _cuda(yr), -1, 1).cpu().numpy()
+    assert np.array_equal(got, oracle.loo(Xr, yr, -1, 1))
+
+
+@pytest.mark.parametrize("n,d,D,m", [(2, 1, -1, 1), (17, 3, 2, 1), (64, 32, -1, 2), (50, 8, 4, 3)])
+def test_loo_random(dt, n, d, D, m):
+    X, y = datagen.random_table(n, n, d, kind="ties", int_y=True)
+    assert np.array_equal(dt.dt_loo(_cuda(X), _cuda(y), D, m).cpu().numpy(), oracle.loo(X, y, D, m))
+
+
+# ------------------------------------------------------------------ generator ----------
+
+@pytest.mark.parametrize("d,real", [(16, False), (16, True), (32, False)])
+def test_generator_bitexact(dt, d, real):
+    for row0, n in ((0, 1000), (123_456_789, 517)):
+        Xg, yg = dt.dt_gen_table(11, n, d=d, real=real, row0=row0)
+        Xh, yh = datagen.cnn_gpu_table(11, n, d=d, real=real, row0=row0)
+        assert np.array_equal(Xg.cpu().numpy(), Xh)
+        assert np.array_equal(yg.cpu().numpy(), yh)
+
+
+def test_dse_generator_bitexact(dt):
+    for row0 in (0, (1 << 30) - 2048):
+        Xg = dt.dt_gen_dse(3, row0, 2048, 10).cpu().numpy()
+        assert np.array_equal(Xg, datagen.dse_candidates(3, row0, 2048))
