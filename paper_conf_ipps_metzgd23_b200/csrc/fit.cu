@@ -272,6 +272,32 @@ __global__ void __launch_bounds__(256) presort_build_kernel(const unsigned long 
 
 // ----------------------------------------------------------------------------- scan ----
 
+// Cursor over the segments of a level's concatenated feature lists: segment (f, k)
+// occupies global positions [f*A + start_k, f*A + start_k + N_k).
+struct Seg {
+  int64_t start, end, fbase;
+  uint32_t k;
+  int f;
+};
+__device__ __forceinline__ void seg_at(Seg& s, const NodeL* __restrict__ nodes, uint32_t K,
+                                       uint64_t A, int64_t p) {
+  s.f = (int)(p / (int64_t)A);
+  s.fbase = (int64_t)s.f * (int64_t)A;
+  s.k = find_node(nodes, K, (uint32_t)(p - s.fbase));
+  s.start = s.fbase + __ldg(&nodes[s.k].start);
+  s.end = s.start + __ldg(&nodes[s.k].N);
+}
+__device__ __forceinline__ void seg_next(Seg& s, const NodeL* __restrict__ nodes, uint32_t K,
+                                         uint64_t A) {
+  if (++s.k == K) {
+    s.k = 0;
+    ++s.f;
+    s.fbase += (int64_t)A;
+  }
+  s.start = s.fbase + __ldg(&nodes[s.k].start);
+  s.end = s.start + __ldg(&nodes[s.k].N);
+}
+
 struct ScanArgs {
   const float* lx;
   const double* ly;
@@ -282,7 +308,8 @@ struct ScanArgs {
   int d;           // feature count (slot stride)
   int64_t min_leaf;
   uint32_t* counter;  // tile counter (zeroed per launch)
-  TileSlots<SumP> ts;
+  uint64_t* lb_agg;   // [ntiles] (kUnpublished before every launch)
+  uint64_t* lb_inc;
   Cand* head_cand;  // [K*d]
   Cand* cont_cand;  // [ntiles]
   Stat* head_stat;  // [K]
@@ -316,12 +343,44 @@ __device__ __forceinline__ double split_gain(double sl, double sc, uint32_t i, u
   return __ddiv_rn(__dmul_rn(D, D), __dmul_rn(__dmul_rn(Nd, nl), nr));
 }
 
-__global__ void __launch_bounds__(kThreads) scan_kernel(ScanArgs a) {
+// Loads kItems consecutive x (f32) and y (f64) entries starting at p0 (vectorised when
+// the whole run is in bounds; p0 is a multiple of kItems, so 16-byte aligned).
+__device__ __forceinline__ void load_items(const float* __restrict__ lx, const double* __restrict__ ly,
+                                           int64_t p0, int64_t total, float* xv, double* yv) {
+  if (p0 + kItems <= total) {
+    const float4* x4 = reinterpret_cast<const float4*>(lx + p0);
+    const double2* y2 = reinterpret_cast<const double2*>(ly + p0);
+#pragma unroll
+    for (int j = 0; j < kItems / 4; ++j) {
+      const float4 t = __ldcs(x4 + j);
+      xv[4 * j] = t.x; xv[4 * j + 1] = t.y; xv[4 * j + 2] = t.z; xv[4 * j + 3] = t.w;
+    }
+#pragma unroll
+    for (int j = 0; j < kItems / 2; ++j) {
+      const double2 t = __ldcs(y2 + j);
+      yv[2 * j] = t.x; yv[2 * j + 1] = t.y;
+    }
+  } else {
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+      const bool ok = p0 + j < total;
+      xv[j] = ok ? lx[p0 + j] : 0.f;
+      yv[j] = ok ? ly[p0 + j] : 0.0;
+    }
+  }
+}
+
+__global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
   __shared__ SumP sh_sum[33];
   __shared__ ArgP sh_arg[33];
   __shared__ StatP sh_stat[33];
+  __shared__ SumP lb_buf[kLookbackMax];
   __shared__ int64_t sh_tile;
   __shared__ SumP sh_carry;
+  // per-thread best of the run before its first head (read back at the flush)
+  __shared__ double fr_gain[kThreads], fr_sl[kThreads], fs_sse[kThreads], fs_min[kThreads],
+      fs_max[kThreads], fs_s1[kThreads];
+  __shared__ uint32_t fr_i[kThreads];
 
   const uint32_t K = a.ctl->K[a.parity];
   const uint64_t A = a.ctl->A[a.parity];
@@ -329,203 +388,162 @@ __global__ void __launch_bounds__(kThreads) scan_kernel(ScanArgs a) {
   const int64_t total = (int64_t)A * a.dl;
   const int64_t ntiles = (total + kTile - 1) / kTile;
   const int tid = threadIdx.x;
+  const uint32_t m = (uint32_t)min(a.min_leaf, (int64_t)0xffffffff);
+  const SumP sum0{0u, 0.0};
+  const ArgP arg0{0u, 0xffffffffu, -1.0, 0.0};
+  const StatP stat0{0u, 0.0, INFINITY, -INFINITY, 0.0};
 
   for (;;) {
     if (tid == 0) sh_tile = (int64_t)atomicAdd(a.counter, 1u);
     __syncthreads();
     const int64_t tile = sh_tile;
-    __syncthreads();
     if (tile >= ntiles) break;
     const int64_t p0 = tile * kTile + (int64_t)tid * kItems;
+    const bool any = p0 < total;
 
-    // ---- locate my first item, load items
     float xv[kItems];
     double yv[kItems];
-    int f0 = 0;
-    uint32_t q0 = 0, k0 = 0;
-    const bool any = p0 < total;
+    Seg sg{0, 0, 0, 0u, 0};
     if (any) {
-      f0 = (int)(p0 / (int64_t)A);
-      q0 = (uint32_t)(p0 - (int64_t)f0 * (int64_t)A);
-      k0 = find_node(a.nodes, K, q0);
-      if (p0 + kItems <= total) {
-        const float4* x4 = reinterpret_cast<const float4*>(a.lx + p0);
-        const double2* y2 = reinterpret_cast<const double2*>(a.ly + p0);
-#pragma unroll
-        for (int j = 0; j < kItems / 4; ++j) {
-          float4 t = __ldcs(x4 + j);
-          xv[4 * j] = t.x; xv[4 * j + 1] = t.y; xv[4 * j + 2] = t.z; xv[4 * j + 3] = t.w;
-        }
-#pragma unroll
-        for (int j = 0; j < kItems / 2; ++j) {
-          double2 t = __ldcs(y2 + j);
-          yv[2 * j] = t.x; yv[2 * j + 1] = t.y;
-        }
-      } else {
-#pragma unroll
-        for (int j = 0; j < kItems; ++j) {
-          const bool ok = p0 + j < total;
-          xv[j] = ok ? a.lx[p0 + j] : 0.f;
-          yv[j] = ok ? a.ly[p0 + j] : 0.0;
-        }
-      }
+      load_items(a.lx, a.ly, p0, total, xv, yv);
+      seg_at(sg, a.nodes, K, A, p0);
     }
 
     // ---- pass 1: thread aggregate of the segmented sum of (y - c)
-    SumP tagg{0u, 0.0};
-    {
-      int f = f0;
-      uint32_t q = q0, k = k0;
-      uint32_t kend = any ? __ldg(&a.nodes[k].start) + __ldg(&a.nodes[k].N) : 0;
-      uint32_t kstart = any ? __ldg(&a.nodes[k].start) : 0;
-      double c = any ? __ldg(&a.nodes[k].c) : 0.0;
+    SumP tagg = sum0;
+    if (any) {
+      Seg s = sg;
+      double c = __ldg(&a.nodes[s.k].c);
 #pragma unroll
       for (int j = 0; j < kItems; ++j) {
-        if (p0 + j < total) {
-          if (q >= (uint32_t)A) { ++f; q = 0; k = 0; kstart = 0; kend = __ldg(&a.nodes[0].N); c = __ldg(&a.nodes[0].c); }
-          while (q >= kend) { ++k; kstart = kend; kend = kstart + __ldg(&a.nodes[k].N); c = __ldg(&a.nodes[k].c); }
+        const int64_t p = p0 + j;
+        if (p < total) {
+          if (p == s.end) {
+            seg_next(s, a.nodes, K, A);
+            c = __ldg(&a.nodes[s.k].c);
+          }
           const double e = __dsub_rn(yv[j], c);
-          if (q == kstart) { tagg.flag = 1u; tagg.s = e; }
+          if (p == s.start) { tagg.flag = 1u; tagg.s = e; }
           else tagg.s = __dadd_rn(tagg.s, e);
-          ++q;
         }
       }
     }
-    // tile's first element is a segment head?
     SumP tile_agg;
-    SumP texcl = block_exclusive_scan(tagg, SumP{0u, 0.0}, tile_agg, sh_sum);
-    if (tid == 0) {
-      const bool head0 = (q0 == __ldg(&a.nodes[k0].start));  // tid 0 is always "any"
-      if (head0 || tile == 0) {
-        publish(a.ts, tile, tile_agg, 2);
-        sh_carry = SumP{0u, 0.0};
+    const SumP texcl = block_exclusive_scan(tagg, sum0, tile_agg, sh_sum);
+    // ---- tile carry: publish the aggregate, look back (warp 0), publish the inclusive
+    if (tid < 32) {
+      const bool head0 = __shfl_sync(0xffffffffu, p0 == sg.start ? 1 : 0, 0) != 0;
+      if (tid == 0) publish(a.lb_agg + tile, tile_agg);
+      if (head0) {
+        if (tid == 0) {
+          publish(a.lb_inc + tile, tile_agg);
+          sh_carry = sum0;
+        }
       } else {
-        publish(a.ts, tile, tile_agg, 1);
-        SumP carry = lookback(a.ts, tile, SumP{0u, 0.0});
-        publish(a.ts, tile, combine(carry, tile_agg), 2);
-        sh_carry = carry;
+        const int64_t stop_tile = __shfl_sync(0xffffffffu, sg.start, 0) / kTile;
+        const SumP carry = warp_lookback(a.lb_agg, a.lb_inc, tile, stop_tile, lb_buf);
+        if (tid == 0) {
+          publish(a.lb_inc + tile, combine(carry, tile_agg));
+          sh_carry = carry;
+        }
       }
     }
     __syncthreads();
-    const SumP carry = sh_carry;
-    // my exclusive prefix value at item 0 (meaningless if item 0 is a head)
-    double S = combine(carry, texcl).s;
+    double S = combine(sh_carry, texcl).s;  // exclusive prefix at my item 0
 
     // ---- pass 2: prefixes, gains, per-run best; flush runs that end in this thread
-    ArgP run{0u, 0xffffffffu, -1.0, 0.0};   // current run's best
-    StatP srun{0u, 0.0, INFINITY, -INFINITY};
-    bool seen_head = false;                  // a head occurred in this thread
-    ArgP first_run{0u, 0xffffffffu, -1.0, 0.0};
-    StatP first_srun{0u, 0.0, INFINITY, -INFINITY};
-    // open-segment identity at the end of this thread
-    int last_f = f0;
-    uint32_t last_k = k0;
+    ArgP run = arg0;
+    StatP srun = stat0;
+    bool seen_head = false;
+    int last_f = sg.f;
+    uint32_t last_k = sg.k;
     const bool stats_tile = (tile * kTile) < (int64_t)A;  // tile holds feature-0 items
-    {
-      int f = f0;
-      uint32_t q = q0, k = k0;
-      uint32_t kstart = any ? __ldg(&a.nodes[k].start) : 0;
-      uint32_t N = any ? __ldg(&a.nodes[k].N) : 0;
-      uint32_t kend = kstart + N;
-      double c = any ? __ldg(&a.nodes[k].c) : 0.0;
-      double sc = any ? __ldg(&a.nodes[k].sc) : 0.0;
-      double v = any ? __ldg(&a.nodes[k].v) : 0.0;
-      int srch = any ? __ldg(&a.nodes[k].searchable) : 0;
-      float xprev = (any && q0 > kstart) ? a.lx[p0 - 1] : 0.f;
-      const uint32_t m = (uint32_t)min(a.min_leaf, (int64_t)0xffffffff);
+    if (any) {
+      Seg s = sg;
+      double nc = __ldg(&a.nodes[s.k].c), nsc = __ldg(&a.nodes[s.k].sc), nv = __ldg(&a.nodes[s.k].v);
+      uint32_t nN = __ldg(&a.nodes[s.k].N);
+      int nsrch = __ldg(&a.nodes[s.k].searchable);
+      float xprev = (p0 > sg.start) ? a.lx[p0 - 1] : 0.f;
 #pragma unroll
       for (int j = 0; j < kItems; ++j) {
-        if (p0 + j < total) {
-          bool newseg = false;
-          if (q >= (uint32_t)A) { ++f; q = 0; k = 0; kstart = 0; newseg = true; }
-          else if (q >= kend) { ++k; kstart = kend; newseg = true; }
-          if (newseg) {
-            while (true) {
-              N = __ldg(&a.nodes[k].N);
-              kend = kstart + N;
-              if (q < kend) break;
-              ++k; kstart = kend;
-            }
-            c = __ldg(&a.nodes[k].c);
-            sc = __ldg(&a.nodes[k].sc);
-            v = __ldg(&a.nodes[k].v);
-            srch = __ldg(&a.nodes[k].searchable);
+        const int64_t p = p0 + j;
+        if (p < total) {
+          if (p == s.end) {
+            seg_next(s, a.nodes, K, A);
+            nc = __ldg(&a.nodes[s.k].c);
+            nsc = __ldg(&a.nodes[s.k].sc);
+            nv = __ldg(&a.nodes[s.k].v);
+            nN = __ldg(&a.nodes[s.k].N);
+            nsrch = __ldg(&a.nodes[s.k].searchable);
           }
-          const bool head = (q == kstart);
-          if (head) {
-            // close the run before this head
-            if (!seen_head) { first_run = run; first_srun = srun; }
-            else {
-              // a run strictly inside this thread: complete segment, started in this tile
-              const int pf = (k == 0) ? f - 1 : f;            // previous segment
-              const uint32_t pkk = (k == 0) ? (K - 1) : k - 1;
-              write_cand(a.head_cand + (int64_t)pkk * a.d + pf, run);
-              if (pf == 0) write_stat(a.head_stat + pkk, srun);
+          if (p == s.start) {
+            if (!seen_head) {
+              fr_gain[tid] = run.gain; fr_sl[tid] = run.sl; fr_i[tid] = run.i;
+              fs_sse[tid] = srun.sse; fs_min[tid] = srun.ymin; fs_max[tid] = srun.ymax;
+              fs_s1[tid] = srun.s1;
+            } else {
+              // the previous run is a whole segment that started in this thread
+              const int pf = (s.k == 0) ? s.f - 1 : s.f;
+              const uint32_t pk = (s.k == 0) ? (K - 1) : s.k - 1;
+              write_cand(a.head_cand + (int64_t)pk * a.d + pf, run);
+              if (pf == 0) write_stat(a.head_stat + pk, srun);
             }
             seen_head = true;
-            run = ArgP{1u, 0xffffffffu, -1.0, 0.0};
-            srun = StatP{1u, 0.0, INFINITY, -INFINITY, 0.0};
+            run = arg0;
+            run.flag = 1u;
+            srun = stat0;
+            srun.flag = 1u;
             S = 0.0;
           }
-          const uint32_t i = q - kstart;
-          const float x = xv[j];
-          if (srch && i >= m && N - i >= m && i >= 1) {
+          const uint32_t i = (uint32_t)(p - s.start);
+          if (nsrch && i >= 1 && i >= m && nN - i >= m) {
             const float xp = (j == 0) ? xprev : xv[j - 1];
-            if (xp < x) {
-              const double g = split_gain(S, sc, i, N);
+            if (xp < xv[j]) {
+              const double g = split_gain(S, nsc, i, nN);
               if (g > run.gain) { run.gain = g; run.i = i; run.sl = S; }
             }
           }
-          const double e = __dsub_rn(yv[j], c);
+          const double e = __dsub_rn(yv[j], nc);
           S = __dadd_rn(S, e);
-          if (f == 0) {
-            const double ev = __dsub_rn(yv[j], v);
+          if (s.f == 0) {
+            const double ev = __dsub_rn(yv[j], nv);
             srun.sse = __dadd_rn(srun.sse, __dmul_rn(ev, ev));
             srun.ymin = fmin(srun.ymin, yv[j]);
             srun.ymax = fmax(srun.ymax, yv[j]);
             srun.s1 = __dadd_rn(srun.s1, e);
           }
-          ++q;
-          last_f = f;
-          last_k = k;
+          last_f = s.f;
+          last_k = s.k;
         }
       }
     }
-    if (!seen_head) { first_run = run; first_srun = srun; }
-    // trailing run of this thread (flag = any head in this thread)
     ArgP trail = run;
     trail.flag = seen_head ? 1u : 0u;
     StatP strail = srun;
     strail.flag = seen_head ? 1u : 0u;
 
     ArgP arg_blk;
-    const ArgP aex = block_exclusive_scan(trail, ArgP{0u, 0xffffffffu, -1.0, 0.0}, arg_blk, sh_arg);
-    StatP sex{0u, 0.0, INFINITY, -INFINITY}, st_blk;
-    if (stats_tile) sex = block_exclusive_scan(strail, StatP{0u, 0.0, INFINITY, -INFINITY, 0.0}, st_blk, sh_stat);
+    const ArgP aex = block_exclusive_scan(trail, arg0, arg_blk, sh_arg);
+    StatP sex = stat0, st_blk;
+    if (stats_tile) sex = block_exclusive_scan(strail, stat0, st_blk, sh_stat);
 
     // Flush the open segment that ends at my first head (its earlier part is in aex).
     if (any && seen_head) {
-      // does my first item start a segment?  then the open segment ended before me
-      ArgP done_a;
-      StatP done_s;
-      const bool item0_head = (q0 == __ldg(&a.nodes[k0].start));
+      const bool item0_head = (p0 == sg.start);
       if (!(tid == 0 && item0_head)) {
-        // open segment identity: the segment containing the item before my first head
         int of;
         uint32_t ok;
-        if (!item0_head) { of = f0; ok = k0; }
-        else if (k0 > 0) { of = f0; ok = k0 - 1; }
-        else { of = f0 - 1; ok = K - 1; }
-        ArgP fr = first_run;
-        fr.flag = 0u;
-        done_a = combine(aex, fr);
+        if (!item0_head) { of = sg.f; ok = sg.k; }
+        else if (sg.k > 0) { of = sg.f; ok = sg.k - 1; }
+        else { of = sg.f - 1; ok = K - 1; }
+        const ArgP fr{0u, fr_i[tid], fr_gain[tid], fr_sl[tid]};
+        const ArgP done_a = combine(aex, fr);
         const bool head_in_tile = aex.flag != 0;
         if (head_in_tile) write_cand(a.head_cand + (int64_t)ok * a.d + of, done_a);
         else write_cand(a.cont_cand + tile, done_a);
         if (stats_tile && of == 0) {
-          StatP fs = first_srun;
-          fs.flag = 0u;
-          done_s = combine(sex, fs);
+          const StatP fs{0u, fs_sse[tid], fs_min[tid], fs_max[tid], fs_s1[tid]};
+          const StatP done_s = combine(sex, fs);
           if (head_in_tile) write_stat(a.head_stat + ok, done_s);
           else write_stat(a.cont_stat + tile, done_s);
         }
@@ -533,18 +551,24 @@ __global__ void __launch_bounds__(kThreads) scan_kernel(ScanArgs a) {
     }
     // The last thread closes the segment open at the tile end.
     if (tid == kThreads - 1) {
-      // find the segment of the tile's last valid element
-      const int64_t plast = min(total, tile * kTile + kTile) - 1;
-      const int lf = (int)(plast / (int64_t)A);
-      const uint32_t lq = (uint32_t)(plast - (int64_t)lf * (int64_t)A);
-      const uint32_t lk = any ? last_k : find_node(a.nodes, K, lq);
-      const int lff = any ? last_f : lf;
-      ArgP done_a = seen_head ? run : combine(aex, ArgP{0u, run.i, run.gain, run.sl});
+      uint32_t lk = last_k;
+      int lff = last_f;
+      if (!any) {
+        Seg t;
+        seg_at(t, a.nodes, K, A, min(total, tile * kTile + kTile) - 1);
+        lk = t.k;
+        lff = t.f;
+      }
+      ArgP tr = run;
+      tr.flag = 0u;
+      const ArgP done_a = seen_head ? run : combine(aex, tr);
       const bool head_in_tile = seen_head || aex.flag != 0;
       if (head_in_tile) write_cand(a.head_cand + (int64_t)lk * a.d + lff, done_a);
       else write_cand(a.cont_cand + tile, done_a);
       if (stats_tile && lff == 0) {
-        StatP done_s = seen_head ? srun : combine(sex, StatP{0u, srun.sse, srun.ymin, srun.ymax, srun.s1});
+        StatP ts = srun;
+        ts.flag = 0u;
+        const StatP done_s = seen_head ? srun : combine(sex, ts);
         if (head_in_tile) write_stat(a.head_stat + lk, done_s);
         else write_stat(a.cont_stat + tile, done_s);
       }
@@ -852,13 +876,15 @@ struct PartArgs {
   int dl_in;   // lists in the input (d)
   int dl_out;  // lists to write (d, or 1 before the last level)
   uint32_t* counter;
-  TileSlots<CntP> ts;
+  uint64_t* lb_agg;
+  uint64_t* lb_inc;
 };
 
 // Stable partition of each (node, feature) segment: left rows first then right rows,
 // order preserved; rows of nodes that did not split are dropped.
-__global__ void __launch_bounds__(kThreads) partition_kernel(PartArgs a) {
+__global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
   __shared__ CntP sh[33];
+  __shared__ CntP lb_buf[kLookbackMax];
   __shared__ int64_t sh_tile;
   __shared__ CntP sh_carry;
   const uint32_t K = a.ctl->K[a.parity];
@@ -868,93 +894,103 @@ __global__ void __launch_bounds__(kThreads) partition_kernel(PartArgs a) {
   const int64_t total = (int64_t)A * a.dl_out;  // only the lists we write
   const int64_t ntiles = (total + kTile - 1) / kTile;
   const int tid = threadIdx.x;
+  const CntP cnt0{0u, 0u};
   for (;;) {
     if (tid == 0) sh_tile = (int64_t)atomicAdd(a.counter, 1u);
     __syncthreads();
     const int64_t tile = sh_tile;
-    __syncthreads();
     if (tile >= ntiles) break;
     const int64_t p0 = tile * kTile + (int64_t)tid * kItems;
     const bool any = p0 < total;
-    int f0 = 0;
-    uint32_t q0 = 0, k0 = 0;
     uint32_t rv[kItems];
-    uint8_t gl[kItems];
+    uint32_t glbits = 0;  // go-left flag per item
+    Seg sg{0, 0, 0, 0u, 0};
+    CntP tagg = cnt0;
     if (any) {
-      f0 = (int)(p0 / (int64_t)A);
-      q0 = (uint32_t)(p0 - (int64_t)f0 * (int64_t)A);
-      k0 = find_node(a.nodes, K, q0);
-    }
-    // pass 1: go-left flags and thread aggregate
-    CntP tagg{0u, 0u};
-    {
-      int f = f0;
-      uint32_t q = q0, k = k0;
-      uint32_t kstart = any ? a.nodes[k].start : 0, kend = any ? kstart + a.nodes[k].N : 0;
-      bool split = any ? (a.dec[k].f >= 0) : false;
+      seg_at(sg, a.nodes, K, A, p0);
+      Seg s = sg;
+      bool split = __ldg(&a.dec[s.k].f) >= 0;
+      if (p0 + kItems <= total) {
+        const uint4* r4 = reinterpret_cast<const uint4*>(a.lr + p0);
+#pragma unroll
+        for (int j = 0; j < kItems / 4; ++j) {
+          const uint4 t = __ldcs(r4 + j);
+          rv[4 * j] = t.x; rv[4 * j + 1] = t.y; rv[4 * j + 2] = t.z; rv[4 * j + 3] = t.w;
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) rv[j] = (p0 + j < total) ? a.lr[p0 + j] : 0u;
+      }
 #pragma unroll
       for (int j = 0; j < kItems; ++j) {
-        gl[j] = 0;
-        rv[j] = 0;
-        if (p0 + j < total) {
-          if (q >= (uint32_t)A) { ++f; q = 0; k = 0; kstart = 0; kend = a.nodes[0].N; split = a.dec[0].f >= 0; }
-          while (q >= kend) { ++k; kstart = kend; kend = kstart + a.nodes[k].N; split = a.dec[k].f >= 0; }
-          const bool head = q == kstart;
-          uint32_t g = 0;
-          if (split) {
-            rv[j] = __ldcs(a.lr + p0 + j);
-            g = a.goleft[rv[j]];
+        const int64_t p = p0 + j;
+        if (p < total) {
+          if (p == s.end) {
+            seg_next(s, a.nodes, K, A);
+            split = __ldg(&a.dec[s.k].f) >= 0;
           }
-          gl[j] = (uint8_t)g;
-          if (head) { tagg.flag = 1u; tagg.c = g; }
+          uint32_t g = 0;
+          if (split) g = __ldg(a.goleft + rv[j]);
+          glbits |= g << j;
+          if (p == s.start) { tagg.flag = 1u; tagg.c = g; }
           else tagg.c += g;
-          ++q;
         }
       }
     }
     CntP tile_agg;
-    CntP texcl = block_exclusive_scan(tagg, CntP{0u, 0u}, tile_agg, sh);
-    if (tid == 0) {
-      const bool head0 = (q0 == a.nodes[k0].start);
-      if (head0 || tile == 0) {
-        publish(a.ts, tile, tile_agg, 2);
-        sh_carry = CntP{0u, 0u};
+    const CntP texcl = block_exclusive_scan(tagg, cnt0, tile_agg, sh);
+    if (tid < 32) {
+      const bool head0 = __shfl_sync(0xffffffffu, p0 == sg.start ? 1 : 0, 0) != 0;
+      if (tid == 0) publish(a.lb_agg + tile, tile_agg);
+      if (head0) {
+        if (tid == 0) {
+          publish(a.lb_inc + tile, tile_agg);
+          sh_carry = cnt0;
+        }
       } else {
-        publish(a.ts, tile, tile_agg, 1);
-        CntP carry = lookback(a.ts, tile, CntP{0u, 0u});
-        publish(a.ts, tile, combine(carry, tile_agg), 2);
-        sh_carry = carry;
+        const int64_t stop_tile = __shfl_sync(0xffffffffu, sg.start, 0) / kTile;
+        const CntP carry = warp_lookback(a.lb_agg, a.lb_inc, tile, stop_tile, lb_buf);
+        if (tid == 0) {
+          publish(a.lb_inc + tile, combine(carry, tile_agg));
+          sh_carry = carry;
+        }
       }
     }
     __syncthreads();
     uint32_t cl = combine(sh_carry, texcl).c;  // lefts before my item 0 in its segment
     if (any) {
-      int f = f0;
-      uint32_t q = q0, k = k0;
-      uint32_t kstart = a.nodes[k].start, kend = kstart + a.nodes[k].N;
-      Decision dc = a.dec[k];
-      uint32_t ns = a.new_start[k];
+      float xv[kItems];
+      double yv[kItems];
+      load_items(a.lx, a.ly, p0, total, xv, yv);
+      Seg s = sg;
+      Decision dc = a.dec[s.k];
+      uint32_t ns = __ldg(&a.new_start[s.k]);
+      int64_t obase = (int64_t)s.f * (int64_t)A2;
 #pragma unroll
       for (int j = 0; j < kItems; ++j) {
-        if (p0 + j < total) {
-          bool nseg = false;
-          if (q >= (uint32_t)A) { ++f; q = 0; k = 0; kstart = 0; kend = a.nodes[0].N; nseg = true; }
-          while (q >= kend) { ++k; kstart = kend; kend = kstart + a.nodes[k].N; nseg = true; }
-          if (nseg) { dc = a.dec[k]; ns = a.new_start[k]; }
-          if (q == kstart) cl = 0;
-          if (dc.f >= 0) {
-            const uint32_t i = q - kstart;
-            uint32_t dst;
-            if (gl[j]) dst = ns + cl;
-            else dst = ns + dc.nl + (i - cl);
-            const int64_t o = (int64_t)f * (int64_t)A2 + dst;
-            const int64_t p = p0 + j;
-            a.ox[o] = __ldcs(a.lx + p);
-            a.orow[o] = rv[j];
-            a.oy[o] = __ldcs(a.ly + p);
-            cl += gl[j];
+        const int64_t p = p0 + j;
+        if (p < total) {
+          if (p == s.end) {
+            seg_next(s, a.nodes, K, A);
+            dc = a.dec[s.k];
+            ns = __ldg(&a.new_start[s.k]);
+            obase = (int64_t)s.f * (int64_t)A2;
           }
-          ++q;
+          if (p == s.start) cl = 0;
+          if (dc.f >= 0) {
+            const uint32_t i = (uint32_t)(p - s.start);
+            const uint32_t g = (glbits >> j) & 1u;
+            const uint32_t dst = g ? ns + cl : ns + dc.nl + (i - cl);
+            const int64_t o = obase + dst;
+#ifdef DT_DEBUG_PART
+            if (dst >= A2) printf("BAD tile %lld tid %d j %d p %lld k %u f %d start %lld end %lld i %u cl %u g %u ns %u nl %u A2 %llu carry %u/%u texcl %u/%u\n",
+              (long long)tile, tid, j, (long long)p, s.k, s.f, (long long)s.start, (long long)s.end, i, cl, g, ns, dc.nl, (unsigned long long)A2, sh_carry.flag, sh_carry.c, texcl.flag, texcl.c);
+#endif
+            a.ox[o] = xv[j];
+            a.orow[o] = rv[j];
+            a.oy[o] = yv[j];
+            cl += g;
+          }
         }
       }
     }
@@ -1044,12 +1080,9 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
   // look-back state: [counter | status[max_tiles]] + values
   uint32_t* lb_status;
   DT_CK(ws.get(&lb_status, (size_t)max_tiles + 32));
-  SumP *sum_agg, *sum_inc;
-  CntP *cnt_agg, *cnt_inc;
-  DT_CK(ws.get(&sum_agg, (size_t)max_tiles));
-  DT_CK(ws.get(&sum_inc, (size_t)max_tiles));
-  DT_CK(ws.get(&cnt_agg, (size_t)max_tiles));
-  DT_CK(ws.get(&cnt_inc, (size_t)max_tiles));
+  // tile descriptors (agg | inc), zeroed with the counter before every launch
+  uint64_t* lb_desc;
+  DT_CK(ws.get(&lb_desc, 2 * (size_t)max_tiles));
 
   LevelLog* lvlog;
   DT_CK(ws.get(&lvlog, (size_t)kMaxLogLevels));
@@ -1113,7 +1146,8 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
   const int g_part = persistent_grid((const void*)partition_kernel, kThreads, 0);
   const int g_sel = num_sms() * 4;
   const int g_gl = num_sms() * 8;
-  const size_t lb_bytes = sizeof(uint32_t) * ((size_t)max_tiles + 32);
+  const size_t lb_bytes = sizeof(uint32_t) * 32;
+  const size_t desc_bytes = sizeof(uint64_t) * 2 * (size_t)max_tiles;
 
   int cur = 0;
   for (int level = 0;; ++level) {
@@ -1122,6 +1156,7 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     const int dl = last ? 1 : d;
     // scan (a4)
     DT_CK(cudaMemsetAsync(lb_status, 0, lb_bytes, s));
+    DT_CK(cudaMemsetAsync(lb_desc, 0xFF, desc_bytes, s));
     ScanArgs sa;
     sa.lx = lx[cur];
     sa.ly = ly[cur];
@@ -1132,7 +1167,8 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     sa.d = d;
     sa.min_leaf = min_leaf;
     sa.counter = lb_status;
-    sa.ts = TileSlots<SumP>{lb_status + 32, sum_agg, sum_inc};
+    sa.lb_agg = lb_desc;
+    sa.lb_inc = lb_desc + max_tiles;
     sa.head_cand = head_cand;
     sa.cont_cand = cont_cand;
     sa.head_stat = head_stat;
@@ -1188,6 +1224,7 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     DT_CK(cudaGetLastError());
     // stable partition (a7)
     DT_CK(cudaMemsetAsync(lb_status, 0, lb_bytes, s));
+    DT_CK(cudaMemsetAsync(lb_desc, 0xFF, desc_bytes, s));
     PartArgs pa;
     pa.lx = lx[cur];
     pa.lr = lr[cur];
@@ -1204,7 +1241,8 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     pa.dl_in = d;
     pa.dl_out = (max_depth >= 0 && level + 1 == max_depth) ? 1 : d;
     pa.counter = lb_status;
-    pa.ts = TileSlots<CntP>{lb_status + 32, cnt_agg, cnt_inc};
+    pa.lb_agg = lb_desc;
+    pa.lb_inc = lb_desc + max_tiles;
     pr = prof_begin(PK_PARTITION, s, 1);
     partition_kernel<<<g_part, kThreads, 0, s>>>(pa);
     prof_end(pr, s, 0.0);

@@ -141,61 +141,86 @@ __device__ __forceinline__ T block_exclusive_scan(T v, const T& ident, T& agg, T
 }
 
 // ------------------------------------------------------------------ look-back ------
+//
+// Each tile publishes two 64-bit words with single-copy-atomic relaxed 64-bit stores:
+// agg[t] = the payload of the tile's own segmented aggregate, inc[t] = the payload of its
+// inclusive prefix.  Both arrays are filled with kUnpublished (all ones: never the bits
+// of a finite f64 sum nor of a u32 count) before every launch.  No flags are needed:
+// a tile whose first element is not a segment head looks back exactly to the tile that
+// holds the head of that segment (`stop_tile`), and every tile in between lies inside
+// the segment.
 
-// Per-tile status word: 0 = nothing, 1 = aggregate published, 2 = inclusive published.
-__device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p) {
-  uint32_t v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+constexpr uint64_t kUnpublished = ~0ull;
+
+// Morally-strong relaxed accesses: single-copy atomic 64-bit words (weak .cg accesses
+// carry no such guarantee and were observed torn), no fence, no L1 invalidation.
+__device__ __forceinline__ void st_cg_u64(uint64_t* p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t ld_cg_u64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
-__device__ __forceinline__ void st_release(uint32_t* p, uint32_t v) {
-  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+
+__device__ __forceinline__ uint64_t payload_bits(const SumP& v) { return (uint64_t)__double_as_longlong(v.s); }
+__device__ __forceinline__ uint64_t payload_bits(const CntP& v) { return (uint64_t)v.c; }
+__device__ __forceinline__ void from_bits(SumP& v, uint64_t b) { v.s = __longlong_as_double((long long)b); }
+__device__ __forceinline__ void from_bits(CntP& v, uint64_t b) { v.c = (uint32_t)b; }
+// unflagged fold of two payloads (no segment head between them)
+__device__ __forceinline__ SumP fold(const SumP& a, const SumP& b) { return SumP{0u, __dadd_rn(a.s, b.s)}; }
+__device__ __forceinline__ CntP fold(const CntP& a, const CntP& b) { return CntP{0u, a.c + b.c}; }
+
+template <class T>
+__device__ __forceinline__ void publish(uint64_t* slot, const T& v) {
+  st_cg_u64(slot, payload_bits(v));
 }
 
-template <class T>
-struct TileSlots {
-  uint32_t* status;  // [ntiles]
-  T* agg;            // [ntiles]
-  T* inc;            // [ntiles]
-};
+constexpr int kLookbackMax = 256;  // predecessor values buffered per look-back (smem)
 
+// Called by ONE WARP (all 32 lanes).  Returns (on lane 0, flag 0) the exclusive carry of
+// `tile`: the strict left-to-right fold of the payloads of tiles stop..tile-1, starting
+// from the nearest one that holds a final value (its inclusive prefix, or stop_tile's
+// aggregate).  32 predecessors are polled per step; values are buffered in `buf` and
+// folded in tile order by lane 0, so the result does not depend on timing.
 template <class T>
-__device__ __forceinline__ T ldcg(const T* p) {
-  // L1-bypassing load of a small POD (values published by other CTAs).
-  static_assert(sizeof(T) % 4 == 0, "POD of 32-bit words");
-  T r;
-  const uint32_t* s = reinterpret_cast<const uint32_t*>(p);
-  uint32_t* d = reinterpret_cast<uint32_t*>(&r);
-#pragma unroll
-  for (int i = 0; i < (int)(sizeof(T) / 4); ++i) d[i] = __ldcg(s + i);
-  return r;
-}
-
-template <class T>
-__device__ __forceinline__ void publish(TileSlots<T> ts, int64_t tile, const T& v, uint32_t state) {
-  if (state == 1) ts.agg[tile] = v;
-  else ts.inc[tile] = v;
-  __threadfence();
-  st_release(ts.status + tile, state);
-}
-
-// Called by ONE thread.  Returns the exclusive carry for `tile`: the strict left-to-right
-// fold of every predecessor tile back to the nearest one holding a final value (status 2,
-// or an aggregate that contains a segment head; tile 0's predecessor is the identity).
-template <class T>
-__device__ T lookback(TileSlots<T> ts, int64_t tile, const T& ident) {
-  int64_t t = tile - 1;
-  uint32_t st = 0;
-  while (t >= 0) {
-    do { st = ld_acquire(ts.status + t); } while (st == 0);
-    if (st == 2) break;
-    if (ldcg(ts.agg + t).flag) break;
-    --t;
+__device__ T warp_lookback(const uint64_t* agg, const uint64_t* inc, int64_t tile,
+                           int64_t stop_tile, T* buf) {
+  const int lane = threadIdx.x & 31;
+  for (;;) {
+    int64_t base = tile - 1;
+    int nbuf = 0, stop = -1;
+    while (nbuf + 32 <= kLookbackMax) {
+      const int64_t t = base - lane;
+      bool fin = true;
+      T val;
+      val.flag = 0u;
+      from_bits(val, 0ull);
+      if (t >= stop_tile) {
+        uint64_t av;
+        while ((av = ld_cg_u64(agg + t)) == kUnpublished) {}
+        const uint64_t iv = ld_cg_u64(inc + t);
+        fin = (iv != kUnpublished) || (t == stop_tile);
+        from_bits(val, (iv != kUnpublished) ? iv : av);
+      }
+      const unsigned m = __ballot_sync(0xffffffffu, fin);
+      const int first = m ? (__ffs(m) - 1) : 31;
+      if (lane <= first) buf[nbuf + lane] = val;
+      nbuf += first + 1;
+      if (m) { stop = nbuf - 1; break; }
+      base -= 32;
+    }
+    __syncwarp();
+    if (stop >= 0) {
+      T acc = buf[stop];
+      if (lane == 0)
+        for (int j = stop - 1; j >= 0; --j) acc = fold(acc, buf[j]);
+      __syncwarp();
+      acc.flag = 0u;
+      return acc;
+    }
+    __nanosleep(500);  // chain longer than the buffer: wait for predecessors, retry
   }
-  T acc = ident;
-  if (t >= 0) acc = (st == 2) ? ldcg(ts.inc + t) : ldcg(ts.agg + t);
-  for (int64_t u = t + 1; u < tile; ++u) acc = combine(acc, ldcg(ts.agg + u));
-  return acc;
 }
 
 }  // namespace dtl
