@@ -882,6 +882,15 @@ struct PartArgs {
 
 // Stable partition of each (node, feature) segment: left rows first then right rows,
 // order preserved; rows of nodes that did not split are dropped.
+//
+// Warp-striped: warp w of a tile owns entries [w*512, w*512 + 512) as 16 rows of 32
+// consecutive entries (lane = position in the row).  Within a row the left/right rank
+// of every entry comes from two ballots (go-left mask, segment-head mask), so each
+// child's entries of a row are written to consecutive addresses (coalesced stores).
+// Carries: row -> row inside the warp, warp -> warp by a block scan, tile -> tile by
+// the decoupled look-back (integer counts).
+constexpr int kRows = kTile / kThreads;  // 16 rows of 32 per warp
+
 __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
   __shared__ CntP sh[33];
   __shared__ CntP lb_buf[kLookbackMax];
@@ -893,54 +902,79 @@ __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
   if (K == 0 || A2 == 0) return;
   const int64_t total = (int64_t)A * a.dl_out;  // only the lists we write
   const int64_t ntiles = (total + kTile - 1) / kTile;
-  const int tid = threadIdx.x;
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  const uint32_t lt_mask = (1u << lane) - 1u;
   const CntP cnt0{0u, 0u};
   for (;;) {
     if (tid == 0) sh_tile = (int64_t)atomicAdd(a.counter, 1u);
     __syncthreads();
     const int64_t tile = sh_tile;
     if (tile >= ntiles) break;
-    const int64_t p0 = tile * kTile + (int64_t)tid * kItems;
-    const bool any = p0 < total;
-    uint32_t rv[kItems];
-    uint32_t glbits = 0;  // go-left flag per item
-    Seg sg{0, 0, 0, 0u, 0};
-    CntP tagg = cnt0;
-    if (any) {
-      seg_at(sg, a.nodes, K, A, p0);
-      Seg s = sg;
-      bool split = __ldg(&a.dec[s.k].f) >= 0;
-      if (p0 + kItems <= total) {
-        const uint4* r4 = reinterpret_cast<const uint4*>(a.lr + p0);
+    const int64_t wbase = tile * kTile + (int64_t)w * (kRows * 32);
+    // ---- load rows / x / y (coalesced rows of 32), go-left flags, head flags
+    uint32_t rv[kRows];
+    float xv[kRows];
+    double yv[kRows];
+    uint32_t gbits = 0, hbits = 0, sbits = 0;  // per row: go-left, head, node split
+    Seg s{0, 0, 0, 0u, 0};
+    const bool wany = wbase < total;
+    if (wany) seg_at(s, a.nodes, K, A, min(wbase + lane, total - 1));
+    const Seg s0 = s;
 #pragma unroll
-        for (int j = 0; j < kItems / 4; ++j) {
-          const uint4 t = __ldcs(r4 + j);
-          rv[4 * j] = t.x; rv[4 * j + 1] = t.y; rv[4 * j + 2] = t.z; rv[4 * j + 3] = t.w;
-        }
-      } else {
-#pragma unroll
-        for (int j = 0; j < kItems; ++j) rv[j] = (p0 + j < total) ? a.lr[p0 + j] : 0u;
-      }
-#pragma unroll
-      for (int j = 0; j < kItems; ++j) {
-        const int64_t p = p0 + j;
-        if (p < total) {
-          if (p == s.end) {
-            seg_next(s, a.nodes, K, A);
-            split = __ldg(&a.dec[s.k].f) >= 0;
-          }
-          uint32_t g = 0;
-          if (split) g = __ldg(a.goleft + rv[j]);
-          glbits |= g << j;
-          if (p == s.start) { tagg.flag = 1u; tagg.c = g; }
-          else tagg.c += g;
-        }
+    for (int r = 0; r < kRows; ++r) {
+      const int64_t p = wbase + r * 32 + lane;
+      rv[r] = 0u;
+      xv[r] = 0.f;
+      yv[r] = 0.0;
+      if (p < total) {
+        rv[r] = __ldcs(a.lr + p);
+        xv[r] = __ldcs(a.lx + p);
+        yv[r] = __ldcs(a.ly + p);
       }
     }
+    CntP wagg = cnt0;  // warp aggregate (lefts since the warp's last head)
+#pragma unroll
+    for (int r = 0; r < kRows; ++r) {
+      const int64_t p = wbase + r * 32 + lane;
+      uint32_t g = 0, h = 0;
+      if (p < total) {
+        while (p >= s.end) seg_next(s, a.nodes, K, A);
+        h = (p == s.start) ? 1u : 0u;
+        if (__ldg(&a.dec[s.k].f) >= 0) {
+          sbits |= 1u << r;
+          g = __ldg(a.goleft + rv[r]);
+        }
+      }
+      gbits |= g << r;
+      hbits |= h << r;
+      const uint32_t gm = __ballot_sync(0xffffffffu, g);
+      const uint32_t hm = __ballot_sync(0xffffffffu, h);
+      if (hm) {
+        const int hl = 31 - __clz(hm);
+        wagg.flag = 1u;
+        wagg.c = __popc(gm & ~((1u << hl) - 1u));
+      } else {
+        wagg.c += __popc(gm);
+      }
+    }
+    // ---- warp carries (block scan over warps) and the tile carry (look-back)
     CntP tile_agg;
-    const CntP texcl = block_exclusive_scan(tagg, cnt0, tile_agg, sh);
+    CntP wexcl;
+    {
+      // exclusive scan over the 8 warp aggregates, done by every thread of the warp on
+      // its warp's value (lane 0's value is the warp's)
+      CntP mine = wagg;
+      const CntP ex = block_exclusive_scan(lane == 31 ? mine : cnt0, cnt0, tile_agg, sh);
+      // block_exclusive_scan's per-thread exclusive value for lane 31 of warp w = the
+      // combined aggregate of warps < w (all other lanes contribute the identity)
+      wexcl.flag = __shfl_sync(0xffffffffu, ex.flag, 31);
+      wexcl.c = __shfl_sync(0xffffffffu, ex.c, 31);
+    }
     if (tid < 32) {
-      const bool head0 = __shfl_sync(0xffffffffu, p0 == sg.start ? 1 : 0, 0) != 0;
+      const int64_t p0 = tile * kTile;
+      Seg t0;
+      seg_at(t0, a.nodes, K, A, p0);
+      const bool head0 = (p0 == t0.start);
       if (tid == 0) publish(a.lb_agg + tile, tile_agg);
       if (head0) {
         if (tid == 0) {
@@ -948,7 +982,7 @@ __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
           sh_carry = cnt0;
         }
       } else {
-        const int64_t stop_tile = __shfl_sync(0xffffffffu, sg.start, 0) / kTile;
+        const int64_t stop_tile = t0.start / kTile;
         const CntP carry = warp_lookback(a.lb_agg, a.lb_inc, tile, stop_tile, lb_buf);
         if (tid == 0) {
           publish(a.lb_inc + tile, combine(carry, tile_agg));
@@ -957,40 +991,51 @@ __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
       }
     }
     __syncthreads();
-    uint32_t cl = combine(sh_carry, texcl).c;  // lefts before my item 0 in its segment
-    if (any) {
-      float xv[kItems];
-      double yv[kItems];
-      load_items(a.lx, a.ly, p0, total, xv, yv);
-      Seg s = sg;
-      Decision dc = a.dec[s.k];
-      uint32_t ns = __ldg(&a.new_start[s.k]);
-      int64_t obase = (int64_t)s.f * (int64_t)A2;
+    // ---- pass 2: destinations and coalesced stores
+    uint32_t carry = combine(sh_carry, wexcl).c;  // lefts of the open segment before my warp
+    if (wany) {
+      s = s0;
+      uint32_t nlv = 0, nsv = 0;
+      int64_t obase = 0;
+      uint32_t cur_k = 0xffffffffu;
+      int cur_f = -1;
 #pragma unroll
-      for (int j = 0; j < kItems; ++j) {
-        const int64_t p = p0 + j;
+      for (int r = 0; r < kRows; ++r) {
+        const int64_t p = wbase + r * 32 + lane;
+        const uint32_t g = (gbits >> r) & 1u, h = (hbits >> r) & 1u, sp = (sbits >> r) & 1u;
+        const uint32_t gm = __ballot_sync(0xffffffffu, g);
+        const uint32_t hm = __ballot_sync(0xffffffffu, h);
         if (p < total) {
-          if (p == s.end) {
-            seg_next(s, a.nodes, K, A);
-            dc = a.dec[s.k];
-            ns = __ldg(&a.new_start[s.k]);
-            obase = (int64_t)s.f * (int64_t)A2;
-          }
-          if (p == s.start) cl = 0;
-          if (dc.f >= 0) {
+          while (p >= s.end) seg_next(s, a.nodes, K, A);
+          if (sp) {
+            if (s.k != cur_k || s.f != cur_f) {
+              cur_k = s.k;
+              cur_f = s.f;
+              nlv = __ldg(&a.dec[s.k].nl);
+              nsv = __ldg(&a.new_start[s.k]);
+              obase = (int64_t)s.f * (int64_t)A2;
+            }
+            const uint32_t le = hm & ((lt_mask << 1) | 1u);  // heads at lanes <= me
+            uint32_t rank;
+            if (le) {
+              const int hl = 31 - __clz(le);
+              rank = __popc(gm & lt_mask & ~((1u << hl) - 1u));
+            } else {
+              rank = carry + __popc(gm & lt_mask);
+            }
             const uint32_t i = (uint32_t)(p - s.start);
-            const uint32_t g = (glbits >> j) & 1u;
-            const uint32_t dst = g ? ns + cl : ns + dc.nl + (i - cl);
+            const uint32_t dst = g ? nsv + rank : nsv + nlv + (i - rank);
             const int64_t o = obase + dst;
-#ifdef DT_DEBUG_PART
-            if (dst >= A2) printf("BAD tile %lld tid %d j %d p %lld k %u f %d start %lld end %lld i %u cl %u g %u ns %u nl %u A2 %llu carry %u/%u texcl %u/%u\n",
-              (long long)tile, tid, j, (long long)p, s.k, s.f, (long long)s.start, (long long)s.end, i, cl, g, ns, dc.nl, (unsigned long long)A2, sh_carry.flag, sh_carry.c, texcl.flag, texcl.c);
-#endif
-            a.ox[o] = xv[j];
-            a.orow[o] = rv[j];
-            a.oy[o] = yv[j];
-            cl += g;
+            a.ox[o] = xv[r];
+            a.orow[o] = rv[r];
+            a.oy[o] = yv[r];
           }
+        }
+        if (hm) {
+          const int hl = 31 - __clz(hm);
+          carry = __popc(gm & ~((1u << hl) - 1u));
+        } else {
+          carry += __popc(gm);
         }
       }
     }
