@@ -343,6 +343,23 @@ __device__ __forceinline__ double split_gain(double sl, double sc, uint32_t i, u
   return __ddiv_rn(__dmul_rn(D, D), __dmul_rn(__dmul_rn(Nd, nl), nr));
 }
 
+// Same D and denominator as split_gain; the quotient via a Newton-refined reciprocal
+// (relative error ~3e-16).  Used only to locate the exact argmax (see scan_kernel).
+__device__ __forceinline__ double rcp_nr(double x) {
+  double r;
+  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
+  double e = __fma_rn(-x, r, 1.0);
+  r = __fma_rn(r, e, r);
+  e = __fma_rn(-x, r, 1.0);
+  return __fma_rn(r, e, r);
+}
+__device__ __forceinline__ double split_gain_approx(double sl, double sc, uint32_t i, uint32_t N) {
+  const double nl = (double)i, nr = (double)(N - i), Nd = (double)N;
+  const double sr = __dsub_rn(sc, sl);
+  const double D = __dsub_rn(__dmul_rn(sl, nr), __dmul_rn(sr, nl));
+  return __dmul_rn(__dmul_rn(D, D), rcp_nr(__dmul_rn(__dmul_rn(Nd, nl), nr)));
+}
+
 // Loads kItems consecutive x (f32) and y (f64) entries starting at p0 (vectorised when
 // the whole run is in bounds; p0 is a multiple of kItems, so 16-byte aligned).
 __device__ __forceinline__ void load_items(const float* __restrict__ lx, const double* __restrict__ ly,
@@ -409,22 +426,37 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
       seg_at(sg, a.nodes, K, A, p0);
     }
 
+    // Warp-uniform fast path: every thread's kItems entries lie in ONE segment (a head
+    // may only sit at its item 0).  True for nearly all warps at shallow levels.
+    const bool one_seg = any && (p0 + kItems <= total) && (sg.end >= p0 + kItems);
+    const bool warp_fast = __all_sync(0xffffffffu, one_seg || !any);
+    const bool head0 = any && (p0 == sg.start);
+
     // ---- pass 1: thread aggregate of the segmented sum of (y - c)
     SumP tagg = sum0;
     if (any) {
-      Seg s = sg;
-      double c = __ldg(&a.nodes[s.k].c);
+      if (warp_fast) {
+        const double c = __ldg(&a.nodes[sg.k].c);
+        double t = head0 ? __dsub_rn(yv[0], c) : __dadd_rn(0.0, __dsub_rn(yv[0], c));
 #pragma unroll
-      for (int j = 0; j < kItems; ++j) {
-        const int64_t p = p0 + j;
-        if (p < total) {
-          if (p == s.end) {
-            seg_next(s, a.nodes, K, A);
-            c = __ldg(&a.nodes[s.k].c);
+        for (int j = 1; j < kItems; ++j) t = __dadd_rn(t, __dsub_rn(yv[j], c));
+        tagg.flag = head0 ? 1u : 0u;
+        tagg.s = t;
+      } else {
+        Seg s = sg;
+        double c = __ldg(&a.nodes[s.k].c);
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+          const int64_t p = p0 + j;
+          if (p < total) {
+            if (p == s.end) {
+              seg_next(s, a.nodes, K, A);
+              c = __ldg(&a.nodes[s.k].c);
+            }
+            const double e = __dsub_rn(yv[j], c);
+            if (p == s.start) { tagg.flag = 1u; tagg.s = e; }
+            else tagg.s = __dadd_rn(tagg.s, e);
           }
-          const double e = __dsub_rn(yv[j], c);
-          if (p == s.start) { tagg.flag = 1u; tagg.s = e; }
-          else tagg.s = __dadd_rn(tagg.s, e);
         }
       }
     }
@@ -432,9 +464,9 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
     const SumP texcl = block_exclusive_scan(tagg, sum0, tile_agg, sh_sum);
     // ---- tile carry: publish the aggregate, look back (warp 0), publish the inclusive
     if (tid < 32) {
-      const bool head0 = __shfl_sync(0xffffffffu, p0 == sg.start ? 1 : 0, 0) != 0;
+      const bool t_head0 = __shfl_sync(0xffffffffu, head0 ? 1 : 0, 0) != 0;
       if (tid == 0) publish(a.lb_agg + tile, tile_agg);
-      if (head0) {
+      if (t_head0) {
         if (tid == 0) {
           publish(a.lb_inc + tile, tile_agg);
           sh_carry = sum0;
@@ -453,14 +485,67 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
 
     // ---- pass 2: prefixes, gains, per-run best; flush runs that end in this thread
     ArgP run = arg0;
-    StatP srun = stat0;
     bool seen_head = false;
     int last_f = sg.f;
     uint32_t last_k = sg.k;
     const bool stats_tile = (tile * kTile) < (int64_t)A;  // tile holds feature-0 items
-    if (any) {
+    if (any && warp_fast) {
+      if (head0) {
+        fr_gain[tid] = -1.0; fr_sl[tid] = 0.0; fr_i[tid] = 0xffffffffu;
+        seen_head = true;
+        run.flag = 1u;
+        S = 0.0;
+      }
+      if (__ldg(&a.nodes[sg.k].searchable)) {
+        const double c = __ldg(&a.nodes[sg.k].c), sc = __ldg(&a.nodes[sg.k].sc);
+        const uint32_t N = __ldg(&a.nodes[sg.k].N);
+        const uint32_t i0 = (uint32_t)(p0 - sg.start);
+        const uint32_t ilo = m > 1u ? m : 1u, ihi = N - m;
+        const float xprev = head0 ? 0.f : a.lx[p0 - 1];
+        // loop 1: approximate gains (exact D and denominator, reciprocal by Newton)
+        double Sj = S, bapx = -1.0, bS = 0.0;
+        int bj = -1;
+        bool amb = false;
+        constexpr double kTol = 1e-13;  // >> |approx - exact| / exact (~3e-16)
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+          const uint32_t i = i0 + j;
+          const float xp = (j == 0) ? xprev : xv[j - 1];
+          if (i >= ilo && i <= ihi && xp < xv[j]) {
+            const double g = split_gain_approx(Sj, sc, i, N);
+            if (g > bapx) {
+              if (bapx >= __dmul_rn(g, 1.0 - kTol)) amb = true;
+              bapx = g; bS = Sj; bj = j;
+            } else if (g >= __dmul_rn(bapx, 1.0 - kTol)) {
+              amb = true;
+            }
+          }
+          Sj = __dadd_rn(Sj, __dsub_rn(yv[j], c));
+        }
+        if (bj >= 0 && !amb) {
+          // the exact argmax is the approximate one: exact gain of that position only
+          const uint32_t i = i0 + (uint32_t)bj;
+          run.gain = split_gain(bS, sc, i, N);
+          run.i = i;
+          run.sl = bS;
+        } else if (bj >= 0) {
+          // near-tie: exact gains at every valid position (strict >, position order)
+          Sj = S;
+#pragma unroll
+          for (int j = 0; j < kItems; ++j) {
+            const uint32_t i = i0 + j;
+            const float xp = (j == 0) ? xprev : xv[j - 1];
+            if (i >= ilo && i <= ihi && xp < xv[j]) {
+              const double g = split_gain(Sj, sc, i, N);
+              if (g > run.gain) { run.gain = g; run.i = i; run.sl = Sj; }
+            }
+            Sj = __dadd_rn(Sj, __dsub_rn(yv[j], c));
+          }
+        }
+      }
+    } else if (any) {
       Seg s = sg;
-      double nc = __ldg(&a.nodes[s.k].c), nsc = __ldg(&a.nodes[s.k].sc), nv = __ldg(&a.nodes[s.k].v);
+      double nc = __ldg(&a.nodes[s.k].c), nsc = __ldg(&a.nodes[s.k].sc);
       uint32_t nN = __ldg(&a.nodes[s.k].N);
       int nsrch = __ldg(&a.nodes[s.k].searchable);
       float xprev = (p0 > sg.start) ? a.lx[p0 - 1] : 0.f;
@@ -472,27 +557,21 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
             seg_next(s, a.nodes, K, A);
             nc = __ldg(&a.nodes[s.k].c);
             nsc = __ldg(&a.nodes[s.k].sc);
-            nv = __ldg(&a.nodes[s.k].v);
             nN = __ldg(&a.nodes[s.k].N);
             nsrch = __ldg(&a.nodes[s.k].searchable);
           }
           if (p == s.start) {
             if (!seen_head) {
               fr_gain[tid] = run.gain; fr_sl[tid] = run.sl; fr_i[tid] = run.i;
-              fs_sse[tid] = srun.sse; fs_min[tid] = srun.ymin; fs_max[tid] = srun.ymax;
-              fs_s1[tid] = srun.s1;
             } else {
               // the previous run is a whole segment that started in this thread
               const int pf = (s.k == 0) ? s.f - 1 : s.f;
               const uint32_t pk = (s.k == 0) ? (K - 1) : s.k - 1;
               write_cand(a.head_cand + (int64_t)pk * a.d + pf, run);
-              if (pf == 0) write_stat(a.head_stat + pk, srun);
             }
             seen_head = true;
             run = arg0;
             run.flag = 1u;
-            srun = stat0;
-            srun.flag = 1u;
             S = 0.0;
           }
           const uint32_t i = (uint32_t)(p - s.start);
@@ -503,17 +582,47 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
               if (g > run.gain) { run.gain = g; run.i = i; run.sl = S; }
             }
           }
-          const double e = __dsub_rn(yv[j], nc);
-          S = __dadd_rn(S, e);
+          S = __dadd_rn(S, __dsub_rn(yv[j], nc));
+          last_f = s.f;
+          last_k = s.k;
+        }
+      }
+    }
+    // ---- node statistics (feature-0 tiles only): sum (y - v)^2, min, max, sum (y - c)
+    StatP srun = stat0;
+    if (stats_tile && any) {
+      Seg s = sg;
+      double nc = __ldg(&a.nodes[s.k].c), nv = __ldg(&a.nodes[s.k].v);
+      bool seen = false;
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        const int64_t p = p0 + j;
+        if (p < total) {
+          if (p == s.end) {
+            seg_next(s, a.nodes, K, A);
+            nc = __ldg(&a.nodes[s.k].c);
+            nv = __ldg(&a.nodes[s.k].v);
+          }
+          if (p == s.start) {
+            if (!seen) {
+              fs_sse[tid] = srun.sse; fs_min[tid] = srun.ymin; fs_max[tid] = srun.ymax;
+              fs_s1[tid] = srun.s1;
+            } else {
+              const int pf = (s.k == 0) ? s.f - 1 : s.f;
+              const uint32_t pk = (s.k == 0) ? (K - 1) : s.k - 1;
+              if (pf == 0) write_stat(a.head_stat + pk, srun);
+            }
+            seen = true;
+            srun = stat0;
+            srun.flag = 1u;
+          }
           if (s.f == 0) {
             const double ev = __dsub_rn(yv[j], nv);
             srun.sse = __dadd_rn(srun.sse, __dmul_rn(ev, ev));
             srun.ymin = fmin(srun.ymin, yv[j]);
             srun.ymax = fmax(srun.ymax, yv[j]);
-            srun.s1 = __dadd_rn(srun.s1, e);
+            srun.s1 = __dadd_rn(srun.s1, __dsub_rn(yv[j], nc));
           }
-          last_f = s.f;
-          last_k = s.k;
         }
       }
     }
