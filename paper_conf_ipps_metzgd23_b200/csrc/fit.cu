@@ -31,8 +31,9 @@ namespace dtl {
 namespace {
 
 constexpr int kThreads = 256;
-constexpr int kItems = 16;
-constexpr int kTile = kThreads * kItems;  // 4096 list entries per tile
+constexpr int kItems = 8;
+constexpr int kTile = kThreads * kItems;  // 2048 list entries per tile
+constexpr int kChunkLog = 4;              // chunk -> node lookup granularity (16 entries)
 
 // Per-level node record (level-local index k).
 struct NodeL {
@@ -77,8 +78,9 @@ struct Cand {  // best candidate of one segment piece
   double gain;
   double sl;
   uint32_t i;
+  uint32_t kf;     // segment id k*d + f
+  uint32_t level;  // level that wrote the record
   uint32_t pad;
-  double pad2;
 };
 
 struct Stat {
@@ -272,6 +274,18 @@ __global__ void __launch_bounds__(256) presort_build_kernel(const unsigned long 
 
 // ----------------------------------------------------------------------------- scan ----
 
+// chunk[c] = node containing position c << kChunkLog of the level's lists.
+__global__ void __launch_bounds__(256) chunk_node_kernel(const NodeL* __restrict__ nodes, const Ctl* ctl,
+                                                         int parity, uint32_t* __restrict__ chunk) {
+  const uint32_t K = ctl->K[parity];
+  const uint64_t A = ctl->A[parity];
+  if (K == 0) return;
+  const int64_t nc = (int64_t)((A + (1u << kChunkLog) - 1) >> kChunkLog);
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < nc;
+       c += (int64_t)gridDim.x * blockDim.x)
+    chunk[c] = find_node(nodes, K, (uint32_t)(c << kChunkLog));
+}
+
 // Cursor over the segments of a level's concatenated feature lists: segment (f, k)
 // occupies global positions [f*A + start_k, f*A + start_k + N_k).
 struct Seg {
@@ -279,11 +293,21 @@ struct Seg {
   uint32_t k;
   int f;
 };
+// chunk_node[q >> kChunkLog] = node containing list position (q >> kChunkLog) << kChunkLog,
+// rebuilt for every level (chunk_node_kernel); seg_at = one load + a short forward walk.
+
+__device__ __forceinline__ uint32_t node_of(const NodeL* __restrict__ nodes, const uint32_t* __restrict__ chunk,
+                                            uint32_t K, uint32_t q) {
+  uint32_t k = __ldg(chunk + (q >> kChunkLog));
+  while (k + 1 < K && __ldg(&nodes[k + 1].start) <= q) ++k;
+  return k;
+}
+
 __device__ __forceinline__ void seg_at(Seg& s, const NodeL* __restrict__ nodes, uint32_t K,
-                                       uint64_t A, int64_t p) {
+                                       uint64_t A, int64_t p, const uint32_t* __restrict__ chunk) {
   s.f = (int)(p / (int64_t)A);
   s.fbase = (int64_t)s.f * (int64_t)A;
-  s.k = find_node(nodes, K, (uint32_t)(p - s.fbase));
+  s.k = node_of(nodes, chunk, K, (uint32_t)(p - s.fbase));
   s.start = s.fbase + __ldg(&nodes[s.k].start);
   s.end = s.start + __ldg(&nodes[s.k].N);
 }
@@ -308,22 +332,33 @@ struct ScanArgs {
   int d;           // feature count (slot stride)
   int64_t min_leaf;
   uint32_t* counter;  // tile counter (zeroed per launch)
-  uint64_t* lb_agg;   // [ntiles] (kUnpublished before every launch)
-  uint64_t* lb_inc;
+  const uint32_t* chunk;  // chunk -> node table of this level
+  SumP* chunk_agg;    // [nchunks] phase A: per-warp-chunk aggregate
+  SumP* chunk_excl;   // [nchunks] phase B1: exclusive within its block of chunks
+  SumP* block_agg;    // [nblocks] phase B1: block aggregates
+  SumP* block_carry;  // [nblocks] phase B2: exclusive carry per block of chunks
   Cand* head_cand;  // [K*d]
-  Cand* cont_cand;  // [ntiles]
+  Cand* cont_cand;  // [nchunks]
+  unsigned long long* slot_gain;  // [K*d] running max gain bits (zero between levels)
+  uint32_t level;
   Stat* head_stat;  // [K]
-  Stat* cont_stat;  // [ntiles]
+  Stat* cont_stat;  // [nchunks]
 };
 
-__device__ __forceinline__ void write_cand(Cand* p, const ArgP& a) {
+// Piece record + running per-segment max of the gain (u64 order == f64 order for gains
+// >= 0).  The position of the winner is resolved by piece_pos_kernel (lowest position
+// among pieces whose gain equals the max), so the result is exact and deterministic.
+__device__ __forceinline__ void write_cand(Cand* p, const ArgP& a, uint32_t kf, uint32_t level,
+                                           unsigned long long* slot_gain) {
   Cand c;
   c.gain = a.gain;
   c.sl = a.sl;
   c.i = a.i;
+  c.kf = kf;
+  c.level = level;
   c.pad = 0;
-  c.pad2 = 0;
   *p = c;
+  if (a.gain >= 0.0) atomicMax(slot_gain + kf, (unsigned long long)__double_as_longlong(a.gain));
 }
 __device__ __forceinline__ void write_stat(Stat* p, const StatP& a) {
   Stat s;
@@ -387,14 +422,198 @@ __device__ __forceinline__ void load_items(const float* __restrict__ lx, const d
   }
 }
 
+// Tile staging in shared memory (scan): thread t owns entries [16t, 16t+16) = 4 x-chunks
+// and 8 y-chunks of 16 B.  Chunks are fetched striped across the block (coalesced
+// global reads) and stored XOR-swizzled so that each thread's 128-bit reads of its own
+// chunks are bank-conflict-free.
+__device__ __forceinline__ int xslot(int owner, int q) { return owner * 4 + (q ^ ((owner >> 1) & 3)); }
+__device__ __forceinline__ int yslot(int owner, int q) { return owner * 8 + (q ^ (owner & 7)); }
+
+__device__ __forceinline__ void stage_tile_async(const float* __restrict__ lx, const double* __restrict__ ly,
+                                                 int64_t tbase, int64_t total, float4* sx, double2* sy) {
+  const int tid = threadIdx.x;
+#pragma unroll
+  for (int r = 0; r < kItems / 4; ++r) {  // x: 1024 chunks of 4 entries
+    const int c = r * kThreads + tid;
+    const int64_t e0 = tbase + (int64_t)c * 4;
+    const int64_t left = total - e0;
+    if (left > 0) cp_async16(sx + xslot(c >> 2, c & 3), lx + e0, left >= 4 ? 16 : (int)left * 4);
+  }
+#pragma unroll
+  for (int r = 0; r < kItems / 2; ++r) {  // y: 2048 chunks of 2 entries
+    const int c = r * kThreads + tid;
+    const int64_t e0 = tbase + (int64_t)c * 2;
+    const int64_t left = total - e0;
+    if (left > 0) cp_async16(sy + yslot(c >> 3, c & 7), ly + e0, left >= 2 ? 16 : 8);
+  }
+  cp_async_commit();
+}
+
+__device__ __forceinline__ void unstage_items(const float4* sx, const double2* sy, float* xv, double* yv) {
+  const int tid = threadIdx.x;
+#pragma unroll
+  for (int q = 0; q < kItems / 4; ++q) {
+    const float4 t = sx[xslot(tid, q)];
+    xv[4 * q] = t.x; xv[4 * q + 1] = t.y; xv[4 * q + 2] = t.z; xv[4 * q + 3] = t.w;
+  }
+#pragma unroll
+  for (int q = 0; q < kItems / 2; ++q) {
+    const double2 t = sy[yslot(tid, q)];
+    yv[2 * q] = t.x; yv[2 * q + 1] = t.y;
+  }
+}
+
+// Thread aggregate of the segmented sum of (y - c) over my kItems entries (pass 1).
+// Shared by the tile-aggregate kernel and the main scan, so both see identical values.
+__device__ __forceinline__ SumP thread_sum_agg(const ScanArgs& a, uint32_t K, uint64_t A, int64_t p0,
+                                               int64_t total, bool any, bool warp_fast, bool head0,
+                                               const Seg& sg, const double* yv) {
+  SumP tagg{0u, 0.0};
+  if (!any) return tagg;
+  if (warp_fast) {
+    const double c = __ldg(&a.nodes[sg.k].c);
+    double t = head0 ? __dsub_rn(yv[0], c) : __dadd_rn(0.0, __dsub_rn(yv[0], c));
+#pragma unroll
+    for (int j = 1; j < kItems; ++j) t = __dadd_rn(t, __dsub_rn(yv[j], c));
+    tagg.flag = head0 ? 1u : 0u;
+    tagg.s = t;
+  } else {
+    Seg s = sg;
+    double c = __ldg(&a.nodes[s.k].c);
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+      const int64_t p = p0 + j;
+      if (p < total) {
+        if (p == s.end) {
+          seg_next(s, a.nodes, K, A);
+          c = __ldg(&a.nodes[s.k].c);
+        }
+        const double e = __dsub_rn(yv[j], c);
+        if (p == s.start) { tagg.flag = 1u; tagg.s = e; }
+        else tagg.s = __dadd_rn(tagg.s, e);
+      }
+    }
+  }
+  return tagg;
+}
+
+__device__ __forceinline__ void load_y(const double* __restrict__ ly, int64_t p0, int64_t total, double* yv) {
+  if (p0 + kItems <= total) {
+    const double2* y2 = reinterpret_cast<const double2*>(ly + p0);
+#pragma unroll
+    for (int j = 0; j < kItems / 2; ++j) {
+      const double2 t = __ldcs(y2 + j);
+      yv[2 * j] = t.x; yv[2 * j + 1] = t.y;
+    }
+  } else {
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) yv[j] = (p0 + j < total) ? ly[p0 + j] : 0.0;
+  }
+}
+
+// The scan works on WARP CHUNKS of kChunkW = 32 x kItems list entries (lane L owns
+// entries [kItems*L, kItems*L + kItems) of its warp's chunk).  All scans inside a chunk
+// are warp-shuffle scans (no block barrier); chunk carries come from phase B.
+constexpr int kChunkW = 32 * kItems;           // 256 entries
+constexpr int kBlockChunks = 1024 * 2;         // chunks per phase-B1 block
+
+// Phase A: per-chunk segmented aggregate of (y - c) (reads y only).
+__global__ void __launch_bounds__(kThreads) scan_agg_kernel(ScanArgs a) {
+  const uint32_t K = a.ctl->K[a.parity];
+  const uint64_t A = a.ctl->A[a.parity];
+  if (K == 0 || A == 0) return;
+  const int64_t total = (int64_t)A * a.dl;
+  const int64_t nch = (total + kChunkW - 1) / kChunkW;
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  double yn[kItems];
+  {
+    const int64_t q0 = gw * kChunkW + lane * kItems;
+    if (gw < nch && q0 < total) load_y(a.ly, q0, total, yn);
+  }
+  for (int64_t ch = gw; ch < nch; ch += nw) {
+    const int64_t p0 = ch * kChunkW + lane * kItems;
+    const bool any = p0 < total;
+    double yv[kItems];
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) yv[j] = yn[j];
+    {
+      const int64_t q0 = (ch + nw) * kChunkW + lane * kItems;
+      if (ch + nw < nch && q0 < total) load_y(a.ly, q0, total, yn);
+    }
+    Seg sg{0, 0, 0, 0u, 0};
+    if (any) seg_at(sg, a.nodes, K, A, p0, a.chunk);
+    const bool one_seg = any && (p0 + kItems <= total) && (sg.end >= p0 + kItems);
+    const bool warp_fast = __all_sync(0xffffffffu, one_seg || !any);
+    const bool head0 = any && (p0 == sg.start);
+    const SumP tagg = thread_sum_agg(a, K, A, p0, total, any, warp_fast, head0, sg, yv);
+    SumP wagg;
+    (void)warp_exclusive_scan(tagg, SumP{0u, 0.0}, wagg);
+    if (lane == 0) a.chunk_agg[ch] = wagg;
+  }
+}
+
+// Phase B1: exclusive segmented scan of the chunk aggregates inside blocks of
+// kBlockChunks chunks (8 per thread sequentially, then a block scan); fixed shape.
+__global__ void __launch_bounds__(1024) chunk_scan_kernel(ScanArgs a) {
+  __shared__ SumP sh[33];
+  const uint32_t K = a.ctl->K[a.parity];
+  const uint64_t A = a.ctl->A[a.parity];
+  if (K == 0 || A == 0) return;
+  const int64_t total = (int64_t)A * a.dl;
+  const int64_t nch = (total + kChunkW - 1) / kChunkW;
+  const int64_t b0 = (int64_t)blockIdx.x * kBlockChunks;
+  if (b0 >= nch) return;
+  constexpr int kPer = kBlockChunks / 1024;
+  const int64_t c0 = b0 + (int64_t)threadIdx.x * kPer;
+  SumP v[kPer];
+  SumP agg{0u, 0.0};
+#pragma unroll
+  for (int q = 0; q < kPer; ++q) {
+    v[q] = (c0 + q < nch) ? a.chunk_agg[c0 + q] : SumP{0u, 0.0};
+    agg = (q == 0) ? v[0] : combine(agg, v[q]);
+  }
+  SumP bagg;
+  SumP cur = block_exclusive_scan(agg, SumP{0u, 0.0}, bagg, sh);
+#pragma unroll
+  for (int q = 0; q < kPer; ++q) {
+    if (c0 + q < nch) a.chunk_excl[c0 + q] = cur;
+    cur = combine(cur, v[q]);
+  }
+  if (threadIdx.x == 0) a.block_agg[blockIdx.x] = bagg;
+}
+
+// Phase B2: exclusive segmented scan of the block aggregates (one block, fixed shape).
+__global__ void __launch_bounds__(1024) block_carry_kernel(ScanArgs a) {
+  __shared__ SumP sh[33];
+  __shared__ SumP sh_run;
+  const uint32_t K = a.ctl->K[a.parity];
+  const uint64_t A = a.ctl->A[a.parity];
+  if (K == 0 || A == 0) return;
+  const int64_t total = (int64_t)A * a.dl;
+  const int64_t nch = (total + kChunkW - 1) / kChunkW;
+  const int64_t nb = (nch + kBlockChunks - 1) / kBlockChunks;
+  if (threadIdx.x == 0) sh_run = SumP{0u, 0.0};
+  __syncthreads();
+  for (int64_t base = 0; base < nb; base += blockDim.x) {
+    const int64_t b = base + threadIdx.x;
+    const SumP v = (b < nb) ? a.block_agg[b] : SumP{0u, 0.0};
+    SumP chunk;
+    const SumP ex = block_exclusive_scan(v, SumP{0u, 0.0}, chunk, sh);
+    const SumP run = sh_run;
+    if (b < nb) a.block_carry[b] = combine(run, ex);
+    __syncthreads();
+    if (threadIdx.x == 0) sh_run = combine(run, chunk);
+    __syncthreads();
+  }
+}
+
+// Phase C: the main scan (prefixes, gains, per-piece argmax, node statistics), one warp
+// chunk at a time per warp, no block barriers.
 __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
-  __shared__ SumP sh_sum[33];
-  __shared__ ArgP sh_arg[33];
-  __shared__ StatP sh_stat[33];
-  __shared__ SumP lb_buf[kLookbackMax];
-  __shared__ int64_t sh_tile;
-  __shared__ SumP sh_carry;
-  // per-thread best of the run before its first head (read back at the flush)
+  // per-thread best of the run before its first head (written and read by the same
+  // thread, so no barrier is needed)
   __shared__ double fr_gain[kThreads], fr_sl[kThreads], fs_sse[kThreads], fs_min[kThreads],
       fs_max[kThreads], fs_s1[kThreads];
   __shared__ uint32_t fr_i[kThreads];
@@ -403,92 +622,52 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
   const uint64_t A = a.ctl->A[a.parity];
   if (K == 0 || A == 0) return;
   const int64_t total = (int64_t)A * a.dl;
-  const int64_t ntiles = (total + kTile - 1) / kTile;
-  const int tid = threadIdx.x;
+  const int64_t nch = (total + kChunkW - 1) / kChunkW;
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const uint32_t m = (uint32_t)min(a.min_leaf, (int64_t)0xffffffff);
   const SumP sum0{0u, 0.0};
   const ArgP arg0{0u, 0xffffffffu, -1.0, 0.0};
   const StatP stat0{0u, 0.0, INFINITY, -INFINITY, 0.0};
 
-  for (;;) {
-    if (tid == 0) sh_tile = (int64_t)atomicAdd(a.counter, 1u);
-    __syncthreads();
-    const int64_t tile = sh_tile;
-    if (tile >= ntiles) break;
-    const int64_t p0 = tile * kTile + (int64_t)tid * kItems;
+  // register double buffering: the next chunk's loads are in flight during this chunk
+  float xn[kItems];
+  double yn[kItems];
+  {
+    const int64_t q0 = gw * kChunkW + lane * kItems;
+    if (gw < nch && q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
+  }
+  for (int64_t ch = gw; ch < nch; ch += nw) {
+    const int64_t p0 = ch * kChunkW + lane * kItems;
     const bool any = p0 < total;
-
     float xv[kItems];
     double yv[kItems];
-    Seg sg{0, 0, 0, 0u, 0};
-    if (any) {
-      load_items(a.lx, a.ly, p0, total, xv, yv);
-      seg_at(sg, a.nodes, K, A, p0);
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) { xv[j] = xn[j]; yv[j] = yn[j]; }
+    {
+      const int64_t q0 = (ch + nw) * kChunkW + lane * kItems;
+      if (ch + nw < nch && q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
     }
-
-    // Warp-uniform fast path: every thread's kItems entries lie in ONE segment (a head
-    // may only sit at its item 0).  True for nearly all warps at shallow levels.
+    Seg sg{0, 0, 0, 0u, 0};
+    if (any) seg_at(sg, a.nodes, K, A, p0, a.chunk);
+    // Warp-uniform fast path: every lane's kItems entries lie in ONE segment (a head may
+    // only sit at its item 0).  True for nearly all warps at shallow levels.
     const bool one_seg = any && (p0 + kItems <= total) && (sg.end >= p0 + kItems);
     const bool warp_fast = __all_sync(0xffffffffu, one_seg || !any);
     const bool head0 = any && (p0 == sg.start);
-
-    // ---- pass 1: thread aggregate of the segmented sum of (y - c)
-    SumP tagg = sum0;
-    if (any) {
-      if (warp_fast) {
-        const double c = __ldg(&a.nodes[sg.k].c);
-        double t = head0 ? __dsub_rn(yv[0], c) : __dadd_rn(0.0, __dsub_rn(yv[0], c));
-#pragma unroll
-        for (int j = 1; j < kItems; ++j) t = __dadd_rn(t, __dsub_rn(yv[j], c));
-        tagg.flag = head0 ? 1u : 0u;
-        tagg.s = t;
-      } else {
-        Seg s = sg;
-        double c = __ldg(&a.nodes[s.k].c);
-#pragma unroll
-        for (int j = 0; j < kItems; ++j) {
-          const int64_t p = p0 + j;
-          if (p < total) {
-            if (p == s.end) {
-              seg_next(s, a.nodes, K, A);
-              c = __ldg(&a.nodes[s.k].c);
-            }
-            const double e = __dsub_rn(yv[j], c);
-            if (p == s.start) { tagg.flag = 1u; tagg.s = e; }
-            else tagg.s = __dadd_rn(tagg.s, e);
-          }
-        }
-      }
-    }
-    SumP tile_agg;
-    const SumP texcl = block_exclusive_scan(tagg, sum0, tile_agg, sh_sum);
-    // ---- tile carry: publish the aggregate, look back (warp 0), publish the inclusive
-    if (tid < 32) {
-      const bool t_head0 = __shfl_sync(0xffffffffu, head0 ? 1 : 0, 0) != 0;
-      if (tid == 0) publish(a.lb_agg + tile, tile_agg);
-      if (t_head0) {
-        if (tid == 0) {
-          publish(a.lb_inc + tile, tile_agg);
-          sh_carry = sum0;
-        }
-      } else {
-        const int64_t stop_tile = __shfl_sync(0xffffffffu, sg.start, 0) / kTile;
-        const SumP carry = warp_lookback(a.lb_agg, a.lb_inc, tile, stop_tile, lb_buf);
-        if (tid == 0) {
-          publish(a.lb_inc + tile, combine(carry, tile_agg));
-          sh_carry = carry;
-        }
-      }
-    }
-    __syncthreads();
-    double S = combine(sh_carry, texcl).s;  // exclusive prefix at my item 0
+    const SumP tagg = thread_sum_agg(a, K, A, p0, total, any, warp_fast, head0, sg, yv);
+    SumP wagg;
+    const SumP texcl = warp_exclusive_scan(tagg, sum0, wagg);
+    const SumP carry = combine(a.block_carry[ch / kBlockChunks], a.chunk_excl[ch]);
+    double S = combine(carry, texcl).s;  // exclusive prefix at my item 0
 
     // ---- pass 2: prefixes, gains, per-run best; flush runs that end in this thread
     ArgP run = arg0;
     bool seen_head = false;
     int last_f = sg.f;
     uint32_t last_k = sg.k;
-    const bool stats_tile = (tile * kTile) < (int64_t)A;  // tile holds feature-0 items
+    const bool stats_tile = (ch * kChunkW) < (int64_t)A;  // chunk holds feature-0 items
     if (any && warp_fast) {
       if (head0) {
         fr_gain[tid] = -1.0; fr_sl[tid] = 0.0; fr_i[tid] = 0xffffffffu;
@@ -567,7 +746,7 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
               // the previous run is a whole segment that started in this thread
               const int pf = (s.k == 0) ? s.f - 1 : s.f;
               const uint32_t pk = (s.k == 0) ? (K - 1) : s.k - 1;
-              write_cand(a.head_cand + (int64_t)pk * a.d + pf, run);
+              write_cand(a.head_cand + (int64_t)pk * a.d + pf, run, pk * a.d + pf, a.level, a.slot_gain);
             }
             seen_head = true;
             run = arg0;
@@ -631,15 +810,15 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
     StatP strail = srun;
     strail.flag = seen_head ? 1u : 0u;
 
-    ArgP arg_blk;
-    const ArgP aex = block_exclusive_scan(trail, arg0, arg_blk, sh_arg);
-    StatP sex = stat0, st_blk;
-    if (stats_tile) sex = block_exclusive_scan(strail, stat0, st_blk, sh_stat);
+    ArgP arg_w;
+    const ArgP aex = warp_exclusive_scan(trail, arg0, arg_w);
+    StatP sex = stat0, st_w;
+    if (stats_tile) sex = warp_exclusive_scan(strail, stat0, st_w);
 
     // Flush the open segment that ends at my first head (its earlier part is in aex).
     if (any && seen_head) {
       const bool item0_head = (p0 == sg.start);
-      if (!(tid == 0 && item0_head)) {
+      if (!(lane == 0 && item0_head)) {
         int of;
         uint32_t ok;
         if (!item0_head) { of = sg.f; ok = sg.k; }
@@ -647,41 +826,59 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
         else { of = sg.f - 1; ok = K - 1; }
         const ArgP fr{0u, fr_i[tid], fr_gain[tid], fr_sl[tid]};
         const ArgP done_a = combine(aex, fr);
-        const bool head_in_tile = aex.flag != 0;
-        if (head_in_tile) write_cand(a.head_cand + (int64_t)ok * a.d + of, done_a);
-        else write_cand(a.cont_cand + tile, done_a);
+        const bool head_in_chunk = aex.flag != 0;
+        const uint32_t kf = ok * a.d + of;
+        if (head_in_chunk) write_cand(a.head_cand + kf, done_a, kf, a.level, a.slot_gain);
+        else write_cand(a.cont_cand + ch, done_a, kf, a.level, a.slot_gain);
         if (stats_tile && of == 0) {
           const StatP fs{0u, fs_sse[tid], fs_min[tid], fs_max[tid], fs_s1[tid]};
           const StatP done_s = combine(sex, fs);
-          if (head_in_tile) write_stat(a.head_stat + ok, done_s);
-          else write_stat(a.cont_stat + tile, done_s);
+          if (head_in_chunk) write_stat(a.head_stat + ok, done_s);
+          else write_stat(a.cont_stat + ch, done_s);
         }
       }
     }
-    // The last thread closes the segment open at the tile end.
-    if (tid == kThreads - 1) {
+    // The last lane closes the segment open at the chunk end.
+    if (lane == 31) {
       uint32_t lk = last_k;
       int lff = last_f;
       if (!any) {
         Seg t;
-        seg_at(t, a.nodes, K, A, min(total, tile * kTile + kTile) - 1);
+        seg_at(t, a.nodes, K, A, min(total, ch * kChunkW + kChunkW) - 1, a.chunk);
         lk = t.k;
         lff = t.f;
       }
       ArgP tr = run;
       tr.flag = 0u;
       const ArgP done_a = seen_head ? run : combine(aex, tr);
-      const bool head_in_tile = seen_head || aex.flag != 0;
-      if (head_in_tile) write_cand(a.head_cand + (int64_t)lk * a.d + lff, done_a);
-      else write_cand(a.cont_cand + tile, done_a);
+      const bool head_in_chunk = seen_head || aex.flag != 0;
+      const uint32_t kf = lk * a.d + lff;
+      if (head_in_chunk) write_cand(a.head_cand + kf, done_a, kf, a.level, a.slot_gain);
+      else write_cand(a.cont_cand + ch, done_a, kf, a.level, a.slot_gain);
       if (stats_tile && lff == 0) {
         StatP ts = srun;
         ts.flag = 0u;
         const StatP done_s = seen_head ? srun : combine(sex, ts);
-        if (head_in_tile) write_stat(a.head_stat + lk, done_s);
-        else write_stat(a.cont_stat + tile, done_s);
+        if (head_in_chunk) write_stat(a.head_stat + lk, done_s);
+        else write_stat(a.cont_stat + ch, done_s);
       }
     }
+  }
+}
+
+// Lowest position among the pieces of each segment whose gain equals the segment max.
+__global__ void __launch_bounds__(256) piece_pos_kernel(ScanArgs a, uint32_t* __restrict__ slot_pos) {
+  const uint32_t K = a.ctl->K[a.parity];
+  const uint64_t A = a.ctl->A[a.parity];
+  if (K == 0 || A == 0) return;
+  const int64_t total = (int64_t)A * a.dl;
+  const int64_t nch = (total + kChunkW - 1) / kChunkW;
+  const int64_t nhead = (int64_t)K * a.d;
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < nch + nhead;
+       r += (int64_t)gridDim.x * blockDim.x) {
+    const Cand c = (r < nch) ? a.cont_cand[r] : a.head_cand[r - nch];
+    if (c.level != a.level || !(c.gain >= 0.0) || (int64_t)c.kf >= nhead) continue;
+    if ((unsigned long long)__double_as_longlong(c.gain) == a.slot_gain[c.kf]) atomicMin(slot_pos + c.kf, c.i);
   }
 }
 
@@ -702,6 +899,8 @@ struct SelectArgs {
   Decision* dec;
   dt_node* out;
   LevelLog* log;
+  unsigned long long* slot_gain;
+  uint32_t* slot_pos;
 };
 
 __device__ __forceinline__ bool cand_better(double g1, uint32_t i1, double g2, uint32_t i2) {
@@ -725,32 +924,32 @@ __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
   }
   for (uint32_t k = blockIdx.x; k < K; k += gridDim.x) {
     const NodeL nd = a.nodes[k];
-    // ---- per-feature best (warp w handles features w, w+8, ...)
-    for (int f = w; f < a.d; f += 8) {
+    // ---- per-feature best: max gain (slot_gain) at the lowest position (slot_pos); the
+    // winner's S'_L comes from the piece record that holds that position.  Slots are reset.
+    for (int f = tid; f < a.d; f += blockDim.x) {
       double bg = -1.0, bsl = 0.0;
       uint32_t bi = 0xffffffffu;
+      const uint32_t kf = k * a.d + f;
       if (nd.searchable && f < a.dl && nd.N > 1) {
-        const int64_t s0 = (int64_t)f * (int64_t)A + nd.start;
-        const int64_t s1 = s0 + nd.N - 1;
-        const int64_t t0 = s0 / kTile, t1 = s1 / kTile;
-        // piece 0 = head record, pieces 1.. = cont records of tiles t0+1..t1
-        for (int64_t pc = lane; pc <= t1 - t0; pc += 32) {
-          const Cand c = (pc == 0) ? a.head_cand[(int64_t)k * a.d + f] : a.cont_cand[t0 + pc];
-          if (c.gain >= 0.0 && cand_better(c.gain, c.i, bg, bi)) { bg = c.gain; bi = c.i; bsl = c.sl; }
-        }
-        for (int off = 16; off > 0; off >>= 1) {
-          const double og = __shfl_down_sync(0xffffffffu, bg, off);
-          const uint32_t oi = __shfl_down_sync(0xffffffffu, bi, off);
-          const double osl = __shfl_down_sync(0xffffffffu, bsl, off);
-          if (cand_better(og, oi, bg, bi)) { bg = og; bi = oi; bsl = osl; }
+        const uint32_t pos = a.slot_pos[kf];
+        if (pos != 0xffffffffu) {
+          const int64_t s0 = (int64_t)f * (int64_t)A + nd.start;
+          const int64_t t0 = s0 / kChunkW, c = (s0 + pos) / kChunkW;
+          const Cand rec = (c == t0) ? a.head_cand[kf] : a.cont_cand[c];
+          bg = __longlong_as_double((long long)a.slot_gain[kf]);
+          bi = pos;
+          bsl = rec.sl;
         }
       }
-      if (lane == 0) { s_gain[f] = bg; s_i[f] = bi; s_sl[f] = bsl; }
+      a.slot_gain[kf] = 0ull;
+      a.slot_pos[kf] = 0xffffffffu;
+      s_gain[f] = bg; s_i[f] = bi; s_sl[f] = bsl;
     }
+    __syncthreads();
     // ---- node statistics from the feature-0 list (fixed-shape reduction)
     {
       const int64_t s0 = nd.start, s1 = s0 + nd.N - 1;
-      const int64_t t0 = s0 / kTile, t1 = s1 / kTile;
+      const int64_t t0 = s0 / kChunkW, t1 = s1 / kChunkW;
       Stat acc{0.0, INFINITY, -INFINITY, 0.0};  // s1 accumulates sum (y - c)
       // each thread folds a contiguous run of pieces, then tree
       const int64_t np = t1 - t0 + 1;
@@ -980,6 +1179,7 @@ struct PartArgs {
   const Decision* dec;
   const uint32_t* new_start;
   const uint8_t* goleft;
+  const uint32_t* chunk;
   const Ctl* ctl;
   int parity;
   int dl_in;   // lists in the input (d)
@@ -992,13 +1192,14 @@ struct PartArgs {
 // Stable partition of each (node, feature) segment: left rows first then right rows,
 // order preserved; rows of nodes that did not split are dropped.
 //
-// Warp-striped: warp w of a tile owns entries [w*512, w*512 + 512) as 16 rows of 32
+// Warp-striped: warp w of a tile owns entries [w*kRows*32, (w+1)*kRows*32) as kRows rows of 32
 // consecutive entries (lane = position in the row).  Within a row the left/right rank
 // of every entry comes from two ballots (go-left mask, segment-head mask), so each
 // child's entries of a row are written to consecutive addresses (coalesced stores).
 // Carries: row -> row inside the warp, warp -> warp by a block scan, tile -> tile by
 // the decoupled look-back (integer counts).
-constexpr int kRows = kTile / kThreads;  // 16 rows of 32 per warp
+constexpr int kTileP = 4096;              // partition tile (entries)
+constexpr int kRows = kTileP / kThreads;  // rows of 32 per warp
 
 __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
   __shared__ CntP sh[33];
@@ -1010,7 +1211,7 @@ __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
   const uint64_t A2 = a.ctl->A[a.parity ^ 1];
   if (K == 0 || A2 == 0) return;
   const int64_t total = (int64_t)A * a.dl_out;  // only the lists we write
-  const int64_t ntiles = (total + kTile - 1) / kTile;
+  const int64_t ntiles = (total + kTileP - 1) / kTileP;
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   const uint32_t lt_mask = (1u << lane) - 1u;
   const CntP cnt0{0u, 0u};
@@ -1019,7 +1220,7 @@ __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
     __syncthreads();
     const int64_t tile = sh_tile;
     if (tile >= ntiles) break;
-    const int64_t wbase = tile * kTile + (int64_t)w * (kRows * 32);
+    const int64_t wbase = tile * kTileP + (int64_t)w * (kRows * 32);
     // ---- load rows / x / y (coalesced rows of 32), go-left flags, head flags
     uint32_t rv[kRows];
     float xv[kRows];
@@ -1027,7 +1228,7 @@ __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
     uint32_t gbits = 0, hbits = 0, sbits = 0;  // per row: go-left, head, node split
     Seg s{0, 0, 0, 0u, 0};
     const bool wany = wbase < total;
-    if (wany) seg_at(s, a.nodes, K, A, min(wbase + lane, total - 1));
+    if (wany) seg_at(s, a.nodes, K, A, min(wbase + lane, total - 1), a.chunk);
     const Seg s0 = s;
 #pragma unroll
     for (int r = 0; r < kRows; ++r) {
@@ -1080,9 +1281,9 @@ __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
       wexcl.c = __shfl_sync(0xffffffffu, ex.c, 31);
     }
     if (tid < 32) {
-      const int64_t p0 = tile * kTile;
+      const int64_t p0 = tile * kTileP;
       Seg t0;
-      seg_at(t0, a.nodes, K, A, p0);
+      seg_at(t0, a.nodes, K, A, p0, a.chunk);
       const bool head0 = (p0 == t0.start);
       if (tid == 0) publish(a.lb_agg + tile, tile_agg);
       if (head0) {
@@ -1091,7 +1292,7 @@ __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
           sh_carry = cnt0;
         }
       } else {
-        const int64_t stop_tile = t0.start / kTile;
+        const int64_t stop_tile = t0.start / kTileP;
         const CntP carry = warp_lookback(a.lb_agg, a.lb_inc, tile, stop_tile, lb_buf);
         if (tid == 0) {
           publish(a.lb_inc + tile, combine(carry, tile_agg));
@@ -1221,9 +1422,18 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
   DT_CK(ws.get(&dec, (size_t)kcap));
   DT_CK(ws.get(&new_start, (size_t)kcap));
   DT_CK(ws.get(&head_cand, (size_t)kcap * d));
-  DT_CK(ws.get(&cont_cand, (size_t)max_tiles));
+  unsigned long long* slot_gain;
+  uint32_t* slot_pos;
+  DT_CK(ws.get(&slot_gain, (size_t)kcap * d));
+  DT_CK(ws.get(&slot_pos, (size_t)kcap * d));
+  DT_CK(cudaMemsetAsync(slot_gain, 0, sizeof(unsigned long long) * (size_t)kcap * d, s));
+  // piece records carry the level that wrote them; none may match before it is written
+  DT_CK(cudaMemsetAsync(head_cand, 0xFF, sizeof(Cand) * (size_t)kcap * d, s));
+  DT_CK(cudaMemsetAsync(slot_pos, 0xFF, sizeof(uint32_t) * (size_t)kcap * d, s));
+  DT_CK(ws.get(&cont_cand, (size_t)((total0 + 255) / 256 + 1)));
+  DT_CK(cudaMemsetAsync(cont_cand, 0xFF, sizeof(Cand) * (size_t)((total0 + 255) / 256 + 1), s));
   DT_CK(ws.get(&head_stat, (size_t)kcap));
-  DT_CK(ws.get(&cont_stat, (size_t)max_tiles));
+  DT_CK(ws.get(&cont_stat, (size_t)((total0 + 255) / 256 + 1)));
   uint8_t* goleft;
   DT_CK(ws.get(&goleft, (size_t)n));
   dt_node* dout;
@@ -1297,6 +1507,16 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
   }
 
   const int g_scan = persistent_grid((const void*)scan_kernel, kThreads, 0);
+  const int g_agg = persistent_grid((const void*)scan_agg_kernel, kThreads, 0);
+  uint32_t* chunk;
+  DT_CK(ws.get(&chunk, (size_t)((n >> kChunkLog) + 2)));
+  const int64_t max_chunks = (total0 + kChunkW - 1) / kChunkW + 1;
+  const int64_t max_cblocks = (max_chunks + kBlockChunks - 1) / kBlockChunks + 1;
+  SumP *chunk_agg, *chunk_excl, *block_agg, *block_carry;
+  DT_CK(ws.get(&chunk_agg, (size_t)max_chunks));
+  DT_CK(ws.get(&chunk_excl, (size_t)max_chunks));
+  DT_CK(ws.get(&block_agg, (size_t)max_cblocks));
+  DT_CK(ws.get(&block_carry, (size_t)max_cblocks));
   const int g_part = persistent_grid((const void*)partition_kernel, kThreads, 0);
   const int g_sel = num_sms() * 4;
   const int g_gl = num_sms() * 8;
@@ -1309,9 +1529,10 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     const bool last = (max_depth >= 0 && level == max_depth);
     const int dl = last ? 1 : d;
     // scan (a4)
-    DT_CK(cudaMemsetAsync(lb_status, 0, lb_bytes, s));
-    DT_CK(cudaMemsetAsync(lb_desc, 0xFF, desc_bytes, s));
+    int pr = prof_begin(PK_SCAN, s, 5);
+    chunk_node_kernel<<<num_sms() * 4, 256, 0, s>>>(nodes[parity], ctl, parity, chunk);
     ScanArgs sa;
+    sa.chunk = chunk;
     sa.lx = lx[cur];
     sa.ly = ly[cur];
     sa.nodes = nodes[parity];
@@ -1320,14 +1541,19 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     sa.dl = dl;
     sa.d = d;
     sa.min_leaf = min_leaf;
-    sa.counter = lb_status;
-    sa.lb_agg = lb_desc;
-    sa.lb_inc = lb_desc + max_tiles;
+    sa.chunk_agg = chunk_agg;
+    sa.chunk_excl = chunk_excl;
+    sa.block_agg = block_agg;
+    sa.block_carry = block_carry;
     sa.head_cand = head_cand;
     sa.cont_cand = cont_cand;
     sa.head_stat = head_stat;
     sa.cont_stat = cont_stat;
-    int pr = prof_begin(PK_SCAN, s, 1);
+    sa.slot_gain = slot_gain;
+    sa.level = (uint32_t)level;
+    scan_agg_kernel<<<g_agg, kThreads, 0, s>>>(sa);
+    chunk_scan_kernel<<<(unsigned)max_cblocks, 1024, 0, s>>>(sa);
+    block_carry_kernel<<<1, 1024, 0, s>>>(sa);
     scan_kernel<<<g_scan, kThreads, 0, s>>>(sa);
     prof_end(pr, s, 0.0);
     pending.push_back({pr, level, PK_SCAN, dl});
@@ -1348,7 +1574,10 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     se.dec = dec;
     se.out = dout;
     se.log = lvlog;
-    pr = prof_begin(PK_SELECT, s, 1);
+    se.slot_gain = slot_gain;
+    se.slot_pos = slot_pos;
+    pr = prof_begin(PK_SELECT, s, 2);
+    piece_pos_kernel<<<num_sms() * 4, 256, 0, s>>>(sa, slot_pos);
     select_kernel<<<g_sel, 256, 0, s>>>(se);
     prof_end(pr, s, 0.0);
     DT_CK(cudaGetLastError());
@@ -1390,6 +1619,7 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     pa.dec = dec;
     pa.new_start = new_start;
     pa.goleft = goleft;
+    pa.chunk = chunk;
     pa.ctl = ctl;
     pa.parity = parity;
     pa.dl_in = d;

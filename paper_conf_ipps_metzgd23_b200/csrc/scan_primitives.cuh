@@ -95,6 +95,38 @@ __device__ __forceinline__ StatP shfl_up(const StatP& v, int delta) {
   return r;
 }
 
+__device__ __forceinline__ SumP shfl_idx(const SumP& v, int src) {
+  return SumP{__shfl_sync(0xffffffffu, v.flag, src), __shfl_sync(0xffffffffu, v.s, src)};
+}
+__device__ __forceinline__ ArgP shfl_idx(const ArgP& v, int src) {
+  return ArgP{__shfl_sync(0xffffffffu, v.flag, src), __shfl_sync(0xffffffffu, v.i, src),
+              __shfl_sync(0xffffffffu, v.gain, src), __shfl_sync(0xffffffffu, v.sl, src)};
+}
+__device__ __forceinline__ StatP shfl_idx(const StatP& v, int src) {
+  return StatP{__shfl_sync(0xffffffffu, v.flag, src), __shfl_sync(0xffffffffu, v.sse, src),
+               __shfl_sync(0xffffffffu, v.ymin, src), __shfl_sync(0xffffffffu, v.ymax, src),
+               __shfl_sync(0xffffffffu, v.s1, src)};
+}
+
+// ------------------------------------------------------------------ warp scan ------
+
+// Exclusive segmented scan across the 32 lanes of a warp (fixed Kogge-Stone shape, so
+// deterministic); `agg` receives the warp's inclusive value.  No block barrier.
+template <class T>
+__device__ __forceinline__ T warp_exclusive_scan(T v, const T& ident, T& agg) {
+  const int lane = threadIdx.x & 31;
+  T inc = v;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    T o = shfl_up(inc, d);
+    if (lane >= d) inc = combine(o, inc);
+  }
+  agg = shfl_idx(inc, 31);
+  T ex = shfl_up(inc, 1);
+  if (lane == 0) ex = ident;
+  return ex;
+}
+
 // ------------------------------------------------------------------ block scan -----
 
 // Exclusive segmented scan over the block (threads in order).  `ident` is returned to
@@ -222,5 +254,15 @@ __device__ T warp_lookback(const uint64_t* agg, const uint64_t* inc, int64_t til
     __nanosleep(500);  // chain longer than the buffer: wait for predecessors, retry
   }
 }
+
+// ------------------------------------------------------------------ cp.async ------
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
+  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(sa), "l"(gmem), "r"(src_bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 
 }  // namespace dtl
