@@ -554,55 +554,68 @@ __global__ void __launch_bounds__(kThreads) scan_agg_kernel(ScanArgs a) {
   }
 }
 
-// Phase B1: exclusive segmented scan of the chunk aggregates inside blocks of
-// kBlockChunks chunks (8 per thread sequentially, then a block scan); fixed shape.
-__global__ void __launch_bounds__(1024) chunk_scan_kernel(ScanArgs a) {
-  __shared__ SumP sh[33];
-  const uint32_t K = a.ctl->K[a.parity];
-  const uint64_t A = a.ctl->A[a.parity];
+// Phase B1: exclusive segmented scan of per-chunk aggregates inside blocks of
+// kBlockChunks chunks (kPer per thread sequentially, then a block scan); fixed shape.
+// Used for the scan (SumP) and the partition (CntP).
+template <class T>
+__global__ void __launch_bounds__(1024) chunk_scan_kernel(const Ctl* ctl, int parity, int dl,
+                                                          const T* __restrict__ chunk_agg,
+                                                          T* __restrict__ chunk_excl, T* __restrict__ block_agg) {
+  __shared__ T sh[33];
+  const uint32_t K = ctl->K[parity];
+  const uint64_t A = ctl->A[parity];
   if (K == 0 || A == 0) return;
-  const int64_t total = (int64_t)A * a.dl;
+  const int64_t total = (int64_t)A * dl;
   const int64_t nch = (total + kChunkW - 1) / kChunkW;
   const int64_t b0 = (int64_t)blockIdx.x * kBlockChunks;
   if (b0 >= nch) return;
   constexpr int kPer = kBlockChunks / 1024;
   const int64_t c0 = b0 + (int64_t)threadIdx.x * kPer;
-  SumP v[kPer];
-  SumP agg{0u, 0.0};
+  T zero;
+  zero.flag = 0u;
+  from_bits(zero, 0ull);
+  T v[kPer];
+  T agg = zero;
 #pragma unroll
   for (int q = 0; q < kPer; ++q) {
-    v[q] = (c0 + q < nch) ? a.chunk_agg[c0 + q] : SumP{0u, 0.0};
+    v[q] = (c0 + q < nch) ? chunk_agg[c0 + q] : zero;
     agg = (q == 0) ? v[0] : combine(agg, v[q]);
   }
-  SumP bagg;
-  SumP cur = block_exclusive_scan(agg, SumP{0u, 0.0}, bagg, sh);
+  T bagg;
+  T cur = block_exclusive_scan(agg, zero, bagg, sh);
 #pragma unroll
   for (int q = 0; q < kPer; ++q) {
-    if (c0 + q < nch) a.chunk_excl[c0 + q] = cur;
+    if (c0 + q < nch) chunk_excl[c0 + q] = cur;
     cur = combine(cur, v[q]);
   }
-  if (threadIdx.x == 0) a.block_agg[blockIdx.x] = bagg;
+  if (threadIdx.x == 0) block_agg[blockIdx.x] = bagg;
 }
 
 // Phase B2: exclusive segmented scan of the block aggregates (one block, fixed shape).
-__global__ void __launch_bounds__(1024) block_carry_kernel(ScanArgs a) {
-  __shared__ SumP sh[33];
-  __shared__ SumP sh_run;
-  const uint32_t K = a.ctl->K[a.parity];
-  const uint64_t A = a.ctl->A[a.parity];
+template <class T>
+__global__ void __launch_bounds__(1024) block_carry_kernel(const Ctl* ctl, int parity, int dl,
+                                                           const T* __restrict__ block_agg,
+                                                           T* __restrict__ block_carry) {
+  __shared__ T sh[33];
+  __shared__ T sh_run;
+  const uint32_t K = ctl->K[parity];
+  const uint64_t A = ctl->A[parity];
   if (K == 0 || A == 0) return;
-  const int64_t total = (int64_t)A * a.dl;
+  const int64_t total = (int64_t)A * dl;
   const int64_t nch = (total + kChunkW - 1) / kChunkW;
   const int64_t nb = (nch + kBlockChunks - 1) / kBlockChunks;
-  if (threadIdx.x == 0) sh_run = SumP{0u, 0.0};
+  T zero;
+  zero.flag = 0u;
+  from_bits(zero, 0ull);
+  if (threadIdx.x == 0) sh_run = zero;
   __syncthreads();
   for (int64_t base = 0; base < nb; base += blockDim.x) {
     const int64_t b = base + threadIdx.x;
-    const SumP v = (b < nb) ? a.block_agg[b] : SumP{0u, 0.0};
-    SumP chunk;
-    const SumP ex = block_exclusive_scan(v, SumP{0u, 0.0}, chunk, sh);
-    const SumP run = sh_run;
-    if (b < nb) a.block_carry[b] = combine(run, ex);
+    const T v = (b < nb) ? block_agg[b] : zero;
+    T chunk;
+    const T ex = block_exclusive_scan(v, zero, chunk, sh);
+    const T run = sh_run;
+    if (b < nb) block_carry[b] = combine(run, ex);
     __syncthreads();
     if (threadIdx.x == 0) sh_run = combine(run, chunk);
     __syncthreads();
@@ -1184,169 +1197,178 @@ struct PartArgs {
   int parity;
   int dl_in;   // lists in the input (d)
   int dl_out;  // lists to write (d, or 1 before the last level)
-  uint32_t* counter;
-  uint64_t* lb_agg;
-  uint64_t* lb_inc;
+  CntP* chunk_agg;    // [nchunks] phase A
+  CntP* chunk_excl;   // [nchunks] phase B1
+  CntP* block_agg;
+  CntP* block_carry;
 };
 
 // Stable partition of each (node, feature) segment: left rows first then right rows,
 // order preserved; rows of nodes that did not split are dropped.
 //
-// Warp-striped: warp w of a tile owns entries [w*kRows*32, (w+1)*kRows*32) as kRows rows of 32
-// consecutive entries (lane = position in the row).  Within a row the left/right rank
-// of every entry comes from two ballots (go-left mask, segment-head mask), so each
-// child's entries of a row are written to consecutive addresses (coalesced stores).
-// Carries: row -> row inside the warp, warp -> warp by a block scan, tile -> tile by
-// the decoupled look-back (integer counts).
-constexpr int kTileP = 4096;              // partition tile (entries)
-constexpr int kRows = kTileP / kThreads;  // rows of 32 per warp
+// Warp chunks of kChunkW = kRows x 32 consecutive entries (row r of a chunk = 32
+// consecutive entries, lane = position in the row).  Within a row the left/right rank of
+// every entry comes from two ballots (go-left mask, segment-head mask), so each child's
+// entries of a row go to consecutive addresses (coalesced stores).  Carries: row to row
+// inside the warp; chunk to chunk from phase A (per-chunk left counts) + the fixed-shape
+// chunk scan (phase B, shared with the split scan).  No block barriers, no look-back.
+constexpr int kRows = kChunkW / 32;  // rows of 32 per warp chunk
 
+// Per-row go-left / head / split masks of a lane's kRows entries (cursor s advanced).
+// The go-left bytes are gathered for every row up front (independent loads in flight),
+// then masked by "node split" while walking the segments.
+__device__ __forceinline__ void part_flags(const PartArgs& a, uint32_t K, uint64_t A, int64_t wbase,
+                                           int64_t total, Seg& s, const uint32_t* rv, uint32_t& gbits,
+                                           uint32_t& hbits, uint32_t& sbits) {
+  const int lane = threadIdx.x & 31;
+  uint32_t graw = 0;
+#pragma unroll
+  for (int r = 0; r < kRows; ++r) graw |= (uint32_t)__ldg(a.goleft + rv[r]) << r;
+  hbits = sbits = 0;
+#pragma unroll
+  for (int r = 0; r < kRows; ++r) {
+    const int64_t p = wbase + r * 32 + lane;
+    if (p < total) {
+      while (p >= s.end) seg_next(s, a.nodes, K, A);
+      if (p == s.start) hbits |= 1u << r;
+      if (__ldg(&a.dec[s.k].f) >= 0) sbits |= 1u << r;
+    }
+  }
+  gbits = graw & sbits;
+}
+
+__device__ __forceinline__ void load_rows(const uint32_t* __restrict__ lr, int64_t wbase, int64_t total, uint32_t* rv) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int r = 0; r < kRows; ++r) {
+    const int64_t p = wbase + r * 32 + lane;
+    rv[r] = (p < total) ? __ldcs(lr + p) : 0u;
+  }
+}
+
+// Phase A: per-chunk aggregate of go-left counts (lefts since the chunk's last head).
+__global__ void __launch_bounds__(kThreads) part_agg_kernel(PartArgs a) {
+  const uint32_t K = a.ctl->K[a.parity];
+  const uint64_t A = a.ctl->A[a.parity];
+  const uint64_t A2 = a.ctl->A[a.parity ^ 1];
+  if (K == 0 || A2 == 0) return;
+  const int64_t total = (int64_t)A * a.dl_out;
+  const int64_t nch = (total + kChunkW - 1) / kChunkW;
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  uint32_t rn[kRows];
+  if (gw < nch) load_rows(a.lr, gw * kChunkW, total, rn);
+  for (int64_t ch = gw; ch < nch; ch += nw) {
+    const int64_t wbase = ch * kChunkW;
+    uint32_t rv[kRows];
+#pragma unroll
+    for (int r = 0; r < kRows; ++r) rv[r] = rn[r];
+    if (ch + nw < nch) load_rows(a.lr, (ch + nw) * kChunkW, total, rn);
+    Seg s{0, 0, 0, 0u, 0};
+    seg_at(s, a.nodes, K, A, min(wbase + lane, total - 1), a.chunk);
+    uint32_t gbits, hbits, sbits;
+    part_flags(a, K, A, wbase, total, s, rv, gbits, hbits, sbits);
+    CntP agg{0u, 0u};
+#pragma unroll
+    for (int r = 0; r < kRows; ++r) {
+      const uint32_t gm = __ballot_sync(0xffffffffu, (gbits >> r) & 1u);
+      const uint32_t hm = __ballot_sync(0xffffffffu, (hbits >> r) & 1u);
+      if (hm) {
+        const int hl = 31 - __clz(hm);
+        agg.flag = 1u;
+        agg.c = __popc(gm & ~((1u << hl) - 1u));
+      } else {
+        agg.c += __popc(gm);
+      }
+    }
+    if (lane == 0) a.chunk_agg[ch] = agg;
+  }
+}
+
+// Phase C: destinations and coalesced stores.
 __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
-  __shared__ CntP sh[33];
-  __shared__ CntP lb_buf[kLookbackMax];
-  __shared__ int64_t sh_tile;
-  __shared__ CntP sh_carry;
   const uint32_t K = a.ctl->K[a.parity];
   const uint64_t A = a.ctl->A[a.parity];
   const uint64_t A2 = a.ctl->A[a.parity ^ 1];
   if (K == 0 || A2 == 0) return;
   const int64_t total = (int64_t)A * a.dl_out;  // only the lists we write
-  const int64_t ntiles = (total + kTileP - 1) / kTileP;
-  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  const int64_t nch = (total + kChunkW - 1) / kChunkW;
+  const int lane = threadIdx.x & 31;
   const uint32_t lt_mask = (1u << lane) - 1u;
-  const CntP cnt0{0u, 0u};
-  for (;;) {
-    if (tid == 0) sh_tile = (int64_t)atomicAdd(a.counter, 1u);
-    __syncthreads();
-    const int64_t tile = sh_tile;
-    if (tile >= ntiles) break;
-    const int64_t wbase = tile * kTileP + (int64_t)w * (kRows * 32);
-    // ---- load rows / x / y (coalesced rows of 32), go-left flags, head flags
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  uint32_t rn[kRows];
+  float xn[kRows];
+  double yn[kRows];
+  auto load = [&](int64_t wbase) {
+#pragma unroll
+    for (int r = 0; r < kRows; ++r) {
+      const int64_t p = wbase + r * 32 + lane;
+      const bool ok = p < total;
+      rn[r] = ok ? __ldcs(a.lr + p) : 0u;
+      xn[r] = ok ? __ldcs(a.lx + p) : 0.f;
+      yn[r] = ok ? __ldcs(a.ly + p) : 0.0;
+    }
+  };
+  if (gw < nch) load(gw * kChunkW);
+  for (int64_t ch = gw; ch < nch; ch += nw) {
+    const int64_t wbase = ch * kChunkW;
     uint32_t rv[kRows];
     float xv[kRows];
     double yv[kRows];
-    uint32_t gbits = 0, hbits = 0, sbits = 0;  // per row: go-left, head, node split
+#pragma unroll
+    for (int r = 0; r < kRows; ++r) { rv[r] = rn[r]; xv[r] = xn[r]; yv[r] = yn[r]; }
+    if (ch + nw < nch) load((ch + nw) * kChunkW);
     Seg s{0, 0, 0, 0u, 0};
-    const bool wany = wbase < total;
-    if (wany) seg_at(s, a.nodes, K, A, min(wbase + lane, total - 1), a.chunk);
+    seg_at(s, a.nodes, K, A, min(wbase + lane, total - 1), a.chunk);
     const Seg s0 = s;
+    uint32_t gbits, hbits, sbits;
+    part_flags(a, K, A, wbase, total, s, rv, gbits, hbits, sbits);
+    const CntP cc = combine(a.block_carry[ch / kBlockChunks], a.chunk_excl[ch]);
+    uint32_t carry = cc.c;  // lefts of the open segment before this chunk
+    s = s0;
+    uint32_t nlv = 0, nsv = 0;
+    int64_t obase = 0;
+    uint32_t cur_k = 0xffffffffu;
+    int cur_f = -1;
 #pragma unroll
     for (int r = 0; r < kRows; ++r) {
       const int64_t p = wbase + r * 32 + lane;
-      rv[r] = 0u;
-      xv[r] = 0.f;
-      yv[r] = 0.0;
-      if (p < total) {
-        rv[r] = __ldcs(a.lr + p);
-        xv[r] = __ldcs(a.lx + p);
-        yv[r] = __ldcs(a.ly + p);
-      }
-    }
-    CntP wagg = cnt0;  // warp aggregate (lefts since the warp's last head)
-#pragma unroll
-    for (int r = 0; r < kRows; ++r) {
-      const int64_t p = wbase + r * 32 + lane;
-      uint32_t g = 0, h = 0;
+      const uint32_t g = (gbits >> r) & 1u, sp = (sbits >> r) & 1u;
+      const uint32_t gm = __ballot_sync(0xffffffffu, g);
+      const uint32_t hm = __ballot_sync(0xffffffffu, (hbits >> r) & 1u);
       if (p < total) {
         while (p >= s.end) seg_next(s, a.nodes, K, A);
-        h = (p == s.start) ? 1u : 0u;
-        if (__ldg(&a.dec[s.k].f) >= 0) {
-          sbits |= 1u << r;
-          g = __ldg(a.goleft + rv[r]);
+        if (sp) {
+          if (s.k != cur_k || s.f != cur_f) {
+            cur_k = s.k;
+            cur_f = s.f;
+            nlv = __ldg(&a.dec[s.k].nl);
+            nsv = __ldg(&a.new_start[s.k]);
+            obase = (int64_t)s.f * (int64_t)A2;
+          }
+          const uint32_t le = hm & ((lt_mask << 1) | 1u);  // heads at lanes <= me
+          uint32_t rank;
+          if (le) {
+            const int hl = 31 - __clz(le);
+            rank = __popc(gm & lt_mask & ~((1u << hl) - 1u));
+          } else {
+            rank = carry + __popc(gm & lt_mask);
+          }
+          const uint32_t i = (uint32_t)(p - s.start);
+          const uint32_t dst = g ? nsv + rank : nsv + nlv + (i - rank);
+          const int64_t o = obase + dst;
+          a.ox[o] = xv[r];
+          a.orow[o] = rv[r];
+          a.oy[o] = yv[r];
         }
       }
-      gbits |= g << r;
-      hbits |= h << r;
-      const uint32_t gm = __ballot_sync(0xffffffffu, g);
-      const uint32_t hm = __ballot_sync(0xffffffffu, h);
       if (hm) {
         const int hl = 31 - __clz(hm);
-        wagg.flag = 1u;
-        wagg.c = __popc(gm & ~((1u << hl) - 1u));
+        carry = __popc(gm & ~((1u << hl) - 1u));
       } else {
-        wagg.c += __popc(gm);
-      }
-    }
-    // ---- warp carries (block scan over warps) and the tile carry (look-back)
-    CntP tile_agg;
-    CntP wexcl;
-    {
-      // exclusive scan over the 8 warp aggregates, done by every thread of the warp on
-      // its warp's value (lane 0's value is the warp's)
-      CntP mine = wagg;
-      const CntP ex = block_exclusive_scan(lane == 31 ? mine : cnt0, cnt0, tile_agg, sh);
-      // block_exclusive_scan's per-thread exclusive value for lane 31 of warp w = the
-      // combined aggregate of warps < w (all other lanes contribute the identity)
-      wexcl.flag = __shfl_sync(0xffffffffu, ex.flag, 31);
-      wexcl.c = __shfl_sync(0xffffffffu, ex.c, 31);
-    }
-    if (tid < 32) {
-      const int64_t p0 = tile * kTileP;
-      Seg t0;
-      seg_at(t0, a.nodes, K, A, p0, a.chunk);
-      const bool head0 = (p0 == t0.start);
-      if (tid == 0) publish(a.lb_agg + tile, tile_agg);
-      if (head0) {
-        if (tid == 0) {
-          publish(a.lb_inc + tile, tile_agg);
-          sh_carry = cnt0;
-        }
-      } else {
-        const int64_t stop_tile = t0.start / kTileP;
-        const CntP carry = warp_lookback(a.lb_agg, a.lb_inc, tile, stop_tile, lb_buf);
-        if (tid == 0) {
-          publish(a.lb_inc + tile, combine(carry, tile_agg));
-          sh_carry = carry;
-        }
-      }
-    }
-    __syncthreads();
-    // ---- pass 2: destinations and coalesced stores
-    uint32_t carry = combine(sh_carry, wexcl).c;  // lefts of the open segment before my warp
-    if (wany) {
-      s = s0;
-      uint32_t nlv = 0, nsv = 0;
-      int64_t obase = 0;
-      uint32_t cur_k = 0xffffffffu;
-      int cur_f = -1;
-#pragma unroll
-      for (int r = 0; r < kRows; ++r) {
-        const int64_t p = wbase + r * 32 + lane;
-        const uint32_t g = (gbits >> r) & 1u, h = (hbits >> r) & 1u, sp = (sbits >> r) & 1u;
-        const uint32_t gm = __ballot_sync(0xffffffffu, g);
-        const uint32_t hm = __ballot_sync(0xffffffffu, h);
-        if (p < total) {
-          while (p >= s.end) seg_next(s, a.nodes, K, A);
-          if (sp) {
-            if (s.k != cur_k || s.f != cur_f) {
-              cur_k = s.k;
-              cur_f = s.f;
-              nlv = __ldg(&a.dec[s.k].nl);
-              nsv = __ldg(&a.new_start[s.k]);
-              obase = (int64_t)s.f * (int64_t)A2;
-            }
-            const uint32_t le = hm & ((lt_mask << 1) | 1u);  // heads at lanes <= me
-            uint32_t rank;
-            if (le) {
-              const int hl = 31 - __clz(le);
-              rank = __popc(gm & lt_mask & ~((1u << hl) - 1u));
-            } else {
-              rank = carry + __popc(gm & lt_mask);
-            }
-            const uint32_t i = (uint32_t)(p - s.start);
-            const uint32_t dst = g ? nsv + rank : nsv + nlv + (i - rank);
-            const int64_t o = obase + dst;
-            a.ox[o] = xv[r];
-            a.orow[o] = rv[r];
-            a.oy[o] = yv[r];
-          }
-        }
-        if (hm) {
-          const int hl = 31 - __clz(hm);
-          carry = __popc(gm & ~((1u << hl) - 1u));
-        } else {
-          carry += __popc(gm);
-        }
+        carry += __popc(gm);
       }
     }
   }
@@ -1517,6 +1539,12 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
   DT_CK(ws.get(&chunk_excl, (size_t)max_chunks));
   DT_CK(ws.get(&block_agg, (size_t)max_cblocks));
   DT_CK(ws.get(&block_carry, (size_t)max_cblocks));
+  CntP *pchunk_agg, *pchunk_excl, *pblock_agg, *pblock_carry;
+  DT_CK(ws.get(&pchunk_agg, (size_t)max_chunks));
+  DT_CK(ws.get(&pchunk_excl, (size_t)max_chunks));
+  DT_CK(ws.get(&pblock_agg, (size_t)max_cblocks));
+  DT_CK(ws.get(&pblock_carry, (size_t)max_cblocks));
+  const int g_pagg = persistent_grid((const void*)part_agg_kernel, kThreads, 0);
   const int g_part = persistent_grid((const void*)partition_kernel, kThreads, 0);
   const int g_sel = num_sms() * 4;
   const int g_gl = num_sms() * 8;
@@ -1552,8 +1580,8 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     sa.slot_gain = slot_gain;
     sa.level = (uint32_t)level;
     scan_agg_kernel<<<g_agg, kThreads, 0, s>>>(sa);
-    chunk_scan_kernel<<<(unsigned)max_cblocks, 1024, 0, s>>>(sa);
-    block_carry_kernel<<<1, 1024, 0, s>>>(sa);
+    chunk_scan_kernel<SumP><<<(unsigned)max_cblocks, 1024, 0, s>>>(ctl, parity, dl, chunk_agg, chunk_excl, block_agg);
+    block_carry_kernel<SumP><<<1, 1024, 0, s>>>(ctl, parity, dl, block_agg, block_carry);
     scan_kernel<<<g_scan, kThreads, 0, s>>>(sa);
     prof_end(pr, s, 0.0);
     pending.push_back({pr, level, PK_SCAN, dl});
@@ -1606,8 +1634,6 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     pending.push_back({pr, level, PK_GOLEFT, 1});
     DT_CK(cudaGetLastError());
     // stable partition (a7)
-    DT_CK(cudaMemsetAsync(lb_status, 0, lb_bytes, s));
-    DT_CK(cudaMemsetAsync(lb_desc, 0xFF, desc_bytes, s));
     PartArgs pa;
     pa.lx = lx[cur];
     pa.lr = lr[cur];
@@ -1624,10 +1650,14 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     pa.parity = parity;
     pa.dl_in = d;
     pa.dl_out = (max_depth >= 0 && level + 1 == max_depth) ? 1 : d;
-    pa.counter = lb_status;
-    pa.lb_agg = lb_desc;
-    pa.lb_inc = lb_desc + max_tiles;
-    pr = prof_begin(PK_PARTITION, s, 1);
+    pa.chunk_agg = pchunk_agg;
+    pa.chunk_excl = pchunk_excl;
+    pa.block_agg = pblock_agg;
+    pa.block_carry = pblock_carry;
+    pr = prof_begin(PK_PARTITION, s, 4);
+    part_agg_kernel<<<g_pagg, kThreads, 0, s>>>(pa);
+    chunk_scan_kernel<CntP><<<(unsigned)max_cblocks, 1024, 0, s>>>(ctl, parity, pa.dl_out, pchunk_agg, pchunk_excl, pblock_agg);
+    block_carry_kernel<CntP><<<1, 1024, 0, s>>>(ctl, parity, pa.dl_out, pblock_agg, pblock_carry);
     partition_kernel<<<g_part, kThreads, 0, s>>>(pa);
     prof_end(pr, s, 0.0);
     pending.push_back({pr, level, PK_PARTITION, pa.dl_out});
