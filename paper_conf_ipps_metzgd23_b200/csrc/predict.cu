@@ -2,6 +2,9 @@
 // :245-247) and the fused accuracy metrics (MAPE, R^2, adj-R^2; Table II
 // :211-217).  HBM-bound: 4d B read + 8 B written per prediction; 16 B per metric element.
 #include <math.h>
+#include <stdlib.h>
+
+#include <algorithm>
 
 #include "dt_internal.cuh"
 
@@ -9,8 +12,6 @@ namespace dtl {
 
 namespace {
 
-constexpr int kPredThreads = 256;
-constexpr int kRowsPerThread = 4;   // independent traversals per thread (ILP)
 constexpr int kMaxSmemNodes = (227 * 1024) / 8;
 
 // One traversal step: go left iff !(x > RD32(t)); for finite x this is exactly
@@ -22,8 +23,11 @@ __device__ __forceinline__ uint32_t step(uint2 nd, const float* __restrict__ xr)
   return (x > __uint_as_float(nd.x)) ? left + 1 : left;
 }
 
-template <bool kSmem>
-__global__ void __launch_bounds__(kPredThreads)
+// kThr threads x kRPT rows in flight per CTA: every row's features are re-read at each of
+// the `depth` levels, so the CTA's rows (kThr * kRPT * 4d bytes) must stay L1-resident
+// next to the smem tree; the host picks (kThr, kRPT) and the smem carveout accordingly.
+template <bool kSmem, int kThr, int kRowsPerThread>
+__global__ void __launch_bounds__(kThr)
 predict_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ value, int count,
                int depth, const float* __restrict__ X, int64_t n, int d,
                double* __restrict__ yhat) {
@@ -53,6 +57,161 @@ predict_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ valu
     for (int j = 0; j < kRowsPerThread; ++j) {
       int64_t r = base + (int64_t)j * blockDim.x;
       if (r < n) yhat[r] = __ldg(value + k[j]);
+    }
+  }
+}
+
+// Staged predict (d = kD, compile time): the CTA's next batch of kThr rows is copied into
+// shared memory by cp.async (4-byte copies, coalesced, row stride kD + 1 words so that the
+// data-dependent feature reads of a warp hit distinct banks) while the current batch is
+// traversed from shared memory; DRAM latency leaves the 20-level dependency chain.
+__device__ __forceinline__ void cp_async4(void* smem, const void* gmem) {
+  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(sa), "l"(gmem) : "memory");
+}
+
+template <int kThr, int kD>
+__global__ void __launch_bounds__(kThr)
+predict_staged_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ value, int count,
+                      int depth, const float* __restrict__ X, int64_t n, double* __restrict__ yhat) {
+  extern __shared__ uint2 sm[];
+  uint2* tree = sm;
+  float* rows = reinterpret_cast<float*>(sm + count);  // [2][kThr * (kD + 1)]
+  constexpr int kStride = kD + 1;
+  constexpr int kRowsPerPass = kThr / kD;  // rows covered by one copy pass of the block
+  const int tid = threadIdx.x;
+  for (int i = tid; i < count; i += kThr) tree[i] = gnodes[i];
+  const int64_t nb = (n + kThr - 1) / kThr;
+  auto stage = [&](int64_t b, int buf) {
+    const int col = tid % kD, r0 = tid / kD;
+    float* dst = rows + buf * (kThr * kStride);
+    const int64_t base = b * kThr;
+#pragma unroll
+    for (int j = 0; j < kD; ++j) {
+      const int rr = r0 + j * kRowsPerPass;
+      const int64_t r = base + rr;
+      if (r < n) cp_async4(dst + rr * kStride + col, X + r * kD + col);
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  int buf = 0;
+  int64_t b = blockIdx.x;
+  if (b < nb) stage(b, 0);
+  for (; b < nb; b += gridDim.x) {
+    const int64_t bn = b + gridDim.x;
+    if (bn < nb) stage(bn, buf ^ 1);
+    else asm volatile("cp.async.commit_group;" ::: "memory");
+    asm volatile("cp.async.wait_group 1;" ::: "memory");
+    __syncthreads();
+    const int64_t r = b * kThr + tid;
+    if (r < n) {
+      const float* row = rows + buf * (kThr * kStride) + tid * kStride;
+      uint32_t k = 0;
+      for (int l = 0; l < depth; ++l) {
+        const uint2 nd = tree[k];
+        const uint32_t left = nd.y & 0xFFFFFFu;
+        k = (row[nd.y >> 24] > __uint_as_float(nd.x)) ? left + 1 : left;
+      }
+      yhat[r] = __ldg(value + k);
+    }
+    __syncthreads();
+    buf ^= 1;
+  }
+}
+
+// Row-prefetch predict (d = 16): each thread fetches its next row with four 128-bit loads
+// before traversing the current one (DRAM latency off the dependency chain); the current
+// row lives in a thread-local array whose data-dependent reads are L1 hits (the carveout
+// leaves L1 everything the smem tree does not need).
+template <int kThr>
+__global__ void __launch_bounds__(kThr)
+predict_rowpf_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ value, int count,
+                     int depth, const float* __restrict__ X, int64_t n, double* __restrict__ yhat) {
+  extern __shared__ uint2 tree[];
+  for (int i = threadIdx.x; i < count; i += kThr) tree[i] = gnodes[i];
+  __syncthreads();
+  const int64_t stride = (int64_t)gridDim.x * kThr;
+  int64_t r = (int64_t)blockIdx.x * kThr + threadIdx.x;
+  float4 nx[4];
+  auto fetch = [&](int64_t rr) {
+    const float4* src = reinterpret_cast<const float4*>(X + rr * 16);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) nx[q] = __ldcs(src + q);
+  };
+  if (r < n) fetch(r);
+  for (; r < n; r += stride) {
+    float row[16];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      row[4 * q] = nx[q].x; row[4 * q + 1] = nx[q].y; row[4 * q + 2] = nx[q].z; row[4 * q + 3] = nx[q].w;
+    }
+    if (r + stride < n) fetch(r + stride);
+    uint32_t k = 0;
+    for (int l = 0; l < depth; ++l) {
+      const uint2 nd = tree[k];
+      const uint32_t left = nd.y & 0xFFFFFFu;
+      k = (row[nd.y >> 24] > __uint_as_float(nd.x)) ? left + 1 : left;
+    }
+    yhat[r] = __ldg(value + k);
+  }
+}
+
+// Column predict: thread t keeps its current row in shared-memory column t (feature-major
+// s[f][t]), so both the 16/32 stores and the data-dependent feature reads of a warp are
+// bank-conflict-free; the next row is prefetched into registers (four or eight 128-bit
+// loads) during the traversal.  No block barrier after the tree load.
+template <int kThr, int kD, int kR>
+__global__ void __launch_bounds__(kThr)
+predict_col_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ value, int count,
+                   int depth, const float* __restrict__ X, int64_t n, double* __restrict__ yhat) {
+  extern __shared__ uint2 sm[];
+  uint2* tree = sm;
+  // kR columns per thread: column j of thread t at cols[(j * kD + f) * kThr + t]
+  float* cols = reinterpret_cast<float*>(sm + count) + threadIdx.x;
+  for (int i = threadIdx.x; i < count; i += kThr) tree[i] = gnodes[i];
+  __syncthreads();
+  const int64_t stride = (int64_t)gridDim.x * kThr * kR;
+  float4 nx[kR][kD / 4];
+  auto fetch = [&](int64_t base) {
+#pragma unroll
+    for (int j = 0; j < kR; ++j) {
+      const int64_t rr = base + j * kThr;
+      if (rr < n) {
+        const float4* src = reinterpret_cast<const float4*>(X + rr * kD);
+#pragma unroll
+        for (int q = 0; q < kD / 4; ++q) nx[j][q] = __ldcs(src + q);
+      }
+    }
+  };
+  int64_t base = (int64_t)blockIdx.x * kThr * kR + threadIdx.x;
+  if (base < n) fetch(base);
+  for (; base < n; base += stride) {
+#pragma unroll
+    for (int j = 0; j < kR; ++j)
+#pragma unroll
+      for (int q = 0; q < kD / 4; ++q) {
+        float* c = cols + (j * kD + 4 * q) * kThr;
+        c[0] = nx[j][q].x;
+        c[kThr] = nx[j][q].y;
+        c[2 * kThr] = nx[j][q].z;
+        c[3 * kThr] = nx[j][q].w;
+      }
+    if (base + stride < n) fetch(base + stride);
+    uint32_t k[kR];
+#pragma unroll
+    for (int j = 0; j < kR; ++j) k[j] = 0;
+    for (int l = 0; l < depth; ++l) {
+#pragma unroll
+      for (int j = 0; j < kR; ++j) {
+        const uint2 nd = tree[k[j]];
+        const uint32_t left = nd.y & 0xFFFFFFu;
+        k[j] = (cols[(j * kD + (nd.y >> 24)) * kThr] > __uint_as_float(nd.x)) ? left + 1 : left;
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < kR; ++j) {
+      const int64_t rr = base + j * kThr;
+      if (rr < n) yhat[rr] = __ldg(value + k[j]);
     }
   }
 }
@@ -169,16 +328,21 @@ eval_final_kernel(const Part* __restrict__ parts, int nparts, int64_t n, int p_p
   }
 }
 
-int pred_grid(int64_t n, size_t smem, bool use_smem) {
+template <bool kSmem, int kThr, int kRPT>
+dt_status launch_predict(const dt_tree* t, const float* X, int64_t n, int32_t d, double* yhat,
+                         cudaStream_t s, int carveout) {
+  const size_t smem = kSmem ? sizeof(uint2) * (size_t)t->count : 0;
+  auto kern = predict_kernel<kSmem, kThr, kRPT>;
+  if (kSmem) DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, carveout));
   int per_sm = 1;
-  if (use_smem)
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, predict_kernel<true>, kPredThreads, smem);
-  else
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, predict_kernel<false>, kPredThreads, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kThr, smem);
   if (per_sm < 1) per_sm = 1;
-  int64_t need = (n + (int64_t)kPredThreads * kRowsPerThread - 1) / ((int64_t)kPredThreads * kRowsPerThread);
-  int64_t g = (int64_t)num_sms() * per_sm;
-  return (int)(need < g ? (need < 1 ? 1 : need) : g);
+  const int64_t need = (n + (int64_t)kThr * kRPT - 1) / ((int64_t)kThr * kRPT);
+  const int64_t g = std::min<int64_t>((int64_t)num_sms() * per_sm, std::max<int64_t>(1, need));
+  kern<<<(unsigned)g, kThr, smem, s>>>(t->dev_packed, t->dev_value, (int)t->count, t->depth, X, n, d, yhat);
+  DT_CK(cudaGetLastError());
+  return DT_OK;
 }
 
 }  // namespace
@@ -187,19 +351,81 @@ dt_status predict_impl(const dt_tree* t, const float* X, int64_t n, int32_t d, d
                        cudaStream_t s) {
   const bool use_smem = t->count <= kMaxSmemNodes;
   const size_t smem = use_smem ? sizeof(uint2) * (size_t)t->count : 0;
-  const int pr = prof_begin(PK_PREDICT, s, 1);
-  if (use_smem) {
-    DT_CK(cudaFuncSetAttribute(predict_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               (int)smem));
-    predict_kernel<true><<<pred_grid(n, smem, true), kPredThreads, smem, s>>>(
-        t->dev_packed, t->dev_value, (int)t->count, t->depth, X, n, d, yhat);
-  } else {
-    predict_kernel<false><<<pred_grid(n, 0, false), kPredThreads, 0, s>>>(
-        t->dev_packed, t->dev_value, (int)t->count, t->depth, X, n, d, yhat);
+  // configuration: DT_PREDICT_CFG=<0..5> overrides (measurement); default by footprint
+  static int cfg_env = -2;
+  if (cfg_env == -2) {
+    const char* e = getenv("DT_PREDICT_CFG");
+    cfg_env = e ? atoi(e) : -1;
   }
+  // carveout in percent of the 228 KB unified L1/smem: just what the tree needs
+  const int carveout = use_smem ? (int)std::min<size_t>(100, (smem + 2048) * 100 / (228 * 1024) + 1) : 0;
+  const int pr = prof_begin(PK_PREDICT, s, 1);
+  dt_status st;
+  int cfg = cfg_env;
+  if (cfg < 0) cfg = 8;  // default: shared-memory column kernel (d = 16 or 32)
+  if (use_smem && (cfg == 8 || cfg == 9) && (d == 16 || d == 32)) {
+    const int thr = (d == 16) ? 1024 : 512;
+    const int rpt = (cfg == 9) ? 2 : 1;
+    const size_t sm = sizeof(uint2) * (size_t)t->count + sizeof(float) * (size_t)thr * d * rpt;
+    if (sm <= 227 * 1024) {
+      auto kern = (d == 16) ? (rpt == 2 ? predict_col_kernel<1024, 16, 2> : predict_col_kernel<1024, 16, 1>)
+                            : (rpt == 2 ? predict_col_kernel<512, 32, 2> : predict_col_kernel<512, 32, 1>);
+      DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+      int per_sm = 1;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, thr, sm);
+      if (per_sm < 1) per_sm = 1;
+      const int64_t g = std::min<int64_t>((int64_t)num_sms() * per_sm,
+                                          std::max<int64_t>(1, (n + (int64_t)thr * rpt - 1) / ((int64_t)thr * rpt)));
+      kern<<<(unsigned)g, thr, sm, s>>>(t->dev_packed, t->dev_value, (int)t->count, t->depth, X, n, yhat);
+      DT_CK(cudaGetLastError());
+      prof_end(pr, s, (4.0 * d + 8.0) * (double)n);
+      return DT_OK;
+    }
+    cfg = 0;  // tree too large for the column layout: generic kernel
+  }
+  if (use_smem && cfg == 7 && d == 16) {
+    constexpr int kThr = 1024;
+    const size_t sm = sizeof(uint2) * (size_t)t->count;
+    auto kern = predict_rowpf_kernel<kThr>;
+    DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, carveout));
+    int per_sm = 1;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kThr, sm);
+    if (per_sm < 1) per_sm = 1;
+    const int64_t g = std::min<int64_t>((int64_t)num_sms() * per_sm, std::max<int64_t>(1, (n + kThr - 1) / kThr));
+    kern<<<(unsigned)g, kThr, sm, s>>>(t->dev_packed, t->dev_value, (int)t->count, t->depth, X, n, yhat);
+    DT_CK(cudaGetLastError());
+    prof_end(pr, s, (4.0 * d + 8.0) * (double)n);
+    return DT_OK;
+  }
+  if (use_smem && cfg >= 6 && (d == 16 || d == 32)) {
+    constexpr int kThr = 512;
+    const size_t sm = sizeof(uint2) * (size_t)t->count + 2 * sizeof(float) * kThr * (size_t)(d + 1);
+    if (sm <= 227 * 1024) {
+      auto kern = (d == 16) ? predict_staged_kernel<kThr, 16> : predict_staged_kernel<kThr, 32>;
+      DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+      int per_sm = 1;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kThr, sm);
+      if (per_sm < 1) per_sm = 1;
+      const int64_t nb = (n + kThr - 1) / kThr;
+      const int64_t g = std::min<int64_t>((int64_t)num_sms() * per_sm, nb);
+      kern<<<(unsigned)g, kThr, sm, s>>>(t->dev_packed, t->dev_value, (int)t->count, t->depth, X, n, yhat);
+      DT_CK(cudaGetLastError());
+      prof_end(pr, s, (4.0 * d + 8.0) * (double)n);
+      return DT_OK;
+    }
+    cfg = 0;
+  }
+  if (cfg >= 6) cfg = 0;
+  if (!use_smem) st = launch_predict<false, 256, 4>(t, X, n, d, yhat, s, carveout);
+  else if (cfg == 0) st = launch_predict<true, 1024, 1>(t, X, n, d, yhat, s, carveout);
+  else if (cfg == 1) st = launch_predict<true, 512, 2>(t, X, n, d, yhat, s, carveout);
+  else if (cfg == 2) st = launch_predict<true, 1024, 2>(t, X, n, d, yhat, s, carveout);
+  else if (cfg == 3) st = launch_predict<true, 256, 4>(t, X, n, d, yhat, s, carveout);
+  else if (cfg == 4) st = launch_predict<true, 512, 1>(t, X, n, d, yhat, s, carveout);
+  else st = launch_predict<true, 256, 2>(t, X, n, d, yhat, s, carveout);
   prof_end(pr, s, (4.0 * d + 8.0) * (double)n);  // row read + f64 written
-  DT_CK(cudaGetLastError());
-  return DT_OK;
+  return st;
 }
 
 dt_status eval_impl(const double* y, const double* yhat, const float* X, const dt_tree* t,
