@@ -224,8 +224,9 @@ def run_ours(args, world, rank, local):
         tree, m = step()
     ev0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     ev1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    dt.dt_profile_reset()
-    dt.dt_profile_enable(True)
+    # ---- timed steps (headline): no profiling, so bounded-depth fits replay their
+    # cached CUDA graph (the library's normal fast path)
+    dt.dt_profile_enable(False)
     launches0 = dt.dt_launch_count()
     evals = 0
     with ClockSampler(local) as clk:
@@ -239,16 +240,32 @@ def run_ours(args, world, rank, local):
             evals += tree.split_evals
         torch.cuda.synchronize()
         barrier(world)
-    dt.dt_profile_enable(False)
     launches = dt.dt_launch_count() - launches0
     ms = [a.elapsed_time(b) for a, b in zip(ev0, ev1)]
     t_total = sum(ms) / 1e3
     t_max = max_over_ranks(t_total, world)
     evals_all = sum_over_ranks(float(evals), world)
     value = evals_all / t_max
+    step_ms = sum(ms) / len(ms)
+
+    # ---- profiled steps (roofline): per-kernel CUDA events recorded by the library on
+    # its stream around every launch (direct enqueue, no graph), live in this process
+    nprof = max(3, min(args.steps, 10))
+    dt.dt_profile_reset()
+    dt.dt_profile_enable(True)
+    pe0, pe1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    prof_ms = 0.0
+    for _ in range(nprof):
+        flush.zero_()
+        pe0.record(stream)
+        step()
+        pe1.record(stream)
+        torch.cuda.synchronize()
+        prof_ms += pe0.elapsed_time(pe1)
+    dt.dt_profile_enable(False)
     prof = dt.dt_profile()
 
-    # roofline of the dominant kernel (largest device time inside the timed steps)
+    # roofline of the dominant kernel (largest device time inside the profiled steps)
     peak, peak_src = peaks()
     fit_kinds = {k: v for k, v in prof.items() if v["alg_bytes"] > 0}
     dom = max(fit_kinds, key=lambda k: fit_kinds[k]["ms"])
@@ -259,12 +276,12 @@ def run_ours(args, world, rank, local):
     if os.path.exists(tpath):
         with open(tpath) as fh:
             traffic = json.load(fh).get(dom)
-    step_ms = sum(ms) / len(ms)
-    share = {k: round(v["ms"] / sum(ms), 4) for k, v in prof.items()}
+    share = {k: round(v["ms"] / prof_ms, 4) for k, v in prof.items()}
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "peak_source": peak_src,
                 "alg_bytes_per_launch": fit_kinds[dom]["alg_bytes"] / fit_kinds[dom]["launches"],
-                "avg_launch_ms": d_ms / fit_kinds[dom]["launches"], "traffic": traffic}
+                "avg_launch_ms": d_ms / fit_kinds[dom]["launches"], "traffic": traffic,
+                "measured": f"{nprof} profiled steps (ms/step {prof_ms / nprof:.3f}), per-launch CUDA events"}
 
     # ---- e2e: through the C ABI with host buffers (pinned), H2D + D2H inside the region
     Xh, yh = X.cpu().pin_memory(), y.cpu().pin_memory()
@@ -343,8 +360,8 @@ def run_ours(args, world, rank, local):
                 "clocks": clk.summary(),
                 "fit": {"split_evals_per_step": evals // args.steps, "tree_nodes": tree.size,
                         "tree_depth": tree.depth, "eval_mape": m["mape"], "eval_r2": m["r2"],
-                        "kernel_share_of_step": share,
-                        "kernel_ms_per_step": {k: v["ms"] / args.steps for k, v in prof.items()}}}
+                        "kernel_share_of_profiled_step": share,
+                        "kernel_ms_per_step": {k: v["ms"] / nprof for k, v in prof.items()}}}
         print(json.dumps(line), flush=True)
 
 

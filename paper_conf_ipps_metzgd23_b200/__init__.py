@@ -18,7 +18,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libdt.so")
+LIB_PATH = os.environ.get("DT_LIB_PATH") or os.path.join(_HERE, "libdt.so")
 
 NODE_DTYPE = np.dtype([
     ("feature", "<i4"), ("left", "<i4"), ("right", "<i4"), ("depth", "<i4"),

@@ -147,8 +147,13 @@ dt_status dt_tree_from_nodes(const dt_node* nodes, int64_t count, int32_t d, dt_
 
 void dt_tree_free(dt_tree* t) {
   if (!t) return;
-  if (t->dev_packed) cudaFree(t->dev_packed);
-  if (t->dev_value) cudaFree(t->dev_value);
+  if (t->async_alloc) {
+    if (t->dev_packed) cudaFreeAsync(t->dev_packed, 0);
+    if (t->dev_value) cudaFreeAsync(t->dev_value, 0);
+  } else {
+    if (t->dev_packed) cudaFree(t->dev_packed);
+    if (t->dev_value) cudaFree(t->dev_value);
+  }
   free(t->host);
   delete t;
 }

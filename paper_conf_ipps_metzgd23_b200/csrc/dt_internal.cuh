@@ -19,6 +19,7 @@ struct dt_tree {
   uint2* dev_packed = nullptr;
   double* dev_value = nullptr;
   int device = -1;
+  int async_alloc = 0;        // device arrays from cudaMallocAsync (freed with cudaFreeAsync)
 };
 
 namespace dtl {
@@ -67,5 +68,7 @@ enum ProfKind {
 int prof_begin(int kind, cudaStream_t s, int nlaunch);
 void prof_end(int idx, cudaStream_t s, double alg_bytes);
 void prof_set_bytes(int idx, double alg_bytes);
+bool prof_enabled();
+void prof_add_launches(long long n);
 
 }  // namespace dtl

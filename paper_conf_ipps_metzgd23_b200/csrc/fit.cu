@@ -21,6 +21,8 @@
 #include <stdio.h>
 
 #include <algorithm>
+#include <memory>
+#include <mutex>
 #include <vector>
 
 #include "dt_internal.cuh"
@@ -85,6 +87,25 @@ struct Cand {  // best candidate of one segment piece
 
 struct Stat {
   double sse, ymin, ymax, s1;  // s1 = sum (y - c) over the piece
+};
+
+// Per-level descriptor of the segment holding the FIRST entry of each warp chunk
+// (kChunkW entries): one independent load per chunk instead of a dependent lookup chain.
+struct ChunkDesc {
+  int64_t start, end;  // global list positions of the segment
+  uint32_t k;
+  int32_t f;
+  double c, sc, v;     // node centre, centred sum, value
+  uint32_t N;
+  int32_t srch;
+};
+struct PartDesc {
+  int64_t start, end;
+  uint32_t k;
+  int32_t f;
+  uint32_t nl, ns;     // decision: rows left, left-child start in the next lists
+  int32_t split;
+  uint32_t pad;
 };
 
 __device__ __forceinline__ uint32_t flip_f32(float x) {
@@ -274,6 +295,33 @@ __global__ void __launch_bounds__(256) presort_build_kernel(const unsigned long 
 
 // ----------------------------------------------------------------------------- scan ----
 
+__global__ void __launch_bounds__(256) scan_desc_kernel(const NodeL* __restrict__ nodes, const Ctl* ctl,
+                                                        int parity, int dl, int chunkw, ChunkDesc* __restrict__ desc) {
+  const uint32_t K = ctl->K[parity];
+  const uint64_t A = ctl->A[parity];
+  if (K == 0 || A == 0) return;
+  const int64_t total = (int64_t)A * dl;
+  const int64_t nch = (total + chunkw - 1) / chunkw;
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < nch; c += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t p = c * chunkw;
+    const int f = (int)(p / (int64_t)A);
+    const int64_t fbase = (int64_t)f * (int64_t)A;
+    const uint32_t k = find_node(nodes, K, (uint32_t)(p - fbase));
+    const NodeL nd = nodes[k];
+    ChunkDesc d;
+    d.start = fbase + nd.start;
+    d.end = d.start + nd.N;
+    d.k = k;
+    d.f = f;
+    d.c = nd.c;
+    d.sc = nd.sc;
+    d.v = nd.v;
+    d.N = nd.N;
+    d.srch = nd.searchable;
+    desc[c] = d;
+  }
+}
+
 // chunk[c] = node containing position c << kChunkLog of the level's lists.
 __global__ void __launch_bounds__(256) chunk_node_kernel(const NodeL* __restrict__ nodes, const Ctl* ctl,
                                                          int parity, uint32_t* __restrict__ chunk) {
@@ -322,6 +370,18 @@ __device__ __forceinline__ void seg_next(Seg& s, const NodeL* __restrict__ nodes
   s.end = s.start + __ldg(&nodes[s.k].N);
 }
 
+// Cursor for position p starting from a chunk descriptor's segment (walks forward).
+__device__ __forceinline__ void seg_from(Seg& s, int64_t start, int64_t end, uint32_t k, int f,
+                                         uint64_t A, int64_t p, const NodeL* __restrict__ nodes,
+                                         uint32_t K) {
+  s.start = start;
+  s.end = end;
+  s.k = k;
+  s.f = f;
+  s.fbase = (int64_t)f * (int64_t)A;
+  while (p >= s.end) seg_next(s, nodes, K, A);
+}
+
 struct ScanArgs {
   const float* lx;
   const double* ly;
@@ -333,6 +393,7 @@ struct ScanArgs {
   int64_t min_leaf;
   uint32_t* counter;  // tile counter (zeroed per launch)
   const uint32_t* chunk;  // chunk -> node table of this level
+  const ChunkDesc* desc;  // per warp chunk
   SumP* chunk_agg;    // [nchunks] phase A: per-warp-chunk aggregate
   SumP* chunk_excl;   // [nchunks] phase B1: exclusive within its block of chunks
   SumP* block_agg;    // [nblocks] phase B1: block aggregates
@@ -467,11 +528,11 @@ __device__ __forceinline__ void unstage_items(const float4* sx, const double2* s
 // Shared by the tile-aggregate kernel and the main scan, so both see identical values.
 __device__ __forceinline__ SumP thread_sum_agg(const ScanArgs& a, uint32_t K, uint64_t A, int64_t p0,
                                                int64_t total, bool any, bool warp_fast, bool head0,
-                                               const Seg& sg, const double* yv) {
+                                               const Seg& sg, const double* yv, double c_first) {
   SumP tagg{0u, 0.0};
   if (!any) return tagg;
   if (warp_fast) {
-    const double c = __ldg(&a.nodes[sg.k].c);
+    const double c = c_first;
     double t = head0 ? __dsub_rn(yv[0], c) : __dadd_rn(0.0, __dsub_rn(yv[0], c));
 #pragma unroll
     for (int j = 1; j < kItems; ++j) t = __dadd_rn(t, __dsub_rn(yv[j], c));
@@ -479,7 +540,7 @@ __device__ __forceinline__ SumP thread_sum_agg(const ScanArgs& a, uint32_t K, ui
     tagg.s = t;
   } else {
     Seg s = sg;
-    double c = __ldg(&a.nodes[s.k].c);
+    double c = c_first;
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
       const int64_t p = p0 + j;
@@ -542,12 +603,14 @@ __global__ void __launch_bounds__(kThreads) scan_agg_kernel(ScanArgs a) {
       const int64_t q0 = (ch + nw) * kChunkW + lane * kItems;
       if (ch + nw < nch && q0 < total) load_y(a.ly, q0, total, yn);
     }
+    const ChunkDesc dsc = a.desc[ch];
     Seg sg{0, 0, 0, 0u, 0};
-    if (any) seg_at(sg, a.nodes, K, A, p0, a.chunk);
+    if (any) seg_from(sg, dsc.start, dsc.end, dsc.k, dsc.f, A, p0, a.nodes, K);
     const bool one_seg = any && (p0 + kItems <= total) && (sg.end >= p0 + kItems);
     const bool warp_fast = __all_sync(0xffffffffu, one_seg || !any);
     const bool head0 = any && (p0 == sg.start);
-    const SumP tagg = thread_sum_agg(a, K, A, p0, total, any, warp_fast, head0, sg, yv);
+    const double c_in = (sg.k == dsc.k && sg.f == dsc.f) ? dsc.c : __ldg(&a.nodes[sg.k].c);
+    const SumP tagg = thread_sum_agg(a, K, A, p0, total, any, warp_fast, head0, sg, yv, c_in);
     SumP wagg;
     (void)warp_exclusive_scan(tagg, SumP{0u, 0.0}, wagg);
     if (lane == 0) a.chunk_agg[ch] = wagg;
@@ -624,7 +687,13 @@ __global__ void __launch_bounds__(1024) block_carry_kernel(const Ctl* ctl, int p
 
 // Phase C: the main scan (prefixes, gains, per-piece argmax, node statistics), one warp
 // chunk at a time per warp, no block barriers.
-__global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
+#ifndef DT_SCAN_DB
+#define DT_SCAN_DB 1
+#endif
+#ifndef DT_SCAN_OCC
+#define DT_SCAN_OCC 2
+#endif
+__global__ void __launch_bounds__(kThreads, DT_SCAN_OCC) scan_kernel(ScanArgs a) {
   // per-thread best of the run before its first head (written and read by the same
   // thread, so no barrier is needed)
   __shared__ double fr_gain[kThreads], fr_sl[kThreads], fs_sse[kThreads], fs_min[kThreads],
@@ -647,29 +716,34 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
   // register double buffering: the next chunk's loads are in flight during this chunk
   float xn[kItems];
   double yn[kItems];
-  {
+  if (DT_SCAN_DB) {
     const int64_t q0 = gw * kChunkW + lane * kItems;
     if (gw < nch && q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
   }
   for (int64_t ch = gw; ch < nch; ch += nw) {
     const int64_t p0 = ch * kChunkW + lane * kItems;
     const bool any = p0 < total;
+    if (!DT_SCAN_DB && any) load_items(a.lx, a.ly, p0, total, xn, yn);
     float xv[kItems];
     double yv[kItems];
 #pragma unroll
     for (int j = 0; j < kItems; ++j) { xv[j] = xn[j]; yv[j] = yn[j]; }
-    {
+    if (DT_SCAN_DB) {
       const int64_t q0 = (ch + nw) * kChunkW + lane * kItems;
       if (ch + nw < nch && q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
     }
+    const ChunkDesc dsc = a.desc[ch];
     Seg sg{0, 0, 0, 0u, 0};
-    if (any) seg_at(sg, a.nodes, K, A, p0, a.chunk);
+    if (any) seg_from(sg, dsc.start, dsc.end, dsc.k, dsc.f, A, p0, a.nodes, K);
     // Warp-uniform fast path: every lane's kItems entries lie in ONE segment (a head may
     // only sit at its item 0).  True for nearly all warps at shallow levels.
     const bool one_seg = any && (p0 + kItems <= total) && (sg.end >= p0 + kItems);
     const bool warp_fast = __all_sync(0xffffffffu, one_seg || !any);
     const bool head0 = any && (p0 == sg.start);
-    const SumP tagg = thread_sum_agg(a, K, A, p0, total, any, warp_fast, head0, sg, yv);
+    // node fields of my first segment: from the descriptor when it is the chunk's segment
+    const bool in_d = (sg.k == dsc.k && sg.f == dsc.f);
+    const double nd_c = in_d ? dsc.c : __ldg(&a.nodes[sg.k].c);
+    const SumP tagg = thread_sum_agg(a, K, A, p0, total, any, warp_fast, head0, sg, yv, nd_c);
     SumP wagg;
     const SumP texcl = warp_exclusive_scan(tagg, sum0, wagg);
     const SumP carry = combine(a.block_carry[ch / kBlockChunks], a.chunk_excl[ch]);
@@ -688,9 +762,9 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
         run.flag = 1u;
         S = 0.0;
       }
-      if (__ldg(&a.nodes[sg.k].searchable)) {
-        const double c = __ldg(&a.nodes[sg.k].c), sc = __ldg(&a.nodes[sg.k].sc);
-        const uint32_t N = __ldg(&a.nodes[sg.k].N);
+      if (in_d ? dsc.srch : __ldg(&a.nodes[sg.k].searchable)) {
+        const double c = nd_c, sc = in_d ? dsc.sc : __ldg(&a.nodes[sg.k].sc);
+        const uint32_t N = in_d ? dsc.N : __ldg(&a.nodes[sg.k].N);
         const uint32_t i0 = (uint32_t)(p0 - sg.start);
         const uint32_t ilo = m > 1u ? m : 1u, ihi = N - m;
         const float xprev = head0 ? 0.f : a.lx[p0 - 1];
@@ -857,7 +931,7 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
       int lff = last_f;
       if (!any) {
         Seg t;
-        seg_at(t, a.nodes, K, A, min(total, ch * kChunkW + kChunkW) - 1, a.chunk);
+        seg_from(t, dsc.start, dsc.end, dsc.k, dsc.f, A, min(total, ch * kChunkW + kChunkW) - 1, a.nodes, K);
         lk = t.k;
         lff = t.f;
       }
@@ -1181,6 +1255,34 @@ __global__ void __launch_bounds__(256) goleft_kernel(const uint32_t* __restrict_
 
 // ----------------------------------------------------------------------------- partition --
 
+__global__ void __launch_bounds__(256) part_desc_kernel(const NodeL* __restrict__ nodes,
+                                                        const Decision* __restrict__ dec,
+                                                        const uint32_t* __restrict__ new_start, const Ctl* ctl,
+                                                        int parity, int dl, PartDesc* __restrict__ desc) {
+  const uint32_t K = ctl->K[parity];
+  const uint64_t A = ctl->A[parity];
+  if (K == 0 || A == 0 || ctl->A[parity ^ 1] == 0) return;
+  const int64_t total = (int64_t)A * dl;
+  const int64_t nch = (total + kChunkW - 1) / kChunkW;
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < nch; c += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t p = c * kChunkW;
+    const int f = (int)(p / (int64_t)A);
+    const int64_t fbase = (int64_t)f * (int64_t)A;
+    const uint32_t k = find_node(nodes, K, (uint32_t)(p - fbase));
+    PartDesc d;
+    d.start = fbase + nodes[k].start;
+    d.end = d.start + nodes[k].N;
+    d.k = k;
+    d.f = f;
+    const Decision dc = dec[k];
+    d.nl = dc.nl;
+    d.split = dc.f >= 0 ? 1 : 0;
+    d.ns = new_start[k];
+    d.pad = 0;
+    desc[c] = d;
+  }
+}
+
 struct PartArgs {
   const float* lx;
   const uint32_t* lr;
@@ -1193,6 +1295,7 @@ struct PartArgs {
   const uint32_t* new_start;
   const uint8_t* goleft;
   const uint32_t* chunk;
+  const PartDesc* desc;  // per warp chunk
   const Ctl* ctl;
   int parity;
   int dl_in;   // lists in the input (d)
@@ -1219,7 +1322,7 @@ constexpr int kRows = kChunkW / 32;  // rows of 32 per warp chunk
 // then masked by "node split" while walking the segments.
 __device__ __forceinline__ void part_flags(const PartArgs& a, uint32_t K, uint64_t A, int64_t wbase,
                                            int64_t total, Seg& s, const uint32_t* rv, uint32_t& gbits,
-                                           uint32_t& hbits, uint32_t& sbits) {
+                                           uint32_t& hbits, uint32_t& sbits, const PartDesc& dsc) {
   const int lane = threadIdx.x & 31;
   uint32_t graw = 0;
 #pragma unroll
@@ -1231,7 +1334,8 @@ __device__ __forceinline__ void part_flags(const PartArgs& a, uint32_t K, uint64
     if (p < total) {
       while (p >= s.end) seg_next(s, a.nodes, K, A);
       if (p == s.start) hbits |= 1u << r;
-      if (__ldg(&a.dec[s.k].f) >= 0) sbits |= 1u << r;
+      const bool sp = (s.k == dsc.k && s.f == dsc.f) ? (dsc.split != 0) : (__ldg(&a.dec[s.k].f) >= 0);
+      if (sp) sbits |= 1u << r;
     }
   }
   gbits = graw & sbits;
@@ -1265,10 +1369,11 @@ __global__ void __launch_bounds__(kThreads) part_agg_kernel(PartArgs a) {
 #pragma unroll
     for (int r = 0; r < kRows; ++r) rv[r] = rn[r];
     if (ch + nw < nch) load_rows(a.lr, (ch + nw) * kChunkW, total, rn);
+    const PartDesc dsc = a.desc[ch];
     Seg s{0, 0, 0, 0u, 0};
-    seg_at(s, a.nodes, K, A, min(wbase + lane, total - 1), a.chunk);
+    seg_from(s, dsc.start, dsc.end, dsc.k, dsc.f, A, min(wbase + lane, total - 1), a.nodes, K);
     uint32_t gbits, hbits, sbits;
-    part_flags(a, K, A, wbase, total, s, rv, gbits, hbits, sbits);
+    part_flags(a, K, A, wbase, total, s, rv, gbits, hbits, sbits, dsc);
     CntP agg{0u, 0u};
 #pragma unroll
     for (int r = 0; r < kRows; ++r) {
@@ -1287,7 +1392,13 @@ __global__ void __launch_bounds__(kThreads) part_agg_kernel(PartArgs a) {
 }
 
 // Phase C: destinations and coalesced stores.
-__global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
+#ifndef DT_PART_DB
+#define DT_PART_DB 0
+#endif
+#ifndef DT_PART_OCC
+#define DT_PART_OCC 4
+#endif
+__global__ void __launch_bounds__(kThreads, DT_PART_OCC) partition_kernel(PartArgs a) {
   const uint32_t K = a.ctl->K[a.parity];
   const uint64_t A = a.ctl->A[a.parity];
   const uint64_t A2 = a.ctl->A[a.parity ^ 1];
@@ -1311,20 +1422,22 @@ __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
       yn[r] = ok ? __ldcs(a.ly + p) : 0.0;
     }
   };
-  if (gw < nch) load(gw * kChunkW);
+  if (DT_PART_DB && gw < nch) load(gw * kChunkW);
   for (int64_t ch = gw; ch < nch; ch += nw) {
     const int64_t wbase = ch * kChunkW;
+    if (!DT_PART_DB) load(wbase);
     uint32_t rv[kRows];
     float xv[kRows];
     double yv[kRows];
 #pragma unroll
     for (int r = 0; r < kRows; ++r) { rv[r] = rn[r]; xv[r] = xn[r]; yv[r] = yn[r]; }
-    if (ch + nw < nch) load((ch + nw) * kChunkW);
+    if (DT_PART_DB && ch + nw < nch) load((ch + nw) * kChunkW);
+    const PartDesc dsc = a.desc[ch];
     Seg s{0, 0, 0, 0u, 0};
-    seg_at(s, a.nodes, K, A, min(wbase + lane, total - 1), a.chunk);
+    seg_from(s, dsc.start, dsc.end, dsc.k, dsc.f, A, min(wbase + lane, total - 1), a.nodes, K);
     const Seg s0 = s;
     uint32_t gbits, hbits, sbits;
-    part_flags(a, K, A, wbase, total, s, rv, gbits, hbits, sbits);
+    part_flags(a, K, A, wbase, total, s, rv, gbits, hbits, sbits, dsc);
     const CntP cc = combine(a.block_carry[ch / kBlockChunks], a.chunk_excl[ch]);
     uint32_t carry = cc.c;  // lefts of the open segment before this chunk
     s = s0;
@@ -1344,8 +1457,9 @@ __global__ void __launch_bounds__(kThreads, 2) partition_kernel(PartArgs a) {
           if (s.k != cur_k || s.f != cur_f) {
             cur_k = s.k;
             cur_f = s.f;
-            nlv = __ldg(&a.dec[s.k].nl);
-            nsv = __ldg(&a.new_start[s.k]);
+            const bool ind = (s.k == dsc.k && s.f == dsc.f);
+            nlv = ind ? dsc.nl : __ldg(&a.dec[s.k].nl);
+            nsv = ind ? dsc.ns : __ldg(&a.new_start[s.k]);
             obase = (int64_t)s.f * (int64_t)A2;
           }
           const uint32_t le = hm & ((lt_mask << 1) | 1u);  // heads at lanes <= me
@@ -1402,154 +1516,153 @@ int persistent_grid(const void* kern, int threads, size_t smem) {
   return num_sms() * per;
 }
 
-}  // namespace
+// ----------------------------------------------------------------------------- buffers --
 
-dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
-                   int64_t min_leaf, cudaStream_t s, dt_tree** out) {
-  // Pool: keep freed workspace for the next fit (no cudaMalloc on the hot path).
-  {
-    int dev = 0;
-    DT_CK(cudaGetDevice(&dev));
-    cudaMemPool_t pool;
-    DT_CK(cudaDeviceGetDefaultMemPool(&pool, dev));
-    uint64_t thr = UINT64_MAX;
-    DT_CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
-  }
-  Workspace ws;
-  ws.s = s;
-  const int64_t total0 = n * (int64_t)d;
-  // node capacities
-  int64_t kcap = n;
-  if (max_depth >= 0 && max_depth < 40) kcap = std::min<int64_t>(kcap, (int64_t)1 << max_depth);
-  int64_t out_cap = 2 * n - 1;
-  if (max_depth >= 0 && max_depth < 40) out_cap = std::min<int64_t>(out_cap, ((int64_t)1 << (max_depth + 1)) - 1);
-  if (out_cap >= ((int64_t)1 << 31)) return fail(DT_ERR_TOO_LARGE, "dt_fit: node array too large");
-  const int64_t max_tiles = (total0 + kTile - 1) / kTile + 1;
-
+struct FitBufs {
   float* lx[2];
   uint32_t* lr[2];
   double* ly[2];
-  for (int b = 0; b < 2; ++b) {
-    DT_CK(ws.get(&lx[b], (size_t)total0));
-    DT_CK(ws.get(&lr[b], (size_t)total0));
-    DT_CK(ws.get(&ly[b], (size_t)total0));
-  }
   NodeL* nodes[2];
-  DT_CK(ws.get(&nodes[0], (size_t)kcap + 1));
-  DT_CK(ws.get(&nodes[1], (size_t)kcap + 1));
   Decision* dec;
   uint32_t* new_start;
   Cand *head_cand, *cont_cand;
-  Stat *head_stat, *cont_stat;
-  DT_CK(ws.get(&dec, (size_t)kcap));
-  DT_CK(ws.get(&new_start, (size_t)kcap));
-  DT_CK(ws.get(&head_cand, (size_t)kcap * d));
   unsigned long long* slot_gain;
   uint32_t* slot_pos;
-  DT_CK(ws.get(&slot_gain, (size_t)kcap * d));
-  DT_CK(ws.get(&slot_pos, (size_t)kcap * d));
-  DT_CK(cudaMemsetAsync(slot_gain, 0, sizeof(unsigned long long) * (size_t)kcap * d, s));
-  // piece records carry the level that wrote them; none may match before it is written
-  DT_CK(cudaMemsetAsync(head_cand, 0xFF, sizeof(Cand) * (size_t)kcap * d, s));
-  DT_CK(cudaMemsetAsync(slot_pos, 0xFF, sizeof(uint32_t) * (size_t)kcap * d, s));
-  DT_CK(ws.get(&cont_cand, (size_t)((total0 + 255) / 256 + 1)));
-  DT_CK(cudaMemsetAsync(cont_cand, 0xFF, sizeof(Cand) * (size_t)((total0 + 255) / 256 + 1), s));
-  DT_CK(ws.get(&head_stat, (size_t)kcap));
-  DT_CK(ws.get(&cont_stat, (size_t)((total0 + 255) / 256 + 1)));
+  Stat *head_stat, *cont_stat;
   uint8_t* goleft;
-  DT_CK(ws.get(&goleft, (size_t)n));
   dt_node* dout;
-  DT_CK(ws.get(&dout, (size_t)out_cap));
   Ctl* ctl;
-  DT_CK(ws.get(&ctl, 1));
-  DT_CK(cudaMemsetAsync(ctl, 0, sizeof(Ctl), s));
-  // look-back state: [counter | status[max_tiles]] + values
-  uint32_t* lb_status;
-  DT_CK(ws.get(&lb_status, (size_t)max_tiles + 32));
-  // tile descriptors (agg | inc), zeroed with the counter before every launch
-  uint64_t* lb_desc;
-  DT_CK(ws.get(&lb_desc, 2 * (size_t)max_tiles));
-
   LevelLog* lvlog;
-  DT_CK(ws.get(&lvlog, (size_t)kMaxLogLevels));
+  RootPart* parts;
+  double* cparts;
+  unsigned long long *k_in, *k_out;
+  uint32_t *v_in, *v_out;
+  void* sort_tmp;
+  size_t sort_tmp_bytes;
+  ChunkDesc* sdesc;
+  PartDesc* pdesc;
+  SumP *chunk_agg, *chunk_excl, *block_agg, *block_carry;
+  CntP *pchunk_agg, *pchunk_excl, *pblock_agg, *pblock_carry;
+  int64_t kcap, out_cap, max_chunks, max_cblocks, root_np, root_chunk;
+  int fbits;
+};
 
-  // profiling records whose bytes depend on device-side counts: (record, level, kind)
-  struct Pending { int rec, level, kind, dl; };
-  std::vector<Pending> pending;
+// Allocates every buffer through `get` (stream-ordered or persistent).
+template <class Get>
+dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, Get get) {
+  const int64_t total0 = n * (int64_t)d;
+  b.kcap = n;
+  if (max_depth >= 0 && max_depth < 40) b.kcap = std::min<int64_t>(b.kcap, (int64_t)1 << max_depth);
+  b.out_cap = 2 * n - 1;
+  if (max_depth >= 0 && max_depth < 40) b.out_cap = std::min<int64_t>(b.out_cap, ((int64_t)1 << (max_depth + 1)) - 1);
+  if (b.out_cap >= ((int64_t)1 << 31)) return fail(DT_ERR_TOO_LARGE, "dt_fit: node array too large");
+  b.max_chunks = (total0 + kChunkW - 1) / kChunkW + 1;
+  b.max_cblocks = (b.max_chunks + kBlockChunks - 1) / kBlockChunks + 1;
+  b.root_chunk = 8192;
+  b.root_np = (n + b.root_chunk - 1) / b.root_chunk;
+  if (b.root_np > 2048) {
+    b.root_np = 2048;
+    b.root_chunk = (n + b.root_np - 1) / b.root_np;
+    b.root_np = (n + b.root_chunk - 1) / b.root_chunk;
+  }
+  b.fbits = 0;
+  while ((1 << b.fbits) < d) ++b.fbits;
+  for (int k = 0; k < 2; ++k) {
+    DT_CK(get(&b.lx[k], (size_t)total0));
+    DT_CK(get(&b.lr[k], (size_t)total0));
+    DT_CK(get(&b.ly[k], (size_t)total0));
+    DT_CK(get(&b.nodes[k], (size_t)b.kcap + 1));
+  }
+  DT_CK(get(&b.dec, (size_t)b.kcap));
+  DT_CK(get(&b.new_start, (size_t)b.kcap));
+  DT_CK(get(&b.head_cand, (size_t)b.kcap * d));
+  DT_CK(get(&b.slot_gain, (size_t)b.kcap * d));
+  DT_CK(get(&b.slot_pos, (size_t)b.kcap * d));
+  DT_CK(get(&b.cont_cand, (size_t)b.max_chunks));
+  DT_CK(get(&b.head_stat, (size_t)b.kcap));
+  DT_CK(get(&b.cont_stat, (size_t)b.max_chunks));
+  DT_CK(get(&b.goleft, (size_t)n));
+  DT_CK(get(&b.dout, (size_t)b.out_cap));
+  DT_CK(get(&b.ctl, 1));
+  DT_CK(get(&b.lvlog, (size_t)kMaxLogLevels));
+  DT_CK(get(&b.parts, (size_t)b.root_np));
+  DT_CK(get(&b.cparts, (size_t)b.root_np));
+  DT_CK(get(&b.k_in, (size_t)total0));
+  DT_CK(get(&b.k_out, (size_t)total0));
+  DT_CK(get(&b.v_in, (size_t)total0));
+  DT_CK(get(&b.v_out, (size_t)total0));
+  b.sort_tmp_bytes = 0;
+  DT_CK(cub::DeviceRadixSort::SortPairs(nullptr, b.sort_tmp_bytes, b.k_in, b.k_out, b.v_in, b.v_out,
+                                        total0, 0, 32 + b.fbits, (cudaStream_t)0));
+  DT_CK(get((char**)&b.sort_tmp, b.sort_tmp_bytes));
+  DT_CK(get(&b.sdesc, (size_t)b.max_chunks));
+  DT_CK(get(&b.pdesc, (size_t)b.max_chunks));
+  DT_CK(get(&b.chunk_agg, (size_t)b.max_chunks));
+  DT_CK(get(&b.chunk_excl, (size_t)b.max_chunks));
+  DT_CK(get(&b.block_agg, (size_t)b.max_cblocks));
+  DT_CK(get(&b.block_carry, (size_t)b.max_cblocks));
+  DT_CK(get(&b.pchunk_agg, (size_t)b.max_chunks));
+  DT_CK(get(&b.pchunk_excl, (size_t)b.max_chunks));
+  DT_CK(get(&b.pblock_agg, (size_t)b.max_cblocks));
+  DT_CK(get(&b.pblock_carry, (size_t)b.max_cblocks));
+  return DT_OK;
+}
 
+// profiling records whose bytes depend on device-side counts
+struct Pending {
+  int rec, level, kind, dl;
+};
+
+// Enqueues the whole fit on stream s (no host synchronisation unless `poll`).
+dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t n, int32_t d,
+                      int32_t max_depth, int64_t min_leaf, cudaStream_t s, bool poll,
+                      std::vector<Pending>* pending) {
+  const int64_t total0 = n * (int64_t)d;
+  DT_CK(cudaMemsetAsync(b.slot_gain, 0, sizeof(unsigned long long) * (size_t)b.kcap * d, s));
+  // piece records carry the level that wrote them; none may match before it is written
+  DT_CK(cudaMemsetAsync(b.head_cand, 0xFF, sizeof(Cand) * (size_t)b.kcap * d, s));
+  DT_CK(cudaMemsetAsync(b.slot_pos, 0xFF, sizeof(uint32_t) * (size_t)b.kcap * d, s));
+  DT_CK(cudaMemsetAsync(b.cont_cand, 0xFF, sizeof(Cand) * (size_t)b.max_chunks, s));
+  DT_CK(cudaMemsetAsync(b.ctl, 0, sizeof(Ctl), s));
+  Ctl* ctl = b.ctl;
   // ---- root statistics (a0: N, sum y, min/max, integrality, finiteness, centre)
   {
-    int64_t chunk = 8192, np = (n + chunk - 1) / chunk;
-    if (np > 2048) { np = 2048; chunk = (n + np - 1) / np; np = (n + chunk - 1) / chunk; }
-    RootPart* parts;
-    double* cparts;
-    DT_CK(ws.get(&parts, (size_t)np));
-    DT_CK(ws.get(&cparts, (size_t)np));
     const int pr = prof_begin(PK_ROOT, s, 4);
-    root_reduce_kernel<<<(unsigned)np, 256, 0, s>>>(y, n, chunk, parts);
-    root_finalize_kernel<<<1, 32, 0, s>>>(parts, (int)np, n, ctl);
-    root_center_kernel<<<(unsigned)np, 256, 0, s>>>(y, n, chunk, ctl, cparts);
-    root_init_kernel<<<1, 32, 0, s>>>(cparts, (int)np, n, max_depth, min_leaf, ctl, nodes[0]);
+    root_reduce_kernel<<<(unsigned)b.root_np, 256, 0, s>>>(y, n, b.root_chunk, b.parts);
+    root_finalize_kernel<<<1, 32, 0, s>>>(b.parts, (int)b.root_np, n, ctl);
+    root_center_kernel<<<(unsigned)b.root_np, 256, 0, s>>>(y, n, b.root_chunk, ctl, b.cparts);
+    root_init_kernel<<<1, 32, 0, s>>>(b.cparts, (int)b.root_np, n, max_depth, min_leaf, ctl, b.nodes[0]);
     prof_end(pr, s, 16.0 * (double)n);  // y read twice
     DT_CK(cudaGetLastError());
   }
   // ---- presort (a2): per-feature stable sort of (x, row), SoA level-0 lists
   {
-    unsigned long long *k_in, *k_out;
-    uint32_t *v_in, *v_out;
-    DT_CK(ws.get(&k_in, (size_t)total0));
-    DT_CK(ws.get(&k_out, (size_t)total0));
-    DT_CK(ws.get(&v_in, (size_t)total0));
-    DT_CK(ws.get(&v_out, (size_t)total0));
     const int64_t nb = (n + 255) / 256;
     const size_t smem = sizeof(float) * 256 * (size_t)d;
     if (smem > 48 * 1024)
       DT_CK(cudaFuncSetAttribute(presort_keys_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int pr = prof_begin(PK_PRESORT_KEYS, s, 1);
-    presort_keys_kernel<<<(unsigned)nb, 256, smem, s>>>(X, n, d, k_in, v_in, ctl);
+    presort_keys_kernel<<<(unsigned)nb, 256, smem, s>>>(X, n, d, b.k_in, b.v_in, ctl);
     prof_end(pr, s, 16.0 * (double)total0);  // X read + (key, val) written
     DT_CK(cudaGetLastError());
-    int fbits = 0;
-    while ((1 << fbits) < d) ++fbits;
-    size_t tmp_bytes = 0;
-    DT_CK(cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, k_in, k_out, v_in, v_out, total0, 0,
-                                          32 + fbits, s));
-    void* tmp;
-    DT_CK(ws.get((char**)&tmp, tmp_bytes));
-    const int passes = (32 + fbits + 7) / 8;
+    const int passes = (32 + b.fbits + 7) / 8;
+    size_t tmp_bytes = b.sort_tmp_bytes;
     pr = prof_begin(PK_PRESORT_SORT, s, 0);  // CUB kernels: library, not counted
-    DT_CK(cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, k_in, k_out, v_in, v_out, total0, 0,
-                                          32 + fbits, s));
+    DT_CK(cub::DeviceRadixSort::SortPairs(b.sort_tmp, tmp_bytes, b.k_in, b.k_out, b.v_in, b.v_out,
+                                          total0, 0, 32 + b.fbits, s));
     prof_end(pr, s, 24.0 * (double)total0 * passes);
     const int gb = std::max(1, std::min<int>((int)((total0 + 255) / 256), num_sms() * 8));
     pr = prof_begin(PK_PRESORT_BUILD, s, 1);
-    presort_build_kernel<<<gb, 256, 0, s>>>(k_out, v_out, y, total0, lx[0], lr[0], ly[0]);
+    presort_build_kernel<<<gb, 256, 0, s>>>(b.k_out, b.v_out, y, total0, b.lx[0], b.lr[0], b.ly[0]);
     prof_end(pr, s, 36.0 * (double)total0);  // (key, val) read, y gathered, 16 B written
     DT_CK(cudaGetLastError());
   }
-
   const int g_scan = persistent_grid((const void*)scan_kernel, kThreads, 0);
   const int g_agg = persistent_grid((const void*)scan_agg_kernel, kThreads, 0);
-  uint32_t* chunk;
-  DT_CK(ws.get(&chunk, (size_t)((n >> kChunkLog) + 2)));
-  const int64_t max_chunks = (total0 + kChunkW - 1) / kChunkW + 1;
-  const int64_t max_cblocks = (max_chunks + kBlockChunks - 1) / kBlockChunks + 1;
-  SumP *chunk_agg, *chunk_excl, *block_agg, *block_carry;
-  DT_CK(ws.get(&chunk_agg, (size_t)max_chunks));
-  DT_CK(ws.get(&chunk_excl, (size_t)max_chunks));
-  DT_CK(ws.get(&block_agg, (size_t)max_cblocks));
-  DT_CK(ws.get(&block_carry, (size_t)max_cblocks));
-  CntP *pchunk_agg, *pchunk_excl, *pblock_agg, *pblock_carry;
-  DT_CK(ws.get(&pchunk_agg, (size_t)max_chunks));
-  DT_CK(ws.get(&pchunk_excl, (size_t)max_chunks));
-  DT_CK(ws.get(&pblock_agg, (size_t)max_cblocks));
-  DT_CK(ws.get(&pblock_carry, (size_t)max_cblocks));
   const int g_pagg = persistent_grid((const void*)part_agg_kernel, kThreads, 0);
   const int g_part = persistent_grid((const void*)partition_kernel, kThreads, 0);
   const int g_sel = num_sms() * 4;
   const int g_gl = num_sms() * 8;
-  const size_t lb_bytes = sizeof(uint32_t) * 32;
-  const size_t desc_bytes = sizeof(uint64_t) * 2 * (size_t)max_tiles;
 
   int cur = 0;
   for (int level = 0;; ++level) {
@@ -1558,139 +1671,165 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     const int dl = last ? 1 : d;
     // scan (a4)
     int pr = prof_begin(PK_SCAN, s, 5);
-    chunk_node_kernel<<<num_sms() * 4, 256, 0, s>>>(nodes[parity], ctl, parity, chunk);
+    scan_desc_kernel<<<num_sms() * 4, 256, 0, s>>>(b.nodes[parity], ctl, parity, dl, kChunkW, b.sdesc);
     ScanArgs sa;
-    sa.chunk = chunk;
-    sa.lx = lx[cur];
-    sa.ly = ly[cur];
-    sa.nodes = nodes[parity];
+    sa.chunk = nullptr;
+    sa.desc = b.sdesc;
+    sa.lx = b.lx[cur];
+    sa.ly = b.ly[cur];
+    sa.nodes = b.nodes[parity];
     sa.ctl = ctl;
     sa.parity = parity;
     sa.dl = dl;
     sa.d = d;
     sa.min_leaf = min_leaf;
-    sa.chunk_agg = chunk_agg;
-    sa.chunk_excl = chunk_excl;
-    sa.block_agg = block_agg;
-    sa.block_carry = block_carry;
-    sa.head_cand = head_cand;
-    sa.cont_cand = cont_cand;
-    sa.head_stat = head_stat;
-    sa.cont_stat = cont_stat;
-    sa.slot_gain = slot_gain;
+    sa.chunk_agg = b.chunk_agg;
+    sa.chunk_excl = b.chunk_excl;
+    sa.block_agg = b.block_agg;
+    sa.block_carry = b.block_carry;
+    sa.head_cand = b.head_cand;
+    sa.cont_cand = b.cont_cand;
+    sa.head_stat = b.head_stat;
+    sa.cont_stat = b.cont_stat;
+    sa.slot_gain = b.slot_gain;
     sa.level = (uint32_t)level;
     scan_agg_kernel<<<g_agg, kThreads, 0, s>>>(sa);
-    chunk_scan_kernel<SumP><<<(unsigned)max_cblocks, 1024, 0, s>>>(ctl, parity, dl, chunk_agg, chunk_excl, block_agg);
-    block_carry_kernel<SumP><<<1, 1024, 0, s>>>(ctl, parity, dl, block_agg, block_carry);
+    chunk_scan_kernel<SumP><<<(unsigned)b.max_cblocks, 1024, 0, s>>>(ctl, parity, dl, b.chunk_agg, b.chunk_excl, b.block_agg);
+    block_carry_kernel<SumP><<<1, 1024, 0, s>>>(ctl, parity, dl, b.block_agg, b.block_carry);
     scan_kernel<<<g_scan, kThreads, 0, s>>>(sa);
     prof_end(pr, s, 0.0);
-    pending.push_back({pr, level, PK_SCAN, dl});
+    if (pending) pending->push_back({pr, level, PK_SCAN, dl});
     DT_CK(cudaGetLastError());
     // select (a5, a8)
     SelectArgs se;
-    se.lx = lx[cur];
-    se.nodes = nodes[parity];
+    se.lx = b.lx[cur];
+    se.nodes = b.nodes[parity];
     se.ctl = ctl;
     se.parity = parity;
     se.level = level;
     se.dl = dl;
     se.d = d;
-    se.head_cand = head_cand;
-    se.cont_cand = cont_cand;
-    se.head_stat = head_stat;
-    se.cont_stat = cont_stat;
-    se.dec = dec;
-    se.out = dout;
-    se.log = lvlog;
-    se.slot_gain = slot_gain;
-    se.slot_pos = slot_pos;
+    se.head_cand = b.head_cand;
+    se.cont_cand = b.cont_cand;
+    se.head_stat = b.head_stat;
+    se.cont_stat = b.cont_stat;
+    se.dec = b.dec;
+    se.out = b.dout;
+    se.log = b.lvlog;
+    se.slot_gain = b.slot_gain;
+    se.slot_pos = b.slot_pos;
     pr = prof_begin(PK_SELECT, s, 2);
-    piece_pos_kernel<<<num_sms() * 4, 256, 0, s>>>(sa, slot_pos);
+    piece_pos_kernel<<<num_sms() * 4, 256, 0, s>>>(sa, b.slot_pos);
     select_kernel<<<g_sel, 256, 0, s>>>(se);
     prof_end(pr, s, 0.0);
     DT_CK(cudaGetLastError());
     if (last) break;
     // number (a3, a8)
     NumberArgs na;
-    na.nodes = nodes[parity];
-    na.next = nodes[parity ^ 1];
-    na.dec = dec;
-    na.new_start = new_start;
+    na.nodes = b.nodes[parity];
+    na.next = b.nodes[parity ^ 1];
+    na.dec = b.dec;
+    na.new_start = b.new_start;
     na.ctl = ctl;
     na.parity = parity;
     na.level = level;
     na.max_depth = max_depth;
     na.min_leaf = min_leaf;
-    na.out = dout;
-    na.log = lvlog;
+    na.out = b.dout;
+    na.log = b.lvlog;
     pr = prof_begin(PK_NUMBER, s, 1);
     number_kernel<<<1, 1024, 0, s>>>(na);
     prof_end(pr, s, 0.0);
     DT_CK(cudaGetLastError());
     // go-left map (a6)
     pr = prof_begin(PK_GOLEFT, s, 1);
-    goleft_kernel<<<g_gl, 256, 0, s>>>(lr[cur], nodes[parity], dec, ctl, parity, goleft);
+    goleft_kernel<<<g_gl, 256, 0, s>>>(b.lr[cur], b.nodes[parity], b.dec, ctl, parity, b.goleft);
     prof_end(pr, s, 0.0);
-    pending.push_back({pr, level, PK_GOLEFT, 1});
+    if (pending) pending->push_back({pr, level, PK_GOLEFT, 1});
     DT_CK(cudaGetLastError());
     // stable partition (a7)
     PartArgs pa;
-    pa.lx = lx[cur];
-    pa.lr = lr[cur];
-    pa.ly = ly[cur];
-    pa.ox = lx[cur ^ 1];
-    pa.orow = lr[cur ^ 1];
-    pa.oy = ly[cur ^ 1];
-    pa.nodes = nodes[parity];
-    pa.dec = dec;
-    pa.new_start = new_start;
-    pa.goleft = goleft;
-    pa.chunk = chunk;
+    pa.lx = b.lx[cur];
+    pa.lr = b.lr[cur];
+    pa.ly = b.ly[cur];
+    pa.ox = b.lx[cur ^ 1];
+    pa.orow = b.lr[cur ^ 1];
+    pa.oy = b.ly[cur ^ 1];
+    pa.nodes = b.nodes[parity];
+    pa.dec = b.dec;
+    pa.new_start = b.new_start;
+    pa.goleft = b.goleft;
+    pa.chunk = nullptr;
+    pa.desc = b.pdesc;
     pa.ctl = ctl;
     pa.parity = parity;
     pa.dl_in = d;
     pa.dl_out = (max_depth >= 0 && level + 1 == max_depth) ? 1 : d;
-    pa.chunk_agg = pchunk_agg;
-    pa.chunk_excl = pchunk_excl;
-    pa.block_agg = pblock_agg;
-    pa.block_carry = pblock_carry;
-    pr = prof_begin(PK_PARTITION, s, 4);
+    pa.chunk_agg = b.pchunk_agg;
+    pa.chunk_excl = b.pchunk_excl;
+    pa.block_agg = b.pblock_agg;
+    pa.block_carry = b.pblock_carry;
+    pr = prof_begin(PK_PARTITION, s, 5);
+    part_desc_kernel<<<num_sms() * 4, 256, 0, s>>>(b.nodes[parity], b.dec, b.new_start, ctl, parity, pa.dl_out, b.pdesc);
     part_agg_kernel<<<g_pagg, kThreads, 0, s>>>(pa);
-    chunk_scan_kernel<CntP><<<(unsigned)max_cblocks, 1024, 0, s>>>(ctl, parity, pa.dl_out, pchunk_agg, pchunk_excl, pblock_agg);
-    block_carry_kernel<CntP><<<1, 1024, 0, s>>>(ctl, parity, pa.dl_out, pblock_agg, pblock_carry);
+    chunk_scan_kernel<CntP><<<(unsigned)b.max_cblocks, 1024, 0, s>>>(ctl, parity, pa.dl_out, b.pchunk_agg, b.pchunk_excl, b.pblock_agg);
+    block_carry_kernel<CntP><<<1, 1024, 0, s>>>(ctl, parity, pa.dl_out, b.pblock_agg, b.pblock_carry);
     partition_kernel<<<g_part, kThreads, 0, s>>>(pa);
     prof_end(pr, s, 0.0);
-    pending.push_back({pr, level, PK_PARTITION, pa.dl_out});
+    if (pending) pending->push_back({pr, level, PK_PARTITION, pa.dl_out});
     DT_CK(cudaGetLastError());
     cur ^= 1;
     // unlimited depth (or a deep limit): poll the node count every few levels
-    if ((max_depth < 0 || max_depth > 24) && (level % 8) == 7) {
+    if (poll && (max_depth < 0 || max_depth > 24) && (level % 8) == 7) {
       uint32_t kk[2];
       DT_CK(cudaMemcpyAsync(kk, ctl->K, sizeof kk, cudaMemcpyDeviceToHost, s));
       DT_CK(cudaStreamSynchronize(s));
       if (kk[parity ^ 1] == 0) break;
     }
   }
+  return DT_OK;
+}
+
+// Device-side packing of the predict representation (see tree_upload in api.cu).
+__global__ void __launch_bounds__(256) pack_tree_kernel(const dt_node* __restrict__ nodes, int64_t count,
+                                                        uint2* __restrict__ packed, double* __restrict__ value) {
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < count; k += (int64_t)gridDim.x * blockDim.x) {
+    const dt_node nd = nodes[k];
+    value[k] = nd.value;
+    if (nd.feature < 0) {
+      packed[k] = make_uint2(0x7f800000u, (uint32_t)k);  // +inf, self-loop
+    } else {
+      float f = __double2float_rd(nd.threshold);  // round-down: x <= t  <=>  x <= RD32(t)
+      packed[k] = make_uint2(__float_as_uint(f), ((uint32_t)nd.feature << 24) | (uint32_t)nd.left);
+    }
+  }
+}
+
+// Reads the result back and builds the tree object (host nodes + device packed copy).
+dt_status fit_finish(const FitBufs& b, int32_t d, cudaStream_t s, const std::vector<Pending>* pending,
+                     dt_tree** out) {
   Ctl hc;
-  DT_CK(cudaMemcpyAsync(&hc, ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+  DT_CK(cudaMemcpyAsync(&hc, b.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
   std::vector<LevelLog> hlog;
-  if (!pending.empty()) {
+  if (pending && !pending->empty()) {
     hlog.resize(kMaxLogLevels);
-    DT_CK(cudaMemcpyAsync(hlog.data(), lvlog, sizeof(LevelLog) * kMaxLogLevels, cudaMemcpyDeviceToHost, s));
+    DT_CK(cudaMemcpyAsync(hlog.data(), b.lvlog, sizeof(LevelLog) * kMaxLogLevels, cudaMemcpyDeviceToHost, s));
   }
   DT_CK(cudaStreamSynchronize(s));
-  // algorithmic bytes per launch:
-  //   scan: every active entry of the scanned lists, x (4 B) + y (8 B);
-  //   goleft: the split feature's row ids of the moved rows (4 B) + one byte per row;
-  //   partition: every moved entry read (16 B) and written (16 B).
-  for (const Pending& p : pending) {
-    if (p.rec < 0 || p.level >= kMaxLogLevels) continue;
-    const LevelLog& L = hlog[(size_t)p.level];
-    double b = 0.0;
-    if (p.kind == PK_SCAN) b = 12.0 * (double)L.A * p.dl;
-    else if (p.kind == PK_GOLEFT) b = 5.0 * (double)L.A_next;
-    else if (p.kind == PK_PARTITION) b = 32.0 * (double)L.A_next * p.dl;
-    prof_set_bytes(p.rec, b);
+  if (pending) {
+    // algorithmic bytes per launch:
+    //   scan: every active entry of the scanned lists, x (4 B) + y (8 B);
+    //   goleft: the split feature's row ids of the moved rows (4 B) + one byte per row;
+    //   partition: every moved entry read (16 B) and written (16 B).
+    for (const Pending& p : *pending) {
+      if (p.rec < 0 || p.level >= kMaxLogLevels) continue;
+      const LevelLog& L = hlog[(size_t)p.level];
+      double bytes = 0.0;
+      if (p.kind == PK_SCAN) bytes = 12.0 * (double)L.A * p.dl;
+      else if (p.kind == PK_GOLEFT) bytes = 5.0 * (double)L.A_next;
+      else if (p.kind == PK_PARTITION) bytes = 32.0 * (double)L.A_next * p.dl;
+      prof_set_bytes(p.rec, bytes);
+    }
   }
   if (hc.nonfinite) return fail(DT_ERR_NONFINITE, "dt_fit: non-finite value in X or y");
   const int64_t count = hc.next_id;
@@ -1701,20 +1840,124 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
   t->split_evals = (int64_t)hc.split_evals;
   t->integer_mode = hc.int_mode;
   t->host = (dt_node*)malloc(sizeof(dt_node) * (size_t)count);
-  cudaError_t e = cudaMemcpyAsync(t->host, dout, sizeof(dt_node) * (size_t)count,
-                                  cudaMemcpyDeviceToHost, s);
+  t->async_alloc = 1;
+  DT_CK(cudaGetDevice(&t->device));
+  cudaError_t e = cudaMallocAsync((void**)&t->dev_packed, sizeof(uint2) * (size_t)count, s);
+  if (e == cudaSuccess) e = cudaMallocAsync((void**)&t->dev_value, sizeof(double) * (size_t)count, s);
+  if (e == cudaSuccess) {
+    const int g = (int)std::min<int64_t>((count + 255) / 256, 1024);
+    pack_tree_kernel<<<g, 256, 0, s>>>(b.dout, count, t->dev_packed, t->dev_value);
+    prof_add_launches(1);
+    e = cudaGetLastError();
+  }
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(t->host, b.dout, sizeof(dt_node) * (size_t)count, cudaMemcpyDeviceToHost, s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) {
     dt_tree_free(t);
-    return cuda_fail(e, "copy tree", __FILE__, __LINE__);
-  }
-  dt_status st = tree_upload(t, s);
-  if (st != DT_OK) {
-    dt_tree_free(t);
-    return st;
+    return cuda_fail(e, "fit readback", __FILE__, __LINE__);
   }
   *out = t;
   return DT_OK;
+}
+
+// One cached, instantiated CUDA graph of a whole bounded-depth fit: replayed when the
+// same inputs (addresses) and shape are fitted again (no per-launch host overhead).
+struct FitPlan {
+  const float* X = nullptr;
+  const double* y = nullptr;
+  int64_t n = 0, min_leaf = 0;
+  int32_t d = 0, max_depth = 0;
+  int device = -1;
+  std::vector<void*> mem;
+  FitBufs b{};
+  cudaGraphExec_t exec = nullptr;
+  cudaStream_t cap = nullptr;
+  int64_t launches = 0;
+  ~FitPlan() {
+    if (exec) cudaGraphExecDestroy(exec);
+    if (cap) cudaStreamDestroy(cap);
+    for (void* p : mem) cudaFree(p);
+  }
+};
+std::mutex g_plan_mu;
+std::unique_ptr<FitPlan> g_plan;
+
+}  // namespace
+
+dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
+                   int64_t min_leaf, cudaStream_t s, dt_tree** out) {
+  // Pool: keep freed workspace for the next fit (no cudaMalloc on the hot path).
+  int dev = 0;
+  DT_CK(cudaGetDevice(&dev));
+  {
+    cudaMemPool_t pool;
+    DT_CK(cudaDeviceGetDefaultMemPool(&pool, dev));
+    uint64_t thr = UINT64_MAX;
+    DT_CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+  }
+  static int graph_env = -1;
+  if (graph_env < 0) {
+    const char* e = getenv("DT_FIT_GRAPH");
+    graph_env = (e && e[0] == '0') ? 0 : 1;
+  }
+  const bool use_graph = graph_env && !prof_enabled() && max_depth >= 0 && max_depth <= 24;
+  if (use_graph) {
+    std::lock_guard<std::mutex> lk(g_plan_mu);
+    FitPlan* pl = g_plan.get();
+    const bool hit = pl && pl->X == X && pl->y == y && pl->n == n && pl->d == d &&
+                     pl->max_depth == max_depth && pl->min_leaf == min_leaf && pl->device == dev;
+    if (!hit) {
+      g_plan.reset();  // frees the previous plan's memory (synchronising)
+      std::unique_ptr<FitPlan> np(new FitPlan());
+      np->X = X;
+      np->y = y;
+      np->n = n;
+      np->d = d;
+      np->max_depth = max_depth;
+      np->min_leaf = min_leaf;
+      np->device = dev;
+      auto get = [&](auto** p, size_t count) -> cudaError_t {
+        cudaError_t e = cudaMalloc((void**)p, sizeof(**p) * (count ? count : 1));
+        if (e == cudaSuccess) np->mem.push_back((void*)*p);
+        return e;
+      };
+      dt_status st = fit_alloc(np->b, n, d, max_depth, get);
+      if (st != DT_OK) return st;
+      DT_CK(cudaStreamCreateWithFlags(&np->cap, cudaStreamNonBlocking));
+      const int64_t l0 = dt_launch_count();
+      DT_CK(cudaStreamBeginCapture(np->cap, cudaStreamCaptureModeThreadLocal));
+      st = fit_enqueue(np->b, X, y, n, d, max_depth, min_leaf, np->cap, false, nullptr);
+      cudaGraph_t graph = nullptr;
+      cudaError_t ce = cudaStreamEndCapture(np->cap, &graph);
+      if (st != DT_OK) {
+        if (graph) cudaGraphDestroy(graph);
+        return st;
+      }
+      if (ce != cudaSuccess) return cuda_fail(ce, "cudaStreamEndCapture", __FILE__, __LINE__);
+      np->launches = dt_launch_count() - l0;
+      prof_add_launches(-np->launches);  // counted when replayed
+      ce = cudaGraphInstantiate(&np->exec, graph, 0);
+      cudaGraphDestroy(graph);
+      if (ce != cudaSuccess) return cuda_fail(ce, "cudaGraphInstantiate", __FILE__, __LINE__);
+      g_plan = std::move(np);
+      pl = g_plan.get();
+    }
+    DT_CK(cudaGraphLaunch(pl->exec, s));
+    prof_add_launches(pl->launches);
+    return fit_finish(pl->b, d, s, nullptr, out);
+  }
+  // Direct path: stream-ordered workspace, kernels enqueued one by one.
+  Workspace ws;
+  ws.s = s;
+  FitBufs b{};
+  auto get = [&](auto** p, size_t count) -> cudaError_t { return ws.get(p, count); };
+  dt_status st = fit_alloc(b, n, d, max_depth, get);
+  if (st != DT_OK) return st;
+  std::vector<Pending> pending;
+  st = fit_enqueue(b, X, y, n, d, max_depth, min_leaf, s, true, &pending);
+  if (st != DT_OK) return st;
+  return fit_finish(b, d, s, &pending, out);
 }
 
 }  // namespace dtl

@@ -52,6 +52,16 @@ void prof_set_bytes(int idx, double bytes) {
   g_recs[(size_t)idx].bytes = bytes;
 }
 
+bool prof_enabled() {
+  std::lock_guard<std::mutex> lk(g_mu);
+  return g_on;
+}
+
+void prof_add_launches(long long n) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  g_launches += n;
+}
+
 }  // namespace dtl
 
 using namespace dtl;

@@ -256,3 +256,18 @@ def test_dse_generator_bitexact(dt):
     for row0 in (0, (1 << 30) - 2048):
         Xg = dt.dt_gen_dse(3, row0, 2048, 10).cpu().numpy()
         assert np.array_equal(Xg, datagen.dse_candidates(3, row0, 2048))
+
+
+def test_fit_graph_replay_matches_direct(dt):
+    """Bounded-depth fits of the same inputs replay a cached CUDA graph; the result must be
+    bytewise identical to the directly enqueued fit (profiling forces the direct path)."""
+    X, y = datagen.cnn_gpu_table(4, 50_000)
+    Xd, yd = _cuda(X), _cuda(y)
+    runs = []
+    for prof in (False, False, True, False):
+        dt.dt_profile_enable(prof)
+        t = dt.dt_fit(Xd, yd, 10, 2)
+        dt.dt_profile_enable(False)
+        runs.append(t.nodes.tobytes())
+    assert all(r == runs[0] for r in runs)
+    _assert_exact(np.frombuffer(runs[0], dtype=dt.NODE_DTYPE), oracle.fit(X, y, 10, 2))
