@@ -157,6 +157,32 @@ dt_status dt_gen_table(uint64_t seed, int64_t row0, int64_t n, int32_t d, int32_
 dt_status dt_gen_dse(uint64_t seed, int64_t row0, int64_t n, int32_t gpu_bits,
                      float* X_dev, void* stream);
 
+/* ------------------------------------------------------------------ multi-GPU ----- */
+
+/* One process (or host thread) per GPU.  Feature-sharded exact fit (DESIGN.md,
+ * "Multi-GPU"): rank r of `world` builds and scans the feature lists of the
+ * global features j*world + r only; per level the ranks allgather their per-node best
+ * splits (reduced in the fixed order of dt_fit: highest gain, then lowest feature, then
+ * lowest threshold) and max-allreduce the go-left byte map.  Every rank passes the FULL
+ * table (X n x d, y) and receives the same tree, identical to dt_fit's (tests/).
+ *   dt_comm_unique_id: 128-byte NCCL id, created by rank 0 and broadcast by the caller
+ *     (e.g. torch.distributed); dt_comm_init: NCCL communicator on the current device
+ *     (libnccl.so.2 is loaded at run time; DT_ERR_NCCL if absent).
+ *   dt_comm_init_local: `world` communicators for host THREADS of one process (device
+ *     copies behind a host barrier), e.g. to run the sharded path on a single GPU.
+ * dt_fit_sharded: world <= d; otherwise as dt_fit (sync). */
+typedef struct dt_comm dt_comm;
+int32_t dt_comm_unique_id_bytes(void);
+dt_status dt_comm_unique_id(void* id_out);
+dt_status dt_comm_init(const void* id, int32_t rank, int32_t world, dt_comm** out);
+dt_status dt_comm_init_local(int32_t world, dt_comm** comms_out);
+void dt_comm_free(dt_comm* comm);
+int32_t dt_comm_rank(const dt_comm* comm);
+int32_t dt_comm_world(const dt_comm* comm);
+dt_status dt_fit_sharded(dt_comm* comm, const float* X_dev, const double* y_dev, int64_t n,
+                         int32_t d, int32_t max_depth, int64_t min_samples_leaf, void* stream,
+                         dt_tree** out);
+
 /* ------------------------------------------------------------------ profiling ----- */
 
 /* Measurement hooks used by bench.py (not needed to use the library).  While enabled,

@@ -32,7 +32,9 @@ SYMBOLS = ("dt_fit", "dt_tree_size", "dt_tree_nodes", "dt_tree_depth", "dt_tree_
            "dt_tree_split_evals", "dt_tree_from_nodes", "dt_tree_free", "dt_predict", "dt_eval",
            "dt_predict_eval", "dt_loo", "dt_gen_table", "dt_gen_dse", "dt_last_error",
            "dt_version", "dt_profile_enable", "dt_profile_reset", "dt_launch_count",
-           "dt_profile_kinds", "dt_profile_get")
+           "dt_profile_kinds", "dt_profile_get", "dt_comm_unique_id_bytes", "dt_comm_unique_id",
+           "dt_comm_init", "dt_comm_init_local", "dt_comm_free", "dt_comm_rank", "dt_comm_world",
+           "dt_fit_sharded")
 
 
 class DTError(RuntimeError):
@@ -75,6 +77,14 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "dt_profile_kinds": ([], I32),
         "dt_profile_get": ([I32, ctypes.POINTER(ctypes.c_char_p), ctypes.POINTER(I64),
                             ctypes.POINTER(D), ctypes.POINTER(D)], ctypes.c_int),
+        "dt_comm_unique_id_bytes": ([], I32),
+        "dt_comm_unique_id": ([P], ctypes.c_int),
+        "dt_comm_init": ([P, I32, I32, ctypes.POINTER(P)], ctypes.c_int),
+        "dt_comm_init_local": ([I32, P], ctypes.c_int),
+        "dt_comm_free": ([P], None),
+        "dt_comm_rank": ([P], I32),
+        "dt_comm_world": ([P], I32),
+        "dt_fit_sharded": ([P, P, P, I64, I32, I32, I64, P, ctypes.POINTER(P)], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -260,6 +270,64 @@ def dt_profile() -> dict:
             out[name.value.decode()] = dict(launches=int(cnt.value), ms=float(ms.value),
                                             alg_bytes=float(by.value))
     return out
+
+
+class Comm:
+    """Owns a ``dt_comm*`` (one rank of a feature-sharded fit)."""
+
+    def __init__(self, handle: ctypes.c_void_p):
+        self._h = handle
+
+    @property
+    def handle(self):
+        return self._h
+
+    @property
+    def rank(self) -> int:
+        return int(_lib.dt_comm_rank(self._h))
+
+    @property
+    def world(self) -> int:
+        return int(_lib.dt_comm_world(self._h))
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h is not None and h.value:
+            _lib.dt_comm_free(h)
+            self._h = None
+
+
+def dt_comm_init_nccl(rank: int, world: int, broadcast) -> Comm:
+    """NCCL communicator; ``broadcast(obj)`` must return rank 0's object on every rank
+    (e.g. a torch.distributed broadcast_object_list wrapper)."""
+    nb = int(_lib.dt_comm_unique_id_bytes())
+    uid = (ctypes.c_char * nb)()
+    if rank == 0:
+        _check(_lib.dt_comm_unique_id(uid))
+    raw = broadcast(bytes(uid) if rank == 0 else None)
+    uid = (ctypes.c_char * nb).from_buffer_copy(raw)
+    h = ctypes.c_void_p()
+    _check(_lib.dt_comm_init(uid, rank, world, ctypes.byref(h)))
+    return Comm(h)
+
+
+def dt_comm_init_local(world: int):
+    """``world`` communicators for host threads of this process (single-GPU sharding)."""
+    arr = (ctypes.c_void_p * world)()
+    _check(_lib.dt_comm_init_local(world, arr))
+    return [Comm(ctypes.c_void_p(arr[i])) for i in range(world)]
+
+
+def dt_fit_sharded(comm: Comm, X, y, max_depth: int = -1, min_samples_leaf: int = 1,
+                   stream=None) -> Tree:
+    import torch
+    xp = _dev(X, torch.float32, 2, "X")
+    yp = _dev(y, torch.float64, 1, "y")
+    n, d = X.shape
+    h = ctypes.c_void_p()
+    _check(_lib.dt_fit_sharded(comm.handle, xp, yp, n, d, max_depth, min_samples_leaf,
+                               _stream(stream), ctypes.byref(h)))
+    return Tree(h)
 
 
 def version() -> str:

@@ -20,6 +20,11 @@ FLAGS = [
     "-cudart", "static",
     "-I", os.path.join(ROOT, "include"),
 ]
+# nccl.h for the communicator types (libnccl.so.2 itself is dlopen'ed at run time)
+for _inc in ("/usr/include", os.path.join(os.path.dirname(os.__file__), "site-packages", "nvidia", "nccl", "include")):
+    if os.path.exists(os.path.join(_inc, "nccl.h")):
+        FLAGS += ["-I", _inc]
+        break
 
 
 def sources():
@@ -59,7 +64,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise RuntimeError("nvcc failed")
     tmp = LIB + f".tmp{os.getpid()}"
     subprocess.check_call([NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared",
-                           "-cudart", "static", "-o", tmp, *objs])
+                           "-cudart", "static", "-o", tmp, *objs, "-ldl"])
     os.replace(tmp, LIB)
     return LIB
 

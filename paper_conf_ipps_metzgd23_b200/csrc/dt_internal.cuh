@@ -41,6 +41,13 @@ dt_status tree_upload(dt_tree* t, cudaStream_t s);
 // Fit driver (fit.cu).
 dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
                    int64_t min_leaf, cudaStream_t s, dt_tree** out);
+dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64_t n, int32_t dg,
+                           int32_t max_depth, int64_t min_leaf, cudaStream_t s, dt_tree** out);
+// Communicators (comm.cu).
+int comm_rank(const dt_comm* c);
+int comm_world(const dt_comm* c);
+dt_status comm_allgather(dt_comm* c, const void* send, void* recv, size_t bytes, cudaStream_t s);
+dt_status comm_allreduce_max_u8(dt_comm* c, uint8_t* buf, int64_t n, cudaStream_t s);
 // Predict / eval (predict.cu).
 dt_status predict_impl(const dt_tree* t, const float* X, int64_t n, int32_t d, double* yhat,
                        cudaStream_t s);

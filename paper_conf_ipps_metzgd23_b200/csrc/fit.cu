@@ -50,10 +50,21 @@ struct NodeL {
 };
 
 struct Decision {
-  int32_t f;    // split feature, -1 = leaf
-  uint32_t nl;  // rows going left (first nl in f-order)
-  double sl;    // S'_L (parent-centred) at the split
-  double thr;   // threshold
+  int32_t f;     // split feature (global index), -1 = leaf
+  uint32_t nl;   // rows going left (first nl in f-order)
+  int32_t floc;  // local list index of f on this rank, -1 if another rank owns f
+  int32_t pad;
+  double sl;     // S'_L (parent-centred) at the split
+  double thr;    // threshold
+};
+
+// Per-node result of one rank's local split search (exchanged across ranks).
+struct ExchRec {
+  double gain;          // -1 = no valid candidate on this rank
+  double sl, thr;
+  uint32_t i;
+  int32_t gf;           // global feature index of the local best
+  double sse, ymin, ymax, s1;  // node statistics from this rank's first feature list
 };
 
 struct Ctl {
@@ -253,14 +264,17 @@ __global__ void root_init_kernel(const double* parts, int nparts, int64_t n, int
 // ----------------------------------------------------------------------------- presort --
 
 // keys[f*n + r] = f << 32 | flip(x[r][f]); vals = r.  X row-major -> feature-major via smem.
+// Feature sharding: this rank's local feature j is global column j * world + rank of the
+// row-major X (row stride dg); keys are built for the d local features only.
 __global__ void __launch_bounds__(256) presort_keys_kernel(const float* __restrict__ X, int64_t n, int d,
                                                            unsigned long long* __restrict__ keys,
-                                                           uint32_t* __restrict__ vals, Ctl* ctl) {
-  extern __shared__ float tileX[];  // 256 rows x d
-  const int64_t r0 = (int64_t)blockIdx.x * 256;
-  const int rows = (int)min((int64_t)256, n - r0);
-  const int64_t base = r0 * d;
-  const int tot = rows * d;
+                                                           uint32_t* __restrict__ vals, Ctl* ctl, int dg,
+                                                           int world, int rank, int rb) {
+  extern __shared__ float tileX[];  // rb rows x dg
+  const int64_t r0 = (int64_t)blockIdx.x * rb;
+  const int rows = (int)min((int64_t)rb, n - r0);
+  const int64_t base = r0 * dg;
+  const int tot = rows * dg;
   bool bad = false;
   for (int i = threadIdx.x; i < tot; i += blockDim.x) {
     float v = X[base + i];
@@ -271,7 +285,7 @@ __global__ void __launch_bounds__(256) presort_keys_kernel(const float* __restri
   for (int f = 0; f < d; ++f) {
     if (threadIdx.x < rows) {
       const int64_t r = r0 + threadIdx.x;
-      const float v = tileX[threadIdx.x * d + f];
+      const float v = tileX[threadIdx.x * dg + f * world + rank];
       keys[(int64_t)f * n + r] = ((unsigned long long)f << 32) | flip_f32(v);
       vals[(int64_t)f * n + r] = (uint32_t)r;
     }
@@ -988,6 +1002,8 @@ struct SelectArgs {
   LevelLog* log;
   unsigned long long* slot_gain;
   uint32_t* slot_pos;
+  ExchRec* exch;       // [K] this rank's records
+  int world, rank, dg;  // feature sharding: local feature j is global j * world + rank
 };
 
 __device__ __forceinline__ bool cand_better(double g1, uint32_t i1, double g2, uint32_t i2) {
@@ -1067,46 +1083,90 @@ __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
       int bf = -1;
       double bg = -1.0, bsl = 0.0;
       uint32_t bi = 0;
-      const bool pure = !(st.ymin < st.ymax);
-      if (nd.searchable && !pure) {
-        for (int f = 0; f < a.d; ++f)
-          if (s_gain[f] > bg) { bg = s_gain[f]; bi = s_i[f]; bsl = s_sl[f]; bf = f; }  // strict >
-        atomicAdd(&a.ctl->split_evals, (unsigned long long)nd.N * (unsigned long long)a.d);
-      }
-      Decision dc;
-      dt_node o;
-      o.depth = a.level;
-      // value = mean of the node's own rows.  Integer mode: exact fl(S/N) from the exact
-      // bookkeeping.  Real mode: centre + fresh sum (y - c) / N, and exactly y for a pure
-      // node (all rows equal), so single-row leaves reproduce their target.
-      if (a.ctl->int_mode) o.value = nd.v;
-      else o.value = pure ? st.ymin : __dadd_rn(nd.c, __ddiv_rn(st.s1, (double)nd.N));
-      o.impurity = __ddiv_rn(st.sse, (double)nd.N);
-      o.n_samples = nd.N;
-      o.left = -1;
-      o.right = -1;
+      for (int f = 0; f < a.d; ++f)
+        if (s_gain[f] > bg) { bg = s_gain[f]; bi = s_i[f]; bsl = s_sl[f]; bf = f; }  // strict >
+      ExchRec r;
+      r.gain = -1.0;
+      r.sl = 0.0;
+      r.thr = 0.0;
+      r.i = 0;
+      r.gf = -1;
       if (bf >= 0 && bg >= 0.0) {
         const int64_t pos = (int64_t)bf * (int64_t)A + nd.start + bi;
         const double xlo = (double)a.lx[pos - 1], xhi = (double)a.lx[pos];
-        dc.f = bf;
-        dc.nl = bi;
-        dc.sl = bsl;
-        dc.thr = __dadd_rn(__ddiv_rn(xlo, 2.0), __ddiv_rn(xhi, 2.0));  // Reading R5
-        o.feature = bf;
-        o.threshold = dc.thr;
-      } else {
-        dc.f = -1;
-        dc.nl = 0;
-        dc.sl = 0.0;
-        dc.thr = 0.0;
-        o.feature = -1;
-        o.threshold = 0.0;
+        r.gain = bg;
+        r.sl = bsl;
+        r.i = bi;
+        r.gf = bf * a.world + a.rank;
+        r.thr = __dadd_rn(__ddiv_rn(xlo, 2.0), __ddiv_rn(xhi, 2.0));  // Reading R5
       }
-      a.dec[k] = dc;
-      a.out[nd.id] = o;
-      atomicMax(&a.ctl->max_depth_seen, a.level);
+      r.sse = st.sse;
+      r.ymin = st.ymin;
+      r.ymax = st.ymax;
+      r.s1 = st.s1;
+      a.exch[k] = r;
     }
     __syncthreads();
+  }
+}
+
+// Combines the ranks' records of every node (fixed order: highest gain, then lowest
+// global feature, Reading R4; statistics from rank 0, which owns feature 0) and applies
+// the leaf rules (Reading R8).  Identical inputs on every rank -> identical trees.
+__global__ void __launch_bounds__(256) decide_kernel(SelectArgs a, const ExchRec* __restrict__ all,
+                                                     int64_t stride) {
+  const uint32_t K = a.ctl->K[a.parity];
+  for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < K; k += gridDim.x * blockDim.x) {
+    const NodeL nd = a.nodes[k];
+    const ExchRec st = all[k];  // rank 0
+    const bool pure = !(st.ymin < st.ymax);
+    int bf = -1;
+    ExchRec best;
+    best.gain = -1.0;
+    if (nd.searchable && !pure) {
+      for (int r = 0; r < a.world; ++r) {
+        const ExchRec c = all[(int64_t)r * stride + k];
+        if (c.gain < 0.0) continue;
+        if (bf < 0 || c.gain > best.gain || (c.gain == best.gain && c.gf < bf)) {
+          best = c;
+          bf = c.gf;
+        }
+      }
+      atomicAdd(&a.ctl->split_evals, (unsigned long long)nd.N * (unsigned long long)a.dg);
+    }
+    Decision dc;
+    dt_node o;
+    o.depth = a.level;
+    // value = mean of the node's own rows.  Integer mode: exact fl(S/N) from the exact
+    // bookkeeping.  Real mode: centre + fresh sum (y - c) / N, and exactly y for a pure
+    // node (all rows equal), so single-row leaves reproduce their target.
+    if (a.ctl->int_mode) o.value = nd.v;
+    else o.value = pure ? st.ymin : __dadd_rn(nd.c, __ddiv_rn(st.s1, (double)nd.N));
+    o.impurity = __ddiv_rn(st.sse, (double)nd.N);
+    o.n_samples = nd.N;
+    o.left = -1;
+    o.right = -1;
+    dc.pad = 0;
+    if (bf >= 0) {
+      dc.f = bf;
+      dc.floc = (bf % a.world == a.rank) ? bf / a.world : -1;
+      dc.nl = best.i;
+      dc.sl = best.sl;
+      dc.thr = best.thr;
+      o.feature = bf;
+      o.threshold = best.thr;
+    } else {
+      dc.f = -1;
+      dc.floc = -1;
+      dc.nl = 0;
+      dc.sl = 0.0;
+      dc.thr = 0.0;
+      o.feature = -1;
+      o.threshold = 0.0;
+    }
+    a.dec[k] = dc;
+    a.out[nd.id] = o;
+    atomicMax(&a.ctl->max_depth_seen, a.level);
   }
 }
 
@@ -1245,8 +1305,8 @@ __global__ void __launch_bounds__(256) goleft_kernel(const uint32_t* __restrict_
       const uint32_t q = (uint32_t)q0 + j;
       while (q >= kend) { ++k; kstart = kend; kend = kstart + nodes[k].N; }
       const Decision dc = dec[k];
-      if (dc.f >= 0) {
-        const uint32_t r = lr[(int64_t)dc.f * (int64_t)A + q];
+      if (dc.floc >= 0) {
+        const uint32_t r = lr[(int64_t)dc.floc * (int64_t)A + q];
         goleft[r] = (q - kstart < dc.nl) ? 1 : 0;
       }
     }
@@ -1543,13 +1603,20 @@ struct FitBufs {
   PartDesc* pdesc;
   SumP *chunk_agg, *chunk_excl, *block_agg, *block_carry;
   CntP *pchunk_agg, *pchunk_excl, *pblock_agg, *pblock_carry;
+  ExchRec *exch_send, *exch_all;
   int64_t kcap, out_cap, max_chunks, max_cblocks, root_np, root_chunk;
   int fbits;
 };
 
+// Feature sharding context: this rank owns global features j * world + rank.
+struct ShardCtx {
+  dt_comm* comm;
+  int world, rank, dg;
+};
+
 // Allocates every buffer through `get` (stream-ordered or persistent).
 template <class Get>
-dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, Get get) {
+dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, int world, Get get) {
   const int64_t total0 = n * (int64_t)d;
   b.kcap = n;
   if (max_depth >= 0 && max_depth < 40) b.kcap = std::min<int64_t>(b.kcap, (int64_t)1 << max_depth);
@@ -1567,6 +1634,7 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, Get get
   }
   b.fbits = 0;
   while ((1 << b.fbits) < d) ++b.fbits;
+  if (b.fbits > 8) b.fbits = 8;
   for (int k = 0; k < 2; ++k) {
     DT_CK(get(&b.lx[k], (size_t)total0));
     DT_CK(get(&b.lr[k], (size_t)total0));
@@ -1605,6 +1673,9 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, Get get
   DT_CK(get(&b.pchunk_excl, (size_t)b.max_chunks));
   DT_CK(get(&b.pblock_agg, (size_t)b.max_cblocks));
   DT_CK(get(&b.pblock_carry, (size_t)b.max_cblocks));
+  DT_CK(get(&b.exch_send, (size_t)b.kcap));
+  if (world > 1) DT_CK(get(&b.exch_all, (size_t)b.kcap * world));
+  else b.exch_all = b.exch_send;
   return DT_OK;
 }
 
@@ -1616,7 +1687,7 @@ struct Pending {
 // Enqueues the whole fit on stream s (no host synchronisation unless `poll`).
 dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t n, int32_t d,
                       int32_t max_depth, int64_t min_leaf, cudaStream_t s, bool poll,
-                      std::vector<Pending>* pending) {
+                      std::vector<Pending>* pending, const ShardCtx& sh) {
   const int64_t total0 = n * (int64_t)d;
   DT_CK(cudaMemsetAsync(b.slot_gain, 0, sizeof(unsigned long long) * (size_t)b.kcap * d, s));
   // piece records carry the level that wrote them; none may match before it is written
@@ -1637,12 +1708,14 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
   }
   // ---- presort (a2): per-feature stable sort of (x, row), SoA level-0 lists
   {
-    const int64_t nb = (n + 255) / 256;
-    const size_t smem = sizeof(float) * 256 * (size_t)d;
+    const int rb = sh.dg <= 48 ? 256 : (sh.dg <= 96 ? 128 : 64);  // rows per block (smem)
+    const int64_t nb = (n + rb - 1) / rb;
+    const size_t smem = sizeof(float) * rb * (size_t)sh.dg;
     if (smem > 48 * 1024)
       DT_CK(cudaFuncSetAttribute(presort_keys_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int pr = prof_begin(PK_PRESORT_KEYS, s, 1);
-    presort_keys_kernel<<<(unsigned)nb, 256, smem, s>>>(X, n, d, b.k_in, b.v_in, ctl);
+    presort_keys_kernel<<<(unsigned)nb, 256, smem, s>>>(X, n, d, b.k_in, b.v_in, ctl, sh.dg, sh.world,
+                                                        sh.rank, rb);
     prof_end(pr, s, 16.0 * (double)total0);  // X read + (key, val) written
     DT_CK(cudaGetLastError());
     const int passes = (32 + b.fbits + 7) / 8;
@@ -1718,9 +1791,21 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     se.log = b.lvlog;
     se.slot_gain = b.slot_gain;
     se.slot_pos = b.slot_pos;
-    pr = prof_begin(PK_SELECT, s, 2);
+    se.exch = b.exch_send;
+    se.world = sh.world;
+    se.rank = sh.rank;
+    se.dg = sh.dg;
+    pr = prof_begin(PK_SELECT, s, 3);
     piece_pos_kernel<<<num_sms() * 4, 256, 0, s>>>(sa, b.slot_pos);
     select_kernel<<<g_sel, 256, 0, s>>>(se);
+    // exchange the per-node local bests (at most min(kcap, 2^level) nodes at this level)
+    const int64_t cnt = (level < 40) ? std::min<int64_t>(b.kcap, (int64_t)1 << level) : b.kcap;
+    if (sh.world > 1) {
+      dt_status cst = comm_allgather(sh.comm, b.exch_send, b.exch_all, sizeof(ExchRec) * (size_t)cnt, s);
+      if (cst != DT_OK) return cst;
+    }
+    decide_kernel<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((cnt + 255) / 256, num_sms() * 4)), 256, 0, s>>>(
+        se, b.exch_all, cnt);
     prof_end(pr, s, 0.0);
     DT_CK(cudaGetLastError());
     if (last) break;
@@ -1743,7 +1828,13 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     DT_CK(cudaGetLastError());
     // go-left map (a6)
     pr = prof_begin(PK_GOLEFT, s, 1);
+    if (sh.world > 1) DT_CK(cudaMemsetAsync(b.goleft, 0, (size_t)n, s));
     goleft_kernel<<<g_gl, 256, 0, s>>>(b.lr[cur], b.nodes[parity], b.dec, ctl, parity, b.goleft);
+    if (sh.world > 1) {
+      // the owner of each split feature wrote its rows' bytes; everyone else wrote 0
+      dt_status cst = comm_allreduce_max_u8(sh.comm, b.goleft, n, s);
+      if (cst != DT_OK) return cst;
+    }
     prof_end(pr, s, 0.0);
     if (pending) pending->push_back({pr, level, PK_GOLEFT, 1});
     DT_CK(cudaGetLastError());
@@ -1807,7 +1898,7 @@ __global__ void __launch_bounds__(256) pack_tree_kernel(const dt_node* __restric
 
 // Reads the result back and builds the tree object (host nodes + device packed copy).
 dt_status fit_finish(const FitBufs& b, int32_t d, cudaStream_t s, const std::vector<Pending>* pending,
-                     dt_tree** out) {
+                     dt_tree** out) {  // d = global feature count
   Ctl hc;
   DT_CK(cudaMemcpyAsync(&hc, b.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
   std::vector<LevelLog> hlog;
@@ -1922,12 +2013,13 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
         if (e == cudaSuccess) np->mem.push_back((void*)*p);
         return e;
       };
-      dt_status st = fit_alloc(np->b, n, d, max_depth, get);
+      dt_status st = fit_alloc(np->b, n, d, max_depth, 1, get);
       if (st != DT_OK) return st;
       DT_CK(cudaStreamCreateWithFlags(&np->cap, cudaStreamNonBlocking));
       const int64_t l0 = dt_launch_count();
       DT_CK(cudaStreamBeginCapture(np->cap, cudaStreamCaptureModeThreadLocal));
-      st = fit_enqueue(np->b, X, y, n, d, max_depth, min_leaf, np->cap, false, nullptr);
+      st = fit_enqueue(np->b, X, y, n, d, max_depth, min_leaf, np->cap, false, nullptr,
+                       ShardCtx{nullptr, 1, 0, d});
       cudaGraph_t graph = nullptr;
       cudaError_t ce = cudaStreamEndCapture(np->cap, &graph);
       if (st != DT_OK) {
@@ -1952,12 +2044,32 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
   ws.s = s;
   FitBufs b{};
   auto get = [&](auto** p, size_t count) -> cudaError_t { return ws.get(p, count); };
-  dt_status st = fit_alloc(b, n, d, max_depth, get);
+  dt_status st = fit_alloc(b, n, d, max_depth, 1, get);
   if (st != DT_OK) return st;
   std::vector<Pending> pending;
-  st = fit_enqueue(b, X, y, n, d, max_depth, min_leaf, s, true, &pending);
+  st = fit_enqueue(b, X, y, n, d, max_depth, min_leaf, s, true, &pending, ShardCtx{nullptr, 1, 0, d});
   if (st != DT_OK) return st;
   return fit_finish(b, d, s, &pending, out);
+}
+
+// Feature-sharded fit: every rank holds the full table and builds /
+// scans the feature lists j * world + rank; per level the ranks exchange their per-node
+// best splits (allgather) and the go-left bytes (max-allreduce).  Same tree on every rank.
+dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64_t n, int32_t dg,
+                           int32_t max_depth, int64_t min_leaf, cudaStream_t s, dt_tree** out) {
+  const int world = comm_world(comm), rank = comm_rank(comm);
+  if (world > dg) return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: world must be <= d (feature sharding)");
+  const int dloc = (dg - rank + world - 1) / world;
+  Workspace ws;
+  ws.s = s;
+  FitBufs b{};
+  auto get = [&](auto** p, size_t count) -> cudaError_t { return ws.get(p, count); };
+  dt_status st = fit_alloc(b, n, dloc, max_depth, world, get);
+  if (st != DT_OK) return st;
+  std::vector<Pending> pending;
+  st = fit_enqueue(b, X, y, n, dloc, max_depth, min_leaf, s, true, &pending, ShardCtx{comm, world, rank, dg});
+  if (st != DT_OK) return st;
+  return fit_finish(b, dg, s, &pending, out);
 }
 
 }  // namespace dtl

@@ -271,3 +271,50 @@ def test_fit_graph_replay_matches_direct(dt):
         runs.append(t.nodes.tobytes())
     assert all(r == runs[0] for r in runs)
     _assert_exact(np.frombuffer(runs[0], dtype=dt.NODE_DTYPE), oracle.fit(X, y, 10, 2))
+
+
+# ------------------------------------------------------------------ feature-sharded fit --
+
+def _sharded_fit_threads(dt, X, y, D, m, world):
+    """world ranks as host threads on this GPU (dt_comm_init_local), one stream each."""
+    import threading
+    comms = dt.dt_comm_init_local(world)
+    Xd, yd = _cuda(X), _cuda(y)
+    trees, errs = [None] * world, []
+
+    def run(r):
+        try:
+            s = torch.cuda.Stream()
+            with torch.cuda.stream(s):
+                trees[r] = dt.dt_fit_sharded(comms[r], Xd, yd, D, m, stream=s)
+        except Exception as e:  # pragma: no cover - reported below
+            errs.append(e)
+
+    th = [threading.Thread(target=run, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    assert not errs, errs
+    return trees
+
+
+@pytest.mark.parametrize("world", [2, 3, 4])
+@pytest.mark.parametrize("case", [("ties", 5000, 8, -1, 1), ("continuous", 20000, 16, 12, 1),
+                                  ("collinear", 3000, 8, -1, 1), ("mixed", 8000, 7, 6, 3)])
+def test_fit_sharded_identical(dt, world, case):
+    kind, n, d, D, m = case
+    X, y = datagen.random_table(n + world, n, d, kind=kind, int_y=True)
+    trees = _sharded_fit_threads(dt, X, y, D, m, world)
+    ref = _fit(dt, X, y, D, m)
+    for t in trees:
+        assert t.nodes.tobytes() == ref.nodes.tobytes()
+        assert t.split_evals == ref.split_evals
+    _assert_exact(trees[0].nodes, oracle.fit(X, y, D, m))
+
+
+def test_fit_sharded_c2_schema(dt):
+    X, y = datagen.cnn_gpu_table(1, 200_000)
+    trees = _sharded_fit_threads(dt, X, y, 12, 1, 4)
+    _assert_exact(trees[0].nodes, oracle.fit(X, y, 12, 1))
+    assert all(t.nodes.tobytes() == trees[0].nodes.tobytes() for t in trees)
