@@ -55,6 +55,8 @@ def parse():
     p.add_argument("--no-dse", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--e2e-steps", type=int, default=10)
+    p.add_argument("--sharded-local", type=int, default=0,
+                   help="N=1 only: also time a feature-sharded fit with this many thread ranks on the GPU")
     return p.parse_args()
 
 
@@ -201,6 +203,60 @@ def run_reference(args, world, rank):
 
 # ---------------------------------------------------------------------- ours (GPU) ----
 
+def sharded_fit_measure(args, world, rank, dev, X, y, stream):
+    """dt_fit_sharded of the configs[1] table (the same table on every rank) split by
+    features over the ranks: strong scaling of ONE fit.  With --sharded-local P on a single
+    process, P host-thread ranks share this GPU (functional check of the sharded path)."""
+    import threading
+
+    import torch
+
+    import paper_conf_ipps_metzgd23_b200 as dt
+    Xs, ys = (X, y) if world > 1 else (X, y)
+    if world > 1:
+        import torch.distributed as dist
+
+        def bcast(obj):
+            lst = [obj]
+            dist.broadcast_object_list(lst, src=0)
+            return lst[0]
+        comms = [dt.dt_comm_init_nccl(rank, world, bcast)]
+    else:
+        comms = dt.dt_comm_init_local(args.sharded_local)
+    steps = max(3, min(args.steps, 10))
+
+    def one_round():
+        trees = [None] * len(comms)
+
+        def run(i):
+            s = torch.cuda.Stream() if len(comms) > 1 else stream
+            with torch.cuda.stream(s):
+                trees[i] = dt.dt_fit_sharded(comms[i], Xs, ys, MAX_DEPTH, MIN_LEAF, stream=s)
+        th = [threading.Thread(target=run, args=(i,)) for i in range(len(comms))]
+        for t in th:
+            t.start()
+        for t in th:
+            t.join()
+        return trees
+
+    for _ in range(2):
+        one_round()
+    barrier(world)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        trees = one_round()
+    torch.cuda.synchronize()
+    dt_s = max_over_ranks(time.perf_counter() - t0, world)
+    ref = dt.dt_fit(X, y, MAX_DEPTH, MIN_LEAF)
+    same = all(t.nodes.tobytes() == ref.nodes.tobytes() for t in trees)
+    evals = trees[0].split_evals
+    return {"ranks": world if world > 1 else args.sharded_local,
+            "backend": "nccl" if world > 1 else "local-threads (one GPU)",
+            "split_evals_per_s": evals * steps / dt_s, "ms_per_fit": dt_s / steps * 1e3,
+            "identical_to_dt_fit": bool(same), "timing": "host wall clock around synchronised fits, max over ranks"}
+
+
 def run_ours(args, world, rank, local):
     import torch
 
@@ -340,6 +396,14 @@ def run_ours(args, world, rank, local):
                             "alg_bytes_per_launch": pp["alg_bytes"] / pp["launches"]}}
         del Xdse, out
 
+    # ---- feature-sharded fit across the N ranks (NCCL): one C2 fit split by features
+    sharded = None
+    if world > 1 or args.sharded_local > 1:
+        try:
+            sharded = sharded_fit_measure(args, world, rank, dev, X, y, stream)
+        except Exception as e:  # never let the extra measurement kill the headline
+            sharded = {"error": f"{type(e).__name__}: {e}"}
+
     # ---- CPU baseline: the oracle on the host (rank 0, N=1 only)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
@@ -356,7 +420,7 @@ def run_ours(args, world, rank, local):
                 "e2e": {"value": e2e_value, "unit": "split evals/s", "h2d_bytes_per_step": h2d,
                         "d2h_bytes_per_step": d2h, "steps": args.e2e_steps},
                 "gpu_launches": launches,
-                "roofline": roofline, "cpu_baseline": cpu, "dse": dse,
+                "roofline": roofline, "cpu_baseline": cpu, "dse": dse, "sharded_fit": sharded,
                 "clocks": clk.summary(),
                 "fit": {"split_evals_per_step": evals // args.steps, "tree_nodes": tree.size,
                         "tree_depth": tree.depth, "eval_mape": m["mape"], "eval_r2": m["r2"],
