@@ -128,6 +128,26 @@ dt_status dt_eval(const double* y_dev, const double* yhat_dev, int64_t n, int32_
 dt_status dt_predict_eval(const dt_tree* tree, const float* X_dev, const double* y_dev,
                           int64_t n, int32_t d, int32_t p, void* stream, dt_metrics* out);
 
+/* dt_tree_truncate -- the tree cut at `depth` (nodes of depth == depth become leaves,
+ * keeping their values).  Greedy CART is prefix-consistent: dt_fit(X, y, D', m) equals
+ * dt_tree_truncate(dt_fit(X, y, D, m), D') for D' <= D (tests), which turns a
+ * (max_depth x min_samples_leaf) grid into one deep fit per m (BASELINE configs[4]).
+ * Host-side renumbering of the BFS prefix; sync. */
+dt_status dt_tree_truncate(const dt_tree* tree, int32_t depth, dt_tree** out);
+
+/* dt_predict_eval_depths -- held-out metrics of EVERY truncation depth 0..D of the tree in
+ * one pass over (X, y): metrics_host[3*l + {0,1,2}] = (MAPE, R^2, adj-R^2) of
+ * dt_tree_truncate(tree, l), l = 0..dt_tree_depth(tree) (<= 32).  Sync. */
+dt_status dt_predict_eval_depths(const dt_tree* tree, const float* X_dev, const double* y_dev,
+                                 int64_t n, int32_t d, int32_t p, void* stream,
+                                 double* metrics_host);
+
+/* dt_importances -- feature importances (Table III; "Gini coefficient"
+ * read as the mean decrease in SSE, Reading R3): importances_host[f] = sum over nodes split
+ * on f of N*imp - N_L*imp_L - N_R*imp_R, normalised to sum 1 (all zero for a single leaf).
+ * importances_host has dt_tree_num_features(tree) entries.  Sync. */
+dt_status dt_importances(const dt_tree* tree, double* importances_host, void* stream);
+
 /* ------------------------------------------------------------------ LOO ----------- */
 
 /* dt_loo -- leave-one-out refits (BASELINE configs[0]; the paper's 70/30 split, P:197,

@@ -34,7 +34,7 @@ SYMBOLS = ("dt_fit", "dt_tree_size", "dt_tree_nodes", "dt_tree_depth", "dt_tree_
            "dt_version", "dt_profile_enable", "dt_profile_reset", "dt_launch_count",
            "dt_profile_kinds", "dt_profile_get", "dt_comm_unique_id_bytes", "dt_comm_unique_id",
            "dt_comm_init", "dt_comm_init_local", "dt_comm_free", "dt_comm_rank", "dt_comm_world",
-           "dt_fit_sharded")
+           "dt_fit_sharded", "dt_tree_truncate", "dt_predict_eval_depths", "dt_importances")
 
 
 class DTError(RuntimeError):
@@ -85,6 +85,9 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "dt_comm_rank": ([P], I32),
         "dt_comm_world": ([P], I32),
         "dt_fit_sharded": ([P, P, P, I64, I32, I32, I64, P, ctypes.POINTER(P)], ctypes.c_int),
+        "dt_tree_truncate": ([P, I32, ctypes.POINTER(P)], ctypes.c_int),
+        "dt_predict_eval_depths": ([P, P, P, I64, I32, I32, P, P], ctypes.c_int),
+        "dt_importances": ([P, P, P], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -270,6 +273,46 @@ def dt_profile() -> dict:
             out[name.value.decode()] = dict(launches=int(cnt.value), ms=float(ms.value),
                                             alg_bytes=float(by.value))
     return out
+
+
+def dt_tree_truncate(tree: Tree, depth: int) -> Tree:
+    h = ctypes.c_void_p()
+    _check(_lib.dt_tree_truncate(tree.handle, depth, ctypes.byref(h)))
+    return Tree(h)
+
+
+def dt_predict_eval_depths(tree: Tree, X, y, p: int, stream=None):
+    """[(mape, r2, adj_r2)] for every truncation depth 0..tree.depth, one pass."""
+    import torch
+    xp = _dev(X, torch.float32, 2, "X")
+    yp = _dev(y, torch.float64, 1, "y")
+    out = np.empty(3 * (tree.depth + 1), dtype=np.float64)
+    _check(_lib.dt_predict_eval_depths(tree.handle, xp, yp, X.shape[0], X.shape[1], p,
+                                       _stream(stream), out.ctypes.data))
+    return [tuple(out[3 * i:3 * i + 3]) for i in range(tree.depth + 1)]
+
+
+def dt_importances(tree: Tree, stream=None) -> np.ndarray:
+    out = np.empty(tree.num_features, dtype=np.float64)
+    _check(_lib.dt_importances(tree.handle, out.ctypes.data, _stream(stream)))
+    return out
+
+
+def grid_search(X, y, Xv, yv, depths, min_leafs, p=None, stream=None):
+    """(max_depth x min_samples_leaf) grid with held-out evaluation (BASELINE configs[4]):
+    one dt_fit at max(depths) per m, then dt_predict_eval_depths -- every (D, m) tree is a
+    truncation of the deep one.  Returns {(D, m): (mape, r2, adj_r2)} and the split evals
+    actually performed."""
+    p = X.shape[1] if p is None else p
+    dmax = max(depths)
+    out, evals = {}, 0
+    for m in min_leafs:
+        t = dt_fit(X, y, dmax, m, stream=stream)
+        evals += t.split_evals
+        per = dt_predict_eval_depths(t, Xv, yv, p, stream=stream)
+        for D in depths:
+            out[(D, m)] = per[min(D, t.depth)]
+    return out, evals
 
 
 class Comm:

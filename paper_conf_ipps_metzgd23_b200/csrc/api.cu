@@ -202,6 +202,48 @@ dt_status dt_predict_eval(const dt_tree* t, const float* X_dev, const double* y_
   return eval_impl(y_dev, nullptr, X_dev, t, n, p, S(stream), out);
 }
 
+dt_status dt_tree_truncate(const dt_tree* t, int32_t depth, dt_tree** out) {
+  if (!out) return fail(DT_ERR_INVALID_ARG, "dt_tree_truncate: out is NULL");
+  *out = nullptr;
+  if (!t || depth < 0) return fail(DT_ERR_INVALID_ARG, "dt_tree_truncate: NULL tree or depth < 0");
+  // BFS order: the nodes of depth <= D are a prefix-closed subset; renumber them in order.
+  std::vector<int64_t> newid((size_t)t->count, -1);
+  int64_t cnt = 0;
+  for (int64_t k = 0; k < t->count; ++k)
+    if (t->host[k].depth <= depth) newid[(size_t)k] = cnt++;
+  std::vector<dt_node> nodes((size_t)cnt);
+  for (int64_t k = 0; k < t->count; ++k) {
+    if (newid[(size_t)k] < 0) continue;
+    dt_node nd = t->host[k];
+    if (nd.depth == depth || nd.feature < 0) {
+      nd.feature = -1;
+      nd.left = nd.right = -1;
+      nd.threshold = 0.0;
+    } else {
+      nd.left = (int32_t)newid[(size_t)nd.left];
+      nd.right = (int32_t)newid[(size_t)nd.right];
+    }
+    nodes[(size_t)newid[(size_t)k]] = nd;
+  }
+  dt_status st = dt_tree_from_nodes(nodes.data(), cnt, t->d, out);
+  if (st == DT_OK) (*out)->split_evals = 0;
+  return st;
+}
+
+dt_status dt_importances(const dt_tree* t, double* importances_host, void* stream) {
+  if (!t || !importances_host) return fail(DT_ERR_INVALID_ARG, "dt_importances: NULL argument");
+  return importances_impl(t, importances_host, S(stream));
+}
+
+dt_status dt_predict_eval_depths(const dt_tree* t, const float* X_dev, const double* y_dev, int64_t n,
+                                 int32_t d, int32_t p, void* stream, double* metrics_host) {
+  if (!t || !X_dev || !y_dev || !metrics_host) return fail(DT_ERR_INVALID_ARG, "dt_predict_eval_depths: NULL argument");
+  if (n < 1) return fail(DT_ERR_INVALID_ARG, "dt_predict_eval_depths: n must be >= 1");
+  if (p < 0) return fail(DT_ERR_INVALID_ARG, "dt_predict_eval_depths: p must be >= 0");
+  if (d != t->d) return fail(DT_ERR_INVALID_ARG, "dt_predict_eval_depths: d differs from the tree's d");
+  return eval_depths_impl(t, X_dev, y_dev, n, p, S(stream), metrics_host);
+}
+
 dt_status dt_loo(const float* X_dev, const double* y_dev, int64_t n, int32_t d, int32_t max_depth,
                  int64_t min_samples_leaf, double* yhat_oof_dev, void* stream) {
   if (!X_dev || !y_dev || !yhat_oof_dev) return fail(DT_ERR_INVALID_ARG, "dt_loo: NULL pointer");

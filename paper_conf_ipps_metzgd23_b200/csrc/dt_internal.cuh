@@ -53,6 +53,9 @@ dt_status predict_impl(const dt_tree* t, const float* X, int64_t n, int32_t d, d
                        cudaStream_t s);
 dt_status eval_impl(const double* y, const double* yhat, const float* X, const dt_tree* t,
                     int64_t n, int32_t p, cudaStream_t s, dt_metrics* out);
+dt_status importances_impl(const dt_tree* t, double* imp_host, cudaStream_t s);
+dt_status eval_depths_impl(const dt_tree* t, const float* X, const double* y, int64_t n, int32_t p,
+                           cudaStream_t s, double* out_host);
 // LOO (loo.cu).
 dt_status loo_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
                    int64_t min_leaf, double* yhat, cudaStream_t s);

@@ -345,7 +345,189 @@ dt_status launch_predict(const dt_tree* t, const float* X, int64_t n, int32_t d,
   return DT_OK;
 }
 
+// ------------------------------------------------------------ multi-depth eval (C5) --
+
+// One pass over held-out rows evaluates EVERY truncation depth 0..D of a tree at once:
+// the depth-l truncation predicts the value of the node the row reaches after l steps
+// (or of the leaf it stopped at).  Per-depth MAPE / SSE partials plus Welford moments of
+// y, fixed-shape reductions (deterministic).  Greedy CART fits are prefix-consistent,
+// fit(D', m) == truncate(fit(D, m), D') (tests), so a (max_depth x m) grid
+// needs one deep fit per m and this pass (BASELINE configs[4]).
+constexpr int kMaxEvalDepth = 32;
+
+struct DepthPart {
+  double ape[kMaxEvalDepth + 1];
+  double sse[kMaxEvalDepth + 1];
+  double cnt, mean, m2;
+};
+
+__global__ void __launch_bounds__(256)
+eval_depths_partial_kernel(const uint2* __restrict__ nodes, const double* __restrict__ value, int depth,
+                           const float* __restrict__ X, int d, const double* __restrict__ y, int64_t n,
+                           int64_t chunk, DepthPart* __restrict__ parts) {
+  __shared__ double sh_ape[8][kMaxEvalDepth + 1];
+  __shared__ double sh_sse[8][kMaxEvalDepth + 1];
+  __shared__ Part sh_y[32];
+  const int64_t lo = (int64_t)blockIdx.x * chunk, hi = min(n, lo + chunk);
+  double ape[kMaxEvalDepth + 1], sse[kMaxEvalDepth + 1];
+#pragma unroll
+  for (int l = 0; l <= kMaxEvalDepth; ++l) { ape[l] = 0.0; sse[l] = 0.0; }
+  Part py{0, 0, 0, 0, 0};
+  for (int64_t r = lo + threadIdx.x; r < hi; r += blockDim.x) {
+    const double yr = y[r];
+    const double den = fmax(fabs(yr), 2.220446049250313e-16);
+    const float* xr = X + r * d;
+    uint32_t k = 0;
+#pragma unroll
+    for (int l = 0; l <= kMaxEvalDepth; ++l) {
+      if (l <= depth) {
+        const double e = yr - __ldg(value + k);
+        ape[l] += __ddiv_rn(fabs(e), den);
+        sse[l] += __dmul_rn(e, e);
+        if (l < depth) k = step(nodes[k], xr);
+      }
+    }
+    py.cnt += 1.0;
+    const double delta = yr - py.mean;
+    py.mean += __ddiv_rn(delta, py.cnt);
+    py.m2 += __dmul_rn(delta, yr - py.mean);
+  }
+  // fixed-shape reduction: warp shuffles, then the 8 warps in order
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+#pragma unroll
+  for (int l = 0; l <= kMaxEvalDepth; ++l) {
+    if (l <= depth) {
+      double a = ape[l], b = sse[l];
+      for (int off = 16; off > 0; off >>= 1) {
+        a += __shfl_down_sync(0xffffffffu, a, off);
+        b += __shfl_down_sync(0xffffffffu, b, off);
+      }
+      if (lane == 0) { sh_ape[w][l] = a; sh_sse[w][l] = b; }
+    }
+  }
+  py = block_reduce(py);
+  if (threadIdx.x == 0) sh_y[0] = py;
+  __syncthreads();
+  if (threadIdx.x <= depth) {
+    const int l = threadIdx.x;
+    double a = 0.0, b = 0.0;
+    for (int ww = 0; ww < (int)(blockDim.x >> 5); ++ww) { a += sh_ape[ww][l]; b += sh_sse[ww][l]; }
+    DepthPart& o = parts[blockIdx.x];
+    o.ape[l] = a;
+    o.sse[l] = b;
+    if (l == 0) {
+      o.cnt = sh_y[0].cnt;
+      o.mean = sh_y[0].mean;
+      o.m2 = sh_y[0].m2;
+    }
+  }
+}
+
+__global__ void eval_depths_final_kernel(const DepthPart* __restrict__ parts, int nparts, int depth,
+                                         int64_t n, int p_pred, double* __restrict__ out) {
+  // thread l folds depth l in part order; thread 32 folds the y moments
+  const int l = threadIdx.x;
+  if (l <= depth) {
+    double ape = 0.0, sse = 0.0;
+    for (int i = 0; i < nparts; ++i) { ape += parts[i].ape[l]; sse += parts[i].sse[l]; }
+    double na = 0, ma = 0, Ma = 0;
+    for (int i = 0; i < nparts; ++i) chan_merge(na, ma, Ma, parts[i].cnt, parts[i].mean, parts[i].m2);
+    const double nn = (double)n;
+    double r2;
+    if (Ma == 0.0) r2 = (sse == 0.0) ? 1.0 : 0.0;
+    else r2 = 1.0 - sse / Ma;
+    double adj;
+    if (nn - (double)p_pred - 1.0 <= 0.0) adj = __longlong_as_double(0x7ff8000000000000ll);
+    else adj = 1.0 - (1.0 - r2) * (nn - 1.0) / (nn - (double)p_pred - 1.0);
+    out[3 * l] = ape / nn;
+    out[3 * l + 1] = r2;
+    out[3 * l + 2] = adj;
+  }
+}
+
+// Feature importances (NEXT-1; Table III, "Gini coefficient" read as mean
+// decrease in SSE, Reading R3): imp[f] = sum over internal nodes split on f of
+// N*imp_P - N_L*imp_L - N_R*imp_R, normalised to sum 1.  One block, fixed order.
+__global__ void __launch_bounds__(256) importances_kernel(const dt_node* __restrict__ nodes, int64_t count,
+                                                          int d, double* __restrict__ imp) {
+  __shared__ double sh[256];
+  __shared__ double tot_sh;
+  const int64_t per = (count + blockDim.x - 1) / blockDim.x;
+  const int64_t k0 = threadIdx.x * per, k1 = min(count, k0 + per);
+  for (int f = 0; f < d; ++f) {
+    double acc = 0.0;
+    for (int64_t k = k0; k < k1; ++k) {
+      const dt_node a = nodes[k];
+      if (a.feature != f) continue;
+      const dt_node L = nodes[a.left], R = nodes[a.right];
+      acc += (double)a.n_samples * a.impurity - (double)L.n_samples * L.impurity -
+             (double)R.n_samples * R.impurity;
+    }
+    sh[threadIdx.x] = acc;
+    __syncthreads();
+    for (int off = 128; off > 0; off >>= 1) {
+      if (threadIdx.x < off) sh[threadIdx.x] += sh[threadIdx.x + off];
+      __syncthreads();
+    }
+    if (threadIdx.x == 0) imp[f] = sh[0];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    double tot = 0.0;
+    for (int f = 0; f < d; ++f) tot += imp[f];
+    tot_sh = tot;
+  }
+  __syncthreads();
+  if (tot_sh > 0.0)
+    for (int f = threadIdx.x; f < d; f += blockDim.x) imp[f] = imp[f] / tot_sh;
+}
+
 }  // namespace
+
+dt_status importances_impl(const dt_tree* t, double* imp_host, cudaStream_t s) {
+  dt_node* dn = nullptr;
+  double* di = nullptr;
+  DT_CK(cudaMallocAsync((void**)&dn, sizeof(dt_node) * (size_t)t->count, s));
+  DT_CK(cudaMallocAsync((void**)&di, sizeof(double) * (size_t)t->d, s));
+  DT_CK(cudaMemcpyAsync(dn, t->host, sizeof(dt_node) * (size_t)t->count, cudaMemcpyHostToDevice, s));
+  const int pr = prof_begin(PK_EVAL, s, 1);
+  importances_kernel<<<1, 256, 0, s>>>(dn, t->count, t->d, di);
+  prof_end(pr, s, 48.0 * (double)t->count);
+  DT_CK(cudaGetLastError());
+  DT_CK(cudaMemcpyAsync(imp_host, di, sizeof(double) * (size_t)t->d, cudaMemcpyDeviceToHost, s));
+  DT_CK(cudaFreeAsync(dn, s));
+  DT_CK(cudaFreeAsync(di, s));
+  DT_CK(cudaStreamSynchronize(s));
+  return DT_OK;
+}
+
+dt_status eval_depths_impl(const dt_tree* t, const float* X, const double* y, int64_t n, int32_t p,
+                           cudaStream_t s, double* out_host) {
+  const int depth = t->depth;
+  if (depth > kMaxEvalDepth) return fail(DT_ERR_TOO_LARGE, "dt_predict_eval_depths: tree depth > 32");
+  int64_t chunk = 8192;
+  int64_t nparts = (n + chunk - 1) / chunk;
+  if (nparts > 2048) {
+    nparts = 2048;
+    chunk = (n + nparts - 1) / nparts;
+    nparts = (n + chunk - 1) / chunk;
+  }
+  DepthPart* parts = nullptr;
+  double* dout = nullptr;
+  DT_CK(cudaMallocAsync((void**)&parts, sizeof(DepthPart) * (size_t)nparts, s));
+  DT_CK(cudaMallocAsync((void**)&dout, sizeof(double) * 3 * (size_t)(depth + 1), s));
+  const int pr = prof_begin(PK_EVAL, s, 2);
+  eval_depths_partial_kernel<<<(unsigned)nparts, 256, 0, s>>>(t->dev_packed, t->dev_value, depth, X, t->d, y,
+                                                              n, chunk, parts);
+  eval_depths_final_kernel<<<1, 64, 0, s>>>(parts, (int)nparts, depth, n, p, dout);
+  prof_end(pr, s, (4.0 * t->d + 8.0) * (double)n);
+  DT_CK(cudaGetLastError());
+  DT_CK(cudaMemcpyAsync(out_host, dout, sizeof(double) * 3 * (size_t)(depth + 1), cudaMemcpyDeviceToHost, s));
+  DT_CK(cudaFreeAsync(parts, s));
+  DT_CK(cudaFreeAsync(dout, s));
+  DT_CK(cudaStreamSynchronize(s));
+  return DT_OK;
+}
 
 dt_status predict_impl(const dt_tree* t, const float* X, int64_t n, int32_t d, double* yhat,
                        cudaStream_t s) {

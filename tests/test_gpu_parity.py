@@ -318,3 +318,42 @@ def test_fit_sharded_c2_schema(dt):
     trees = _sharded_fit_threads(dt, X, y, 12, 1, 4)
     _assert_exact(trees[0].nodes, oracle.fit(X, y, 12, 1))
     assert all(t.nodes.tobytes() == trees[0].nodes.tobytes() for t in trees)
+
+
+# ------------------------------------------------------------------ grid / importances --
+
+def test_truncation_equals_shallow_fit(dt):
+    """SURVEY A.5 on the GPU: truncate(fit(D=10)) == fit(D') for every D' (integer mode)."""
+    X, y = datagen.cnn_gpu_table(5, 30000)
+    deep = _fit(dt, X, y, 10, 3)
+    for Dp in (0, 1, 4, 7, 10):
+        t = dt.dt_tree_truncate(deep, Dp).nodes
+        g = _fit(dt, X, y, Dp, 3).nodes
+        for f in ("feature", "left", "right", "depth", "n_samples", "threshold", "value", "impurity"):
+            assert np.array_equal(t[f], g[f]), (Dp, f)
+
+
+def test_grid_search_matches_oracle(dt):
+    """BASELINE configs[4] shape, small: (max_depth x min_samples_leaf) grid with held-out
+    metrics via one deep fit per m + the fused multi-depth evaluation."""
+    X, y = datagen.cnn_gpu_table(5, 20000)
+    hold = datagen.holdout_mask(5, 20000)
+    Xt, yt, Xv, yv = X[~hold], y[~hold], X[hold], y[hold]
+    depths, ms = [1, 2, 3, 5, 8], [1, 4, 32]
+    res, _ = dt.grid_search(_cuda(Xt), _cuda(yt), _cuda(Xv), _cuda(yv), depths, ms)
+    for D in depths:
+        for m in ms:
+            o = oracle.fit(Xt, yt, D, m)
+            want = oracle.evaluate(yv, oracle.predict(o, Xv), 16)
+            got = res[(D, m)]
+            for a, b in zip(got, want):
+                assert _close(a, b), (D, m, got, want)
+
+
+def test_importances_match_oracle(dt):
+    X, y = datagen.cnn_gpu_table(6, 50000)
+    t = _fit(dt, X, y, 12, 1)
+    got = dt.dt_importances(t)
+    want = oracle.importances(t.nodes, 16)
+    np.testing.assert_allclose(got, want, rtol=1e-12, atol=1e-15)
+    assert abs(got.sum() - 1.0) < 1e-12
