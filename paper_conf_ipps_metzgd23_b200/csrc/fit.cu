@@ -267,7 +267,7 @@ __global__ void root_init_kernel(const double* parts, int nparts, int64_t n, int
 // Feature sharding: this rank's local feature j is global column j * world + rank of the
 // row-major X (row stride dg); keys are built for the d local features only.
 __global__ void __launch_bounds__(256) presort_keys_kernel(const float* __restrict__ X, int64_t n, int d,
-                                                           unsigned long long* __restrict__ keys,
+                                                           uint32_t* __restrict__ keys,
                                                            uint32_t* __restrict__ vals, Ctl* ctl, int dg,
                                                            int world, int rank, int rb) {
   extern __shared__ float tileX[];  // rb rows x dg
@@ -286,14 +286,14 @@ __global__ void __launch_bounds__(256) presort_keys_kernel(const float* __restri
     if (threadIdx.x < rows) {
       const int64_t r = r0 + threadIdx.x;
       const float v = tileX[threadIdx.x * dg + f * world + rank];
-      keys[(int64_t)f * n + r] = ((unsigned long long)f << 32) | flip_f32(v);
+      keys[(int64_t)f * n + r] = flip_f32(v);
       vals[(int64_t)f * n + r] = (uint32_t)r;
     }
   }
 }
 
 // SoA level-0 lists from the sorted pairs: x = unflip(key), row = val, y = y[row].
-__global__ void __launch_bounds__(256) presort_build_kernel(const unsigned long long* __restrict__ keys,
+__global__ void __launch_bounds__(256) presort_build_kernel(const uint32_t* __restrict__ keys,
                                                             const uint32_t* __restrict__ vals,
                                                             const double* __restrict__ y, int64_t total,
                                                             float* __restrict__ lx, uint32_t* __restrict__ lr,
@@ -301,7 +301,7 @@ __global__ void __launch_bounds__(256) presort_build_kernel(const unsigned long 
   for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < total;
        p += (int64_t)gridDim.x * blockDim.x) {
     const uint32_t r = vals[p];
-    lx[p] = unflip_f32((uint32_t)keys[p]);
+    lx[p] = unflip_f32(keys[p]);
     lr[p] = r;
     ly[p] = __ldg(y + r);
   }
@@ -1595,9 +1595,9 @@ struct FitBufs {
   LevelLog* lvlog;
   RootPart* parts;
   double* cparts;
-  unsigned long long *k_in, *k_out;
+  uint32_t *k_in, *k_out;  // per feature: n keys flip(x), stable-sorted feature by feature
   uint32_t *v_in, *v_out;
-  void* sort_tmp;
+  void* sort_tmp;           // d slices of sort_tmp_bytes (one CUB sort per feature)
   size_t sort_tmp_bytes;
   ChunkDesc* sdesc;
   PartDesc* pdesc;
@@ -1661,8 +1661,9 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, int wor
   DT_CK(get(&b.v_out, (size_t)total0));
   b.sort_tmp_bytes = 0;
   DT_CK(cub::DeviceRadixSort::SortPairs(nullptr, b.sort_tmp_bytes, b.k_in, b.k_out, b.v_in, b.v_out,
-                                        total0, 0, 32 + b.fbits, (cudaStream_t)0));
-  DT_CK(get((char**)&b.sort_tmp, b.sort_tmp_bytes));
+                                        n, 0, 32, (cudaStream_t)0));
+  b.sort_tmp_bytes = (b.sort_tmp_bytes + 255) & ~(size_t)255;
+  DT_CK(get((char**)&b.sort_tmp, b.sort_tmp_bytes * (size_t)d));
   DT_CK(get(&b.sdesc, (size_t)b.max_chunks));
   DT_CK(get(&b.pdesc, (size_t)b.max_chunks));
   DT_CK(get(&b.chunk_agg, (size_t)b.max_chunks));
@@ -1677,6 +1678,24 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, int wor
   if (world > 1) DT_CK(get(&b.exch_all, (size_t)b.kcap * world));
   else b.exch_all = b.exch_send;
   return DT_OK;
+}
+
+// Per-host-thread pool of side streams for the forked per-feature sorts.
+struct SideStreams {
+  static constexpr int kN = 8;
+  cudaStream_t st[kN];
+  cudaEvent_t fork, join[kN];
+  SideStreams() {
+    for (int j = 0; j < kN; ++j) {
+      cudaStreamCreateWithFlags(&st[j], cudaStreamNonBlocking);
+      cudaEventCreateWithFlags(&join[j], cudaEventDisableTiming);
+    }
+    cudaEventCreateWithFlags(&fork, cudaEventDisableTiming);
+  }
+};
+SideStreams& side_streams() {
+  static thread_local SideStreams ss;
+  return ss;
 }
 
 // profiling records whose bytes depend on device-side counts
@@ -1718,12 +1737,27 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
                                                         sh.rank, rb);
     prof_end(pr, s, 16.0 * (double)total0);  // X read + (key, val) written
     DT_CK(cudaGetLastError());
-    const int passes = (32 + b.fbits + 7) / 8;
-    size_t tmp_bytes = b.sort_tmp_bytes;
+    // stable 32-bit radix sort of every feature's n keys (4 passes each; ties keep the
+    // row order -> (x, row id) order), the d sorts forked over side streams
     pr = prof_begin(PK_PRESORT_SORT, s, 0);  // CUB kernels: library, not counted
-    DT_CK(cub::DeviceRadixSort::SortPairs(b.sort_tmp, tmp_bytes, b.k_in, b.k_out, b.v_in, b.v_out,
-                                          total0, 0, 32 + b.fbits, s));
-    prof_end(pr, s, 24.0 * (double)total0 * passes);
+    {
+      SideStreams& ss = side_streams();
+      DT_CK(cudaEventRecord(ss.fork, s));
+      const int nside = std::min(d, SideStreams::kN);
+      for (int j = 0; j < nside; ++j) DT_CK(cudaStreamWaitEvent(ss.st[j], ss.fork, 0));
+      for (int f = 0; f < d; ++f) {
+        size_t tb = b.sort_tmp_bytes;
+        const int64_t o = (int64_t)f * n;
+        DT_CK(cub::DeviceRadixSort::SortPairs((char*)b.sort_tmp + (size_t)f * b.sort_tmp_bytes, tb,
+                                              b.k_in + o, b.k_out + o, b.v_in + o, b.v_out + o, n, 0, 32,
+                                              ss.st[f % SideStreams::kN]));
+      }
+      for (int j = 0; j < nside; ++j) {
+        DT_CK(cudaEventRecord(ss.join[j], ss.st[j]));
+        DT_CK(cudaStreamWaitEvent(s, ss.join[j], 0));
+      }
+    }
+    prof_end(pr, s, 16.0 * (double)total0 * 4);
     const int gb = std::max(1, std::min<int>((int)((total0 + 255) / 256), num_sms() * 8));
     pr = prof_begin(PK_PRESORT_BUILD, s, 1);
     presort_build_kernel<<<gb, 256, 0, s>>>(b.k_out, b.v_out, y, total0, b.lx[0], b.lr[0], b.ly[0]);
