@@ -34,8 +34,6 @@ namespace {
 
 constexpr int kThreads = 256;
 constexpr int kItems = 8;
-constexpr int kTile = kThreads * kItems;  // 2048 list entries per tile
-constexpr int kChunkLog = 4;              // chunk -> node lookup granularity (16 entries)
 
 // Per-level node record (level-local index k).
 struct NodeL {
@@ -336,18 +334,6 @@ __global__ void __launch_bounds__(256) scan_desc_kernel(const NodeL* __restrict_
   }
 }
 
-// chunk[c] = node containing position c << kChunkLog of the level's lists.
-__global__ void __launch_bounds__(256) chunk_node_kernel(const NodeL* __restrict__ nodes, const Ctl* ctl,
-                                                         int parity, uint32_t* __restrict__ chunk) {
-  const uint32_t K = ctl->K[parity];
-  const uint64_t A = ctl->A[parity];
-  if (K == 0) return;
-  const int64_t nc = (int64_t)((A + (1u << kChunkLog) - 1) >> kChunkLog);
-  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < nc;
-       c += (int64_t)gridDim.x * blockDim.x)
-    chunk[c] = find_node(nodes, K, (uint32_t)(c << kChunkLog));
-}
-
 // Cursor over the segments of a level's concatenated feature lists: segment (f, k)
 // occupies global positions [f*A + start_k, f*A + start_k + N_k).
 struct Seg {
@@ -355,24 +341,6 @@ struct Seg {
   uint32_t k;
   int f;
 };
-// chunk_node[q >> kChunkLog] = node containing list position (q >> kChunkLog) << kChunkLog,
-// rebuilt for every level (chunk_node_kernel); seg_at = one load + a short forward walk.
-
-__device__ __forceinline__ uint32_t node_of(const NodeL* __restrict__ nodes, const uint32_t* __restrict__ chunk,
-                                            uint32_t K, uint32_t q) {
-  uint32_t k = __ldg(chunk + (q >> kChunkLog));
-  while (k + 1 < K && __ldg(&nodes[k + 1].start) <= q) ++k;
-  return k;
-}
-
-__device__ __forceinline__ void seg_at(Seg& s, const NodeL* __restrict__ nodes, uint32_t K,
-                                       uint64_t A, int64_t p, const uint32_t* __restrict__ chunk) {
-  s.f = (int)(p / (int64_t)A);
-  s.fbase = (int64_t)s.f * (int64_t)A;
-  s.k = node_of(nodes, chunk, K, (uint32_t)(p - s.fbase));
-  s.start = s.fbase + __ldg(&nodes[s.k].start);
-  s.end = s.start + __ldg(&nodes[s.k].N);
-}
 __device__ __forceinline__ void seg_next(Seg& s, const NodeL* __restrict__ nodes, uint32_t K,
                                          uint64_t A) {
   if (++s.k == K) {
@@ -406,7 +374,6 @@ struct ScanArgs {
   int d;           // feature count (slot stride)
   int64_t min_leaf;
   uint32_t* counter;  // tile counter (zeroed per launch)
-  const uint32_t* chunk;  // chunk -> node table of this level
   const ChunkDesc* desc;  // per warp chunk
   SumP* chunk_agg;    // [nchunks] phase A: per-warp-chunk aggregate
   SumP* chunk_excl;   // [nchunks] phase B1: exclusive within its block of chunks
@@ -494,47 +461,6 @@ __device__ __forceinline__ void load_items(const float* __restrict__ lx, const d
       xv[j] = ok ? lx[p0 + j] : 0.f;
       yv[j] = ok ? ly[p0 + j] : 0.0;
     }
-  }
-}
-
-// Tile staging in shared memory (scan): thread t owns entries [16t, 16t+16) = 4 x-chunks
-// and 8 y-chunks of 16 B.  Chunks are fetched striped across the block (coalesced
-// global reads) and stored XOR-swizzled so that each thread's 128-bit reads of its own
-// chunks are bank-conflict-free.
-__device__ __forceinline__ int xslot(int owner, int q) { return owner * 4 + (q ^ ((owner >> 1) & 3)); }
-__device__ __forceinline__ int yslot(int owner, int q) { return owner * 8 + (q ^ (owner & 7)); }
-
-__device__ __forceinline__ void stage_tile_async(const float* __restrict__ lx, const double* __restrict__ ly,
-                                                 int64_t tbase, int64_t total, float4* sx, double2* sy) {
-  const int tid = threadIdx.x;
-#pragma unroll
-  for (int r = 0; r < kItems / 4; ++r) {  // x: 1024 chunks of 4 entries
-    const int c = r * kThreads + tid;
-    const int64_t e0 = tbase + (int64_t)c * 4;
-    const int64_t left = total - e0;
-    if (left > 0) cp_async16(sx + xslot(c >> 2, c & 3), lx + e0, left >= 4 ? 16 : (int)left * 4);
-  }
-#pragma unroll
-  for (int r = 0; r < kItems / 2; ++r) {  // y: 2048 chunks of 2 entries
-    const int c = r * kThreads + tid;
-    const int64_t e0 = tbase + (int64_t)c * 2;
-    const int64_t left = total - e0;
-    if (left > 0) cp_async16(sy + yslot(c >> 3, c & 7), ly + e0, left >= 2 ? 16 : 8);
-  }
-  cp_async_commit();
-}
-
-__device__ __forceinline__ void unstage_items(const float4* sx, const double2* sy, float* xv, double* yv) {
-  const int tid = threadIdx.x;
-#pragma unroll
-  for (int q = 0; q < kItems / 4; ++q) {
-    const float4 t = sx[xslot(tid, q)];
-    xv[4 * q] = t.x; xv[4 * q + 1] = t.y; xv[4 * q + 2] = t.z; xv[4 * q + 3] = t.w;
-  }
-#pragma unroll
-  for (int q = 0; q < kItems / 2; ++q) {
-    const double2 t = sy[yslot(tid, q)];
-    yv[2 * q] = t.x; yv[2 * q + 1] = t.y;
   }
 }
 
@@ -701,13 +627,7 @@ __global__ void __launch_bounds__(1024) block_carry_kernel(const Ctl* ctl, int p
 
 // Phase C: the main scan (prefixes, gains, per-piece argmax, node statistics), one warp
 // chunk at a time per warp, no block barriers.
-#ifndef DT_SCAN_DB
-#define DT_SCAN_DB 1
-#endif
-#ifndef DT_SCAN_OCC
-#define DT_SCAN_OCC 2
-#endif
-__global__ void __launch_bounds__(kThreads, DT_SCAN_OCC) scan_kernel(ScanArgs a) {
+__global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
   // per-thread best of the run before its first head (written and read by the same
   // thread, so no barrier is needed)
   __shared__ double fr_gain[kThreads], fr_sl[kThreads], fs_sse[kThreads], fs_min[kThreads],
@@ -730,19 +650,18 @@ __global__ void __launch_bounds__(kThreads, DT_SCAN_OCC) scan_kernel(ScanArgs a)
   // register double buffering: the next chunk's loads are in flight during this chunk
   float xn[kItems];
   double yn[kItems];
-  if (DT_SCAN_DB) {
+  {
     const int64_t q0 = gw * kChunkW + lane * kItems;
     if (gw < nch && q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
   }
   for (int64_t ch = gw; ch < nch; ch += nw) {
     const int64_t p0 = ch * kChunkW + lane * kItems;
     const bool any = p0 < total;
-    if (!DT_SCAN_DB && any) load_items(a.lx, a.ly, p0, total, xn, yn);
     float xv[kItems];
     double yv[kItems];
 #pragma unroll
     for (int j = 0; j < kItems; ++j) { xv[j] = xn[j]; yv[j] = yn[j]; }
-    if (DT_SCAN_DB) {
+    {
       const int64_t q0 = (ch + nw) * kChunkW + lane * kItems;
       if (ch + nw < nch && q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
     }
@@ -1005,10 +924,6 @@ struct SelectArgs {
   ExchRec* exch;       // [K] this rank's records
   int world, rank, dg;  // feature sharding: local feature j is global j * world + rank
 };
-
-__device__ __forceinline__ bool cand_better(double g1, uint32_t i1, double g2, uint32_t i2) {
-  return g1 > g2 || (g1 == g2 && i1 < i2);
-}
 
 // One block per node (grid-stride over the level's nodes).
 __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
@@ -1354,7 +1269,6 @@ struct PartArgs {
   const Decision* dec;
   const uint32_t* new_start;
   const uint8_t* goleft;
-  const uint32_t* chunk;
   const PartDesc* desc;  // per warp chunk
   const Ctl* ctl;
   int parity;
@@ -1452,13 +1366,9 @@ __global__ void __launch_bounds__(kThreads) part_agg_kernel(PartArgs a) {
 }
 
 // Phase C: destinations and coalesced stores.
-#ifndef DT_PART_DB
-#define DT_PART_DB 0
-#endif
-#ifndef DT_PART_OCC
-#define DT_PART_OCC 4
-#endif
-__global__ void __launch_bounds__(kThreads, DT_PART_OCC) partition_kernel(PartArgs a) {
+// 4 CTAs/SM (64 registers) and no register double buffering: occupancy hides the load
+// latency better than prefetching at 2 CTAs/SM (measured).
+__global__ void __launch_bounds__(kThreads, 4) partition_kernel(PartArgs a) {
   const uint32_t K = a.ctl->K[a.parity];
   const uint64_t A = a.ctl->A[a.parity];
   const uint64_t A2 = a.ctl->A[a.parity ^ 1];
@@ -1482,16 +1392,14 @@ __global__ void __launch_bounds__(kThreads, DT_PART_OCC) partition_kernel(PartAr
       yn[r] = ok ? __ldcs(a.ly + p) : 0.0;
     }
   };
-  if (DT_PART_DB && gw < nch) load(gw * kChunkW);
   for (int64_t ch = gw; ch < nch; ch += nw) {
     const int64_t wbase = ch * kChunkW;
-    if (!DT_PART_DB) load(wbase);
+    load(wbase);
     uint32_t rv[kRows];
     float xv[kRows];
     double yv[kRows];
 #pragma unroll
     for (int r = 0; r < kRows; ++r) { rv[r] = rn[r]; xv[r] = xn[r]; yv[r] = yn[r]; }
-    if (DT_PART_DB && ch + nw < nch) load((ch + nw) * kChunkW);
     const PartDesc dsc = a.desc[ch];
     Seg s{0, 0, 0, 0u, 0};
     seg_from(s, dsc.start, dsc.end, dsc.k, dsc.f, A, min(wbase + lane, total - 1), a.nodes, K);
@@ -1780,7 +1688,6 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     int pr = prof_begin(PK_SCAN, s, 5);
     scan_desc_kernel<<<num_sms() * 4, 256, 0, s>>>(b.nodes[parity], ctl, parity, dl, kChunkW, b.sdesc);
     ScanArgs sa;
-    sa.chunk = nullptr;
     sa.desc = b.sdesc;
     sa.lx = b.lx[cur];
     sa.ly = b.ly[cur];
@@ -1884,7 +1791,6 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     pa.dec = b.dec;
     pa.new_start = b.new_start;
     pa.goleft = b.goleft;
-    pa.chunk = nullptr;
     pa.desc = b.pdesc;
     pa.ctl = ctl;
     pa.parity = parity;

@@ -1,13 +1,12 @@
-// Segmented block-scan and decoupled look-back primitives used by the fit kernels.
+// Segmented warp- and block-scan primitives used by the fit kernels.
 //
 // A "segment" is one (node, feature) run of a level's sorted feature list.  Every scan
 // payload carries a head flag; combine(a, b) resets at b's head:
 //   combine(a, b) = b.flag ? b : a (+) b,   flag = a.flag | b.flag.
-// All block scans have a fixed shape (Kogge-Stone within a warp, then across warps), so
-// results are bit-reproducible for a given blockDim.  The look-back folds predecessor
-// tiles strictly left to right from the nearest tile that holds a final value, which
-// makes the carried prefix identical to the sequential tile-by-tile definition whatever
-// the timing (deterministic fp64 prefixes).
+// All scans have a fixed shape (Kogge-Stone within a warp, then across warps / blocks in
+// index order), so fp64 results are bit-reproducible run to run.  Chunk carries come
+// from fixed-shape chunk/block scans (fit.cu, phase B) rather than a decoupled
+// look-back, which measured slower in every variant tried.
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -172,97 +171,8 @@ __device__ __forceinline__ T block_exclusive_scan(T v, const T& ident, T& agg, T
   return res;
 }
 
-// ------------------------------------------------------------------ look-back ------
-//
-// Each tile publishes two 64-bit words with single-copy-atomic relaxed 64-bit stores:
-// agg[t] = the payload of the tile's own segmented aggregate, inc[t] = the payload of its
-// inclusive prefix.  Both arrays are filled with kUnpublished (all ones: never the bits
-// of a finite f64 sum nor of a u32 count) before every launch.  No flags are needed:
-// a tile whose first element is not a segment head looks back exactly to the tile that
-// holds the head of that segment (`stop_tile`), and every tile in between lies inside
-// the segment.
-
-constexpr uint64_t kUnpublished = ~0ull;
-
-// Morally-strong relaxed accesses: single-copy atomic 64-bit words (weak .cg accesses
-// carry no such guarantee and were observed torn), no fence, no L1 invalidation.
-__device__ __forceinline__ void st_cg_u64(uint64_t* p, uint64_t v) {
-  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ uint64_t ld_cg_u64(const uint64_t* p) {
-  uint64_t v;
-  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-
-__device__ __forceinline__ uint64_t payload_bits(const SumP& v) { return (uint64_t)__double_as_longlong(v.s); }
-__device__ __forceinline__ uint64_t payload_bits(const CntP& v) { return (uint64_t)v.c; }
+// payload <-> 64-bit word helpers (identity element construction in the chunk scans)
 __device__ __forceinline__ void from_bits(SumP& v, uint64_t b) { v.s = __longlong_as_double((long long)b); }
 __device__ __forceinline__ void from_bits(CntP& v, uint64_t b) { v.c = (uint32_t)b; }
-// unflagged fold of two payloads (no segment head between them)
-__device__ __forceinline__ SumP fold(const SumP& a, const SumP& b) { return SumP{0u, __dadd_rn(a.s, b.s)}; }
-__device__ __forceinline__ CntP fold(const CntP& a, const CntP& b) { return CntP{0u, a.c + b.c}; }
-
-template <class T>
-__device__ __forceinline__ void publish(uint64_t* slot, const T& v) {
-  st_cg_u64(slot, payload_bits(v));
-}
-
-constexpr int kLookbackMax = 256;  // predecessor values buffered per look-back (smem)
-
-// Called by ONE WARP (all 32 lanes).  Returns (on lane 0, flag 0) the exclusive carry of
-// `tile`: the strict left-to-right fold of the payloads of tiles stop..tile-1, starting
-// from the nearest one that holds a final value (its inclusive prefix, or stop_tile's
-// aggregate).  32 predecessors are polled per step; values are buffered in `buf` and
-// folded in tile order by lane 0, so the result does not depend on timing.
-template <class T>
-__device__ T warp_lookback(const uint64_t* agg, const uint64_t* inc, int64_t tile,
-                           int64_t stop_tile, T* buf) {
-  const int lane = threadIdx.x & 31;
-  for (;;) {
-    int64_t base = tile - 1;
-    int nbuf = 0, stop = -1;
-    while (nbuf + 32 <= kLookbackMax) {
-      const int64_t t = base - lane;
-      bool fin = true;
-      T val;
-      val.flag = 0u;
-      from_bits(val, 0ull);
-      if (t >= stop_tile) {
-        uint64_t av;
-        while ((av = ld_cg_u64(agg + t)) == kUnpublished) {}
-        const uint64_t iv = ld_cg_u64(inc + t);
-        fin = (iv != kUnpublished) || (t == stop_tile);
-        from_bits(val, (iv != kUnpublished) ? iv : av);
-      }
-      const unsigned m = __ballot_sync(0xffffffffu, fin);
-      const int first = m ? (__ffs(m) - 1) : 31;
-      if (lane <= first) buf[nbuf + lane] = val;
-      nbuf += first + 1;
-      if (m) { stop = nbuf - 1; break; }
-      base -= 32;
-    }
-    __syncwarp();
-    if (stop >= 0) {
-      T acc = buf[stop];
-      if (lane == 0)
-        for (int j = stop - 1; j >= 0; --j) acc = fold(acc, buf[j]);
-      __syncwarp();
-      acc.flag = 0u;
-      return acc;
-    }
-    __nanosleep(500);  // chain longer than the buffer: wait for predecessors, retry
-  }
-}
-
-// ------------------------------------------------------------------ cp.async ------
-
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
-  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(sa), "l"(gmem), "r"(src_bytes)
-               : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 
 }  // namespace dtl
