@@ -17,7 +17,8 @@ import sys
 
 # kernel name -> library profiling kind (dt_profile_* kinds, csrc/prof.cu)
 KIND = {
-    "chunk_node_kernel": "scan", "scan_agg_kernel": "scan", "scan_kernel": "scan",
+    "scan_desc_kernel": "scan", "scan_agg_kernel": "scan", "scan_kernel": "scan",
+    "part_desc_kernel": "partition", "decide_kernel": "select",
     "chunk_scan_kernel<SumP>": "scan", "block_carry_kernel<SumP>": "scan",
     "part_agg_kernel": "partition", "partition_kernel": "partition",
     "chunk_scan_kernel<CntP>": "partition", "block_carry_kernel<CntP>": "partition",
@@ -59,17 +60,21 @@ def main():
         a[0] += 1
         a[1] += v.get("gpu__time_duration.sum", 0.0)
         a[2] += v.get("dram__bytes_read.sum", 0.0) + v.get("dram__bytes_write.sum", 0.0)
+    nfit = max(1, agg.get("root_init_kernel", [1])[0])  # one root_init launch per fit
+    for k in agg:
+        agg[k] = [agg[k][0] / nfit, agg[k][1] / nfit, agg[k][2] / nfit]
     tot = sum(a[1] for a in agg.values())
-    lines = [f"# ncu launch list: `{os.path.basename(src)}`", "",
+    lines = [f"# ncu launch list: `{os.path.basename(src)}` (per fit; {nfit} fits captured)", "",
              "Cold-cache, serialised per-launch times (ncu `--clock-control none`); the bench's",
              "live CUDA-event times are the reference for absolutes. Share = fraction of the",
-             "summed kernel time.", "",
+             "summed kernel time.  ncu serialises the per-feature CUB sorts that the library",
+             "runs concurrently on side streams, so `cub_radix_sort` is overstated here.", "",
              "| kernel | launches | time (us) | share | DRAM (MB) | GB/s |",
              "|---|---:|---:|---:|---:|---:|"]
     for n, (c, t, b) in sorted(agg.items(), key=lambda kv: -kv[1][1]):
-        lines.append(f"| {n} | {c} | {t / 1e3:.1f} | {t / tot:.3f} | {b / 1e6:.1f} | "
+        lines.append(f"| {n} | {c:g} | {t / 1e3:.1f} | {t / tot:.3f} | {b / 1e6:.1f} | "
                      f"{(b / t if t else 0):.0f} |")
-    lines.append(f"| **total** | {sum(a[0] for a in agg.values())} | {tot / 1e3:.1f} | 1.000 | | |")
+    lines.append(f"| **total** | {sum(a[0] for a in agg.values()):g} | {tot / 1e3:.1f} | 1.000 | | |")
     with open(out + ".md", "w") as fh:
         fh.write("\n".join(lines) + "\n")
     # traffic per launch of each profiling kind (a kind's launch = one library region)
