@@ -87,11 +87,11 @@ struct LocalGroup {
   }
 };
 
-__global__ void max_u8_kernel(const uint8_t* const* __restrict__ src, int nsrc, uint8_t* __restrict__ dst,
+__global__ void or_u32_kernel(const uint32_t* const* __restrict__ src, int nsrc, uint32_t* __restrict__ dst,
                               int64_t n) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    uint8_t m = 0;
-    for (int r = 0; r < nsrc; ++r) m = max(m, src[r][i]);
+    uint32_t m = 0;
+    for (int r = 0; r < nsrc; ++r) m |= src[r][i];
     dst[i] = m;
   }
 }
@@ -103,7 +103,7 @@ struct CommImpl {
   int backend = 0;  // 0 = NCCL, 1 = local
   ncclComm_t nccl = nullptr;
   std::shared_ptr<LocalGroup> group;
-  uint8_t** dev_ptrs = nullptr;  // local backend: device array of peer pointers
+  uint32_t** dev_ptrs = nullptr;  // local backend: device array of peer pointers
 };
 
 }  // namespace dtl
@@ -141,30 +141,32 @@ dt_status comm_allgather(dt_comm* c, const void* send, void* recv, size_t bytes,
   return DT_OK;
 }
 
-// buf[i] = max over ranks of buf[i] (u8), in place.
-dt_status comm_allreduce_max_u8(dt_comm* c, uint8_t* buf, int64_t n, cudaStream_t s) {
+// buf[i] = OR over ranks of buf[i], in place, for bitmaps whose set bits are disjoint
+// across ranks (each row's go-left bit is set by exactly one rank): NCCL sums the words,
+// which equals the OR when no two ranks set the same bit.
+dt_status comm_allreduce_or_u32(dt_comm* c, uint32_t* buf, int64_t n, cudaStream_t s) {
   CommImpl& m = c->impl;
   if (m.world == 1) return DT_OK;
   if (m.backend == 0) {
-    ncclResult_t r = g_nccl.AllReduce(buf, buf, (size_t)n, ncclUint8, ncclMax, m.nccl, s);
+    ncclResult_t r = g_nccl.AllReduce(buf, buf, (size_t)n, ncclUint32, ncclSum, m.nccl, s);
     if (r != ncclSuccess) return nccl_fail(r, "ncclAllReduce");
     return DT_OK;
   }
   LocalGroup& g = *m.group;
-  // every rank computes the max of all ranks' (unchanged) inputs into a private copy
-  uint8_t* tmp = nullptr;
-  DT_CK(cudaMallocAsync((void**)&tmp, (size_t)n, s));
+  // every rank computes the OR of all ranks' (unchanged) inputs into a private copy
+  uint32_t* tmp = nullptr;
+  DT_CK(cudaMallocAsync((void**)&tmp, sizeof(uint32_t) * (size_t)n, s));
   DT_CK(cudaStreamSynchronize(s));
   g.send[(size_t)m.rank] = buf;
   g.barrier();
-  std::vector<uint8_t*> ptrs((size_t)m.world);
-  for (int r = 0; r < m.world; ++r) ptrs[(size_t)r] = (uint8_t*)g.send[(size_t)r];
-  DT_CK(cudaMemcpyAsync(m.dev_ptrs, ptrs.data(), sizeof(uint8_t*) * ptrs.size(), cudaMemcpyHostToDevice, s));
-  max_u8_kernel<<<num_sms() * 4, 256, 0, s>>>(m.dev_ptrs, m.world, tmp, n);
+  std::vector<uint32_t*> ptrs((size_t)m.world);
+  for (int r = 0; r < m.world; ++r) ptrs[(size_t)r] = (uint32_t*)g.send[(size_t)r];
+  DT_CK(cudaMemcpyAsync(m.dev_ptrs, ptrs.data(), sizeof(uint32_t*) * ptrs.size(), cudaMemcpyHostToDevice, s));
+  or_u32_kernel<<<num_sms() * 4, 256, 0, s>>>(m.dev_ptrs, m.world, tmp, n);
   DT_CK(cudaGetLastError());
   DT_CK(cudaStreamSynchronize(s));
   g.barrier();  // everybody has read every input
-  DT_CK(cudaMemcpyAsync(buf, tmp, (size_t)n, cudaMemcpyDeviceToDevice, s));
+  DT_CK(cudaMemcpyAsync(buf, tmp, sizeof(uint32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
   DT_CK(cudaFreeAsync(tmp, s));
   DT_CK(cudaStreamSynchronize(s));
   return DT_OK;
@@ -217,7 +219,7 @@ dt_status dt_comm_init_local(int32_t world, dt_comm** comms_out) {
     c->impl.world = world;
     c->impl.backend = 1;
     c->impl.group = g;
-    cudaError_t e = cudaMalloc((void**)&c->impl.dev_ptrs, sizeof(uint8_t*) * (size_t)world);
+    cudaError_t e = cudaMalloc((void**)&c->impl.dev_ptrs, sizeof(uint32_t*) * (size_t)world);
     if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc", __FILE__, __LINE__);
     comms_out[r] = c;
   }

@@ -47,7 +47,7 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
 int comm_rank(const dt_comm* c);
 int comm_world(const dt_comm* c);
 dt_status comm_allgather(dt_comm* c, const void* send, void* recv, size_t bytes, cudaStream_t s);
-dt_status comm_allreduce_max_u8(dt_comm* c, uint8_t* buf, int64_t n, cudaStream_t s);
+dt_status comm_allreduce_or_u32(dt_comm* c, uint32_t* buf, int64_t n, cudaStream_t s);
 // Predict / eval (predict.cu).
 dt_status predict_impl(const dt_tree* t, const float* X, int64_t n, int32_t d, double* yhat,
                        cudaStream_t s);

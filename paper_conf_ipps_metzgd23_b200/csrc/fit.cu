@@ -10,7 +10,7 @@
 //                              per-node SSE / min / max from the feature-0 list;
 //                    select    per node: combine pieces, leaf rules, best feature;
 //                    number    BFS numbering of the children, child statistics, offsets;
-//                    goleft    byte per row: 1 if the row goes to the left child;
+//                    goleft    bit per row: 1 if the row goes to the left child;
 //                    partition stable partition of every feature list into the children
 //                              (sorted order preserved, rows of leaves dropped).
 // No host synchronisation inside the level loop (counts live on the device); kernels
@@ -544,6 +544,21 @@ __global__ void __launch_bounds__(kThreads) scan_agg_kernel(ScanArgs a) {
       if (ch + nw < nch && q0 < total) load_y(a.ly, q0, total, yn);
     }
     const ChunkDesc dsc = a.desc[ch];
+    if (dsc.start <= ch * kChunkW && dsc.end >= ch * kChunkW + kChunkW) {
+      // whole chunk in one segment: the general path's sums without the segment logic
+      const bool head = dsc.start == ch * kChunkW;
+      const double c = dsc.c;
+      double t = (head && lane == 0) ? __dsub_rn(yv[0], c) : __dadd_rn(0.0, __dsub_rn(yv[0], c));
+#pragma unroll
+      for (int j = 1; j < kItems; ++j) t = __dadd_rn(t, __dsub_rn(yv[j], c));
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const double o = __shfl_up_sync(0xffffffffu, t, d);
+        if (lane >= d) t = __dadd_rn(o, t);
+      }
+      if (lane == 31) a.chunk_agg[ch] = SumP{head ? 1u : 0u, t};
+      continue;
+    }
     Seg sg{0, 0, 0, 0u, 0};
     if (any) seg_from(sg, dsc.start, dsc.end, dsc.k, dsc.f, A, p0, a.nodes, K);
     const bool one_seg = any && (p0 + kItems <= total) && (sg.end >= p0 + kItems);
@@ -625,6 +640,109 @@ __global__ void __launch_bounds__(1024) block_carry_kernel(const Ctl* ctl, int p
   }
 }
 
+// Whole warp chunk inside ONE segment (a head can only sit at the chunk's first entry) --
+// true for nearly every chunk at shallow levels.  Same sums in the same order as the
+// general path (thread sums item by item, Kogge-Stone prefix, carry), so the results are
+// bitwise identical; the per-chunk argmax is a warp max-reduction + lowest winning lane
+// (exact selection, ties to the lowest position like ArgP's combine).
+__device__ __forceinline__ void scan_single(const ScanArgs& a, int64_t ch, int64_t cbase, const ChunkDesc& dsc,
+                                            const float* xv, const double* yv, uint32_t m) {
+  const int lane = threadIdx.x & 31;
+  const bool head = dsc.start == cbase;
+  const bool head0 = head && lane == 0;
+  const double c = dsc.c;
+  double t = head0 ? __dsub_rn(yv[0], c) : __dadd_rn(0.0, __dsub_rn(yv[0], c));
+#pragma unroll
+  for (int j = 1; j < kItems; ++j) t = __dadd_rn(t, __dsub_rn(yv[j], c));
+  double inc = t;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const double o = __shfl_up_sync(0xffffffffu, inc, d);
+    if (lane >= d) inc = __dadd_rn(o, inc);
+  }
+  double S = __shfl_up_sync(0xffffffffu, inc, 1);
+  if (lane == 0) S = 0.0;
+  if (!head) S = __dadd_rn(combine(a.block_carry[ch / kBlockChunks], a.chunk_excl[ch]).s, S);
+
+  ArgP run{0u, 0xffffffffu, -1.0, 0.0};
+  if (dsc.srch) {
+    const double sc = dsc.sc;
+    const uint32_t N = dsc.N;
+    const uint32_t i0 = (uint32_t)(cbase + lane * kItems - dsc.start);
+    const uint32_t ilo = m > 1u ? m : 1u, ihi = N - m;
+    float xprev = __shfl_up_sync(0xffffffffu, xv[kItems - 1], 1);
+    if (lane == 0) xprev = head ? 0.f : a.lx[cbase - 1];
+    double Sj = S, bapx = -1.0, bS = 0.0;
+    int bj = -1;
+    bool amb = false;
+    constexpr double kTol = 1e-13;  // >> |approx - exact| / exact (~3e-16)
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+      const uint32_t i = i0 + j;
+      const float xp = (j == 0) ? xprev : xv[j - 1];
+      if (i >= ilo && i <= ihi && xp < xv[j]) {
+        const double g = split_gain_approx(Sj, sc, i, N);
+        if (g > bapx) {
+          if (bapx >= __dmul_rn(g, 1.0 - kTol)) amb = true;
+          bapx = g; bS = Sj; bj = j;
+        } else if (g >= __dmul_rn(bapx, 1.0 - kTol)) {
+          amb = true;
+        }
+      }
+      Sj = __dadd_rn(Sj, __dsub_rn(yv[j], c));
+    }
+    if (bj >= 0 && !amb) {
+      const uint32_t i = i0 + (uint32_t)bj;
+      run.gain = split_gain(bS, sc, i, N);
+      run.i = i;
+      run.sl = bS;
+    } else if (bj >= 0) {
+      Sj = S;
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        const uint32_t i = i0 + j;
+        const float xp = (j == 0) ? xprev : xv[j - 1];
+        if (i >= ilo && i <= ihi && xp < xv[j]) {
+          const double g = split_gain(Sj, sc, i, N);
+          if (g > run.gain) { run.gain = g; run.i = i; run.sl = Sj; }
+        }
+        Sj = __dadd_rn(Sj, __dsub_rn(yv[j], c));
+      }
+    }
+  }
+  double g = run.gain;
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) g = fmax(g, __shfl_xor_sync(0xffffffffu, g, off));
+  const uint32_t win = __ballot_sync(0xffffffffu, run.gain == g);
+  const int src = win ? __ffs(win) - 1 : 0;
+  const uint32_t bi = __shfl_sync(0xffffffffu, run.i, src);
+  const double bsl = __shfl_sync(0xffffffffu, run.sl, src);
+  const uint32_t kf = dsc.k * a.d + dsc.f;
+  const double bg = __shfl_sync(0xffffffffu, run.gain, src);
+  if (lane == 0) write_cand(head ? a.head_cand + kf : a.cont_cand + ch, ArgP{0u, bi, bg, bsl}, kf, a.level,
+                            a.slot_gain);
+  // node statistics from the feature-0 list (same scan as the general path)
+  if (dsc.f == 0) {
+    const double v = dsc.v;
+    StatP srun{head0 ? 1u : 0u, 0.0, INFINITY, -INFINITY, 0.0};
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+      const double ev = __dsub_rn(yv[j], v);
+      srun.sse = __dadd_rn(srun.sse, __dmul_rn(ev, ev));
+      srun.ymin = fmin(srun.ymin, yv[j]);
+      srun.ymax = fmax(srun.ymax, yv[j]);
+      srun.s1 = __dadd_rn(srun.s1, __dsub_rn(yv[j], c));
+    }
+    StatP st_w;
+    const StatP sex = warp_exclusive_scan(srun, StatP{0u, 0.0, INFINITY, -INFINITY, 0.0}, st_w);
+    if (lane == 31) {
+      StatP ts = srun;
+      ts.flag = 0u;
+      write_stat(head ? a.head_stat + dsc.k : a.cont_stat + ch, combine(sex, ts));
+    }
+  }
+}
+
 // Phase C: the main scan (prefixes, gains, per-piece argmax, node statistics), one warp
 // chunk at a time per warp, no block barriers.
 __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
@@ -666,6 +784,10 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
       if (ch + nw < nch && q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
     }
     const ChunkDesc dsc = a.desc[ch];
+    if (dsc.start <= ch * kChunkW && dsc.end >= ch * kChunkW + kChunkW) {
+      scan_single(a, ch, ch * kChunkW, dsc, xv, yv, m);
+      continue;
+    }
     Seg sg{0, 0, 0, 0u, 0};
     if (any) seg_from(sg, dsc.start, dsc.end, dsc.k, dsc.f, A, p0, a.nodes, K);
     // Warp-uniform fast path: every lane's kItems entries lie in ONE segment (a head may
@@ -1204,10 +1326,12 @@ __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
 
 // ----------------------------------------------------------------------------- goleft --
 
-// goleft[row] = 1 iff the row goes to the left child (rows of split nodes only).
+// Go-left bitmap: bit r of gbits is set iff row r goes to the left child (rows of split
+// nodes only; zeroed before every level).  Only the first nl positions of a split node
+// in its split feature's list go left, so only those row ids are read.
 __global__ void __launch_bounds__(256) goleft_kernel(const uint32_t* __restrict__ lr, const NodeL* nodes,
                                                      const Decision* dec, const Ctl* ctl, int parity,
-                                                     uint8_t* __restrict__ goleft) {
+                                                     uint32_t* __restrict__ gbits) {
   const uint32_t K = ctl->K[parity];
   const uint64_t A = ctl->A[parity];
   if (K == 0) return;
@@ -1220,9 +1344,9 @@ __global__ void __launch_bounds__(256) goleft_kernel(const uint32_t* __restrict_
       const uint32_t q = (uint32_t)q0 + j;
       while (q >= kend) { ++k; kstart = kend; kend = kstart + nodes[k].N; }
       const Decision dc = dec[k];
-      if (dc.floc >= 0) {
+      if (dc.floc >= 0 && q - kstart < dc.nl) {
         const uint32_t r = lr[(int64_t)dc.floc * (int64_t)A + q];
-        goleft[r] = (q - kstart < dc.nl) ? 1 : 0;
+        atomicOr(gbits + (r >> 5), 1u << (r & 31));
       }
     }
   }
@@ -1268,7 +1392,9 @@ struct PartArgs {
   const NodeL* nodes;
   const Decision* dec;
   const uint32_t* new_start;
-  const uint8_t* goleft;
+  const uint32_t* gbits;  // go-left bitmap (global)
+  uint32_t* gmask;        // [nchunks * kRows] go-left ballots per row of 32 entries (phase A -> C)
+  int64_t nwords;         // bitmap words
   const PartDesc* desc;  // per warp chunk
   const Ctl* ctl;
   int parity;
@@ -1291,16 +1417,12 @@ struct PartArgs {
 // chunk scan (phase B, shared with the split scan).  No block barriers, no look-back.
 constexpr int kRows = kChunkW / 32;  // rows of 32 per warp chunk
 
-// Per-row go-left / head / split masks of a lane's kRows entries (cursor s advanced).
-// The go-left bytes are gathered for every row up front (independent loads in flight),
-// then masked by "node split" while walking the segments.
+// Per-row head / split masks of a lane's kRows entries (cursor s advanced); gbits = the
+// raw go-left bits masked by "node split".
 __device__ __forceinline__ void part_flags(const PartArgs& a, uint32_t K, uint64_t A, int64_t wbase,
-                                           int64_t total, Seg& s, const uint32_t* rv, uint32_t& gbits,
+                                           int64_t total, Seg& s, uint32_t graw, uint32_t& gbits,
                                            uint32_t& hbits, uint32_t& sbits, const PartDesc& dsc) {
   const int lane = threadIdx.x & 31;
-  uint32_t graw = 0;
-#pragma unroll
-  for (int r = 0; r < kRows; ++r) graw |= (uint32_t)__ldg(a.goleft + rv[r]) << r;
   hbits = sbits = 0;
 #pragma unroll
   for (int r = 0; r < kRows; ++r) {
@@ -1324,8 +1446,18 @@ __device__ __forceinline__ void load_rows(const uint32_t* __restrict__ lr, int64
   }
 }
 
-// Phase A: per-chunk aggregate of go-left counts (lefts since the chunk's last head).
-__global__ void __launch_bounds__(kThreads) part_agg_kernel(PartArgs a) {
+// Largest go-left bitmap kept in shared memory by part_agg_kernel<true> (rows <= 1.8M).
+constexpr int64_t kMaxSmemBitmapBytes = 227 * 1024;
+constexpr int kAggSmemThreads = 1024;
+
+// Phase A: per-chunk aggregate of go-left counts (lefts since the chunk's last head), and
+// the chunk's raw go-left ballots (one word per row of 32 entries) for phase C, so the
+// partition itself gathers nothing.  kSmem: the whole bitmap is staged in shared memory
+// (one CTA per SM), so the per-entry gathers are shared-memory loads, not L2 round trips.
+template <bool kSmem>
+__global__ void __launch_bounds__(kSmem ? kAggSmemThreads : kThreads) part_agg_kernel(PartArgs a) {
+  extern __shared__ uint4 smem_bits4[];
+  const uint32_t* __restrict__ bits = kSmem ? reinterpret_cast<const uint32_t*>(smem_bits4) : a.gbits;
   const uint32_t K = a.ctl->K[a.parity];
   const uint64_t A = a.ctl->A[a.parity];
   const uint64_t A2 = a.ctl->A[a.parity ^ 1];
@@ -1337,6 +1469,12 @@ __global__ void __launch_bounds__(kThreads) part_agg_kernel(PartArgs a) {
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   uint32_t rn[kRows];
   if (gw < nch) load_rows(a.lr, gw * kChunkW, total, rn);
+  if (kSmem) {
+    const int64_t n4 = (a.nwords + 3) / 4;
+    const uint4* g4 = reinterpret_cast<const uint4*>(a.gbits);
+    for (int64_t i = threadIdx.x; i < n4; i += blockDim.x) smem_bits4[i] = __ldg(g4 + i);
+    __syncthreads();
+  }
   for (int64_t ch = gw; ch < nch; ch += nw) {
     const int64_t wbase = ch * kChunkW;
     uint32_t rv[kRows];
@@ -1344,24 +1482,43 @@ __global__ void __launch_bounds__(kThreads) part_agg_kernel(PartArgs a) {
     for (int r = 0; r < kRows; ++r) rv[r] = rn[r];
     if (ch + nw < nch) load_rows(a.lr, (ch + nw) * kChunkW, total, rn);
     const PartDesc dsc = a.desc[ch];
-    Seg s{0, 0, 0, 0u, 0};
-    seg_from(s, dsc.start, dsc.end, dsc.k, dsc.f, A, min(wbase + lane, total - 1), a.nodes, K);
-    uint32_t gbits, hbits, sbits;
-    part_flags(a, K, A, wbase, total, s, rv, gbits, hbits, sbits, dsc);
-    CntP agg{0u, 0u};
+    uint32_t graw = 0;
 #pragma unroll
-    for (int r = 0; r < kRows; ++r) {
-      const uint32_t gm = __ballot_sync(0xffffffffu, (gbits >> r) & 1u);
-      const uint32_t hm = __ballot_sync(0xffffffffu, (hbits >> r) & 1u);
-      if (hm) {
-        const int hl = 31 - __clz(hm);
-        agg.flag = 1u;
-        agg.c = __popc(gm & ~((1u << hl) - 1u));
-      } else {
-        agg.c += __popc(gm);
+    for (int r = 0; r < kRows; ++r) graw |= ((bits[rv[r] >> 5] >> (rv[r] & 31)) & 1u) << r;
+    uint32_t my_mask = 0;
+    if (dsc.start <= wbase && dsc.end >= wbase + kChunkW) {
+      // whole chunk in one segment (a head can only be its first entry)
+      uint32_t c = 0;
+#pragma unroll
+      for (int r = 0; r < kRows; ++r) {
+        const uint32_t gm = __ballot_sync(0xffffffffu, (graw >> r) & 1u);
+        if (lane == r) my_mask = gm;
+        c += __popc(gm);
       }
+      if (lane == 0) a.chunk_agg[ch] = CntP{dsc.start == wbase ? 1u : 0u, dsc.split ? c : 0u};
+    } else {
+      Seg s{0, 0, 0, 0u, 0};
+      seg_from(s, dsc.start, dsc.end, dsc.k, dsc.f, A, min(wbase + lane, total - 1), a.nodes, K);
+      uint32_t gbits, hbits, sbits;
+      part_flags(a, K, A, wbase, total, s, graw, gbits, hbits, sbits, dsc);
+      CntP agg{0u, 0u};
+#pragma unroll
+      for (int r = 0; r < kRows; ++r) {
+        const uint32_t rm = __ballot_sync(0xffffffffu, (graw >> r) & 1u);
+        if (lane == r) my_mask = rm;
+        const uint32_t gm = __ballot_sync(0xffffffffu, (gbits >> r) & 1u);
+        const uint32_t hm = __ballot_sync(0xffffffffu, (hbits >> r) & 1u);
+        if (hm) {
+          const int hl = 31 - __clz(hm);
+          agg.flag = 1u;
+          agg.c = __popc(gm & ~((1u << hl) - 1u));
+        } else {
+          agg.c += __popc(gm);
+        }
+      }
+      if (lane == 0) a.chunk_agg[ch] = agg;
     }
-    if (lane == 0) a.chunk_agg[ch] = agg;
+    if (lane < kRows) a.gmask[ch * kRows + lane] = my_mask;
   }
 }
 
@@ -1401,11 +1558,39 @@ __global__ void __launch_bounds__(kThreads, 4) partition_kernel(PartArgs a) {
 #pragma unroll
     for (int r = 0; r < kRows; ++r) { rv[r] = rn[r]; xv[r] = xn[r]; yv[r] = yn[r]; }
     const PartDesc dsc = a.desc[ch];
+    // raw go-left bits of my kRows entries, from the chunk's ballots (phase A)
+    const uint32_t mword = (lane < kRows) ? __ldcs(a.gmask + ch * kRows + lane) : 0u;
+    uint32_t graw = 0;
+#pragma unroll
+    for (int r = 0; r < kRows; ++r) graw |= ((__shfl_sync(0xffffffffu, mword, r) >> lane) & 1u) << r;
+    if (dsc.start <= wbase && dsc.end >= wbase + kChunkW) {
+      // whole chunk in one segment: ranks from the go-left ballots and one carry
+      if (!dsc.split) continue;  // rows of leaves are dropped
+      uint32_t carry = (dsc.start == wbase) ? 0u : combine(a.block_carry[ch / kBlockChunks], a.chunk_excl[ch]).c;
+      const uint32_t i0 = (uint32_t)(wbase - dsc.start) + lane;
+      const uint32_t nsl = dsc.ns + dsc.nl;
+      float* const ox = a.ox + (int64_t)dsc.f * (int64_t)A2;
+      uint32_t* const orow = a.orow + (int64_t)dsc.f * (int64_t)A2;
+      double* const oy = a.oy + (int64_t)dsc.f * (int64_t)A2;
+#pragma unroll
+      for (int r = 0; r < kRows; ++r) {
+        const uint32_t g = (graw >> r) & 1u;
+        const uint32_t gm = __ballot_sync(0xffffffffu, g);
+        const uint32_t rank = carry + __popc(gm & lt_mask);
+        const uint32_t i = i0 + r * 32;
+        const uint32_t dst = g ? dsc.ns + rank : nsl + (i - rank);
+        ox[dst] = xv[r];
+        orow[dst] = rv[r];
+        oy[dst] = yv[r];
+        carry += __popc(gm);
+      }
+      continue;
+    }
     Seg s{0, 0, 0, 0u, 0};
     seg_from(s, dsc.start, dsc.end, dsc.k, dsc.f, A, min(wbase + lane, total - 1), a.nodes, K);
     const Seg s0 = s;
     uint32_t gbits, hbits, sbits;
-    part_flags(a, K, A, wbase, total, s, rv, gbits, hbits, sbits, dsc);
+    part_flags(a, K, A, wbase, total, s, graw, gbits, hbits, sbits, dsc);
     const CntP cc = combine(a.block_carry[ch / kBlockChunks], a.chunk_excl[ch]);
     uint32_t carry = cc.c;  // lefts of the open segment before this chunk
     s = s0;
@@ -1497,7 +1682,9 @@ struct FitBufs {
   unsigned long long* slot_gain;
   uint32_t* slot_pos;
   Stat *head_stat, *cont_stat;
-  uint8_t* goleft;
+  uint32_t* gbits;  // go-left bitmap, nwords4 words
+  uint32_t* gmask;  // [max_chunks * kRows]
+  int64_t nwords4;
   dt_node* dout;
   Ctl* ctl;
   LevelLog* lvlog;
@@ -1557,7 +1744,9 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, int wor
   DT_CK(get(&b.cont_cand, (size_t)b.max_chunks));
   DT_CK(get(&b.head_stat, (size_t)b.kcap));
   DT_CK(get(&b.cont_stat, (size_t)b.max_chunks));
-  DT_CK(get(&b.goleft, (size_t)n));
+  b.nwords4 = ((n + 127) / 128) * 4;  // whole uint4s
+  DT_CK(get(&b.gbits, (size_t)b.nwords4));
+  DT_CK(get(&b.gmask, (size_t)b.max_chunks * kRows));
   DT_CK(get(&b.dout, (size_t)b.out_cap));
   DT_CK(get(&b.ctl, 1));
   DT_CK(get(&b.lvlog, (size_t)kMaxLogLevels));
@@ -1674,7 +1863,11 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
   }
   const int g_scan = persistent_grid((const void*)scan_kernel, kThreads, 0);
   const int g_agg = persistent_grid((const void*)scan_agg_kernel, kThreads, 0);
-  const int g_pagg = persistent_grid((const void*)part_agg_kernel, kThreads, 0);
+  const int g_pagg = persistent_grid((const void*)part_agg_kernel<false>, kThreads, 0);
+  size_t agg_smem = sizeof(uint32_t) * (size_t)b.nwords4;
+  if ((int64_t)agg_smem > kMaxSmemBitmapBytes) agg_smem = 0;
+  else DT_CK(cudaFuncSetAttribute((const void*)part_agg_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)agg_smem));
   const int g_part = persistent_grid((const void*)partition_kernel, kThreads, 0);
   const int g_sel = num_sms() * 4;
   const int g_gl = num_sms() * 8;
@@ -1769,11 +1962,11 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     DT_CK(cudaGetLastError());
     // go-left map (a6)
     pr = prof_begin(PK_GOLEFT, s, 1);
-    if (sh.world > 1) DT_CK(cudaMemsetAsync(b.goleft, 0, (size_t)n, s));
-    goleft_kernel<<<g_gl, 256, 0, s>>>(b.lr[cur], b.nodes[parity], b.dec, ctl, parity, b.goleft);
+    DT_CK(cudaMemsetAsync(b.gbits, 0, sizeof(uint32_t) * (size_t)b.nwords4, s));
+    goleft_kernel<<<g_gl, 256, 0, s>>>(b.lr[cur], b.nodes[parity], b.dec, ctl, parity, b.gbits);
     if (sh.world > 1) {
-      // the owner of each split feature wrote its rows' bytes; everyone else wrote 0
-      dt_status cst = comm_allreduce_max_u8(sh.comm, b.goleft, n, s);
+      // only the owner of each split feature set its rows' bits: OR over the ranks
+      dt_status cst = comm_allreduce_or_u32(sh.comm, b.gbits, b.nwords4, s);
       if (cst != DT_OK) return cst;
     }
     prof_end(pr, s, 0.0);
@@ -1790,7 +1983,9 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     pa.nodes = b.nodes[parity];
     pa.dec = b.dec;
     pa.new_start = b.new_start;
-    pa.goleft = b.goleft;
+    pa.gbits = b.gbits;
+    pa.gmask = b.gmask;
+    pa.nwords = b.nwords4;
     pa.desc = b.pdesc;
     pa.ctl = ctl;
     pa.parity = parity;
@@ -1802,7 +1997,8 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     pa.block_carry = b.pblock_carry;
     pr = prof_begin(PK_PARTITION, s, 5);
     part_desc_kernel<<<num_sms() * 4, 256, 0, s>>>(b.nodes[parity], b.dec, b.new_start, ctl, parity, pa.dl_out, b.pdesc);
-    part_agg_kernel<<<g_pagg, kThreads, 0, s>>>(pa);
+    if (agg_smem) part_agg_kernel<true><<<num_sms(), kAggSmemThreads, agg_smem, s>>>(pa);
+    else part_agg_kernel<false><<<g_pagg, kThreads, 0, s>>>(pa);
     chunk_scan_kernel<CntP><<<(unsigned)b.max_cblocks, 1024, 0, s>>>(ctl, parity, pa.dl_out, b.pchunk_agg, b.pchunk_excl, b.pblock_agg);
     block_carry_kernel<CntP><<<1, 1024, 0, s>>>(ctl, parity, pa.dl_out, b.pblock_agg, b.pblock_carry);
     partition_kernel<<<g_part, kThreads, 0, s>>>(pa);
@@ -1850,14 +2046,15 @@ dt_status fit_finish(const FitBufs& b, int32_t d, cudaStream_t s, const std::vec
   if (pending) {
     // algorithmic bytes per launch:
     //   scan: every active entry of the scanned lists, x (4 B) + y (8 B);
-    //   goleft: the split feature's row ids of the moved rows (4 B) + one byte per row;
+    //   goleft: the split feature's row ids of the moved rows (4 B, left rows only read, counted
+    //           for all) + one bit per row;
     //   partition: every moved entry read (16 B) and written (16 B).
     for (const Pending& p : *pending) {
       if (p.rec < 0 || p.level >= kMaxLogLevels) continue;
       const LevelLog& L = hlog[(size_t)p.level];
       double bytes = 0.0;
       if (p.kind == PK_SCAN) bytes = 12.0 * (double)L.A * p.dl;
-      else if (p.kind == PK_GOLEFT) bytes = 5.0 * (double)L.A_next;
+      else if (p.kind == PK_GOLEFT) bytes = 4.125 * (double)L.A_next;
       else if (p.kind == PK_PARTITION) bytes = 32.0 * (double)L.A_next * p.dl;
       prof_set_bytes(p.rec, bytes);
     }
@@ -1994,7 +2191,7 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
 
 // Feature-sharded fit: every rank holds the full table and builds /
 // scans the feature lists j * world + rank; per level the ranks exchange their per-node
-// best splits (allgather) and the go-left bytes (max-allreduce).  Same tree on every rank.
+// best splits (allgather) and the go-left bitmap (OR-allreduce).  Same tree on every rank.
 dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64_t n, int32_t dg,
                            int32_t max_depth, int64_t min_leaf, cudaStream_t s, dt_tree** out) {
   const int world = comm_world(comm), rank = comm_rank(comm);
