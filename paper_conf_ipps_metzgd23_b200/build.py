@@ -9,7 +9,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
-LIB = os.path.join(HERE, "libdt.so")
+LIB = os.environ.get("DT_BUILD_OUT", os.path.join(HERE, "libdt.so"))  # override: experiments
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 FLAGS = [
@@ -19,7 +19,7 @@ FLAGS = [
     "-Xcompiler", "-fPIC", "-Xcompiler", "-O2",
     "-cudart", "static",
     "-I", os.path.join(ROOT, "include"),
-]
+] + os.environ.get("DT_EXTRA_NVCC", "").split()  # experiments (e.g. -DDT_GAIN_BATCH=8)
 # nccl.h for the communicator types (libnccl.so.2 itself is dlopen'ed at run time)
 for _inc in ("/usr/include", os.path.join(os.path.dirname(os.__file__), "site-packages", "nvidia", "nccl", "include")):
     if os.path.exists(os.path.join(_inc, "nccl.h")):
@@ -43,7 +43,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
     objs = []
-    bdir = os.path.join(HERE, "build")
+    bdir = os.path.join(HERE, "build" + os.environ.get("DT_BUILD_TAG", ""))
     os.makedirs(bdir, exist_ok=True)
     procs = []
     for src in sources():

@@ -26,6 +26,7 @@
 #include <vector>
 
 #include "dt_internal.cuh"
+#include "bulk.cuh"
 #include "scan_primitives.cuh"
 
 namespace dtl {
@@ -77,6 +78,9 @@ struct Ctl {
   double ysum, ymin, ymax, ysc;
   int32_t all_integral;
   int32_t pad;
+  // chunk lists of the level (single-segment chunks from the front, others from the back)
+  uint32_t scnt[2];  // scan: singles, others
+  uint32_t pcnt[2];  // partition: singles, others
 };
 
 struct LevelLog {  // per-level counts, for algorithmic-byte accounting (profiling)
@@ -100,7 +104,7 @@ struct Stat {
 
 // Per-level descriptor of the segment holding the FIRST entry of each warp chunk
 // (kChunkW entries): one independent load per chunk instead of a dependent lookup chain.
-struct ChunkDesc {
+struct __align__(64) ChunkDesc {  // 64 B: one bulk copy
   int64_t start, end;  // global list positions of the segment
   uint32_t k;
   int32_t f;
@@ -108,6 +112,7 @@ struct ChunkDesc {
   uint32_t N;
   int32_t srch;
 };
+static_assert(sizeof(ChunkDesc) == 64, "ChunkDesc is copied with one 64-byte bulk copy");
 struct PartDesc {
   int64_t start, end;
   uint32_t k;
@@ -307,10 +312,32 @@ __global__ void __launch_bounds__(256) presort_build_kernel(const uint32_t* __re
 
 // ----------------------------------------------------------------------------- scan ----
 
-__global__ void __launch_bounds__(256) scan_desc_kernel(const NodeL* __restrict__ nodes, const Ctl* ctl,
-                                                        int parity, int dl, int chunkw, ChunkDesc* __restrict__ desc) {
+// Appends chunk c to a level's chunk list: single-segment chunks from the front, the
+// others from the back (warp-aggregated atomics; the order inside a list is irrelevant,
+// every chunk's results are independent of when it is processed).
+__device__ __forceinline__ void list_chunk(uint32_t* cnt, uint32_t* list, int64_t nch, int64_t c, bool single) {
+  const unsigned am = __activemask();
+  const int lane = threadIdx.x & 31;
+  const unsigned ms = __ballot_sync(am, single);
+  const int leader = __ffs(am) - 1;
+  uint32_t bs = 0, bg = 0;
+  if (lane == leader) {
+    bs = atomicAdd(cnt, (uint32_t)__popc(ms));
+    bg = atomicAdd(cnt + 1, (uint32_t)__popc(am & ~ms));
+  }
+  bs = __shfl_sync(am, bs, leader);
+  bg = __shfl_sync(am, bg, leader);
+  const unsigned lt = (1u << lane) - 1u;
+  if (single) list[bs + __popc(ms & lt)] = (uint32_t)c;
+  else list[nch - 1 - (bg + __popc(am & ~ms & lt))] = (uint32_t)c;
+}
+
+__global__ void __launch_bounds__(256) scan_desc_kernel(const NodeL* __restrict__ nodes, Ctl* ctl,
+                                                        int parity, int dl, int chunkw, ChunkDesc* __restrict__ desc,
+                                                        uint32_t* __restrict__ list) {
   const uint32_t K = ctl->K[parity];
   const uint64_t A = ctl->A[parity];
+  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->pcnt[0] = ctl->pcnt[1] = 0;  // this level's partition lists
   if (K == 0 || A == 0) return;
   const int64_t total = (int64_t)A * dl;
   const int64_t nch = (total + chunkw - 1) / chunkw;
@@ -331,6 +358,7 @@ __global__ void __launch_bounds__(256) scan_desc_kernel(const NodeL* __restrict_
     d.N = nd.N;
     d.srch = nd.searchable;
     desc[c] = d;
+    list_chunk(ctl->scnt, list, nch, c, d.start <= p && d.end >= p + chunkw);
   }
 }
 
@@ -375,6 +403,7 @@ struct ScanArgs {
   int64_t min_leaf;
   uint32_t* counter;  // tile counter (zeroed per launch)
   const ChunkDesc* desc;  // per warp chunk
+  const uint32_t* list;   // chunk list (scan_desc_kernel): singles first, others from the back
   SumP* chunk_agg;    // [nchunks] phase A: per-warp-chunk aggregate
   SumP* chunk_excl;   // [nchunks] phase B1: exclusive within its block of chunks
   SumP* block_agg;    // [nblocks] phase B1: block aggregates
@@ -646,7 +675,8 @@ __global__ void __launch_bounds__(1024) block_carry_kernel(const Ctl* ctl, int p
 // bitwise identical; the per-chunk argmax is a warp max-reduction + lowest winning lane
 // (exact selection, ties to the lowest position like ArgP's combine).
 __device__ __forceinline__ void scan_single(const ScanArgs& a, int64_t ch, int64_t cbase, const ChunkDesc& dsc,
-                                            const float* xv, const double* yv, uint32_t m) {
+                                            const float* xv, const double* yv, uint32_t m, const SumP& carry,
+                                            float xp0) {
   const int lane = threadIdx.x & 31;
   const bool head = dsc.start == cbase;
   const bool head0 = head && lane == 0;
@@ -662,7 +692,7 @@ __device__ __forceinline__ void scan_single(const ScanArgs& a, int64_t ch, int64
   }
   double S = __shfl_up_sync(0xffffffffu, inc, 1);
   if (lane == 0) S = 0.0;
-  if (!head) S = __dadd_rn(combine(a.block_carry[ch / kBlockChunks], a.chunk_excl[ch]).s, S);
+  if (!head) S = __dadd_rn(carry.s, S);
 
   ArgP run{0u, 0xffffffffu, -1.0, 0.0};
   if (dsc.srch) {
@@ -671,42 +701,65 @@ __device__ __forceinline__ void scan_single(const ScanArgs& a, int64_t ch, int64
     const uint32_t i0 = (uint32_t)(cbase + lane * kItems - dsc.start);
     const uint32_t ilo = m > 1u ? m : 1u, ihi = N - m;
     float xprev = __shfl_up_sync(0xffffffffu, xv[kItems - 1], 1);
-    if (lane == 0) xprev = head ? 0.f : a.lx[cbase - 1];
-    double Sj = S, bapx = -1.0, bS = 0.0;
-    int bj = -1;
-    bool amb = false;
-    constexpr double kTol = 1e-13;  // >> |approx - exact| / exact (~3e-16)
+    if (lane == 0) xprev = head ? 0.f : xp0;
+    // Argmax without divisions: candidate j's gain is n_j / d_j with n_j = D_j^2 and
+    // d_j = (N n_L) n_R exactly as in split_gain, so g_a < g_b <=> n_a d_b < n_b d_a up to
+    // two roundings (relative 2.2e-16).  A fixed 8 -> 4 -> 2 -> 1 tournament (earlier item
+    // wins unless the later is strictly larger) finds the argmax; a comparison whose two
+    // sides are within kTol flags a near-tie on the winner's path, and then every valid
+    // item's exact gain decides (strict >, in order).  Otherwise only the winner's exact
+    // gain is computed.  Exactly the argmax and gain of the plain per-item loop.
+    constexpr double kTol = 1e-13;  // >> 2 roundings
+    const double Nd = (double)N;
+    double tn[kItems], td[kItems], ts[kItems];
+    int tj[kItems];
+    bool tamb[kItems];
+    double Sj = S;
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
       const uint32_t i = i0 + j;
       const float xp = (j == 0) ? xprev : xv[j - 1];
-      if (i >= ilo && i <= ihi && xp < xv[j]) {
-        const double g = split_gain_approx(Sj, sc, i, N);
-        if (g > bapx) {
-          if (bapx >= __dmul_rn(g, 1.0 - kTol)) amb = true;
-          bapx = g; bS = Sj; bj = j;
-        } else if (g >= __dmul_rn(bapx, 1.0 - kTol)) {
-          amb = true;
-        }
-      }
+      const bool ok = i >= ilo && i <= ihi && xp < xv[j];
+      const double nl = (double)i, nr = __dsub_rn(Nd, nl);
+      const double sr = __dsub_rn(sc, Sj);
+      const double D = __dsub_rn(__dmul_rn(Sj, nr), __dmul_rn(sr, nl));
+      tn[j] = ok ? __dmul_rn(D, D) : -1.0;
+      td[j] = ok ? __dmul_rn(__dmul_rn(Nd, nl), nr) : 1.0;
+      ts[j] = Sj;
+      tj[j] = j;
+      tamb[j] = false;
       Sj = __dadd_rn(Sj, __dsub_rn(yv[j], c));
     }
-    if (bj >= 0 && !amb) {
-      const uint32_t i = i0 + (uint32_t)bj;
-      run.gain = split_gain(bS, sc, i, N);
-      run.i = i;
-      run.sl = bS;
-    } else if (bj >= 0) {
-      Sj = S;
 #pragma unroll
-      for (int j = 0; j < kItems; ++j) {
-        const uint32_t i = i0 + j;
-        const float xp = (j == 0) ? xprev : xv[j - 1];
-        if (i >= ilo && i <= ihi && xp < xv[j]) {
-          const double g = split_gain(Sj, sc, i, N);
-          if (g > run.gain) { run.gain = g; run.i = i; run.sl = Sj; }
+    for (int w = 1; w < kItems; w <<= 1) {
+#pragma unroll
+      for (int q = 0; q < kItems; q += 2 * w) {
+        const double L = __dmul_rn(tn[q], td[q + w]), R = __dmul_rn(tn[q + w], td[q]);
+        const bool bw = R > L;  // the later candidate wins only if strictly larger
+        const double hi = bw ? R : L, lo = bw ? L : R;
+        const bool near = lo >= __dmul_rn(hi, 1.0 - kTol);
+        if (bw) { tn[q] = tn[q + w]; td[q] = td[q + w]; ts[q] = ts[q + w]; tj[q] = tj[q + w]; tamb[q] = tamb[q + w]; }
+        tamb[q] = tamb[q] || near;
+      }
+    }
+    if (tn[0] >= 0.0) {
+      if (!tamb[0]) {
+        const uint32_t i = i0 + (uint32_t)tj[0];
+        run.gain = split_gain(ts[0], sc, i, N);
+        run.i = i;
+        run.sl = ts[0];
+      } else {
+        Sj = S;
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+          const uint32_t i = i0 + j;
+          const float xp = (j == 0) ? xprev : xv[j - 1];
+          if (i >= ilo && i <= ihi && xp < xv[j]) {
+            const double g = split_gain(Sj, sc, i, N);
+            if (g > run.gain) { run.gain = g; run.i = i; run.sl = Sj; }
+          }
+          Sj = __dadd_rn(Sj, __dsub_rn(yv[j], c));
         }
-        Sj = __dadd_rn(Sj, __dsub_rn(yv[j], c));
       }
     }
   }
@@ -743,6 +796,91 @@ __device__ __forceinline__ void scan_single(const ScanArgs& a, int64_t ch, int64
   }
 }
 
+// One pipeline stage of scan_single_kernel: everything one chunk needs, brought in by
+// TMA bulk copies (x, y, descriptor, the two carry words, the entry before the chunk).
+constexpr int kScanStages = 3;
+struct __align__(128) ScanStage {
+  float x[kChunkW];
+  double y[kChunkW];
+  ChunkDesc d;
+  SumP cb, ce;   // block carry, chunk-exclusive carry
+  float xp[4];   // x[cbase - 4 .. cbase)
+  uint32_t ch;
+};
+
+// Phase C for the single-segment chunks with a per-warp TMA pipeline: lane 0 keeps
+// kScanStages chunks in flight (bulk copies completing on one mbarrier per stage); the
+// lanes read their items from shared memory, so no registers hold in-flight data.
+__global__ void __launch_bounds__(kThreads, 2) scan_single_kernel(ScanArgs a) {
+  extern __shared__ __align__(128) unsigned char scan_smem[];
+  const uint32_t K = a.ctl->K[a.parity];
+  const uint64_t A = a.ctl->A[a.parity];
+  if (K == 0 || A == 0) return;
+  const int64_t ns = a.ctl->scnt[0];
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  if (gw >= ns) return;  // warp-uniform; no block barriers below
+  const uint32_t m = (uint32_t)min(a.min_leaf, (int64_t)0xffffffff);
+  ScanStage* st = reinterpret_cast<ScanStage*>(scan_smem) + wib * kScanStages;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(scan_smem + sizeof(ScanStage) * kScanStages * (kThreads / 32)) +
+                  wib * kScanStages;
+  auto issue = [&](int s, int64_t ch) {  // lane 0
+    ScanStage& t = st[s];
+    t.ch = (uint32_t)ch;
+    const uint32_t bytes = (uint32_t)(sizeof(t.x) + sizeof(t.y) + sizeof(ChunkDesc) + 2 * sizeof(SumP)) +
+                           (ch > 0 ? 16u : 0u);
+    fence_proxy_async_smem();
+    mbar_arrive_expect_tx(bar + s, bytes);
+    bulk_g2s(t.x, a.lx + ch * kChunkW, sizeof(t.x), bar + s);
+    bulk_g2s(t.y, a.ly + ch * kChunkW, sizeof(t.y), bar + s);
+    bulk_g2s(&t.d, a.desc + ch, sizeof(ChunkDesc), bar + s);
+    bulk_g2s(&t.cb, a.block_carry + ch / kBlockChunks, sizeof(SumP), bar + s);
+    bulk_g2s(&t.ce, a.chunk_excl + ch, sizeof(SumP), bar + s);
+    if (ch > 0) bulk_g2s(t.xp, a.lx + ch * kChunkW - 4, 16, bar + s);
+  };
+  if (lane == 0) {
+    for (int s = 0; s < kScanStages; ++s) mbar_init(bar + s, 1);
+    mbar_init_fence();
+    for (int s = 0; s < kScanStages; ++s)
+      if (gw + s * nw < ns) issue(s, (int64_t)a.list[gw + s * nw]);
+  }
+  __syncwarp();
+  int s = 0;
+  uint32_t phase = 0;
+  for (int64_t idx = gw; idx < ns; idx += nw) {
+    const int64_t nxt = idx + kScanStages * nw;
+    const uint32_t ch_ahead = (lane == 0 && nxt < ns) ? a.list[nxt] : 0u;  // consumed after the chunk
+    mbar_wait(bar + s, phase);
+    const ScanStage& t = st[s];
+    float xv[kItems];
+    double yv[kItems];
+    {
+      const float4* x4 = reinterpret_cast<const float4*>(t.x + lane * kItems);
+      const double2* y2 = reinterpret_cast<const double2*>(t.y + lane * kItems);
+#pragma unroll
+      for (int j = 0; j < kItems / 4; ++j) {
+        const float4 q = x4[j];
+        xv[4 * j] = q.x; xv[4 * j + 1] = q.y; xv[4 * j + 2] = q.z; xv[4 * j + 3] = q.w;
+      }
+#pragma unroll
+      for (int j = 0; j < kItems / 2; ++j) {
+        const double2 q = y2[j];
+        yv[2 * j] = q.x; yv[2 * j + 1] = q.y;
+      }
+    }
+    const ChunkDesc dsc = t.d;
+    const int64_t ch = t.ch;
+    const SumP carry = combine(t.cb, t.ce);
+    const float xp0 = t.xp[3];
+    __syncwarp();  // every lane has read the stage
+    if (lane == 0 && nxt < ns) issue(s, (int64_t)ch_ahead);
+    scan_single(a, ch, ch * kChunkW, dsc, xv, yv, m, carry, xp0);
+    if (++s == kScanStages) { s = 0; phase ^= 1u; }
+  }
+}
+constexpr size_t kScanSingleSmem = (sizeof(ScanStage) + sizeof(uint64_t)) * kScanStages * (kThreads / 32);
+
 // Phase C: the main scan (prefixes, gains, per-piece argmax, node statistics), one warp
 // chunk at a time per warp, no block barriers.
 __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
@@ -765,29 +903,30 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
   const ArgP arg0{0u, 0xffffffffu, -1.0, 0.0};
   const StatP stat0{0u, 0.0, INFINITY, -INFINITY, 0.0};
 
-  // register double buffering: the next chunk's loads are in flight during this chunk
+  // the chunks with a segment boundary inside (list tail); register double buffering:
+  // the next chunk's loads are in flight during this chunk
+  const int64_t ng = a.ctl->scnt[1];
   float xn[kItems];
   double yn[kItems];
+  int64_t ch_next = (gw < ng) ? (int64_t)a.list[nch - 1 - gw] : 0;
   {
-    const int64_t q0 = gw * kChunkW + lane * kItems;
-    if (gw < nch && q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
+    const int64_t q0 = ch_next * kChunkW + lane * kItems;
+    if (gw < ng && q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
   }
-  for (int64_t ch = gw; ch < nch; ch += nw) {
+  for (int64_t idx = gw; idx < ng; idx += nw) {
+    const int64_t ch = ch_next;
     const int64_t p0 = ch * kChunkW + lane * kItems;
     const bool any = p0 < total;
     float xv[kItems];
     double yv[kItems];
 #pragma unroll
     for (int j = 0; j < kItems; ++j) { xv[j] = xn[j]; yv[j] = yn[j]; }
-    {
-      const int64_t q0 = (ch + nw) * kChunkW + lane * kItems;
-      if (ch + nw < nch && q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
+    if (idx + nw < ng) {
+      ch_next = (int64_t)a.list[nch - 1 - (idx + nw)];
+      const int64_t q0 = ch_next * kChunkW + lane * kItems;
+      if (q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
     }
     const ChunkDesc dsc = a.desc[ch];
-    if (dsc.start <= ch * kChunkW && dsc.end >= ch * kChunkW + kChunkW) {
-      scan_single(a, ch, ch * kChunkW, dsc, xv, yv, m);
-      continue;
-    }
     Seg sg{0, 0, 0, 0u, 0};
     if (any) seg_from(sg, dsc.start, dsc.end, dsc.k, dsc.f, A, p0, a.nodes, K);
     // Warp-uniform fast path: every lane's kItems entries lie in ONE segment (a head may
@@ -1356,10 +1495,12 @@ __global__ void __launch_bounds__(256) goleft_kernel(const uint32_t* __restrict_
 
 __global__ void __launch_bounds__(256) part_desc_kernel(const NodeL* __restrict__ nodes,
                                                         const Decision* __restrict__ dec,
-                                                        const uint32_t* __restrict__ new_start, const Ctl* ctl,
-                                                        int parity, int dl, PartDesc* __restrict__ desc) {
+                                                        const uint32_t* __restrict__ new_start, Ctl* ctl,
+                                                        int parity, int dl, PartDesc* __restrict__ desc,
+                                                        uint32_t* __restrict__ list) {
   const uint32_t K = ctl->K[parity];
   const uint64_t A = ctl->A[parity];
+  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->scnt[0] = ctl->scnt[1] = 0;  // next level's scan lists
   if (K == 0 || A == 0 || ctl->A[parity ^ 1] == 0) return;
   const int64_t total = (int64_t)A * dl;
   const int64_t nch = (total + kChunkW - 1) / kChunkW;
@@ -1379,6 +1520,9 @@ __global__ void __launch_bounds__(256) part_desc_kernel(const NodeL* __restrict_
     d.ns = new_start[k];
     d.pad = 0;
     desc[c] = d;
+    // single-segment chunks of leaves have nothing to move: in neither list
+    const bool single = d.start <= p && d.end >= p + kChunkW;
+    if (!single || d.split) list_chunk(ctl->pcnt, list, nch, c, single);
   }
 }
 
@@ -1396,6 +1540,7 @@ struct PartArgs {
   uint32_t* gmask;        // [nchunks * kRows] go-left ballots per row of 32 entries (phase A -> C)
   int64_t nwords;         // bitmap words
   const PartDesc* desc;  // per warp chunk
+  const uint32_t* list;   // chunk list (part_desc_kernel): split singles first, others from the back
   const Ctl* ctl;
   int parity;
   int dl_in;   // lists in the input (d)
@@ -1522,9 +1667,123 @@ __global__ void __launch_bounds__(kSmem ? kAggSmemThreads : kThreads) part_agg_k
   }
 }
 
-// Phase C: destinations and coalesced stores.
-// 4 CTAs/SM (64 registers) and no register double buffering: occupancy hides the load
-// latency better than prefetching at 2 CTAs/SM (measured).
+// Phase C, one chunk inside ONE segment of a split node: ranks from the chunk's go-left
+// ballots plus one carry; each child's entries of a row go to consecutive addresses.
+__device__ __forceinline__ void partition_single_chunk(const PartArgs& a, uint64_t A2, int64_t ch) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t lt_mask = (1u << lane) - 1u;
+  const int64_t wbase = ch * kChunkW;
+  uint32_t rv[kRows];
+  float xv[kRows];
+  double yv[kRows];
+#pragma unroll
+  for (int r = 0; r < kRows; ++r) {
+    const int64_t p = wbase + r * 32 + lane;
+    rv[r] = __ldcs(a.lr + p);
+    xv[r] = __ldcs(a.lx + p);
+    yv[r] = __ldcs(a.ly + p);
+  }
+  const PartDesc dsc = a.desc[ch];
+  const uint32_t mword = (lane < kRows) ? __ldcs(a.gmask + ch * kRows + lane) : 0u;
+  uint32_t carry = (dsc.start == wbase) ? 0u : combine(a.block_carry[ch / kBlockChunks], a.chunk_excl[ch]).c;
+  const uint32_t i0 = (uint32_t)(wbase - dsc.start) + lane;
+  const uint32_t nsl = dsc.ns + dsc.nl;
+  float* const ox = a.ox + (int64_t)dsc.f * (int64_t)A2;
+  uint32_t* const orow = a.orow + (int64_t)dsc.f * (int64_t)A2;
+  double* const oy = a.oy + (int64_t)dsc.f * (int64_t)A2;
+#pragma unroll
+  for (int r = 0; r < kRows; ++r) {
+    const uint32_t gm = __shfl_sync(0xffffffffu, mword, r);
+    const uint32_t g = (gm >> lane) & 1u;
+    const uint32_t rank = carry + __popc(gm & lt_mask);
+    const uint32_t i = i0 + r * 32;
+    const uint32_t dst = g ? dsc.ns + rank : nsl + (i - rank);
+    ox[dst] = xv[r];
+    orow[dst] = rv[r];
+    oy[dst] = yv[r];
+    carry += __popc(gm);
+  }
+}
+
+// Phase C, one chunk with segment boundaries inside.
+__device__ __forceinline__ void partition_general_chunk(const PartArgs& a, uint32_t K, uint64_t A, uint64_t A2,
+                                                      int64_t total, int64_t ch) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t lt_mask = (1u << lane) - 1u;
+  const int64_t wbase = ch * kChunkW;
+  uint32_t rv[kRows];
+  float xv[kRows];
+  double yv[kRows];
+#pragma unroll
+  for (int r = 0; r < kRows; ++r) {
+    const int64_t p = wbase + r * 32 + lane;
+    const bool ok = p < total;
+    rv[r] = ok ? __ldcs(a.lr + p) : 0u;
+    xv[r] = ok ? __ldcs(a.lx + p) : 0.f;
+    yv[r] = ok ? __ldcs(a.ly + p) : 0.0;
+  }
+  const PartDesc dsc = a.desc[ch];
+  // raw go-left bits of my kRows entries, from the chunk's ballots (phase A)
+  const uint32_t mword = (lane < kRows) ? __ldcs(a.gmask + ch * kRows + lane) : 0u;
+  uint32_t graw = 0;
+#pragma unroll
+  for (int r = 0; r < kRows; ++r) graw |= ((__shfl_sync(0xffffffffu, mword, r) >> lane) & 1u) << r;
+  Seg s{0, 0, 0, 0u, 0};
+  seg_from(s, dsc.start, dsc.end, dsc.k, dsc.f, A, min(wbase + lane, total - 1), a.nodes, K);
+  const Seg s0 = s;
+  uint32_t gbits, hbits, sbits;
+  part_flags(a, K, A, wbase, total, s, graw, gbits, hbits, sbits, dsc);
+  const CntP cc = combine(a.block_carry[ch / kBlockChunks], a.chunk_excl[ch]);
+  uint32_t carry = cc.c;  // lefts of the open segment before this chunk
+  s = s0;
+  uint32_t nlv = 0, nsv = 0;
+  int64_t obase = 0;
+  uint32_t cur_k = 0xffffffffu;
+  int cur_f = -1;
+#pragma unroll
+  for (int r = 0; r < kRows; ++r) {
+    const int64_t p = wbase + r * 32 + lane;
+    const uint32_t g = (gbits >> r) & 1u, sp = (sbits >> r) & 1u;
+    const uint32_t gm = __ballot_sync(0xffffffffu, g);
+    const uint32_t hm = __ballot_sync(0xffffffffu, (hbits >> r) & 1u);
+    if (p < total) {
+      while (p >= s.end) seg_next(s, a.nodes, K, A);
+      if (sp) {
+        if (s.k != cur_k || s.f != cur_f) {
+          cur_k = s.k;
+          cur_f = s.f;
+          const bool ind = (s.k == dsc.k && s.f == dsc.f);
+          nlv = ind ? dsc.nl : __ldg(&a.dec[s.k].nl);
+          nsv = ind ? dsc.ns : __ldg(&a.new_start[s.k]);
+          obase = (int64_t)s.f * (int64_t)A2;
+        }
+        const uint32_t le = hm & ((lt_mask << 1) | 1u);  // heads at lanes <= me
+        uint32_t rank;
+        if (le) {
+          const int hl = 31 - __clz(le);
+          rank = __popc(gm & lt_mask & ~((1u << hl) - 1u));
+        } else {
+          rank = carry + __popc(gm & lt_mask);
+        }
+        const uint32_t i = (uint32_t)(p - s.start);
+        const uint32_t dst = g ? nsv + rank : nsv + nlv + (i - rank);
+        const int64_t o = obase + dst;
+        a.ox[o] = xv[r];
+        a.orow[o] = rv[r];
+        a.oy[o] = yv[r];
+      }
+    }
+    if (hm) {
+      const int hl = 31 - __clz(hm);
+      carry = __popc(gm & ~((1u << hl) - 1u));
+    } else {
+      carry += __popc(gm);
+    }
+  }
+}
+
+// Phase C: the level's chunk list, single-segment chunks of split nodes first, then the
+// chunks with segment boundaries (chunks of leaves inside one segment are not listed).
 __global__ void __launch_bounds__(kThreads, 4) partition_kernel(PartArgs a) {
   const uint32_t K = a.ctl->K[a.parity];
   const uint64_t A = a.ctl->A[a.parity];
@@ -1532,112 +1791,12 @@ __global__ void __launch_bounds__(kThreads, 4) partition_kernel(PartArgs a) {
   if (K == 0 || A2 == 0) return;
   const int64_t total = (int64_t)A * a.dl_out;  // only the lists we write
   const int64_t nch = (total + kChunkW - 1) / kChunkW;
-  const int lane = threadIdx.x & 31;
-  const uint32_t lt_mask = (1u << lane) - 1u;
+  const int64_t ns = a.ctl->pcnt[0], ng = a.ctl->pcnt[1];
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  uint32_t rn[kRows];
-  float xn[kRows];
-  double yn[kRows];
-  auto load = [&](int64_t wbase) {
-#pragma unroll
-    for (int r = 0; r < kRows; ++r) {
-      const int64_t p = wbase + r * 32 + lane;
-      const bool ok = p < total;
-      rn[r] = ok ? __ldcs(a.lr + p) : 0u;
-      xn[r] = ok ? __ldcs(a.lx + p) : 0.f;
-      yn[r] = ok ? __ldcs(a.ly + p) : 0.0;
-    }
-  };
-  for (int64_t ch = gw; ch < nch; ch += nw) {
-    const int64_t wbase = ch * kChunkW;
-    load(wbase);
-    uint32_t rv[kRows];
-    float xv[kRows];
-    double yv[kRows];
-#pragma unroll
-    for (int r = 0; r < kRows; ++r) { rv[r] = rn[r]; xv[r] = xn[r]; yv[r] = yn[r]; }
-    const PartDesc dsc = a.desc[ch];
-    // raw go-left bits of my kRows entries, from the chunk's ballots (phase A)
-    const uint32_t mword = (lane < kRows) ? __ldcs(a.gmask + ch * kRows + lane) : 0u;
-    uint32_t graw = 0;
-#pragma unroll
-    for (int r = 0; r < kRows; ++r) graw |= ((__shfl_sync(0xffffffffu, mword, r) >> lane) & 1u) << r;
-    if (dsc.start <= wbase && dsc.end >= wbase + kChunkW) {
-      // whole chunk in one segment: ranks from the go-left ballots and one carry
-      if (!dsc.split) continue;  // rows of leaves are dropped
-      uint32_t carry = (dsc.start == wbase) ? 0u : combine(a.block_carry[ch / kBlockChunks], a.chunk_excl[ch]).c;
-      const uint32_t i0 = (uint32_t)(wbase - dsc.start) + lane;
-      const uint32_t nsl = dsc.ns + dsc.nl;
-      float* const ox = a.ox + (int64_t)dsc.f * (int64_t)A2;
-      uint32_t* const orow = a.orow + (int64_t)dsc.f * (int64_t)A2;
-      double* const oy = a.oy + (int64_t)dsc.f * (int64_t)A2;
-#pragma unroll
-      for (int r = 0; r < kRows; ++r) {
-        const uint32_t g = (graw >> r) & 1u;
-        const uint32_t gm = __ballot_sync(0xffffffffu, g);
-        const uint32_t rank = carry + __popc(gm & lt_mask);
-        const uint32_t i = i0 + r * 32;
-        const uint32_t dst = g ? dsc.ns + rank : nsl + (i - rank);
-        ox[dst] = xv[r];
-        orow[dst] = rv[r];
-        oy[dst] = yv[r];
-        carry += __popc(gm);
-      }
-      continue;
-    }
-    Seg s{0, 0, 0, 0u, 0};
-    seg_from(s, dsc.start, dsc.end, dsc.k, dsc.f, A, min(wbase + lane, total - 1), a.nodes, K);
-    const Seg s0 = s;
-    uint32_t gbits, hbits, sbits;
-    part_flags(a, K, A, wbase, total, s, graw, gbits, hbits, sbits, dsc);
-    const CntP cc = combine(a.block_carry[ch / kBlockChunks], a.chunk_excl[ch]);
-    uint32_t carry = cc.c;  // lefts of the open segment before this chunk
-    s = s0;
-    uint32_t nlv = 0, nsv = 0;
-    int64_t obase = 0;
-    uint32_t cur_k = 0xffffffffu;
-    int cur_f = -1;
-#pragma unroll
-    for (int r = 0; r < kRows; ++r) {
-      const int64_t p = wbase + r * 32 + lane;
-      const uint32_t g = (gbits >> r) & 1u, sp = (sbits >> r) & 1u;
-      const uint32_t gm = __ballot_sync(0xffffffffu, g);
-      const uint32_t hm = __ballot_sync(0xffffffffu, (hbits >> r) & 1u);
-      if (p < total) {
-        while (p >= s.end) seg_next(s, a.nodes, K, A);
-        if (sp) {
-          if (s.k != cur_k || s.f != cur_f) {
-            cur_k = s.k;
-            cur_f = s.f;
-            const bool ind = (s.k == dsc.k && s.f == dsc.f);
-            nlv = ind ? dsc.nl : __ldg(&a.dec[s.k].nl);
-            nsv = ind ? dsc.ns : __ldg(&a.new_start[s.k]);
-            obase = (int64_t)s.f * (int64_t)A2;
-          }
-          const uint32_t le = hm & ((lt_mask << 1) | 1u);  // heads at lanes <= me
-          uint32_t rank;
-          if (le) {
-            const int hl = 31 - __clz(le);
-            rank = __popc(gm & lt_mask & ~((1u << hl) - 1u));
-          } else {
-            rank = carry + __popc(gm & lt_mask);
-          }
-          const uint32_t i = (uint32_t)(p - s.start);
-          const uint32_t dst = g ? nsv + rank : nsv + nlv + (i - rank);
-          const int64_t o = obase + dst;
-          a.ox[o] = xv[r];
-          a.orow[o] = rv[r];
-          a.oy[o] = yv[r];
-        }
-      }
-      if (hm) {
-        const int hl = 31 - __clz(hm);
-        carry = __popc(gm & ~((1u << hl) - 1u));
-      } else {
-        carry += __popc(gm);
-      }
-    }
+  for (int64_t idx = gw; idx < ns + ng; idx += nw) {
+    if (idx < ns) partition_single_chunk(a, A2, (int64_t)a.list[idx]);
+    else partition_general_chunk(a, K, A, A2, total, (int64_t)a.list[nch - 1 - (idx - ns)]);
   }
 }
 
@@ -1695,6 +1854,7 @@ struct FitBufs {
   void* sort_tmp;           // d slices of sort_tmp_bytes (one CUB sort per feature)
   size_t sort_tmp_bytes;
   ChunkDesc* sdesc;
+  uint32_t *slist, *plist;  // per-level chunk lists (scan, partition)
   PartDesc* pdesc;
   SumP *chunk_agg, *chunk_excl, *block_agg, *block_carry;
   CntP *pchunk_agg, *pchunk_excl, *pblock_agg, *pblock_carry;
@@ -1762,6 +1922,8 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, int wor
   b.sort_tmp_bytes = (b.sort_tmp_bytes + 255) & ~(size_t)255;
   DT_CK(get((char**)&b.sort_tmp, b.sort_tmp_bytes * (size_t)d));
   DT_CK(get(&b.sdesc, (size_t)b.max_chunks));
+  DT_CK(get(&b.slist, (size_t)b.max_chunks));
+  DT_CK(get(&b.plist, (size_t)b.max_chunks));
   DT_CK(get(&b.pdesc, (size_t)b.max_chunks));
   DT_CK(get(&b.chunk_agg, (size_t)b.max_chunks));
   DT_CK(get(&b.chunk_excl, (size_t)b.max_chunks));
@@ -1862,6 +2024,9 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     DT_CK(cudaGetLastError());
   }
   const int g_scan = persistent_grid((const void*)scan_kernel, kThreads, 0);
+  DT_CK(cudaFuncSetAttribute((const void*)scan_single_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)kScanSingleSmem));
+  const int g_scan1 = persistent_grid((const void*)scan_single_kernel, kThreads, kScanSingleSmem);
   const int g_agg = persistent_grid((const void*)scan_agg_kernel, kThreads, 0);
   const int g_pagg = persistent_grid((const void*)part_agg_kernel<false>, kThreads, 0);
   size_t agg_smem = sizeof(uint32_t) * (size_t)b.nwords4;
@@ -1878,10 +2043,11 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     const bool last = (max_depth >= 0 && level == max_depth);
     const int dl = last ? 1 : d;
     // scan (a4)
-    int pr = prof_begin(PK_SCAN, s, 5);
-    scan_desc_kernel<<<num_sms() * 4, 256, 0, s>>>(b.nodes[parity], ctl, parity, dl, kChunkW, b.sdesc);
+    int pr = prof_begin(PK_SCAN, s, 6);
+    scan_desc_kernel<<<num_sms() * 4, 256, 0, s>>>(b.nodes[parity], ctl, parity, dl, kChunkW, b.sdesc, b.slist);
     ScanArgs sa;
     sa.desc = b.sdesc;
+    sa.list = b.slist;
     sa.lx = b.lx[cur];
     sa.ly = b.ly[cur];
     sa.nodes = b.nodes[parity];
@@ -1903,6 +2069,7 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     scan_agg_kernel<<<g_agg, kThreads, 0, s>>>(sa);
     chunk_scan_kernel<SumP><<<(unsigned)b.max_cblocks, 1024, 0, s>>>(ctl, parity, dl, b.chunk_agg, b.chunk_excl, b.block_agg);
     block_carry_kernel<SumP><<<1, 1024, 0, s>>>(ctl, parity, dl, b.block_agg, b.block_carry);
+    scan_single_kernel<<<g_scan1, kThreads, kScanSingleSmem, s>>>(sa);
     scan_kernel<<<g_scan, kThreads, 0, s>>>(sa);
     prof_end(pr, s, 0.0);
     if (pending) pending->push_back({pr, level, PK_SCAN, dl});
@@ -1996,7 +2163,9 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     pa.block_agg = b.pblock_agg;
     pa.block_carry = b.pblock_carry;
     pr = prof_begin(PK_PARTITION, s, 5);
-    part_desc_kernel<<<num_sms() * 4, 256, 0, s>>>(b.nodes[parity], b.dec, b.new_start, ctl, parity, pa.dl_out, b.pdesc);
+    pa.list = b.plist;
+    part_desc_kernel<<<num_sms() * 4, 256, 0, s>>>(b.nodes[parity], b.dec, b.new_start, ctl, parity, pa.dl_out, b.pdesc,
+                                                   b.plist);
     if (agg_smem) part_agg_kernel<true><<<num_sms(), kAggSmemThreads, agg_smem, s>>>(pa);
     else part_agg_kernel<false><<<g_pagg, kThreads, 0, s>>>(pa);
     chunk_scan_kernel<CntP><<<(unsigned)b.max_cblocks, 1024, 0, s>>>(ctl, parity, pa.dl_out, b.pchunk_agg, b.pchunk_excl, b.pblock_agg);
