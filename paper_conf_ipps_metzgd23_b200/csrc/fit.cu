@@ -81,6 +81,8 @@ struct Ctl {
   // chunk lists of the level (single-segment chunks from the front, others from the back)
   uint32_t scnt[2];  // scan: singles, others
   uint32_t pcnt[2];  // partition: singles, others
+  uint32_t ticket;   // chunk_scan_kernel: blocks done (the last one computes the block carries)
+  uint32_t pad2;
 };
 
 struct LevelLog {  // per-level counts, for algorithmic-byte accounting (profiling)
@@ -101,6 +103,20 @@ struct Cand {  // best candidate of one segment piece
 struct Stat {
   double sse, ymin, ymax, s1;  // s1 = sum (y - c) over the piece
 };
+
+// L2 (coherent) loads of a carry payload written by other blocks of the same launch.
+__device__ __forceinline__ SumP ld_cg(const SumP* p) {
+  SumP r;
+  r.flag = __ldcg(&p->flag);
+  r.s = __ldcg(&p->s);
+  return r;
+}
+__device__ __forceinline__ CntP ld_cg(const CntP* p) {
+  CntP r;
+  r.flag = __ldcg(&p->flag);
+  r.c = __ldcg(&p->c);
+  return r;
+}
 
 // Per-level descriptor of the segment holding the FIRST entry of each warp chunk
 // (kChunkW entries): one independent load per chunk instead of a dependent lookup chain.
@@ -601,68 +617,66 @@ __global__ void __launch_bounds__(kThreads) scan_agg_kernel(ScanArgs a) {
   }
 }
 
-// Phase B1: exclusive segmented scan of per-chunk aggregates inside blocks of
-// kBlockChunks chunks (kPer per thread sequentially, then a block scan); fixed shape.
-// Used for the scan (SumP) and the partition (CntP).
+// Phase B: exclusive segmented scan of per-chunk aggregates inside blocks of
+// kBlockChunks chunks (kPer per thread sequentially, then a block scan), then -- by the
+// last block to finish (ticket) -- the exclusive scan of the block aggregates (carries).
+// Fixed shape, so deterministic.  Used for the scan (SumP) and the partition (CntP).
 template <class T>
-__global__ void __launch_bounds__(1024) chunk_scan_kernel(const Ctl* ctl, int parity, int dl,
+__global__ void __launch_bounds__(1024) chunk_scan_kernel(Ctl* ctl, int parity, int dl,
                                                           const T* __restrict__ chunk_agg,
-                                                          T* __restrict__ chunk_excl, T* __restrict__ block_agg) {
-  __shared__ T sh[33];
-  const uint32_t K = ctl->K[parity];
-  const uint64_t A = ctl->A[parity];
-  if (K == 0 || A == 0) return;
-  const int64_t total = (int64_t)A * dl;
-  const int64_t nch = (total + kChunkW - 1) / kChunkW;
-  const int64_t b0 = (int64_t)blockIdx.x * kBlockChunks;
-  if (b0 >= nch) return;
-  constexpr int kPer = kBlockChunks / 1024;
-  const int64_t c0 = b0 + (int64_t)threadIdx.x * kPer;
-  T zero;
-  zero.flag = 0u;
-  from_bits(zero, 0ull);
-  T v[kPer];
-  T agg = zero;
-#pragma unroll
-  for (int q = 0; q < kPer; ++q) {
-    v[q] = (c0 + q < nch) ? chunk_agg[c0 + q] : zero;
-    agg = (q == 0) ? v[0] : combine(agg, v[q]);
-  }
-  T bagg;
-  T cur = block_exclusive_scan(agg, zero, bagg, sh);
-#pragma unroll
-  for (int q = 0; q < kPer; ++q) {
-    if (c0 + q < nch) chunk_excl[c0 + q] = cur;
-    cur = combine(cur, v[q]);
-  }
-  if (threadIdx.x == 0) block_agg[blockIdx.x] = bagg;
-}
-
-// Phase B2: exclusive segmented scan of the block aggregates (one block, fixed shape).
-template <class T>
-__global__ void __launch_bounds__(1024) block_carry_kernel(const Ctl* ctl, int parity, int dl,
-                                                           const T* __restrict__ block_agg,
-                                                           T* __restrict__ block_carry) {
+                                                          T* __restrict__ chunk_excl, T* block_agg,
+                                                          T* __restrict__ block_carry) {
   __shared__ T sh[33];
   __shared__ T sh_run;
+  __shared__ bool s_last;
   const uint32_t K = ctl->K[parity];
   const uint64_t A = ctl->A[parity];
-  if (K == 0 || A == 0) return;
-  const int64_t total = (int64_t)A * dl;
+  const int64_t total = (K == 0) ? 0 : (int64_t)A * dl;
   const int64_t nch = (total + kChunkW - 1) / kChunkW;
-  const int64_t nb = (nch + kBlockChunks - 1) / kBlockChunks;
+  const int64_t b0 = (int64_t)blockIdx.x * kBlockChunks;
   T zero;
   zero.flag = 0u;
   from_bits(zero, 0ull);
-  if (threadIdx.x == 0) sh_run = zero;
+  if (b0 < nch) {  // block-uniform
+    constexpr int kPer = kBlockChunks / 1024;
+    const int64_t c0 = b0 + (int64_t)threadIdx.x * kPer;
+    T v[kPer];
+    T agg = zero;
+#pragma unroll
+    for (int q = 0; q < kPer; ++q) {
+      v[q] = (c0 + q < nch) ? chunk_agg[c0 + q] : zero;
+      agg = (q == 0) ? v[0] : combine(agg, v[q]);
+    }
+    T bagg;
+    T cur = block_exclusive_scan(agg, zero, bagg, sh);
+#pragma unroll
+    for (int q = 0; q < kPer; ++q) {
+      if (c0 + q < nch) chunk_excl[c0 + q] = cur;
+      cur = combine(cur, v[q]);
+    }
+    if (threadIdx.x == 0) block_agg[blockIdx.x] = bagg;
+  }
+  // the last block to arrive scans the block aggregates
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) s_last = atomicAdd(&ctl->ticket, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  if (threadIdx.x == 0) {
+    ctl->ticket = 0u;  // ready for the next launch
+    sh_run = zero;
+  }
+  const int64_t nb = (nch + kBlockChunks - 1) / kBlockChunks;
   __syncthreads();
   for (int64_t base = 0; base < nb; base += blockDim.x) {
-    const int64_t b = base + threadIdx.x;
-    const T v = (b < nb) ? block_agg[b] : zero;
+    const int64_t bi = base + threadIdx.x;
+    T v = zero;
+    if (bi < nb) v = ld_cg(block_agg + bi);
     T chunk;
     const T ex = block_exclusive_scan(v, zero, chunk, sh);
     const T run = sh_run;
-    if (b < nb) block_carry[b] = combine(run, ex);
+    if (bi < nb) block_carry[bi] = combine(run, ex);
     __syncthreads();
     if (threadIdx.x == 0) sh_run = combine(run, chunk);
     __syncthreads();
@@ -1186,6 +1200,60 @@ struct SelectArgs {
   int world, rank, dg;  // feature sharding: local feature j is global j * world + rank
 };
 
+// Leaf rules and the decision of node k from the ranks' records (see decide_kernel).
+__device__ __forceinline__ void decide_node(const SelectArgs& a, uint32_t k, const NodeL& nd,
+                                            const ExchRec* __restrict__ all, int64_t stride) {
+  const ExchRec st = all[k];  // rank 0
+  const bool pure = !(st.ymin < st.ymax);
+  int bf = -1;
+  ExchRec best;
+  best.gain = -1.0;
+  if (nd.searchable && !pure) {
+    for (int r = 0; r < a.world; ++r) {
+      const ExchRec c = all[(int64_t)r * stride + k];
+      if (c.gain < 0.0) continue;
+      if (bf < 0 || c.gain > best.gain || (c.gain == best.gain && c.gf < bf)) {
+        best = c;
+        bf = c.gf;
+      }
+    }
+    atomicAdd(&a.ctl->split_evals, (unsigned long long)nd.N * (unsigned long long)a.dg);
+  }
+  Decision dc;
+  dt_node o;
+  o.depth = a.level;
+  // value = mean of the node's own rows.  Integer mode: exact fl(S/N) from the exact
+  // bookkeeping.  Real mode: centre + fresh sum (y - c) / N, and exactly y for a pure
+  // node (all rows equal), so single-row leaves reproduce their target.
+  if (a.ctl->int_mode) o.value = nd.v;
+  else o.value = pure ? st.ymin : __dadd_rn(nd.c, __ddiv_rn(st.s1, (double)nd.N));
+  o.impurity = __ddiv_rn(st.sse, (double)nd.N);
+  o.n_samples = nd.N;
+  o.left = -1;
+  o.right = -1;
+  dc.pad = 0;
+  if (bf >= 0) {
+    dc.f = bf;
+    dc.floc = (bf % a.world == a.rank) ? bf / a.world : -1;
+    dc.nl = best.i;
+    dc.sl = best.sl;
+    dc.thr = best.thr;
+    o.feature = bf;
+    o.threshold = best.thr;
+  } else {
+    dc.f = -1;
+    dc.floc = -1;
+    dc.nl = 0;
+    dc.sl = 0.0;
+    dc.thr = 0.0;
+    o.feature = -1;
+    o.threshold = 0.0;
+  }
+  a.dec[k] = dc;
+  a.out[nd.id] = o;
+  atomicMax(&a.ctl->max_depth_seen, a.level);
+}
+
 // One block per node (grid-stride over the level's nodes).
 __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
   const uint32_t K = a.ctl->K[a.parity];
@@ -1281,6 +1349,7 @@ __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
       r.ymax = st.ymax;
       r.s1 = st.s1;
       a.exch[k] = r;
+      if (a.world == 1) decide_node(a, k, nd, a.exch, 0);  // single rank: decide in place
     }
     __syncthreads();
   }
@@ -1292,58 +1361,8 @@ __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
 __global__ void __launch_bounds__(256) decide_kernel(SelectArgs a, const ExchRec* __restrict__ all,
                                                      int64_t stride) {
   const uint32_t K = a.ctl->K[a.parity];
-  for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < K; k += gridDim.x * blockDim.x) {
-    const NodeL nd = a.nodes[k];
-    const ExchRec st = all[k];  // rank 0
-    const bool pure = !(st.ymin < st.ymax);
-    int bf = -1;
-    ExchRec best;
-    best.gain = -1.0;
-    if (nd.searchable && !pure) {
-      for (int r = 0; r < a.world; ++r) {
-        const ExchRec c = all[(int64_t)r * stride + k];
-        if (c.gain < 0.0) continue;
-        if (bf < 0 || c.gain > best.gain || (c.gain == best.gain && c.gf < bf)) {
-          best = c;
-          bf = c.gf;
-        }
-      }
-      atomicAdd(&a.ctl->split_evals, (unsigned long long)nd.N * (unsigned long long)a.dg);
-    }
-    Decision dc;
-    dt_node o;
-    o.depth = a.level;
-    // value = mean of the node's own rows.  Integer mode: exact fl(S/N) from the exact
-    // bookkeeping.  Real mode: centre + fresh sum (y - c) / N, and exactly y for a pure
-    // node (all rows equal), so single-row leaves reproduce their target.
-    if (a.ctl->int_mode) o.value = nd.v;
-    else o.value = pure ? st.ymin : __dadd_rn(nd.c, __ddiv_rn(st.s1, (double)nd.N));
-    o.impurity = __ddiv_rn(st.sse, (double)nd.N);
-    o.n_samples = nd.N;
-    o.left = -1;
-    o.right = -1;
-    dc.pad = 0;
-    if (bf >= 0) {
-      dc.f = bf;
-      dc.floc = (bf % a.world == a.rank) ? bf / a.world : -1;
-      dc.nl = best.i;
-      dc.sl = best.sl;
-      dc.thr = best.thr;
-      o.feature = bf;
-      o.threshold = best.thr;
-    } else {
-      dc.f = -1;
-      dc.floc = -1;
-      dc.nl = 0;
-      dc.sl = 0.0;
-      dc.thr = 0.0;
-      o.feature = -1;
-      o.threshold = 0.0;
-    }
-    a.dec[k] = dc;
-    a.out[nd.id] = o;
-    atomicMax(&a.ctl->max_depth_seen, a.level);
-  }
+  for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < K; k += gridDim.x * blockDim.x)
+    decide_node(a, k, a.nodes[k], all, stride);
 }
 
 // ----------------------------------------------------------------------------- number --
@@ -1453,6 +1472,8 @@ __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
   }
   if (tid == 0) {
     const int np = a.parity ^ 1;
+    a.ctl->pcnt[0] = a.ctl->pcnt[1] = 0;  // this level's partition lists (prep_kernel)
+    a.ctl->scnt[0] = a.ctl->scnt[1] = 0;  // the next level's scan lists (prep_kernel)
     a.ctl->K[np] = 2 * base_split;
     a.ctl->A[np] = base_rows;
     a.ctl->next_id = next_id0 + 2 * (int)base_split;
@@ -1465,64 +1486,117 @@ __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
 
 // ----------------------------------------------------------------------------- goleft --
 
-// Go-left bitmap: bit r of gbits is set iff row r goes to the left child (rows of split
-// nodes only; zeroed before every level).  Only the first nl positions of a split node
-// in its split feature's list go left, so only those row ids are read.
-__global__ void __launch_bounds__(256) goleft_kernel(const uint32_t* __restrict__ lr, const NodeL* nodes,
-                                                     const Decision* dec, const Ctl* ctl, int parity,
-                                                     uint32_t* __restrict__ gbits) {
-  const uint32_t K = ctl->K[parity];
-  const uint64_t A = ctl->A[parity];
-  if (K == 0) return;
-  constexpr int kI = 8;
-  for (int64_t q0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * kI; q0 < (int64_t)A;
-       q0 += (int64_t)gridDim.x * blockDim.x * kI) {
-    uint32_t k = find_node(nodes, K, (uint32_t)q0);
-    uint32_t kstart = nodes[k].start, kend = kstart + nodes[k].N;
-    for (int j = 0; j < kI && q0 + j < (int64_t)A; ++j) {
-      const uint32_t q = (uint32_t)q0 + j;
-      while (q >= kend) { ++k; kstart = kend; kend = kstart + nodes[k].N; }
-      const Decision dc = dec[k];
-      if (dc.floc >= 0 && q - kstart < dc.nl) {
-        const uint32_t r = lr[(int64_t)dc.floc * (int64_t)A + q];
-        atomicOr(gbits + (r >> 5), 1u << (r & 31));
-      }
-    }
-  }
-}
-
 // ----------------------------------------------------------------------------- partition --
 
-__global__ void __launch_bounds__(256) part_desc_kernel(const NodeL* __restrict__ nodes,
-                                                        const Decision* __restrict__ dec,
-                                                        const uint32_t* __restrict__ new_start, Ctl* ctl,
-                                                        int parity, int dl, PartDesc* __restrict__ desc,
-                                                        uint32_t* __restrict__ list) {
-  const uint32_t K = ctl->K[parity];
-  const uint64_t A = ctl->A[parity];
-  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->scnt[0] = ctl->scnt[1] = 0;  // next level's scan lists
-  if (K == 0 || A == 0 || ctl->A[parity ^ 1] == 0) return;
-  const int64_t total = (int64_t)A * dl;
-  const int64_t nch = (total + kChunkW - 1) / kChunkW;
-  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < nch; c += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t p = c * kChunkW;
-    const int f = (int)(p / (int64_t)A);
-    const int64_t fbase = (int64_t)f * (int64_t)A;
-    const uint32_t k = find_node(nodes, K, (uint32_t)(p - fbase));
-    PartDesc d;
-    d.start = fbase + nodes[k].start;
-    d.end = d.start + nodes[k].N;
-    d.k = k;
-    d.f = f;
-    const Decision dc = dec[k];
-    d.nl = dc.nl;
-    d.split = dc.f >= 0 ? 1 : 0;
-    d.ns = new_start[k];
-    d.pad = 0;
-    desc[c] = d;
-    // single-segment chunks of leaves have nothing to move: in neither list
-    const bool single = d.start <= p && d.end >= p + kChunkW;
-    if (!single || d.split) list_chunk(ctl->pcnt, list, nch, c, single);
+// Binary search over a level's node starts cached in shared memory: largest k with
+// st[k] <= q.
+__device__ __forceinline__ uint32_t find_start(const uint32_t* st, uint32_t K, uint32_t q) {
+  uint32_t lo = 0, hi = K;
+  while (hi - lo > 1) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (st[mid] <= q) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+
+struct PrepArgs {
+  const uint32_t* lr;         // this level's row lists
+  const NodeL* nodes;         // this level's nodes
+  const NodeL* next;          // next level's nodes (from number_kernel)
+  const Decision* dec;
+  const uint32_t* new_start;
+  uint32_t* gbits;            // zeroed go-left bitmap
+  PartDesc* pdesc;
+  uint32_t* plist;
+  ChunkDesc* sdesc;
+  uint32_t* slist;
+  Ctl* ctl;
+  int parity;
+  int dl_out;   // lists the partition writes (= lists the next level scans)
+};
+constexpr int kPrepCache = 12288;  // node starts of both levels cached per block (48 KB)
+constexpr int kPrepThreads = 1024;
+
+// Everything between the numbering of level l and its partition, in one launch (one
+// block per SM, the node starts of levels l and l+1 in shared memory):
+//   goleft:    bit per row of every split node's left rows (a6);
+//   part desc: level-l partition chunk descriptors and chunk lists;
+//   scan desc: level-(l+1) scan chunk descriptors and chunk lists.
+// The three index spaces are independent; the list counters were reset by number_kernel.
+__global__ void __launch_bounds__(kPrepThreads) prep_kernel(PrepArgs a) {
+  __shared__ uint32_t st[kPrepCache];
+  const uint32_t K = a.ctl->K[a.parity], K2 = a.ctl->K[a.parity ^ 1];
+  const uint64_t A = a.ctl->A[a.parity], A2 = a.ctl->A[a.parity ^ 1];
+  if (K == 0 || A == 0 || A2 == 0) return;  // nothing splits: nothing moves, no next level
+  const bool cache = (uint64_t)K + K2 <= (uint64_t)kPrepCache;
+  uint32_t* s1 = st;
+  uint32_t* s2 = st + K;
+  if (cache) {
+    for (uint32_t i = threadIdx.x; i < K; i += blockDim.x) s1[i] = __ldg(&a.nodes[i].start);
+    for (uint32_t i = threadIdx.x; i < K2; i += blockDim.x) s2[i] = __ldg(&a.next[i].start);
+    __syncthreads();
+  }
+  constexpr int kI = 8;  // goleft positions per work item
+  const int64_t G = ((int64_t)A + kI - 1) / kI;
+  const int64_t P = ((int64_t)A * a.dl_out + kChunkW - 1) / kChunkW;
+  const int64_t S = ((int64_t)A2 * a.dl_out + kChunkW - 1) / kChunkW;
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < G + P + S;
+       t += (int64_t)gridDim.x * blockDim.x) {
+    if (t < G) {
+      const uint32_t q0 = (uint32_t)(t * kI);
+      uint32_t k = cache ? find_start(s1, K, q0) : find_node(a.nodes, K, q0);
+      uint32_t kstart = __ldg(&a.nodes[k].start), kend = kstart + __ldg(&a.nodes[k].N);
+      for (int j = 0; j < kI && (uint64_t)q0 + j < A; ++j) {
+        const uint32_t q = q0 + j;
+        while (q >= kend) { ++k; kstart = kend; kend = kstart + __ldg(&a.nodes[k].N); }
+        const int32_t floc = __ldg(&a.dec[k].floc);
+        if (floc >= 0 && q - kstart < __ldg(&a.dec[k].nl)) {
+          const uint32_t r = __ldg(&a.lr[(int64_t)floc * (int64_t)A + q]);
+          atomicOr(a.gbits + (r >> 5), 1u << (r & 31));
+        }
+      }
+    } else if (t < G + P) {
+      const int64_t c = t - G;
+      const int64_t p = c * kChunkW;
+      const int f = (int)(p / (int64_t)A);
+      const int64_t fbase = (int64_t)f * (int64_t)A;
+      const uint32_t q = (uint32_t)(p - fbase);
+      const uint32_t k = cache ? find_start(s1, K, q) : find_node(a.nodes, K, q);
+      PartDesc d;
+      d.start = fbase + __ldg(&a.nodes[k].start);
+      d.end = d.start + __ldg(&a.nodes[k].N);
+      d.k = k;
+      d.f = f;
+      const Decision dc = a.dec[k];
+      d.nl = dc.nl;
+      d.split = dc.f >= 0 ? 1 : 0;
+      d.ns = __ldg(&a.new_start[k]);
+      d.pad = 0;
+      a.pdesc[c] = d;
+      // single-segment chunks of leaves have nothing to move: in neither list
+      const bool single = d.start <= p && d.end >= p + kChunkW;
+      if (!single || d.split) list_chunk(a.ctl->pcnt, a.plist, P, c, single);
+    } else {
+      const int64_t c = t - G - P;
+      const int64_t p = c * kChunkW;
+      const int f = (int)(p / (int64_t)A2);
+      const int64_t fbase = (int64_t)f * (int64_t)A2;
+      const uint32_t q = (uint32_t)(p - fbase);
+      const uint32_t k = cache ? find_start(s2, K2, q) : find_node(a.next, K2, q);
+      const NodeL nd = a.next[k];
+      ChunkDesc d;
+      d.start = fbase + nd.start;
+      d.end = d.start + nd.N;
+      d.k = k;
+      d.f = f;
+      d.c = nd.c;
+      d.sc = nd.sc;
+      d.v = nd.v;
+      d.N = nd.N;
+      d.srch = nd.searchable;
+      a.sdesc[c] = d;
+      list_chunk(a.ctl->scnt, a.slist, S, c, d.start <= p && d.end >= p + kChunkW);
+    }
   }
 }
 
@@ -1540,7 +1614,7 @@ struct PartArgs {
   uint32_t* gmask;        // [nchunks * kRows] go-left ballots per row of 32 entries (phase A -> C)
   int64_t nwords;         // bitmap words
   const PartDesc* desc;  // per warp chunk
-  const uint32_t* list;   // chunk list (part_desc_kernel): split singles first, others from the back
+  const uint32_t* list;   // chunk list (prep_kernel): split singles first, others from the back
   const Ctl* ctl;
   int parity;
   int dl_in;   // lists in the input (d)
@@ -2043,8 +2117,9 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     const bool last = (max_depth >= 0 && level == max_depth);
     const int dl = last ? 1 : d;
     // scan (a4)
-    int pr = prof_begin(PK_SCAN, s, 6);
-    scan_desc_kernel<<<num_sms() * 4, 256, 0, s>>>(b.nodes[parity], ctl, parity, dl, kChunkW, b.sdesc, b.slist);
+    int pr = prof_begin(PK_SCAN, s, level == 0 ? 5 : 4);
+    // level 0's chunk descriptors; deeper levels' come from the previous level's prep_kernel
+    if (level == 0) scan_desc_kernel<<<num_sms() * 4, 256, 0, s>>>(b.nodes[parity], ctl, parity, dl, kChunkW, b.sdesc, b.slist);
     ScanArgs sa;
     sa.desc = b.sdesc;
     sa.list = b.slist;
@@ -2067,8 +2142,8 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     sa.slot_gain = b.slot_gain;
     sa.level = (uint32_t)level;
     scan_agg_kernel<<<g_agg, kThreads, 0, s>>>(sa);
-    chunk_scan_kernel<SumP><<<(unsigned)b.max_cblocks, 1024, 0, s>>>(ctl, parity, dl, b.chunk_agg, b.chunk_excl, b.block_agg);
-    block_carry_kernel<SumP><<<1, 1024, 0, s>>>(ctl, parity, dl, b.block_agg, b.block_carry);
+    chunk_scan_kernel<SumP><<<(unsigned)b.max_cblocks, 1024, 0, s>>>(ctl, parity, dl, b.chunk_agg, b.chunk_excl,
+                                                                     b.block_agg, b.block_carry);
     scan_single_kernel<<<g_scan1, kThreads, kScanSingleSmem, s>>>(sa);
     scan_kernel<<<g_scan, kThreads, 0, s>>>(sa);
     prof_end(pr, s, 0.0);
@@ -2096,7 +2171,7 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     se.world = sh.world;
     se.rank = sh.rank;
     se.dg = sh.dg;
-    pr = prof_begin(PK_SELECT, s, 3);
+    pr = prof_begin(PK_SELECT, s, sh.world > 1 ? 3 : 2);
     piece_pos_kernel<<<num_sms() * 4, 256, 0, s>>>(sa, b.slot_pos);
     select_kernel<<<g_sel, 256, 0, s>>>(se);
     // exchange the per-node local bests (at most min(kcap, 2^level) nodes at this level)
@@ -2105,8 +2180,9 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
       dt_status cst = comm_allgather(sh.comm, b.exch_send, b.exch_all, sizeof(ExchRec) * (size_t)cnt, s);
       if (cst != DT_OK) return cst;
     }
-    decide_kernel<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((cnt + 255) / 256, num_sms() * 4)), 256, 0, s>>>(
-        se, b.exch_all, cnt);
+    if (sh.world > 1)  // (a single rank decides inside select_kernel)
+      decide_kernel<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((cnt + 255) / 256, num_sms() * 4)), 256, 0, s>>>(
+          se, b.exch_all, cnt);
     prof_end(pr, s, 0.0);
     DT_CK(cudaGetLastError());
     if (last) break;
@@ -2127,10 +2203,28 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     number_kernel<<<1, 1024, 0, s>>>(na);
     prof_end(pr, s, 0.0);
     DT_CK(cudaGetLastError());
-    // go-left map (a6)
+    // go-left map (a6) + this level's partition descriptors + the next level's scan
+    // descriptors (one launch)
+    const int dl_out = (max_depth >= 0 && level + 1 == max_depth) ? 1 : d;
     pr = prof_begin(PK_GOLEFT, s, 1);
     DT_CK(cudaMemsetAsync(b.gbits, 0, sizeof(uint32_t) * (size_t)b.nwords4, s));
-    goleft_kernel<<<g_gl, 256, 0, s>>>(b.lr[cur], b.nodes[parity], b.dec, ctl, parity, b.gbits);
+    {
+      PrepArgs pp;
+      pp.lr = b.lr[cur];
+      pp.nodes = b.nodes[parity];
+      pp.next = b.nodes[parity ^ 1];
+      pp.dec = b.dec;
+      pp.new_start = b.new_start;
+      pp.gbits = b.gbits;
+      pp.pdesc = b.pdesc;
+      pp.plist = b.plist;
+      pp.sdesc = b.sdesc;
+      pp.slist = b.slist;
+      pp.ctl = ctl;
+      pp.parity = parity;
+      pp.dl_out = dl_out;
+      prep_kernel<<<num_sms(), kPrepThreads, 0, s>>>(pp);
+    }
     if (sh.world > 1) {
       // only the owner of each split feature set its rows' bits: OR over the ranks
       dt_status cst = comm_allreduce_or_u32(sh.comm, b.gbits, b.nwords4, s);
@@ -2157,19 +2251,17 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     pa.ctl = ctl;
     pa.parity = parity;
     pa.dl_in = d;
-    pa.dl_out = (max_depth >= 0 && level + 1 == max_depth) ? 1 : d;
+    pa.dl_out = dl_out;
     pa.chunk_agg = b.pchunk_agg;
     pa.chunk_excl = b.pchunk_excl;
     pa.block_agg = b.pblock_agg;
     pa.block_carry = b.pblock_carry;
-    pr = prof_begin(PK_PARTITION, s, 5);
+    pr = prof_begin(PK_PARTITION, s, 3);
     pa.list = b.plist;
-    part_desc_kernel<<<num_sms() * 4, 256, 0, s>>>(b.nodes[parity], b.dec, b.new_start, ctl, parity, pa.dl_out, b.pdesc,
-                                                   b.plist);
     if (agg_smem) part_agg_kernel<true><<<num_sms(), kAggSmemThreads, agg_smem, s>>>(pa);
     else part_agg_kernel<false><<<g_pagg, kThreads, 0, s>>>(pa);
-    chunk_scan_kernel<CntP><<<(unsigned)b.max_cblocks, 1024, 0, s>>>(ctl, parity, pa.dl_out, b.pchunk_agg, b.pchunk_excl, b.pblock_agg);
-    block_carry_kernel<CntP><<<1, 1024, 0, s>>>(ctl, parity, pa.dl_out, b.pblock_agg, b.pblock_carry);
+    chunk_scan_kernel<CntP><<<(unsigned)b.max_cblocks, 1024, 0, s>>>(ctl, parity, pa.dl_out, b.pchunk_agg,
+                                                                     b.pchunk_excl, b.pblock_agg, b.pblock_carry);
     partition_kernel<<<g_part, kThreads, 0, s>>>(pa);
     prof_end(pr, s, 0.0);
     if (pending) pending->push_back({pr, level, PK_PARTITION, pa.dl_out});
