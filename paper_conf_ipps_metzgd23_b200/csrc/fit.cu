@@ -326,6 +326,164 @@ __global__ void __launch_bounds__(256) presort_build_kernel(const uint32_t* __re
   }
 }
 
+// Batched LSD radix sort of the d per-feature key lists (n <= kTileSortMaxRows): 4 passes
+// of 8-bit digits; per pass three launches, each over all d features (grid.y = feature):
+//   rs_count:   per-tile digit counts;
+//   rs_offset:  per (feature, digit) exclusive scan of the counts over the tiles, and the
+//               digit totals;
+//   rs_scatter: every key's stable rank inside its tile (warp match_any per step of 32
+//               keys + per-warp digit counters; keys in tile order), then its destination
+//               = (keys of smaller digits) + (same digit, earlier tiles) + rank.
+// Stable within a feature, so equal keys keep the row order: (x, row id) order (R6).
+constexpr int kTS = 256, kTI = 8, kTile = kTS * kTI;
+constexpr int64_t kTileSortMaxRows = int64_t(1) << 24;
+
+__global__ void __launch_bounds__(kTS) rs_count_kernel(const uint32_t* __restrict__ keys, int64_t n, int shift,
+                                                       int tiles, uint32_t* __restrict__ cnt) {
+  __shared__ uint32_t h[256];
+  const int f = blockIdx.y, tile = blockIdx.x;
+  h[threadIdx.x] = 0u;
+  __syncthreads();
+  const int64_t base = (int64_t)f * n + (int64_t)tile * kTile;
+  const int m = (int)min((int64_t)kTile, n - (int64_t)tile * kTile);
+  for (int i = threadIdx.x; i < m; i += kTS) atomicAdd(&h[(__ldg(keys + base + i) >> shift) & 255u], 1u);
+  __syncthreads();
+  cnt[((int64_t)f * 256 + threadIdx.x) * tiles + tile] = h[threadIdx.x];
+}
+
+// grid (256 digits, d features): exclusive prefix of one digit's counts over the tiles
+// (fixed shape; integers), and the digit's total.
+__global__ void __launch_bounds__(1024) rs_offset_kernel(const uint32_t* __restrict__ cnt, int tiles,
+                                                         uint32_t* __restrict__ off, uint32_t* __restrict__ tot) {
+  __shared__ uint32_t sw[32];
+  __shared__ uint32_t s_run;
+  const int64_t base = ((int64_t)blockIdx.y * 256 + blockIdx.x) * tiles;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  if (threadIdx.x == 0) s_run = 0u;
+  __syncthreads();
+  for (int t0 = 0; t0 < tiles; t0 += blockDim.x) {
+    const int t = t0 + threadIdx.x;
+    const uint32_t c = (t < tiles) ? __ldg(cnt + base + t) : 0u;
+    uint32_t inc = c;
+#pragma unroll
+    for (int dd = 1; dd < 32; dd <<= 1) {
+      const uint32_t o = __shfl_up_sync(0xffffffffu, inc, dd);
+      if (lane >= dd) inc += o;
+    }
+    if (lane == 31) sw[w] = inc;
+    __syncthreads();
+    if (w == 0) {
+      const uint32_t v = (lane < (int)(blockDim.x >> 5)) ? sw[lane] : 0u;
+      uint32_t vi = v;
+#pragma unroll
+      for (int dd = 1; dd < 32; dd <<= 1) {
+        const uint32_t o = __shfl_up_sync(0xffffffffu, vi, dd);
+        if (lane >= dd) vi += o;
+      }
+      sw[lane] = vi - v;  // exclusive prefix of the warp totals
+    }
+    __syncthreads();
+    const uint32_t run = s_run;
+    if (t < tiles) off[base + t] = run + sw[w] + inc - c;
+    __syncthreads();
+    if (threadIdx.x == blockDim.x - 1) s_run = run + sw[w] + inc;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) tot[(int64_t)blockIdx.y * 256 + blockIdx.x] = s_run;
+}
+
+__global__ void __launch_bounds__(kTS) rs_scatter_kernel(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ vin,
+                                                         uint32_t* __restrict__ kout, uint32_t* __restrict__ vout,
+                                                         int64_t n, int shift, int tiles, const uint32_t* __restrict__ off,
+                                                         const uint32_t* __restrict__ tot) {
+  __shared__ uint32_t wc[kTS / 32][256];  // per-warp digit counters -> per-warp prefixes
+  __shared__ uint32_t s_base[256];        // digit base of this tile: smaller digits + earlier tiles
+  __shared__ uint32_t s_start[256];       // digit starts inside the tile
+  __shared__ uint32_t skey[kTile], sval[kTile];
+  __shared__ uint32_t sw[kTS / 32], sw2[kTS / 32];
+  const int f = blockIdx.y, tile = blockIdx.x;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int64_t base = (int64_t)f * n + (int64_t)tile * kTile;
+  const int m = (int)min((int64_t)kTile, n - (int64_t)tile * kTile);
+  for (int q = lane; q < 256; q += 32) wc[w][q] = 0u;
+  // keys of warp w: tile positions w * 256 + j * 32 + lane (coalesced, in tile order)
+  uint32_t keys[kTI], vals[kTI], rk[kTI];
+#pragma unroll
+  for (int j = 0; j < kTI; ++j) {
+    const int i = w * 256 + j * 32 + lane;
+    keys[j] = (i < m) ? __ldg(kin + base + i) : 0u;
+    vals[j] = (i < m) ? __ldg(vin + base + i) : 0u;
+  }
+  __syncwarp();
+  const uint32_t lt = (1u << lane) - 1u;
+#pragma unroll
+  for (int j = 0; j < kTI; ++j) {
+    const int i = w * 256 + j * 32 + lane;
+    const bool v = i < m;
+    const uint32_t dg = v ? ((keys[j] >> shift) & 255u) : 256u;  // padding: its own class
+    const uint32_t peers = __match_any_sync(0xffffffffu, dg);
+    const uint32_t before = wc[w][dg & 255u];
+    rk[j] = before + __popc(peers & lt);
+    __syncwarp();
+    if (v && (peers & lt) == 0u) wc[w][dg] = before + __popc(peers);  // lowest peer updates
+    __syncwarp();
+  }
+  __syncthreads();
+  // thread = digit: exclusive prefix over the warps, the tile's digit starts (exclusive
+  // scan of its digit counts) and the digit's global base for this tile
+  {
+    const int dgt = threadIdx.x;
+    uint32_t run = 0u;
+#pragma unroll
+    for (int q = 0; q < kTS / 32; ++q) {
+      const uint32_t c = wc[q][dgt];
+      wc[q][dgt] = run;
+      run += c;
+    }
+    uint32_t inc = run;  // tile count of this digit
+#pragma unroll
+    for (int dd = 1; dd < 32; dd <<= 1) {
+      const uint32_t o = __shfl_up_sync(0xffffffffu, inc, dd);
+      if (lane >= dd) inc += o;
+    }
+    if (lane == 31) sw[w] = inc;
+    // exclusive prefix of the digit totals of this feature
+    const uint32_t t = __ldg(tot + (int64_t)f * 256 + dgt);
+    uint32_t tinc = t;
+#pragma unroll
+    for (int dd = 1; dd < 32; dd <<= 1) {
+      const uint32_t o = __shfl_up_sync(0xffffffffu, tinc, dd);
+      if (lane >= dd) tinc += o;
+    }
+    if (lane == 31) sw2[w] = tinc;
+    __syncthreads();
+    uint32_t wp = 0u, wp2 = 0u;
+    for (int q = 0; q < w; ++q) { wp += sw[q]; wp2 += sw2[q]; }
+    s_start[dgt] = wp + inc - run;
+    s_base[dgt] = wp2 + tinc - t + __ldg(off + ((int64_t)f * 256 + dgt) * tiles + tile);
+  }
+  __syncthreads();
+  // local (tile-sorted) order in shared memory, then coalesced runs to global memory
+#pragma unroll
+  for (int j = 0; j < kTI; ++j) {
+    const int i = w * 256 + j * 32 + lane;
+    if (i < m) {
+      const uint32_t dg = (keys[j] >> shift) & 255u;
+      const uint32_t lp = s_start[dg] + wc[w][dg] + rk[j];
+      skey[lp] = keys[j];
+      sval[lp] = vals[j];
+    }
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < m; i += kTS) {
+    const uint32_t key = skey[i];
+    const uint32_t dg = (key >> shift) & 255u;
+    const int64_t dst = (int64_t)f * n + s_base[dg] + ((uint32_t)i - s_start[dg]);
+    kout[dst] = key;
+    vout[dst] = sval[i];
+  }
+}
+
 // ----------------------------------------------------------------------------- scan ----
 
 // Appends chunk c to a level's chunk list: single-segment chunks from the front, the
@@ -1927,6 +2085,9 @@ struct FitBufs {
   uint32_t *v_in, *v_out;
   void* sort_tmp;           // d slices of sort_tmp_bytes (one CUB sort per feature)
   size_t sort_tmp_bytes;
+  uint32_t *rs_cnt, *rs_off;  // batched tile sort: per (feature, digit, tile) counts / offsets
+  uint32_t* rs_tot;           // per (feature, digit) totals
+  int rs_tiles;               // tiles per feature (0: per-feature CUB sorts instead)
   ChunkDesc* sdesc;
   uint32_t *slist, *plist;  // per-level chunk lists (scan, partition)
   PartDesc* pdesc;
@@ -1990,11 +2151,19 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, int wor
   DT_CK(get(&b.k_out, (size_t)total0));
   DT_CK(get(&b.v_in, (size_t)total0));
   DT_CK(get(&b.v_out, (size_t)total0));
+  b.rs_tiles = (n <= kTileSortMaxRows) ? (int)((n + kTile - 1) / kTile) : 0;
+  b.rs_cnt = b.rs_off = b.rs_tot = nullptr;
+  if (b.rs_tiles) {
+    DT_CK(get(&b.rs_cnt, (size_t)d * 256 * b.rs_tiles));
+    DT_CK(get(&b.rs_off, (size_t)d * 256 * b.rs_tiles));
+    DT_CK(get(&b.rs_tot, (size_t)d * 256));
+  }
   b.sort_tmp_bytes = 0;
-  DT_CK(cub::DeviceRadixSort::SortPairs(nullptr, b.sort_tmp_bytes, b.k_in, b.k_out, b.v_in, b.v_out,
+  if (!b.rs_tiles) DT_CK(cub::DeviceRadixSort::SortPairs(nullptr, b.sort_tmp_bytes, b.k_in, b.k_out, b.v_in, b.v_out,
                                         n, 0, 32, (cudaStream_t)0));
   b.sort_tmp_bytes = (b.sort_tmp_bytes + 255) & ~(size_t)255;
-  DT_CK(get((char**)&b.sort_tmp, b.sort_tmp_bytes * (size_t)d));
+  if (!b.rs_tiles) DT_CK(get((char**)&b.sort_tmp, b.sort_tmp_bytes * (size_t)d));
+  else b.sort_tmp = nullptr;
   DT_CK(get(&b.sdesc, (size_t)b.max_chunks));
   DT_CK(get(&b.slist, (size_t)b.max_chunks));
   DT_CK(get(&b.plist, (size_t)b.max_chunks));
@@ -2072,28 +2241,50 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     DT_CK(cudaGetLastError());
     // stable 32-bit radix sort of every feature's n keys (4 passes each; ties keep the
     // row order -> (x, row id) order), the d sorts forked over side streams
-    pr = prof_begin(PK_PRESORT_SORT, s, 0);  // CUB kernels: library, not counted
-    {
-      SideStreams& ss = side_streams();
-      DT_CK(cudaEventRecord(ss.fork, s));
-      const int nside = std::min(d, SideStreams::kN);
-      for (int j = 0; j < nside; ++j) DT_CK(cudaStreamWaitEvent(ss.st[j], ss.fork, 0));
-      for (int f = 0; f < d; ++f) {
-        size_t tb = b.sort_tmp_bytes;
-        const int64_t o = (int64_t)f * n;
-        DT_CK(cub::DeviceRadixSort::SortPairs((char*)b.sort_tmp + (size_t)f * b.sort_tmp_bytes, tb,
-                                              b.k_in + o, b.k_out + o, b.v_in + o, b.v_out + o, n, 0, 32,
-                                              ss.st[f % SideStreams::kN]));
+    const uint32_t* sk = b.k_out;  // sorted keys / rows
+    const uint32_t* sv = b.v_out;
+    if (b.rs_tiles) {
+      // batched tile radix sort of all d lists: 4 passes x 3 launches (ping-pong, ends in _in)
+      pr = prof_begin(PK_PRESORT_SORT, s, 12);
+      uint32_t *ki = b.k_in, *ko = b.k_out, *vi = b.v_in, *vo = b.v_out;
+      const dim3 g((unsigned)b.rs_tiles, (unsigned)d);
+      for (int pass = 0; pass < 4; ++pass) {
+        const int shift = 8 * pass;
+        rs_count_kernel<<<g, kTS, 0, s>>>(ki, n, shift, b.rs_tiles, b.rs_cnt);
+        rs_offset_kernel<<<dim3(256, (unsigned)d), std::min(1024, (b.rs_tiles + 31) / 32 * 32), 0, s>>>(
+            b.rs_cnt, b.rs_tiles, b.rs_off, b.rs_tot);
+        rs_scatter_kernel<<<g, kTS, 0, s>>>(ki, vi, ko, vo, n, shift, b.rs_tiles, b.rs_off, b.rs_tot);
+        std::swap(ki, ko);
+        std::swap(vi, vo);
       }
-      for (int j = 0; j < nside; ++j) {
-        DT_CK(cudaEventRecord(ss.join[j], ss.st[j]));
-        DT_CK(cudaStreamWaitEvent(s, ss.join[j], 0));
+      prof_end(pr, s, 4.0 * 24.0 * (double)total0);  // per pass: keys read twice, pairs read + written
+      DT_CK(cudaGetLastError());
+      sk = ki;
+      sv = vi;
+    } else {
+      pr = prof_begin(PK_PRESORT_SORT, s, 0);  // CUB kernels: library, not counted
+      {
+        SideStreams& ss = side_streams();
+        DT_CK(cudaEventRecord(ss.fork, s));
+        const int nside = std::min(d, SideStreams::kN);
+        for (int j = 0; j < nside; ++j) DT_CK(cudaStreamWaitEvent(ss.st[j], ss.fork, 0));
+        for (int f = 0; f < d; ++f) {
+          size_t tb = b.sort_tmp_bytes;
+          const int64_t o = (int64_t)f * n;
+          DT_CK(cub::DeviceRadixSort::SortPairs((char*)b.sort_tmp + (size_t)f * b.sort_tmp_bytes, tb,
+                                                b.k_in + o, b.k_out + o, b.v_in + o, b.v_out + o, n, 0, 32,
+                                                ss.st[f % SideStreams::kN]));
+        }
+        for (int j = 0; j < nside; ++j) {
+          DT_CK(cudaEventRecord(ss.join[j], ss.st[j]));
+          DT_CK(cudaStreamWaitEvent(s, ss.join[j], 0));
+        }
       }
+      prof_end(pr, s, 16.0 * (double)total0 * 4);
     }
-    prof_end(pr, s, 16.0 * (double)total0 * 4);
     const int gb = std::max(1, std::min<int>((int)((total0 + 255) / 256), num_sms() * 8));
     pr = prof_begin(PK_PRESORT_BUILD, s, 1);
-    presort_build_kernel<<<gb, 256, 0, s>>>(b.k_out, b.v_out, y, total0, b.lx[0], b.lr[0], b.ly[0]);
+    presort_build_kernel<<<gb, 256, 0, s>>>(sk, sv, y, total0, b.lx[0], b.lr[0], b.ly[0]);
     prof_end(pr, s, 36.0 * (double)total0);  // (key, val) read, y gathered, 16 B written
     DT_CK(cudaGetLastError());
   }
