@@ -25,7 +25,9 @@ KIND = {
     "piece_pos_kernel": "select", "select_kernel": "select", "number_kernel": "number",
     "goleft_kernel": "goleft", "presort_keys_kernel": "presort_keys",
     "presort_build_kernel": "presort_build", "predict_kernel<true>": "predict",
-    "predict_kernel<false>": "predict",
+    "predict_kernel<false>": "predict", "scan_single_kernel": "scan", "prep_kernel": "goleft",
+    "rs_count_kernel": "presort_sort(cub)", "rs_offset_kernel": "presort_sort(cub)",
+    "rs_scatter_kernel": "presort_sort(cub)", "predict_col_kernel": "predict",
 }
 
 
@@ -85,7 +87,9 @@ def main():
             per_kind[k][0] += b
     region_launches = {"scan": agg.get("scan_kernel", [1])[0],
                        "partition": agg.get("partition_kernel", [1])[0],
-                       "select": agg.get("select_kernel", [1])[0]}
+                       "select": agg.get("select_kernel", [1])[0],
+                       "goleft": agg.get("prep_kernel", [1])[0],
+                       "presort_sort(cub)": 1}
     tpath = os.path.join(os.path.dirname(os.path.abspath(__file__)), "..", "profiles", "traffic.json")
     traffic = json.load(open(tpath)) if os.path.exists(tpath) else {}
     for k, (b, _) in per_kind.items():
