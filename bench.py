@@ -57,6 +57,8 @@ def parse():
     p.add_argument("--e2e-steps", type=int, default=10)
     p.add_argument("--no-extra", action="store_true", help="skip configs[0] LOO and configs[4] grid")
     p.add_argument("--grid-rows", type=int, default=10_000_000, help="configs[4] rows (0 = skip)")
+    p.add_argument("--c3-rows", type=int, default=100_000_000,
+                   help="configs[2] rows (x 32 features, depth 16; 0 = skip)")
     p.add_argument("--sharded-local", type=int, default=0,
                    help="N=1 only: also time a feature-sharded fit with this many thread ranks on the GPU")
     return p.parse_args()
@@ -314,6 +316,66 @@ def extra_configs(args, dev, stream):
     return out
 
 
+def c3_measure(args, world, rank, dev, stream):
+    """BASELINE configs[2]: 100M x 32 (S32, seed 3), max_depth 16, min_samples_leaf 1.
+    N=1: dt_fit on one B200 (~110 GB of HBM: the level lists, double-buffered, hold the
+    presort buffers).  N>1: dt_fit_sharded over NCCL, features split over the ranks (every
+    rank holds the whole table; strong scaling of one fit).  Device-timed with CUDA events
+    on the fit's stream, max over ranks; the first fit (planning + graph capture) is
+    untimed.  One extra profiled fit splits presort / levels."""
+    import torch
+
+    import paper_conf_ipps_metzgd23_b200 as dt
+    n, d, depth = args.c3_rows, 32, 16
+    dt.dt_release_workspace()
+    torch.cuda.empty_cache()
+    X, y = dt.dt_gen_table(3, n, d=d, cnn_pool_bits=22, gpu_pool_bits=12, device=dev)
+    comm = None
+    if world > 1:
+        import torch.distributed as dist
+
+        def bcast(obj):
+            lst = [obj]
+            dist.broadcast_object_list(lst, src=0)
+            return lst[0]
+        comm = dt.dt_comm_init_nccl(rank, world, bcast)
+
+    def fit():
+        if comm is None:
+            return dt.dt_fit(X, y, depth, 1)
+        return dt.dt_fit_sharded(comm, X, y, depth, 1, stream=stream)
+    tree = fit()
+    reps = 3
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier(world)
+    torch.cuda.synchronize()
+    a.record(stream)
+    for _ in range(reps):
+        tree = fit()
+    b.record(stream)
+    torch.cuda.synchronize()
+    t = max_over_ranks(a.elapsed_time(b) / 1e3 / reps, world)
+    # one profiled fit (direct enqueue) for the presort / level split; the cached graph
+    # plan's buffers are released first (the direct path allocates its own)
+    dt.dt_release_workspace()
+    dt.dt_profile_reset()
+    dt.dt_profile_enable(True)
+    fit()
+    dt.dt_profile_enable(False)
+    prof = dt.dt_profile()
+    dt.dt_release_workspace()
+    del X, y
+    torch.cuda.empty_cache()
+    presort = sum(v["ms"] for k, v in prof.items() if k.startswith("presort"))
+    levels = sum(v["ms"] for k, v in prof.items() if not k.startswith("presort"))
+    return {"workload": f"configs[2]: {n} x {d} (S32, seed 3, pools 2^22 x 2^12), max_depth {depth}, min_samples_leaf 1",
+            "mode": "dt_fit (1 GPU)" if world == 1 else f"dt_fit_sharded over NCCL ({world} ranks, features split)",
+            "ms_per_fit": t * 1e3, "split_evals_per_fit": tree.split_evals,
+            "split_evals_per_s": tree.split_evals / t, "tree_nodes": tree.size, "tree_depth": tree.depth,
+            "profiled_fit_ms": {"presort": presort, "levels": levels},
+            "timing": "CUDA events around 3 fits after 1 untimed, max over ranks"}
+
+
 def run_ours(args, world, rank, local):
     import torch
 
@@ -456,6 +518,38 @@ def run_ours(args, world, rank, local):
                             "unit": "GB/s", "frac": pach / peak,
                             "alg_bytes_per_launch": pp["alg_bytes"] / pp["launches"]}}
         del Xdse, out
+        # factored DSE: the full configs[3] cross product, 2^20 CNNs x
+        # 2^10 GPU configs = 2^30 candidates, composed on the fly from the two tables
+        import datagen
+        n_cnn, n_gpu = 1 << 20, 1 << 10
+        cnn, gpu, src = datagen.dse_tables(3 + rank, 0, n_cnn, n_gpu)
+        cnn_d, gpu_d = torch.from_numpy(cnn).to(dev), torch.from_numpy(gpu).to(dev)
+        out = torch.empty(n_cnn * n_gpu, dtype=torch.float64, device=dev)
+        for _ in range(3):
+            dt.dt_predict_dse(tdse, cnn_d, gpu_d, src, out=out)
+        torch.cuda.synchronize()
+        dt.dt_profile_reset()
+        dt.dt_profile_enable(True)
+        a.record(stream)
+        for _ in range(reps):
+            dt.dt_predict_dse(tdse, cnn_d, gpu_d, src, out=out)
+        b.record(stream)
+        torch.cuda.synchronize()
+        dt.dt_profile_enable(False)
+        pp = dt.dt_profile().get("predict")
+        t = a.elapsed_time(b) / 1e3
+        tmax = max_over_ranks(t, world)
+        fpreds = sum_over_ranks(float(n_cnn * n_gpu * reps), world) / tmax
+        fach = pp["alg_bytes"] / (pp["ms"] / 1e3) / 1e9
+        dse["factored"] = {
+            "workload": "configs[3]: 2^20 CNNs x 2^10 GPU configs = 2^30 candidates per rank, "
+                        "composed from the two tables (dt_predict_dse), same tree",
+            "predictions_per_s": fpreds, "ms_per_pass": t / reps * 1e3,
+            "roofline": {"bound": "hbm", "kernel": "predict_dse", "achieved": fach, "peak": peak,
+                         "unit": "GB/s", "frac": fach / peak,
+                         "alg_bytes_per_launch": pp["alg_bytes"] / pp["launches"],
+                         "note": "8 B yhat write per prediction; the traversal is issue-bound"}}
+        del out, cnn_d, gpu_d
 
     # ---- feature-sharded fit across the N ranks (NCCL): one C2 fit split by features
     sharded = None
@@ -471,6 +565,14 @@ def run_ours(args, world, rank, local):
             extra = extra_configs(args, dev, stream)
         except Exception as e:
             extra = {"error": f"{type(e).__name__}: {e}"}
+
+    c3 = None
+    if args.c3_rows > 0:
+        del Xd, yd, Xvd, yvd
+        try:
+            c3 = c3_measure(args, world, rank, dev, stream)
+        except Exception as e:
+            c3 = {"error": f"{type(e).__name__}: {e}"}
 
     # ---- CPU baseline: the oracle on the host (rank 0, N=1 only)
     cpu = None
@@ -489,6 +591,7 @@ def run_ours(args, world, rank, local):
                         "d2h_bytes_per_step": d2h, "steps": args.e2e_steps},
                 "gpu_launches": launches,
                 "roofline": roofline, "cpu_baseline": cpu, "dse": dse, "sharded_fit": sharded, "extra_configs": extra,
+                "c3_fit": c3,
                 "clocks": clk.summary(),
                 "fit": {"split_evals_per_step": evals // args.steps, "tree_nodes": tree.size,
                         "tree_depth": tree.depth, "eval_mape": m["mape"], "eval_r2": m["r2"],

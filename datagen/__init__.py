@@ -178,6 +178,21 @@ def dse_candidates(seed: int, row0: int, n: int, cnn_bits: int = 20, gpu_bits: i
     return _assemble(_cnn_cols(seed, cid), _gpu_cols(seed, gid), False)
 
 
+def dse_tables(seed: int, cnn_row0: int, n_cnn: int, n_gpu: int):
+    """The factors of the DSE cross product (factored predict, include/dt.h
+    dt_predict_dse): CNN pool rows cnn_row0 .. cnn_row0 + n_cnn - 1 (the 10 CNN-side S16
+    columns) and GPU pool rows 0 .. n_gpu - 1 (the 6 GPU-side columns), plus feature_src
+    (S16 column f -> CNN column f for f < 10, GPU column f - 10 as -1 - (f - 10)).
+    Candidate (i, j) composes to dse_candidates(seed, ((cnn_row0 + i) << b) + j, 1, b)
+    for n_gpu == 2^b."""
+    cid = np.arange(cnn_row0, cnn_row0 + n_cnn, dtype=np.uint64)
+    gid = np.arange(n_gpu, dtype=np.uint64)
+    cnn = _assemble(_cnn_cols(seed, cid), _gpu_cols(seed, np.zeros(n_cnn, dtype=np.uint64)), False)[:, :10]
+    gpu = _assemble(_cnn_cols(seed, np.zeros(n_gpu, dtype=np.uint64)), _gpu_cols(seed, gid), False)[:, 10:]
+    src = list(range(10)) + [-1 - g for g in range(6)]
+    return np.ascontiguousarray(cnn), np.ascontiguousarray(gpu), src
+
+
 def holdout_mask(seed: int, n: int):
     """Reading R11: row r is held out for evaluation iff h(seed, r) mod 10 < 3 (~30%)."""
     rows = np.arange(n, dtype=np.uint64)

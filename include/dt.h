@@ -116,6 +116,23 @@ void dt_tree_free(dt_tree* tree);
 dt_status dt_predict(const dt_tree* tree, const float* X_dev, int64_t n, int32_t d,
                      double* yhat_dev, void* stream);
 
+/* dt_predict_dse -- factored design-space exploration (the PM
+ * estimates ONE CNN on n candidate GPUs, T_est = t_dca + n * t_pm):
+ * the candidates are the cross product of a CNN table and a GPU table, never
+ * materialised.  cnn_dev: n_cnn x dc f32 row-major (the CNN-side features of each CNN);
+ * gpu_dev: n_gpu x dg f32 row-major (the GPU-side features of each configuration).
+ * feature_src (HOST, dt_tree_num_features(tree) entries) says where tree feature f comes
+ * from: c >= 0 -> CNN column c, -1 - g -> GPU column g.  Candidate (i, j) is the row
+ * x[f] = feature_src[f] >= 0 ? cnn[i][feature_src[f]] : gpu[j][-1 - feature_src[f]], and
+ * yhat_dev[i * n_gpu + j] (f64, n_cnn * n_gpu entries, CNN-major) is exactly what
+ * dt_predict returns for that row.  1 <= dc, dg <= 128; the GPU table must fit shared
+ * memory (dg * n_gpu * 4 B <= ~220 KB, e.g. 6 x 1024 GPUs); n_gpu < 2^24.  The tree sits
+ * in shared memory when it fits beside the GPU table, else it is read through L1/L2.
+ * Errors: INVALID_ARG (NULL pointers, bad feature_src), TOO_LARGE.  Async on stream. */
+dt_status dt_predict_dse(const dt_tree* tree, const float* cnn_dev, int64_t n_cnn, int32_t dc,
+                         const float* gpu_dev, int64_t n_gpu, int32_t dg,
+                         const int32_t* feature_src, double* yhat_dev, void* stream);
+
 /* ------------------------------------------------------------------ eval ---------- */
 
 /* dt_eval -- MAPE, R^2, adjusted R^2 of yhat against y (Table II).
@@ -218,6 +235,18 @@ int64_t dt_launch_count(void);
 int32_t dt_profile_kinds(void);
 dt_status dt_profile_get(int32_t kind, const char** name, int64_t* launches, double* ms,
                          double* alg_bytes);
+
+/* ------------------------------------------------------------------ memory -------- */
+
+/* Workspace is kept between calls so that repeated fits allocate nothing: the cached
+ * CUDA-graph plan of the last bounded-depth dt_fit (its buffers are ~32 B per training
+ * entry, i.e. 32 * n * d bytes) and the freed blocks of the device's default memory pool
+ * (stream-ordered workspace of the other calls).  dt_release_workspace synchronises the
+ * device, frees the cached plan and trims the pool of the CURRENT device to zero, so that
+ * a following large allocation (e.g. the 100M x 32 fit of BASELINE configs[2], ~110 GB)
+ * can use the whole HBM.  Always safe to call; the next fit re-plans.  Returns DT_OK, or
+ * DT_ERR_CUDA if the device synchronisation fails. */
+dt_status dt_release_workspace(void);
 
 /* ------------------------------------------------------------------ misc ---------- */
 

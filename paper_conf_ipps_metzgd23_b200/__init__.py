@@ -88,6 +88,8 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "dt_tree_truncate": ([P, I32, ctypes.POINTER(P)], ctypes.c_int),
         "dt_predict_eval_depths": ([P, P, P, I64, I32, I32, P, P], ctypes.c_int),
         "dt_importances": ([P, P, P], ctypes.c_int),
+        "dt_release_workspace": ([], ctypes.c_int),
+        "dt_predict_dse": ([P, P, I64, I32, P, I64, I32, P, P, P], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -188,6 +190,23 @@ def dt_predict(tree: Tree, X, out=None, stream=None):
         out = torch.empty(n, dtype=torch.float64, device=X.device)
     op = _dev(out, torch.float64, 1, "out")
     _check(_lib.dt_predict(tree.handle, xp, n, d, op, _stream(stream)))
+    return out
+
+
+def dt_predict_dse(tree: Tree, cnn, gpu, feature_src, out=None, stream=None):
+    """Factored DSE predict (include/dt.h): yhat[i * n_gpu + j] = prediction of CNN row i
+    composed with GPU row j; feature_src[f] = CNN column c >= 0 or -1 - GPU column."""
+    import torch
+    n_cnn, dc = cnn.shape
+    n_gpu, dg = gpu.shape
+    src = (ctypes.c_int32 * len(feature_src))(*[int(v) for v in feature_src])
+    if len(feature_src) != tree.num_features:
+        raise ValueError("feature_src needs one entry per tree feature")
+    if out is None:
+        out = torch.empty(n_cnn * n_gpu, dtype=torch.float64, device=cnn.device)
+    _check(_lib.dt_predict_dse(tree.handle, _dev(cnn, torch.float32, 2, "cnn"), n_cnn, dc,
+                               _dev(gpu, torch.float32, 2, "gpu"), n_gpu, dg, src,
+                               _dev(out, torch.float64, 1, "out"), _stream(stream)))
     return out
 
 
@@ -371,6 +390,11 @@ def dt_fit_sharded(comm: Comm, X, y, max_depth: int = -1, min_samples_leaf: int 
     _check(_lib.dt_fit_sharded(comm.handle, xp, yp, n, d, max_depth, min_samples_leaf,
                                _stream(stream), ctypes.byref(h)))
     return Tree(h)
+
+
+def dt_release_workspace():
+    """Free the cached fit plan and trim the device memory pool (include/dt.h)."""
+    _check(_lib.dt_release_workspace())
 
 
 def version() -> str:

@@ -64,7 +64,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise RuntimeError("nvcc failed")
     tmp = LIB + f".tmp{os.getpid()}"
     subprocess.check_call([NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared",
-                           "-cudart", "static", "-o", tmp, *objs, "-ldl"])
+                           "-cudart", "static", "-Xlinker", "-z,defs", "-o", tmp, *objs, "-ldl", "-lpthread", "-lrt"])
     os.replace(tmp, LIB)
     return LIB
 

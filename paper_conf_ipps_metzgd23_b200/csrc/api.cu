@@ -183,6 +183,20 @@ dt_status dt_predict(const dt_tree* t, const float* X_dev, int64_t n, int32_t d,
   return predict_impl(t, X_dev, n, d, yhat_dev, S(stream));
 }
 
+dt_status dt_predict_dse(const dt_tree* t, const float* cnn_dev, int64_t n_cnn, int32_t dc,
+                         const float* gpu_dev, int64_t n_gpu, int32_t dg, const int32_t* feature_src,
+                         double* yhat_dev, void* stream) {
+  if (!t) return fail(DT_ERR_INVALID_ARG, "dt_predict_dse: tree is NULL");
+  if (n_cnn < 0 || n_gpu < 0) return fail(DT_ERR_INVALID_ARG, "dt_predict_dse: n_cnn, n_gpu must be >= 0");
+  if (n_cnn == 0 || n_gpu == 0) return DT_OK;
+  if (!cnn_dev || !gpu_dev || !yhat_dev || !feature_src)
+    return fail(DT_ERR_INVALID_ARG, "dt_predict_dse: NULL pointer");
+  if (dc < 1 || dg < 1 || dc > 128 || dg > 128) return fail(DT_ERR_INVALID_ARG, "dt_predict_dse: dc, dg in [1, 128]");
+  if (n_gpu >= ((int64_t)1 << 24)) return fail(DT_ERR_TOO_LARGE, "dt_predict_dse: n_gpu >= 2^24");
+  if (n_cnn >= ((int64_t)1 << 62) / n_gpu) return fail(DT_ERR_TOO_LARGE, "dt_predict_dse: n_cnn * n_gpu >= 2^62");
+  return predict_dse_impl(t, cnn_dev, n_cnn, dc, gpu_dev, n_gpu, dg, feature_src, yhat_dev, S(stream));
+}
+
 dt_status dt_eval(const double* y_dev, const double* yhat_dev, int64_t n, int32_t p,
                   void* stream, dt_metrics* out) {
   if (!out) return fail(DT_ERR_INVALID_ARG, "dt_eval: out is NULL");
@@ -277,5 +291,7 @@ dt_status dt_gen_dse(uint64_t seed, int64_t row0, int64_t n, int32_t gpu_bits, f
   if (n == 0) return DT_OK;
   return gen_dse_impl(seed, row0, n, gpu_bits, X_dev, S(stream));
 }
+
+dt_status dt_release_workspace(void) { return release_workspace_impl(); }
 
 }  // extern "C"

@@ -39,6 +39,7 @@ dt_status cuda_fail(cudaError_t e, const char* what, const char* file, int line)
 dt_status tree_upload(dt_tree* t, cudaStream_t s);
 
 // Fit driver (fit.cu).
+dt_status release_workspace_impl();
 dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
                    int64_t min_leaf, cudaStream_t s, dt_tree** out);
 dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64_t n, int32_t dg,
@@ -49,6 +50,8 @@ int comm_world(const dt_comm* c);
 dt_status comm_allgather(dt_comm* c, const void* send, void* recv, size_t bytes, cudaStream_t s);
 dt_status comm_allreduce_or_u32(dt_comm* c, uint32_t* buf, int64_t n, cudaStream_t s);
 // Predict / eval (predict.cu).
+dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, int32_t dc, const float* gpu,
+                           int64_t n_gpu, int32_t dg, const int32_t* src, double* yhat, cudaStream_t s);
 dt_status predict_impl(const dt_tree* t, const float* X, int64_t n, int32_t d, double* yhat,
                        cudaStream_t s);
 dt_status eval_impl(const double* y, const double* yhat, const float* X, const dt_tree* t,

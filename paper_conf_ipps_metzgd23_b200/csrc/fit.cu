@@ -616,11 +616,17 @@ __device__ __forceinline__ void write_stat(Stat* p, const StatP& a) {
 
 // Gain of candidate "first i rows left" (Reading R19), no FMA contraction:
 //   D = S'_L n_R - S'_R n_L,  gain = D^2 / ((N n_L) n_R).
-__device__ __forceinline__ double split_gain(double sl, double sc, uint32_t i, uint32_t N) {
-  const double nl = (double)i, nr = (double)(N - i), Nd = (double)N;
+// nl, Nd: the left count and the node size as doubles (exact integers).  Callers in the
+// per-item loops pass nl = (double)i0 + j (exact), so no int->f64 conversion (an XU-pipe
+// op, the scan's former bottleneck) runs per item; the values are identical.
+__device__ __forceinline__ double split_gain_d(double sl, double sc, double nl, double Nd) {
+  const double nr = __dsub_rn(Nd, nl);
   const double sr = __dsub_rn(sc, sl);
   const double D = __dsub_rn(__dmul_rn(sl, nr), __dmul_rn(sr, nl));
   return __ddiv_rn(__dmul_rn(D, D), __dmul_rn(__dmul_rn(Nd, nl), nr));
+}
+__device__ __forceinline__ double split_gain(double sl, double sc, uint32_t i, uint32_t N) {
+  return split_gain_d(sl, sc, (double)i, (double)N);
 }
 
 // Same D and denominator as split_gain; the quotient via a Newton-refined reciprocal
@@ -633,8 +639,8 @@ __device__ __forceinline__ double rcp_nr(double x) {
   e = __fma_rn(-x, r, 1.0);
   return __fma_rn(r, e, r);
 }
-__device__ __forceinline__ double split_gain_approx(double sl, double sc, uint32_t i, uint32_t N) {
-  const double nl = (double)i, nr = (double)(N - i), Nd = (double)N;
+__device__ __forceinline__ double split_gain_approx_d(double sl, double sc, double nl, double Nd) {
+  const double nr = __dsub_rn(Nd, nl);
   const double sr = __dsub_rn(sc, sl);
   const double D = __dsub_rn(__dmul_rn(sl, nr), __dmul_rn(sr, nl));
   return __dmul_rn(__dmul_rn(D, D), rcp_nr(__dmul_rn(__dmul_rn(Nd, nl), nr)));
@@ -846,9 +852,16 @@ __global__ void __launch_bounds__(1024) chunk_scan_kernel(Ctl* ctl, int parity, 
 // general path (thread sums item by item, Kogge-Stone prefix, carry), so the results are
 // bitwise identical; the per-chunk argmax is a warp max-reduction + lowest winning lane
 // (exact selection, ties to the lowest position like ArgP's combine).
+// Valid split positions of one chunk, compacted (position order) for the exact gains.
+constexpr int kCompactMax = kChunkW;
+struct CompactBuf {
+  double sl[kCompactMax];
+  uint32_t i[kCompactMax];
+};
+
 __device__ __forceinline__ void scan_single(const ScanArgs& a, int64_t ch, int64_t cbase, const ChunkDesc& dsc,
                                             const float* xv, const double* yv, uint32_t m, const SumP& carry,
-                                            float xp0) {
+                                            float xp0, CompactBuf& cb) {
   const int lane = threadIdx.x & 31;
   const bool head = dsc.start == cbase;
   const bool head0 = head && lane == 0;
@@ -866,7 +879,13 @@ __device__ __forceinline__ void scan_single(const ScanArgs& a, int64_t ch, int64
   if (lane == 0) S = 0.0;
   if (!head) S = __dadd_rn(carry.s, S);
 
-  ArgP run{0u, 0xffffffffu, -1.0, 0.0};
+  // Valid positions (x_prev < x, both children >= m) are few on tied data (a column with
+  // V distinct values has < V boundaries per node): the (prefix, position) pairs of the
+  // chunk's valid positions are compacted, in position order, into shared memory and the
+  // EXACT gain of each is computed once, lane q taking entries q, q + 32, .. (strict >
+  // per lane, then a warp (max gain, lowest index) reduction == the lowest position
+  // among the maxima).  On tied data one round of 32 gains covers a whole chunk.
+  ArgP best{0u, 0xffffffffu, -1.0, 0.0};
   if (dsc.srch) {
     const double sc = dsc.sc;
     const uint32_t N = dsc.N;
@@ -874,78 +893,55 @@ __device__ __forceinline__ void scan_single(const ScanArgs& a, int64_t ch, int64
     const uint32_t ilo = m > 1u ? m : 1u, ihi = N - m;
     float xprev = __shfl_up_sync(0xffffffffu, xv[kItems - 1], 1);
     if (lane == 0) xprev = head ? 0.f : xp0;
-    // Argmax without divisions: candidate j's gain is n_j / d_j with n_j = D_j^2 and
-    // d_j = (N n_L) n_R exactly as in split_gain, so g_a < g_b <=> n_a d_b < n_b d_a up to
-    // two roundings (relative 2.2e-16).  A fixed 8 -> 4 -> 2 -> 1 tournament (earlier item
-    // wins unless the later is strictly larger) finds the argmax; a comparison whose two
-    // sides are within kTol flags a near-tie on the winner's path, and then every valid
-    // item's exact gain decides (strict >, in order).  Otherwise only the winner's exact
-    // gain is computed.  Exactly the argmax and gain of the plain per-item loop.
-    constexpr double kTol = 1e-13;  // >> 2 roundings
-    const double Nd = (double)N;
-    double tn[kItems], td[kItems], ts[kItems];
-    int tj[kItems];
-    bool tamb[kItems];
-    double Sj = S;
+    uint32_t vm = 0u;
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
       const uint32_t i = i0 + j;
       const float xp = (j == 0) ? xprev : xv[j - 1];
-      const bool ok = i >= ilo && i <= ihi && xp < xv[j];
-      const double nl = (double)i, nr = __dsub_rn(Nd, nl);
-      const double sr = __dsub_rn(sc, Sj);
-      const double D = __dsub_rn(__dmul_rn(Sj, nr), __dmul_rn(sr, nl));
-      tn[j] = ok ? __dmul_rn(D, D) : -1.0;
-      td[j] = ok ? __dmul_rn(__dmul_rn(Nd, nl), nr) : 1.0;
-      ts[j] = Sj;
-      tj[j] = j;
-      tamb[j] = false;
-      Sj = __dadd_rn(Sj, __dsub_rn(yv[j], c));
+      if (i >= ilo && i <= ihi && xp < xv[j]) vm |= 1u << j;
     }
+    const uint32_t nv = __popc(vm);
+    uint32_t vinc = nv;
 #pragma unroll
-    for (int w = 1; w < kItems; w <<= 1) {
-#pragma unroll
-      for (int q = 0; q < kItems; q += 2 * w) {
-        const double L = __dmul_rn(tn[q], td[q + w]), R = __dmul_rn(tn[q + w], td[q]);
-        const bool bw = R > L;  // the later candidate wins only if strictly larger
-        const double hi = bw ? R : L, lo = bw ? L : R;
-        const bool near = lo >= __dmul_rn(hi, 1.0 - kTol);
-        if (bw) { tn[q] = tn[q + w]; td[q] = td[q + w]; ts[q] = ts[q + w]; tj[q] = tj[q + w]; tamb[q] = tamb[q + w]; }
-        tamb[q] = tamb[q] || near;
-      }
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t o = __shfl_up_sync(0xffffffffu, vinc, d);
+      if (lane >= d) vinc += o;
     }
-    if (tn[0] >= 0.0) {
-      if (!tamb[0]) {
-        const uint32_t i = i0 + (uint32_t)tj[0];
-        run.gain = split_gain(ts[0], sc, i, N);
-        run.i = i;
-        run.sl = ts[0];
-      } else {
-        Sj = S;
+    const uint32_t vtot = __shfl_sync(0xffffffffu, vinc, 31);
+    if (vtot != 0u) {
+      uint32_t q = vinc - nv;
+      double Sj = S;
 #pragma unroll
-        for (int j = 0; j < kItems; ++j) {
-          const uint32_t i = i0 + j;
-          const float xp = (j == 0) ? xprev : xv[j - 1];
-          if (i >= ilo && i <= ihi && xp < xv[j]) {
-            const double g = split_gain(Sj, sc, i, N);
-            if (g > run.gain) { run.gain = g; run.i = i; run.sl = Sj; }
-          }
-          Sj = __dadd_rn(Sj, __dsub_rn(yv[j], c));
+      for (int j = 0; j < kItems; ++j) {
+        if (vm & (1u << j)) {
+          cb.sl[q] = Sj;
+          cb.i[q] = i0 + j;
+          ++q;
         }
+        Sj = __dadd_rn(Sj, __dsub_rn(yv[j], c));
       }
+      __syncwarp();
+      const double Nd = (double)N;
+      double bg = -1.0;
+      uint32_t bq = 0xffffffffu;
+      for (uint32_t e = lane; e < vtot; e += 32) {
+        const double sl = cb.sl[e];
+        const double g = split_gain_d(sl, sc, (double)cb.i[e], Nd);
+        if (g > bg) { bg = g; bq = e; }
+      }
+      // warp max of the gains, then the lowest index holding it (one redux)
+      double g = bg;
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) g = fmax(g, __shfl_xor_sync(0xffffffffu, g, off));
+      bq = __reduce_min_sync(0xffffffffu, bg == g ? bq : 0xffffffffu);
+      best = ArgP{0u, cb.i[bq], g, cb.sl[bq]};  // bq < vtot: gains are >= 0 > -1
+      __syncwarp();  // the buffer is rewritten by the next chunk
     }
   }
-  double g = run.gain;
-#pragma unroll
-  for (int off = 16; off > 0; off >>= 1) g = fmax(g, __shfl_xor_sync(0xffffffffu, g, off));
-  const uint32_t win = __ballot_sync(0xffffffffu, run.gain == g);
-  const int src = win ? __ffs(win) - 1 : 0;
-  const uint32_t bi = __shfl_sync(0xffffffffu, run.i, src);
-  const double bsl = __shfl_sync(0xffffffffu, run.sl, src);
-  const uint32_t kf = dsc.k * a.d + dsc.f;
-  const double bg = __shfl_sync(0xffffffffu, run.gain, src);
-  if (lane == 0) write_cand(head ? a.head_cand + kf : a.cont_cand + ch, ArgP{0u, bi, bg, bsl}, kf, a.level,
-                            a.slot_gain);
+  if (lane == 0) {
+    const uint32_t kf = dsc.k * a.d + dsc.f;
+    write_cand(head ? a.head_cand + kf : a.cont_cand + ch, best, kf, a.level, a.slot_gain);
+  }
   // node statistics from the feature-0 list (same scan as the general path)
   if (dsc.f == 0) {
     const double v = dsc.v;
@@ -997,6 +993,8 @@ __global__ void __launch_bounds__(kThreads, 2) scan_single_kernel(ScanArgs a) {
   ScanStage* st = reinterpret_cast<ScanStage*>(scan_smem) + wib * kScanStages;
   uint64_t* bar = reinterpret_cast<uint64_t*>(scan_smem + sizeof(ScanStage) * kScanStages * (kThreads / 32)) +
                   wib * kScanStages;
+  CompactBuf* cbuf = reinterpret_cast<CompactBuf*>(scan_smem + (sizeof(ScanStage) + sizeof(uint64_t)) * kScanStages *
+                                                                   (kThreads / 32));
   auto issue = [&](int s, int64_t ch) {  // lane 0
     ScanStage& t = st[s];
     t.ch = (uint32_t)ch;
@@ -1047,11 +1045,12 @@ __global__ void __launch_bounds__(kThreads, 2) scan_single_kernel(ScanArgs a) {
     const float xp0 = t.xp[3];
     __syncwarp();  // every lane has read the stage
     if (lane == 0 && nxt < ns) issue(s, (int64_t)ch_ahead);
-    scan_single(a, ch, ch * kChunkW, dsc, xv, yv, m, carry, xp0);
+    scan_single(a, ch, ch * kChunkW, dsc, xv, yv, m, carry, xp0, cbuf[wib]);
     if (++s == kScanStages) { s = 0; phase ^= 1u; }
   }
 }
-constexpr size_t kScanSingleSmem = (sizeof(ScanStage) + sizeof(uint64_t)) * kScanStages * (kThreads / 32);
+constexpr size_t kScanSingleSmem =
+    (sizeof(ScanStage) + sizeof(uint64_t)) * kScanStages * (kThreads / 32) + sizeof(CompactBuf) * (kThreads / 32);
 
 // Phase C: the main scan (prefixes, gains, per-piece argmax, node statistics), one warp
 // chunk at a time per warp, no block barriers.
@@ -1134,6 +1133,7 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
         const uint32_t i0 = (uint32_t)(p0 - sg.start);
         const uint32_t ilo = m > 1u ? m : 1u, ihi = N - m;
         const float xprev = head0 ? 0.f : a.lx[p0 - 1];
+        const double Nd = (double)N, nl0 = (double)i0;
         // loop 1: approximate gains (exact D and denominator, reciprocal by Newton)
         double Sj = S, bapx = -1.0, bS = 0.0;
         int bj = -1;
@@ -1144,7 +1144,7 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
           const uint32_t i = i0 + j;
           const float xp = (j == 0) ? xprev : xv[j - 1];
           if (i >= ilo && i <= ihi && xp < xv[j]) {
-            const double g = split_gain_approx(Sj, sc, i, N);
+            const double g = split_gain_approx_d(Sj, sc, __dadd_rn(nl0, (double)j), Nd);
             if (g > bapx) {
               if (bapx >= __dmul_rn(g, 1.0 - kTol)) amb = true;
               bapx = g; bS = Sj; bj = j;
@@ -1157,7 +1157,7 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
         if (bj >= 0 && !amb) {
           // the exact argmax is the approximate one: exact gain of that position only
           const uint32_t i = i0 + (uint32_t)bj;
-          run.gain = split_gain(bS, sc, i, N);
+          run.gain = split_gain_d(bS, sc, __dadd_rn(nl0, (double)bj), Nd);
           run.i = i;
           run.sl = bS;
         } else if (bj >= 0) {
@@ -1168,7 +1168,7 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
             const uint32_t i = i0 + j;
             const float xp = (j == 0) ? xprev : xv[j - 1];
             if (i >= ilo && i <= ihi && xp < xv[j]) {
-              const double g = split_gain(Sj, sc, i, N);
+              const double g = split_gain_d(Sj, sc, __dadd_rn(nl0, (double)j), Nd);
               if (g > run.gain) { run.gain = g; run.i = i; run.sl = Sj; }
             }
             Sj = __dadd_rn(Sj, __dsub_rn(yv[j], c));
@@ -2083,7 +2083,7 @@ struct FitBufs {
   double* cparts;
   uint32_t *k_in, *k_out;  // per feature: n keys flip(x), stable-sorted feature by feature
   uint32_t *v_in, *v_out;
-  void* sort_tmp;           // d slices of sort_tmp_bytes (one CUB sort per feature)
+  void* sort_tmp;           // min(d, kSideStreams) slices of sort_tmp_bytes (CUB path)
   size_t sort_tmp_bytes;
   uint32_t *rs_cnt, *rs_off;  // batched tile sort: per (feature, digit, tile) counts / offsets
   uint32_t* rs_tot;           // per (feature, digit) totals
@@ -2103,6 +2103,8 @@ struct ShardCtx {
   dt_comm* comm;
   int world, rank, dg;
 };
+
+constexpr int kSideStreams = 8;  // side streams of the forked per-feature sorts
 
 // Allocates every buffer through `get` (stream-ordered or persistent).
 template <class Get>
@@ -2147,10 +2149,13 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, int wor
   DT_CK(get(&b.lvlog, (size_t)kMaxLogLevels));
   DT_CK(get(&b.parts, (size_t)b.root_np));
   DT_CK(get(&b.cparts, (size_t)b.root_np));
-  DT_CK(get(&b.k_in, (size_t)total0));
-  DT_CK(get(&b.k_out, (size_t)total0));
-  DT_CK(get(&b.v_in, (size_t)total0));
-  DT_CK(get(&b.v_out, (size_t)total0));
+  // the presort's key / row buffers live in the level-1 lists (16 B per entry = exactly
+  // the four 4-B arrays): they are dead once presort_build has written the level-0 lists,
+  // before level 0's partition first writes lists[1].  Saves 16 B per entry (C3: 51 GB).
+  b.k_in = reinterpret_cast<uint32_t*>(b.lx[1]);
+  b.k_out = b.lr[1];
+  b.v_in = reinterpret_cast<uint32_t*>(b.ly[1]);
+  b.v_out = reinterpret_cast<uint32_t*>(b.ly[1]) + total0;
   b.rs_tiles = (n <= kTileSortMaxRows) ? (int)((n + kTile - 1) / kTile) : 0;
   b.rs_cnt = b.rs_off = b.rs_tot = nullptr;
   if (b.rs_tiles) {
@@ -2162,7 +2167,8 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, int wor
   if (!b.rs_tiles) DT_CK(cub::DeviceRadixSort::SortPairs(nullptr, b.sort_tmp_bytes, b.k_in, b.k_out, b.v_in, b.v_out,
                                         n, 0, 32, (cudaStream_t)0));
   b.sort_tmp_bytes = (b.sort_tmp_bytes + 255) & ~(size_t)255;
-  if (!b.rs_tiles) DT_CK(get((char**)&b.sort_tmp, b.sort_tmp_bytes * (size_t)d));
+  // one temp slice per side stream: sorts that share a stream run one after another
+  if (!b.rs_tiles) DT_CK(get((char**)&b.sort_tmp, b.sort_tmp_bytes * (size_t)std::min(d, kSideStreams)));
   else b.sort_tmp = nullptr;
   DT_CK(get(&b.sdesc, (size_t)b.max_chunks));
   DT_CK(get(&b.slist, (size_t)b.max_chunks));
@@ -2184,7 +2190,7 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, int wor
 
 // Per-host-thread pool of side streams for the forked per-feature sorts.
 struct SideStreams {
-  static constexpr int kN = 8;
+  static constexpr int kN = kSideStreams;
   cudaStream_t st[kN];
   cudaEvent_t fork, join[kN];
   SideStreams() {
@@ -2271,7 +2277,7 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
         for (int f = 0; f < d; ++f) {
           size_t tb = b.sort_tmp_bytes;
           const int64_t o = (int64_t)f * n;
-          DT_CK(cub::DeviceRadixSort::SortPairs((char*)b.sort_tmp + (size_t)f * b.sort_tmp_bytes, tb,
+          DT_CK(cub::DeviceRadixSort::SortPairs((char*)b.sort_tmp + (size_t)(f % SideStreams::kN) * b.sort_tmp_bytes, tb,
                                                 b.k_in + o, b.k_out + o, b.v_in + o, b.v_out + o, n, 0, 32,
                                                 ss.st[f % SideStreams::kN]));
         }
@@ -2564,6 +2570,20 @@ std::mutex g_plan_mu;
 std::unique_ptr<FitPlan> g_plan;
 
 }  // namespace
+
+dt_status release_workspace_impl() {
+  {
+    std::lock_guard<std::mutex> lk(g_plan_mu);
+    g_plan.reset();
+  }
+  DT_CK(cudaDeviceSynchronize());
+  int dev = 0;
+  DT_CK(cudaGetDevice(&dev));
+  cudaMemPool_t pool;
+  DT_CK(cudaDeviceGetDefaultMemPool(&pool, dev));
+  DT_CK(cudaMemPoolTrimTo(pool, 0));
+  return DT_OK;
+}
 
 dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
                    int64_t min_leaf, cudaStream_t s, dt_tree** out) {

@@ -482,7 +482,111 @@ __global__ void __launch_bounds__(256) importances_kernel(const dt_node* __restr
     for (int f = threadIdx.x; f < d; f += blockDim.x) imp[f] = imp[f] / tot_sh;
 }
 
+
+// ------------------------------------------------------- factored DSE predict (NEXT-3) --
+
+// The paper's design-space exploration estimates one CNN on n GPU configurations
+// (T_est = t_dca + n * t_pm): candidate (i, j) = CNN row i composed with
+// GPU row j, never materialised.  A CTA keeps the tree (features re-encoded: 0x80 | g =
+// GPU column g, c = CNN column c), the transposed GPU table (thread j reads column
+// entries j: conflict-free) and kR CNN rows in shared memory; thread j walks kR
+// candidates (i0 + r, j) at once (independent chains) and writes yhat[(i0 + r) * n_gpu + j]
+// (coalesced).  Output-write bound: 8 B per prediction (the inputs are O(n_cnn + n_gpu)).
+struct DseMap {
+  uint8_t code[256];  // tree feature f -> 0x80 | GPU column, or CNN column
+};
+
+template <bool kSmemTree, int kR>
+__global__ void __launch_bounds__(1024, 1)
+predict_dse_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ value, int count, int depth,
+                   const float* __restrict__ cnn, int64_t n_cnn, int dc, const float* __restrict__ gpu,
+                   int n_gpu, int dg, DseMap map, double* __restrict__ yhat) {
+  extern __shared__ __align__(16) unsigned char dse_smem[];
+  uint2* snodes = reinterpret_cast<uint2*>(dse_smem);
+  float* gpu_t = reinterpret_cast<float*>(dse_smem + (kSmemTree ? sizeof(uint2) * (size_t)count : 0));
+  float* cnn_s = gpu_t + (size_t)dg * n_gpu;
+  const int tid = threadIdx.x;
+  if (kSmemTree) {
+    for (int k = tid; k < count; k += blockDim.x) {
+      uint2 nd = gnodes[k];
+      nd.y = ((uint32_t)map.code[nd.y >> 24] << 24) | (nd.y & 0xFFFFFFu);
+      snodes[k] = nd;
+    }
+  }
+  for (int e = tid; e < dg * n_gpu; e += blockDim.x) {
+    const int g = e / n_gpu, j = e - g * n_gpu;
+    gpu_t[e] = __ldg(gpu + (int64_t)j * dg + g);
+  }
+  const int64_t nblk = (n_cnn + kR - 1) / kR;
+  for (int64_t b = blockIdx.x; b < nblk; b += gridDim.x) {
+    const int64_t i0 = b * kR;
+    __syncthreads();  // previous CNN rows consumed (and the tables above written)
+    for (int e = tid; e < kR * dc; e += blockDim.x) {
+      const int r = e / dc;
+      cnn_s[e] = (i0 + r < n_cnn) ? __ldg(cnn + (i0 + r) * dc + (e - r * dc)) : 0.f;
+    }
+    __syncthreads();
+    for (int j = tid; j < n_gpu; j += blockDim.x) {
+      uint32_t k[kR];
+#pragma unroll
+      for (int r = 0; r < kR; ++r) k[r] = 0;
+      for (int l = 0; l < depth; ++l) {
+#pragma unroll
+        for (int r = 0; r < kR; ++r) {
+          uint2 nd;
+          if (kSmemTree) {
+            nd = snodes[k[r]];
+          } else {
+            nd = __ldg(gnodes + k[r]);
+            nd.y = ((uint32_t)map.code[nd.y >> 24] << 24) | (nd.y & 0xFFFFFFu);
+          }
+          const uint32_t code = nd.y >> 24, left = nd.y & 0xFFFFFFu;
+          const float* src = (code & 0x80u) ? gpu_t + (code & 0x7Fu) * (uint32_t)n_gpu + j
+                                            : cnn_s + r * dc + code;
+          // go left iff !(x > RD32(t)) (Reading R5); leaves self-loop
+          k[r] = (*src > __uint_as_float(nd.x)) ? left + 1 : left;
+        }
+      }
+#pragma unroll
+      for (int r = 0; r < kR; ++r)
+        if (i0 + r < n_cnn) yhat[(i0 + r) * (int64_t)n_gpu + j] = __ldg(value + k[r]);
+    }
+  }
+}
+
 }  // namespace
+
+dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, int32_t dc, const float* gpu,
+                           int64_t n_gpu, int32_t dg, const int32_t* src, double* yhat, cudaStream_t s) {
+  DseMap map{};
+  for (int f = 0; f < t->d; ++f) {
+    if (src[f] >= 0) {
+      if (src[f] >= dc) return fail(DT_ERR_INVALID_ARG, "dt_predict_dse: bad CNN column in feature_src");
+      map.code[f] = (uint8_t)src[f];
+    } else {
+      const int g = -1 - src[f];
+      if (g >= dg) return fail(DT_ERR_INVALID_ARG, "dt_predict_dse: bad GPU column in feature_src");
+      map.code[f] = (uint8_t)(0x80 | g);
+    }
+  }
+  constexpr int kR = 2, kThr = 1024;
+  const size_t tables = sizeof(float) * ((size_t)dg * (size_t)n_gpu + (size_t)kR * dc);
+  const size_t tree = sizeof(uint2) * (size_t)t->count;
+  const size_t cap = 227 * 1024;
+  if (tables > cap) return fail(DT_ERR_TOO_LARGE, "dt_predict_dse: GPU table too large for shared memory");
+  const bool smem_tree = tree + tables <= cap;
+  const size_t sm = (smem_tree ? tree : 0) + tables;
+  auto kern = smem_tree ? predict_dse_kernel<true, kR> : predict_dse_kernel<false, kR>;
+  DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+  const int64_t nblk = (n_cnn + kR - 1) / kR;
+  const int64_t g = std::min<int64_t>((int64_t)num_sms(), nblk);
+  const int pr = prof_begin(PK_PREDICT, s, 1);
+  kern<<<(unsigned)g, kThr, sm, s>>>(t->dev_packed, t->dev_value, (int)t->count, t->depth, cnn, n_cnn, dc, gpu,
+                                     (int)n_gpu, dg, map, yhat);
+  prof_end(pr, s, 8.0 * (double)n_cnn * (double)n_gpu);  // the yhat write (inputs are O(n_cnn + n_gpu))
+  DT_CK(cudaGetLastError());
+  return DT_OK;
+}
 
 dt_status importances_impl(const dt_tree* t, double* imp_host, cudaStream_t s) {
   dt_node* dn = nullptr;

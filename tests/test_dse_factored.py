@@ -1,0 +1,104 @@
+"""Factored DSE predict (T_est = t_dca + n * t_pm):
+candidate (i, j) = CNN row i composed with GPU row j, never materialised.
+
+The oracle side is the plain definition: compose every candidate row explicitly and
+predict it with oracle.predict (the CPU tree walk).  Predictions from the same tree must
+be bit-exact (BASELINE.json contract).
+"""
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+
+
+def test_dse_tables_compose_to_candidates():
+    """The factor tables are the shared recipe's cross product (no GPU)."""
+    cnn, gpu, src = datagen.dse_tables(3, 5, 7, 16)
+    X = datagen.dse_candidates(3, 5 << 4, 7 << 4, gpu_bits=4)
+    comp = np.concatenate([np.repeat(cnn, 16, axis=0), np.tile(gpu, (7, 1))], axis=1)
+    assert np.array_equal(comp, X)
+    assert src == list(range(10)) + [-1, -2, -3, -4, -5, -6]
+
+
+def _compose(cnn, gpu, src):
+    n_cnn, n_gpu = len(cnn), len(gpu)
+    X = np.empty((n_cnn * n_gpu, len(src)), dtype=np.float32)
+    for f, c in enumerate(src):
+        X[:, f] = np.repeat(cnn[:, c], n_gpu) if c >= 0 else np.tile(gpu[:, -1 - c], n_cnn)
+    return X
+
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def dt():
+    import paper_conf_ipps_metzgd23_b200 as m
+    return m
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("n_cnn,n_gpu,D,m", [(1, 1, 3, 1), (7, 1024, 20, 128), (33, 37, 12, 1),
+                                           (256, 1000, 8, 4)])
+def test_predict_dse_matches_oracle(dt, n_cnn, n_gpu, D, m):
+    X, y = datagen.cnn_gpu_table(1, 50_000)
+    nodes = oracle.fit(X, y, D, m)
+    tree = dt.dt_tree_from_nodes(nodes, 16)
+    cnn, gpu, src = datagen.dse_tables(3, 11, n_cnn, n_gpu)
+    out = dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), torch.from_numpy(gpu).cuda(), src)
+    want = oracle.predict(nodes, _compose(cnn, gpu, src))
+    assert np.array_equal(out.cpu().numpy(), want)
+
+
+@pytest.mark.gpu
+def test_predict_dse_interleaved_columns_and_global_tree(dt):
+    """Arbitrary feature_src (CNN and GPU columns interleaved, one column used twice) and
+    a tree too large for shared memory beside the GPU table (read through L1/L2)."""
+    rng = np.random.default_rng(4)
+    n = 120_000
+    X = rng.integers(0, 1000, size=(n, 6)).astype(np.float32)
+    y = np.floor(rng.random(n) * 1e6)
+    nodes = oracle.fit(X, y, -1, 1)
+    assert len(nodes) * 8 > 227 * 1024  # forces the global-tree path
+    tree = dt.dt_tree_from_nodes(nodes, 6)
+    cnn = rng.integers(0, 1000, size=(5, 3)).astype(np.float32)
+    gpu = rng.integers(0, 1000, size=(4000, 4)).astype(np.float32)
+    src = [-3, 0, -1, 2, 0, -4]
+    out = dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), torch.from_numpy(gpu).cuda(), src)
+    assert np.array_equal(out.cpu().numpy(), oracle.predict(nodes, _compose(cnn, gpu, src)))
+    # the same candidates through dt_predict (materialised rows)
+    Xc = torch.from_numpy(_compose(cnn, gpu, src)).cuda()
+    assert torch.equal(dt.dt_predict(tree, Xc), out)
+
+
+@pytest.mark.gpu
+def test_predict_dse_bench_size_sampled(dt):
+    """bench.py's factored line: 2^20 CNNs x 2^10 GPUs (BASELINE configs[3]) on the
+    depth-20 / min_samples_leaf-128 tree; sampled CNN rows checked bit for bit."""
+    X, y = dt.dt_gen_table(1, 1_000_000, d=16, device="cuda")
+    tree = dt.dt_fit(X, y, 20, 128)
+    n_cnn, n_gpu = 1 << 20, 1 << 10
+    cnn, gpu, src = datagen.dse_tables(3, 0, n_cnn, n_gpu)
+    out = dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), torch.from_numpy(gpu).cuda(), src)
+    torch.cuda.synchronize()
+    rows = np.unique(np.concatenate([[0, 1, n_cnn - 1], np.random.default_rng(2).integers(0, n_cnn, 40)]))
+    for i in rows:
+        want = oracle.predict(tree.nodes, _compose(cnn[i:i + 1], gpu, src))
+        assert np.array_equal(out[i * n_gpu:(i + 1) * n_gpu].cpu().numpy(), want), i
+    del out
+    torch.cuda.empty_cache()
+
+
+@pytest.mark.gpu
+def test_predict_dse_rejects_bad_args(dt):
+    X, y = datagen.cnn_gpu_table(1, 1000)
+    tree = dt.dt_tree_from_nodes(oracle.fit(X, y, 3, 1), 16)
+    cnn, gpu, src = datagen.dse_tables(3, 0, 2, 4)
+    bad = list(src)
+    bad[0] = 10  # CNN column out of range
+    with pytest.raises(dt.DTError):
+        dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), torch.from_numpy(gpu).cuda(), bad)
+    big = torch.zeros((1 << 16, 6), dtype=torch.float32, device="cuda")  # 1.5 MB table
+    with pytest.raises(dt.DTError):
+        dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), big, src)

@@ -1,0 +1,134 @@
+"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py times.
+
+The oracle cannot fit 100M x 32 (hours single-threaded), so at full size the GPU result
+is checked ("sampled outputs ... else via properties that hold at any size"):
+
+* properties of the whole node array that hold at any size: BFS links, child counts sum
+  to the parent's, the parent's value is the count-weighted mean of its children's, leaf
+  counts sum to n, depth <= max_depth, the root value equals the fp64 mean of y;
+* sampled nodes, one by one: the rows that reach a node are gathered (kept in row order)
+  and the oracle fits a depth-1 tree on exactly those rows; in integer mode (the
+  generator's integer-microsecond targets) its split feature, threshold, child counts
+  and value must equal the node's bit for bit (greedy CART decides every node from its
+  own rows only, Readings R4/R8);
+* DSE prediction (configs[3] shape on one GPU, 2^28 candidates, depth-20 tree): sampled
+  candidates predicted by the oracle must match bit for bit.
+"""
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def dt():
+    import paper_conf_ipps_metzgd23_b200 as m
+    return m
+
+
+def _check_array(nodes, n, max_depth):
+    feat, left, right = nodes["feature"], nodes["left"], nodes["right"]
+    cnt, val, dep = nodes["n_samples"], nodes["value"], nodes["depth"]
+    assert cnt[0] == n
+    internal = feat >= 0
+    assert np.all(right[internal] == left[internal] + 1)
+    assert np.all(left[~internal] == -1)
+    li, ri = left[internal], right[internal]
+    assert np.all(li > np.nonzero(internal)[0])  # BFS: children after the parent
+    assert np.array_equal(cnt[li] + cnt[ri], cnt[internal])
+    assert np.all(dep[li] == dep[internal] + 1)
+    wmean = (val[li] * cnt[li] + val[ri] * cnt[ri]) / cnt[internal]
+    np.testing.assert_allclose(wmean, val[internal], rtol=1e-9, atol=1e-12)
+    assert cnt[~internal].sum() == n
+    assert dep.max() <= max_depth
+
+
+def _route(nodes, X, depth):
+    """Node index of every row after `depth` steps down the tree (torch on the GPU: test
+    infrastructure; leaves keep their rows)."""
+    feat = torch.from_numpy(nodes["feature"].astype(np.int64)).cuda()
+    thr = torch.from_numpy(nodes["threshold"]).cuda()
+    left = torch.from_numpy(nodes["left"].astype(np.int64)).cuda()
+    node = torch.zeros(X.shape[0], dtype=torch.int64, device=X.device)
+    for _ in range(depth):
+        f = feat[node]
+        internal = f >= 0
+        x = torch.gather(X, 1, f.clamp(min=0).unsqueeze(1)).squeeze(1).double()
+        child = left[node] + (x > thr[node]).long()
+        node = torch.where(internal, child, node)
+    return node
+
+
+def _sampled_nodes(nodes, lo, hi, k, rng):
+    internal = np.nonzero((nodes["feature"] >= 0) & (nodes["n_samples"] >= lo) & (nodes["n_samples"] <= hi))[0]
+    assert len(internal) > 0
+    deep = sorted(internal, key=lambda i: -int(nodes["depth"][i]))[: max(1, k // 2)]
+    rest = rng.choice(internal, size=min(k - len(deep), len(internal)), replace=False)
+    return sorted(set(int(i) for i in list(deep) + list(rest)))
+
+
+def test_fit_c3_full_size(dt):
+    """BASELINE configs[2] at full size on one B200: 100M x 32 (S32, seed 3, pools 2^22 CNNs x
+    2^12 GPUs), depth 16."""
+    n, d, D = 100_000_000, 32, 16
+    dt.dt_release_workspace()
+    torch.cuda.empty_cache()
+    X, y = dt.dt_gen_table(3, n, d=d, cnn_pool_bits=22, gpu_pool_bits=12, device="cuda")
+    # the device generator is the shared input recipe: spot-check rows against datagen
+    for r0 in (0, n // 2 + 17, n - 1000):
+        Xh, yh = datagen.cnn_gpu_table(3, 1000, d=d, row0=r0, cnn_pool_bits=22, gpu_pool_bits=12)
+        assert np.array_equal(X[r0:r0 + 1000].cpu().numpy(), Xh)
+        assert np.array_equal(y[r0:r0 + 1000].cpu().numpy(), yh)
+    tree = dt.dt_fit(X, y, D, 1)
+    torch.cuda.synchronize()
+    dt.dt_release_workspace()
+    nodes = tree.nodes
+    _check_array(nodes, n, D)
+    mean = float(y.sum().item()) / n
+    assert abs(nodes["value"][0] - mean) <= 1e-9 * abs(mean)
+    # integer mode (Reading R17): integral targets, max|y| * n < 2^52
+    assert bool((torch.floor(y) == y).all()) and float(y.abs().max()) * n < 2.0 ** 52
+    rng = np.random.default_rng(0)
+    picks = _sampled_nodes(nodes, 2000, 400_000, 6, rng)
+    for k in picks:
+        at = _route(nodes, X, int(nodes["depth"][k]))
+        idx = torch.nonzero(at == k).squeeze(1)  # ascending row order
+        assert idx.numel() == nodes["n_samples"][k]
+        Xs, ys = X[idx].cpu().numpy(), y[idx].cpu().numpy()
+        o = oracle.fit(Xs, ys, 1, 1)
+        L = nodes["left"][k]
+        assert o["feature"][0] == nodes["feature"][k], k
+        assert o["threshold"][0] == nodes["threshold"][k], k
+        assert o["value"][0] == nodes["value"][k], k
+        assert o["n_samples"][1] == nodes["n_samples"][L], k
+        assert o["n_samples"][2] == nodes["n_samples"][L + 1], k
+    del X, y
+    torch.cuda.empty_cache()
+
+
+def test_dse_predict_bench_size_sampled(dt):
+    """bench.py's DSE line: 2^28 candidates (configs[3] shape on one GPU) on the depth-20,
+    min_samples_leaf-128 tree fitted on the configs[1] table; sampled predictions must
+    equal the oracle's bit for bit."""
+    dt.dt_release_workspace()
+    torch.cuda.empty_cache()
+    X, y = dt.dt_gen_table(1, 1_000_000, d=16, device="cuda")
+    tree = dt.dt_fit(X, y, 20, 128)
+    nd = 1 << 28
+    Xd = dt.dt_gen_dse(3, 0, nd, 10, device="cuda")
+    out = dt.dt_predict(tree, Xd)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(1)
+    idx = np.unique(np.concatenate([rng.integers(0, nd, 200_000), np.arange(1000), np.arange(nd - 1000, nd)]))
+    ti = torch.from_numpy(idx).cuda()
+    Xs = Xd[ti].cpu().numpy()
+    # the candidates are the shared recipe's rows
+    Xr = datagen.dse_candidates(3, 0, 1000)
+    assert np.array_equal(Xs[:1000], Xr)
+    assert np.array_equal(out[ti].cpu().numpy(), oracle.predict(tree.nodes, Xs))
+    del Xd, out
+    torch.cuda.empty_cache()

@@ -8,7 +8,7 @@ TESTS=${2:-1}
 mkdir -p gpurun_out
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,memory.total --format=csv > gpurun_out/${TAG}_smi.txt 2>&1
 if [ "$TESTS" = 1 ]; then
-  timeout 1500 python -m pytest tests -x -q -m gpu > gpurun_out/${TAG}_pytest_gpu.log 2>&1
+  timeout 1500 python -m pytest tests -q -m gpu > gpurun_out/${TAG}_pytest_gpu.log 2>&1
   echo "pytest exit $?" >> gpurun_out/${TAG}_pytest_gpu.log
   timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TAG}_smoke.log 2>&1
   echo "smoke exit $?" >> gpurun_out/${TAG}_smoke.log
@@ -21,6 +21,9 @@ timeout 600 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__byte
 echo "ncu launch exit $?" >> gpurun_out/${TAG}_ncu_launch.log
 timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base function \
   -k regex:'^(scan_kernel|scan_single_kernel|partition_kernel|part_agg_kernel|scan_agg_kernel|predict_col_kernel|rs_scatter_kernel)$' \
-  --launch-count 40 -o gpurun_out/${TAG}_full -f \
+  --launch-count 12 -o /tmp/${TAG}_full -f \
   python bench.py --steps 1 --warmup 0 --no-cpu --no-extra --e2e-steps 0 --dse-log2 24 > gpurun_out/${TAG}_ncu_full.log 2>&1
 echo "ncu full exit $?" >> gpurun_out/${TAG}_ncu_full.log
+ncu -i /tmp/${TAG}_full.ncu-rep --page raw --csv > gpurun_out/${TAG}_full_raw.csv 2>/dev/null
+ncu -i /tmp/${TAG}_full.ncu-rep --page details --csv > gpurun_out/${TAG}_full_details.csv 2>/dev/null
+ls -la /tmp/${TAG}_full.ncu-rep >> gpurun_out/${TAG}_ncu_full.log
