@@ -1427,6 +1427,94 @@ __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
     a.log[a.level].A_next = 0;
     a.log[a.level].K_next = 0;
   }
+  if (K > gridDim.x) {
+    // Many (small) nodes: one warp per node, no block barriers.  Same per-feature bests;
+    // node statistics by a fixed-shape warp reduction (contiguous runs of pieces per lane,
+    // then an xor tree); the feature argmax keeps the lowest feature among equal gains.
+    const int nwarps = blockDim.x >> 5;
+    for (uint32_t k = blockIdx.x * nwarps + w; k < K; k += gridDim.x * nwarps) {
+      const NodeL nd = a.nodes[k];
+      double bg = -1.0, bsl = 0.0;
+      uint32_t bi = 0xffffffffu;
+      int bf = 0x7fffffff;
+      for (int f = lane; f < a.d; f += 32) {
+        const uint32_t kf = k * a.d + f;
+        if (nd.searchable && f < a.dl && nd.N > 1) {
+          const uint32_t pos = a.slot_pos[kf];
+          if (pos != 0xffffffffu) {
+            const double g = __longlong_as_double((long long)a.slot_gain[kf]);
+            if (g > bg) {  // strict >: the lowest of this lane's features wins ties
+              const int64_t s0 = (int64_t)f * (int64_t)A + nd.start;
+              const int64_t t0 = s0 / kChunkW, c = (s0 + pos) / kChunkW;
+              bsl = ((c == t0) ? a.head_cand[kf] : a.cont_cand[c]).sl;
+              bg = g;
+              bi = pos;
+              bf = f;
+            }
+          }
+        }
+        a.slot_gain[kf] = 0ull;
+        a.slot_pos[kf] = 0xffffffffu;
+      }
+      double gmax = bg;
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) gmax = fmax(gmax, __shfl_xor_sync(0xffffffffu, gmax, off));
+      const int wf = __reduce_min_sync(0xffffffffu, (bg == gmax && bg >= 0.0) ? bf : 0x7fffffff);
+      const int src = __ffs(__ballot_sync(0xffffffffu, bf == wf)) - 1;
+      const uint32_t wi = __shfl_sync(0xffffffffu, bi, src < 0 ? 0 : src);
+      const double wsl = __shfl_sync(0xffffffffu, bsl, src < 0 ? 0 : src);
+      // node statistics from the feature-0 list
+      const int64_t s0 = nd.start, s1 = s0 + nd.N - 1;
+      const int64_t t0 = s0 / kChunkW, t1 = s1 / kChunkW;
+      const int64_t np = t1 - t0 + 1;
+      const int64_t per = (np + 31) / 32;
+      Stat acc{0.0, INFINITY, -INFINITY, 0.0};
+      for (int64_t pc = lane * per; pc < min(np, (lane + 1) * per); ++pc) {
+        const Stat st = (pc == 0) ? a.head_stat[k] : a.cont_stat[t0 + pc];
+        acc.sse = __dadd_rn(acc.sse, st.sse);
+        acc.ymin = fmin(acc.ymin, st.ymin);
+        acc.ymax = fmax(acc.ymax, st.ymax);
+        acc.s1 = __dadd_rn(acc.s1, st.s1);
+      }
+#pragma unroll
+      for (int off = 1; off < 32; off <<= 1) {  // lane l absorbs lane l + off (fixed shape)
+        const double o_sse = __shfl_down_sync(0xffffffffu, acc.sse, off);
+        const double o_min = __shfl_down_sync(0xffffffffu, acc.ymin, off);
+        const double o_max = __shfl_down_sync(0xffffffffu, acc.ymax, off);
+        const double o_s1 = __shfl_down_sync(0xffffffffu, acc.s1, off);
+        if ((lane & (2 * off - 1)) == 0) {
+          acc.sse = __dadd_rn(acc.sse, o_sse);
+          acc.ymin = fmin(acc.ymin, o_min);
+          acc.ymax = fmax(acc.ymax, o_max);
+          acc.s1 = __dadd_rn(acc.s1, o_s1);
+        }
+      }
+      if (lane == 0) {
+        ExchRec r;
+        r.gain = -1.0;
+        r.sl = 0.0;
+        r.thr = 0.0;
+        r.i = 0;
+        r.gf = -1;
+        if (wf != 0x7fffffff) {
+          const int64_t pos = (int64_t)wf * (int64_t)A + nd.start + wi;
+          const double xlo = (double)a.lx[pos - 1], xhi = (double)a.lx[pos];
+          r.gain = gmax;
+          r.sl = wsl;
+          r.i = wi;
+          r.gf = wf * a.world + a.rank;
+          r.thr = __dadd_rn(__ddiv_rn(xlo, 2.0), __ddiv_rn(xhi, 2.0));  // Reading R5
+        }
+        r.sse = acc.sse;
+        r.ymin = acc.ymin;
+        r.ymax = acc.ymax;
+        r.s1 = acc.s1;
+        a.exch[k] = r;
+        if (a.world == 1) decide_node(a, k, nd, a.exch, 0);  // single rank: decide in place
+      }
+    }
+    return;
+  }
   for (uint32_t k = blockIdx.x; k < K; k += gridDim.x) {
     const NodeL nd = a.nodes[k];
     // ---- per-feature best: max gain (slot_gain) at the lowest position (slot_pos); the
