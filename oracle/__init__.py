@@ -58,6 +58,9 @@ def _load():
                                    ctypes.c_int64, P]
         lib.oracle_loo.restype = ctypes.c_int
         lib.oracle_importances.argtypes = [P, ctypes.c_int64, ctypes.c_int32, P]
+        lib.oracle_bootstrap.argtypes = [ctypes.c_uint64, ctypes.c_int32, ctypes.c_int64, P]
+        lib.oracle_forest_predict.argtypes = [P, P, ctypes.c_int32, P, ctypes.c_int64,
+                                              ctypes.c_int32, P]
         _lib = lib
     return _lib
 
@@ -149,3 +152,38 @@ def importances(nodes, d: int):
     imp = np.empty(d, dtype=np.float64)
     lib.oracle_importances(nodes.ctypes.data, len(nodes), d, imp.ctypes.data)
     return imp
+
+
+# ------------------------------------------------------------ random forest (NEXT-2) ----
+
+def bootstrap(seed: int, t: int, n: int):
+    """Row indices of tree t's bootstrap sample (n draws with replacement, Reading R21)."""
+    lib = _load()
+    idx = np.empty(n, dtype=np.uint32)
+    lib.oracle_bootstrap(ctypes.c_uint64(seed), t, n, idx.ctypes.data)
+    return idx
+
+
+def forest_fit(X, y, n_trees: int, max_depth: int = -1, min_samples_leaf: int = 1, seed: int = 0):
+    """Bagged CART (Reading R20): tree t = fit on (X[idx_t], y[idx_t])."""
+    X = _f32(X)
+    y = _f64(y)
+    trees = []
+    for t in range(n_trees):
+        idx = bootstrap(seed, t, X.shape[0])
+        trees.append(fit(X[idx], y[idx], max_depth, min_samples_leaf))
+    return trees
+
+
+def forest_predict(trees, X):
+    """Mean of the trees' predictions, summed in tree order, divided by T."""
+    lib = _load()
+    X = _f32(X)
+    arrs = [np.ascontiguousarray(t, dtype=NODE_DTYPE) for t in trees]
+    ptrs = (ctypes.c_void_p * len(arrs))(*[a.ctypes.data for a in arrs])
+    counts = np.array([len(a) for a in arrs], dtype=np.int64)
+    yhat = np.empty(X.shape[0], dtype=np.float64)
+    lib.oracle_forest_predict(ptrs, counts.ctypes.data, len(arrs), X.ctypes.data, X.shape[0],
+                              X.shape[1], yhat.ctypes.data)
+    return yhat
+

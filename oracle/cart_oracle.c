@@ -318,3 +318,39 @@ void oracle_importances(const oracle_node* nodes, int64_t count, int32_t d, doub
   for (int32_t f = 0; f < d; ++f) tot += imp[f];
   if (tot > 0.0) for (int32_t f = 0; f < d; ++f) imp[f] /= tot;
 }
+
+/* ------------------------------------------------------- random forest (NEXT-2) -- */
+
+/* Random Forest = bagged CART ("the Random Forest Tree is an ensemble of Decision
+ * Trees"; "the decision is taken based on the average value of all included
+ * Decision Trees").  Reading R20: tree t is grown by oracle_fit on the bootstrap sample
+ * X[idx_t], y[idx_t] (n draws with replacement, in draw order; duplicates count towards
+ * min_samples_leaf); every split considers all d features (sklearn's regression default,
+ * max_features = 1.0).  Draw i of tree t (counter-based SplitMix64, Reading R21):
+ *   z = seed + 0x9E3779B97F4A7C15 * ((t << 32) + i + 1)   (mod 2^64)
+ *   z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9; z = (z ^ (z >> 27)) * 0x94D049BB133111EB;
+ *   z ^= z >> 31;  idx = z mod n. */
+void oracle_bootstrap(uint64_t seed, int32_t t, int64_t n, uint32_t* idx) {
+  for (int64_t i = 0; i < n; ++i) {
+    uint64_t z = seed + 0x9E3779B97F4A7C15ull * ((((uint64_t)(uint32_t)t) << 32) + (uint64_t)i + 1ull);
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    z ^= z >> 31;
+    idx[i] = (uint32_t)(z % (uint64_t)n);
+  }
+}
+
+/* Forest prediction: the mean of the trees' predictions, summed in tree order (plain
+ * fp64, no compensation: T is small), then divided by T. */
+void oracle_forest_predict(const oracle_node* const* trees, const int64_t* counts, int32_t n_trees,
+                           const float* X, int64_t n, int32_t d, double* yhat) {
+  for (int64_t r = 0; r < n; ++r) {
+    double acc = 0.0;
+    for (int32_t t = 0; t < n_trees; ++t) {
+      double v;
+      oracle_predict(trees[t], counts[t], X + r * d, 1, d, &v);
+      acc = acc + v;
+    }
+    yhat[r] = acc / (double)n_trees;
+  }
+}
