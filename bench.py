@@ -566,6 +566,39 @@ def run_ours(args, world, rank, local):
         except Exception as e:
             extra = {"error": f"{type(e).__name__}: {e}"}
 
+    # ---- Random Forest: 16 bagged trees of the configs[1] table
+    forest = None
+    if not args.no_extra:
+        try:
+            T = 16
+            fo = dt.dt_forest_fit(X, y, 2, MAX_DEPTH, MIN_LEAF, seed=1)  # warm-up (plans the graph)
+            torch.cuda.synchronize()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            barrier(world)
+            a.record(stream)
+            fo = dt.dt_forest_fit(X, y, T, MAX_DEPTH, MIN_LEAF, seed=1)
+            b.record(stream)
+            torch.cuda.synchronize()
+            tf = max_over_ranks(a.elapsed_time(b) / 1e3, world)
+            outv = torch.empty(Xv.shape[0], dtype=torch.float64, device=dev)
+            dt.dt_forest_predict(fo, Xv, out=outv)
+            torch.cuda.synchronize()
+            a.record(stream)
+            for _ in range(5):
+                dt.dt_forest_predict(fo, Xv, out=outv)
+            b.record(stream)
+            torch.cuda.synchronize()
+            tp = a.elapsed_time(b) / 1e3 / 5
+            mf = dt.dt_eval(yv, outv, D)
+            forest = {"workload": f"{T} bagged trees (bootstrap seed 1) of the configs[1] table, depth "
+                                  f"{MAX_DEPTH}; predict + eval on the 1M held-out rows",
+                      "split_evals_per_s": sum_over_ranks(float(fo.split_evals), world) / tf,
+                      "ms_per_forest_fit": tf * 1e3, "predict_ms": tp * 1e3,
+                      "predictions_per_s": Xv.shape[0] / tp, "eval_mape": mf["mape"], "eval_r2": mf["r2"]}
+            del fo, outv
+        except Exception as e:
+            forest = {"error": f"{type(e).__name__}: {e}"}
+
     c3 = None
     if args.c3_rows > 0:
         del Xd, yd, Xvd, yvd
@@ -591,7 +624,7 @@ def run_ours(args, world, rank, local):
                         "d2h_bytes_per_step": d2h, "steps": args.e2e_steps},
                 "gpu_launches": launches,
                 "roofline": roofline, "cpu_baseline": cpu, "dse": dse, "sharded_fit": sharded, "extra_configs": extra,
-                "c3_fit": c3,
+                "c3_fit": c3, "forest": forest,
                 "clocks": clk.summary(),
                 "fit": {"split_evals_per_step": evals // args.steps, "tree_nodes": tree.size,
                         "tree_depth": tree.depth, "eval_mape": m["mape"], "eval_r2": m["r2"],

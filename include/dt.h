@@ -165,6 +165,35 @@ dt_status dt_predict_eval_depths(const dt_tree* tree, const float* X_dev, const 
  * importances_host has dt_tree_num_features(tree) entries.  Sync. */
 dt_status dt_importances(const dt_tree* tree, double* importances_host, void* stream);
 
+/* ------------------------------------------------------------------ random forest - */
+
+/* Random Forest = bagged CART ("an ensemble of Decision
+ * Trees", :231 "the decision is taken based on the average value of all included
+ * Decision Trees"; Readings R20, R21).  Tree t (0 <= t < n_trees) is exactly dt_fit's
+ * tree of its bootstrap sample: the n rows X[idx_t[i]], y[idx_t[i]], i = 0..n-1 in draw
+ * order (duplicates count towards min_samples_leaf), all d features at every split.
+ * Draw i of tree t (dt_bootstrap): z = seed + 0x9E3779B97F4A7C15 * ((t << 32) + i + 1),
+ * z = (z ^ z >> 30) * 0xBF58476D1CE4E5B9, z = (z ^ z >> 27) * 0x94D049BB133111EB,
+ * z ^= z >> 31, idx = z mod n (all mod 2^64).  Prediction: the mean of the trees'
+ * predictions, summed in fp64 in tree order, then divided by n_trees.
+ * dt_forest_fit: X_dev n x d f32 row-major, y_dev n f64 (as dt_fit); n_trees >= 1; the
+ * library allocates one n x d bootstrap sample for the duration of the call; returns
+ * when every tree is complete.  The forest owns its trees: dt_forest_tree returns a
+ * borrowed pointer valid until dt_forest_free.  Errors as dt_fit. */
+typedef struct dt_forest dt_forest;
+dt_status dt_forest_fit(const float* X_dev, const double* y_dev, int64_t n, int32_t d,
+                        int32_t n_trees, int32_t max_depth, int64_t min_samples_leaf,
+                        uint64_t seed, void* stream, dt_forest** out);
+int32_t dt_forest_num_trees(const dt_forest* forest);
+const dt_tree* dt_forest_tree(const dt_forest* forest, int32_t t);
+int64_t dt_forest_split_evals(const dt_forest* forest);  /* sum over the trees */
+/* yhat_dev[r] = forest mean for row r of X_dev (n x d f32); async on stream. */
+dt_status dt_forest_predict(const dt_forest* forest, const float* X_dev, int64_t n, int32_t d,
+                            double* yhat_dev, void* stream);
+void dt_forest_free(dt_forest* forest);
+/* The bootstrap draws of tree t: idx_dev[i], i < n (u32, device); async on stream. */
+dt_status dt_bootstrap(uint64_t seed, int32_t tree, int64_t n, uint32_t* idx_dev, void* stream);
+
 /* ------------------------------------------------------------------ LOO ----------- */
 
 /* dt_loo -- leave-one-out refits (BASELINE configs[0]; the paper's 70/30 split, P:197,

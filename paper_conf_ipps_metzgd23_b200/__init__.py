@@ -90,6 +90,13 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "dt_importances": ([P, P, P], ctypes.c_int),
         "dt_release_workspace": ([], ctypes.c_int),
         "dt_predict_dse": ([P, P, I64, I32, P, I64, I32, P, P, P], ctypes.c_int),
+        "dt_forest_fit": ([P, P, I64, I32, I32, I32, I64, U64, P, ctypes.POINTER(P)], ctypes.c_int),
+        "dt_forest_num_trees": ([P], I32),
+        "dt_forest_tree": ([P, I32], P),
+        "dt_forest_split_evals": ([P], I64),
+        "dt_forest_predict": ([P, P, I64, I32, P, P], ctypes.c_int),
+        "dt_forest_free": ([P], None),
+        "dt_bootstrap": ([U64, I32, I64, P, P], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -124,10 +131,12 @@ def _dev(t, dtype, ndim, name):
 
 
 class Tree:
-    """Owns a ``dt_tree*``.  ``nodes`` is a numpy structured copy (BFS, 48 B/node)."""
+    """Owns a ``dt_tree*`` (or borrows one from its ``owner``, e.g. a Forest).  ``nodes``
+    is a numpy structured copy (BFS, 48 B/node)."""
 
-    def __init__(self, handle: ctypes.c_void_p):
+    def __init__(self, handle: ctypes.c_void_p, owner=None):
         self._h = handle
+        self._owner = owner
 
     @property
     def handle(self):
@@ -135,9 +144,9 @@ class Tree:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h is not None and h.value:
+        if h is not None and h.value and getattr(self, "_owner", None) is None:
             _lib.dt_tree_free(h)
-            self._h = None
+        self._h = None
 
     @property
     def size(self) -> int:
@@ -390,6 +399,69 @@ def dt_fit_sharded(comm: Comm, X, y, max_depth: int = -1, min_samples_leaf: int 
     _check(_lib.dt_fit_sharded(comm.handle, xp, yp, n, d, max_depth, min_samples_leaf,
                                _stream(stream), ctypes.byref(h)))
     return Tree(h)
+
+
+class Forest:
+    """Owns a ``dt_forest*`` (bagged CART, include/dt.h)."""
+
+    def __init__(self, handle: ctypes.c_void_p):
+        self._h = handle
+
+    @property
+    def handle(self):
+        return self._h
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h is not None and h.value:
+            _lib.dt_forest_free(h)
+        self._h = None
+
+    @property
+    def num_trees(self) -> int:
+        return int(_lib.dt_forest_num_trees(self._h))
+
+    @property
+    def split_evals(self) -> int:
+        return int(_lib.dt_forest_split_evals(self._h))
+
+    def tree(self, t: int) -> Tree:
+        p = _lib.dt_forest_tree(self._h, t)
+        if not p:
+            raise IndexError(t)
+        return Tree(ctypes.c_void_p(p), owner=self)
+
+
+def dt_forest_fit(X, y, n_trees: int, max_depth: int = -1, min_samples_leaf: int = 1,
+                  seed: int = 0, stream=None) -> Forest:
+    import torch
+    xp = _dev(X, torch.float32, 2, "X")
+    yp = _dev(y, torch.float64, 1, "y")
+    n, d = X.shape
+    if y.shape[0] != n:
+        raise ValueError("y must have n elements")
+    h = ctypes.c_void_p()
+    _check(_lib.dt_forest_fit(xp, yp, n, d, n_trees, max_depth, min_samples_leaf,
+                              ctypes.c_uint64(seed), _stream(stream), ctypes.byref(h)))
+    return Forest(h)
+
+
+def dt_forest_predict(forest: Forest, X, out=None, stream=None):
+    import torch
+    n, d = X.shape
+    if out is None:
+        out = torch.empty(n, dtype=torch.float64, device=X.device)
+    _check(_lib.dt_forest_predict(forest.handle, _dev(X, torch.float32, 2, "X"), n, d,
+                                  _dev(out, torch.float64, 1, "out"), _stream(stream)))
+    return out
+
+
+def dt_bootstrap(seed: int, tree: int, n: int, device="cuda", stream=None):
+    import torch
+    out = torch.empty(n, dtype=torch.int32, device=device)  # u32 bits
+    _check(_lib.dt_bootstrap(ctypes.c_uint64(seed), tree, n, ctypes.c_void_p(out.data_ptr()),
+                             _stream(stream)))
+    return out
 
 
 def dt_release_workspace():

@@ -294,4 +294,38 @@ dt_status dt_gen_dse(uint64_t seed, int64_t row0, int64_t n, int32_t gpu_bits, f
 
 dt_status dt_release_workspace(void) { return release_workspace_impl(); }
 
+dt_status dt_bootstrap(uint64_t seed, int32_t tree, int64_t n, uint32_t* idx_dev, void* stream) {
+  if (!idx_dev) return fail(DT_ERR_INVALID_ARG, "dt_bootstrap: idx is NULL");
+  if (tree < 0) return fail(DT_ERR_INVALID_ARG, "dt_bootstrap: tree must be >= 0");
+  if (n < 1) return fail(DT_ERR_INVALID_ARG, "dt_bootstrap: n must be >= 1");
+  if (n >= (int64_t)1 << 32) return fail(DT_ERR_TOO_LARGE, "dt_bootstrap: n must be < 2^32");
+  return bootstrap_impl(seed, tree, n, idx_dev, S(stream));
+}
+
+dt_status dt_forest_fit(const float* X_dev, const double* y_dev, int64_t n, int32_t d, int32_t n_trees,
+                        int32_t max_depth, int64_t min_samples_leaf, uint64_t seed, void* stream,
+                        dt_forest** out) {
+  if (!out) return fail(DT_ERR_INVALID_ARG, "dt_forest_fit: out is NULL");
+  *out = nullptr;
+  if (!X_dev || !y_dev) return fail(DT_ERR_INVALID_ARG, "dt_forest_fit: NULL X or y");
+  if (n < 1) return fail(DT_ERR_INVALID_ARG, "dt_forest_fit: n must be >= 1");
+  if (d < 1 || d > 255) return fail(DT_ERR_INVALID_ARG, "dt_forest_fit: d must be in [1, 255]");
+  if (n_trees < 1) return fail(DT_ERR_INVALID_ARG, "dt_forest_fit: n_trees must be >= 1");
+  if (min_samples_leaf < 1) return fail(DT_ERR_INVALID_ARG, "dt_forest_fit: min_samples_leaf must be >= 1");
+  if (max_depth < -1) return fail(DT_ERR_INVALID_ARG, "dt_forest_fit: max_depth must be >= -1");
+  if (n >= (int64_t)1 << 32) return fail(DT_ERR_TOO_LARGE, "dt_forest_fit: n must be < 2^32");
+  return forest_fit_impl(X_dev, y_dev, n, d, n_trees, max_depth, min_samples_leaf, seed, S(stream), out);
+}
+
+dt_status dt_forest_predict(const dt_forest* forest, const float* X_dev, int64_t n, int32_t d,
+                            double* yhat_dev, void* stream) {
+  if (!forest) return fail(DT_ERR_INVALID_ARG, "dt_forest_predict: forest is NULL");
+  if (n < 0) return fail(DT_ERR_INVALID_ARG, "dt_forest_predict: n < 0");
+  if (n == 0) return DT_OK;
+  if (!X_dev || !yhat_dev) return fail(DT_ERR_INVALID_ARG, "dt_forest_predict: NULL X or yhat");
+  if (d != dt_tree_num_features(dt_forest_tree(forest, 0)))
+    return fail(DT_ERR_INVALID_ARG, "dt_forest_predict: d differs from the forest's d");
+  return forest_predict_impl(forest, X_dev, n, d, yhat_dev, S(stream));
+}
+
 }  // extern "C"

@@ -59,6 +59,12 @@ dt_status eval_impl(const double* y, const double* yhat, const float* X, const d
 dt_status importances_impl(const dt_tree* t, double* imp_host, cudaStream_t s);
 dt_status eval_depths_impl(const dt_tree* t, const float* X, const double* y, int64_t n, int32_t p,
                            cudaStream_t s, double* out_host);
+// Random forest (forest.cu).
+dt_status bootstrap_impl(uint64_t seed, int32_t t, int64_t n, uint32_t* idx, cudaStream_t s);
+dt_status forest_fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t n_trees,
+                          int32_t max_depth, int64_t min_leaf, uint64_t seed, cudaStream_t s, dt_forest** out);
+dt_status forest_predict_impl(const dt_forest* fo, const float* X, int64_t n, int32_t d, double* yhat,
+                              cudaStream_t s);
 // LOO (loo.cu).
 dt_status loo_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
                    int64_t min_leaf, double* yhat, cudaStream_t s);
