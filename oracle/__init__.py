@@ -58,6 +58,8 @@ def _load():
                                    ctypes.c_int64, P]
         lib.oracle_loo.restype = ctypes.c_int
         lib.oracle_importances.argtypes = [P, ctypes.c_int64, ctypes.c_int32, P]
+        lib.oracle_knn.argtypes = [P, P, ctypes.c_int64, ctypes.c_int32, P, ctypes.c_int64,
+                                   ctypes.c_int32, P]
         lib.oracle_bootstrap.argtypes = [ctypes.c_uint64, ctypes.c_int32, ctypes.c_int64, P]
         lib.oracle_forest_predict.argtypes = [P, P, ctypes.c_int32, P, ctypes.c_int64,
                                               ctypes.c_int32, P]
@@ -185,5 +187,23 @@ def forest_predict(trees, X):
     yhat = np.empty(X.shape[0], dtype=np.float64)
     lib.oracle_forest_predict(ptrs, counts.ctypes.data, len(arrs), X.ctypes.data, X.shape[0],
                               X.shape[1], yhat.ctypes.data)
+    return yhat
+
+
+# ------------------------------------------------------------- KNN regression (NEXT-4) ----
+
+def knn_predict(Xtr, ytr, Xq, k: int = 5):
+    """KNN regression (Table II; Reading R22): mean y of the k nearest training rows
+    by fp64 squared Euclidean distance (fma-accumulated in feature order), ties to the
+    lower training row index."""
+    lib = _load()
+    Xtr = _f32(Xtr)
+    ytr = _f64(ytr)
+    Xq = _f32(Xq)
+    if not (1 <= k <= Xtr.shape[0]):
+        raise ValueError("need 1 <= k <= n_train")
+    yhat = np.empty(Xq.shape[0], dtype=np.float64)
+    lib.oracle_knn(Xtr.ctypes.data, ytr.ctypes.data, Xtr.shape[0], Xtr.shape[1], Xq.ctypes.data,
+                   Xq.shape[0], k, yhat.ctypes.data)
     return yhat
 

@@ -354,3 +354,44 @@ void oracle_forest_predict(const oracle_node* const* trees, const int64_t* count
     yhat[r] = acc / (double)n_trees;
   }
 }
+
+/* ------------------------------------------------------- K-nearest neighbours (NEXT-4) */
+
+/* KNN regression ("K-Nearest Neighbors ... non-linear dependencies", Table II
+ * P:214; sklearn KNeighborsRegressor defaults: k = 5, uniform weights, Euclidean).
+ * Reading R22: dist(q, x) = sum over f = 0..d-1, in feature order, of (q_f - x_f)^2,
+ * each term fused into the running sum: acc = fma(q_f - x_f, q_f - x_f, acc), with
+ * q_f - x_f taken in fp64 from the f32 inputs (one rounding).  Squared distance orders
+ * exactly like the Euclidean one.  Neighbours: the k training rows with the smallest
+ * (dist, row index) -- ties go to the lower index; yhat = (sum of their y in that
+ * order) / k.  k <= n_train. */
+void oracle_knn(const float* Xtr, const double* ytr, int64_t ntr, int32_t d, const float* Xq,
+                int64_t nq, int32_t k, double* yhat) {
+  double* bd = (double*)malloc(sizeof(double) * (size_t)k);
+  int64_t* bi = (int64_t*)malloc(sizeof(int64_t) * (size_t)k);
+  for (int64_t q = 0; q < nq; ++q) {
+    int32_t cnt = 0;  /* bd/bi sorted ascending by (dist, index) */
+    for (int64_t r = 0; r < ntr; ++r) {
+      double acc = 0.0;
+      for (int32_t f = 0; f < d; ++f) {
+        double df = (double)Xq[q * d + f] - (double)Xtr[r * d + f];
+        acc = fma(df, df, acc);
+      }
+      if (cnt == k && !(acc < bd[k - 1])) continue;  /* equal distance: the lower index stays */
+      int32_t pos = (cnt < k) ? cnt : k - 1;
+      while (pos > 0 && acc < bd[pos - 1]) {  /* strict: earlier (lower) index first on ties */
+        bd[pos] = bd[pos - 1];
+        bi[pos] = bi[pos - 1];
+        --pos;
+      }
+      bd[pos] = acc;
+      bi[pos] = r;
+      if (cnt < k) ++cnt;
+    }
+    double s = 0.0;
+    for (int32_t j = 0; j < k; ++j) s = s + ytr[bi[j]];
+    yhat[q] = s / (double)k;
+  }
+  free(bd);
+  free(bi);
+}

@@ -17,13 +17,19 @@ timeout 600 python bench.py > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_
 echo "bench exit $?" >> gpurun_out/${TAG}_bench.err
 timeout 600 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none \
   --csv --log-file gpurun_out/${TAG}_launches.csv \
-  python bench.py --steps 1 --warmup 0 --no-cpu --no-extra --e2e-steps 0 --no-dse > gpurun_out/${TAG}_ncu_launch.log 2>&1
+  python bench.py --steps 1 --warmup 0 --no-cpu --no-extra --e2e-steps 0 --no-dse --c3-rows 0 > gpurun_out/${TAG}_ncu_launch.log 2>&1
 echo "ncu launch exit $?" >> gpurun_out/${TAG}_ncu_launch.log
 timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base function \
-  -k regex:'^(scan_kernel|scan_single_kernel|partition_kernel|part_agg_kernel|scan_agg_kernel|predict_col_kernel|rs_scatter_kernel)$' \
+  -k regex:'^(scan_kernel|scan_single_kernel|partition_kernel|part_agg_kernel|scan_agg_kernel|rs_scatter_kernel|select_kernel|prep_kernel)$' \
   --launch-count 12 -o /tmp/${TAG}_full -f \
-  python bench.py --steps 1 --warmup 0 --no-cpu --no-extra --e2e-steps 0 --dse-log2 24 > gpurun_out/${TAG}_ncu_full.log 2>&1
+  python bench.py --steps 1 --warmup 0 --no-cpu --no-extra --e2e-steps 0 --no-dse --c3-rows 0 > gpurun_out/${TAG}_ncu_full.log 2>&1
 echo "ncu full exit $?" >> gpurun_out/${TAG}_ncu_full.log
 ncu -i /tmp/${TAG}_full.ncu-rep --page raw --csv > gpurun_out/${TAG}_full_raw.csv 2>/dev/null
 ncu -i /tmp/${TAG}_full.ncu-rep --page details --csv > gpurun_out/${TAG}_full_details.csv 2>/dev/null
 ls -la /tmp/${TAG}_full.ncu-rep >> gpurun_out/${TAG}_ncu_full.log
+# predict kernels (materialised rows and the factored DSE), one launch each
+timeout 600 ncu --set full --clock-control none --import-source on --kernel-name-base function \
+  -k regex:'^(predict_col_kernel|predict_dse_kernel|forest_predict_kernel)$' --launch-count 3 -o /tmp/${TAG}_pred -f \
+  python bench.py --steps 1 --warmup 0 --no-cpu --e2e-steps 0 --dse-log2 24 --c3-rows 0 --grid-rows 0 > gpurun_out/${TAG}_ncu_pred.log 2>&1
+echo "ncu pred exit $?" >> gpurun_out/${TAG}_ncu_pred.log
+ncu -i /tmp/${TAG}_pred.ncu-rep --page raw --csv > gpurun_out/${TAG}_pred_raw.csv 2>/dev/null
