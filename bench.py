@@ -599,6 +599,39 @@ def run_ours(args, world, rank, local):
         except Exception as e:
             forest = {"error": f"{type(e).__name__}: {e}"}
 
+    # ---- KNN regression: 2^16 training rows of the configs[1] table,
+    # 2^20 queries (held-out rows), k = 5 (sklearn default); fp64 CUDA-core brute force
+    knn = None
+    if not args.no_extra:
+        try:
+            ntr, nqk = 1 << 16, 1 << 20
+            Xtr, ytr = X[:ntr].contiguous(), y[:ntr].contiguous()
+            Xq = Xv[:nqk].contiguous()
+            outk = torch.empty(nqk, dtype=torch.float64, device=dev)
+            dt.dt_knn_predict(Xtr, ytr, Xq[:4096], 5, out=outk[:4096])  # warm-up
+            torch.cuda.synchronize()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            dt.dt_knn_predict(Xtr, ytr, Xq, 5, out=outk)
+            b.record(stream)
+            torch.cuda.synchronize()
+            tk = a.elapsed_time(b) / 1e3
+            pairs = float(ntr) * nqk
+            # fp64 pipe: 64 lanes / SM / clock (B200 FP64 37 TFLOPS = 2 x 64 x 148 x 1.965 GHz),
+            # 2 instructions (DSUB, DFMA) per (query, row, feature)
+            ops = 2.0 * D * pairs
+            peak_ops = 64.0 * 148 * 1.965e9
+            knn = {"workload": f"{ntr} training rows (configs[1] table) x {nqk} queries (held-out rows), "
+                               f"d {D}, k 5", "ms": tk * 1e3, "distance_pairs_per_s": pairs / tk,
+                   "predictions_per_s": nqk / tk,
+                   "roofline": {"bound": "alu", "kernel": "knn (fp64 pipe)", "achieved": ops / tk / 1e12,
+                                "peak": peak_ops / 1e12, "unit": "T fp64 instr/s",
+                                "frac": ops / tk / peak_ops,
+                                "peak_source": "derived: 64 fp64 lanes/SM/clk x 148 SMs x 1.965 GHz"}}
+            del outk, Xtr, ytr, Xq
+        except Exception as e:
+            knn = {"error": f"{type(e).__name__}: {e}"}
+
     c3 = None
     if args.c3_rows > 0:
         del Xd, yd, Xvd, yvd
@@ -624,7 +657,7 @@ def run_ours(args, world, rank, local):
                         "d2h_bytes_per_step": d2h, "steps": args.e2e_steps},
                 "gpu_launches": launches,
                 "roofline": roofline, "cpu_baseline": cpu, "dse": dse, "sharded_fit": sharded, "extra_configs": extra,
-                "c3_fit": c3, "forest": forest,
+                "c3_fit": c3, "forest": forest, "knn": knn,
                 "clocks": clk.summary(),
                 "fit": {"split_evals_per_step": evals // args.steps, "tree_nodes": tree.size,
                         "tree_depth": tree.depth, "eval_mape": m["mape"], "eval_r2": m["r2"],

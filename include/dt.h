@@ -194,6 +194,20 @@ void dt_forest_free(dt_forest* forest);
 /* The bootstrap draws of tree t: idx_dev[i], i < n (u32, device); async on stream. */
 dt_status dt_bootstrap(uint64_t seed, int32_t tree, int64_t n, uint32_t* idx_dev, void* stream);
 
+/* ------------------------------------------------------------------ KNN ----------- */
+
+/* dt_knn_predict -- KNN regression (Table II :214;
+ * sklearn KNeighborsRegressor defaults: uniform weights, Euclidean; Reading R22):
+ * yhat_dev[q] = (sum of y over the k nearest training rows, in (distance, row) order) / k,
+ * distance(q, x) = fp64 sum over f in feature order of (q_f - x_f)^2, each term fused
+ * (acc = fma(df, df, acc), df = (double)q_f - (double)x_f); equal distances go to the
+ * lower training row.  Xtr_dev n_train x d f32, ytr_dev n_train f64, Xq_dev n_query x d
+ * f32 (row-major, device); 1 <= k <= min(16, n_train); d in 1..8, 10, 12, 16, 32.
+ * Brute force, fp64 CUDA cores (bound: the fp64 pipe).  Async on stream. */
+dt_status dt_knn_predict(const float* Xtr_dev, const double* ytr_dev, int64_t n_train, int32_t d,
+                         const float* Xq_dev, int64_t n_query, int32_t k, double* yhat_dev,
+                         void* stream);
+
 /* ------------------------------------------------------------------ LOO ----------- */
 
 /* dt_loo -- leave-one-out refits (BASELINE configs[0]; the paper's 70/30 split, P:197,

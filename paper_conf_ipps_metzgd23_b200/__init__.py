@@ -97,6 +97,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "dt_forest_predict": ([P, P, I64, I32, P, P], ctypes.c_int),
         "dt_forest_free": ([P], None),
         "dt_bootstrap": ([U64, I32, I64, P, P], ctypes.c_int),
+        "dt_knn_predict": ([P, P, I64, I32, P, I64, I32, P, P], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -461,6 +462,21 @@ def dt_bootstrap(seed: int, tree: int, n: int, device="cuda", stream=None):
     out = torch.empty(n, dtype=torch.int32, device=device)  # u32 bits
     _check(_lib.dt_bootstrap(ctypes.c_uint64(seed), tree, n, ctypes.c_void_p(out.data_ptr()),
                              _stream(stream)))
+    return out
+
+
+def dt_knn_predict(Xtr, ytr, Xq, k: int = 5, out=None, stream=None):
+    """KNN regression (include/dt.h dt_knn_predict)."""
+    import torch
+    ntr, d = Xtr.shape
+    nq = Xq.shape[0]
+    if Xq.shape[1] != d or ytr.shape[0] != ntr:
+        raise ValueError("shape mismatch")
+    if out is None:
+        out = torch.empty(nq, dtype=torch.float64, device=Xq.device)
+    _check(_lib.dt_knn_predict(_dev(Xtr, torch.float32, 2, "Xtr"), _dev(ytr, torch.float64, 1, "ytr"), ntr, d,
+                               _dev(Xq, torch.float32, 2, "Xq"), nq, k, _dev(out, torch.float64, 1, "out"),
+                               _stream(stream)))
     return out
 
 

@@ -328,4 +328,15 @@ dt_status dt_forest_predict(const dt_forest* forest, const float* X_dev, int64_t
   return forest_predict_impl(forest, X_dev, n, d, yhat_dev, S(stream));
 }
 
+dt_status dt_knn_predict(const float* Xtr_dev, const double* ytr_dev, int64_t n_train, int32_t d,
+                         const float* Xq_dev, int64_t n_query, int32_t k, double* yhat_dev, void* stream) {
+  if (!Xtr_dev || !ytr_dev) return fail(DT_ERR_INVALID_ARG, "dt_knn_predict: NULL training data");
+  if (n_train < 1) return fail(DT_ERR_INVALID_ARG, "dt_knn_predict: n_train must be >= 1");
+  if (k < 1 || k > n_train) return fail(DT_ERR_INVALID_ARG, "dt_knn_predict: need 1 <= k <= n_train");
+  if (n_query < 0) return fail(DT_ERR_INVALID_ARG, "dt_knn_predict: n_query < 0");
+  if (n_query == 0) return DT_OK;
+  if (!Xq_dev || !yhat_dev) return fail(DT_ERR_INVALID_ARG, "dt_knn_predict: NULL queries or yhat");
+  return knn_impl(Xtr_dev, ytr_dev, n_train, d, Xq_dev, n_query, k, yhat_dev, S(stream));
+}
+
 }  // extern "C"

@@ -65,6 +65,9 @@ dt_status forest_fit_impl(const float* X, const double* y, int64_t n, int32_t d,
                           int32_t max_depth, int64_t min_leaf, uint64_t seed, cudaStream_t s, dt_forest** out);
 dt_status forest_predict_impl(const dt_forest* fo, const float* X, int64_t n, int32_t d, double* yhat,
                               cudaStream_t s);
+// KNN regression (knn.cu).
+dt_status knn_impl(const float* Xtr, const double* ytr, int64_t ntr, int32_t d, const float* Xq, int64_t nq,
+                   int32_t k, double* yhat, cudaStream_t s);
 // LOO (loo.cu).
 dt_status loo_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
                    int64_t min_leaf, double* yhat, cudaStream_t s);
