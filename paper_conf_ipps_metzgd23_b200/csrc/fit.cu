@@ -966,7 +966,7 @@ __device__ __forceinline__ void scan_single(const ScanArgs& a, int64_t ch, int64
 
 // One pipeline stage of scan_single_kernel: everything one chunk needs, brought in by
 // TMA bulk copies (x, y, descriptor, the two carry words, the entry before the chunk).
-constexpr int kScanStages = 3;
+constexpr int kScanStages = 2;
 struct __align__(128) ScanStage {
   float x[kChunkW];
   double y[kChunkW];
@@ -979,7 +979,7 @@ struct __align__(128) ScanStage {
 // Phase C for the single-segment chunks with a per-warp TMA pipeline: lane 0 keeps
 // kScanStages chunks in flight (bulk copies completing on one mbarrier per stage); the
 // lanes read their items from shared memory, so no registers hold in-flight data.
-__global__ void __launch_bounds__(kThreads, 2) scan_single_kernel(ScanArgs a) {
+__global__ void __launch_bounds__(kThreads, 3) scan_single_kernel(ScanArgs a) {
   extern __shared__ __align__(128) unsigned char scan_smem[];
   const uint32_t K = a.ctl->K[a.parity];
   const uint64_t A = a.ctl->A[a.parity];
@@ -1625,11 +1625,14 @@ struct NumberArgs {
   int64_t min_leaf;
   dt_node* out;
   LevelLog* log;
+  uint4* gbits;    // go-left bitmap, zeroed here for this level's prep_kernel
+  int64_t nvec;    // uint4 words of the bitmap
 };
 
 // Single block: BFS numbering (children appended left, right in node order), child
 // statistics, next-level offsets.  Integer mode keeps every quantity exact (int64).
 __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
+  for (int64_t i = threadIdx.x; i < a.nvec; i += blockDim.x) a.gbits[i] = make_uint4(0u, 0u, 0u, 0u);
   __shared__ CntP sh[33];
   __shared__ unsigned long long sh_rows[33];
   __shared__ uint32_t base_split;
@@ -2484,6 +2487,8 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     na.min_leaf = min_leaf;
     na.out = b.dout;
     na.log = b.lvlog;
+    na.gbits = reinterpret_cast<uint4*>(b.gbits);
+    na.nvec = b.nwords4 / 4;
     pr = prof_begin(PK_NUMBER, s, 1);
     number_kernel<<<1, 1024, 0, s>>>(na);
     prof_end(pr, s, 0.0);
@@ -2492,7 +2497,6 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     // descriptors (one launch)
     const int dl_out = (max_depth >= 0 && level + 1 == max_depth) ? 1 : d;
     pr = prof_begin(PK_GOLEFT, s, 1);
-    DT_CK(cudaMemsetAsync(b.gbits, 0, sizeof(uint32_t) * (size_t)b.nwords4, s));
     {
       PrepArgs pp;
       pp.lr = b.lr[cur];
