@@ -332,6 +332,7 @@ dt_status dt_knn_predict(const float* Xtr_dev, const double* ytr_dev, int64_t n_
                          const float* Xq_dev, int64_t n_query, int32_t k, double* yhat_dev, void* stream) {
   if (!Xtr_dev || !ytr_dev) return fail(DT_ERR_INVALID_ARG, "dt_knn_predict: NULL training data");
   if (n_train < 1) return fail(DT_ERR_INVALID_ARG, "dt_knn_predict: n_train must be >= 1");
+  if (n_train >= (int64_t)1 << 32) return fail(DT_ERR_TOO_LARGE, "dt_knn_predict: n_train must be < 2^32");
   if (k < 1 || k > n_train) return fail(DT_ERR_INVALID_ARG, "dt_knn_predict: need 1 <= k <= n_train");
   if (n_query < 0) return fail(DT_ERR_INVALID_ARG, "dt_knn_predict: n_query < 0");
   if (n_query == 0) return DT_OK;

@@ -6,8 +6,8 @@
 //
 // Brute force on the CUDA cores in fp64 (the exact distance of the definition; a GEMM
 // expansion |q|^2 + |x|^2 - 2 q.x on the tensor cores rounds differently and would
-// change the neighbour sets near ties).  One query per thread, kQ = 2 queries per thread
-// for ILP; the block streams the training set through shared memory in tiles of kTile
+// change the neighbour sets near ties).  kQ = 2 queries per thread (ILP and
+// shared-memory reuse); the block streams the training set through shared memory in tiles of kTile
 // rows (converted to f64 once per tile, read as warp-broadcasts); each thread keeps its
 // queries' k best (distance, row) pairs sorted in registers.  Bound: the fp64 pipe, two
 // instructions (DADD, DFMA) per (query, train row, feature).
@@ -21,9 +21,9 @@ namespace {
 
 constexpr int kKnnThreads = 128;
 constexpr int kKnnTile = 64;  // training rows per shared-memory tile
-constexpr int kKMax = 16;
+constexpr int kKMaxAll = 16;
 
-template <int D, int Q>
+template <int D, int Q, int kKMax>
 __global__ void __launch_bounds__(kKnnThreads)
 knn_kernel(const float* __restrict__ Xtr, const double* __restrict__ ytr, int64_t ntr, const float* __restrict__ Xq,
            int64_t nq, int k, double* __restrict__ yhat) {
@@ -37,13 +37,13 @@ knn_kernel(const float* __restrict__ Xtr, const double* __restrict__ ytr, int64_
     for (int f = 0; f < D; ++f) qv[a][f] = (double)__ldg(Xq + q * D + f);
   }
   double bd[Q][kKMax];
-  int64_t bi[Q][kKMax];
+  uint32_t bi[Q][kKMax];
   double worst[Q];
 #pragma unroll
   for (int a = 0; a < Q; ++a) {
     worst[a] = INFINITY;
 #pragma unroll
-    for (int j = 0; j < kKMax; ++j) { bd[a][j] = INFINITY; bi[a][j] = -1; }
+    for (int j = 0; j < kKMax; ++j) { bd[a][j] = INFINITY; bi[a][j] = 0u; }
   }
   for (int64_t t0 = 0; t0 < ntr; t0 += kKnnTile) {
     const int rows = (int)min((int64_t)kKnnTile, ntr - t0);
@@ -81,7 +81,7 @@ knn_kernel(const float* __restrict__ Xtr, const double* __restrict__ ytr, int64_
 #pragma unroll
       for (int a = 0; a < Q; ++a) {
         if (acc[a] < worst[a]) {  // strict: an equal distance keeps the earlier (lower) row
-          const int64_t row = t0 + r;
+          const uint32_t row = (uint32_t)(t0 + r);
           bool placed = false;
 #pragma unroll
           for (int j = kKMax - 1; j >= 0; --j) {
@@ -115,19 +115,22 @@ knn_kernel(const float* __restrict__ Xtr, const double* __restrict__ ytr, int64_
   }
 }
 
+// Two queries per thread (measured: 3 or 4 need > 200 registers and run ~2x slower);
+// the k-best lists sized 8 when k <= 8 (the sklearn default k = 5), else 16.
 template <int D>
 void launch_knn(const float* Xtr, const double* ytr, int64_t ntr, const float* Xq, int64_t nq, int k, double* yhat,
                 cudaStream_t s) {
   constexpr int Q = 2;
-  const int64_t per = (int64_t)kKnnThreads * Q;
-  knn_kernel<D, Q><<<(unsigned)((nq + per - 1) / per), kKnnThreads, 0, s>>>(Xtr, ytr, ntr, Xq, nq, k, yhat);
+  const unsigned g = (unsigned)((nq + Q * kKnnThreads - 1) / (Q * kKnnThreads));
+  if (k <= 8) knn_kernel<D, Q, 8><<<g, kKnnThreads, 0, s>>>(Xtr, ytr, ntr, Xq, nq, k, yhat);
+  else knn_kernel<D, Q, 16><<<g, kKnnThreads, 0, s>>>(Xtr, ytr, ntr, Xq, nq, k, yhat);
 }
 
 }  // namespace
 
 dt_status knn_impl(const float* Xtr, const double* ytr, int64_t ntr, int32_t d, const float* Xq, int64_t nq,
                    int32_t k, double* yhat, cudaStream_t s) {
-  if (k > kKMax) return fail(DT_ERR_TOO_LARGE, "dt_knn_predict: k must be <= 16");
+  if (k > kKMaxAll) return fail(DT_ERR_TOO_LARGE, "dt_knn_predict: k must be <= 16");
   const int pr = prof_begin(PK_PREDICT, s, 1);
   switch (d) {  // the query row lives in registers: d is a compile-time constant
 #define DT_KNN_CASE(D) \
