@@ -263,6 +263,14 @@ dt_status dt_fit_sharded(dt_comm* comm, const float* X_dev, const double* y_dev,
                          int32_t d, int32_t max_depth, int64_t min_samples_leaf, void* stream,
                          dt_tree** out);
 
+/* dt_eval_sharded -- MAPE / R^2 / adj-R^2 of rows split over the ranks (SURVEY 8e
+ * "Eval"; Table II): each rank reduces its n_local rows (y_dev, yhat_dev f64,
+ * device; n_local may be 0) to one partial (sum of |e|/max(|y|, eps), SSE, count and the
+ * Welford mean / M2 of y), the partials are allgathered and merged in rank order (Chan),
+ * so every rank returns bitwise the same metrics; out->n = the total row count.  Sync. */
+dt_status dt_eval_sharded(dt_comm* comm, const double* y_dev, const double* yhat_dev,
+                          int64_t n_local, int32_t p, void* stream, dt_metrics* out);
+
 /* ------------------------------------------------------------------ profiling ----- */
 
 /* Measurement hooks used by bench.py (not needed to use the library).  While enabled,

@@ -98,6 +98,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "dt_forest_free": ([P], None),
         "dt_bootstrap": ([U64, I32, I64, P, P], ctypes.c_int),
         "dt_knn_predict": ([P, P, I64, I32, P, I64, I32, P, P], ctypes.c_int),
+        "dt_eval_sharded": ([P, P, P, I64, I32, P, ctypes.POINTER(dt_metrics)], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -483,6 +484,19 @@ def dt_knn_predict(Xtr, ytr, Xq, k: int = 5, out=None, stream=None):
 def dt_release_workspace():
     """Free the cached fit plan and trim the device memory pool (include/dt.h)."""
     _check(_lib.dt_release_workspace())
+
+
+def dt_eval_sharded(comm: "Comm", y, yhat, p: int, stream=None) -> dict:
+    """Metrics of rows split over the ranks (include/dt.h); same result on every rank."""
+    import torch
+    m = dt_metrics()
+    n = y.shape[0]
+    if yhat.shape[0] != n:
+        raise ValueError("y and yhat differ in length")
+    yp = _dev(y, torch.float64, 1, "y") if n else ctypes.c_void_p(0)
+    hp = _dev(yhat, torch.float64, 1, "yhat") if n else ctypes.c_void_p(0)
+    _check(_lib.dt_eval_sharded(comm.handle, yp, hp, n, p, _stream(stream), ctypes.byref(m)))
+    return _metrics(m)
 
 
 def version() -> str:

@@ -340,4 +340,14 @@ dt_status dt_knn_predict(const float* Xtr_dev, const double* ytr_dev, int64_t n_
   return knn_impl(Xtr_dev, ytr_dev, n_train, d, Xq_dev, n_query, k, yhat_dev, S(stream));
 }
 
+dt_status dt_eval_sharded(dt_comm* comm, const double* y_dev, const double* yhat_dev, int64_t n_local, int32_t p,
+                          void* stream, dt_metrics* out) {
+  if (!comm) return fail(DT_ERR_INVALID_ARG, "dt_eval_sharded: comm is NULL");
+  if (!out) return fail(DT_ERR_INVALID_ARG, "dt_eval_sharded: out is NULL");
+  if (n_local < 0) return fail(DT_ERR_INVALID_ARG, "dt_eval_sharded: n_local < 0");
+  if (n_local > 0 && (!y_dev || !yhat_dev)) return fail(DT_ERR_INVALID_ARG, "dt_eval_sharded: NULL y or yhat");
+  if (p < 0) return fail(DT_ERR_INVALID_ARG, "dt_eval_sharded: p must be >= 0");
+  return eval_sharded_impl(comm, y_dev, yhat_dev, n_local, p, S(stream), out);
+}
+
 }  // extern "C"

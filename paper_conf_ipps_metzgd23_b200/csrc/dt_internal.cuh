@@ -56,6 +56,8 @@ dt_status predict_impl(const dt_tree* t, const float* X, int64_t n, int32_t d, d
                        cudaStream_t s);
 dt_status eval_impl(const double* y, const double* yhat, const float* X, const dt_tree* t,
                     int64_t n, int32_t p, cudaStream_t s, dt_metrics* out);
+dt_status eval_sharded_impl(dt_comm* comm, const double* y, const double* yhat, int64_t n, int32_t p,
+                            cudaStream_t s, dt_metrics* out);
 dt_status importances_impl(const dt_tree* t, double* imp_host, cudaStream_t s);
 dt_status eval_depths_impl(const dt_tree* t, const float* X, const double* y, int64_t n, int32_t p,
                            cudaStream_t s, double* out_host);

@@ -328,6 +328,35 @@ eval_final_kernel(const Part* __restrict__ parts, int nparts, int64_t n, int p_p
   }
 }
 
+// Merges a rank's block partials into ONE partial (fixed shape), for the allgather of
+// dt_eval_sharded.
+__global__ void __launch_bounds__(1024) eval_local_kernel(const Part* __restrict__ parts, int nparts,
+                                                          Part* __restrict__ out) {
+  Part acc{0, 0, 0, 0, 0};
+  for (int i = threadIdx.x; i < nparts; i += blockDim.x) part_merge(acc, parts[i]);
+  acc = block_reduce(acc);
+  if (threadIdx.x == 0) *out = acc;
+}
+
+// The ranks' partials merged in rank order (every rank runs the same sequence, so every
+// rank gets bitwise the same metrics); n = the merged count.
+__global__ void eval_ranks_kernel(const Part* __restrict__ parts, int world, int p_pred, double* __restrict__ out) {
+  if (threadIdx.x != 0) return;
+  Part acc{0, 0, 0, 0, 0};
+  for (int r = 0; r < world; ++r) part_merge(acc, parts[r]);
+  const double nn = acc.cnt;
+  double r2;
+  if (acc.m2 == 0.0) r2 = (acc.sse == 0.0) ? 1.0 : 0.0;  // Reading R13
+  else r2 = 1.0 - acc.sse / acc.m2;
+  double adj;
+  if (nn - (double)p_pred - 1.0 <= 0.0) adj = __longlong_as_double(0x7ff8000000000000ll);
+  else adj = 1.0 - (1.0 - r2) * (nn - 1.0) / (nn - (double)p_pred - 1.0);  // R14
+  out[0] = acc.ape / nn;
+  out[1] = r2;
+  out[2] = adj;
+  out[3] = nn;
+}
+
 template <bool kSmem, int kThr, int kRPT>
 dt_status launch_predict(const dt_tree* t, const float* X, int64_t n, int32_t d, double* yhat,
                          cudaStream_t s, int carveout) {
@@ -749,6 +778,50 @@ dt_status eval_impl(const double* y, const double* yhat, const float* X, const d
   out->r2 = h[1];
   out->adj_r2 = h[2];
   out->n = n;
+  out->p = p;
+  return DT_OK;
+}
+
+// dt_eval_sharded: each rank reduces its rows to one partial (sums + Welford moments),
+// the partials are allgathered and merged in rank order (SURVEY 8e "Eval").
+dt_status eval_sharded_impl(dt_comm* comm, const double* y, const double* yhat, int64_t n, int32_t p,
+                            cudaStream_t s, dt_metrics* out) {
+  const int world = comm_world(comm);
+  int64_t chunk = 4096;
+  int64_t nparts = n > 0 ? (n + chunk - 1) / chunk : 0;
+  if (nparts > 4096) {
+    nparts = 4096;
+    chunk = (n + nparts - 1) / nparts;
+    nparts = (n + chunk - 1) / chunk;
+  }
+  Part *parts = nullptr, *mine = nullptr, *all = nullptr;
+  double* dout = nullptr;
+  DT_CK(cudaMallocAsync(&parts, sizeof(Part) * (size_t)std::max<int64_t>(1, nparts), s));
+  DT_CK(cudaMallocAsync(&mine, sizeof(Part), s));
+  DT_CK(cudaMallocAsync(&all, sizeof(Part) * (size_t)world, s));
+  DT_CK(cudaMallocAsync(&dout, sizeof(double) * 4, s));
+  const int pr = prof_begin(PK_EVAL, s, 3);
+  if (nparts > 0)
+    eval_partial_kernel<false><<<(unsigned)nparts, 256, 0, s>>>(y, yhat, nullptr, nullptr, 0, nullptr, 0, n, chunk,
+                                                                parts);
+  eval_local_kernel<<<1, 1024, 0, s>>>(parts, (int)nparts, mine);
+  DT_CK(cudaGetLastError());
+  dt_status cst = comm_allgather(comm, mine, all, sizeof(Part), s);
+  if (cst != DT_OK) return cst;
+  eval_ranks_kernel<<<1, 32, 0, s>>>(all, world, p, dout);
+  prof_end(pr, s, 16.0 * (double)n);
+  DT_CK(cudaGetLastError());
+  double h[4];
+  DT_CK(cudaMemcpyAsync(h, dout, sizeof h, cudaMemcpyDeviceToHost, s));
+  DT_CK(cudaFreeAsync(parts, s));
+  DT_CK(cudaFreeAsync(mine, s));
+  DT_CK(cudaFreeAsync(all, s));
+  DT_CK(cudaFreeAsync(dout, s));
+  DT_CK(cudaStreamSynchronize(s));
+  out->mape = h[0];
+  out->r2 = h[1];
+  out->adj_r2 = h[2];
+  out->n = (int64_t)h[3];
   out->p = p;
   return DT_OK;
 }

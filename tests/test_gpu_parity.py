@@ -357,3 +357,38 @@ def test_importances_match_oracle(dt):
     want = oracle.importances(t.nodes, 16)
     np.testing.assert_allclose(got, want, rtol=1e-12, atol=1e-15)
     assert abs(got.sum() - 1.0) < 1e-12
+
+
+@pytest.mark.parametrize("world,sizes", [(2, [500_000, 500_001]), (3, [0, 17, 100_000]), (4, [1, 2, 3, 4])])
+def test_eval_sharded(dt, world, sizes):
+    """dt_eval_sharded over thread ranks: every rank gets bitwise the same metrics, equal
+    (1e-9 relative) to the oracle's metrics of the concatenated rows."""
+    import threading
+    rng = np.random.default_rng(world)
+    n = sum(sizes)
+    y = rng.uniform(1, 1e6, n)
+    yh = y * (1 + 0.1 * rng.standard_normal(n))
+    comms = dt.dt_comm_init_local(world)
+    offs = np.concatenate([[0], np.cumsum(sizes)])
+    out, errs = [None] * world, []
+
+    def run(r):
+        try:
+            s = torch.cuda.Stream()
+            with torch.cuda.stream(s):
+                a, b = offs[r], offs[r + 1]
+                out[r] = dt.dt_eval_sharded(comms[r], _cuda(y[a:b]), _cuda(yh[a:b]), 5, stream=s)
+        except Exception as e:  # pragma: no cover - reported below
+            errs.append(e)
+
+    th = [threading.Thread(target=run, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    assert not errs, errs
+    assert all(o == out[0] for o in out)
+    assert out[0]["n"] == n
+    mape, r2, adj = oracle.evaluate(y, yh, 5)
+    for got, want in ((out[0]["mape"], mape), (out[0]["r2"], r2), (out[0]["adj_r2"], adj)):
+        assert abs(got - want) <= 1e-9 * abs(want) + 1e-12

@@ -100,3 +100,55 @@ def test_feature_sharded_decomposition_gloo():
         p.join(timeout=60)
     assert sorted(r for r, _ in res) == [0, 1]
     assert all(ok for _, ok in res)
+
+
+def _eval_worker(rank, world, port, q):
+    """Row-sharded evaluation (dt_eval_sharded's decomposition): each rank reduces its rows
+    to (sum |e|/max(|y|, eps), SSE, n, mean, M2), the ranks all_gather the partials and
+    merge them in rank order (Chan); every rank must get the full-array metrics."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import oracle
+    rng = np.random.default_rng(0)
+    y = rng.uniform(1, 1e4, 1001)
+    yh = y + rng.standard_normal(1001) * 50
+    lo, hi = (0, 400) if rank == 0 else (400, 1001)
+    ys, hs = y[lo:hi], yh[lo:hi]
+    e = ys - hs
+    mean = ys.mean()
+    part = torch.tensor([np.sum(np.abs(e) / np.maximum(np.abs(ys), np.finfo(float).eps)), np.sum(e * e),
+                         float(len(ys)), mean, np.sum((ys - mean) ** 2)], dtype=torch.float64)
+    parts = [torch.zeros(5, dtype=torch.float64) for _ in range(world)]
+    dist.all_gather(parts, part)
+    ape = sse = n = m = M2 = 0.0
+    for p in parts:  # rank order
+        pa, ps, pn, pm, pM = p.tolist()
+        ape, sse = ape + pa, sse + ps
+        if n == 0:
+            n, m, M2 = pn, pm, pM
+        else:
+            tot = n + pn
+            delta = pm - m
+            m = m + delta * (pn / tot)
+            M2 = M2 + pM + delta * delta * (n * pn / tot)
+            n = tot
+    r2 = 1 - sse / M2
+    mape, r2o, _ = oracle.evaluate(y, yh, 3)
+    q.put((rank, abs(ape / n - mape) <= 1e-12 * mape and abs(r2 - r2o) <= 1e-12 * abs(r2o) and n == 1001))
+    dist.destroy_process_group()
+
+
+def test_row_sharded_eval_decomposition_gloo():
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_eval_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    assert sorted(r for r, _ in res) == [0, 1]
+    assert all(ok for _, ok in res)
