@@ -146,7 +146,7 @@ class Tree:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h is not None and h.value and getattr(self, "_owner", None) is None:
+        if h is not None and h.value and getattr(self, "_owner", None) is None and _lib is not None:
             _lib.dt_tree_free(h)
         self._h = None
 
@@ -365,7 +365,7 @@ class Comm:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h is not None and h.value:
+        if h is not None and h.value and _lib is not None:
             _lib.dt_comm_free(h)
             self._h = None
 
@@ -415,7 +415,7 @@ class Forest:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h is not None and h.value:
+        if h is not None and h.value and _lib is not None:
             _lib.dt_forest_free(h)
         self._h = None
 

@@ -525,26 +525,68 @@ struct DseMap {
   uint8_t code[256];  // tree feature f -> 0x80 | GPU column, or CNN column
 };
 
-template <bool kSmemTree, int kR>
+template <bool kSmemTree, bool kSorted, int kR>
 __global__ void __launch_bounds__(1024, 1)
 predict_dse_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ value, int count, int depth,
                    const float* __restrict__ cnn, int64_t n_cnn, int dc, const float* __restrict__ gpu,
-                   int n_gpu, int dg, DseMap map, double* __restrict__ yhat) {
+                   int n_gpu, int dg, int p2, DseMap map, double* __restrict__ yhat) {
   extern __shared__ __align__(16) unsigned char dse_smem[];
   uint2* snodes = reinterpret_cast<uint2*>(dse_smem);
   float* gpu_t = reinterpret_cast<float*>(dse_smem + (kSmemTree ? sizeof(uint2) * (size_t)count : 0));
   float* cnn_s = gpu_t + (size_t)dg * n_gpu;
+  // kSorted: sort keys (p2 >= n_gpu, a power of two), the GPU order, output staging
+  unsigned long long* skey = reinterpret_cast<unsigned long long*>(
+      reinterpret_cast<unsigned char*>(cnn_s) + ((sizeof(float) * kR * dc + 15) & ~(size_t)15));
+  uint32_t* perm = reinterpret_cast<uint32_t*>(skey + (kSorted ? p2 : 0));
+  double* out_s = reinterpret_cast<double*>(perm + (kSorted ? ((n_gpu + 3) & ~3) : 0));
   const int tid = threadIdx.x;
+  auto recode = [&](uint2 nd) {
+    nd.y = ((uint32_t)map.code[nd.y >> 24] << 24) | (nd.y & 0xFFFFFFu);
+    return nd;
+  };
   if (kSmemTree) {
-    for (int k = tid; k < count; k += blockDim.x) {
-      uint2 nd = gnodes[k];
-      nd.y = ((uint32_t)map.code[nd.y >> 24] << 24) | (nd.y & 0xFFFFFFu);
-      snodes[k] = nd;
+    for (int k = tid; k < count; k += blockDim.x) snodes[k] = recode(gnodes[k]);
+    __syncthreads();
+  }
+  if (kSorted) {
+    // GPU rows grouped by the leaf they reach with CNN row 0: neighbouring threads then
+    // share most of their GPU-side decisions for any CNN, so a warp's node reads hit
+    // fewer distinct shared-memory words (broadcasts instead of bank conflicts).
+    for (int j = tid; j < p2; j += blockDim.x) {
+      unsigned long long key = ~0ull;
+      if (j < n_gpu) {
+        uint32_t k = 0;
+        for (int l = 0; l < depth; ++l) {
+          const uint2 nd = kSmemTree ? snodes[k] : recode(__ldg(gnodes + k));
+          const uint32_t code = nd.y >> 24, left = nd.y & 0xFFFFFFu;
+          const float x = (code & 0x80u) ? __ldg(gpu + (int64_t)j * dg + (code & 0x7Fu)) : __ldg(cnn + code);
+          k = (x > __uint_as_float(nd.x)) ? left + 1 : left;
+        }
+        key = ((unsigned long long)k << 32) | (uint32_t)j;
+      }
+      skey[j] = key;
     }
+    __syncthreads();
+    for (int kk = 2; kk <= p2; kk <<= 1) {  // bitonic sort of (leaf, row)
+      for (int jj = kk >> 1; jj > 0; jj >>= 1) {
+        for (int i = tid; i < p2; i += blockDim.x) {
+          const int ixj = i ^ jj;
+          if (ixj > i) {
+            const unsigned long long u = skey[i], v = skey[ixj];
+            const bool up = (i & kk) == 0;
+            if ((u > v) == up) { skey[i] = v; skey[ixj] = u; }
+          }
+        }
+        __syncthreads();
+      }
+    }
+    for (int j = tid; j < n_gpu; j += blockDim.x) perm[j] = (uint32_t)skey[j];
+    __syncthreads();
   }
   for (int e = tid; e < dg * n_gpu; e += blockDim.x) {
     const int g = e / n_gpu, j = e - g * n_gpu;
-    gpu_t[e] = __ldg(gpu + (int64_t)j * dg + g);
+    const int src = kSorted ? (int)perm[j] : j;
+    gpu_t[e] = __ldg(gpu + (int64_t)src * dg + g);
   }
   const int64_t nblk = (n_cnn + kR - 1) / kR;
   for (int64_t b = blockIdx.x; b < nblk; b += gridDim.x) {
@@ -562,13 +604,7 @@ predict_dse_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ 
       for (int l = 0; l < depth; ++l) {
 #pragma unroll
         for (int r = 0; r < kR; ++r) {
-          uint2 nd;
-          if (kSmemTree) {
-            nd = snodes[k[r]];
-          } else {
-            nd = __ldg(gnodes + k[r]);
-            nd.y = ((uint32_t)map.code[nd.y >> 24] << 24) | (nd.y & 0xFFFFFFu);
-          }
+          const uint2 nd = kSmemTree ? snodes[k[r]] : recode(__ldg(gnodes + k[r]));
           const uint32_t code = nd.y >> 24, left = nd.y & 0xFFFFFFu;
           const float* src = (code & 0x80u) ? gpu_t + (code & 0x7Fu) * (uint32_t)n_gpu + j
                                             : cnn_s + r * dc + code;
@@ -577,8 +613,17 @@ predict_dse_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ 
         }
       }
 #pragma unroll
-      for (int r = 0; r < kR; ++r)
-        if (i0 + r < n_cnn) yhat[(i0 + r) * (int64_t)n_gpu + j] = __ldg(value + k[r]);
+      for (int r = 0; r < kR; ++r) {
+        if (kSorted) out_s[r * n_gpu + perm[j]] = __ldg(value + k[r]);
+        else if (i0 + r < n_cnn) yhat[(i0 + r) * (int64_t)n_gpu + j] = __ldg(value + k[r]);
+      }
+    }
+    if (kSorted) {  // the staged rows, in GPU order, coalesced
+      __syncthreads();
+      for (int e = tid; e < kR * n_gpu; e += blockDim.x) {
+        const int r = e / n_gpu;
+        if (i0 + r < n_cnn) yhat[i0 * (int64_t)n_gpu + e] = out_s[e];
+      }
     }
   }
 }
@@ -599,19 +644,31 @@ dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, in
     }
   }
   constexpr int kR = 2, kThr = 1024;
-  const size_t tables = sizeof(float) * ((size_t)dg * (size_t)n_gpu + (size_t)kR * dc);
+  const size_t cnn_bytes = (sizeof(float) * kR * (size_t)dc + 15) & ~(size_t)15;
+  const size_t tables = sizeof(float) * (size_t)dg * (size_t)n_gpu + cnn_bytes;
+  int p2 = 1;
+  while (p2 < n_gpu) p2 <<= 1;
+  const size_t sort_bytes = sizeof(unsigned long long) * (size_t)p2 + sizeof(uint32_t) * (size_t)((n_gpu + 3) & ~3) +
+                            sizeof(double) * kR * (size_t)n_gpu;
   const size_t tree = sizeof(uint2) * (size_t)t->count;
   const size_t cap = 227 * 1024;
   if (tables > cap) return fail(DT_ERR_TOO_LARGE, "dt_predict_dse: GPU table too large for shared memory");
+  static int sort_env = -1;
+  if (sort_env < 0) {
+    const char* e = getenv("DT_DSE_SORT");
+    sort_env = (e && e[0] == '0') ? 0 : 1;
+  }
   const bool smem_tree = tree + tables <= cap;
-  const size_t sm = (smem_tree ? tree : 0) + tables;
-  auto kern = smem_tree ? predict_dse_kernel<true, kR> : predict_dse_kernel<false, kR>;
+  const bool sorted = sort_env && (smem_tree ? tree : 0) + tables + sort_bytes <= cap;
+  const size_t sm = (smem_tree ? tree : 0) + tables + (sorted ? sort_bytes : 0);
+  auto kern = smem_tree ? (sorted ? predict_dse_kernel<true, true, kR> : predict_dse_kernel<true, false, kR>)
+                        : (sorted ? predict_dse_kernel<false, true, kR> : predict_dse_kernel<false, false, kR>);
   DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
   const int64_t nblk = (n_cnn + kR - 1) / kR;
   const int64_t g = std::min<int64_t>((int64_t)num_sms(), nblk);
   const int pr = prof_begin(PK_PREDICT, s, 1);
   kern<<<(unsigned)g, kThr, sm, s>>>(t->dev_packed, t->dev_value, (int)t->count, t->depth, cnn, n_cnn, dc, gpu,
-                                     (int)n_gpu, dg, map, yhat);
+                                     (int)n_gpu, dg, p2, map, yhat);
   prof_end(pr, s, 8.0 * (double)n_cnn * (double)n_gpu);  // the yhat write (inputs are O(n_cnn + n_gpu))
   DT_CK(cudaGetLastError());
   return DT_OK;
