@@ -77,7 +77,7 @@ struct Ctl {
   // root reduction
   double ysum, ymin, ymax, ysc;
   int32_t all_integral;
-  int32_t pad;
+  int32_t y32;  // the level lists hold y as int32 (Reading R24)
   // chunk lists of the level (single-segment chunks from the front, others from the back)
   uint32_t scnt[2];  // scan: singles, others
   uint32_t pcnt[2];  // partition: singles, others
@@ -230,6 +230,9 @@ __global__ void root_finalize_kernel(const RootPart* parts, int nparts, int64_t 
   const double amax = fmax(fabs(mn), fabs(mx));
   // Reading R17: integer mode iff every y integral and max|y| * n < 2^52.
   ctl->int_mode = (integral && finite && amax * (double)n < 4503599627370496.0) ? 1 : 0;
+  // Reading R24: integral targets with |y| < 2^31 travel through the level lists as int32
+  // (4 B instead of 8 per entry; converted exactly to f64 where used)
+  ctl->y32 = (ctl->int_mode && amax < 2147483647.0) ? 1 : 0;
 }
 
 // S'_0 = sum (y - c0) over all rows (second pass; c0 from the finalised root sum).
@@ -316,13 +319,16 @@ __global__ void __launch_bounds__(256) presort_build_kernel(const uint32_t* __re
                                                             const uint32_t* __restrict__ vals,
                                                             const double* __restrict__ y, int64_t total,
                                                             float* __restrict__ lx, uint32_t* __restrict__ lr,
-                                                            double* __restrict__ ly) {
+                                                            double* __restrict__ ly, const Ctl* ctl) {
+  const bool y32 = ctl->y32 != 0;
   for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < total;
        p += (int64_t)gridDim.x * blockDim.x) {
     const uint32_t r = vals[p];
     lx[p] = unflip_f32(keys[p]);
     lr[p] = r;
-    ly[p] = __ldg(y + r);
+    const double v = __ldg(y + r);
+    if (y32) reinterpret_cast<int32_t*>(ly)[p] = (int32_t)v;
+    else ly[p] = v;
   }
 }
 
@@ -648,27 +654,48 @@ __device__ __forceinline__ double split_gain_approx_d(double sl, double sc, doub
 
 // Loads kItems consecutive x (f32) and y (f64) entries starting at p0 (vectorised when
 // the whole run is in bounds; p0 is a multiple of kItems, so 16-byte aligned).
-__device__ __forceinline__ void load_items(const float* __restrict__ lx, const double* __restrict__ ly,
-                                           int64_t p0, int64_t total, float* xv, double* yv) {
-  if (p0 + kItems <= total) {
-    const float4* x4 = reinterpret_cast<const float4*>(lx + p0);
-    const double2* y2 = reinterpret_cast<const double2*>(ly + p0);
+// y list element p: int32 storage when y32 (Reading R24), else f64.
+__device__ __forceinline__ double yget(const double* __restrict__ ly, int64_t p, bool y32) {
+  return y32 ? (double)reinterpret_cast<const int32_t*>(ly)[p] : ly[p];
+}
+
+// kItems consecutive y entries from p0 (p0 + kItems <= total; p0 a multiple of kItems).
+__device__ __forceinline__ void load_y_vec(const double* __restrict__ ly, int64_t p0, bool y32, double* yv) {
+  if (y32) {
+    const int4* y4 = reinterpret_cast<const int4*>(reinterpret_cast<const int32_t*>(ly) + p0);
 #pragma unroll
     for (int j = 0; j < kItems / 4; ++j) {
-      const float4 t = __ldcs(x4 + j);
-      xv[4 * j] = t.x; xv[4 * j + 1] = t.y; xv[4 * j + 2] = t.z; xv[4 * j + 3] = t.w;
+      const int4 t = __ldcs(y4 + j);
+      yv[4 * j] = (double)t.x; yv[4 * j + 1] = (double)t.y; yv[4 * j + 2] = (double)t.z; yv[4 * j + 3] = (double)t.w;
     }
+  } else {
+    const double2* y2 = reinterpret_cast<const double2*>(ly + p0);
 #pragma unroll
     for (int j = 0; j < kItems / 2; ++j) {
       const double2 t = __ldcs(y2 + j);
       yv[2 * j] = t.x; yv[2 * j + 1] = t.y;
     }
+  }
+}
+
+// Loads kItems consecutive x (f32) and y entries starting at p0 (vectorised when the
+// whole run is in bounds; p0 is a multiple of kItems, so 16-byte aligned).
+__device__ __forceinline__ void load_items(const float* __restrict__ lx, const double* __restrict__ ly,
+                                           int64_t p0, int64_t total, float* xv, double* yv, bool y32) {
+  if (p0 + kItems <= total) {
+    const float4* x4 = reinterpret_cast<const float4*>(lx + p0);
+#pragma unroll
+    for (int j = 0; j < kItems / 4; ++j) {
+      const float4 t = __ldcs(x4 + j);
+      xv[4 * j] = t.x; xv[4 * j + 1] = t.y; xv[4 * j + 2] = t.z; xv[4 * j + 3] = t.w;
+    }
+    load_y_vec(ly, p0, y32, yv);
   } else {
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
       const bool ok = p0 + j < total;
       xv[j] = ok ? lx[p0 + j] : 0.f;
-      yv[j] = ok ? ly[p0 + j] : 0.0;
+      yv[j] = ok ? yget(ly, p0 + j, y32) : 0.0;
     }
   }
 }
@@ -707,17 +734,13 @@ __device__ __forceinline__ SumP thread_sum_agg(const ScanArgs& a, uint32_t K, ui
   return tagg;
 }
 
-__device__ __forceinline__ void load_y(const double* __restrict__ ly, int64_t p0, int64_t total, double* yv) {
+__device__ __forceinline__ void load_y(const double* __restrict__ ly, int64_t p0, int64_t total, double* yv,
+                                       bool y32) {
   if (p0 + kItems <= total) {
-    const double2* y2 = reinterpret_cast<const double2*>(ly + p0);
-#pragma unroll
-    for (int j = 0; j < kItems / 2; ++j) {
-      const double2 t = __ldcs(y2 + j);
-      yv[2 * j] = t.x; yv[2 * j + 1] = t.y;
-    }
+    load_y_vec(ly, p0, y32, yv);
   } else {
 #pragma unroll
-    for (int j = 0; j < kItems; ++j) yv[j] = (p0 + j < total) ? ly[p0 + j] : 0.0;
+    for (int j = 0; j < kItems; ++j) yv[j] = (p0 + j < total) ? yget(ly, p0 + j, y32) : 0.0;
   }
 }
 
@@ -737,10 +760,11 @@ __global__ void __launch_bounds__(kThreads) scan_agg_kernel(ScanArgs a) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const bool y32 = a.ctl->y32 != 0;
   double yn[kItems];
   {
     const int64_t q0 = gw * kChunkW + lane * kItems;
-    if (gw < nch && q0 < total) load_y(a.ly, q0, total, yn);
+    if (gw < nch && q0 < total) load_y(a.ly, q0, total, yn, y32);
   }
   for (int64_t ch = gw; ch < nch; ch += nw) {
     const int64_t p0 = ch * kChunkW + lane * kItems;
@@ -750,7 +774,7 @@ __global__ void __launch_bounds__(kThreads) scan_agg_kernel(ScanArgs a) {
     for (int j = 0; j < kItems; ++j) yv[j] = yn[j];
     {
       const int64_t q0 = (ch + nw) * kChunkW + lane * kItems;
-      if (ch + nw < nch && q0 < total) load_y(a.ly, q0, total, yn);
+      if (ch + nw < nch && q0 < total) load_y(a.ly, q0, total, yn, y32);
     }
     const ChunkDesc dsc = a.desc[ch];
     if (dsc.start <= ch * kChunkW && dsc.end >= ch * kChunkW + kChunkW) {
@@ -995,15 +1019,17 @@ __global__ void __launch_bounds__(kThreads, 3) scan_single_kernel(ScanArgs a) {
                   wib * kScanStages;
   CompactBuf* cbuf = reinterpret_cast<CompactBuf*>(scan_smem + (sizeof(ScanStage) + sizeof(uint64_t)) * kScanStages *
                                                                    (kThreads / 32));
+  const bool y32 = a.ctl->y32 != 0;
+  const uint32_t ybytes = (uint32_t)(y32 ? sizeof(int32_t) : sizeof(double)) * kChunkW;
   auto issue = [&](int s, int64_t ch) {  // lane 0
     ScanStage& t = st[s];
     t.ch = (uint32_t)ch;
-    const uint32_t bytes = (uint32_t)(sizeof(t.x) + sizeof(t.y) + sizeof(ChunkDesc) + 2 * sizeof(SumP)) +
+    const uint32_t bytes = (uint32_t)(sizeof(t.x) + sizeof(ChunkDesc) + 2 * sizeof(SumP)) + ybytes +
                            (ch > 0 ? 16u : 0u);
     fence_proxy_async_smem();
     mbar_arrive_expect_tx(bar + s, bytes);
     bulk_g2s(t.x, a.lx + ch * kChunkW, sizeof(t.x), bar + s);
-    bulk_g2s(t.y, a.ly + ch * kChunkW, sizeof(t.y), bar + s);
+    bulk_g2s(t.y, reinterpret_cast<const char*>(a.ly) + ch * (int64_t)ybytes, ybytes, bar + s);
     bulk_g2s(&t.d, a.desc + ch, sizeof(ChunkDesc), bar + s);
     bulk_g2s(&t.cb, a.block_carry + ch / kBlockChunks, sizeof(SumP), bar + s);
     bulk_g2s(&t.ce, a.chunk_excl + ch, sizeof(SumP), bar + s);
@@ -1033,10 +1059,19 @@ __global__ void __launch_bounds__(kThreads, 3) scan_single_kernel(ScanArgs a) {
         const float4 q = x4[j];
         xv[4 * j] = q.x; xv[4 * j + 1] = q.y; xv[4 * j + 2] = q.z; xv[4 * j + 3] = q.w;
       }
+      if (y32) {
+        const int4* y4 = reinterpret_cast<const int4*>(reinterpret_cast<const int32_t*>(t.y) + lane * kItems);
 #pragma unroll
-      for (int j = 0; j < kItems / 2; ++j) {
-        const double2 q = y2[j];
-        yv[2 * j] = q.x; yv[2 * j + 1] = q.y;
+        for (int j = 0; j < kItems / 4; ++j) {
+          const int4 q = y4[j];
+          yv[4 * j] = (double)q.x; yv[4 * j + 1] = (double)q.y; yv[4 * j + 2] = (double)q.z; yv[4 * j + 3] = (double)q.w;
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < kItems / 2; ++j) {
+          const double2 q = y2[j];
+          yv[2 * j] = q.x; yv[2 * j + 1] = q.y;
+        }
       }
     }
     const ChunkDesc dsc = t.d;
@@ -1079,10 +1114,11 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
   const int64_t ng = a.ctl->scnt[1];
   float xn[kItems];
   double yn[kItems];
+  const bool y32 = a.ctl->y32 != 0;
   int64_t ch_next = (gw < ng) ? (int64_t)a.list[nch - 1 - gw] : 0;
   {
     const int64_t q0 = ch_next * kChunkW + lane * kItems;
-    if (gw < ng && q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
+    if (gw < ng && q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn, y32);
   }
   for (int64_t idx = gw; idx < ng; idx += nw) {
     const int64_t ch = ch_next;
@@ -1095,7 +1131,7 @@ __global__ void __launch_bounds__(kThreads, 2) scan_kernel(ScanArgs a) {
     if (idx + nw < ng) {
       ch_next = (int64_t)a.list[nch - 1 - (idx + nw)];
       const int64_t q0 = ch_next * kChunkW + lane * kItems;
-      if (q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn);
+      if (q0 < total) load_items(a.lx, a.ly, q0, total, xn, yn, y32);
     }
     const ChunkDesc dsc = a.desc[ch];
     Seg sg{0, 0, 0, 0u, 0};
@@ -1992,19 +2028,29 @@ __global__ void __launch_bounds__(kSmem ? kAggSmemThreads : kThreads) part_agg_k
 
 // Phase C, one chunk inside ONE segment of a split node: ranks from the chunk's go-left
 // ballots plus one carry; each child's entries of a row go to consecutive addresses.
-__device__ __forceinline__ void partition_single_chunk(const PartArgs& a, uint64_t A2, int64_t ch) {
+// y moves as raw bits: 4 B (y32) or 8 B per entry.
+__device__ __forceinline__ unsigned long long yload_raw(const double* __restrict__ ly, int64_t p, bool y32) {
+  return y32 ? (unsigned long long)__ldcs(reinterpret_cast<const unsigned int*>(ly) + p)
+             : (unsigned long long)__ldcs(reinterpret_cast<const unsigned long long*>(ly) + p);
+}
+__device__ __forceinline__ void ystore_raw(double* __restrict__ oy, int64_t o, unsigned long long v, bool y32) {
+  if (y32) reinterpret_cast<unsigned int*>(oy)[o] = (unsigned int)v;
+  else reinterpret_cast<unsigned long long*>(oy)[o] = v;
+}
+
+__device__ __forceinline__ void partition_single_chunk(const PartArgs& a, uint64_t A2, int64_t ch, bool y32) {
   const int lane = threadIdx.x & 31;
   const uint32_t lt_mask = (1u << lane) - 1u;
   const int64_t wbase = ch * kChunkW;
   uint32_t rv[kRows];
   float xv[kRows];
-  double yv[kRows];
+  unsigned long long yv[kRows];
 #pragma unroll
   for (int r = 0; r < kRows; ++r) {
     const int64_t p = wbase + r * 32 + lane;
     rv[r] = __ldcs(a.lr + p);
     xv[r] = __ldcs(a.lx + p);
-    yv[r] = __ldcs(a.ly + p);
+    yv[r] = yload_raw(a.ly, p, y32);
   }
   const PartDesc dsc = a.desc[ch];
   const uint32_t mword = (lane < kRows) ? __ldcs(a.gmask + ch * kRows + lane) : 0u;
@@ -2013,7 +2059,7 @@ __device__ __forceinline__ void partition_single_chunk(const PartArgs& a, uint64
   const uint32_t nsl = dsc.ns + dsc.nl;
   float* const ox = a.ox + (int64_t)dsc.f * (int64_t)A2;
   uint32_t* const orow = a.orow + (int64_t)dsc.f * (int64_t)A2;
-  double* const oy = a.oy + (int64_t)dsc.f * (int64_t)A2;
+  const int64_t ybase = (int64_t)dsc.f * (int64_t)A2;
 #pragma unroll
   for (int r = 0; r < kRows; ++r) {
     const uint32_t gm = __shfl_sync(0xffffffffu, mword, r);
@@ -2023,27 +2069,27 @@ __device__ __forceinline__ void partition_single_chunk(const PartArgs& a, uint64
     const uint32_t dst = g ? dsc.ns + rank : nsl + (i - rank);
     ox[dst] = xv[r];
     orow[dst] = rv[r];
-    oy[dst] = yv[r];
+    ystore_raw(a.oy, ybase + dst, yv[r], y32);
     carry += __popc(gm);
   }
 }
 
 // Phase C, one chunk with segment boundaries inside.
 __device__ __forceinline__ void partition_general_chunk(const PartArgs& a, uint32_t K, uint64_t A, uint64_t A2,
-                                                      int64_t total, int64_t ch) {
+                                                      int64_t total, int64_t ch, bool y32) {
   const int lane = threadIdx.x & 31;
   const uint32_t lt_mask = (1u << lane) - 1u;
   const int64_t wbase = ch * kChunkW;
   uint32_t rv[kRows];
   float xv[kRows];
-  double yv[kRows];
+  unsigned long long yv[kRows];
 #pragma unroll
   for (int r = 0; r < kRows; ++r) {
     const int64_t p = wbase + r * 32 + lane;
     const bool ok = p < total;
     rv[r] = ok ? __ldcs(a.lr + p) : 0u;
     xv[r] = ok ? __ldcs(a.lx + p) : 0.f;
-    yv[r] = ok ? __ldcs(a.ly + p) : 0.0;
+    yv[r] = ok ? yload_raw(a.ly, p, y32) : 0ull;
   }
   const PartDesc dsc = a.desc[ch];
   // raw go-left bits of my kRows entries, from the chunk's ballots (phase A)
@@ -2093,7 +2139,7 @@ __device__ __forceinline__ void partition_general_chunk(const PartArgs& a, uint3
         const int64_t o = obase + dst;
         a.ox[o] = xv[r];
         a.orow[o] = rv[r];
-        a.oy[o] = yv[r];
+        ystore_raw(a.oy, o, yv[r], y32);
       }
     }
     if (hm) {
@@ -2117,9 +2163,10 @@ __global__ void __launch_bounds__(kThreads, 4) partition_kernel(PartArgs a) {
   const int64_t ns = a.ctl->pcnt[0], ng = a.ctl->pcnt[1];
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const bool y32 = a.ctl->y32 != 0;
   for (int64_t idx = gw; idx < ns + ng; idx += nw) {
-    if (idx < ns) partition_single_chunk(a, A2, (int64_t)a.list[idx]);
-    else partition_general_chunk(a, K, A, A2, total, (int64_t)a.list[nch - 1 - (idx - ns)]);
+    if (idx < ns) partition_single_chunk(a, A2, (int64_t)a.list[idx], y32);
+    else partition_general_chunk(a, K, A, A2, total, (int64_t)a.list[nch - 1 - (idx - ns)], y32);
   }
 }
 
@@ -2381,7 +2428,7 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     }
     const int gb = std::max(1, std::min<int>((int)((total0 + 255) / 256), num_sms() * 8));
     pr = prof_begin(PK_PRESORT_BUILD, s, 1);
-    presort_build_kernel<<<gb, 256, 0, s>>>(sk, sv, y, total0, b.lx[0], b.lr[0], b.ly[0]);
+    presort_build_kernel<<<gb, 256, 0, s>>>(sk, sv, y, total0, b.lx[0], b.lr[0], b.ly[0], ctl);
     prof_end(pr, s, 36.0 * (double)total0);  // (key, val) read, y gathered, 16 B written
     DT_CK(cudaGetLastError());
   }
@@ -2595,17 +2642,18 @@ dt_status fit_finish(const FitBufs& b, int32_t d, cudaStream_t s, const std::vec
   DT_CK(cudaStreamSynchronize(s));
   if (pending) {
     // algorithmic bytes per launch:
-    //   scan: every active entry of the scanned lists, x (4 B) + y (8 B);
+    //   scan: every active entry of the scanned lists, x (4 B) + y (8 B, or 4 B as int32);
     //   goleft: the split feature's row ids of the moved rows (4 B, left rows only read, counted
     //           for all) + one bit per row;
-    //   partition: every moved entry read (16 B) and written (16 B).
+    //   partition: every moved entry read and written (x 4 + row 4 + y 8 or 4 B, each way).
     for (const Pending& p : *pending) {
       if (p.rec < 0 || p.level >= kMaxLogLevels) continue;
       const LevelLog& L = hlog[(size_t)p.level];
       double bytes = 0.0;
-      if (p.kind == PK_SCAN) bytes = 12.0 * (double)L.A * p.dl;
+      const double yb = hc.y32 ? 4.0 : 8.0;  // y bytes per entry (Reading R24)
+      if (p.kind == PK_SCAN) bytes = (4.0 + yb) * (double)L.A * p.dl;
       else if (p.kind == PK_GOLEFT) bytes = 4.125 * (double)L.A_next;
-      else if (p.kind == PK_PARTITION) bytes = 32.0 * (double)L.A_next * p.dl;
+      else if (p.kind == PK_PARTITION) bytes = 2.0 * (8.0 + yb) * (double)L.A_next * p.dl;
       prof_set_bytes(p.rec, bytes);
     }
   }
