@@ -751,57 +751,112 @@ constexpr int kChunkW = 32 * kItems;           // 256 entries
 constexpr int kBlockChunks = 1024 * 2;         // chunks per phase-B1 block
 
 // Phase A: per-chunk segmented aggregate of (y - c) (reads y only).
+// One chunk's segmented aggregate of (y - c) into chunk_agg[ch].
+__device__ __forceinline__ void agg_chunk(const ScanArgs& a, uint32_t K, uint64_t A, int64_t total, int64_t ch,
+                                          const double* yv, const ChunkDesc& dsc) {
+  const int lane = threadIdx.x & 31;
+  const int64_t p0 = ch * kChunkW + lane * kItems;
+  const bool any = p0 < total;
+  if (dsc.start <= ch * kChunkW && dsc.end >= ch * kChunkW + kChunkW) {
+    // whole chunk in one segment: the general path's sums without the segment logic
+    const bool head = dsc.start == ch * kChunkW;
+    const double c = dsc.c;
+    double t = (head && lane == 0) ? __dsub_rn(yv[0], c) : __dadd_rn(0.0, __dsub_rn(yv[0], c));
+#pragma unroll
+    for (int j = 1; j < kItems; ++j) t = __dadd_rn(t, __dsub_rn(yv[j], c));
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const double o = __shfl_up_sync(0xffffffffu, t, d);
+      if (lane >= d) t = __dadd_rn(o, t);
+    }
+    if (lane == 31) a.chunk_agg[ch] = SumP{head ? 1u : 0u, t};
+    return;
+  }
+  Seg sg{0, 0, 0, 0u, 0};
+  if (any) seg_from(sg, dsc.start, dsc.end, dsc.k, dsc.f, A, p0, a.nodes, K);
+  const bool one_seg = any && (p0 + kItems <= total) && (sg.end >= p0 + kItems);
+  const bool warp_fast = __all_sync(0xffffffffu, one_seg || !any);
+  const bool head0 = any && (p0 == sg.start);
+  const double c_in = (sg.k == dsc.k && sg.f == dsc.f) ? dsc.c : __ldg(&a.nodes[sg.k].c);
+  const SumP tagg = thread_sum_agg(a, K, A, p0, total, any, warp_fast, head0, sg, yv, c_in);
+  SumP wagg;
+  (void)warp_exclusive_scan(tagg, SumP{0u, 0.0}, wagg);
+  if (lane == 0) a.chunk_agg[ch] = wagg;
+}
+
+// Phase A over the level's full chunks with a per-warp TMA pipeline (kAggStages chunks of
+// y and their descriptors in flight per warp: the pass is a pure stream of y); a partial
+// last chunk goes through registers.
+constexpr int kAggStages = 3;
+struct __align__(128) AggStage {
+  double y[kChunkW];  // 256 f64 or 256 int32 (first half)
+  ChunkDesc d;
+};
+constexpr size_t kScanAggSmem = (sizeof(AggStage) + sizeof(uint64_t)) * kAggStages * (kThreads / 32);
+
 __global__ void __launch_bounds__(kThreads) scan_agg_kernel(ScanArgs a) {
+  extern __shared__ __align__(128) unsigned char agg_smem[];
   const uint32_t K = a.ctl->K[a.parity];
   const uint64_t A = a.ctl->A[a.parity];
   if (K == 0 || A == 0) return;
   const int64_t total = (int64_t)A * a.dl;
-  const int64_t nch = (total + kChunkW - 1) / kChunkW;
-  const int lane = threadIdx.x & 31;
+  const int64_t nfull = total / kChunkW;
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const bool y32 = a.ctl->y32 != 0;
-  double yn[kItems];
-  {
-    const int64_t q0 = gw * kChunkW + lane * kItems;
-    if (gw < nch && q0 < total) load_y(a.ly, q0, total, yn, y32);
-  }
-  for (int64_t ch = gw; ch < nch; ch += nw) {
-    const int64_t p0 = ch * kChunkW + lane * kItems;
-    const bool any = p0 < total;
+  if (gw == 0 && nfull * kChunkW < total) {  // the partial last chunk
     double yv[kItems];
+    const int64_t p0 = nfull * kChunkW + lane * kItems;
 #pragma unroll
-    for (int j = 0; j < kItems; ++j) yv[j] = yn[j];
-    {
-      const int64_t q0 = (ch + nw) * kChunkW + lane * kItems;
-      if (ch + nw < nch && q0 < total) load_y(a.ly, q0, total, yn, y32);
-    }
-    const ChunkDesc dsc = a.desc[ch];
-    if (dsc.start <= ch * kChunkW && dsc.end >= ch * kChunkW + kChunkW) {
-      // whole chunk in one segment: the general path's sums without the segment logic
-      const bool head = dsc.start == ch * kChunkW;
-      const double c = dsc.c;
-      double t = (head && lane == 0) ? __dsub_rn(yv[0], c) : __dadd_rn(0.0, __dsub_rn(yv[0], c));
+    for (int j = 0; j < kItems; ++j) yv[j] = 0.0;
+    if (p0 < total) load_y(a.ly, p0, total, yv, y32);
+    agg_chunk(a, K, A, total, nfull, yv, a.desc[nfull]);
+  }
+  if (gw >= nfull) return;  // warp-uniform
+  AggStage* st = reinterpret_cast<AggStage*>(agg_smem) + wib * kAggStages;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(agg_smem + sizeof(AggStage) * kAggStages * (kThreads / 32)) +
+                  wib * kAggStages;
+  const uint32_t ybytes = (uint32_t)(y32 ? sizeof(int32_t) : sizeof(double)) * kChunkW;
+  auto issue = [&](int q, int64_t ch) {  // lane 0
+    fence_proxy_async_smem();
+    mbar_arrive_expect_tx(bar + q, ybytes + (uint32_t)sizeof(ChunkDesc));
+    bulk_g2s(st[q].y, reinterpret_cast<const char*>(a.ly) + ch * (int64_t)ybytes, ybytes, bar + q);
+    bulk_g2s(&st[q].d, a.desc + ch, sizeof(ChunkDesc), bar + q);
+  };
+  if (lane == 0) {
+    for (int q = 0; q < kAggStages; ++q) mbar_init(bar + q, 1);
+    mbar_init_fence();
+    for (int q = 0; q < kAggStages; ++q)
+      if (gw + q * nw < nfull) issue(q, gw + q * nw);
+  }
+  __syncwarp();
+  int q = 0;
+  uint32_t phase = 0;
+  for (int64_t ch = gw; ch < nfull; ch += nw) {
+    mbar_wait(bar + q, phase);
+    double yv[kItems];
+    if (y32) {
+      const int4* y4 = reinterpret_cast<const int4*>(reinterpret_cast<const int32_t*>(st[q].y) + lane * kItems);
 #pragma unroll
-      for (int j = 1; j < kItems; ++j) t = __dadd_rn(t, __dsub_rn(yv[j], c));
-#pragma unroll
-      for (int d = 1; d < 32; d <<= 1) {
-        const double o = __shfl_up_sync(0xffffffffu, t, d);
-        if (lane >= d) t = __dadd_rn(o, t);
+      for (int j = 0; j < kItems / 4; ++j) {
+        const int4 v = y4[j];
+        yv[4 * j] = (double)v.x; yv[4 * j + 1] = (double)v.y; yv[4 * j + 2] = (double)v.z; yv[4 * j + 3] = (double)v.w;
       }
-      if (lane == 31) a.chunk_agg[ch] = SumP{head ? 1u : 0u, t};
-      continue;
+    } else {
+      const double2* y2 = reinterpret_cast<const double2*>(st[q].y + lane * kItems);
+#pragma unroll
+      for (int j = 0; j < kItems / 2; ++j) {
+        const double2 v = y2[j];
+        yv[2 * j] = v.x; yv[2 * j + 1] = v.y;
+      }
     }
-    Seg sg{0, 0, 0, 0u, 0};
-    if (any) seg_from(sg, dsc.start, dsc.end, dsc.k, dsc.f, A, p0, a.nodes, K);
-    const bool one_seg = any && (p0 + kItems <= total) && (sg.end >= p0 + kItems);
-    const bool warp_fast = __all_sync(0xffffffffu, one_seg || !any);
-    const bool head0 = any && (p0 == sg.start);
-    const double c_in = (sg.k == dsc.k && sg.f == dsc.f) ? dsc.c : __ldg(&a.nodes[sg.k].c);
-    const SumP tagg = thread_sum_agg(a, K, A, p0, total, any, warp_fast, head0, sg, yv, c_in);
-    SumP wagg;
-    (void)warp_exclusive_scan(tagg, SumP{0u, 0.0}, wagg);
-    if (lane == 0) a.chunk_agg[ch] = wagg;
+    const ChunkDesc dsc = st[q].d;
+    __syncwarp();  // every lane has read the stage
+    const int64_t nxt = ch + kAggStages * nw;
+    if (lane == 0 && nxt < nfull) issue(q, nxt);
+    agg_chunk(a, K, A, total, ch, yv, dsc);
+    if (++q == kAggStages) { q = 0; phase ^= 1u; }
   }
 }
 
@@ -2436,7 +2491,9 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
   DT_CK(cudaFuncSetAttribute((const void*)scan_single_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)kScanSingleSmem));
   const int g_scan1 = persistent_grid((const void*)scan_single_kernel, kThreads, kScanSingleSmem);
-  const int g_agg = persistent_grid((const void*)scan_agg_kernel, kThreads, 0);
+  DT_CK(cudaFuncSetAttribute((const void*)scan_agg_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)kScanAggSmem));
+  const int g_agg = persistent_grid((const void*)scan_agg_kernel, kThreads, kScanAggSmem);
   const int g_pagg = persistent_grid((const void*)part_agg_kernel<false>, kThreads, 0);
   size_t agg_smem = sizeof(uint32_t) * (size_t)b.nwords4;
   if ((int64_t)agg_smem > kMaxSmemBitmapBytes) agg_smem = 0;
@@ -2476,7 +2533,7 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     sa.cont_stat = b.cont_stat;
     sa.slot_gain = b.slot_gain;
     sa.level = (uint32_t)level;
-    scan_agg_kernel<<<g_agg, kThreads, 0, s>>>(sa);
+    scan_agg_kernel<<<g_agg, kThreads, kScanAggSmem, s>>>(sa);
     chunk_scan_kernel<SumP><<<(unsigned)b.max_cblocks, 1024, 0, s>>>(ctl, parity, dl, b.chunk_agg, b.chunk_excl,
                                                                      b.block_agg, b.block_carry);
     scan_single_kernel<<<g_scan1, kThreads, kScanSingleSmem, s>>>(sa);
