@@ -11,9 +11,12 @@ N>1 (torchrun): every rank fits its own replica table (seed 1 + rank): "replicas
 weak scaling, no data-path collective (Multi-GPU); max over ranks.
 
 Also reported: e2e (same metric through the C-ABI with host buffers, H2D/D2H inside the
-timed region), DSE predictions/s (BASELINE configs[3] shape on one GPU: 2^28 candidates
-by default, depth-20 / min_samples_leaf-128 tree), the dominant kernel's roofline, and
-the oracle timed on the host as cpu_baseline.
+timed region), DSE predictions/s (BASELINE configs[3] shape on one GPU: 2^28 materialised
+candidates by default, depth-20 / min_samples_leaf-128 tree; and the full 2^30 cross
+product through the factored predictor), the dominant kernel's roofline, the oracle timed
+on the host as cpu_baseline, configs[0] LOO, configs[4] grid, configs[2] (100M x 32,
+depth 16) on one GPU (feature-sharded over NCCL at N>1), a 16-tree Random Forest and
+KNN regression.
 
 --impl reference: the oracle (the slow CPU reference of this tier) timed on the host.
 """
