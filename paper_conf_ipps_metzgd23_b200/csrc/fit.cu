@@ -342,7 +342,10 @@ __global__ void __launch_bounds__(256) presort_build_kernel(const uint32_t* __re
 //               = (keys of smaller digits) + (same digit, earlier tiles) + rank.
 // Stable within a feature, so equal keys keep the row order: (x, row id) order (R6).
 constexpr int kTS = 256, kTI = 8, kTile = kTS * kTI;
-constexpr int64_t kTileSortMaxRows = int64_t(1) << 24;
+#ifndef DT_TILE_SORT_LOG2
+#define DT_TILE_SORT_LOG2 24  // above 2^this rows the presort uses CUB onesweep per feature
+#endif
+constexpr int64_t kTileSortMaxRows = int64_t(1) << DT_TILE_SORT_LOG2;
 
 __global__ void __launch_bounds__(kTS) rs_count_kernel(const uint32_t* __restrict__ keys, int64_t n, int shift,
                                                        int tiles, uint32_t* __restrict__ cnt) {
@@ -787,7 +790,10 @@ __device__ __forceinline__ void agg_chunk(const ScanArgs& a, uint32_t K, uint64_
 // Phase A over the level's full chunks with a per-warp TMA pipeline (kAggStages chunks of
 // y and their descriptors in flight per warp: the pass is a pure stream of y); a partial
 // last chunk goes through registers.
-constexpr int kAggStages = 3;
+#ifndef DT_AGG_STAGES
+#define DT_AGG_STAGES 3
+#endif
+constexpr int kAggStages = DT_AGG_STAGES;
 struct __align__(128) AggStage {
   double y[kChunkW];  // 256 f64 or 256 int32 (first half)
   ChunkDesc d;
@@ -1045,7 +1051,13 @@ __device__ __forceinline__ void scan_single(const ScanArgs& a, int64_t ch, int64
 
 // One pipeline stage of scan_single_kernel: everything one chunk needs, brought in by
 // TMA bulk copies (x, y, descriptor, the two carry words, the entry before the chunk).
-constexpr int kScanStages = 2;
+#ifndef DT_SCAN_STAGES  // experiments: -DDT_SCAN_STAGES=n -DDT_SCAN_MINB=b (DT_EXTRA_NVCC)
+#define DT_SCAN_STAGES 2
+#endif
+#ifndef DT_SCAN_MINB
+#define DT_SCAN_MINB 3
+#endif
+constexpr int kScanStages = DT_SCAN_STAGES;
 struct __align__(128) ScanStage {
   float x[kChunkW];
   double y[kChunkW];
@@ -1058,7 +1070,7 @@ struct __align__(128) ScanStage {
 // Phase C for the single-segment chunks with a per-warp TMA pipeline: lane 0 keeps
 // kScanStages chunks in flight (bulk copies completing on one mbarrier per stage); the
 // lanes read their items from shared memory, so no registers hold in-flight data.
-__global__ void __launch_bounds__(kThreads, 3) scan_single_kernel(ScanArgs a) {
+__global__ void __launch_bounds__(kThreads, DT_SCAN_MINB) scan_single_kernel(ScanArgs a) {
   extern __shared__ __align__(128) unsigned char scan_smem[];
   const uint32_t K = a.ctl->K[a.parity];
   const uint64_t A = a.ctl->A[a.parity];
@@ -1883,18 +1895,34 @@ __global__ void __launch_bounds__(kPrepThreads) prep_kernel(PrepArgs a) {
   for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < G + P + S;
        t += (int64_t)gridDim.x * blockDim.x) {
     if (t < G) {
+      // positions q0 .. q0 + kI - 1 of the split features' lists: all row loads first
+      // (independent), then the bit atomics
       const uint32_t q0 = (uint32_t)(t * kI);
       uint32_t k = cache ? find_start(s1, K, q0) : find_node(a.nodes, K, q0);
       uint32_t kstart = __ldg(&a.nodes[k].start), kend = kstart + __ldg(&a.nodes[k].N);
-      for (int j = 0; j < kI && (uint64_t)q0 + j < A; ++j) {
+      int32_t floc = __ldg(&a.dec[k].floc);
+      uint32_t nl = __ldg(&a.dec[k].nl);
+      uint32_t rr[kI];
+      bool go[kI];
+#pragma unroll
+      for (int j = 0; j < kI; ++j) {
         const uint32_t q = q0 + j;
-        while (q >= kend) { ++k; kstart = kend; kend = kstart + __ldg(&a.nodes[k].N); }
-        const int32_t floc = __ldg(&a.dec[k].floc);
-        if (floc >= 0 && q - kstart < __ldg(&a.dec[k].nl)) {
-          const uint32_t r = __ldg(&a.lr[(int64_t)floc * (int64_t)A + q]);
-          atomicOr(a.gbits + (r >> 5), 1u << (r & 31));
+        go[j] = false;
+        if ((uint64_t)q < A) {
+          while (q >= kend) {
+            ++k;
+            kstart = kend;
+            kend = kstart + __ldg(&a.nodes[k].N);
+            floc = __ldg(&a.dec[k].floc);
+            nl = __ldg(&a.dec[k].nl);
+          }
+          go[j] = floc >= 0 && q - kstart < nl;
+          rr[j] = go[j] ? __ldg(&a.lr[(int64_t)floc * (int64_t)A + q]) : 0u;
         }
       }
+#pragma unroll
+      for (int j = 0; j < kI; ++j)
+        if (go[j]) atomicOr(a.gbits + (rr[j] >> 5), 1u << (rr[j] & 31));
     } else if (t < G + P) {
       const int64_t c = t - G;
       const int64_t p = c * kChunkW;
