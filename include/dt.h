@@ -278,8 +278,7 @@ dt_status dt_eval_sharded(dt_comm* comm, const double* y_dev, const double* yhat
  * launches, tagged with the kernel kind and the launch's ALGORITHMIC bytes (DESIGN.md,
  * "Roofline"); dt_profile_get synchronises those events and returns, for one kind, the
  * number of launches, the summed device time (ms) and the summed algorithmic bytes.
- * dt_launch_count counts this library's own kernel launches (library kernels such as
- * the CUB radix sort inside the presort are not counted) since the last reset. */
+ * dt_launch_count counts this library's own kernel launches since the last reset. */
 void dt_profile_enable(int on);
 void dt_profile_reset(void);
 int64_t dt_launch_count(void);

@@ -3,9 +3,11 @@
 //
 // Level-synchronous, exact (every feature, every threshold, every node):
 //   presort (once)   X row-major -> per-feature lists sorted by (x, row id), SoA
-//                    {x f32, row u32, y f64}; CUB radix sort of (f<<32 | flip(x), row).
+//                    {x f32, row u32, y f64 or int32 (R24)}; batched tile LSD radix sort
+//                    of flip(x) with the row id as value (stable: ties keep row order).
 //   per level l:     scan      segmented prefix of (y - c_node) over every (node, feature)
-//                              segment (deterministic decoupled look-back), gain at every
+//                              segment (three fixed-shape phases: chunk aggregates,
+//                              chunk-carry scan, main pass), gain at every
 //                              valid position, per-(node,feature) argmax pieces, and
 //                              per-node SSE / min / max from the feature-0 list;
 //                    select    per node: combine pieces, leaf rules, best feature;
@@ -15,7 +17,6 @@
 //                              (sorted order preserved, rows of leaves dropped).
 // No host synchronisation inside the level loop (counts live on the device); kernels
 // are persistent and read the level's node/entry counts from device memory.
-#include <cub/device/device_radix_sort.cuh>
 
 #include <math.h>
 #include <stdio.h>
@@ -332,7 +333,7 @@ __global__ void __launch_bounds__(256) presort_build_kernel(const uint32_t* __re
   }
 }
 
-// Batched LSD radix sort of the d per-feature key lists (n <= kTileSortMaxRows): 4 passes
+// Batched LSD radix sort of the d per-feature key lists (any n < 2^32): 4 passes
 // of 8-bit digits; per pass three launches, each over all d features (grid.y = feature):
 //   rs_count:   per-tile digit counts;
 //   rs_offset:  per (feature, digit) exclusive scan of the counts over the tiles, and the
@@ -342,10 +343,6 @@ __global__ void __launch_bounds__(256) presort_build_kernel(const uint32_t* __re
 //               = (keys of smaller digits) + (same digit, earlier tiles) + rank.
 // Stable within a feature, so equal keys keep the row order: (x, row id) order (R6).
 constexpr int kTS = 256, kTI = 8, kTile = kTS * kTI;
-#ifndef DT_TILE_SORT_LOG2
-#define DT_TILE_SORT_LOG2 24  // above 2^this rows the presort uses CUB onesweep per feature
-#endif
-constexpr int64_t kTileSortMaxRows = int64_t(1) << DT_TILE_SORT_LOG2;
 
 __global__ void __launch_bounds__(kTS) rs_count_kernel(const uint32_t* __restrict__ keys, int64_t n, int shift,
                                                        int tiles, uint32_t* __restrict__ cnt) {
@@ -2304,11 +2301,9 @@ struct FitBufs {
   double* cparts;
   uint32_t *k_in, *k_out;  // per feature: n keys flip(x), stable-sorted feature by feature
   uint32_t *v_in, *v_out;
-  void* sort_tmp;           // min(d, kSideStreams) slices of sort_tmp_bytes (CUB path)
-  size_t sort_tmp_bytes;
   uint32_t *rs_cnt, *rs_off;  // batched tile sort: per (feature, digit, tile) counts / offsets
   uint32_t* rs_tot;           // per (feature, digit) totals
-  int rs_tiles;               // tiles per feature (0: per-feature CUB sorts instead)
+  int rs_tiles;               // radix-sort tiles per feature
   ChunkDesc* sdesc;
   uint32_t *slist, *plist;  // per-level chunk lists (scan, partition)
   PartDesc* pdesc;
@@ -2324,8 +2319,6 @@ struct ShardCtx {
   dt_comm* comm;
   int world, rank, dg;
 };
-
-constexpr int kSideStreams = 8;  // side streams of the forked per-feature sorts
 
 // Allocates every buffer through `get` (stream-ordered or persistent).
 template <class Get>
@@ -2377,20 +2370,10 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, int wor
   b.k_out = b.lr[1];
   b.v_in = reinterpret_cast<uint32_t*>(b.ly[1]);
   b.v_out = reinterpret_cast<uint32_t*>(b.ly[1]) + total0;
-  b.rs_tiles = (n <= kTileSortMaxRows) ? (int)((n + kTile - 1) / kTile) : 0;
-  b.rs_cnt = b.rs_off = b.rs_tot = nullptr;
-  if (b.rs_tiles) {
-    DT_CK(get(&b.rs_cnt, (size_t)d * 256 * b.rs_tiles));
-    DT_CK(get(&b.rs_off, (size_t)d * 256 * b.rs_tiles));
-    DT_CK(get(&b.rs_tot, (size_t)d * 256));
-  }
-  b.sort_tmp_bytes = 0;
-  if (!b.rs_tiles) DT_CK(cub::DeviceRadixSort::SortPairs(nullptr, b.sort_tmp_bytes, b.k_in, b.k_out, b.v_in, b.v_out,
-                                        n, 0, 32, (cudaStream_t)0));
-  b.sort_tmp_bytes = (b.sort_tmp_bytes + 255) & ~(size_t)255;
-  // one temp slice per side stream: sorts that share a stream run one after another
-  if (!b.rs_tiles) DT_CK(get((char**)&b.sort_tmp, b.sort_tmp_bytes * (size_t)std::min(d, kSideStreams)));
-  else b.sort_tmp = nullptr;
+  b.rs_tiles = (int)((n + kTile - 1) / kTile);
+  DT_CK(get(&b.rs_cnt, (size_t)d * 256 * b.rs_tiles));
+  DT_CK(get(&b.rs_off, (size_t)d * 256 * b.rs_tiles));
+  DT_CK(get(&b.rs_tot, (size_t)d * 256));
   DT_CK(get(&b.sdesc, (size_t)b.max_chunks));
   DT_CK(get(&b.slist, (size_t)b.max_chunks));
   DT_CK(get(&b.plist, (size_t)b.max_chunks));
@@ -2409,23 +2392,6 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int32_t d, int32_t max_depth, int wor
   return DT_OK;
 }
 
-// Per-host-thread pool of side streams for the forked per-feature sorts.
-struct SideStreams {
-  static constexpr int kN = kSideStreams;
-  cudaStream_t st[kN];
-  cudaEvent_t fork, join[kN];
-  SideStreams() {
-    for (int j = 0; j < kN; ++j) {
-      cudaStreamCreateWithFlags(&st[j], cudaStreamNonBlocking);
-      cudaEventCreateWithFlags(&join[j], cudaEventDisableTiming);
-    }
-    cudaEventCreateWithFlags(&fork, cudaEventDisableTiming);
-  }
-};
-SideStreams& side_streams() {
-  static thread_local SideStreams ss;
-  return ss;
-}
 
 // profiling records whose bytes depend on device-side counts
 struct Pending {
@@ -2470,7 +2436,7 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     // row order -> (x, row id) order), the d sorts forked over side streams
     const uint32_t* sk = b.k_out;  // sorted keys / rows
     const uint32_t* sv = b.v_out;
-    if (b.rs_tiles) {
+    {
       // batched tile radix sort of all d lists: 4 passes x 3 launches (ping-pong, ends in _in)
       pr = prof_begin(PK_PRESORT_SORT, s, 12);
       uint32_t *ki = b.k_in, *ko = b.k_out, *vi = b.v_in, *vo = b.v_out;
@@ -2488,26 +2454,6 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
       DT_CK(cudaGetLastError());
       sk = ki;
       sv = vi;
-    } else {
-      pr = prof_begin(PK_PRESORT_SORT, s, 0);  // CUB kernels: library, not counted
-      {
-        SideStreams& ss = side_streams();
-        DT_CK(cudaEventRecord(ss.fork, s));
-        const int nside = std::min(d, SideStreams::kN);
-        for (int j = 0; j < nside; ++j) DT_CK(cudaStreamWaitEvent(ss.st[j], ss.fork, 0));
-        for (int f = 0; f < d; ++f) {
-          size_t tb = b.sort_tmp_bytes;
-          const int64_t o = (int64_t)f * n;
-          DT_CK(cub::DeviceRadixSort::SortPairs((char*)b.sort_tmp + (size_t)(f % SideStreams::kN) * b.sort_tmp_bytes, tb,
-                                                b.k_in + o, b.k_out + o, b.v_in + o, b.v_out + o, n, 0, 32,
-                                                ss.st[f % SideStreams::kN]));
-        }
-        for (int j = 0; j < nside; ++j) {
-          DT_CK(cudaEventRecord(ss.join[j], ss.st[j]));
-          DT_CK(cudaStreamWaitEvent(s, ss.join[j], 0));
-        }
-      }
-      prof_end(pr, s, 16.0 * (double)total0 * 4);
     }
     const int gb = std::max(1, std::min<int>((int)((total0 + 255) / 256), num_sms() * 8));
     pr = prof_begin(PK_PRESORT_BUILD, s, 1);

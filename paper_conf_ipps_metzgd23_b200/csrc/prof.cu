@@ -19,7 +19,7 @@ std::mutex g_mu;
 bool g_on = false;
 std::vector<Rec> g_recs;
 long long g_launches = 0;
-const char* kNames[] = {"presort_keys", "presort_sort(cub)", "presort_build", "root_stats",
+const char* kNames[] = {"presort_keys", "presort_sort", "presort_build", "root_stats",
                         "scan", "select", "number", "goleft", "partition", "predict",
                         "eval", "loo", "gen", "memset"};
 constexpr int kNumKinds = sizeof(kNames) / sizeof(kNames[0]);

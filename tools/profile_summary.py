@@ -26,8 +26,8 @@ KIND = {
     "goleft_kernel": "goleft", "presort_keys_kernel": "presort_keys",
     "presort_build_kernel": "presort_build", "predict_kernel<true>": "predict",
     "predict_kernel<false>": "predict", "scan_single_kernel": "scan", "prep_kernel": "goleft",
-    "rs_count_kernel": "presort_sort(cub)", "rs_offset_kernel": "presort_sort(cub)",
-    "rs_scatter_kernel": "presort_sort(cub)", "predict_col_kernel": "predict",
+    "rs_count_kernel": "presort_sort", "rs_offset_kernel": "presort_sort",
+    "rs_scatter_kernel": "presort_sort", "predict_col_kernel": "predict",
 }
 
 
@@ -69,8 +69,7 @@ def main():
     lines = [f"# ncu launch list: `{os.path.basename(src)}` (per fit; {nfit} fits captured)", "",
              "Cold-cache, serialised per-launch times (ncu `--clock-control none`); the bench's",
              "live CUDA-event times are the reference for absolutes. Share = fraction of the",
-             "summed kernel time.  ncu serialises the per-feature CUB sorts that the library",
-             "runs concurrently on side streams, so `cub_radix_sort` is overstated here.", "",
+             "summed kernel time.", "",
              "| kernel | launches | time (us) | share | DRAM (MB) | GB/s |",
              "|---|---:|---:|---:|---:|---:|"]
     for n, (c, t, b) in sorted(agg.items(), key=lambda kv: -kv[1][1]):
@@ -89,7 +88,7 @@ def main():
                        "partition": agg.get("partition_kernel", [1])[0],
                        "select": agg.get("select_kernel", [1])[0],
                        "goleft": agg.get("prep_kernel", [1])[0],
-                       "presort_sort(cub)": 1}
+                       "presort_sort": 1}
     tpath = os.path.join(os.path.dirname(os.path.abspath(__file__)), "..", "profiles", "traffic.json")
     traffic = json.load(open(tpath)) if os.path.exists(tpath) else {}
     for k, (b, _) in per_kind.items():
