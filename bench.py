@@ -475,13 +475,19 @@ def run_ours(args, world, rank, local):
     dt.dt_predict_eval(dt.dt_fit(Xd, yd, MAX_DEPTH, MIN_LEAF), Xv, yv, D)
     torch.cuda.synchronize()
     barrier(world)
+    # the held-out rows travel on a second stream while the tree is fitted (after the
+    # training rows, so they do not share the link with them)
+    side = torch.cuda.Stream()
     t0 = time.perf_counter()
     for _ in range(args.e2e_steps):
         Xd.copy_(Xh, non_blocking=True)
         yd.copy_(yh, non_blocking=True)
-        Xvd.copy_(Xvh, non_blocking=True)
-        yvd.copy_(yvh, non_blocking=True)
+        side.wait_stream(stream)  # training rows issued; the previous eval is done
+        with torch.cuda.stream(side):
+            Xvd.copy_(Xvh, non_blocking=True)
+            yvd.copy_(yvh, non_blocking=True)
         tr = dt.dt_fit(Xd, yd, MAX_DEPTH, MIN_LEAF)   # returns the node array on the host
+        stream.wait_stream(side)
         mm = dt.dt_predict_eval(tr, Xvd, yvd, D)      # metrics to the host
         e_evals += tr.split_evals
         h2d = sum(t.numel() * t.element_size() for t in (Xh, yh, Xvh, yvh))
