@@ -392,3 +392,39 @@ def test_eval_sharded(dt, world, sizes):
     mape, r2, adj = oracle.evaluate(y, yh, 5)
     for got, want in ((out[0]["mape"], mape), (out[0]["r2"], r2), (out[0]["adj_r2"], adj)):
         assert abs(got - want) <= 1e-9 * abs(want) + 1e-12
+
+
+# ------------------------------------------------------------------ edge cases --
+
+def _edge_table(case):
+    rng = np.random.default_rng(7)
+    if case == "d255":
+        return rng.integers(0, 8, size=(3000, 255)).astype(np.float32), rng.integers(0, 100, 3000).astype(np.float64)
+    if case == "d100":
+        X, y = datagen.random_table(11, 5000, 100, kind="continuous", int_y=True)
+        return X, y
+    if case == "y_beyond_int32":   # integer mode, but the lists keep f64 targets (R24)
+        return (rng.integers(0, 50, size=(4000, 6)).astype(np.float32),
+                3e9 + rng.integers(0, 1000, 4000).astype(np.float64))
+    if case == "y_negative":
+        return rng.integers(0, 50, size=(4000, 6)).astype(np.float32), rng.integers(-10**6, 10, 4000).astype(np.float64)
+    if case == "y_constant":
+        return rng.random((500, 3)).astype(np.float32), np.full(500, 7.0)
+    if case == "chain":            # alternating 0/1 along x: every level peels one row, depth n - 1
+        n = 60
+        return np.arange(n, dtype=np.float32)[:, None], (np.arange(n) % 2).astype(np.float64)
+    raise KeyError(case)
+
+
+@pytest.mark.parametrize("case,D,m", [("d255", 6, 1), ("d100", -1, 2), ("y_beyond_int32", 10, 1),
+                                      ("y_negative", -1, 1), ("y_constant", -1, 1), ("chain", 24, 1),
+                                      ("chain", 25, 1), ("chain", -1, 1), ("d255", 3, 2000)])
+def test_fit_edge_cases(dt, case, D, m):
+    """Maximum d, wide tables, targets outside int32 / negative / constant, depth around
+    the graph-replay limit (24) and unlimited depth (polled), min_samples_leaf > n / 2."""
+    X, y = _edge_table(case)
+    o, mode = oracle.fit(X, y, D, m, return_mode=True)
+    assert mode
+    _assert_exact(_fit(dt, X, y, D, m).nodes, o)
+    if case == "chain" and D < 0:
+        assert int(o["depth"].max()) == len(y) - 1
