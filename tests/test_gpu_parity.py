@@ -428,3 +428,18 @@ def test_fit_edge_cases(dt, case, D, m):
     _assert_exact(_fit(dt, X, y, D, m).nodes, o)
     if case == "chain" and D < 0:
         assert int(o["depth"].max()) == len(y) - 1
+
+
+def test_nccl_communicator_single_rank(dt):
+    """The NCCL backend of dt_comm (libnccl.so.2 loaded at run time, ncclCommInitRank,
+    allgather / OR-allreduce on the fit's stream) with one rank: the sharded fit equals
+    dt_fit bytewise and the sharded metrics equal dt_eval."""
+    comm = dt.dt_comm_init_nccl(0, 1, lambda obj: obj)
+    X, y = datagen.cnn_gpu_table(4, 30_000)
+    Xd, yd = _cuda(X), _cuda(y)
+    t = dt.dt_fit_sharded(comm, Xd, yd, 10, 2)
+    assert t.nodes.tobytes() == _fit(dt, X, y, 10, 2).nodes.tobytes()
+    yh = dt.dt_predict(t, Xd)
+    m = dt.dt_eval_sharded(comm, yd, yh, 16)
+    ref = dt.dt_eval(yd, yh, 16)
+    assert (m["mape"], m["r2"], m["adj_r2"], m["n"]) == (ref["mape"], ref["r2"], ref["adj_r2"], ref["n"])
