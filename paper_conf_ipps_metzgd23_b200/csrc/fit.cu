@@ -1512,6 +1512,30 @@ __device__ __forceinline__ void decide_node(const SelectArgs& a, uint32_t k, con
   atomicMax(&a.ctl->max_depth_seen, a.level);
 }
 
+// Folds the node-statistics pieces [lo, hi) of node k in index order: loads issued in
+// batches of 8 ahead of the (sequential, order-preserving) combination, so a long run
+// costs one memory latency per 8 pieces instead of one per piece.
+__device__ __forceinline__ void fold_stats(const SelectArgs& a, uint32_t k, int64_t t0, int64_t lo, int64_t hi,
+                                           Stat& acc) {
+  for (int64_t b = lo; b < hi; b += 8) {
+    Stat v[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int64_t pc = b + u;
+      if (pc < hi) v[u] = (pc == 0) ? a.head_stat[k] : a.cont_stat[t0 + pc];
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      if (b + u < hi) {
+        acc.sse = __dadd_rn(acc.sse, v[u].sse);
+        acc.ymin = fmin(acc.ymin, v[u].ymin);
+        acc.ymax = fmax(acc.ymax, v[u].ymax);
+        acc.s1 = __dadd_rn(acc.s1, v[u].s1);
+      }
+    }
+  }
+}
+
 // One block per node (grid-stride over the level's nodes).
 __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
   const uint32_t K = a.ctl->K[a.parity];
@@ -1569,13 +1593,7 @@ __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
       const int64_t np = t1 - t0 + 1;
       const int64_t per = (np + 31) / 32;
       Stat acc{0.0, INFINITY, -INFINITY, 0.0};
-      for (int64_t pc = lane * per; pc < min(np, (lane + 1) * per); ++pc) {
-        const Stat st = (pc == 0) ? a.head_stat[k] : a.cont_stat[t0 + pc];
-        acc.sse = __dadd_rn(acc.sse, st.sse);
-        acc.ymin = fmin(acc.ymin, st.ymin);
-        acc.ymax = fmax(acc.ymax, st.ymax);
-        acc.s1 = __dadd_rn(acc.s1, st.s1);
-      }
+      fold_stats(a, k, t0, lane * per, min(np, (lane + 1) * per), acc);
 #pragma unroll
       for (int off = 1; off < 32; off <<= 1) {  // lane l absorbs lane l + off (fixed shape)
         const double o_sse = __shfl_down_sync(0xffffffffu, acc.sse, off);
@@ -1647,13 +1665,7 @@ __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
       // each thread folds a contiguous run of pieces, then tree
       const int64_t np = t1 - t0 + 1;
       const int64_t per = (np + blockDim.x - 1) / blockDim.x;
-      for (int64_t pc = tid * per; pc < min(np, (tid + 1) * per); ++pc) {
-        const Stat s = (pc == 0) ? a.head_stat[k] : a.cont_stat[t0 + pc];
-        acc.sse = __dadd_rn(acc.sse, s.sse);
-        acc.ymin = fmin(acc.ymin, s.ymin);
-        acc.ymax = fmax(acc.ymax, s.ymax);
-        acc.s1 = __dadd_rn(acc.s1, s.s1);
-      }
+      fold_stats(a, k, t0, tid * per, min(np, (tid + 1) * per), acc);
       s_stat[tid] = acc;
       __syncthreads();
       for (int off = 128; off > 0; off >>= 1) {
