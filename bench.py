@@ -455,11 +455,18 @@ def run_ours(args, world, rank, local):
         with open(tpath) as fh:
             traffic = json.load(fh).get(dom)
     share = {k: round(v["ms"] / prof_ms, 4) for k, v in prof.items()}
+    # every kernel kind with algorithmic bytes (the north star names scan, partition and
+    # predict): achieved GB/s over its launches and the fraction of the measured peak
+    by_kernel = {k: {"achieved_gbs": round(v["alg_bytes"] / (v["ms"] / 1e3) / 1e9, 1),
+                     "frac": round(v["alg_bytes"] / (v["ms"] / 1e3) / 1e9 / peak, 4),
+                     "ms_per_step": round(v["ms"] / nprof, 4)}
+                 for k, v in fit_kinds.items()}
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "peak_source": peak_src,
                 "alg_bytes_per_launch": fit_kinds[dom]["alg_bytes"] / fit_kinds[dom]["launches"],
                 "avg_launch_ms": d_ms / fit_kinds[dom]["launches"], "traffic": traffic,
-                "measured": f"{nprof} profiled steps (ms/step {prof_ms / nprof:.3f}), per-launch CUDA events"}
+                "measured": f"{nprof} profiled steps (ms/step {prof_ms / nprof:.3f}), per-launch CUDA events",
+                "by_kernel": by_kernel}
 
     # ---- e2e: through the C ABI with host buffers (pinned), H2D + D2H inside the region
     Xh, yh = X.cpu().pin_memory(), y.cpu().pin_memory()
