@@ -398,7 +398,10 @@ __global__ void __launch_bounds__(1024) rs_offset_kernel(const uint32_t* __restr
   if (threadIdx.x == 0) tot[(int64_t)blockIdx.y * 256 + blockIdx.x] = s_run;
 }
 
-__global__ void __launch_bounds__(kTS) rs_scatter_kernel(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ vin,
+#ifndef DT_RS_MINB
+#define DT_RS_MINB 4  // 4 CTAs/SM (64 registers): more tiles in flight (measured 4.04 -> 3.95 ms/step)
+#endif
+__global__ void __launch_bounds__(kTS, DT_RS_MINB) rs_scatter_kernel(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ vin,
                                                          uint32_t* __restrict__ kout, uint32_t* __restrict__ vout,
                                                          int64_t n, int shift, int tiles, const uint32_t* __restrict__ off,
                                                          const uint32_t* __restrict__ tot) {
