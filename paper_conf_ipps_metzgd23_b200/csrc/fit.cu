@@ -751,7 +751,10 @@ __device__ __forceinline__ void load_y(const double* __restrict__ ly, int64_t p0
 // entries [kItems*L, kItems*L + kItems) of its warp's chunk).  All scans inside a chunk
 // are warp-shuffle scans (no block barrier); chunk carries come from phase B.
 constexpr int kChunkW = 32 * kItems;           // 256 entries
-constexpr int kBlockChunks = 1024 * 2;         // chunks per phase-B1 block
+#ifndef DT_BLOCK_CHUNKS
+#define DT_BLOCK_CHUNKS 1024  // one chunk per thread (measured: 2048 -> 1024 saves ~1% of the step)
+#endif
+constexpr int kBlockChunks = DT_BLOCK_CHUNKS;  // chunks per phase-B block (1024 threads)
 
 // Phase A: per-chunk segmented aggregate of (y - c) (reads y only).
 // One chunk's segmented aggregate of (y - c) into chunk_agg[ch].
@@ -1885,7 +1888,10 @@ struct PrepArgs {
   int dl_out;   // lists the partition writes (= lists the next level scans)
 };
 constexpr int kPrepCache = 12288;  // node starts of both levels cached per block (48 KB)
-constexpr int kPrepThreads = 1024;
+#ifndef DT_PREP_THREADS
+#define DT_PREP_THREADS 1024
+#endif
+constexpr int kPrepThreads = DT_PREP_THREADS;
 
 // Everything between the numbering of level l and its partition, in one launch (one
 // block per SM, the node starts of levels l and l+1 in shared memory):
@@ -2614,7 +2620,7 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
       pp.ctl = ctl;
       pp.parity = parity;
       pp.dl_out = dl_out;
-      prep_kernel<<<num_sms(), kPrepThreads, 0, s>>>(pp);
+      prep_kernel<<<num_sms() * (1024 / kPrepThreads), kPrepThreads, 0, s>>>(pp);
     }
     if (sh.world > 1) {
       // only the owner of each split feature set its rows' bits: OR over the ranks
