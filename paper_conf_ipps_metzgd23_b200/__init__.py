@@ -34,7 +34,10 @@ SYMBOLS = ("dt_fit", "dt_tree_size", "dt_tree_nodes", "dt_tree_depth", "dt_tree_
            "dt_version", "dt_profile_enable", "dt_profile_reset", "dt_launch_count",
            "dt_profile_kinds", "dt_profile_get", "dt_comm_unique_id_bytes", "dt_comm_unique_id",
            "dt_comm_init", "dt_comm_init_local", "dt_comm_free", "dt_comm_rank", "dt_comm_world",
-           "dt_fit_sharded", "dt_tree_truncate", "dt_predict_eval_depths", "dt_importances")
+           "dt_fit_sharded", "dt_eval_sharded", "dt_tree_truncate", "dt_predict_eval_depths",
+           "dt_importances", "dt_release_workspace", "dt_predict_dse", "dt_forest_fit",
+           "dt_forest_num_trees", "dt_forest_tree", "dt_forest_split_evals", "dt_forest_predict",
+           "dt_forest_free", "dt_bootstrap", "dt_knn_predict")
 
 
 class DTError(RuntimeError):
