@@ -584,7 +584,6 @@ struct ScanArgs {
   int dl;          // feature lists present at this level (d, or 1 at the last level)
   int d;           // feature count (slot stride)
   int64_t min_leaf;
-  uint32_t* counter;  // tile counter (zeroed per launch)
   const ChunkDesc* desc;  // per warp chunk
   const uint32_t* list;   // chunk list (scan_desc_kernel): singles first, others from the back
   SumP* chunk_agg;    // [nchunks] phase A: per-warp-chunk aggregate
