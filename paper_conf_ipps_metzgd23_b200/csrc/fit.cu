@@ -35,7 +35,10 @@ namespace dtl {
 namespace {
 
 constexpr int kThreads = 256;
-constexpr int kItems = 8;
+#ifndef DT_KITEMS
+#define DT_KITEMS 8  // entries per lane of a warp chunk (chunk = 32 x kItems)
+#endif
+constexpr int kItems = DT_KITEMS;
 
 // Per-level node record (level-local index k).
 struct NodeL {
