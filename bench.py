@@ -167,15 +167,53 @@ def barrier(world):
 
 # ---------------------------------------------------------------------- oracle (CPU) --
 
+def _one_core():
+    """Pin this process to one host core for a CPU timing; returns the previous mask."""
+    try:
+        prev = os.sched_getaffinity(0)
+        os.sched_setaffinity(0, {min(prev)})
+        return prev
+    except (AttributeError, OSError):
+        return None
+
+
+def _cpu_model():
+    try:
+        with open("/proc/cpuinfo") as fh:
+            for line in fh:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
 def oracle_rate(rows: int, seed: int = 1):
-    """Oracle fit on the first `rows` rows of the workload table; returns (evals/s, s, evals)."""
+    """Oracle fit on the first `rows` rows of the workload table, pinned to one host core;
+    returns (evals/s, s, evals, sklearn) where sklearn is DecisionTreeRegressor's time on
+    the same sample (the paper's presumed tool) or None."""
     import datagen
     import oracle
     X, y = datagen.cnn_gpu_table(seed, rows)
-    t0 = time.perf_counter()
-    _, ev = oracle.fit(X, y, MAX_DEPTH, MIN_LEAF, return_evals=True)
-    dt = time.perf_counter() - t0
-    return ev / dt, dt, ev
+    prev = _one_core()
+    try:
+        t0 = time.perf_counter()
+        _, ev = oracle.fit(X, y, MAX_DEPTH, MIN_LEAF, return_evals=True)
+        dt = time.perf_counter() - t0
+        sk = None
+        try:
+            from sklearn.tree import DecisionTreeRegressor
+            t1 = time.perf_counter()
+            DecisionTreeRegressor(max_depth=MAX_DEPTH, min_samples_leaf=MIN_LEAF).fit(X, y)
+            ts = time.perf_counter() - t1
+            sk = {"value": ev / ts, "unit": "split evals/s", "seconds": ts,
+                  "note": "sklearn DecisionTreeRegressor (Cython, single thread), same sample and numerator"}
+        except ImportError:
+            pass
+    finally:
+        if prev:
+            os.sched_setaffinity(0, prev)
+    return ev / dt, dt, ev, sk
 
 
 def run_reference(args, world, rank):
@@ -185,6 +223,7 @@ def run_reference(args, world, rank):
     import oracle
     oracle.build()
     X, y = datagen.cnn_gpu_table(1, REF_SAMPLE_ROWS)
+    prev = _one_core()
     for _ in range(args.warmup):
         oracle.fit(X, y, MAX_DEPTH, MIN_LEAF)
     t0 = time.perf_counter()
@@ -193,6 +232,8 @@ def run_reference(args, world, rank):
         _, ev = oracle.fit(X, y, MAX_DEPTH, MIN_LEAF, return_evals=True)
         ev_tot += ev
     dt = time.perf_counter() - t0
+    if prev:
+        os.sched_setaffinity(0, prev)
     v = ev_tot / dt
     sample = (f"oracle fit (single-threaded C, -O2) on the first {REF_SAMPLE_ROWS} rows of the "
               f"configs[1] table (seed 1), depth {MAX_DEPTH}; per step")
@@ -202,7 +243,8 @@ def run_reference(args, world, rank):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": workload_config(1),
             "cpu_baseline": {"value": v, "unit": "split evals/s", "cores": 1, "kind": "oracle",
-                             "sample": sample},
+                             "sample": sample, "cpu_model": _cpu_model(),
+                             "host_cores_available": os.cpu_count()},
             "e2e": {"value": v, "unit": "split evals/s", "h2d_bytes_per_step": 0,
                     "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -659,10 +701,12 @@ def run_ours(args, world, rank, local):
     # ---- CPU baseline: the oracle on the host (rank 0, N=1 only)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
-        rate, secs, ev = oracle_rate(CPU_SAMPLE_ROWS)
+        rate, secs, ev, sk = oracle_rate(CPU_SAMPLE_ROWS)
         cpu = {"value": rate, "unit": "split evals/s", "cores": 1, "kind": "oracle",
                "sample": f"oracle fit on the first {CPU_SAMPLE_ROWS} of the {N_TRAIN} rows "
-                         f"(seed 1), depth {MAX_DEPTH}: {ev} split evals in {secs:.1f} s"}
+                         f"(seed 1), depth {MAX_DEPTH}: {ev} split evals in {secs:.1f} s",
+               "cpu_model": _cpu_model(), "host_cores_available": os.cpu_count(),
+               "pinned": "one core (sched_setaffinity)", "sklearn": sk}
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "split evals/s", "n_gpus": world,
