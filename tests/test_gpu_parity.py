@@ -179,6 +179,17 @@ def test_fit_c2_full(dt):
     assert g.depth == int(o["depth"].max())
 
 
+def test_fit_c2_full_real_target(dt):
+    """BASELINE configs[1] at full size with real-valued targets: the f64 level lists
+    (Reading R24 does not apply) through every streaming kernel at 1M x 16, depth 12;
+    structure by root path with exact-tie adjudication, values within 1e-9."""
+    X, y = datagen.cnn_gpu_table(1, 1_000_000, real=True)
+    o, mode = oracle.fit(X, y, 12, 1, return_mode=True)
+    assert not mode
+    st = treecmp.compare(_fit(dt, X, y, 12, 1).nodes, o, X, y)
+    assert st["compared"] > 1000
+
+
 def test_fit_real_target_c2_schema(dt):
     X, y = datagen.cnn_gpu_table(3, 100_000, real=True)
     o = oracle.fit(X, y, 10, 2)
