@@ -331,20 +331,31 @@ def dt_importances(tree: Tree, stream=None) -> np.ndarray:
     return out
 
 
-def grid_search(X, y, Xv, yv, depths, min_leafs, p=None, stream=None):
+def grid_search(X, y, Xv, yv, depths, min_leafs, p=None, stream=None, rank=0, world=1, gather=None):
     """(max_depth x min_samples_leaf) grid with held-out evaluation (BASELINE configs[4]):
     one dt_fit at max(depths) per m, then dt_predict_eval_depths -- every (D, m) tree is a
     truncation of the deep one.  Returns {(D, m): (mape, r2, adj_r2)} and the split evals
-    actually performed."""
+    actually performed.
+
+    Multi-GPU ("LOO / grid"): with ``world`` ranks each fits the m values
+    ``min_leafs[rank::world]`` on its own GPU (data replicated) and ``gather(obj)`` --
+    e.g. a torch.distributed all_gather_object wrapper returning the list of every rank's
+    object -- merges the per-fit results, so every rank returns the whole grid."""
     p = X.shape[1] if p is None else p
     dmax = max(depths)
     out, evals = {}, 0
-    for m in min_leafs:
+    for m in list(min_leafs)[rank::world]:
         t = dt_fit(X, y, dmax, m, stream=stream)
         evals += t.split_evals
         per = dt_predict_eval_depths(t, Xv, yv, p, stream=stream)
         for D in depths:
             out[(D, m)] = per[min(D, t.depth)]
+    if world > 1:
+        parts = gather((out, evals))
+        out, evals = {}, 0
+        for o, e in parts:
+            out.update(o)
+            evals += e
     return out, evals
 
 

@@ -152,3 +152,51 @@ def test_row_sharded_eval_decomposition_gloo():
         p.join(timeout=60)
     assert sorted(r for r, _ in res) == [0, 1]
     assert all(ok for _, ok in res)
+
+
+def _grid_worker(rank, world, port, q):
+    """grid_search's rank split + gather (SURVEY 8e "LOO / grid") across real processes, with
+    the library's fit / all-depth eval replaced by deterministic stand-ins (no GPU): every
+    rank must return exactly the single-process grid."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import types
+    src = open(os.path.join(os.path.dirname(__file__), "..", "paper_conf_ipps_metzgd23_b200", "__init__.py")).read()
+    body = src[src.index("def grid_search("):src.index("\nclass Comm")]
+    ns = {}
+
+    class FakeTree:
+        def __init__(self, m):
+            self.split_evals, self.depth = 1000 + m, 5
+
+    ns["dt_fit"] = lambda X, y, D, m, stream=None: FakeTree(m)
+    ns["dt_predict_eval_depths"] = lambda t, Xv, yv, p, stream=None: [
+        (t.split_evals * 1e-3 + d, float(d), -float(d)) for d in range(t.depth + 1)]
+    exec(body, ns)
+    X = types.SimpleNamespace(shape=(10, 4))
+
+    def gather(obj):
+        lst = [None] * world
+        dist.all_gather_object(lst, obj)
+        return lst
+    depths, ms = list(range(1, 9)), [1, 2, 4, 8, 16, 32, 64]
+    got = ns["grid_search"](X, None, None, None, depths, ms, rank=rank, world=world, gather=gather)
+    want = ns["grid_search"](X, None, None, None, depths, ms)
+    q.put((rank, got == want and len(got[0]) == len(depths) * len(ms)))
+    dist.destroy_process_group()
+
+
+def test_grid_search_rank_split_gloo():
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_grid_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    assert sorted(r for r, _ in res) == [0, 1]
+    assert all(ok for _, ok in res)
