@@ -7,7 +7,10 @@
  * (CNN, GPU) candidates in a design-space exploration (T_est = t_dca + n*t_pm,
  * PAPER.md:245-247), and judged by MAPE, R^2 and adjusted R^2 (Table II
  * :211-217).  The paper fixes no hyper-parameter, tie rule or threshold rule; the
- * readings used here are listed in DESIGN.md ("Readings", R1-R19).
+ * readings used here are listed in DESIGN.md ("Readings", R1-R24).  Beyond the tree, the
+ * library carries the paper's other non-linear models (Random Forest as bagged CART,
+ * KNN regression), a factored DSE predictor and row / feature sharded
+ * multi-GPU calls.
  *
  * Conventions (all calls):
  *  - Every call returns dt_status; DT_OK == 0.  On error, dt_last_error() returns a
@@ -81,6 +84,9 @@ typedef struct {
  * threshold; threshold = x[i-1]/2 + x[i]/2 in fp64 (R4, R5, R19).  A node is a leaf if
  * depth == max_depth, N < 2*min_samples_leaf, all its y are equal, or no position is
  * valid (R8).
+ * Storage: integral targets with |y| < 2^31 travel through the level lists as int32
+ * (R24); every sum and gain is still the same f64 value.  Repeated bounded-depth fits
+ * (max_depth <= 24) of the same shape replay a cached CUDA graph (dt_release_workspace).
  * Sync: returns once the tree is complete; *out is owned by the caller (dt_tree_free).
  * Errors: INVALID_ARG (n, d, max_depth, min_samples_leaf, null pointers), NONFINITE,
  * TOO_LARGE (n >= 2^32 or workspace beyond device memory), OOM, CUDA. */
