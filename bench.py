@@ -261,7 +261,8 @@ def sharded_fit_measure(args, world, rank, dev, X, y, stream):
     import torch
 
     import paper_conf_ipps_metzgd23_b200 as dt
-    Xs, ys = (X, y) if world > 1 else (X, y)
+    # the SAME table on every rank (the replicas of the headline use seed 1 + rank)
+    Xs, ys = dt.dt_gen_table(1, N_TRAIN, d=D, device=dev) if world > 1 else (X, y)
     if world > 1:
         import torch.distributed as dist
 
@@ -297,7 +298,7 @@ def sharded_fit_measure(args, world, rank, dev, X, y, stream):
         trees = one_round()
     torch.cuda.synchronize()
     dt_s = max_over_ranks(time.perf_counter() - t0, world)
-    ref = dt.dt_fit(X, y, MAX_DEPTH, MIN_LEAF)
+    ref = dt.dt_fit(Xs, ys, MAX_DEPTH, MIN_LEAF)
     same = all(t.nodes.tobytes() == ref.nodes.tobytes() for t in trees)
     evals = trees[0].split_evals
     return {"ranks": world if world > 1 else args.sharded_local,
