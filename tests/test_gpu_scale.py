@@ -12,7 +12,9 @@ is checked ("sampled outputs ... else via properties that hold at any
   and value must equal the node's bit for bit (greedy CART decides every node from its
   own rows only, Readings R4/R8);
 * DSE prediction (configs[3] shape on one GPU, 2^28 candidates, depth-20 tree): sampled
-  candidates predicted by the oracle must match bit for bit.
+  candidates predicted by the oracle must match bit for bit;
+* the bench's KNN (2^16 x 2^20) and Random Forest (16 trees of 1M rows) lines: sampled
+  queries / rows against the oracle, one full-size bootstrap tree exactly.
 """
 import numpy as np
 import pytest
@@ -132,3 +134,36 @@ def test_dse_predict_bench_size_sampled(dt):
     assert np.array_equal(out[ti].cpu().numpy(), oracle.predict(tree.nodes, Xs))
     del Xd, out
     torch.cuda.empty_cache()
+
+
+def test_knn_bench_size_sampled(dt):
+    """bench.py's KNN line: 2^16 training rows of the configs[1] table x 2^20 held-out
+    queries, k = 5; sampled queries equal the oracle's bit for bit."""
+    X, y = dt.dt_gen_table(1, 1 << 16, d=16, device="cuda")
+    Xq, _ = dt.dt_gen_table(2, 1 << 20, d=16, device="cuda")
+    out = dt.dt_knn_predict(X, y, Xq, 5)
+    torch.cuda.synchronize()
+    idx = np.unique(np.concatenate([[0, (1 << 20) - 1], np.random.default_rng(5).integers(0, 1 << 20, 300)]))
+    ti = torch.from_numpy(idx).cuda()
+    want = oracle.knn_predict(X.cpu().numpy(), y.cpu().numpy(), Xq[ti].cpu().numpy(), 5)
+    assert np.array_equal(out[ti].cpu().numpy(), want)
+
+
+def test_forest_bench_size(dt):
+    """bench.py's forest line (16 bagged trees of the configs[1] table, depth 12): tree 0
+    equals the oracle's tree of the same bootstrap sample at full size (integer mode), and
+    sampled forest predictions equal the oracle's tree-order mean of the GPU's trees."""
+    X, y = dt.dt_gen_table(1, 1_000_000, d=16, device="cuda")
+    fo = dt.dt_forest_fit(X, y, 16, 12, 1, seed=1)
+    Xh, yh = X.cpu().numpy(), y.cpu().numpy()
+    idx = oracle.bootstrap(1, 0, len(yh))
+    o = oracle.fit(Xh[idx], yh[idx], 12, 1)
+    g = fo.tree(0).nodes
+    for f in ("feature", "threshold", "left", "n_samples", "value"):
+        assert np.array_equal(g[f], o[f]), f
+    Xv, _ = dt.dt_gen_table(2, 1_000_000, d=16, device="cuda")
+    out = dt.dt_forest_predict(fo, Xv)
+    rows = np.random.default_rng(6).integers(0, 1_000_000, 5000)
+    trees = [fo.tree(t).nodes for t in range(16)]
+    Xs = Xv[torch.from_numpy(rows).cuda()].cpu().numpy()
+    assert np.array_equal(out[torch.from_numpy(rows).cuda()].cpu().numpy(), oracle.forest_predict(trees, Xs))
