@@ -454,3 +454,31 @@ def test_nccl_communicator_single_rank(dt):
     m = dt.dt_eval_sharded(comm, yd, yh, 16)
     ref = dt.dt_eval(yd, yh, 16)
     assert (m["mape"], m["r2"], m["adj_r2"], m["n"]) == (ref["mape"], ref["r2"], ref["adj_r2"], ref["n"])
+
+
+def test_concurrent_fits_from_threads(dt):
+    """Two host threads fitting different tables of the same shape at once (the cached
+    graph plan is shared under a lock and re-planned per input): both trees exact."""
+    import threading
+    tabs = [datagen.random_table(40 + i, 30_000, 8, kind="ties", int_y=True) for i in range(2)]
+    want = [oracle.fit(X, y, 10, 1) for X, y in tabs]
+    got, errs = [None, None], []
+
+    def run(i):
+        try:
+            s = torch.cuda.Stream()
+            with torch.cuda.stream(s):
+                X, y = tabs[i]
+                for _ in range(3):
+                    got[i] = dt.dt_fit(_cuda(X), _cuda(y), 10, 1, stream=s).nodes
+        except Exception as e:  # pragma: no cover - reported below
+            errs.append(e)
+
+    th = [threading.Thread(target=run, args=(i,)) for i in range(2)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    assert not errs, errs
+    for g, o in zip(got, want):
+        _assert_exact(g, o)
