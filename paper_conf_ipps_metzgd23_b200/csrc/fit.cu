@@ -2763,21 +2763,28 @@ struct FitPlan {
   cudaGraphExec_t exec = nullptr;
   cudaStream_t cap = nullptr;
   int64_t launches = 0;
+  uint64_t last_use = 0;
   ~FitPlan() {
     if (exec) cudaGraphExecDestroy(exec);
     if (cap) cudaStreamDestroy(cap);
     for (void* p : mem) cudaFree(p);
   }
 };
+// Two cached plans (least recently used replaced): a caller alternating between two
+// input buffers -- e.g. double-buffered host->device copies overlapping the previous fit
+// -- replays both graphs without re-capture.  A plan whose workspace does not fit beside
+// the other evicts it.
+constexpr int kPlans = 2;
 std::mutex g_plan_mu;
-std::unique_ptr<FitPlan> g_plan;
+std::unique_ptr<FitPlan> g_plans[kPlans];
+uint64_t g_plan_tick = 0;
 
 }  // namespace
 
 dt_status release_workspace_impl() {
   {
     std::lock_guard<std::mutex> lk(g_plan_mu);
-    g_plan.reset();
+    for (auto& p : g_plans) p.reset();
   }
   DT_CK(cudaDeviceSynchronize());
   int dev = 0;
@@ -2807,24 +2814,31 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
   const bool use_graph = graph_env && !prof_enabled() && max_depth >= 0 && max_depth <= 24;
   if (use_graph) {
     std::lock_guard<std::mutex> lk(g_plan_mu);
-    FitPlan* pl = g_plan.get();
-    const bool hit = pl && pl->X == X && pl->y == y && pl->n == n && pl->d == d &&
-                     pl->max_depth == max_depth && pl->min_leaf == min_leaf && pl->device == dev;
-    if (!hit) {
+    FitPlan* pl = nullptr;
+    for (auto& p : g_plans)
+      if (p && p->X == X && p->y == y && p->n == n && p->d == d && p->max_depth == max_depth &&
+          p->min_leaf == min_leaf && p->device == dev)
+        pl = p.get();
+    if (!pl) {
+      // victim slot: an empty one, else the least recently used
+      int v = 0;
+      for (int i = 0; i < kPlans; ++i) {
+        if (!g_plans[i]) { v = i; break; }
+        if (g_plans[i]->last_use < g_plans[v]->last_use) v = i;
+      }
+      FitPlan* old = g_plans[v].get();
       std::unique_ptr<FitPlan> np(new FitPlan());
-      const bool same_shape = pl && pl->n == n && pl->d == d && pl->max_depth == max_depth && pl->device == dev;
+      const bool same_shape = old && old->n == n && old->d == d && old->max_depth == max_depth && old->device == dev;
       if (same_shape) {
         // same buffer shapes (e.g. a min_samples_leaf grid, or new input addresses): keep
         // the workspace, re-capture only -- no cudaFree / cudaMalloc of ~32 B per entry
         DT_CK(cudaDeviceSynchronize());  // the old graph may still run on another stream
-        np->mem.swap(pl->mem);
-        np->b = pl->b;
-        np->cap = pl->cap;
-        pl->cap = nullptr;
-        g_plan.reset();
-      } else {
-        g_plan.reset();  // frees the previous plan's memory (synchronising)
+        np->mem.swap(old->mem);
+        np->b = old->b;
+        np->cap = old->cap;
+        old->cap = nullptr;
       }
+      g_plans[v].reset();  // frees the victim's memory unless it was taken over (synchronising)
       np->X = X;
       np->y = y;
       np->n = n;
@@ -2839,13 +2853,25 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
           return e;
         };
         dt_status st = fit_alloc(np->b, n, d, max_depth, 1, get);
-        if (st != DT_OK) return st;
+        if (st != DT_OK) {
+          // no room beside the other cached plan(s): drop them and try once more
+          bool others = false;
+          for (auto& p : g_plans) others |= (bool)p;
+          if (!others) return st;
+          (void)cudaGetLastError();  // the failed cudaMalloc (not sticky)
+          for (void* m : np->mem) cudaFree(m);
+          np->mem.clear();
+          np->b = FitBufs{};
+          for (auto& p : g_plans) p.reset();
+          st = fit_alloc(np->b, n, d, max_depth, 1, get);
+          if (st != DT_OK) return st;
+        }
         DT_CK(cudaStreamCreateWithFlags(&np->cap, cudaStreamNonBlocking));
       }
       const int64_t l0 = dt_launch_count();
       DT_CK(cudaStreamBeginCapture(np->cap, cudaStreamCaptureModeThreadLocal));
       dt_status st = fit_enqueue(np->b, X, y, n, d, max_depth, min_leaf, np->cap, false, nullptr,
-                       ShardCtx{nullptr, 1, 0, d});
+                                 ShardCtx{nullptr, 1, 0, d});
       cudaGraph_t graph = nullptr;
       cudaError_t ce = cudaStreamEndCapture(np->cap, &graph);
       if (st != DT_OK) {
@@ -2858,9 +2884,10 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
       ce = cudaGraphInstantiate(&np->exec, graph, 0);
       cudaGraphDestroy(graph);
       if (ce != cudaSuccess) return cuda_fail(ce, "cudaGraphInstantiate", __FILE__, __LINE__);
-      g_plan = std::move(np);
-      pl = g_plan.get();
+      g_plans[v] = std::move(np);
+      pl = g_plans[v].get();
     }
+    pl->last_use = ++g_plan_tick;
     DT_CK(cudaGraphLaunch(pl->exec, s));
     prof_add_launches(pl->launches);
     return fit_finish(pl->b, d, s, nullptr, out);
