@@ -295,13 +295,14 @@ dt_status dt_profile_get(int32_t kind, const char** name, int64_t* launches, dou
 /* ------------------------------------------------------------------ memory -------- */
 
 /* Workspace is kept between calls so that repeated fits allocate nothing: the cached
- * CUDA-graph plan of the last bounded-depth dt_fit (its buffers are ~32 B per training
- * entry, i.e. 32 * n * d bytes) and the freed blocks of the device's default memory pool
- * (stream-ordered workspace of the other calls).  dt_release_workspace synchronises the
- * device, frees the cached plan and trims the pool of the CURRENT device to zero, so that
- * a following large allocation (e.g. the 100M x 32 fit of BASELINE configs[2], ~110 GB)
- * can use the whole HBM.  Always safe to call; the next fit re-plans.  Returns DT_OK, or
- * DT_ERR_CUDA if the device synchronisation fails. */
+ * CUDA-graph plans of the last two bounded-depth dt_fit inputs (least recently used
+ * replaced; buffers ~32 B per training entry, i.e. 32 * n * d bytes each; a plan that
+ * does not fit beside the other evicts it) and the freed blocks of the device's default
+ * memory pool (stream-ordered workspace of the other calls).  dt_release_workspace
+ * synchronises the device, frees the cached plans and trims the pool of the CURRENT
+ * device to zero, so that a following large allocation (e.g. the 100M x 32 fit of
+ * BASELINE configs[2], ~110 GB) can use the whole HBM.  Always safe to call; the next fit
+ * re-plans.  Returns DT_OK, or DT_ERR_CUDA if the device synchronisation fails. */
 dt_status dt_release_workspace(void);
 
 /* ------------------------------------------------------------------ misc ---------- */
