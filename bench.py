@@ -651,6 +651,10 @@ def run_ours(args, world, rank, local):
     if not args.no_extra:
         try:
             T = 16
+            # earlier sections leave cached fit plans (up to 2, e.g. the C5 grid's 10M-row
+            # workspace); start from a clean pool so the timed forest holds only its own
+            dt.dt_release_workspace()
+            torch.cuda.empty_cache()
             fo = dt.dt_forest_fit(X, y, 2, MAX_DEPTH, MIN_LEAF, seed=1)  # warm-up (plans the graph)
             torch.cuda.synchronize()
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
