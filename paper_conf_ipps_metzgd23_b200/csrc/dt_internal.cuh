@@ -40,6 +40,8 @@ dt_status tree_upload(dt_tree* t, cudaStream_t s);
 
 // Fit driver (fit.cu).
 dt_status release_workspace_impl();
+// frees the forest's cached bootstrap scratch table (forest.cu); called by release_workspace_impl
+void forest_release_scratch();
 dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
                    int64_t min_leaf, cudaStream_t s, dt_tree** out);
 dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64_t n, int32_t dg,

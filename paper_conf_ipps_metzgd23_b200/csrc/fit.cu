@@ -2786,6 +2786,7 @@ dt_status release_workspace_impl() {
     std::lock_guard<std::mutex> lk(g_plan_mu);
     for (auto& p : g_plans) p.reset();
   }
+  forest_release_scratch();
   DT_CK(cudaDeviceSynchronize());
   int dev = 0;
   DT_CK(cudaGetDevice(&dev));
