@@ -85,3 +85,22 @@ def test_forest_rejects_bad_args(dt):
     fo = dt.dt_forest_fit(_cuda(X), _cuda(y), 1)
     with pytest.raises(dt.DTError):
         dt.dt_forest_predict(fo, _cuda(np.zeros((4, 2), np.float32)))
+
+
+def test_forest_scratch_reuse_across_shapes(dt):
+    """The bootstrap scratch is cached across dt_forest_fit calls (csrc/forest.cu): the
+    same forest again, a different shape in between, and after dt_release_workspace all
+    give the oracle's trees (integer mode, bit-exact)."""
+    tabs = {n: datagen.random_table(n, n, 6, kind="mixed", int_y=True) for n in (4000, 2500)}
+    want = {n: oracle.forest_fit(X, y, 2, 6, 2, seed=3) for n, (X, y) in tabs.items()}
+    for step, n in enumerate((4000, 4000, 2500, 4000, "release", 2500)):
+        if n == "release":
+            dt.dt_release_workspace()
+            continue
+        X, y = tabs[n]
+        fo = dt.dt_forest_fit(_cuda(X), _cuda(y), 2, 6, 2, seed=3)
+        for t in range(2):
+            g, o = fo.tree(t).nodes, want[n][t]
+            assert len(g) == len(o), (step, t)
+            for f in ("feature", "left", "threshold", "n_samples", "value"):
+                assert np.array_equal(g[f], o[f]), (step, t, f)
