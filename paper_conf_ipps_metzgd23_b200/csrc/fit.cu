@@ -1449,6 +1449,8 @@ __global__ void __launch_bounds__(256) piece_pos_kernel(ScanArgs a, uint32_t* __
 // ----------------------------------------------------------------------------- select --
 
 struct SelectArgs {
+  uint4* gbits;  // go-left bitmap: zeroed here (grid-stride) for this level's prep_kernel
+  int64_t nvec;
   const float* lx;
   const NodeL* nodes;
   Ctl* ctl;
@@ -1559,6 +1561,11 @@ __global__ void __launch_bounds__(256, DT_SEL_MINB) select_kernel(SelectArgs a) 
   __shared__ double s_sl[256];
   __shared__ Stat s_stat[256];
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  // nothing reads the bitmap between the previous level's partition and this level's
+  // prep_kernel; clearing it here spreads the 128 KB (C2) / 12.5 MB (C3) over the whole
+  // grid instead of number_kernel's single block
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + tid; i < a.nvec; i += (int64_t)gridDim.x * blockDim.x)
+    a.gbits[i] = make_uint4(0u, 0u, 0u, 0u);
   if (blockIdx.x == 0 && tid == 0 && a.level < kMaxLogLevels) {
     a.log[a.level].A = A;
     a.log[a.level].K = K;
@@ -1751,14 +1758,11 @@ struct NumberArgs {
   int64_t min_leaf;
   dt_node* out;
   LevelLog* log;
-  uint4* gbits;    // go-left bitmap, zeroed here for this level's prep_kernel
-  int64_t nvec;    // uint4 words of the bitmap
 };
 
 // Single block: BFS numbering (children appended left, right in node order), child
 // statistics, next-level offsets.  Integer mode keeps every quantity exact (int64).
 __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
-  for (int64_t i = threadIdx.x; i < a.nvec; i += blockDim.x) a.gbits[i] = make_uint4(0u, 0u, 0u, 0u);
   __shared__ CntP sh[33];
   __shared__ unsigned long long sh_rows[33];
   __shared__ uint32_t base_split;
@@ -1880,7 +1884,7 @@ struct PrepArgs {
   const NodeL* next;          // next level's nodes (from number_kernel)
   const Decision* dec;
   const uint32_t* new_start;
-  uint32_t* gbits;            // zeroed go-left bitmap
+  uint32_t* gbits;            // go-left bitmap (zeroed by select_kernel)
   PartDesc* pdesc;
   uint32_t* plist;
   ChunkDesc* sdesc;
@@ -2566,6 +2570,8 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     se.slot_gain = b.slot_gain;
     se.slot_pos = b.slot_pos;
     se.exch = b.exch_send;
+    se.gbits = reinterpret_cast<uint4*>(b.gbits);
+    se.nvec = b.nwords4 / 4;
     se.world = sh.world;
     se.rank = sh.rank;
     se.dg = sh.dg;
@@ -2597,8 +2603,6 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     na.min_leaf = min_leaf;
     na.out = b.dout;
     na.log = b.lvlog;
-    na.gbits = reinterpret_cast<uint4*>(b.gbits);
-    na.nvec = b.nwords4 / 4;
     pr = prof_begin(PK_NUMBER, s, 1);
     number_kernel<<<1, 1024, 0, s>>>(na);
     prof_end(pr, s, 0.0);
