@@ -241,7 +241,9 @@ def run_reference(args, world, rank):
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": dt / args.steps * 1e3, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": workload_config(1),
+            "config": dict(workload_config(1), n_train=REF_SAMPLE_ROWS,
+                           sample=f"bounded sample: each step fits the first {REF_SAMPLE_ROWS} of the "
+                                  f"{N_TRAIN} configs[1] rows (a 1M-row oracle fit takes ~20 s)"),
             "cpu_baseline": {"value": v, "unit": "split evals/s", "cores": 1, "kind": "oracle",
                              "sample": sample, "cpu_model": _cpu_model(),
                              "host_cores_available": os.cpu_count()},

@@ -135,6 +135,18 @@ def _dev(t, dtype, ndim, name):
     return ctypes.c_void_p(t.data_ptr())
 
 
+def _same(*pairs):
+    """Argument checks before any device work: every tensor on one device, and every
+    (name, actual, expected) length equal.  A short output or label vector would make
+    the kernels read or write past its allocation."""
+    devs = {t.device for t in pairs[0] if t is not None}
+    if len(devs) > 1:
+        raise ValueError(f"tensors on different devices: {sorted(map(str, devs))}")
+    for name, got, want in pairs[1:]:
+        if got != want:
+            raise ValueError(f"{name} has {got} elements, expected {want}")
+
+
 class Tree:
     """Owns a ``dt_tree*`` (or borrows one from its ``owner``, e.g. a Forest).  ``nodes``
     is a numpy structured copy (BFS, 48 B/node)."""
@@ -182,8 +194,7 @@ def dt_fit(X, y, max_depth: int = -1, min_samples_leaf: int = 1, stream=None) ->
     xp = _dev(X, torch.float32, 2, "X")
     yp = _dev(y, torch.float64, 1, "y")
     n, d = X.shape
-    if y.shape[0] != n:
-        raise ValueError("y must have n elements")
+    _same((X, y), ("y", y.shape[0], n))
     h = ctypes.c_void_p()
     _check(_lib.dt_fit(xp, yp, n, d, max_depth, min_samples_leaf, _stream(stream), ctypes.byref(h)))
     return Tree(h)
@@ -203,6 +214,7 @@ def dt_predict(tree: Tree, X, out=None, stream=None):
     if out is None:
         out = torch.empty(n, dtype=torch.float64, device=X.device)
     op = _dev(out, torch.float64, 1, "out")
+    _same((X, out), ("out", out.shape[0], n))
     _check(_lib.dt_predict(tree.handle, xp, n, d, op, _stream(stream)))
     return out
 
@@ -218,6 +230,7 @@ def dt_predict_dse(tree: Tree, cnn, gpu, feature_src, out=None, stream=None):
         raise ValueError("feature_src needs one entry per tree feature")
     if out is None:
         out = torch.empty(n_cnn * n_gpu, dtype=torch.float64, device=cnn.device)
+    _same((cnn, gpu, out), ("out", out.numel(), n_cnn * n_gpu))
     _check(_lib.dt_predict_dse(tree.handle, _dev(cnn, torch.float32, 2, "cnn"), n_cnn, dc,
                                _dev(gpu, torch.float32, 2, "gpu"), n_gpu, dg, src,
                                _dev(out, torch.float64, 1, "out"), _stream(stream)))
@@ -232,6 +245,7 @@ def dt_eval(y, yhat, p: int, stream=None) -> dict:
     import torch
     yp = _dev(y, torch.float64, 1, "y")
     hp = _dev(yhat, torch.float64, 1, "yhat")
+    _same((y, yhat), ("yhat", yhat.shape[0], y.shape[0]))
     m = dt_metrics()
     _check(_lib.dt_eval(yp, hp, y.shape[0], p, _stream(stream), ctypes.byref(m)))
     return _metrics(m)
@@ -241,6 +255,7 @@ def dt_predict_eval(tree: Tree, X, y, p: int, stream=None) -> dict:
     import torch
     xp = _dev(X, torch.float32, 2, "X")
     yp = _dev(y, torch.float64, 1, "y")
+    _same((X, y), ("y", y.shape[0], X.shape[0]))
     m = dt_metrics()
     _check(_lib.dt_predict_eval(tree.handle, xp, yp, X.shape[0], X.shape[1], p, _stream(stream),
                                 ctypes.byref(m)))
@@ -255,6 +270,7 @@ def dt_loo(X, y, max_depth: int = -1, min_samples_leaf: int = 1, out=None, strea
     if out is None:
         out = torch.empty(n, dtype=torch.float64, device=X.device)
     op = _dev(out, torch.float64, 1, "out")
+    _same((X, y, out), ("y", y.shape[0], n), ("out", out.shape[0], n))
     _check(_lib.dt_loo(xp, yp, n, d, max_depth, min_samples_leaf, op, _stream(stream)))
     return out
 
@@ -276,6 +292,9 @@ def dt_gen_dse(seed: int, row0: int, n: int, gpu_bits: int = 10, out=None, devic
     import torch
     if out is None:
         out = torch.empty((n, 16), dtype=torch.float32, device=device)
+    if not out.is_cuda or out.dtype != torch.float32 or not out.is_contiguous():
+        raise TypeError("out must be a contiguous float32 CUDA tensor")
+    _same((out,), ("out", out.numel(), n * 16))
     _check(_lib.dt_gen_dse(seed, row0, n, gpu_bits, ctypes.c_void_p(out.data_ptr()), _stream(stream)))
     return out
 
@@ -319,6 +338,7 @@ def dt_predict_eval_depths(tree: Tree, X, y, p: int, stream=None):
     import torch
     xp = _dev(X, torch.float32, 2, "X")
     yp = _dev(y, torch.float64, 1, "y")
+    _same((X, y), ("y", y.shape[0], X.shape[0]))
     out = np.empty(3 * (tree.depth + 1), dtype=np.float64)
     _check(_lib.dt_predict_eval_depths(tree.handle, xp, yp, X.shape[0], X.shape[1], p,
                                        _stream(stream), out.ctypes.data))
@@ -454,8 +474,7 @@ def dt_forest_fit(X, y, n_trees: int, max_depth: int = -1, min_samples_leaf: int
     xp = _dev(X, torch.float32, 2, "X")
     yp = _dev(y, torch.float64, 1, "y")
     n, d = X.shape
-    if y.shape[0] != n:
-        raise ValueError("y must have n elements")
+    _same((X, y), ("y", y.shape[0], n))
     h = ctypes.c_void_p()
     _check(_lib.dt_forest_fit(xp, yp, n, d, n_trees, max_depth, min_samples_leaf,
                               ctypes.c_uint64(seed), _stream(stream), ctypes.byref(h)))
@@ -467,6 +486,7 @@ def dt_forest_predict(forest: Forest, X, out=None, stream=None):
     n, d = X.shape
     if out is None:
         out = torch.empty(n, dtype=torch.float64, device=X.device)
+    _same((X, out), ("out", out.shape[0], n))
     _check(_lib.dt_forest_predict(forest.handle, _dev(X, torch.float32, 2, "X"), n, d,
                                   _dev(out, torch.float64, 1, "out"), _stream(stream)))
     return out
@@ -485,10 +505,11 @@ def dt_knn_predict(Xtr, ytr, Xq, k: int = 5, out=None, stream=None):
     import torch
     ntr, d = Xtr.shape
     nq = Xq.shape[0]
-    if Xq.shape[1] != d or ytr.shape[0] != ntr:
-        raise ValueError("shape mismatch")
+    if Xq.shape[1] != d:
+        raise ValueError("Xq must have the training rows' d columns")
     if out is None:
         out = torch.empty(nq, dtype=torch.float64, device=Xq.device)
+    _same((Xtr, ytr, Xq, out), ("ytr", ytr.shape[0], ntr), ("out", out.shape[0], nq))
     _check(_lib.dt_knn_predict(_dev(Xtr, torch.float32, 2, "Xtr"), _dev(ytr, torch.float64, 1, "ytr"), ntr, d,
                                _dev(Xq, torch.float32, 2, "Xq"), nq, k, _dev(out, torch.float64, 1, "out"),
                                _stream(stream)))
@@ -505,8 +526,7 @@ def dt_eval_sharded(comm: "Comm", y, yhat, p: int, stream=None) -> dict:
     import torch
     m = dt_metrics()
     n = y.shape[0]
-    if yhat.shape[0] != n:
-        raise ValueError("y and yhat differ in length")
+    _same((y, yhat), ("yhat", yhat.shape[0], n))
     yp = _dev(y, torch.float64, 1, "y") if n else ctypes.c_void_p(0)
     hp = _dev(yhat, torch.float64, 1, "yhat") if n else ctypes.c_void_p(0)
     _check(_lib.dt_eval_sharded(comm.handle, yp, hp, n, p, _stream(stream), ctypes.byref(m)))

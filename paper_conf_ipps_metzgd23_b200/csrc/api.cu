@@ -41,30 +41,40 @@ int num_sms() {
 // x, Reading R5), y = feature << 24 | left.  A leaf self-loops (feature 0, +inf, left =
 // self) so every row runs exactly `depth` iterations without divergence on exit.
 dt_status tree_upload(dt_tree* t, cudaStream_t s) {
-  std::vector<uint2> packed((size_t)t->count);
+  const bool wide = t->count >= kWideNodes;
+  std::vector<uint2> packed(wide ? 0 : (size_t)t->count);
+  std::vector<uint4> wnodes(wide ? (size_t)t->count : 0);
   std::vector<double> val((size_t)t->count);
   for (int64_t k = 0; k < t->count; ++k) {
     const dt_node& nd = t->host[k];
     val[(size_t)k] = nd.value;
+    uint32_t bits, left, feat;
     if (nd.feature < 0) {
       float inf = INFINITY;
-      uint32_t bits;
       memcpy(&bits, &inf, 4);
-      packed[(size_t)k] = make_uint2(bits, (uint32_t)k);
+      left = (uint32_t)k;
+      feat = 0;
     } else {
       // round-down of the fp64 threshold to f32
       float f = (float)nd.threshold;
       if ((double)f > nd.threshold) f = nextafterf(f, -INFINITY);
-      uint32_t bits;
       memcpy(&bits, &f, 4);
-      packed[(size_t)k] = make_uint2(bits, ((uint32_t)nd.feature << 24) | (uint32_t)nd.left);
+      left = (uint32_t)nd.left;
+      feat = (uint32_t)nd.feature;
     }
+    if (wide) wnodes[(size_t)k] = make_uint4(bits, left, feat, 0u);
+    else packed[(size_t)k] = make_uint2(bits, (feat << 24) | left);
   }
   DT_CK(cudaGetDevice(&t->device));
-  DT_CK(cudaMalloc(&t->dev_packed, sizeof(uint2) * (size_t)t->count));
+  if (wide) {
+    DT_CK(cudaMalloc(&t->dev_wide, sizeof(uint4) * (size_t)t->count));
+    DT_CK(cudaMemcpyAsync(t->dev_wide, wnodes.data(), sizeof(uint4) * (size_t)t->count, cudaMemcpyHostToDevice, s));
+  } else {
+    DT_CK(cudaMalloc(&t->dev_packed, sizeof(uint2) * (size_t)t->count));
+    DT_CK(cudaMemcpyAsync(t->dev_packed, packed.data(), sizeof(uint2) * (size_t)t->count,
+                          cudaMemcpyHostToDevice, s));
+  }
   DT_CK(cudaMalloc(&t->dev_value, sizeof(double) * (size_t)t->count));
-  DT_CK(cudaMemcpyAsync(t->dev_packed, packed.data(), sizeof(uint2) * (size_t)t->count,
-                        cudaMemcpyHostToDevice, s));
   DT_CK(cudaMemcpyAsync(t->dev_value, val.data(), sizeof(double) * (size_t)t->count,
                         cudaMemcpyHostToDevice, s));
   DT_CK(cudaStreamSynchronize(s));
@@ -121,7 +131,7 @@ dt_status dt_tree_from_nodes(const dt_node* nodes, int64_t count, int32_t d, dt_
   *out = nullptr;
   if (!nodes || count < 1) return fail(DT_ERR_INVALID_ARG, "dt_tree_from_nodes: empty");
   if (d < 1 || d > 255) return fail(DT_ERR_INVALID_ARG, "dt_tree_from_nodes: d must be in [1, 255]");
-  if (count >= (1 << 24)) return fail(DT_ERR_TOO_LARGE, "dt_tree_from_nodes: >= 2^24 nodes");
+  if (count >= ((int64_t)1 << 31)) return fail(DT_ERR_TOO_LARGE, "dt_tree_from_nodes: >= 2^31 nodes");
   std::vector<int> refs((size_t)count, 0);
   int32_t depth = 0;
   if (nodes[0].depth != 0) return fail(DT_ERR_INVALID_ARG, "root depth != 0");
@@ -161,13 +171,11 @@ dt_status dt_tree_from_nodes(const dt_node* nodes, int64_t count, int32_t d, dt_
 
 void dt_tree_free(dt_tree* t) {
   if (!t) return;
-  if (t->async_alloc) {
-    if (t->dev_packed) cudaFreeAsync(t->dev_packed, 0);
-    if (t->dev_value) cudaFreeAsync(t->dev_value, 0);
-  } else {
-    if (t->dev_packed) cudaFree(t->dev_packed);
-    if (t->dev_value) cudaFree(t->dev_value);
-  }
+  // cudaFree synchronises the device: an asynchronous predict still reading the nodes on
+  // another (non-blocking) stream finishes before the memory can be reused
+  if (t->dev_packed) cudaFree(t->dev_packed);
+  if (t->dev_wide) cudaFree(t->dev_wide);
+  if (t->dev_value) cudaFree(t->dev_value);
   free(t->host);
   delete t;
 }

@@ -121,13 +121,13 @@ int comm_world(const dt_comm* c) { return c->impl.world; }
 // (stream synchronised) for the local backend.
 dt_status comm_allgather(dt_comm* c, const void* send, void* recv, size_t bytes, cudaStream_t s) {
   CommImpl& m = c->impl;
-  if (m.world == 1) {
-    if (send != recv) DT_CK(cudaMemcpyAsync(recv, send, bytes, cudaMemcpyDeviceToDevice, s));
-    return DT_OK;
-  }
-  if (m.backend == 0) {
+  if (m.backend == 0) {  // NCCL, any world size (a 1-rank communicator runs the real collective)
     ncclResult_t r = g_nccl.AllGather(send, recv, bytes, ncclUint8, m.nccl, s);
     if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather");
+    return DT_OK;
+  }
+  if (m.world == 1) {
+    if (send != recv) DT_CK(cudaMemcpyAsync(recv, send, bytes, cudaMemcpyDeviceToDevice, s));
     return DT_OK;
   }
   LocalGroup& g = *m.group;
@@ -146,12 +146,12 @@ dt_status comm_allgather(dt_comm* c, const void* send, void* recv, size_t bytes,
 // which equals the OR when no two ranks set the same bit.
 dt_status comm_allreduce_or_u32(dt_comm* c, uint32_t* buf, int64_t n, cudaStream_t s) {
   CommImpl& m = c->impl;
-  if (m.world == 1) return DT_OK;
   if (m.backend == 0) {
     ncclResult_t r = g_nccl.AllReduce(buf, buf, (size_t)n, ncclUint32, ncclSum, m.nccl, s);
     if (r != ncclSuccess) return nccl_fail(r, "ncclAllReduce");
     return DT_OK;
   }
+  if (m.world == 1) return DT_OK;
   LocalGroup& g = *m.group;
   // every rank computes the OR of all ranks' (unchanged) inputs into a private copy
   uint32_t* tmp = nullptr;
@@ -199,13 +199,11 @@ dt_status dt_comm_init(const void* id, int32_t rank, int32_t world, dt_comm** ou
   c->impl.rank = rank;
   c->impl.world = world;
   c->impl.backend = 0;
-  if (world > 1) {
-    if (!load_nccl()) return fail(DT_ERR_NCCL, "dt_comm_init: libnccl.so.2 not loadable");
-    ncclUniqueId uid;
-    memcpy(&uid, id, sizeof(uid));
-    ncclResult_t r = g_nccl.CommInitRank(&c->impl.nccl, world, uid, rank);
-    if (r != ncclSuccess) return nccl_fail(r, "ncclCommInitRank");
-  }
+  if (!load_nccl()) return fail(DT_ERR_NCCL, "dt_comm_init: libnccl.so.2 not loadable");
+  ncclUniqueId uid;
+  memcpy(&uid, id, sizeof(uid));
+  ncclResult_t r = g_nccl.CommInitRank(&c->impl.nccl, world, uid, rank);
+  if (r != ncclSuccess) return nccl_fail(r, "ncclCommInitRank");
   *out = c.release();
   return DT_OK;
 }

@@ -16,11 +16,16 @@ struct dt_tree {
   dt_node* host = nullptr;    // count nodes, BFS
   // Device copy for prediction: packed 8-byte nodes {f32 thr (round-down), u32 f<<24|left}
   // (leaves self-loop: feature 0, thr +inf, left = self) plus f64 values.
+  // Trees of >= kWideNodes nodes do not fit the 24-bit child field: they get the WIDE
+  // form instead, 16-byte nodes {f32 bits of RD32(thr), left, feature, 0} (same
+  // self-looping leaves), and dev_packed stays NULL (dt_predict / dt_predict_eval only).
   uint2* dev_packed = nullptr;
+  uint4* dev_wide = nullptr;
   double* dev_value = nullptr;
   int device = -1;
-  int async_alloc = 0;        // device arrays from cudaMallocAsync (freed with cudaFreeAsync)
 };
+
+constexpr int64_t kWideNodes = (int64_t)1 << 24;
 
 namespace dtl {
 

@@ -2681,18 +2681,26 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
   return DT_OK;
 }
 
-// Device-side packing of the predict representation (see tree_upload in api.cu).
+// Device-side packing of the predict representation (see tree_upload in api.cu): the
+// 8-byte packed form, or the 16-byte wide form for trees of >= kWideNodes nodes.
 __global__ void __launch_bounds__(256) pack_tree_kernel(const dt_node* __restrict__ nodes, int64_t count,
-                                                        uint2* __restrict__ packed, double* __restrict__ value) {
+                                                        uint2* __restrict__ packed, uint4* __restrict__ wide,
+                                                        double* __restrict__ value) {
   for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < count; k += (int64_t)gridDim.x * blockDim.x) {
     const dt_node nd = nodes[k];
     value[k] = nd.value;
+    uint32_t bits, left, feat;
     if (nd.feature < 0) {
-      packed[k] = make_uint2(0x7f800000u, (uint32_t)k);  // +inf, self-loop
+      bits = 0x7f800000u;  // +inf, self-loop
+      left = (uint32_t)k;
+      feat = 0u;
     } else {
-      float f = __double2float_rd(nd.threshold);  // round-down: x <= t  <=>  x <= RD32(t)
-      packed[k] = make_uint2(__float_as_uint(f), ((uint32_t)nd.feature << 24) | (uint32_t)nd.left);
+      bits = __float_as_uint(__double2float_rd(nd.threshold));  // x <= t  <=>  x <= RD32(t)
+      left = (uint32_t)nd.left;
+      feat = (uint32_t)nd.feature;
     }
+    if (wide) wide[k] = make_uint4(bits, left, feat, 0u);
+    else packed[k] = make_uint2(bits, (feat << 24) | left);
   }
 }
 
@@ -2733,13 +2741,14 @@ dt_status fit_finish(const FitBufs& b, int32_t d, cudaStream_t s, const std::vec
   t->split_evals = (int64_t)hc.split_evals;
   t->integer_mode = hc.int_mode;
   t->host = (dt_node*)malloc(sizeof(dt_node) * (size_t)count);
-  t->async_alloc = 1;
   DT_CK(cudaGetDevice(&t->device));
-  cudaError_t e = cudaMallocAsync((void**)&t->dev_packed, sizeof(uint2) * (size_t)count, s);
-  if (e == cudaSuccess) e = cudaMallocAsync((void**)&t->dev_value, sizeof(double) * (size_t)count, s);
+  const bool wide = count >= kWideNodes;
+  cudaError_t e = wide ? cudaMalloc((void**)&t->dev_wide, sizeof(uint4) * (size_t)count)
+                       : cudaMalloc((void**)&t->dev_packed, sizeof(uint2) * (size_t)count);
+  if (e == cudaSuccess) e = cudaMalloc((void**)&t->dev_value, sizeof(double) * (size_t)count);
   if (e == cudaSuccess) {
     const int g = (int)std::min<int64_t>((count + 255) / 256, 1024);
-    pack_tree_kernel<<<g, 256, 0, s>>>(b.dout, count, t->dev_packed, t->dev_value);
+    pack_tree_kernel<<<g, 256, 0, s>>>(b.dout, count, t->dev_packed, t->dev_wide, t->dev_value);
     prof_add_launches(1);
     e = cudaGetLastError();
   }

@@ -180,6 +180,8 @@ dt_status forest_fit_impl(const float* X, const double* y, int64_t n, int32_t d,
   std::vector<const double*> hv(n_trees);
   std::vector<int32_t> hd(n_trees);
   for (int32_t t = 0; t < n_trees; ++t) {
+    if (!fo->trees[t]->dev_packed)
+      return cleanup(fail(DT_ERR_TOO_LARGE, "dt_forest_fit: a tree has >= 2^24 nodes (no packed predict form)"));
     hn[t] = fo->trees[t]->dev_packed;
     hv[t] = fo->trees[t]->dev_value;
     hd[t] = fo->trees[t]->depth;

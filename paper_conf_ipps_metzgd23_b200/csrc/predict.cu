@@ -61,101 +61,6 @@ predict_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ valu
   }
 }
 
-// Staged predict (d = kD, compile time): the CTA's next batch of kThr rows is copied into
-// shared memory by cp.async (4-byte copies, coalesced, row stride kD + 1 words so that the
-// data-dependent feature reads of a warp hit distinct banks) while the current batch is
-// traversed from shared memory; DRAM latency leaves the 20-level dependency chain.
-__device__ __forceinline__ void cp_async4(void* smem, const void* gmem) {
-  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(sa), "l"(gmem) : "memory");
-}
-
-template <int kThr, int kD>
-__global__ void __launch_bounds__(kThr)
-predict_staged_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ value, int count,
-                      int depth, const float* __restrict__ X, int64_t n, double* __restrict__ yhat) {
-  extern __shared__ uint2 sm[];
-  uint2* tree = sm;
-  float* rows = reinterpret_cast<float*>(sm + count);  // [2][kThr * (kD + 1)]
-  constexpr int kStride = kD + 1;
-  constexpr int kRowsPerPass = kThr / kD;  // rows covered by one copy pass of the block
-  const int tid = threadIdx.x;
-  for (int i = tid; i < count; i += kThr) tree[i] = gnodes[i];
-  const int64_t nb = (n + kThr - 1) / kThr;
-  auto stage = [&](int64_t b, int buf) {
-    const int col = tid % kD, r0 = tid / kD;
-    float* dst = rows + buf * (kThr * kStride);
-    const int64_t base = b * kThr;
-#pragma unroll
-    for (int j = 0; j < kD; ++j) {
-      const int rr = r0 + j * kRowsPerPass;
-      const int64_t r = base + rr;
-      if (r < n) cp_async4(dst + rr * kStride + col, X + r * kD + col);
-    }
-    asm volatile("cp.async.commit_group;" ::: "memory");
-  };
-  int buf = 0;
-  int64_t b = blockIdx.x;
-  if (b < nb) stage(b, 0);
-  for (; b < nb; b += gridDim.x) {
-    const int64_t bn = b + gridDim.x;
-    if (bn < nb) stage(bn, buf ^ 1);
-    else asm volatile("cp.async.commit_group;" ::: "memory");
-    asm volatile("cp.async.wait_group 1;" ::: "memory");
-    __syncthreads();
-    const int64_t r = b * kThr + tid;
-    if (r < n) {
-      const float* row = rows + buf * (kThr * kStride) + tid * kStride;
-      uint32_t k = 0;
-      for (int l = 0; l < depth; ++l) {
-        const uint2 nd = tree[k];
-        const uint32_t left = nd.y & 0xFFFFFFu;
-        k = (row[nd.y >> 24] > __uint_as_float(nd.x)) ? left + 1 : left;
-      }
-      yhat[r] = __ldg(value + k);
-    }
-    __syncthreads();
-    buf ^= 1;
-  }
-}
-
-// Row-prefetch predict (d = 16): each thread fetches its next row with four 128-bit loads
-// before traversing the current one (DRAM latency off the dependency chain); the current
-// row lives in a thread-local array whose data-dependent reads are L1 hits (the carveout
-// leaves L1 everything the smem tree does not need).
-template <int kThr>
-__global__ void __launch_bounds__(kThr)
-predict_rowpf_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ value, int count,
-                     int depth, const float* __restrict__ X, int64_t n, double* __restrict__ yhat) {
-  extern __shared__ uint2 tree[];
-  for (int i = threadIdx.x; i < count; i += kThr) tree[i] = gnodes[i];
-  __syncthreads();
-  const int64_t stride = (int64_t)gridDim.x * kThr;
-  int64_t r = (int64_t)blockIdx.x * kThr + threadIdx.x;
-  float4 nx[4];
-  auto fetch = [&](int64_t rr) {
-    const float4* src = reinterpret_cast<const float4*>(X + rr * 16);
-#pragma unroll
-    for (int q = 0; q < 4; ++q) nx[q] = __ldcs(src + q);
-  };
-  if (r < n) fetch(r);
-  for (; r < n; r += stride) {
-    float row[16];
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      row[4 * q] = nx[q].x; row[4 * q + 1] = nx[q].y; row[4 * q + 2] = nx[q].z; row[4 * q + 3] = nx[q].w;
-    }
-    if (r + stride < n) fetch(r + stride);
-    uint32_t k = 0;
-    for (int l = 0; l < depth; ++l) {
-      const uint2 nd = tree[k];
-      const uint32_t left = nd.y & 0xFFFFFFu;
-      k = (row[nd.y >> 24] > __uint_as_float(nd.x)) ? left + 1 : left;
-    }
-    yhat[r] = __ldg(value + k);
-  }
-}
-
 // Column predict: thread t keeps its current row in shared-memory column t (feature-major
 // s[f][t]), so both the 16/32 stores and the data-dependent feature reads of a warp are
 // bank-conflict-free; the next row is prefetched into registers (four or eight 128-bit
@@ -632,6 +537,7 @@ predict_dse_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ 
 
 dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, int32_t dc, const float* gpu,
                            int64_t n_gpu, int32_t dg, const int32_t* src, double* yhat, cudaStream_t s) {
+  if (!t->dev_packed) return fail(DT_ERR_TOO_LARGE, "dt_predict_dse: tree has >= 2^24 nodes");
   DseMap map{};
   for (int f = 0; f < t->d; ++f) {
     if (src[f] >= 0) {
@@ -653,13 +559,8 @@ dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, in
   const size_t tree = sizeof(uint2) * (size_t)t->count;
   const size_t cap = 227 * 1024;
   if (tables > cap) return fail(DT_ERR_TOO_LARGE, "dt_predict_dse: GPU table too large for shared memory");
-  static int sort_env = -1;
-  if (sort_env < 0) {
-    const char* e = getenv("DT_DSE_SORT");
-    sort_env = (e && e[0] == '0') ? 0 : 1;
-  }
   const bool smem_tree = tree + tables <= cap;
-  const bool sorted = sort_env && (smem_tree ? tree : 0) + tables + sort_bytes <= cap;
+  const bool sorted = (smem_tree ? tree : 0) + tables + sort_bytes <= cap;
   const size_t sm = (smem_tree ? tree : 0) + tables + (sorted ? sort_bytes : 0);
   auto kern = smem_tree ? (sorted ? predict_dse_kernel<true, true, kR> : predict_dse_kernel<true, false, kR>)
                         : (sorted ? predict_dse_kernel<false, true, kR> : predict_dse_kernel<false, false, kR>);
@@ -695,6 +596,7 @@ dt_status eval_depths_impl(const dt_tree* t, const float* X, const double* y, in
                            cudaStream_t s, double* out_host) {
   const int depth = t->depth;
   if (depth > kMaxEvalDepth) return fail(DT_ERR_TOO_LARGE, "dt_predict_eval_depths: tree depth > 32");
+  if (!t->dev_packed) return fail(DT_ERR_TOO_LARGE, "dt_predict_eval_depths: tree has >= 2^24 nodes");
   int64_t chunk = 8192;
   int64_t nparts = (n + chunk - 1) / chunk;
   if (nparts > 2048) {
@@ -719,89 +621,73 @@ dt_status eval_depths_impl(const dt_tree* t, const float* X, const double* y, in
   return DT_OK;
 }
 
+// Wide-format traversal (trees of >= 2^24 nodes, see dt_internal.cuh): node k =
+// {f32 bits of RD32(threshold), left, feature, 0}; leaves self-loop like the packed form.
+__global__ void __launch_bounds__(256) predict_wide_kernel(const uint4* __restrict__ nodes,
+                                                           const double* __restrict__ value, int depth,
+                                                           const float* __restrict__ X, int64_t n, int d,
+                                                           double* __restrict__ yhat) {
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
+    const float* xr = X + r * d;
+    uint32_t k = 0;
+    for (int l = 0; l < depth; ++l) {
+      const uint4 nd = __ldg(nodes + k);
+      k = (__ldg(xr + nd.z) > __uint_as_float(nd.x)) ? nd.y + 1 : nd.y;
+    }
+    yhat[r] = __ldg(value + k);
+  }
+}
+
 dt_status predict_impl(const dt_tree* t, const float* X, int64_t n, int32_t d, double* yhat,
                        cudaStream_t s) {
+  const int pr = prof_begin(PK_PREDICT, s, 1);
+  if (t->dev_wide) {
+    const int64_t g = std::min<int64_t>((int64_t)num_sms() * 8, std::max<int64_t>(1, (n + 255) / 256));
+    predict_wide_kernel<<<(unsigned)g, 256, 0, s>>>(t->dev_wide, t->dev_value, t->depth, X, n, d, yhat);
+    DT_CK(cudaGetLastError());
+    prof_end(pr, s, (4.0 * d + 8.0) * (double)n);
+    return DT_OK;
+  }
   const bool use_smem = t->count <= kMaxSmemNodes;
   const size_t smem = use_smem ? sizeof(uint2) * (size_t)t->count : 0;
-  // configuration: DT_PREDICT_CFG=<0..5> overrides (measurement); default by footprint
-  static int cfg_env = -2;
-  if (cfg_env == -2) {
-    const char* e = getenv("DT_PREDICT_CFG");
-    cfg_env = e ? atoi(e) : -1;
-  }
   // carveout in percent of the 228 KB unified L1/smem: just what the tree needs
   const int carveout = use_smem ? (int)std::min<size_t>(100, (smem + 2048) * 100 / (228 * 1024) + 1) : 0;
-  const int pr = prof_begin(PK_PREDICT, s, 1);
-  dt_status st;
-  int cfg = cfg_env;
-  if (cfg < 0) cfg = 8;  // default: shared-memory column kernel (d = 16 or 32)
-  if (use_smem && (cfg == 8 || cfg == 9) && (d == 16 || d == 32)) {
+  if (use_smem && (d == 16 || d == 32)) {
+    // shared-memory column kernel: tree + one smem column per thread
     const int thr = (d == 16) ? 1024 : 512;
-    const int rpt = (cfg == 9) ? 2 : 1;
-    const size_t sm = sizeof(uint2) * (size_t)t->count + sizeof(float) * (size_t)thr * d * rpt;
+    const size_t sm = sizeof(uint2) * (size_t)t->count + sizeof(float) * (size_t)thr * d;
     if (sm <= 227 * 1024) {
-      auto kern = (d == 16) ? (rpt == 2 ? predict_col_kernel<1024, 16, 2> : predict_col_kernel<1024, 16, 1>)
-                            : (rpt == 2 ? predict_col_kernel<512, 32, 2> : predict_col_kernel<512, 32, 1>);
+      auto kern = (d == 16) ? predict_col_kernel<1024, 16, 1> : predict_col_kernel<512, 32, 1>;
       DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
       int per_sm = 1;
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, thr, sm);
       if (per_sm < 1) per_sm = 1;
       const int64_t g = std::min<int64_t>((int64_t)num_sms() * per_sm,
-                                          std::max<int64_t>(1, (n + (int64_t)thr * rpt - 1) / ((int64_t)thr * rpt)));
+                                          std::max<int64_t>(1, (n + (int64_t)thr - 1) / (int64_t)thr));
       kern<<<(unsigned)g, thr, sm, s>>>(t->dev_packed, t->dev_value, (int)t->count, t->depth, X, n, yhat);
       DT_CK(cudaGetLastError());
       prof_end(pr, s, (4.0 * d + 8.0) * (double)n);
       return DT_OK;
     }
-    cfg = 0;  // tree too large for the column layout: generic kernel
   }
-  if (use_smem && cfg == 7 && d == 16) {
-    constexpr int kThr = 1024;
-    const size_t sm = sizeof(uint2) * (size_t)t->count;
-    auto kern = predict_rowpf_kernel<kThr>;
-    DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
-    DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, carveout));
-    int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kThr, sm);
-    if (per_sm < 1) per_sm = 1;
-    const int64_t g = std::min<int64_t>((int64_t)num_sms() * per_sm, std::max<int64_t>(1, (n + kThr - 1) / kThr));
-    kern<<<(unsigned)g, kThr, sm, s>>>(t->dev_packed, t->dev_value, (int)t->count, t->depth, X, n, yhat);
-    DT_CK(cudaGetLastError());
-    prof_end(pr, s, (4.0 * d + 8.0) * (double)n);
-    return DT_OK;
-  }
-  if (use_smem && cfg >= 6 && (d == 16 || d == 32)) {
-    constexpr int kThr = 512;
-    const size_t sm = sizeof(uint2) * (size_t)t->count + 2 * sizeof(float) * kThr * (size_t)(d + 1);
-    if (sm <= 227 * 1024) {
-      auto kern = (d == 16) ? predict_staged_kernel<kThr, 16> : predict_staged_kernel<kThr, 32>;
-      DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
-      int per_sm = 1;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kThr, sm);
-      if (per_sm < 1) per_sm = 1;
-      const int64_t nb = (n + kThr - 1) / kThr;
-      const int64_t g = std::min<int64_t>((int64_t)num_sms() * per_sm, nb);
-      kern<<<(unsigned)g, kThr, sm, s>>>(t->dev_packed, t->dev_value, (int)t->count, t->depth, X, n, yhat);
-      DT_CK(cudaGetLastError());
-      prof_end(pr, s, (4.0 * d + 8.0) * (double)n);
-      return DT_OK;
-    }
-    cfg = 0;
-  }
-  if (cfg >= 6) cfg = 0;
-  if (!use_smem) st = launch_predict<false, 256, 4>(t, X, n, d, yhat, s, carveout);
-  else if (cfg == 0) st = launch_predict<true, 1024, 1>(t, X, n, d, yhat, s, carveout);
-  else if (cfg == 1) st = launch_predict<true, 512, 2>(t, X, n, d, yhat, s, carveout);
-  else if (cfg == 2) st = launch_predict<true, 1024, 2>(t, X, n, d, yhat, s, carveout);
-  else if (cfg == 3) st = launch_predict<true, 256, 4>(t, X, n, d, yhat, s, carveout);
-  else if (cfg == 4) st = launch_predict<true, 512, 1>(t, X, n, d, yhat, s, carveout);
-  else st = launch_predict<true, 256, 2>(t, X, n, d, yhat, s, carveout);
+  // generic: tree in shared memory when it fits, rows through L1
+  dt_status st = use_smem ? launch_predict<true, 1024, 1>(t, X, n, d, yhat, s, carveout)
+                          : launch_predict<false, 256, 4>(t, X, n, d, yhat, s, carveout);
   prof_end(pr, s, (4.0 * d + 8.0) * (double)n);  // row read + f64 written
   return st;
 }
 
 dt_status eval_impl(const double* y, const double* yhat, const float* X, const dt_tree* t,
                     int64_t n, int32_t p, cudaStream_t s, dt_metrics* out) {
+  if (t && !t->dev_packed) {
+    // wide tree (>= 2^24 nodes): predict into a scratch vector, then the plain metrics
+    double* tmp = nullptr;
+    DT_CK(cudaMallocAsync((void**)&tmp, sizeof(double) * (size_t)n, s));
+    dt_status st = predict_impl(t, X, n, t->d, tmp, s);
+    if (st == DT_OK) st = eval_impl(y, tmp, nullptr, nullptr, n, p, s, out);
+    cudaFreeAsync(tmp, s);
+    return st;
+  }
   // Fixed partition of [0, n) into nparts chunks (deterministic for a given n).
   int64_t chunk = 4096;
   int64_t nparts = (n + chunk - 1) / chunk;

@@ -139,7 +139,10 @@ def test_fit_real_mode_contract(dt, d, n, kind, D, m):
     o = oracle.fit(X, y, D, m)
     g = _fit(dt, X, y, D, m).nodes
     st = treecmp.compare(g, o, X, y)
-    assert st["compared"] >= 1
+    # exemptions (exact gain gap <= 1e-12 relative) must stay rare, and must not hide
+    # the tree: nearly every node is compared by root path
+    assert st["exempt"] <= 2, st
+    assert st["compared"] >= 0.95 * min(len(g), len(o)), (st, len(g), len(o))
 
 
 def test_fit_collinear_ties_exact(dt):
@@ -482,3 +485,24 @@ def test_concurrent_fits_from_threads(dt):
     assert not errs, errs
     for g, o in zip(got, want):
         _assert_exact(g, o)
+
+
+def test_binding_rejects_short_or_misplaced_tensors(dt):
+    """The binding checks lengths and devices before any launch (a short output would be
+    written past its allocation by the kernels)."""
+    X, y = datagen.random_table(3, 100, 4)
+    Xd, yd = _cuda(X), _cuda(y)
+    t = dt.dt_fit(Xd, yd, 3, 1)
+    short = torch.empty(99, dtype=torch.float64, device="cuda")
+    with pytest.raises(ValueError):
+        dt.dt_predict(t, Xd, out=short)
+    with pytest.raises(ValueError):
+        dt.dt_fit(Xd, yd[:50])
+    with pytest.raises(ValueError):
+        dt.dt_eval(yd, short, 4)
+    with pytest.raises(ValueError):
+        dt.dt_predict_eval(t, Xd, yd[:10], 4)
+    with pytest.raises(ValueError):
+        dt.dt_loo(Xd[:20], yd[:20], out=short)
+    with pytest.raises(ValueError):
+        dt.dt_knn_predict(Xd, yd[:99], Xd, 5)

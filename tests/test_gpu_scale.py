@@ -167,3 +167,35 @@ def test_forest_bench_size(dt):
     trees = [fo.tree(t).nodes for t in range(16)]
     Xs = Xv[torch.from_numpy(rows).cuda()].cpu().numpy()
     assert np.array_equal(out[torch.from_numpy(rows).cuda()].cpu().numpy(), oracle.forest_predict(trees, Xs))
+
+
+def test_fit_predict_beyond_2_24_nodes(dt):
+    """A fully grown tree with more than 2^24 nodes (distinct x and y, max_depth -1, Reading
+    R2): the packed 8-byte predict node has a 24-bit child field, so such trees take the
+    16-byte wide form (dt_internal.cuh).  Checks: node array properties, every training row
+    predicts its own target (interpolation), sampled rows bit-exact against the oracle's
+    predict on the GPU's node array, and dt_predict_eval through the wide form."""
+    n = (1 << 23) + 4099
+    rng = np.random.default_rng(24)
+    X = rng.permutation(n).astype(np.float32)[:, None]
+    y = rng.permutation(n).astype(np.float64)
+    Xd, yd = torch.from_numpy(X).cuda(), torch.from_numpy(y).cuda()
+    t = dt.dt_fit(Xd, yd, -1, 1)
+    nodes = t.nodes
+    assert len(nodes) == 2 * n - 1 and len(nodes) >= (1 << 24)
+    _check_array(nodes, n, 10_000)
+    yh = dt.dt_predict(t, Xd)
+    assert torch.equal(yh, yd)
+    m = dt.dt_predict_eval(t, Xd, yd, 1)
+    assert m["mape"] == 0.0 and m["r2"] == 1.0
+    # unseen rows (between the training values) against the oracle, sampled
+    q = (rng.integers(0, n, 4096) + rng.uniform(-0.6, 0.6, 4096)).astype(np.float32)[:, None]
+    got = dt.dt_predict(t, torch.from_numpy(q).cuda()).cpu().numpy()
+    assert np.array_equal(got, oracle.predict(nodes, q))
+    # the same node array through dt_tree_from_nodes (host-built wide form)
+    t2 = dt.dt_tree_from_nodes(nodes, 1)
+    assert np.array_equal(dt.dt_predict(t2, torch.from_numpy(q).cuda()).cpu().numpy(), got)
+    with pytest.raises(dt.DTError):
+        dt.dt_predict_eval_depths(t, Xd, yd, 1)
+    del t, t2
+    dt.dt_release_workspace()
