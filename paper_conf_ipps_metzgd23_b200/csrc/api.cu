@@ -171,11 +171,18 @@ dt_status dt_tree_from_nodes(const dt_node* nodes, int64_t count, int32_t d, dt_
 
 void dt_tree_free(dt_tree* t) {
   if (!t) return;
-  // cudaFree synchronises the device: an asynchronous predict still reading the nodes on
-  // another (non-blocking) stream finishes before the memory can be reused
-  if (t->dev_packed) cudaFree(t->dev_packed);
-  if (t->dev_wide) cudaFree(t->dev_wide);
-  if (t->dev_value) cudaFree(t->dev_value);
+  // The device is synchronised first: an asynchronous predict still reading the nodes on
+  // another (non-blocking) stream finishes before the memory can be reused.
+  if (t->async_alloc) {
+    cudaDeviceSynchronize();
+    if (t->dev_packed) cudaFreeAsync(t->dev_packed, 0);
+    if (t->dev_wide) cudaFreeAsync(t->dev_wide, 0);
+    if (t->dev_value) cudaFreeAsync(t->dev_value, 0);
+  } else {
+    if (t->dev_packed) cudaFree(t->dev_packed);
+    if (t->dev_wide) cudaFree(t->dev_wide);
+    if (t->dev_value) cudaFree(t->dev_value);
+  }
   free(t->host);
   delete t;
 }

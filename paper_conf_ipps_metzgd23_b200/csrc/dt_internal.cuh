@@ -23,6 +23,7 @@ struct dt_tree {
   uint4* dev_wide = nullptr;
   double* dev_value = nullptr;
   int device = -1;
+  int async_alloc = 0;        // device arrays from cudaMallocAsync (dt_fit's pool)
 };
 
 constexpr int64_t kWideNodes = (int64_t)1 << 24;

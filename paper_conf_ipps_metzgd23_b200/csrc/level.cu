@@ -1,0 +1,1172 @@
+// The fused per-level pass of the exact CART fit:
+// stable partition of the level-l feature lists into the children's level-(l+1) lists
+// AND evaluation of every split candidate of every child (every feature, every
+// threshold), in one pass over the entries.
+//
+//   F_A  level_agg_kernel   per warp chunk (256 entries): go-left bit of every entry
+//                           (bitmap lookup by row id), and the chunk aggregate AggP
+//                           (left count, child-centred sums of both sides, last x of
+//                           both sides) since the chunk's last segment head;
+//   F_B  agg_scan_kernel    fixed-shape exclusive scan of the chunk aggregates -> the
+//                           carry of every chunk (blocks of 1024 chunks + block carries);
+//   F_C  fused_kernel       per warp chunk, a TMA bulk-copy pipeline (x, row, y, bits,
+//                           segment plan, carries): the chunk's entries are written to
+//                           their child lists (stable: left entries in order, then right
+//                           entries in order) with coalesced row-wise stores, and the
+//                           children's prefix sums S'_L, positions and neighbour x give
+//                           the exact gain of every valid position (compacted, one gain
+//                           per valid position); per (child segment, chunk) the best
+//                           candidate is recorded, per child node the statistics
+//                           (sum (y - v)^2, min, max, sum (y - c)) from feature 0.
+// All sums run in a fixed order (within a lane sequentially, across lanes Kogge-Stone,
+// across chunks the F_B tree), so results are bit-reproducible; in integer mode every
+// sum is exact, so the trees are independent of the summation order (Reading R17).
+#include <algorithm>
+
+#include "bulk.cuh"
+#include "fit_core.cuh"
+
+namespace dtl {
+
+namespace {
+
+constexpr int kThreads = 256;
+constexpr float kNaN = __builtin_nanf("");
+
+__device__ __forceinline__ double y_at(const double* __restrict__ ly, int64_t p, bool y32) {
+  return y32 ? (double)reinterpret_cast<const int32_t*>(ly)[p] : ly[p];
+}
+
+// ----------------------------------------------------------------------------- F_A --
+
+struct AggArgs {
+  const uint32_t* lr;
+  const double* ly;
+  const float* lx;
+  const uint32_t* desc;
+  const PSeg* pseg;
+  const uint32_t* gbits;
+  uint8_t* gm;
+  AggP* agg;
+  AggP* tails;
+  const Ctl* ctl;
+  int par;
+  int64_t nwords;
+};
+
+__device__ __forceinline__ void load_rows_y(const AggArgs& a, int64_t p0, int64_t T, bool y32, bool need_rows,
+                                            uint32_t* rv, double* yv) {
+  if (p0 + kItems <= T) {
+    if (need_rows) {
+      const uint4* r4 = reinterpret_cast<const uint4*>(a.lr + p0);
+      const uint4 q0 = __ldcs(r4), q1 = __ldcs(r4 + 1);
+      rv[0] = q0.x; rv[1] = q0.y; rv[2] = q0.z; rv[3] = q0.w;
+      rv[4] = q1.x; rv[5] = q1.y; rv[6] = q1.z; rv[7] = q1.w;
+    }
+    if (y32) {
+      const int4* y4 = reinterpret_cast<const int4*>(reinterpret_cast<const int32_t*>(a.ly) + p0);
+      const int4 q0 = __ldcs(y4), q1 = __ldcs(y4 + 1);
+      yv[0] = q0.x; yv[1] = q0.y; yv[2] = q0.z; yv[3] = q0.w;
+      yv[4] = q1.x; yv[5] = q1.y; yv[6] = q1.z; yv[7] = q1.w;
+    } else {
+      const double2* y2 = reinterpret_cast<const double2*>(a.ly + p0);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const double2 t = __ldcs(y2 + q);
+        yv[2 * q] = t.x;
+        yv[2 * q + 1] = t.y;
+      }
+    }
+  } else {
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+      const bool ok = p0 + j < T;
+      rv[j] = (ok && need_rows) ? a.lr[p0 + j] : 0u;
+      yv[j] = ok ? y_at(a.ly, p0 + j, y32) : 0.0;
+    }
+  }
+}
+
+// Kogge-Stone inclusive scan of two f64 values across the warp (fixed shape).
+__device__ __forceinline__ void warp_incl2(double& a, double& b) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const double oa = __shfl_up_sync(0xffffffffu, a, d);
+    const double ob = __shfl_up_sync(0xffffffffu, b, d);
+    if (lane >= d) {
+      a = __dadd_rn(oa, a);
+      b = __dadd_rn(ob, b);
+    }
+  }
+}
+
+template <class T>
+__device__ __forceinline__ T warp_excl_seg(T v, const T& ident, T& agg) {
+  const int lane = threadIdx.x & 31;
+  T inc = v;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    T o = shfl_up(inc, d);
+    if (lane >= d) inc = combine(o, inc);
+  }
+  agg = shfl_idx(inc, 31);
+  T ex = shfl_up(inc, 1);
+  if (lane == 0) ex = ident;
+  return ex;
+}
+
+// Segment plan fields the aggregate pass needs.
+struct SegLite {
+  uint64_t start, end;
+  uint32_t flags;
+  double c0, c1;
+};
+__device__ __forceinline__ SegLite seg_lite(const PSeg* __restrict__ ps, uint32_t s) {
+  SegLite r;
+  r.start = __ldg(&ps[s].start);
+  r.end = r.start + __ldg(&ps[s].cnt);
+  r.flags = __ldg(&ps[s].flags);
+  r.c0 = __ldg(&ps[s].c[0]);
+  r.c1 = __ldg(&ps[s].c[1]);
+  return r;
+}
+
+template <bool kSmemBits, bool kTails>
+__global__ void __launch_bounds__(kSmemBits ? 1024 : kThreads) level_agg_kernel(AggArgs a) {
+  extern __shared__ uint4 smem_bits4[];
+  const uint32_t* __restrict__ bits = kSmemBits ? reinterpret_cast<const uint32_t*>(smem_bits4) : a.gbits;
+  const uint64_t T = a.ctl->T[a.par];
+  const bool full = a.ctl->nsrch > 0;  // children searched: every list; else feature 0 (statistics)
+  const uint64_t Tw = full ? T : a.ctl->T0[a.par];
+  const int64_t nch = (int64_t)((Tw + kChunkW - 1) / kChunkW);
+  const bool y32 = a.ctl->y32 != 0;
+  if (kSmemBits) {
+    const int64_t n4 = a.nwords / 4;
+    const uint4* g4 = reinterpret_cast<const uint4*>(a.gbits);
+    for (int64_t i = threadIdx.x; i < n4; i += blockDim.x) smem_bits4[i] = __ldg(g4 + i);
+    __syncthreads();
+  }
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t ch = gw; ch < nch; ch += nw) {
+    const uint64_t cbase = (uint64_t)ch * kChunkW;
+    const int64_t p0 = (int64_t)cbase + lane * kItems;
+    uint32_t s = __ldg(a.desc + ch);
+    SegLite sg = seg_lite(a.pseg, s);
+    const bool fast = sg.start <= cbase && sg.end >= cbase + kChunkW;  // warp-uniform
+    if (fast) {
+      AggP out = agg_ident();
+      out.flag = sg.start == cbase ? 1u : 0u;
+      uint32_t gbyte = 0u;
+      if (sg.flags & PS_SPLIT) {
+        const bool all_left = (sg.flags & PS_ALLLEFT) != 0;
+        uint32_t rv[kItems];
+        double yv[kItems];
+        load_rows_y(a, p0, (int64_t)T, y32, !all_left, rv, yv);
+        double sl = 0.0, sr = 0.0;
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+          const uint32_t g = all_left ? 1u : ((bits[rv[j] >> 5] >> (rv[j] & 31)) & 1u);
+          gbyte |= g << j;
+          if (g) sl = __dadd_rn(sl, __dsub_rn(yv[j], sg.c0));
+          else sr = __dadd_rn(sr, __dsub_rn(yv[j], sg.c1));
+        }
+        warp_incl2(sl, sr);
+        const uint32_t Lm = __ballot_sync(0xffffffffu, gbyte != 0u);
+        const uint32_t Rm = __ballot_sync(0xffffffffu, gbyte != 0xffu);
+        float xl = kNaN, xr = kNaN;
+        if (Lm) {
+          const int h = 31 - __clz(Lm);
+          float v = 0.f;
+          if (lane == h) v = a.lx[p0 + 31 - __clz(gbyte)];
+          xl = __shfl_sync(0xffffffffu, v, h);
+        }
+        if (Rm) {
+          const int h = 31 - __clz(Rm);
+          float v = 0.f;
+          if (lane == h) v = a.lx[p0 + 31 - __clz(~gbyte & 0xffu)];
+          xr = __shfl_sync(0xffffffffu, v, h);
+        }
+        uint32_t nl = __popc(gbyte);
+        nl = __reduce_add_sync(0xffffffffu, nl);
+        out.nl = nl;
+        out.sl = __shfl_sync(0xffffffffu, sl, 31);
+        out.sr = __shfl_sync(0xffffffffu, sr, 31);
+        out.xl = xl;
+        out.xr = xr;
+      }
+      a.gm[cbase / 8 + lane] = (uint8_t)gbyte;
+      if (lane == 0) {
+        a.agg[ch] = out;
+        if (kTails && (sg.flags & PS_SPLIT) && sg.end == cbase + kChunkW) a.tails[s] = out;
+      }
+      continue;
+    }
+    // ---- general chunk: segment heads inside; per item walk
+    uint32_t rv[kItems];
+    double yv[kItems];
+    load_rows_y(a, p0, (int64_t)T, y32, true, rv, yv);
+    uint32_t gbyte = 0u;
+    AggP run = agg_ident();  // trailing run of the lane
+    int lastL = -1, lastR = -1;
+    {
+      uint32_t sc = s;
+      SegLite g2 = sg;
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        const uint64_t p = (uint64_t)p0 + j;
+        if (p < T) {
+          while (p >= g2.end) g2 = seg_lite(a.pseg, ++sc);
+          if (p == g2.start) {
+            run = agg_ident();
+            run.flag = 1u;
+            lastL = lastR = -1;
+          }
+          if (g2.flags & PS_SPLIT) {
+            const uint32_t g = (g2.flags & PS_ALLLEFT) ? 1u : ((bits[rv[j] >> 5] >> (rv[j] & 31)) & 1u);
+            gbyte |= g << j;
+            if (g) {
+              run.nl += 1u;
+              run.sl = __dadd_rn(run.sl, __dsub_rn(yv[j], g2.c0));
+              lastL = j;
+            } else {
+              run.sr = __dadd_rn(run.sr, __dsub_rn(yv[j], g2.c1));
+              lastR = j;
+            }
+          }
+        }
+      }
+    }
+    if (lastL >= 0) run.xl = a.lx[p0 + lastL];
+    if (lastR >= 0) run.xr = a.lx[p0 + lastR];
+    AggP wagg;
+    const AggP ex = warp_excl_seg(run, agg_ident(), wagg);
+    a.gm[cbase / 8 + lane] = (uint8_t)gbyte;
+    if (lane == 0) a.agg[ch] = wagg;
+    if (kTails) {
+      // per split segment ending in this lane: its aggregate from max(segment start,
+      // chunk start) to its last entry (segcount adds the chunk carry)
+      uint32_t sc = s;
+      SegLite g2 = sg;
+      AggP r = ex;  // the open segment's part before this lane
+      int lL = -1, lR = -1;
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        const uint64_t p = (uint64_t)p0 + j;
+        if (p < T) {
+          while (p >= g2.end) g2 = seg_lite(a.pseg, ++sc);
+          if (p == g2.start) {
+            r = agg_ident();
+            r.flag = 1u;
+            lL = lR = -1;
+          }
+          if (g2.flags & PS_SPLIT) {
+            if ((gbyte >> j) & 1u) {
+              r.nl += 1u;
+              r.sl = __dadd_rn(r.sl, __dsub_rn(yv[j], g2.c0));
+              lL = j;
+            } else {
+              r.sr = __dadd_rn(r.sr, __dsub_rn(yv[j], g2.c1));
+              lR = j;
+            }
+            if (p + 1 == g2.end) {
+              AggP t = r;
+              if (lL >= 0) t.xl = a.lx[p0 + lL];
+              if (lR >= 0) t.xr = a.lx[p0 + lR];
+              a.tails[sc] = t;
+            }
+          }
+        }
+      }
+    }
+  }
+}
+
+// ----------------------------------------------------------------------------- F_B --
+
+// Exclusive segmented scan of the chunk aggregates inside blocks of kBlockChunks chunks,
+// then -- by the last block to finish (ticket) -- the exclusive scan of the block
+// aggregates (block carries).  Fixed shape: deterministic.
+__device__ __forceinline__ AggP block_excl_agg(AggP v, AggP& bagg, AggP* sh) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int nw = blockDim.x >> 5;
+  AggP inc = v;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    AggP o = shfl_up(inc, d);
+    if (lane >= d) inc = combine(o, inc);
+  }
+  if (lane == 31) sh[w] = inc;
+  __syncthreads();
+  if (w == 0) {
+    AggP wv = (lane < nw) ? sh[lane] : agg_ident();
+    AggP wi = wv;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      AggP o = shfl_up(wi, d);
+      if (lane >= d) wi = combine(o, wi);
+    }
+    AggP ex = shfl_up(wi, 1);
+    if (lane == 0) ex = agg_ident();
+    __syncwarp();
+    if (lane < nw) sh[lane] = ex;
+    if (lane == nw - 1) sh[nw] = wi;
+  }
+  __syncthreads();
+  const AggP wpre = sh[w];
+  bagg = sh[nw];
+  AggP ex = shfl_up(inc, 1);
+  AggP res = (lane == 0) ? wpre : combine(wpre, ex);
+  __syncthreads();
+  return res;
+}
+
+__device__ __forceinline__ AggP ld_cg_agg(const AggP* p) {
+  AggP r;
+  r.flag = __ldcg(&p->flag);
+  r.nl = __ldcg(&p->nl);
+  r.sl = __ldcg(&p->sl);
+  r.sr = __ldcg(&p->sr);
+  r.xl = __ldcg(&p->xl);
+  r.xr = __ldcg(&p->xr);
+  return r;
+}
+
+__global__ void __launch_bounds__(1024) agg_scan_kernel(Ctl* ctl, int par, const AggP* __restrict__ agg,
+                                                       AggP* __restrict__ cexcl, AggP* bagg, AggP* __restrict__ bcarry) {
+  __shared__ AggP sh[33];
+  __shared__ AggP sh_run;
+  __shared__ bool s_last;
+  const bool full = ctl->nsrch > 0;
+  const uint64_t T = full ? ctl->T[par] : 0;  // carries are only used when children are searched
+  const int64_t nch = (int64_t)((T + kChunkW - 1) / kChunkW);
+  const int64_t b0 = (int64_t)blockIdx.x * kBlockChunks;
+  if (b0 < nch) {  // block-uniform
+    const int64_t c = b0 + threadIdx.x;
+    const AggP v = (c < nch) ? agg[c] : agg_ident();
+    AggP ba;
+    const AggP ex = block_excl_agg(v, ba, sh);
+    if (c < nch) cexcl[c] = ex;
+    if (threadIdx.x == 0) bagg[blockIdx.x] = ba;
+  }
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) s_last = atomicAdd(&ctl->ticket, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  if (threadIdx.x == 0) {
+    ctl->ticket = 0u;
+    sh_run = agg_ident();
+  }
+  const int64_t nb = (nch + kBlockChunks - 1) / kBlockChunks;
+  __syncthreads();
+  for (int64_t base = 0; base < nb; base += blockDim.x) {
+    const int64_t bi = base + threadIdx.x;
+    const AggP v = (bi < nb) ? ld_cg_agg(bagg + bi) : agg_ident();
+    AggP chunk;
+    const AggP ex = block_excl_agg(v, chunk, sh);
+    const AggP run = sh_run;
+    if (bi < nb) bcarry[bi] = combine(run, ex);
+    __syncthreads();
+    if (threadIdx.x == 0) sh_run = combine(run, chunk);
+    __syncthreads();
+  }
+}
+
+// ----------------------------------------------------------------------------- F_C --
+
+struct FusedArgs {
+  const float* lx;
+  const uint32_t* lr;
+  const double* ly;
+  float* ox;
+  uint32_t* orow;
+  double* oy;
+  const uint32_t* desc;
+  uint32_t* desc_next;
+  const PSeg* pseg;
+  const uint8_t* gm;
+  const AggP* cexcl;
+  const AggP* bcarry;
+  Cand2* head_cand;
+  Cand2* cont_cand;
+  unsigned long long* slot_gain;
+  Stat* head_stat;
+  Stat* cont_stat;
+  uint32_t* gen_list;  // chunks with segment heads inside (fused_general_kernel)
+  Ctl* ctl;
+  int par;
+  uint32_t level;   // level of the children (written into the pieces)
+  uint32_t m;       // min_samples_leaf (clamped)
+  uint32_t ystride; // bytes of one y entry (4 or 8)
+  uint32_t stage_bytes;
+};
+
+// Stage layout (bytes): x[256] f32 | row[256] u32 | y[256] (4 or 8 B) | gm[32] | PSeg |
+// chunk carry | block carry | meta.
+constexpr uint32_t kOffX = 0, kOffR = 1024, kOffY = 2048;
+__device__ __forceinline__ uint32_t off_gm(uint32_t yb) { return kOffY + 256u * yb; }
+__device__ __forceinline__ uint32_t off_ps(uint32_t yb) { return off_gm(yb) + 32u; }
+__device__ __forceinline__ uint32_t off_ce(uint32_t yb) { return off_ps(yb) + (uint32_t)sizeof(PSeg); }
+__device__ __forceinline__ uint32_t off_cb(uint32_t yb) { return off_ce(yb) + 32u; }
+__device__ __forceinline__ uint32_t off_meta(uint32_t yb) { return off_cb(yb) + 32u; }
+__host__ __device__ constexpr uint32_t stage_bytes_for(uint32_t yb) { return 2048u + 256u * yb + 32u + (uint32_t)sizeof(PSeg) + 64u + 16u; }
+
+struct Meta {
+  int64_t ch;
+  uint32_t skip, pad;
+};
+
+// Compacted valid positions of one chunk (per warp).
+struct Compact {
+  double S[kChunkW];
+  uint32_t js[kChunkW];  // global child position | side << 31
+  float xp[kChunkW];
+  float xv[kChunkW];
+};
+
+struct ArgQ {  // segmented argmax: ties keep the earlier position
+  uint32_t flag, j;
+  double gain, sl, thr;
+};
+__device__ __forceinline__ ArgQ argq_ident() { return ArgQ{0u, 0u, -1.0, 0.0, 0.0}; }
+__device__ __forceinline__ ArgQ combine(const ArgQ& a, const ArgQ& b) {
+  if (b.flag) return b;
+  ArgQ r = (b.gain > a.gain) ? b : a;
+  r.flag = a.flag;
+  return r;
+}
+__device__ __forceinline__ ArgQ shfl_up(const ArgQ& v, int d) {
+  return ArgQ{__shfl_up_sync(0xffffffffu, v.flag, d), __shfl_up_sync(0xffffffffu, v.j, d),
+              __shfl_up_sync(0xffffffffu, v.gain, d), __shfl_up_sync(0xffffffffu, v.sl, d),
+              __shfl_up_sync(0xffffffffu, v.thr, d)};
+}
+__device__ __forceinline__ ArgQ shfl_idx(const ArgQ& v, int s) {
+  return ArgQ{__shfl_sync(0xffffffffu, v.flag, s), __shfl_sync(0xffffffffu, v.j, s),
+              __shfl_sync(0xffffffffu, v.gain, s), __shfl_sync(0xffffffffu, v.sl, s),
+              __shfl_sync(0xffffffffu, v.thr, s)};
+}
+struct StatQ {
+  uint32_t flag;
+  double sse, ymin, ymax, s1;
+};
+__device__ __forceinline__ StatQ statq_ident() { return StatQ{0u, 0.0, INFINITY, -INFINITY, 0.0}; }
+__device__ __forceinline__ StatQ combine(const StatQ& a, const StatQ& b) {
+  if (b.flag) return b;
+  return StatQ{a.flag, __dadd_rn(a.sse, b.sse), fmin(a.ymin, b.ymin), fmax(a.ymax, b.ymax), __dadd_rn(a.s1, b.s1)};
+}
+__device__ __forceinline__ StatQ shfl_up(const StatQ& v, int d) {
+  return StatQ{__shfl_up_sync(0xffffffffu, v.flag, d), __shfl_up_sync(0xffffffffu, v.sse, d),
+               __shfl_up_sync(0xffffffffu, v.ymin, d), __shfl_up_sync(0xffffffffu, v.ymax, d),
+               __shfl_up_sync(0xffffffffu, v.s1, d)};
+}
+__device__ __forceinline__ StatQ shfl_idx(const StatQ& v, int s) {
+  return StatQ{__shfl_sync(0xffffffffu, v.flag, s), __shfl_sync(0xffffffffu, v.sse, s),
+               __shfl_sync(0xffffffffu, v.ymin, s), __shfl_sync(0xffffffffu, v.ymax, s),
+               __shfl_sync(0xffffffffu, v.s1, s)};
+}
+__device__ __forceinline__ void stat_add(StatQ& st, double y, double v, double c) {
+  const double e = __dsub_rn(y, v);
+  st.sse = __dadd_rn(st.sse, __dmul_rn(e, e));
+  st.ymin = fmin(st.ymin, y);
+  st.ymax = fmax(st.ymax, y);
+  st.s1 = __dadd_rn(st.s1, __dsub_rn(y, c));
+}
+
+__device__ __forceinline__ void put_cand(const FusedArgs& a, bool head, int64_t ch, int side, uint32_t cs,
+                                         double gain, double sl, double thr, uint32_t j) {
+  Cand2 c;
+  c.gain = gain;
+  c.sl = sl;
+  c.thr = thr;
+  c.j = j;
+  c.sp = cs;
+  c.level = a.level;
+  c.pad = 0u;
+  if (head) a.head_cand[cs] = c;
+  else a.cont_cand[2 * ch + side] = c;
+  atomicMax(a.slot_gain + cs, (unsigned long long)__double_as_longlong(gain));
+}
+__device__ __forceinline__ void put_stat(const FusedArgs& a, bool head, int64_t ch, int side, uint32_t kc,
+                                         const StatQ& q) {
+  Stat s{q.sse, q.ymin, q.ymax, q.s1};
+  if (head) a.head_stat[kc] = s;
+  else a.cont_stat[2 * ch + side] = s;
+}
+
+
+// Loads the plan fields of segment s (global memory; general path).
+struct SegCtx {
+  uint64_t start, end;
+  uint32_t flags, kid;
+  int32_t f;
+  uint32_t cs[2];
+  uint64_t os[2];
+  double c[2], v[2], sc[2], soff[2];
+  uint32_t N[2], ioff[2];
+  float xp[2];
+};
+__device__ __forceinline__ void load_ctx(SegCtx& c, const PSeg* __restrict__ P) {
+  c.start = __ldg(&P->start);
+  c.end = c.start + __ldg(&P->cnt);
+  c.flags = __ldg(&P->flags);
+  c.kid = __ldg(&P->kid);
+  c.f = __ldg(&P->f);
+#pragma unroll
+  for (int q = 0; q < 2; ++q) {
+    c.cs[q] = __ldg(&P->cs[q]);
+    c.os[q] = __ldg(&P->ostart[q]);
+    c.c[q] = __ldg(&P->c[q]);
+    c.v[q] = __ldg(&P->v[q]);
+    c.sc[q] = __ldg(&P->sc[q]);
+    c.soff[q] = __ldg(&P->soff[q]);
+    c.N[q] = __ldg(&P->N[q]);
+    c.ioff[q] = __ldg(&P->ioff[q]);
+    c.xp[q] = __ldg(&P->xprev[q]);
+  }
+}
+
+__device__ __forceinline__ void store_entry(const FusedArgs& a, bool y32, uint64_t dst, float x, uint32_t r,
+                                            const unsigned char* ysrc, uint32_t cs) {
+  a.ox[dst] = x;
+  a.orow[dst] = r;
+  if (y32) reinterpret_cast<uint32_t*>(a.oy)[dst] = *reinterpret_cast<const uint32_t*>(ysrc);
+  else reinterpret_cast<unsigned long long*>(a.oy)[dst] = *reinterpret_cast<const unsigned long long*>(ysrc);
+  if ((dst & (kChunkW - 1)) == 0) a.desc_next[dst / kChunkW] = cs;
+}
+
+// y storage (int32 or f64, Reading R24) is decided on the device (root statistics): the
+// stage always has room for f64 entries; int32 lists copy and read half of it.
+__global__ void __launch_bounds__(kThreads, 2) fused_kernel(FusedArgs a) {
+  extern __shared__ __align__(128) unsigned char fsm[];
+  constexpr uint32_t YB = 8u;
+  constexpr uint32_t SB = (stage_bytes_for(YB) + 127u) & ~127u;
+  constexpr int kWarps = kThreads / 32;
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  unsigned char* my = fsm + (size_t)wib * 2 * SB;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(fsm + (size_t)kWarps * 2 * SB) + wib * 2;
+  PSeg* cur = reinterpret_cast<PSeg*>(fsm + (size_t)kWarps * 2 * SB + kWarps * 2 * sizeof(uint64_t)) + wib;
+  Compact& cbuf = reinterpret_cast<Compact*>(fsm + (size_t)kWarps * 2 * SB + kWarps * 2 * sizeof(uint64_t) +
+                                             kWarps * sizeof(PSeg))[wib];
+  const uint64_t T = a.ctl->T[a.par];
+  const bool full = a.ctl->nsrch > 0;
+  const uint64_t Tw = full ? T : a.ctl->T0[a.par];
+  const int64_t nch = (int64_t)((Tw + kChunkW - 1) / kChunkW);
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->nch_last = (uint32_t)nch;  // for piece_pos
+  if (gw >= nch) return;  // warp-uniform; no block barriers below
+  const uint32_t m = a.m;
+  const uint32_t ilo = m > 1u ? m : 1u;
+  const bool y32 = a.ctl->y32 != 0;
+  const uint32_t yb = y32 ? 4u : 8u;
+  const uint32_t lt = (1u << lane) - 1u;
+
+  auto issue = [&](int s, int64_t ch) {  // lane 0
+    unsigned char* st = my + (size_t)s * SB;
+    Meta* mt = reinterpret_cast<Meta*>(st + off_meta(YB));
+    mt->ch = ch;
+    const uint64_t cbase = (uint64_t)ch * kChunkW;
+    const uint32_t sid = __ldg(a.desc + ch);
+    const PSeg* P = a.pseg + sid;
+    const uint64_t s0 = __ldg(&P->start), e0 = s0 + __ldg(&P->cnt);
+    const bool single = s0 <= cbase && e0 >= cbase + kChunkW;
+    if (!single || !(__ldg(&P->flags) & PS_SPLIT)) {
+      // whole chunk in one segment of a node that does not split: nothing to do; a chunk
+      // with segment heads inside: listed for fused_general_kernel
+      if (!single) a.gen_list[atomicAdd(&a.ctl->ngen, 1u)] = (uint32_t)ch;
+      mt->skip = 1u;
+      mbar_arrive(bar + s);
+      return;
+    }
+    mt->skip = 0u;
+    const uint32_t bytes = 2048u + 256u * yb + 32u + (uint32_t)sizeof(PSeg) + 64u;
+    fence_proxy_async_smem();
+    mbar_arrive_expect_tx(bar + s, bytes);
+    bulk_g2s(st + kOffX, a.lx + cbase, 1024u, bar + s);
+    bulk_g2s(st + kOffR, a.lr + cbase, 1024u, bar + s);
+    bulk_g2s(st + kOffY, reinterpret_cast<const unsigned char*>(a.ly) + cbase * yb, 256u * yb, bar + s);
+    bulk_g2s(st + off_gm(YB), a.gm + cbase / 8, 32u, bar + s);
+    bulk_g2s(st + off_ps(YB), P, (uint32_t)sizeof(PSeg), bar + s);
+    bulk_g2s(st + off_ce(YB), a.cexcl + ch, 32u, bar + s);
+    bulk_g2s(st + off_cb(YB), a.bcarry + ch / kBlockChunks, 32u, bar + s);
+  };
+  if (lane == 0) {
+    mbar_init(bar, 1);
+    mbar_init(bar + 1, 1);
+    mbar_init_fence();
+    issue(0, gw);
+    if (gw + nw < nch) issue(1, gw + nw);
+  }
+  __syncwarp();
+  int s = 0;
+  uint32_t phase = 0;
+  for (int64_t ch = gw; ch < nch; ch += nw) {
+    mbar_wait(bar + s, phase);
+    unsigned char* st = my + (size_t)s * SB;
+    const int64_t nxt = ch + 2 * nw;
+    const bool skip = reinterpret_cast<const Meta*>(st + off_meta(YB))->skip != 0u;
+    if (skip) {
+      __syncwarp();
+      if (lane == 0 && nxt < nch) issue(s, nxt);
+      if (++s == 2) { s = 0; phase ^= 1u; }
+      continue;
+    }
+    const uint64_t cbase = (uint64_t)ch * kChunkW;
+    // the plan of the chunk's first segment: kept in this warp's slot (the stage is
+    // refilled before the candidates are evaluated)
+    if (lane < (int)(sizeof(PSeg) / 16))
+      reinterpret_cast<uint4*>(cur)[lane] = reinterpret_cast<const uint4*>(st + off_ps(YB))[lane];
+    __syncwarp();
+    const PSeg& ps = *cur;
+    const float* sx = reinterpret_cast<const float*>(st + kOffX);
+    const uint32_t* sr = reinterpret_cast<const uint32_t*>(st + kOffR);
+    const unsigned char* sy = st + kOffY;
+    const uint8_t* sgm = st + off_gm(YB);
+    const uint32_t* sw = reinterpret_cast<const uint32_t*>(sgm);
+    const bool headc = ps.start == cbase;
+    AggP carry = agg_ident();
+    if (full && !headc) carry = combine(*reinterpret_cast<const AggP*>(st + off_cb(YB)),
+                                        *reinterpret_cast<const AggP*>(st + off_ce(YB)));
+    // lane items
+    float xv[kItems];
+    double yv[kItems];
+    {
+      const float4* x4 = reinterpret_cast<const float4*>(sx + lane * kItems);
+      const float4 q0 = x4[0], q1 = x4[1];
+      xv[0] = q0.x; xv[1] = q0.y; xv[2] = q0.z; xv[3] = q0.w;
+      xv[4] = q1.x; xv[5] = q1.y; xv[6] = q1.z; xv[7] = q1.w;
+      if (y32) {
+        const int4* y4 = reinterpret_cast<const int4*>(sy) + lane * 2;
+        const int4 r0 = y4[0], r1 = y4[1];
+        yv[0] = r0.x; yv[1] = r0.y; yv[2] = r0.z; yv[3] = r0.w;
+        yv[4] = r1.x; yv[5] = r1.y; yv[6] = r1.z; yv[7] = r1.w;
+      } else {
+        const double2* y2 = reinterpret_cast<const double2*>(sy) + lane * 4;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const double2 t = y2[q];
+          yv[2 * q] = t.x;
+          yv[2 * q + 1] = t.y;
+        }
+      }
+    }
+    const uint32_t gbyte = sgm[lane];
+    {
+      // =================== whole chunk inside one split segment =====================
+      const uint32_t flags = ps.flags;
+      const uint64_t ibase = cbase - ps.start;  // local index of the chunk's entry 0
+      // ---- partition: row-wise coalesced stores (row r = entries 32r .. 32r+31)
+      if (full && (flags & (PS_WR0 | PS_WR1))) {
+        uint32_t pre = carry.nl;
+#pragma unroll
+        for (int r = 0; r < kItems; ++r) {
+          const uint32_t wr = sw[r];
+          const uint32_t g = (wr >> lane) & 1u;
+          const uint32_t rk = pre + __popc(wr & lt);
+          const int e = 32 * r + lane;
+          if (g ? (flags & PS_WR0) : (flags & PS_WR1)) {
+            const uint64_t dst = g ? ps.ostart[0] + rk : ps.ostart[1] + (ibase + (uint64_t)e - rk);
+            store_entry(a, y32, dst, sx[e], sr[e], sy + (size_t)e * yb, ps.cs[g ? 0 : 1]);
+          }
+          pre += __popc(wr);
+        }
+      }
+      // ---- left count before my items, neighbour x across lanes
+      uint32_t nl = carry.nl;
+      {
+        const int wq = lane >> 2;
+#pragma unroll
+        for (int r = 0; r < kItems; ++r)
+          if (r < wq) nl += __popc(sw[r]);
+        nl += __popc(sw[wq] & ((1u << (8 * (lane & 3))) - 1u));
+      }
+      const uint32_t Lm = __ballot_sync(0xffffffffu, gbyte != 0u) & lt;
+      const uint32_t Rm = __ballot_sync(0xffffffffu, gbyte != 0xffu) & lt;
+      float xl = carry.xl, xr = carry.xr;
+      if (Lm) {
+        const int h = 31 - __clz(Lm);
+        xl = sx[8 * h + 31 - __clz((uint32_t)sgm[h])];
+      }
+      if (Rm) {
+        const int h = 31 - __clz(Rm);
+        xr = sx[8 * h + 31 - __clz(~(uint32_t)sgm[h] & 0xffu)];
+      }
+      if (isnan(xl)) xl = ps.xprev[0];
+      if (isnan(xr)) xr = ps.xprev[1];
+      __syncwarp();  // the stage is read completely: refill it
+      if (lane == 0 && nxt < nch) issue(s, nxt);
+      // ---- children's prefix sums: lane sums, Kogge-Stone across lanes, chunk carry
+      const double c0 = ps.c[0], c1 = ps.c[1];
+      double sl = 0.0, srr = 0.0;
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        if ((gbyte >> j) & 1u) sl = __dadd_rn(sl, __dsub_rn(yv[j], c0));
+        else srr = __dadd_rn(srr, __dsub_rn(yv[j], c1));
+      }
+      double il = sl, ir = srr;
+      warp_incl2(il, ir);
+      double SL = __shfl_up_sync(0xffffffffu, il, 1), SR = __shfl_up_sync(0xffffffffu, ir, 1);
+      if (lane == 0) { SL = 0.0; SR = 0.0; }
+      SL = __dadd_rn(carry.sl, SL);
+      SR = __dadd_rn(carry.sr, SR);
+      // ---- valid positions of both children, compacted
+      if (full && (flags & (PS_SRCH0 | PS_SRCH1))) {
+        const uint32_t i0 = (uint32_t)(ibase + (uint64_t)(lane * kItems));
+        double tS[kItems];
+        uint32_t tJ[kItems];
+        float tP[kItems];
+        uint32_t vm = 0u;
+        uint32_t nlj = nl;
+        double SLj = SL, SRj = SR;
+        float xlj = xl, xrj = xr;
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+          const float x = xv[j];
+          if ((gbyte >> j) & 1u) {
+            const uint32_t jg = ps.ioff[0] + nlj;
+            if ((flags & PS_SRCH0) && jg >= ilo && ps.N[0] - jg >= m && xlj < x) {
+              vm |= 1u << j;
+              tS[j] = __dadd_rn(ps.soff[0], SLj);
+              tJ[j] = jg;
+              tP[j] = xlj;
+            }
+            SLj = __dadd_rn(SLj, __dsub_rn(yv[j], c0));
+            ++nlj;
+            xlj = x;
+          } else {
+            const uint32_t jg = ps.ioff[1] + (i0 + j - nlj);
+            if ((flags & PS_SRCH1) && jg >= ilo && ps.N[1] - jg >= m && xrj < x) {
+              vm |= 1u << j;
+              tS[j] = __dadd_rn(ps.soff[1], SRj);
+              tJ[j] = jg | 0x80000000u;
+              tP[j] = xrj;
+            }
+            SRj = __dadd_rn(SRj, __dsub_rn(yv[j], c1));
+            xrj = x;
+          }
+        }
+        const uint32_t nv = __popc(vm);
+        uint32_t vinc = nv;
+#pragma unroll
+        for (int dd = 1; dd < 32; dd <<= 1) {
+          const uint32_t o = __shfl_up_sync(0xffffffffu, vinc, dd);
+          if (lane >= dd) vinc += o;
+        }
+        const uint32_t vtot = __shfl_sync(0xffffffffu, vinc, 31);
+        if (vtot) {
+          uint32_t q = vinc - nv;
+#pragma unroll
+          for (int j = 0; j < kItems; ++j) {
+            if ((vm >> j) & 1u) {
+              cbuf.S[q] = tS[j];
+              cbuf.js[q] = tJ[j];
+              cbuf.xp[q] = tP[j];
+              cbuf.xv[q] = xv[j];
+              ++q;
+            }
+          }
+          __syncwarp();
+          double bg[2] = {-1.0, -1.0};
+          uint32_t bj[2] = {0xffffffffu, 0xffffffffu}, be[2] = {0u, 0u};
+          const double N0 = (double)ps.N[0], N1 = (double)ps.N[1];
+          const double sc0 = ps.sc[0], sc1 = ps.sc[1];
+          for (uint32_t e = lane; e < vtot; e += 32) {
+            const uint32_t js = cbuf.js[e];
+            const int side = (int)(js >> 31);
+            const uint32_t jg = js & 0x7fffffffu;
+            const double g = split_gain_d(cbuf.S[e], side ? sc1 : sc0, (double)jg, side ? N1 : N0);
+            if (side == 0) {
+              if (g > bg[0]) { bg[0] = g; bj[0] = jg; be[0] = e; }
+            } else {
+              if (g > bg[1]) { bg[1] = g; bj[1] = jg; be[1] = e; }
+            }
+          }
+#pragma unroll
+          for (int side = 0; side < 2; ++side) {
+            double gmx = bg[side];
+#pragma unroll
+            for (int off = 16; off > 0; off >>= 1) gmx = fmax(gmx, __shfl_xor_sync(0xffffffffu, gmx, off));
+            if (gmx >= 0.0) {
+              const uint32_t jmin = __reduce_min_sync(0xffffffffu, bg[side] == gmx ? bj[side] : 0xffffffffu);
+              const int src = __ffs(__ballot_sync(0xffffffffu, bg[side] == gmx && bj[side] == jmin)) - 1;
+              const uint32_t e = __shfl_sync(0xffffffffu, be[side], src);
+              if (lane == 0)
+                put_cand(a, headc, ch, side, ps.cs[side], gmx, cbuf.S[e], mid_threshold(cbuf.xp[e], cbuf.xv[e]), jmin);
+            }
+          }
+          __syncwarp();  // the buffer is rewritten by the next chunk
+        }
+      }
+      // ---- children's statistics from feature 0
+      if (ps.f == 0) {
+        StatQ q0 = statq_ident(), q1 = statq_ident();
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+          if ((gbyte >> j) & 1u) stat_add(q0, yv[j], ps.v[0], c0);
+          else stat_add(q1, yv[j], ps.v[1], c1);
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) {
+          q0.sse = __dadd_rn(q0.sse, __shfl_xor_sync(0xffffffffu, q0.sse, off));
+          q0.ymin = fmin(q0.ymin, __shfl_xor_sync(0xffffffffu, q0.ymin, off));
+          q0.ymax = fmax(q0.ymax, __shfl_xor_sync(0xffffffffu, q0.ymax, off));
+          q0.s1 = __dadd_rn(q0.s1, __shfl_xor_sync(0xffffffffu, q0.s1, off));
+          q1.sse = __dadd_rn(q1.sse, __shfl_xor_sync(0xffffffffu, q1.sse, off));
+          q1.ymin = fmin(q1.ymin, __shfl_xor_sync(0xffffffffu, q1.ymin, off));
+          q1.ymax = fmax(q1.ymax, __shfl_xor_sync(0xffffffffu, q1.ymax, off));
+          q1.s1 = __dadd_rn(q1.s1, __shfl_xor_sync(0xffffffffu, q1.s1, off));
+        }
+        if (lane == 0) {
+          put_stat(a, headc, ch, 0, ps.kid, q0);
+          if (!(flags & PS_ALLLEFT)) put_stat(a, headc, ch, 1, ps.kid + 1, q1);
+        }
+      }
+    }
+    if (++s == 2) { s = 0; phase ^= 1u; }
+  }
+}
+
+// F_C for the chunks with segment heads inside (listed by fused_kernel): one warp per
+// chunk, the entries read directly (these chunks appear at deep levels, where nodes are
+// small); per lane a walk over its 8 entries' segments, segmented warp scans of the lanes'
+// runs for the candidate / statistics pieces of every segment in the chunk.
+__global__ void __launch_bounds__(kThreads) fused_general_kernel(FusedArgs a) {
+  const int lane = threadIdx.x & 31;
+  const int64_t ngen = a.ctl->ngen;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const uint64_t T = a.ctl->T[a.par];
+  const bool full = a.ctl->nsrch > 0;
+  const bool y32 = a.ctl->y32 != 0;
+  const uint32_t yb = y32 ? 4u : 8u;
+  const uint32_t m = a.m;
+  const uint32_t ilo = m > 1u ? m : 1u;
+  for (int64_t idx = gw; idx < ngen; idx += nw) {
+    const int64_t ch = (int64_t)a.gen_list[idx];
+    const uint64_t cbase = (uint64_t)ch * kChunkW;
+    const float* sx = a.lx + cbase;
+    const uint32_t* sr = a.lr + cbase;
+    const unsigned char* sy = reinterpret_cast<const unsigned char*>(a.ly) + cbase * yb;
+    const uint32_t sid0 = __ldg(a.desc + ch);
+    const uint64_t ps_start = __ldg(&a.pseg[sid0].start);
+    const int32_t ps_f = __ldg(&a.pseg[sid0].f);
+    const bool headc = ps_start == cbase;
+    AggP carry = agg_ident();
+    if (full && !headc) carry = combine(a.bcarry[ch / kBlockChunks], a.cexcl[ch]);
+    float xv[kItems];
+    double yv[kItems];
+    const uint64_t pl = cbase + (uint64_t)(lane * kItems);
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+      const bool ok = pl + j < T;
+      xv[j] = ok ? sx[lane * kItems + j] : 0.f;
+      yv[j] = ok ? y_at(a.ly, (int64_t)(pl + j), y32) : 0.0;
+    }
+    const uint32_t gbyte = a.gm[cbase / 8 + lane];
+      // =================== general chunk: segment heads inside =======================
+      const uint64_t p0 = cbase + (uint64_t)(lane * kItems);
+      // pass 1: my trailing run's aggregate (segments walked from the chunk's first)
+      uint32_t sid = __ldg(a.desc + ch);
+      SegCtx cx;
+      load_ctx(cx, a.pseg + sid);
+      AggP run = agg_ident();
+      int lastL = -1, lastR = -1;
+      {
+        uint32_t s2 = sid;
+        uint64_t e2 = cx.end, st2 = cx.start;
+        uint32_t fl2 = cx.flags;
+        double c20 = cx.c[0], c21 = cx.c[1];
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+          const uint64_t p = p0 + j;
+          if (p < T) {
+            while (p >= e2) {
+              ++s2;
+              st2 = __ldg(&a.pseg[s2].start);
+              e2 = st2 + __ldg(&a.pseg[s2].cnt);
+              fl2 = __ldg(&a.pseg[s2].flags);
+              c20 = __ldg(&a.pseg[s2].c[0]);
+              c21 = __ldg(&a.pseg[s2].c[1]);
+            }
+            if (p == st2) {
+              run = agg_ident();
+              run.flag = 1u;
+              lastL = lastR = -1;
+            }
+            if (fl2 & PS_SPLIT) {
+              if ((gbyte >> j) & 1u) {
+                run.nl += 1u;
+                run.sl = __dadd_rn(run.sl, __dsub_rn(yv[j], c20));
+                lastL = j;
+              } else {
+                run.sr = __dadd_rn(run.sr, __dsub_rn(yv[j], c21));
+                lastR = j;
+              }
+            }
+          }
+        }
+      }
+      if (lastL >= 0) run.xl = sx[lane * kItems + lastL];
+      if (lastR >= 0) run.xr = sx[lane * kItems + lastR];
+      AggP wagg;
+      const AggP ex = warp_excl_seg(run, agg_ident(), wagg);
+      const AggP E = combine(carry, ex);  // the open segment's state at my first item
+      // pass 2: positions, candidates, statistics, stores
+      const bool stats_chunk = ps_f == 0;
+      // walk to the segment of my first item
+      {
+        uint64_t q = p0 < T ? p0 : T - 1;
+        while (q >= cx.end) load_ctx(cx, a.pseg + (++sid));
+      }
+      uint32_t nl = E.nl;
+      double SL = E.sl, SR = E.sr;
+      float xl = isnan(E.xl) ? cx.xp[0] : E.xl, xr = isnan(E.xr) ? cx.xp[1] : E.xr;
+      // runs: the one open at my first item (its part before my first head: "first")
+      // and the current one
+      ArgQ fa0 = argq_ident(), fa1 = argq_ident(), ca0 = argq_ident(), ca1 = argq_ident();
+      StatQ fs0 = statq_ident(), fs1 = statq_ident(), cs0 = statq_ident(), cs1 = statq_ident();
+      bool seen = false;
+      // ids of the run's segment
+      uint32_t rcs0 = cx.cs[0], rcs1 = cx.cs[1], rkid = cx.kid, rfl = cx.flags;
+      int rf = cx.f;
+      const uint32_t fcs0 = cx.cs[0], fcs1 = cx.cs[1], fkid = cx.kid, ffl = cx.flags;
+      const int ff = cx.f;
+      bool item0_head = false;
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        const uint64_t p = p0 + j;
+        if (p < T) {
+          while (p >= cx.end) load_ctx(cx, a.pseg + (++sid));
+          if (p == cx.start) {
+            if (j == 0) item0_head = true;
+            if (!seen) {
+              fa0 = ca0; fa1 = ca1; fs0 = cs0; fs1 = cs1;
+            } else {
+              // a run that started at a head inside this lane ends here: complete piece
+              if (full && (rfl & PS_SPLIT)) {
+                if ((rfl & PS_SRCH0) && ca0.gain >= 0.0) put_cand(a, true, ch, 0, rcs0, ca0.gain, ca0.sl, ca0.thr, ca0.j);
+                if ((rfl & PS_SRCH1) && ca1.gain >= 0.0) put_cand(a, true, ch, 1, rcs1, ca1.gain, ca1.sl, ca1.thr, ca1.j);
+              }
+              if (rf == 0 && (rfl & PS_SPLIT)) {
+                put_stat(a, true, ch, 0, rkid, cs0);
+                if (!(rfl & PS_ALLLEFT)) put_stat(a, true, ch, 1, rkid + 1, cs1);
+              }
+            }
+            seen = true;
+            ca0 = argq_ident(); ca1 = argq_ident(); ca0.flag = ca1.flag = 1u;
+            cs0 = statq_ident(); cs1 = statq_ident(); cs0.flag = cs1.flag = 1u;
+            nl = 0u;
+            SL = 0.0;
+            SR = 0.0;
+            xl = cx.xp[0];
+            xr = cx.xp[1];
+            rcs0 = cx.cs[0]; rcs1 = cx.cs[1]; rkid = cx.kid; rfl = cx.flags; rf = cx.f;
+          }
+          if (cx.flags & PS_SPLIT) {
+            const float x = xv[j];
+            const double y = yv[j];
+            const uint32_t i = (uint32_t)(p - cx.start);
+            if ((gbyte >> j) & 1u) {
+              if (full) {
+                const uint32_t jg = cx.ioff[0] + nl;
+                if ((cx.flags & PS_SRCH0) && jg >= ilo && cx.N[0] - jg >= m && xl < x) {
+                  const double S = __dadd_rn(cx.soff[0], SL);
+                  const double g = split_gain_d(S, cx.sc[0], (double)jg, (double)cx.N[0]);
+                  if (g > ca0.gain) { ca0.gain = g; ca0.j = jg; ca0.sl = S; ca0.thr = mid_threshold(xl, x); }
+                }
+                if (cx.flags & PS_WR0)
+                  store_entry(a, y32, cx.os[0] + nl, x, sr[lane * kItems + j], sy + (size_t)(lane * kItems + j) * yb, cx.cs[0]);
+              }
+              if (cx.f == 0) stat_add(cs0, y, cx.v[0], cx.c[0]);
+              SL = __dadd_rn(SL, __dsub_rn(y, cx.c[0]));
+              ++nl;
+              xl = x;
+            } else {
+              if (full) {
+                const uint32_t jr = i - nl;
+                const uint32_t jg = cx.ioff[1] + jr;
+                if ((cx.flags & PS_SRCH1) && jg >= ilo && cx.N[1] - jg >= m && xr < x) {
+                  const double S = __dadd_rn(cx.soff[1], SR);
+                  const double g = split_gain_d(S, cx.sc[1], (double)jg, (double)cx.N[1]);
+                  if (g > ca1.gain) { ca1.gain = g; ca1.j = jg; ca1.sl = S; ca1.thr = mid_threshold(xr, x); }
+                }
+                if (cx.flags & PS_WR1)
+                  store_entry(a, y32, cx.os[1] + jr, x, sr[lane * kItems + j], sy + (size_t)(lane * kItems + j) * yb, cx.cs[1]);
+              }
+              if (cx.f == 0) stat_add(cs1, y, cx.v[1], cx.c[1]);
+              SR = __dadd_rn(SR, __dsub_rn(y, cx.c[1]));
+              xr = x;
+            }
+          }
+        }
+      }
+      if (!seen) { fa0 = ca0; fa1 = ca1; fs0 = cs0; fs1 = cs1; }
+      // segmented scans of the lane trails (the last run, flagged when it began at a head)
+      ArgQ ta0 = ca0, ta1 = ca1;
+      ta0.flag = ta1.flag = seen ? 1u : 0u;
+      ArgQ w0, w1;
+      const ArgQ ax0 = warp_excl_seg(ta0, argq_ident(), w0);
+      const ArgQ ax1 = warp_excl_seg(ta1, argq_ident(), w1);
+      StatQ sx0 = statq_ident(), sx1 = statq_ident();
+      if (stats_chunk) {
+        StatQ ts0 = cs0, ts1 = cs1, v0, v1;
+        ts0.flag = ts1.flag = seen ? 1u : 0u;
+        sx0 = warp_excl_seg(ts0, statq_ident(), v0);
+        sx1 = warp_excl_seg(ts1, statq_ident(), v1);
+      }
+      // the segment open at my first item ends in this lane: its piece = earlier lanes + "first"
+      if (seen && !(lane == 0 && item0_head) && !item0_head) {
+        const bool h = ax0.flag != 0;  // its head lies in an earlier lane of this chunk
+        if (full && (ffl & PS_SPLIT)) {
+          const ArgQ d0 = combine(ax0, fa0), d1 = combine(ax1, fa1);
+          if ((ffl & PS_SRCH0) && d0.gain >= 0.0) put_cand(a, h, ch, 0, fcs0, d0.gain, d0.sl, d0.thr, d0.j);
+          if ((ffl & PS_SRCH1) && d1.gain >= 0.0) put_cand(a, h, ch, 1, fcs1, d1.gain, d1.sl, d1.thr, d1.j);
+        }
+        if (ff == 0 && (ffl & PS_SPLIT)) {
+          put_stat(a, h, ch, 0, fkid, combine(sx0, fs0));
+          if (!(ffl & PS_ALLLEFT)) put_stat(a, h, ch, 1, fkid + 1, combine(sx1, fs1));
+        }
+      } else if (seen && item0_head && lane > 0) {
+        // my first item is a head: the segment open before me ended in an earlier lane;
+        // its piece (earlier lanes only) is closed here
+        // the previous non-empty segment: the one holding position p0 - 1
+        SegCtx pc;
+        {
+          uint32_t t2 = __ldg(a.desc + ch);
+          load_ctx(pc, a.pseg + t2);
+          while (p0 - 1 >= pc.end) load_ctx(pc, a.pseg + (++t2));
+        }
+        const bool h = ax0.flag != 0;
+        if (full && (pc.flags & PS_SPLIT)) {
+          if ((pc.flags & PS_SRCH0) && ax0.gain >= 0.0) put_cand(a, h, ch, 0, pc.cs[0], ax0.gain, ax0.sl, ax0.thr, ax0.j);
+          if ((pc.flags & PS_SRCH1) && ax1.gain >= 0.0) put_cand(a, h, ch, 1, pc.cs[1], ax1.gain, ax1.sl, ax1.thr, ax1.j);
+        }
+        if (pc.f == 0 && (pc.flags & PS_SPLIT)) {
+          put_stat(a, h, ch, 0, pc.kid, sx0);
+          if (!(pc.flags & PS_ALLLEFT)) put_stat(a, h, ch, 1, pc.kid + 1, sx1);
+        }
+      }
+      // the last lane closes the segment open at the chunk's end
+      if (lane == 31) {
+        SegCtx lc;
+        bool lh;
+        ArgQ d0, d1;
+        StatQ e0, e1;
+        if (p0 < T && seen) {
+          lc = cx;  // my last run began at a head in my items
+          lh = true;
+          d0 = ca0; d1 = ca1; e0 = cs0; e1 = cs1;
+        } else {
+          // no head in my items (or no items): earlier lanes + my run
+          const uint64_t last = (cbase + kChunkW <= T ? cbase + kChunkW : T) - 1;
+          uint32_t t2 = __ldg(a.desc + ch);
+          load_ctx(lc, a.pseg + t2);
+          while (last >= lc.end) load_ctx(lc, a.pseg + (++t2));
+          lh = ax0.flag != 0;
+          d0 = combine(ax0, ca0); d1 = combine(ax1, ca1);
+          e0 = combine(sx0, cs0); e1 = combine(sx1, cs1);
+        }
+        if (full && (lc.flags & PS_SPLIT)) {
+          if ((lc.flags & PS_SRCH0) && d0.gain >= 0.0) put_cand(a, lh, ch, 0, lc.cs[0], d0.gain, d0.sl, d0.thr, d0.j);
+          if ((lc.flags & PS_SRCH1) && d1.gain >= 0.0) put_cand(a, lh, ch, 1, lc.cs[1], d1.gain, d1.sl, d1.thr, d1.j);
+        }
+        if (lc.f == 0 && (lc.flags & PS_SPLIT)) {
+          put_stat(a, lh, ch, 0, lc.kid, e0);
+          if (!(lc.flags & PS_ALLLEFT)) put_stat(a, lh, ch, 1, lc.kid + 1, e1);
+        }
+      }
+  }
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------------ launchers --
+
+namespace {
+int grid_for(const void* kern, int threads, size_t smem) {
+  int per = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, kern, threads, smem);
+  if (per < 1) per = 1;
+  return num_sms() * per;
+}
+constexpr int64_t kMaxSmemBits = 227 * 1024;
+}  // namespace
+
+// F_A + F_B of the pass whose parent level is la.level (la.level = -1: the virtual root).
+dt_status level_agg_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t s) {
+  AggArgs a;
+  a.lr = b.lr[la.cur];
+  a.ly = b.ly[la.cur];
+  a.lx = b.lx[la.cur];
+  a.desc = b.desc[la.par];
+  a.pseg = b.pseg;
+  a.gbits = b.gbits;
+  a.gm = b.gm;
+  a.agg = b.agg;
+  a.tails = b.tails;
+  a.ctl = b.ctl;
+  a.par = la.par;
+  a.nwords = b.nwords4;
+  const size_t bytes = sizeof(uint32_t) * (size_t)b.nwords4;
+  if ((int64_t)bytes <= kMaxSmemBits) {
+    auto k = la.tails ? level_agg_kernel<true, true> : level_agg_kernel<true, false>;
+    DT_CK(cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes));
+    k<<<num_sms(), 1024, bytes, s>>>(a);
+  } else {
+    auto k = la.tails ? level_agg_kernel<false, true> : level_agg_kernel<false, false>;
+    k<<<grid_for((const void*)k, kThreads, 0), kThreads, 0, s>>>(a);
+  }
+  DT_CK(cudaGetLastError());
+  agg_scan_kernel<<<(unsigned)b.max_cblocks, 1024, 0, s>>>(b.ctl, la.par, b.agg, b.cexcl, b.bagg, b.bcarry);
+  DT_CK(cudaGetLastError());
+  return DT_OK;
+}
+
+size_t fused_smem() {
+  const size_t sb = (stage_bytes_for(8u) + 127u) & ~127u;
+  constexpr int kWarps = kThreads / 32;
+  return sb * 2 * kWarps + kWarps * 2 * sizeof(uint64_t) + kWarps * sizeof(PSeg) + kWarps * sizeof(Compact);
+}
+
+// F_C of the pass whose parent level is la.level.
+dt_status level_fused_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t s) {
+  FusedArgs a;
+  a.lx = b.lx[la.cur];
+  a.lr = b.lr[la.cur];
+  a.ly = b.ly[la.cur];
+  a.ox = b.lx[la.cur ^ 1];
+  a.orow = b.lr[la.cur ^ 1];
+  a.oy = b.ly[la.cur ^ 1];
+  a.desc = b.desc[la.par];
+  a.desc_next = b.desc[la.par ^ 1];
+  a.pseg = b.pseg;
+  a.gm = b.gm;
+  a.cexcl = b.cexcl;
+  a.bcarry = b.bcarry;
+  a.head_cand = b.head_cand;
+  a.cont_cand = b.cont_cand;
+  a.slot_gain = b.slot_gain;
+  a.head_stat = b.head_stat;
+  a.cont_stat = b.cont_stat;
+  a.ctl = b.ctl;
+  a.par = la.par;
+  a.level = (uint32_t)(la.level + 1);
+  a.m = (uint32_t)std::min<int64_t>(la.min_leaf, 0x7fffffff);
+  a.ystride = 0;
+  a.stage_bytes = 0;
+  const size_t sm = fused_smem();
+  a.gen_list = b.gen_list;
+  auto k = fused_kernel;
+  DT_CK(cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+  k<<<grid_for((const void*)k, kThreads, sm), kThreads, sm, s>>>(a);
+  DT_CK(cudaGetLastError());
+  fused_general_kernel<<<grid_for((const void*)fused_general_kernel, kThreads, 0), kThreads, 0, s>>>(a);
+  DT_CK(cudaGetLastError());
+  return DT_OK;
+}
+
+}  // namespace dtl

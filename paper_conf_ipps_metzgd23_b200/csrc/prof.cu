@@ -20,7 +20,7 @@ bool g_on = false;
 std::vector<Rec> g_recs;
 long long g_launches = 0;
 const char* kNames[] = {"presort_keys", "presort_sort", "presort_build", "root_stats",
-                        "scan", "select", "number", "goleft", "partition", "predict",
+                        "agg", "select", "number", "goleft", "fused", "predict",
                         "eval", "loo", "gen", "memset"};
 constexpr int kNumKinds = sizeof(kNames) / sizeof(kNames[0]);
 }  // namespace
