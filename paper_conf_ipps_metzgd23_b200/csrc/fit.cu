@@ -210,7 +210,7 @@ __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
   // nothing reads the bitmap between the previous level's F_A and this level's goleft
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + tid; i < a.nvec; i += (int64_t)gridDim.x * blockDim.x)
     a.gbits[i] = make_uint4(0u, 0u, 0u, 0u);
-  if (blockIdx.x == 0 && tid == 0) a.ctl->ngen = 0u;  // the next fused pass lists its general chunks
+  if (blockIdx.x == 0 && tid == 0) a.ctl->nfast = a.ctl->ngen = a.ctl->nunit = a.ctl->nbig = 0u;  // next chunk plan
   if (blockIdx.x == 0 && tid == 0 && a.level < kMaxLogLevels) {
     a.log[a.level].T = a.ctl->T[a.par];
     a.log[a.level].K = K;
@@ -674,6 +674,9 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int64_t n_global, int32_t d, int32_t 
   GET(b.bcarry, b.max_cblocks);
   GET(b.gm, b.max_chunks * 32);
   GET(b.gen_list, b.max_chunks);
+  GET(b.fast_list, b.max_chunks);
+  GET(b.unit_list, b.max_chunks * 9);  // <= 8 pieces per listed chunk (kMaxPieces)
+  GET(b.big_list, b.max_chunks);
   GET(b.head_cand, b.segcap);
   GET(b.cont_cand, 2 * b.max_chunks);
   GET(b.slot_gain, b.segcap);

@@ -182,7 +182,10 @@ struct Ctl {
   uint32_t ticket;
   uint32_t nsrch;            // searchable children of the current pass (0: statistics only)
   uint32_t nch_last;         // chunks processed by the last fused pass (its candidate pieces)
-  uint32_t ngen;             // chunks with segment heads inside, listed by the fused pass
+  uint32_t nfast;            // chunk plan of the pass: chunks inside one split segment,
+  uint32_t ngen;             //   chunks with segment heads inside,
+  uint32_t nunit;            //   split segment pieces of chunks (the fused pass),
+  uint32_t nbig;             //   chunks with too many pieces
   unsigned long long split_evals;
   double ysum, ymin, ymax, ysc;
 };
@@ -242,7 +245,10 @@ struct FitBufs {
   AggP *agg, *cexcl, *bagg, *bcarry;
   AggP* tails;         // sharded: per parent segment, its aggregate from its last chunk
   uint8_t* gm;         // go-left bits per chunk entry (32 B per chunk)
-  uint32_t* gen_list;  // chunks with segment heads inside (per fused pass)
+  uint2* fast_list;    // chunk plan of the pass: {chunk, segment} inside one split segment
+  uint32_t* gen_list;  // chunks with segment heads inside
+  uint2* unit_list;    // {chunk, segment}: split segment pieces of chunks (fused pass)
+  uint32_t* big_list;  // chunks with more than kMaxPieces pieces
   Cand2 *head_cand, *cont_cand;
   unsigned long long *slot_gain, *slot_pos;
   Stat *head_stat, *cont_stat;

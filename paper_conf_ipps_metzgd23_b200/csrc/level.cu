@@ -22,6 +22,7 @@
 // across chunks the F_B tree), so results are bit-reproducible; in integer mode every
 // sum is exact, so the trees are independent of the summation order (Reading R17).
 #include <algorithm>
+#include <type_traits>
 
 #include "bulk.cuh"
 #include "fit_core.cuh"
@@ -31,6 +32,9 @@ namespace dtl {
 namespace {
 
 constexpr int kThreads = 256;
+#ifndef DT_FUSED_MINB
+#define DT_FUSED_MINB 2  // CTAs per SM of the fused pass (register budget; 3 spills: slower)
+#endif
 constexpr float kNaN = __builtin_nanf("");
 
 __device__ __forceinline__ double y_at(const double* __restrict__ ly, int64_t p, bool y32) {
@@ -49,6 +53,8 @@ struct AggArgs {
   uint8_t* gm;
   AggP* agg;
   AggP* tails;
+  const uint2* fast_list;
+  const uint32_t* gen_list;
   const Ctl* ctl;
   int par;
   int64_t nwords;
@@ -132,15 +138,154 @@ __device__ __forceinline__ SegLite seg_lite(const PSeg* __restrict__ ps, uint32_
   return r;
 }
 
+// Chunk plan of a pass (thread per chunk).  A chunk inside ONE segment: of a split node
+// -> fast list {chunk, segment} (F_A fast path) and unit list (F_C); of a node that does
+// not split -> nothing to do (its aggregate is written here).  A chunk with segment heads
+// inside -> gen list (F_A general path) and, per split segment piece, the unit list when
+// it has at most kMaxPieces such pieces (F_C processes the chunk once per piece, masked to
+// the piece's entries), else the big list (fused_general_kernel).  Warp-aggregated appends.
+constexpr int kMaxPieces = 8;
+
+__device__ __forceinline__ uint32_t warp_append(uint32_t cnt, uint32_t* counter) {
+  const int lane = threadIdx.x & 31;
+  uint32_t inc = cnt;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t o = __shfl_up_sync(0xffffffffu, inc, d);
+    if (lane >= d) inc += o;
+  }
+  const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
+  uint32_t base = 0;
+  if (lane == 31 && tot) base = atomicAdd(counter, tot);
+  base = __shfl_sync(0xffffffffu, base, 31);
+  return base + inc - cnt;
+}
+
+__global__ void __launch_bounds__(256) chunk_plan_kernel(Ctl* ctl, int par, int d, const uint32_t* __restrict__ desc,
+                                                         const PSeg* __restrict__ pseg, AggP* __restrict__ agg,
+                                                         uint2* __restrict__ fast_list, uint32_t* __restrict__ gen_list,
+                                                         uint2* __restrict__ unit_list, uint32_t* __restrict__ big_list) {
+  const uint64_t T = ctl->T[par];
+  const bool full = ctl->nsrch > 0;  // children searched: every list; else feature 0 (statistics)
+  const uint64_t Tw = full ? T : ctl->T0[par];
+  const int64_t nch = (int64_t)((Tw + kChunkW - 1) / kChunkW);
+  const uint32_t nseg = ctl->K[par] * (uint32_t)d;  // segments of the parent level
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < nch; base += stride) {  // warp-uniform trip count
+    const int64_t ch = base + threadIdx.x;
+    bool fast = false, gen = false, big = false;
+    uint32_t npieces = 0;
+    uint32_t s = 0;
+    if (ch < nch) {
+      const uint64_t cbase = (uint64_t)ch * kChunkW, cend = min(cbase + kChunkW, T);
+      s = __ldg(desc + ch);
+      const uint64_t st = __ldg(&pseg[s].start), en = st + __ldg(&pseg[s].cnt);
+      const bool split = (__ldg(&pseg[s].flags) & PS_SPLIT) != 0;
+      if (st <= cbase && en >= cbase + kChunkW) {
+        if (split) fast = true;
+        else {
+          AggP z = agg_ident();
+          z.flag = st == cbase ? 1u : 0u;
+          agg[ch] = z;
+        }
+      } else {
+        gen = true;
+        for (uint32_t t = s; t < nseg; ++t) {  // split segment pieces of this chunk
+          const uint64_t ts = __ldg(&pseg[t].start);
+          if (ts >= cend) break;
+          if (__ldg(&pseg[t].cnt) && (__ldg(&pseg[t].flags) & PS_SPLIT)) ++npieces;
+          if (npieces > (uint32_t)kMaxPieces) break;
+        }
+        if (npieces > (uint32_t)kMaxPieces) {
+          big = true;
+          npieces = 0;
+        }
+      }
+    }
+    const uint32_t pf = warp_append(fast ? 1u : 0u, &ctl->nfast);
+    const uint32_t pg = warp_append(gen ? 1u : 0u, &ctl->ngen);
+    const uint32_t pb = warp_append(big ? 1u : 0u, &ctl->nbig);
+    uint32_t pu = warp_append(fast ? 1u : npieces, &ctl->nunit);
+    if (fast) {
+      fast_list[pf] = make_uint2((uint32_t)ch, s);
+      unit_list[pu] = make_uint2((uint32_t)ch, s);
+    }
+    if (gen) gen_list[pg] = (uint32_t)ch;
+    if (big) big_list[pb] = (uint32_t)ch;
+    if (npieces) {
+      const uint64_t cend = min((uint64_t)ch * kChunkW + kChunkW, T);
+      for (uint32_t t = s; t < nseg; ++t) {
+        if (__ldg(&pseg[t].start) >= cend) break;
+        if (__ldg(&pseg[t].cnt) && (__ldg(&pseg[t].flags) & PS_SPLIT)) unit_list[pu++] = make_uint2((uint32_t)ch, t);
+      }
+    }
+  }
+}
+
+// One fast chunk of the aggregate pass: go-left bits, sums, last x of both sides.
+template <bool kSmemBits, bool kTails>
+__device__ __forceinline__ void agg_fast_chunk(const AggArgs& a, const uint32_t* __restrict__ bits, int64_t ch,
+                                               uint32_t s, const uint32_t* rv, const double* yv) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t cbase = (uint64_t)ch * kChunkW;
+  const int64_t p0 = (int64_t)cbase + lane * kItems;
+  const uint64_t st = __ldg(&a.pseg[s].start);
+  const uint32_t flags = __ldg(&a.pseg[s].flags);
+  const double c0 = __ldg(&a.pseg[s].c[0]), c1 = __ldg(&a.pseg[s].c[1]);
+  uint32_t gbyte = 0xffu;
+  if (!(flags & PS_ALLLEFT)) {
+    uint32_t wv[kItems];
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) wv[j] = bits[rv[j] >> 5];  // independent shared-memory loads
+    gbyte = 0u;
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) gbyte |= ((wv[j] >> (rv[j] & 31)) & 1u) << j;
+  }
+  double sl = 0.0, sr = 0.0;
+#pragma unroll
+  for (int j = 0; j < kItems; ++j) {
+    const bool g = (gbyte >> j) & 1u;
+    const double d = __dsub_rn(yv[j], g ? c0 : c1);
+    // adding +0.0 is exact: a sum of (y - c) terms is never -0.0
+    sl = __dadd_rn(sl, g ? d : 0.0);
+    sr = __dadd_rn(sr, g ? 0.0 : d);
+  }
+  warp_incl2(sl, sr);
+  const uint32_t Lm = __ballot_sync(0xffffffffu, gbyte != 0u);
+  const uint32_t Rm = __ballot_sync(0xffffffffu, gbyte != 0xffu);
+  AggP out;
+  out.flag = st == cbase ? 1u : 0u;
+  out.nl = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(gbyte));
+  out.sl = __shfl_sync(0xffffffffu, sl, 31);
+  out.sr = __shfl_sync(0xffffffffu, sr, 31);
+  out.xl = kNaN;
+  out.xr = kNaN;
+  if (Lm) {
+    const int h = 31 - __clz(Lm);
+    float v = 0.f;
+    if (lane == h) v = a.lx[p0 + 31 - __clz(gbyte)];
+    out.xl = __shfl_sync(0xffffffffu, v, h);
+  }
+  if (Rm) {
+    const int h = 31 - __clz(Rm);
+    float v = 0.f;
+    if (lane == h) v = a.lx[p0 + 31 - __clz(~gbyte & 0xffu)];
+    out.xr = __shfl_sync(0xffffffffu, v, h);
+  }
+  a.gm[cbase / 8 + lane] = (uint8_t)gbyte;
+  if (lane == 0) {
+    a.agg[ch] = out;
+    if (kTails && st + __ldg(&a.pseg[s].cnt) == cbase + kChunkW) a.tails[s] = out;
+  }
+}
+
 template <bool kSmemBits, bool kTails>
 __global__ void __launch_bounds__(kSmemBits ? 1024 : kThreads) level_agg_kernel(AggArgs a) {
   extern __shared__ uint4 smem_bits4[];
   const uint32_t* __restrict__ bits = kSmemBits ? reinterpret_cast<const uint32_t*>(smem_bits4) : a.gbits;
   const uint64_t T = a.ctl->T[a.par];
-  const bool full = a.ctl->nsrch > 0;  // children searched: every list; else feature 0 (statistics)
-  const uint64_t Tw = full ? T : a.ctl->T0[a.par];
-  const int64_t nch = (int64_t)((Tw + kChunkW - 1) / kChunkW);
   const bool y32 = a.ctl->y32 != 0;
+  const int64_t nfast = a.ctl->nfast, ngen = a.ctl->ngen;
   if (kSmemBits) {
     const int64_t n4 = a.nwords / 4;
     const uint4* g4 = reinterpret_cast<const uint4*>(a.gbits);
@@ -150,61 +295,46 @@ __global__ void __launch_bounds__(kSmemBits ? 1024 : kThreads) level_agg_kernel(
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t ch = gw; ch < nch; ch += nw) {
+  // ---- fast chunks: the next chunk's rows and y are in flight during this chunk
+  if (y32) {
+    uint2 e = gw < nfast ? a.fast_list[gw] : make_uint2(0u, 0u);
+    uint4 r0 = make_uint4(0, 0, 0, 0), r1 = r0;
+    int4 q0 = make_int4(0, 0, 0, 0), q1 = q0;
+    auto fetch = [&](const uint2& en) {
+      const int64_t p0 = (int64_t)en.x * kChunkW + lane * kItems;
+      const uint4* r4 = reinterpret_cast<const uint4*>(a.lr + p0);
+      const int4* y4 = reinterpret_cast<const int4*>(reinterpret_cast<const int32_t*>(a.ly) + p0);
+      r0 = __ldcs(r4); r1 = __ldcs(r4 + 1);
+      q0 = __ldcs(y4); q1 = __ldcs(y4 + 1);
+    };
+    if (gw < nfast) fetch(e);
+    for (int64_t i = gw; i < nfast; i += nw) {
+      const uint2 cur = e;
+      const uint32_t rv[kItems] = {r0.x, r0.y, r0.z, r0.w, r1.x, r1.y, r1.z, r1.w};
+      const double yv[kItems] = {(double)q0.x, (double)q0.y, (double)q0.z, (double)q0.w,
+                                 (double)q1.x, (double)q1.y, (double)q1.z, (double)q1.w};
+      if (i + nw < nfast) {
+        e = a.fast_list[i + nw];
+        fetch(e);
+      }
+      agg_fast_chunk<kSmemBits, kTails>(a, bits, (int64_t)cur.x, cur.y, rv, yv);
+    }
+  } else {
+    for (int64_t i = gw; i < nfast; i += nw) {
+      const uint2 cur = a.fast_list[i];
+      uint32_t rv[kItems];
+      double yv[kItems];
+      load_rows_y(a, (int64_t)cur.x * kChunkW + lane * kItems, (int64_t)T, false, true, rv, yv);
+      agg_fast_chunk<kSmemBits, kTails>(a, bits, (int64_t)cur.x, cur.y, rv, yv);
+    }
+  }
+  // ---- general chunks: segment heads inside; per item walk
+  for (int64_t gi = gw; gi < ngen; gi += nw) {
+    const int64_t ch = (int64_t)a.gen_list[gi];
     const uint64_t cbase = (uint64_t)ch * kChunkW;
     const int64_t p0 = (int64_t)cbase + lane * kItems;
-    uint32_t s = __ldg(a.desc + ch);
-    SegLite sg = seg_lite(a.pseg, s);
-    const bool fast = sg.start <= cbase && sg.end >= cbase + kChunkW;  // warp-uniform
-    if (fast) {
-      AggP out = agg_ident();
-      out.flag = sg.start == cbase ? 1u : 0u;
-      uint32_t gbyte = 0u;
-      if (sg.flags & PS_SPLIT) {
-        const bool all_left = (sg.flags & PS_ALLLEFT) != 0;
-        uint32_t rv[kItems];
-        double yv[kItems];
-        load_rows_y(a, p0, (int64_t)T, y32, !all_left, rv, yv);
-        double sl = 0.0, sr = 0.0;
-#pragma unroll
-        for (int j = 0; j < kItems; ++j) {
-          const uint32_t g = all_left ? 1u : ((bits[rv[j] >> 5] >> (rv[j] & 31)) & 1u);
-          gbyte |= g << j;
-          if (g) sl = __dadd_rn(sl, __dsub_rn(yv[j], sg.c0));
-          else sr = __dadd_rn(sr, __dsub_rn(yv[j], sg.c1));
-        }
-        warp_incl2(sl, sr);
-        const uint32_t Lm = __ballot_sync(0xffffffffu, gbyte != 0u);
-        const uint32_t Rm = __ballot_sync(0xffffffffu, gbyte != 0xffu);
-        float xl = kNaN, xr = kNaN;
-        if (Lm) {
-          const int h = 31 - __clz(Lm);
-          float v = 0.f;
-          if (lane == h) v = a.lx[p0 + 31 - __clz(gbyte)];
-          xl = __shfl_sync(0xffffffffu, v, h);
-        }
-        if (Rm) {
-          const int h = 31 - __clz(Rm);
-          float v = 0.f;
-          if (lane == h) v = a.lx[p0 + 31 - __clz(~gbyte & 0xffu)];
-          xr = __shfl_sync(0xffffffffu, v, h);
-        }
-        uint32_t nl = __popc(gbyte);
-        nl = __reduce_add_sync(0xffffffffu, nl);
-        out.nl = nl;
-        out.sl = __shfl_sync(0xffffffffu, sl, 31);
-        out.sr = __shfl_sync(0xffffffffu, sr, 31);
-        out.xl = xl;
-        out.xr = xr;
-      }
-      a.gm[cbase / 8 + lane] = (uint8_t)gbyte;
-      if (lane == 0) {
-        a.agg[ch] = out;
-        if (kTails && (sg.flags & PS_SPLIT) && sg.end == cbase + kChunkW) a.tails[s] = out;
-      }
-      continue;
-    }
-    // ---- general chunk: segment heads inside; per item walk
+    const uint32_t s = __ldg(a.desc + ch);
+    const SegLite sg = seg_lite(a.pseg, s);
     uint32_t rv[kItems];
     double yv[kItems];
     load_rows_y(a, p0, (int64_t)T, y32, true, rv, yv);
@@ -247,7 +377,7 @@ __global__ void __launch_bounds__(kSmemBits ? 1024 : kThreads) level_agg_kernel(
     if (lane == 0) a.agg[ch] = wagg;
     if (kTails) {
       // per split segment ending in this lane: its aggregate from max(segment start,
-      // chunk start) to its last entry (segcount adds the chunk carry)
+      // chunk start) to its last entry (the boundary pass adds the chunk carry)
       uint32_t sc = s;
       SegLite g2 = sg;
       AggP r = ex;  // the open segment's part before this lane
@@ -396,7 +526,8 @@ struct FusedArgs {
   unsigned long long* slot_gain;
   Stat* head_stat;
   Stat* cont_stat;
-  uint32_t* gen_list;  // chunks with segment heads inside (fused_general_kernel)
+  const uint2* unit_list;    // {chunk, segment}: a split segment's piece of a chunk
+  const uint32_t* big_list;  // chunks with more than kMaxPieces pieces (fused_general_kernel)
   Ctl* ctl;
   int par;
   uint32_t level;   // level of the children (written into the pieces)
@@ -418,14 +549,6 @@ __host__ __device__ constexpr uint32_t stage_bytes_for(uint32_t yb) { return 204
 struct Meta {
   int64_t ch;
   uint32_t skip, pad;
-};
-
-// Compacted valid positions of one chunk (per warp).
-struct Compact {
-  double S[kChunkW];
-  uint32_t js[kChunkW];  // global child position | side << 31
-  float xp[kChunkW];
-  float xv[kChunkW];
 };
 
 struct ArgQ {  // segmented argmax: ties keep the earlier position
@@ -538,9 +661,129 @@ __device__ __forceinline__ void store_entry(const FusedArgs& a, bool y32, uint64
   if ((dst & (kChunkW - 1)) == 0) a.desc_next[dst / kChunkW] = cs;
 }
 
+// Row-wise stores of one fast chunk (lane = column of a row of 32 entries): left entries
+// to the left child's run, right entries to the right child's, both in order.  Returns
+// the left count through the chunk (segment-local).
+template <bool kY32>
+__device__ __forceinline__ uint32_t store_rows(const FusedArgs& a, const PSeg& ps, const uint32_t* w, uint32_t pre,
+                                               uint32_t ib, int e_lo, int e_hi, const float* sx, const uint32_t* sr,
+                                               const unsigned char* sy, bool w0, bool w1) {
+  using YT = typename std::conditional<kY32, uint32_t, unsigned long long>::type;
+  const int lane = threadIdx.x & 31;
+  const uint32_t lt = (1u << lane) - 1u;
+  float* const x0 = a.ox + ps.ostart[0];
+  float* const x1 = a.ox + ps.ostart[1];
+  uint32_t* const r0 = a.orow + ps.ostart[0];
+  uint32_t* const r1 = a.orow + ps.ostart[1];
+  YT* const y0 = reinterpret_cast<YT*>(a.oy) + ps.ostart[0];
+  YT* const y1 = reinterpret_cast<YT*>(a.oy) + ps.ostart[1];
+  const YT* const ys = reinterpret_cast<const YT*>(sy);
+#pragma unroll
+  for (int r = 0; r < kItems; ++r) {
+    const int e = 32 * r + lane;
+    const bool in = e >= e_lo && e < e_hi;
+    const uint32_t wr = w[r] & __ballot_sync(0xffffffffu, in);  // left entries of this segment
+    const bool g = (wr >> lane) & 1u;
+    const uint32_t rk = pre + __popc(wr & lt);
+    // segment-local index of entry e: ib + e (mod 2^32); right position = index - lefts before
+    const uint32_t off = g ? rk : ib + (uint32_t)e - rk;
+    if (in && (g ? w0 : w1)) {
+      (g ? x0 : x1)[off] = sx[e];
+      (g ? r0 : r1)[off] = sr[e];
+      (g ? y0 : y1)[off] = ys[e];
+    }
+    pre += __popc(wr);
+  }
+  return pre;
+}
+
+// rcp with two Newton steps: relative error ~3e-16 (a filter only; the winner's gain is
+// exact)
+__device__ __forceinline__ double rcp_nr(double x) {
+  double r;
+  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
+  double e = __fma_rn(-x, r, 1.0);
+  r = __fma_rn(r, e, r);
+  e = __fma_rn(-x, r, 1.0);
+  return __fma_rn(r, e, r);
+}
+
+// One child's candidate search over a lane's items: running prefix S (child-centred), the
+// child position, the neighbour x; best candidate by a Newton-reciprocal gain with a
+// near-tie flag (then the exact pass decides), exact gain of the winner.
+struct Side {
+  double S, sc, Nd, jd;         // prefix (rank carry included), S' of the child, N, position (f64)
+  uint32_t jl, lo, hi;          // local position, valid local range [lo, hi)
+  float xp;                     // x of the previous entry of this child
+  double bg, bs;                // best gain (approximate pass: approximate), its S'_L
+  uint32_t bj;                  // best global position
+  float bxp, bx;
+  __device__ __forceinline__ void init(const PSeg& ps, int side, uint32_t ilo, uint32_t m, bool srch, double S0,
+                                       float x0, uint32_t j0) {
+    S = __dadd_rn(ps.soff[side], S0);
+    sc = ps.sc[side];
+    Nd = (double)ps.N[side];
+    jl = j0;
+    jd = (double)(ps.ioff[side] + j0);
+    lo = ilo > ps.ioff[side] ? ilo - ps.ioff[side] : 0u;
+    hi = (srch && ps.N[side] >= m + ps.ioff[side]) ? ps.N[side] - m - ps.ioff[side] + 1u : 0u;
+    xp = x0;
+    bg = -1.0;
+    bs = 0.0;
+    bj = 0xffffffffu;
+    bxp = bx = 0.f;
+  }
+  // approximate pass; returns true on a near tie with the current best
+  __device__ __forceinline__ bool step(float x, double d) {
+    bool amb = false;
+    if (jl >= lo && jl < hi && xp < x) {
+      const double nr = __dsub_rn(Nd, jd);
+      const double D = __dsub_rn(__dmul_rn(S, nr), __dmul_rn(__dsub_rn(sc, S), jd));
+      const double ga = __dmul_rn(__dmul_rn(D, D), rcp_nr(__dmul_rn(__dmul_rn(Nd, jd), nr)));
+      constexpr double kTol = 1e-13;  // >> |approx - exact| / exact (~3e-16)
+      if (ga > bg) {
+        amb = bg >= __dmul_rn(ga, 1.0 - kTol);
+        bg = ga;
+        bs = S;
+        bj = (uint32_t)jd;
+        bxp = xp;
+        bx = x;
+      } else {
+        amb = ga >= __dmul_rn(bg, 1.0 - kTol);
+      }
+    }
+    S = __dadd_rn(S, d);
+    ++jl;
+    jd = __dadd_rn(jd, 1.0);
+    xp = x;
+    return amb;
+  }
+  __device__ __forceinline__ void step_exact(float x, double d) {
+    if (jl >= lo && jl < hi && xp < x) {
+      const double g = split_gain_d(S, sc, jd, Nd);
+      if (g > bg) {  // strict >: the lowest position wins exact ties
+        bg = g;
+        bs = S;
+        bj = (uint32_t)jd;
+        bxp = xp;
+        bx = x;
+      }
+    }
+    S = __dadd_rn(S, d);
+    ++jl;
+    jd = __dadd_rn(jd, 1.0);
+    xp = x;
+  }
+  __device__ __forceinline__ void finish() {  // the exact gain of the approximate winner
+    if (bg >= 0.0) bg = split_gain_d(bs, sc, (double)bj, Nd);
+  }
+};
+
 // y storage (int32 or f64, Reading R24) is decided on the device (root statistics): the
 // stage always has room for f64 entries; int32 lists copy and read half of it.
-__global__ void __launch_bounds__(kThreads, 2) fused_kernel(FusedArgs a) {
+// Work: the fast chunks listed by chunk_plan_kernel (whole chunk inside one segment of a
+// split node); a warp per chunk, two bulk-copy stages in flight per warp.
+__global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArgs a) {
   extern __shared__ __align__(128) unsigned char fsm[];
   constexpr uint32_t YB = 8u;
   constexpr uint32_t SB = (stage_bytes_for(YB) + 127u) & ~127u;
@@ -549,40 +792,26 @@ __global__ void __launch_bounds__(kThreads, 2) fused_kernel(FusedArgs a) {
   unsigned char* my = fsm + (size_t)wib * 2 * SB;
   uint64_t* bar = reinterpret_cast<uint64_t*>(fsm + (size_t)kWarps * 2 * SB) + wib * 2;
   PSeg* cur = reinterpret_cast<PSeg*>(fsm + (size_t)kWarps * 2 * SB + kWarps * 2 * sizeof(uint64_t)) + wib;
-  Compact& cbuf = reinterpret_cast<Compact*>(fsm + (size_t)kWarps * 2 * SB + kWarps * 2 * sizeof(uint64_t) +
-                                             kWarps * sizeof(PSeg))[wib];
-  const uint64_t T = a.ctl->T[a.par];
   const bool full = a.ctl->nsrch > 0;
-  const uint64_t Tw = full ? T : a.ctl->T0[a.par];
-  const int64_t nch = (int64_t)((Tw + kChunkW - 1) / kChunkW);
+  const int64_t nfast = a.ctl->nunit;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  if (blockIdx.x == 0 && threadIdx.x == 0) a.ctl->nch_last = (uint32_t)nch;  // for piece_pos
-  if (gw >= nch) return;  // warp-uniform; no block barriers below
+  if (blockIdx.x == 0 && threadIdx.x == 0) {  // for piece_pos: the chunks of this pass
+    const uint64_t Tw = full ? a.ctl->T[a.par] : a.ctl->T0[a.par];
+    a.ctl->nch_last = (uint32_t)((Tw + kChunkW - 1) / kChunkW);
+  }
+  if (gw >= nfast) return;  // warp-uniform; no block barriers below
   const uint32_t m = a.m;
   const uint32_t ilo = m > 1u ? m : 1u;
   const bool y32 = a.ctl->y32 != 0;
   const uint32_t yb = y32 ? 4u : 8u;
   const uint32_t lt = (1u << lane) - 1u;
 
-  auto issue = [&](int s, int64_t ch) {  // lane 0
+  auto issue = [&](int s, const uint2 en) {  // lane 0
     unsigned char* st = my + (size_t)s * SB;
-    Meta* mt = reinterpret_cast<Meta*>(st + off_meta(YB));
-    mt->ch = ch;
+    const int64_t ch = (int64_t)en.x;
+    reinterpret_cast<Meta*>(st + off_meta(YB))->ch = ch;
     const uint64_t cbase = (uint64_t)ch * kChunkW;
-    const uint32_t sid = __ldg(a.desc + ch);
-    const PSeg* P = a.pseg + sid;
-    const uint64_t s0 = __ldg(&P->start), e0 = s0 + __ldg(&P->cnt);
-    const bool single = s0 <= cbase && e0 >= cbase + kChunkW;
-    if (!single || !(__ldg(&P->flags) & PS_SPLIT)) {
-      // whole chunk in one segment of a node that does not split: nothing to do; a chunk
-      // with segment heads inside: listed for fused_general_kernel
-      if (!single) a.gen_list[atomicAdd(&a.ctl->ngen, 1u)] = (uint32_t)ch;
-      mt->skip = 1u;
-      mbar_arrive(bar + s);
-      return;
-    }
-    mt->skip = 0u;
     const uint32_t bytes = 2048u + 256u * yb + 32u + (uint32_t)sizeof(PSeg) + 64u;
     fence_proxy_async_smem();
     mbar_arrive_expect_tx(bar + s, bytes);
@@ -590,34 +819,30 @@ __global__ void __launch_bounds__(kThreads, 2) fused_kernel(FusedArgs a) {
     bulk_g2s(st + kOffR, a.lr + cbase, 1024u, bar + s);
     bulk_g2s(st + kOffY, reinterpret_cast<const unsigned char*>(a.ly) + cbase * yb, 256u * yb, bar + s);
     bulk_g2s(st + off_gm(YB), a.gm + cbase / 8, 32u, bar + s);
-    bulk_g2s(st + off_ps(YB), P, (uint32_t)sizeof(PSeg), bar + s);
+    bulk_g2s(st + off_ps(YB), a.pseg + en.y, (uint32_t)sizeof(PSeg), bar + s);
     bulk_g2s(st + off_ce(YB), a.cexcl + ch, 32u, bar + s);
     bulk_g2s(st + off_cb(YB), a.bcarry + ch / kBlockChunks, 32u, bar + s);
   };
+  uint2 ahead = make_uint2(0u, 0u);  // lane 0: the list entry two chunks ahead
   if (lane == 0) {
     mbar_init(bar, 1);
     mbar_init(bar + 1, 1);
     mbar_init_fence();
-    issue(0, gw);
-    if (gw + nw < nch) issue(1, gw + nw);
+    issue(0, a.unit_list[gw]);
+    if (gw + nw < nfast) issue(1, a.unit_list[gw + nw]);
+    if (gw + 2 * nw < nfast) ahead = a.unit_list[gw + 2 * nw];
   }
   __syncwarp();
   int s = 0;
   uint32_t phase = 0;
-  for (int64_t ch = gw; ch < nch; ch += nw) {
+  for (int64_t idx = gw; idx < nfast; idx += nw) {
     mbar_wait(bar + s, phase);
     unsigned char* st = my + (size_t)s * SB;
-    const int64_t nxt = ch + 2 * nw;
-    const bool skip = reinterpret_cast<const Meta*>(st + off_meta(YB))->skip != 0u;
-    if (skip) {
-      __syncwarp();
-      if (lane == 0 && nxt < nch) issue(s, nxt);
-      if (++s == 2) { s = 0; phase ^= 1u; }
-      continue;
-    }
+    const int64_t nxt = idx + 2 * nw;
+    const int64_t ch = reinterpret_cast<const Meta*>(st + off_meta(YB))->ch;
     const uint64_t cbase = (uint64_t)ch * kChunkW;
-    // the plan of the chunk's first segment: kept in this warp's slot (the stage is
-    // refilled before the candidates are evaluated)
+    // the plan of the chunk's segment: kept in this warp's slot (the stage is refilled
+    // before the candidates are evaluated)
     if (lane < (int)(sizeof(PSeg) / 16))
       reinterpret_cast<uint4*>(cur)[lane] = reinterpret_cast<const uint4*>(st + off_ps(YB))[lane];
     __syncwarp();
@@ -626,8 +851,13 @@ __global__ void __launch_bounds__(kThreads, 2) fused_kernel(FusedArgs a) {
     const uint32_t* sr = reinterpret_cast<const uint32_t*>(st + kOffR);
     const unsigned char* sy = st + kOffY;
     const uint8_t* sgm = st + off_gm(YB);
-    const uint32_t* sw = reinterpret_cast<const uint32_t*>(sgm);
-    const bool headc = ps.start == cbase;
+    const uint4 wq0 = reinterpret_cast<const uint4*>(sgm)[0], wq1 = reinterpret_cast<const uint4*>(sgm)[1];
+    const uint32_t w[kItems] = {wq0.x, wq0.y, wq0.z, wq0.w, wq1.x, wq1.y, wq1.z, wq1.w};
+    // this segment's entries of the chunk: [e_lo, e_hi) (the whole chunk unless segment
+    // heads lie inside; chunk_plan_kernel lists such a chunk once per segment piece)
+    const bool headc = ps.start >= cbase;  // the segment's head lies in this chunk
+    const int e_lo = headc ? (int)(ps.start - cbase) : 0;
+    const int e_hi = (int)min((uint64_t)kChunkW, ps.start + ps.cnt - cbase);
     AggP carry = agg_ident();
     if (full && !headc) carry = combine(*reinterpret_cast<const AggP*>(st + off_cb(YB)),
                                         *reinterpret_cast<const AggP*>(st + off_ce(YB)));
@@ -654,175 +884,144 @@ __global__ void __launch_bounds__(kThreads, 2) fused_kernel(FusedArgs a) {
         }
       }
     }
-    const uint32_t gbyte = sgm[lane];
+    // in-range mask of my items; left / right items of this segment
+    uint32_t mbyte;
     {
-      // =================== whole chunk inside one split segment =====================
-      const uint32_t flags = ps.flags;
-      const uint64_t ibase = cbase - ps.start;  // local index of the chunk's entry 0
-      // ---- partition: row-wise coalesced stores (row r = entries 32r .. 32r+31)
-      if (full && (flags & (PS_WR0 | PS_WR1))) {
-        uint32_t pre = carry.nl;
+      const int lo_i = min(max(e_lo - lane * kItems, 0), kItems);
+      const int hi_i = min(max(e_hi - lane * kItems, 0), kItems);
+      mbyte = ((1u << hi_i) - 1u) & ~((1u << lo_i) - 1u);
+    }
+    const uint32_t graw = (w[lane >> 2] >> (8 * (lane & 3))) & 0xffu;
+    const uint32_t lbyte = graw & mbyte, rbyte = ~graw & mbyte;
+    const uint32_t flags = ps.flags;
+    const uint32_t ib = (uint32_t)(cbase - ps.start);  // segment-local index of entry 0 (mod 2^32)
+    // ---- partition: row-wise coalesced stores (row r = entries 32r .. 32r+31); each
+    // child's entries of a row are consecutive
+    if (full && (flags & (PS_WR0 | PS_WR1))) {
+      const bool w0 = (flags & PS_WR0) != 0, w1 = (flags & PS_WR1) != 0;
+      const uint32_t pre = y32 ? store_rows<true>(a, ps, w, carry.nl, ib, e_lo, e_hi, sx, sr, sy, w0, w1)
+                               : store_rows<false>(a, ps, w, carry.nl, ib, e_lo, e_hi, sx, sr, sy, w0, w1);
+      // chunk descriptors of the next level: a child's run of this piece (<= 256 entries)
+      // crossing a multiple of kChunkW starts that chunk of the child's list
+      if (lane < 2) {
+        const bool g = lane == 0;
+        const uint32_t nL = pre - carry.nl, nR = (uint32_t)(e_hi - e_lo) - nL;
+        const uint64_t lo = g ? ps.ostart[0] + carry.nl : ps.ostart[1] + (uint64_t)(ib + (uint32_t)e_lo - carry.nl);
+        const uint64_t hi = lo + (g ? nL : nR);
+        const uint64_t b0 = (lo + kChunkW - 1) & ~(uint64_t)(kChunkW - 1);
+        if ((g ? w0 : w1) && b0 < hi) a.desc_next[b0 / kChunkW] = ps.cs[g ? 0 : 1];
+      }
+    }
+    // ---- left count before my items, neighbour x across lanes
+    uint32_t nl = carry.nl;
+    {
+      uint32_t cnt = __popc(lbyte);
 #pragma unroll
-        for (int r = 0; r < kItems; ++r) {
-          const uint32_t wr = sw[r];
-          const uint32_t g = (wr >> lane) & 1u;
-          const uint32_t rk = pre + __popc(wr & lt);
-          const int e = 32 * r + lane;
-          if (g ? (flags & PS_WR0) : (flags & PS_WR1)) {
-            const uint64_t dst = g ? ps.ostart[0] + rk : ps.ostart[1] + (ibase + (uint64_t)e - rk);
-            store_entry(a, y32, dst, sx[e], sr[e], sy + (size_t)e * yb, ps.cs[g ? 0 : 1]);
-          }
-          pre += __popc(wr);
-        }
+      for (int dd = 1; dd < 32; dd <<= 1) {
+        const uint32_t o = __shfl_up_sync(0xffffffffu, cnt, dd);
+        if (lane >= dd) cnt += o;
       }
-      // ---- left count before my items, neighbour x across lanes
-      uint32_t nl = carry.nl;
-      {
-        const int wq = lane >> 2;
+      nl += cnt - __popc(lbyte);
+    }
+    const uint32_t Lm = __ballot_sync(0xffffffffu, lbyte != 0u) & lt;
+    const uint32_t Rm = __ballot_sync(0xffffffffu, rbyte != 0u) & lt;
+    float xl = carry.xl, xr = carry.xr;
+    {
+      // x of the last left / right item of the nearest lower lane holding one
+      const int hl = Lm ? 31 - __clz(Lm) : 0, hr = Rm ? 31 - __clz(Rm) : 0;
+      const uint32_t bl = __shfl_sync(0xffffffffu, lbyte, hl), br = __shfl_sync(0xffffffffu, rbyte, hr);
+      if (Lm) xl = sx[8 * hl + 31 - __clz(bl)];
+      if (Rm) xr = sx[8 * hr + 31 - __clz(br)];
+    }
+    if (isnan(xl)) xl = ps.xprev[0];
+    if (isnan(xr)) xr = ps.xprev[1];
+    __syncwarp();  // the stage is read completely: refill it
+    if (lane == 0) {
+      if (nxt < nfast) issue(s, ahead);
+      if (nxt + nw < nfast) ahead = a.unit_list[nxt + nw];
+    }
+    // ---- children's prefix sums: lane sums, Kogge-Stone across lanes, chunk carry
+    const double c0 = ps.c[0], c1 = ps.c[1];
+    double dv[kItems];
+    double sl = 0.0, srr = 0.0;
 #pragma unroll
-        for (int r = 0; r < kItems; ++r)
-          if (r < wq) nl += __popc(sw[r]);
-        nl += __popc(sw[wq] & ((1u << (8 * (lane & 3))) - 1u));
-      }
-      const uint32_t Lm = __ballot_sync(0xffffffffu, gbyte != 0u) & lt;
-      const uint32_t Rm = __ballot_sync(0xffffffffu, gbyte != 0xffu) & lt;
-      float xl = carry.xl, xr = carry.xr;
-      if (Lm) {
-        const int h = 31 - __clz(Lm);
-        xl = sx[8 * h + 31 - __clz((uint32_t)sgm[h])];
-      }
-      if (Rm) {
-        const int h = 31 - __clz(Rm);
-        xr = sx[8 * h + 31 - __clz(~(uint32_t)sgm[h] & 0xffu)];
-      }
-      if (isnan(xl)) xl = ps.xprev[0];
-      if (isnan(xr)) xr = ps.xprev[1];
-      __syncwarp();  // the stage is read completely: refill it
-      if (lane == 0 && nxt < nch) issue(s, nxt);
-      // ---- children's prefix sums: lane sums, Kogge-Stone across lanes, chunk carry
-      const double c0 = ps.c[0], c1 = ps.c[1];
-      double sl = 0.0, srr = 0.0;
+    for (int j = 0; j < kItems; ++j) {
+      const bool g = (lbyte >> j) & 1u, r = (rbyte >> j) & 1u;
+      dv[j] = __dsub_rn(yv[j], g ? c0 : c1);
+      // adding +0.0 is exact: a sum of (y - c) terms is never -0.0
+      sl = __dadd_rn(sl, g ? dv[j] : 0.0);
+      srr = __dadd_rn(srr, r ? dv[j] : 0.0);
+    }
+    // ---- children's statistics from feature 0
+    if (ps.f == 0) {
+      StatQ q0 = statq_ident(), q1 = statq_ident();
 #pragma unroll
       for (int j = 0; j < kItems; ++j) {
-        if ((gbyte >> j) & 1u) sl = __dadd_rn(sl, __dsub_rn(yv[j], c0));
-        else srr = __dadd_rn(srr, __dsub_rn(yv[j], c1));
+        if ((lbyte >> j) & 1u) stat_add(q0, yv[j], ps.v[0], c0);
+        if ((rbyte >> j) & 1u) stat_add(q1, yv[j], ps.v[1], c1);
       }
-      double il = sl, ir = srr;
-      warp_incl2(il, ir);
-      double SL = __shfl_up_sync(0xffffffffu, il, 1), SR = __shfl_up_sync(0xffffffffu, ir, 1);
-      if (lane == 0) { SL = 0.0; SR = 0.0; }
-      SL = __dadd_rn(carry.sl, SL);
-      SR = __dadd_rn(carry.sr, SR);
-      // ---- valid positions of both children, compacted
-      if (full && (flags & (PS_SRCH0 | PS_SRCH1))) {
-        const uint32_t i0 = (uint32_t)(ibase + (uint64_t)(lane * kItems));
-        double tS[kItems];
-        uint32_t tJ[kItems];
-        float tP[kItems];
-        uint32_t vm = 0u;
-        uint32_t nlj = nl;
-        double SLj = SL, SRj = SR;
-        float xlj = xl, xrj = xr;
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) {
+        q0.sse = __dadd_rn(q0.sse, __shfl_xor_sync(0xffffffffu, q0.sse, off));
+        q0.ymin = fmin(q0.ymin, __shfl_xor_sync(0xffffffffu, q0.ymin, off));
+        q0.ymax = fmax(q0.ymax, __shfl_xor_sync(0xffffffffu, q0.ymax, off));
+        q0.s1 = __dadd_rn(q0.s1, __shfl_xor_sync(0xffffffffu, q0.s1, off));
+        q1.sse = __dadd_rn(q1.sse, __shfl_xor_sync(0xffffffffu, q1.sse, off));
+        q1.ymin = fmin(q1.ymin, __shfl_xor_sync(0xffffffffu, q1.ymin, off));
+        q1.ymax = fmax(q1.ymax, __shfl_xor_sync(0xffffffffu, q1.ymax, off));
+        q1.s1 = __dadd_rn(q1.s1, __shfl_xor_sync(0xffffffffu, q1.s1, off));
+      }
+      if (lane == 0) {
+        put_stat(a, headc, ch, 0, ps.kid, q0);
+        if (!(flags & PS_ALLLEFT)) put_stat(a, headc, ch, 1, ps.kid + 1, q1);
+      }
+    }
+    double il = sl, ir = srr;
+    warp_incl2(il, ir);
+    double SL = __shfl_up_sync(0xffffffffu, il, 1), SR = __shfl_up_sync(0xffffffffu, ir, 1);
+    if (lane == 0) { SL = 0.0; SR = 0.0; }
+    SL = __dadd_rn(carry.sl, SL);
+    SR = __dadd_rn(carry.sr, SR);
+    // ---- candidates of both children at every valid position of my items
+    if (full && (flags & (PS_SRCH0 | PS_SRCH1))) {
+      // right position of my first in-range item: its segment-local index - lefts before
+      const uint32_t jr0 = ib + (uint32_t)max(lane * kItems, e_lo) - nl;
+      Side sd[2];
+      sd[0].init(ps, 0, ilo, m, (flags & PS_SRCH0) != 0, SL, xl, nl);
+      sd[1].init(ps, 1, ilo, m, (flags & PS_SRCH1) != 0, SR, xr, jr0);
+      bool amb = false;
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        if ((lbyte >> j) & 1u) amb |= sd[0].step(xv[j], dv[j]);
+        if ((rbyte >> j) & 1u) amb |= sd[1].step(xv[j], dv[j]);
+      }
+      if (__any_sync(0xffffffffu, amb)) {
+        // a near tie of approximate gains in some lane: exact gains at every position
+        sd[0].init(ps, 0, ilo, m, (flags & PS_SRCH0) != 0, SL, xl, nl);
+        sd[1].init(ps, 1, ilo, m, (flags & PS_SRCH1) != 0, SR, xr, jr0);
 #pragma unroll
         for (int j = 0; j < kItems; ++j) {
-          const float x = xv[j];
-          if ((gbyte >> j) & 1u) {
-            const uint32_t jg = ps.ioff[0] + nlj;
-            if ((flags & PS_SRCH0) && jg >= ilo && ps.N[0] - jg >= m && xlj < x) {
-              vm |= 1u << j;
-              tS[j] = __dadd_rn(ps.soff[0], SLj);
-              tJ[j] = jg;
-              tP[j] = xlj;
-            }
-            SLj = __dadd_rn(SLj, __dsub_rn(yv[j], c0));
-            ++nlj;
-            xlj = x;
-          } else {
-            const uint32_t jg = ps.ioff[1] + (i0 + j - nlj);
-            if ((flags & PS_SRCH1) && jg >= ilo && ps.N[1] - jg >= m && xrj < x) {
-              vm |= 1u << j;
-              tS[j] = __dadd_rn(ps.soff[1], SRj);
-              tJ[j] = jg | 0x80000000u;
-              tP[j] = xrj;
-            }
-            SRj = __dadd_rn(SRj, __dsub_rn(yv[j], c1));
-            xrj = x;
-          }
+          if ((lbyte >> j) & 1u) sd[0].step_exact(xv[j], dv[j]);
+          if ((rbyte >> j) & 1u) sd[1].step_exact(xv[j], dv[j]);
         }
-        const uint32_t nv = __popc(vm);
-        uint32_t vinc = nv;
-#pragma unroll
-        for (int dd = 1; dd < 32; dd <<= 1) {
-          const uint32_t o = __shfl_up_sync(0xffffffffu, vinc, dd);
-          if (lane >= dd) vinc += o;
-        }
-        const uint32_t vtot = __shfl_sync(0xffffffffu, vinc, 31);
-        if (vtot) {
-          uint32_t q = vinc - nv;
-#pragma unroll
-          for (int j = 0; j < kItems; ++j) {
-            if ((vm >> j) & 1u) {
-              cbuf.S[q] = tS[j];
-              cbuf.js[q] = tJ[j];
-              cbuf.xp[q] = tP[j];
-              cbuf.xv[q] = xv[j];
-              ++q;
-            }
-          }
-          __syncwarp();
-          double bg[2] = {-1.0, -1.0};
-          uint32_t bj[2] = {0xffffffffu, 0xffffffffu}, be[2] = {0u, 0u};
-          const double N0 = (double)ps.N[0], N1 = (double)ps.N[1];
-          const double sc0 = ps.sc[0], sc1 = ps.sc[1];
-          for (uint32_t e = lane; e < vtot; e += 32) {
-            const uint32_t js = cbuf.js[e];
-            const int side = (int)(js >> 31);
-            const uint32_t jg = js & 0x7fffffffu;
-            const double g = split_gain_d(cbuf.S[e], side ? sc1 : sc0, (double)jg, side ? N1 : N0);
-            if (side == 0) {
-              if (g > bg[0]) { bg[0] = g; bj[0] = jg; be[0] = e; }
-            } else {
-              if (g > bg[1]) { bg[1] = g; bj[1] = jg; be[1] = e; }
-            }
-          }
-#pragma unroll
-          for (int side = 0; side < 2; ++side) {
-            double gmx = bg[side];
-#pragma unroll
-            for (int off = 16; off > 0; off >>= 1) gmx = fmax(gmx, __shfl_xor_sync(0xffffffffu, gmx, off));
-            if (gmx >= 0.0) {
-              const uint32_t jmin = __reduce_min_sync(0xffffffffu, bg[side] == gmx ? bj[side] : 0xffffffffu);
-              const int src = __ffs(__ballot_sync(0xffffffffu, bg[side] == gmx && bj[side] == jmin)) - 1;
-              const uint32_t e = __shfl_sync(0xffffffffu, be[side], src);
-              if (lane == 0)
-                put_cand(a, headc, ch, side, ps.cs[side], gmx, cbuf.S[e], mid_threshold(cbuf.xp[e], cbuf.xv[e]), jmin);
-            }
-          }
-          __syncwarp();  // the buffer is rewritten by the next chunk
-        }
+      } else {
+        sd[0].finish();
+        sd[1].finish();
       }
-      // ---- children's statistics from feature 0
-      if (ps.f == 0) {
-        StatQ q0 = statq_ident(), q1 = statq_ident();
 #pragma unroll
-        for (int j = 0; j < kItems; ++j) {
-          if ((gbyte >> j) & 1u) stat_add(q0, yv[j], ps.v[0], c0);
-          else stat_add(q1, yv[j], ps.v[1], c1);
-        }
-#pragma unroll
-        for (int off = 16; off > 0; off >>= 1) {
-          q0.sse = __dadd_rn(q0.sse, __shfl_xor_sync(0xffffffffu, q0.sse, off));
-          q0.ymin = fmin(q0.ymin, __shfl_xor_sync(0xffffffffu, q0.ymin, off));
-          q0.ymax = fmax(q0.ymax, __shfl_xor_sync(0xffffffffu, q0.ymax, off));
-          q0.s1 = __dadd_rn(q0.s1, __shfl_xor_sync(0xffffffffu, q0.s1, off));
-          q1.sse = __dadd_rn(q1.sse, __shfl_xor_sync(0xffffffffu, q1.sse, off));
-          q1.ymin = fmin(q1.ymin, __shfl_xor_sync(0xffffffffu, q1.ymin, off));
-          q1.ymax = fmax(q1.ymax, __shfl_xor_sync(0xffffffffu, q1.ymax, off));
-          q1.s1 = __dadd_rn(q1.s1, __shfl_xor_sync(0xffffffffu, q1.s1, off));
-        }
-        if (lane == 0) {
-          put_stat(a, headc, ch, 0, ps.kid, q0);
-          if (!(flags & PS_ALLLEFT)) put_stat(a, headc, ch, 1, ps.kid + 1, q1);
+      for (int side = 0; side < 2; ++side) {
+        const double bg = sd[side].bg;
+        const uint32_t bj = sd[side].bj;
+        // warp max of the exact gains (>= 0: the f64 bit patterns order like the values;
+        // key 0 = no candidate), then the lowest position holding it
+        const unsigned long long key = bg >= 0.0 ? (unsigned long long)__double_as_longlong(bg) + 1ull : 0ull;
+        const uint32_t khi = __reduce_max_sync(0xffffffffu, (uint32_t)(key >> 32));
+        const uint32_t klo = __reduce_max_sync(0xffffffffu, (uint32_t)(key >> 32) == khi ? (uint32_t)key : 0u);
+        const unsigned long long kmax = ((unsigned long long)khi << 32) | klo;
+        if (kmax != 0ull) {
+          const uint32_t jmin = __reduce_min_sync(0xffffffffu, key == kmax ? bj : 0xffffffffu);
+          if (key == kmax && bj == jmin)  // exactly one lane holds the winner
+            put_cand(a, headc, ch, side, ps.cs[side], bg, sd[side].bs, mid_threshold(sd[side].bxp, sd[side].bx), jmin);
         }
       }
     }
@@ -836,7 +1035,7 @@ __global__ void __launch_bounds__(kThreads, 2) fused_kernel(FusedArgs a) {
 // runs for the candidate / statistics pieces of every segment in the chunk.
 __global__ void __launch_bounds__(kThreads) fused_general_kernel(FusedArgs a) {
   const int lane = threadIdx.x & 31;
-  const int64_t ngen = a.ctl->ngen;
+  const int64_t ngen = a.ctl->nbig;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const uint64_t T = a.ctl->T[a.par];
@@ -846,7 +1045,7 @@ __global__ void __launch_bounds__(kThreads) fused_general_kernel(FusedArgs a) {
   const uint32_t m = a.m;
   const uint32_t ilo = m > 1u ? m : 1u;
   for (int64_t idx = gw; idx < ngen; idx += nw) {
-    const int64_t ch = (int64_t)a.gen_list[idx];
+    const int64_t ch = (int64_t)a.big_list[idx];
     const uint64_t cbase = (uint64_t)ch * kChunkW;
     const float* sx = a.lx + cbase;
     const uint32_t* sr = a.lr + cbase;
@@ -1108,9 +1307,14 @@ dt_status level_agg_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t 
   a.gm = b.gm;
   a.agg = b.agg;
   a.tails = b.tails;
+  a.fast_list = b.fast_list;
+  a.gen_list = b.gen_list;
   a.ctl = b.ctl;
   a.par = la.par;
   a.nwords = b.nwords4;
+  chunk_plan_kernel<<<num_sms() * 8, 256, 0, s>>>(b.ctl, la.par, la.d, b.desc[la.par], b.pseg, b.agg, b.fast_list,
+                                                  b.gen_list, b.unit_list, b.big_list);
+  DT_CK(cudaGetLastError());
   const size_t bytes = sizeof(uint32_t) * (size_t)b.nwords4;
   if ((int64_t)bytes <= kMaxSmemBits) {
     auto k = la.tails ? level_agg_kernel<true, true> : level_agg_kernel<true, false>;
@@ -1129,7 +1333,7 @@ dt_status level_agg_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t 
 size_t fused_smem() {
   const size_t sb = (stage_bytes_for(8u) + 127u) & ~127u;
   constexpr int kWarps = kThreads / 32;
-  return sb * 2 * kWarps + kWarps * 2 * sizeof(uint64_t) + kWarps * sizeof(PSeg) + kWarps * sizeof(Compact);
+  return sb * 2 * kWarps + kWarps * 2 * sizeof(uint64_t) + kWarps * sizeof(PSeg);
 }
 
 // F_C of the pass whose parent level is la.level.
@@ -1159,7 +1363,8 @@ dt_status level_fused_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_
   a.ystride = 0;
   a.stage_bytes = 0;
   const size_t sm = fused_smem();
-  a.gen_list = b.gen_list;
+  a.unit_list = b.unit_list;
+  a.big_list = b.big_list;
   auto k = fused_kernel;
   DT_CK(cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
   k<<<grid_for((const void*)k, kThreads, sm), kThreads, sm, s>>>(a);
