@@ -455,8 +455,9 @@ __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
 // ----------------------------------------------------------------------------- goleft --
 
 // Bit per row: 1 if the row goes to its node's left child -- the first nl entries of the
-// node's split-feature list (a6).  One warp per chunk of the level's lists; chunks of other
-// features are skipped after one descriptor read.
+// node's split-feature list (a6).  Each thread tests one chunk of the level's lists (does
+// it hold left entries of a split feature?); the warp then sets the bits of the
+// qualifying chunks together.
 __global__ void __launch_bounds__(256) goleft_kernel(const Ctl* __restrict__ ctl, int par, const uint32_t* __restrict__ desc,
                                                      const SegT* __restrict__ segs, const Decision* __restrict__ dec,
                                                      const uint32_t* __restrict__ lr, uint32_t* __restrict__ gbits) {
@@ -464,48 +465,68 @@ __global__ void __launch_bounds__(256) goleft_kernel(const Ctl* __restrict__ ctl
   if (ctl->K[par ^ 1] == 0) return;  // nothing splits
   const int64_t nch = (int64_t)((T + kChunkW - 1) / kChunkW);
   const int lane = threadIdx.x & 31;
+  // warp gw tests chunks gw + (32 it + lane) nw: qualifying chunks (contiguous runs of a
+  // split feature's list) spread over all warps
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t ch = gw; ch < nch; ch += nw) {
-    const uint64_t cbase = (uint64_t)ch * kChunkW;
-    uint32_t s = __ldg(desc + ch);
-    uint64_t st = __ldg(&segs[s].start), en = st + __ldg(&segs[s].cnt);
-    if (st <= cbase && en >= cbase + kChunkW) {  // one segment: warp-uniform skip test
-      const uint32_t k = __ldg(&segs[s].k);
-      const int f = __ldg(&segs[s].f);
-      if (__ldg(&dec[k].f) != f) continue;
-      const uint32_t ioff = __ldg(&segs[s].ioff), nl = __ldg(&dec[k].nl);
-      // local positions i < nl - ioff go left
-      const uint64_t lim = (nl > ioff) ? st + (nl - ioff) : st;
+  for (int64_t it = 0; gw + it * 32 * nw < nch; ++it) {
+    const int64_t mych = gw + (it * 32 + lane) * nw;
+    bool q = false;
+    if (mych < nch) {
+      const uint64_t cbase = (uint64_t)mych * kChunkW;
+      const uint32_t s = __ldg(desc + mych);
+      const uint64_t st = __ldg(&segs[s].start), en = st + __ldg(&segs[s].cnt);
+      if (st <= cbase && en >= cbase + kChunkW) {
+        const uint32_t k = __ldg(&segs[s].k);
+        const uint32_t ioff = __ldg(&segs[s].ioff);
+        q = __ldg(&dec[k].f) == __ldg(&segs[s].f) && cbase < st + (uint64_t)(__ldg(&dec[k].nl) - min(ioff, __ldg(&dec[k].nl)));
+      } else {
+        q = true;  // segment heads inside: walk it
+      }
+    }
+    uint32_t qm = __ballot_sync(0xffffffffu, q);
+    while (qm) {
+      const int c = __ffs(qm) - 1;
+      qm &= qm - 1u;
+      const int64_t ch = gw + (it * 32 + c) * nw;
+      const uint64_t cbase = (uint64_t)ch * kChunkW;
+      uint32_t s = __ldg(desc + ch);
+      uint64_t st = __ldg(&segs[s].start), en = st + __ldg(&segs[s].cnt);
+      uint32_t k = __ldg(&segs[s].k);
+      int f = __ldg(&segs[s].f);
+      uint32_t ioff = __ldg(&segs[s].ioff);
+      if (st <= cbase && en >= cbase + kChunkW) {
+        // one segment: its local positions i < nl - ioff go left (rows read coalesced)
+        const uint32_t nl = __ldg(&dec[k].nl);
+        const uint64_t lim = (nl > ioff) ? st + (nl - ioff) : st;
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+          const uint64_t p = cbase + (uint64_t)(j * 32 + lane);
+          if (p < lim) {
+            const uint32_t r = __ldg(lr + p);
+            atomicOr(gbits + (r >> 5), 1u << (r & 31));
+          }
+        }
+        continue;
+      }
+      // segment heads inside: lane owns entries 8 lane .. 8 lane + 7, walks their segments
+      const uint64_t p0 = cbase + (uint64_t)(lane * kItems);
+#pragma unroll
       for (int j = 0; j < kItems; ++j) {
-        const uint64_t p = cbase + (uint64_t)(j * 32 + lane);
-        if (p < lim) {
+        const uint64_t p = p0 + j;
+        if (p >= T) break;
+        while (p >= en) {
+          ++s;
+          st = __ldg(&segs[s].start);
+          en = st + __ldg(&segs[s].cnt);
+          k = __ldg(&segs[s].k);
+          f = __ldg(&segs[s].f);
+          ioff = __ldg(&segs[s].ioff);
+        }
+        if (__ldg(&dec[k].f) == f && ioff + (uint32_t)(p - st) < __ldg(&dec[k].nl)) {
           const uint32_t r = __ldg(lr + p);
           atomicOr(gbits + (r >> 5), 1u << (r & 31));
         }
-      }
-      continue;
-    }
-    // general chunk: walk the segments item by item (lane owns entries 8 lane .. 8 lane + 7)
-    const uint64_t p0 = cbase + (uint64_t)(lane * kItems);
-    uint32_t k = __ldg(&segs[s].k);
-    int f = __ldg(&segs[s].f);
-    uint32_t ioff = __ldg(&segs[s].ioff);
-#pragma unroll
-    for (int j = 0; j < kItems; ++j) {
-      const uint64_t p = p0 + j;
-      if (p >= T) break;
-      while (p >= en) {
-        ++s;
-        st = __ldg(&segs[s].start);
-        en = st + __ldg(&segs[s].cnt);
-        k = __ldg(&segs[s].k);
-        f = __ldg(&segs[s].f);
-        ioff = __ldg(&segs[s].ioff);
-      }
-      if (__ldg(&dec[k].f) == f && ioff + (uint32_t)(p - st) < __ldg(&dec[k].nl)) {
-        const uint32_t r = __ldg(lr + p);
-        atomicOr(gbits + (r >> 5), 1u << (r & 31));
       }
     }
   }
