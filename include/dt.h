@@ -245,18 +245,30 @@ dt_status dt_gen_dse(uint64_t seed, int64_t row0, int64_t n, int32_t gpu_bits,
 
 /* ------------------------------------------------------------------ multi-GPU ----- */
 
-/* One process (or host thread) per GPU.  Feature-sharded exact fit (DESIGN.md,
- * "Multi-GPU"): rank r of `world` builds and scans the feature lists of the
- * global features j*world + r only; per level the ranks allgather their per-node best
- * splits (reduced in the fixed order of dt_fit: highest gain, then lowest feature, then
- * lowest threshold) and max-allreduce the go-left byte map.  Every rank passes the FULL
- * table (X n x d, y) and receives the same tree, identical to dt_fit's (tests/).
+/* One process (or host thread) per GPU.  Value-range ROW-sharded exact fit (
+ * BASELINE north_star "rows shard naturally across the GPUs ... allreduce / allgather of
+ * the per-node, per-feature candidate statistics").  Rank p of P
+ * passes only ITS rows: X_local_dev (n_local x d f32 row-major) and y_local_dev (n_local
+ * f64) are rows row_offset .. row_offset + n_local - 1 of the n_global-row table, ranks
+ * in row order (row_offset of rank p = sum of n_local of ranks < p; n_local may be 0).
+ *  - presort: a local sort, exact splitters by bisection on the key (flip(x) << 32 | row)
+ *    with a sum-allreduce per round, an all-to-all of 16-byte entries (x, row, y): rank p
+ *    then holds global sorted positions [p n / P, (p + 1) n / P) of every feature list;
+ *  - per level: allgather of the per-node local bests (reduced in rank order: highest
+ *    gain, then lowest feature, then lowest position), OR-allreduce of the n_global-bit
+ *    go-left map, allgather of the children's boundary records (count, last x, S') ->
+ *    the carries of every child segment.  Entries never move between ranks after the
+ *    presort.
+ * Every rank returns the same tree: identical to dt_fit's in integer mode except the
+ * impurity (summed in another order; within 1e-12 relative), within the parity contract
+ * otherwise.  Sync (one host synchronisation per level).
  *   dt_comm_unique_id: 128-byte NCCL id, created by rank 0 and broadcast by the caller
  *     (e.g. torch.distributed); dt_comm_init: NCCL communicator on the current device
- *     (libnccl.so.2 is loaded at run time; DT_ERR_NCCL if absent).
+ *     (libnccl.so.2 is loaded at run time; DT_ERR_NCCL if absent); a 1-rank communicator
+ *     runs the real NCCL collectives.
  *   dt_comm_init_local: `world` communicators for host THREADS of one process (device
  *     copies behind a host barrier), e.g. to run the sharded path on a single GPU.
- * dt_fit_sharded: world <= d; otherwise as dt_fit (sync). */
+ * Errors: as dt_fit; INVALID_ARG also for row_offset + n_local > n_global; NCCL. */
 typedef struct dt_comm dt_comm;
 int32_t dt_comm_unique_id_bytes(void);
 dt_status dt_comm_unique_id(void* id_out);
@@ -265,9 +277,9 @@ dt_status dt_comm_init_local(int32_t world, dt_comm** comms_out);
 void dt_comm_free(dt_comm* comm);
 int32_t dt_comm_rank(const dt_comm* comm);
 int32_t dt_comm_world(const dt_comm* comm);
-dt_status dt_fit_sharded(dt_comm* comm, const float* X_dev, const double* y_dev, int64_t n,
-                         int32_t d, int32_t max_depth, int64_t min_samples_leaf, void* stream,
-                         dt_tree** out);
+dt_status dt_fit_sharded(dt_comm* comm, const float* X_local_dev, const double* y_local_dev, int64_t n_local,
+                         int64_t row_offset, int64_t n_global, int32_t d, int32_t max_depth,
+                         int64_t min_samples_leaf, void* stream, dt_tree** out);
 
 /* dt_eval_sharded -- MAPE / R^2 / adj-R^2 of rows split over the ranks (SURVEY 8e
  * "Eval"; Table II): each rank reduces its n_local rows (y_dev, yhat_dev f64,

@@ -87,7 +87,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "dt_comm_free": ([P], None),
         "dt_comm_rank": ([P], I32),
         "dt_comm_world": ([P], I32),
-        "dt_fit_sharded": ([P, P, P, I64, I32, I32, I64, P, ctypes.POINTER(P)], ctypes.c_int),
+        "dt_fit_sharded": ([P, P, P, I64, I64, I64, I32, I32, I64, P, ctypes.POINTER(P)], ctypes.c_int),
         "dt_tree_truncate": ([P, I32, ctypes.POINTER(P)], ctypes.c_int),
         "dt_predict_eval_depths": ([P, P, P, I64, I32, I32, P, P], ctypes.c_int),
         "dt_importances": ([P, P, P], ctypes.c_int),
@@ -380,7 +380,7 @@ def grid_search(X, y, Xv, yv, depths, min_leafs, p=None, stream=None, rank=0, wo
 
 
 class Comm:
-    """Owns a ``dt_comm*`` (one rank of a feature-sharded fit)."""
+    """Owns a ``dt_comm*`` (one rank of a row-sharded fit)."""
 
     def __init__(self, handle: ctypes.c_void_p):
         self._h = handle
@@ -425,14 +425,17 @@ def dt_comm_init_local(world: int):
     return [Comm(ctypes.c_void_p(arr[i])) for i in range(world)]
 
 
-def dt_fit_sharded(comm: Comm, X, y, max_depth: int = -1, min_samples_leaf: int = 1,
-                   stream=None) -> Tree:
+def dt_fit_sharded(comm: Comm, X_local, y_local, row_offset: int, n_global: int, max_depth: int = -1,
+                   min_samples_leaf: int = 1, stream=None) -> Tree:
+    """Value-range row-sharded fit (include/dt.h): this rank's rows row_offset ..
+    row_offset + n_local - 1 of the n_global-row table; every rank returns the same tree."""
     import torch
-    xp = _dev(X, torch.float32, 2, "X")
-    yp = _dev(y, torch.float64, 1, "y")
-    n, d = X.shape
+    n, d = X_local.shape
+    _same((X_local, y_local), ("y_local", y_local.shape[0], n))
+    xp = _dev(X_local, torch.float32, 2, "X_local") if n else ctypes.c_void_p(0)
+    yp = _dev(y_local, torch.float64, 1, "y_local") if n else ctypes.c_void_p(0)
     h = ctypes.c_void_p()
-    _check(_lib.dt_fit_sharded(comm.handle, xp, yp, n, d, max_depth, min_samples_leaf,
+    _check(_lib.dt_fit_sharded(comm.handle, xp, yp, n, row_offset, n_global, d, max_depth, min_samples_leaf,
                                _stream(stream), ctypes.byref(h)))
     return Tree(h)
 

@@ -106,18 +106,22 @@ dt_status dt_fit(const float* X_dev, const double* y_dev, int64_t n, int32_t d,
   return fit_impl(X_dev, y_dev, n, d, max_depth, min_samples_leaf, S(stream), out);
 }
 
-dt_status dt_fit_sharded(dt_comm* comm, const float* X_dev, const double* y_dev, int64_t n, int32_t d,
-                         int32_t max_depth, int64_t min_samples_leaf, void* stream, dt_tree** out) {
+dt_status dt_fit_sharded(dt_comm* comm, const float* X_local_dev, const double* y_local_dev, int64_t n_local,
+                         int64_t row_offset, int64_t n_global, int32_t d, int32_t max_depth, int64_t min_samples_leaf,
+                         void* stream, dt_tree** out) {
   if (!out) return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: out is NULL");
   *out = nullptr;
   if (!comm) return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: comm is NULL");
-  if (!X_dev || !y_dev) return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: NULL X or y");
-  if (n < 1) return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: n must be >= 1");
-  if (n >= (int64_t)1 << 32) return fail(DT_ERR_TOO_LARGE, "dt_fit_sharded: n must be < 2^32");
+  if (n_local < 0 || row_offset < 0) return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: n_local, row_offset must be >= 0");
+  if (n_local > 0 && (!X_local_dev || !y_local_dev)) return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: NULL X or y");
+  if (n_global < 1) return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: n_global must be >= 1");
+  if (n_global >= (int64_t)1 << 32) return fail(DT_ERR_TOO_LARGE, "dt_fit_sharded: n_global must be < 2^32");
+  if (row_offset + n_local > n_global) return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: row_offset + n_local > n_global");
   if (d < 1 || d > 255) return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: d must be in [1, 255]");
   if (max_depth < -1) return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: max_depth must be >= -1");
   if (min_samples_leaf < 1) return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: min_samples_leaf must be >= 1");
-  return fit_sharded_impl(comm, X_dev, y_dev, n, d, max_depth, min_samples_leaf, S(stream), out);
+  return fit_sharded_impl(comm, X_local_dev, y_local_dev, n_local, row_offset, n_global, d, max_depth,
+                          min_samples_leaf, S(stream), out);
 }
 
 int64_t dt_tree_size(const dt_tree* t) { return t ? t->count : 0; }

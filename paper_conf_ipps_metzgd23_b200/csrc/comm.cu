@@ -31,6 +31,10 @@ struct NcclApi {
   ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
   ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
                             cudaStream_t) = nullptr;
+  ncclResult_t (*Send)(const void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*GroupStart)() = nullptr;
+  ncclResult_t (*GroupEnd)() = nullptr;
   const char* (*GetErrorString)(ncclResult_t) = nullptr;
   bool ok = false;
 };
@@ -53,9 +57,14 @@ bool load_nccl() {
   LOAD(AllGather, "ncclAllGather");
   LOAD(AllReduce, "ncclAllReduce");
   LOAD(GetErrorString, "ncclGetErrorString");
+  LOAD(Send, "ncclSend");
+  LOAD(Recv, "ncclRecv");
+  LOAD(GroupStart, "ncclGroupStart");
+  LOAD(GroupEnd, "ncclGroupEnd");
 #undef LOAD
   g_nccl.ok = g_nccl.GetUniqueId && g_nccl.CommInitRank && g_nccl.CommDestroy && g_nccl.AllGather &&
-              g_nccl.AllReduce && g_nccl.GetErrorString;
+              g_nccl.AllReduce && g_nccl.GetErrorString && g_nccl.Send && g_nccl.Recv && g_nccl.GroupStart &&
+              g_nccl.GroupEnd;
   return g_nccl.ok;
 }
 
@@ -73,7 +82,8 @@ struct LocalGroup {
   long long gen = 0;
   std::vector<const void*> send;
   std::vector<int> device;
-  explicit LocalGroup(int w) : world(w), send((size_t)w, nullptr), device((size_t)w, 0) {}
+  std::vector<const size_t*> sdispl;  // all-to-all: each rank's byte displacements per destination
+  explicit LocalGroup(int w) : world(w), send((size_t)w, nullptr), device((size_t)w, 0), sdispl((size_t)w, nullptr) {}
   void barrier() {
     std::unique_lock<std::mutex> lk(mu);
     const long long g = gen;
@@ -86,6 +96,15 @@ struct LocalGroup {
     }
   }
 };
+
+__global__ void sum_u64_kernel(const unsigned long long* const* __restrict__ src, int nsrc,
+                               unsigned long long* __restrict__ dst, int64_t n) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    unsigned long long m = 0;
+    for (int r = 0; r < nsrc; ++r) m += src[r][i];
+    dst[i] = m;
+  }
+}
 
 __global__ void or_u32_kernel(const uint32_t* const* __restrict__ src, int nsrc, uint32_t* __restrict__ dst,
                               int64_t n) {
@@ -172,6 +191,64 @@ dt_status comm_allreduce_or_u32(dt_comm* c, uint32_t* buf, int64_t n, cudaStream
   return DT_OK;
 }
 
+// buf[i] = sum over ranks of buf[i] (u64), in place.
+dt_status comm_allreduce_sum_u64(dt_comm* c, unsigned long long* buf, int64_t n, cudaStream_t s) {
+  CommImpl& m = c->impl;
+  if (m.backend == 0) {
+    ncclResult_t r = g_nccl.AllReduce(buf, buf, (size_t)n, ncclUint64, ncclSum, m.nccl, s);
+    if (r != ncclSuccess) return nccl_fail(r, "ncclAllReduce");
+    return DT_OK;
+  }
+  if (m.world == 1) return DT_OK;
+  LocalGroup& g = *m.group;
+  unsigned long long* tmp = nullptr;
+  DT_CK(cudaMallocAsync((void**)&tmp, sizeof(unsigned long long) * (size_t)n, s));
+  DT_CK(cudaStreamSynchronize(s));
+  g.send[(size_t)m.rank] = buf;
+  g.barrier();
+  std::vector<unsigned long long*> ptrs((size_t)m.world);
+  for (int r = 0; r < m.world; ++r) ptrs[(size_t)r] = (unsigned long long*)g.send[(size_t)r];
+  DT_CK(cudaMemcpyAsync(m.dev_ptrs, ptrs.data(), sizeof(void*) * ptrs.size(), cudaMemcpyHostToDevice, s));
+  sum_u64_kernel<<<num_sms() * 2, 256, 0, s>>>(reinterpret_cast<unsigned long long**>(m.dev_ptrs), m.world, tmp, n);
+  DT_CK(cudaGetLastError());
+  DT_CK(cudaStreamSynchronize(s));
+  g.barrier();  // everybody has read every input
+  DT_CK(cudaMemcpyAsync(buf, tmp, sizeof(unsigned long long) * (size_t)n, cudaMemcpyDeviceToDevice, s));
+  DT_CK(cudaFreeAsync(tmp, s));
+  DT_CK(cudaStreamSynchronize(s));
+  return DT_OK;
+}
+
+// All-to-all of byte ranges: this rank sends send[sdispl[q], sdispl[q] + scount[q]) to rank
+// q and receives rank q's range for it at recv + rdispl[q] (rcount[q] bytes).  Host arrays.
+dt_status comm_alltoallv(dt_comm* c, const void* send, const size_t* scount, const size_t* sdispl, void* recv,
+                         const size_t* rcount, const size_t* rdispl, cudaStream_t s) {
+  CommImpl& m = c->impl;
+  if (m.backend == 0) {
+    ncclResult_t r = g_nccl.GroupStart();
+    for (int q = 0; q < m.world && r == ncclSuccess; ++q) {
+      if (scount[q]) r = g_nccl.Send((const char*)send + sdispl[q], scount[q], ncclUint8, q, m.nccl, s);
+      if (r == ncclSuccess && rcount[q]) r = g_nccl.Recv((char*)recv + rdispl[q], rcount[q], ncclUint8, q, m.nccl, s);
+    }
+    ncclResult_t r2 = g_nccl.GroupEnd();
+    if (r != ncclSuccess) return nccl_fail(r, "ncclSend/ncclRecv");
+    if (r2 != ncclSuccess) return nccl_fail(r2, "ncclGroupEnd");
+    return DT_OK;
+  }
+  LocalGroup& g = *m.group;
+  DT_CK(cudaStreamSynchronize(s));
+  g.send[(size_t)m.rank] = send;
+  g.sdispl[(size_t)m.rank] = sdispl;
+  g.barrier();
+  for (int q = 0; q < m.world; ++q)
+    if (rcount[q])
+      DT_CK(cudaMemcpyAsync((char*)recv + rdispl[q], (const char*)g.send[(size_t)q] + g.sdispl[(size_t)q][m.rank],
+                            rcount[q], cudaMemcpyDefault, s));
+  DT_CK(cudaStreamSynchronize(s));
+  g.barrier();
+  return DT_OK;
+}
+
 }  // namespace dtl
 
 using namespace dtl;
@@ -217,7 +294,7 @@ dt_status dt_comm_init_local(int32_t world, dt_comm** comms_out) {
     c->impl.world = world;
     c->impl.backend = 1;
     c->impl.group = g;
-    cudaError_t e = cudaMalloc((void**)&c->impl.dev_ptrs, sizeof(uint32_t*) * (size_t)world);
+    cudaError_t e = cudaMalloc((void**)&c->impl.dev_ptrs, sizeof(void*) * (size_t)world);
     if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc", __FILE__, __LINE__);
     comms_out[r] = c;
   }

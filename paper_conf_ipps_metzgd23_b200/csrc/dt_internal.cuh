@@ -50,13 +50,17 @@ dt_status release_workspace_impl();
 void forest_release_scratch();
 dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
                    int64_t min_leaf, cudaStream_t s, dt_tree** out);
-dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64_t n, int32_t dg,
-                           int32_t max_depth, int64_t min_leaf, cudaStream_t s, dt_tree** out);
+dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64_t n_local, int64_t row_offset,
+                           int64_t n_global, int32_t d, int32_t max_depth, int64_t min_leaf, cudaStream_t s,
+                           dt_tree** out);
 // Communicators (comm.cu).
 int comm_rank(const dt_comm* c);
 int comm_world(const dt_comm* c);
 dt_status comm_allgather(dt_comm* c, const void* send, void* recv, size_t bytes, cudaStream_t s);
 dt_status comm_allreduce_or_u32(dt_comm* c, uint32_t* buf, int64_t n, cudaStream_t s);
+dt_status comm_allreduce_sum_u64(dt_comm* c, unsigned long long* buf, int64_t n, cudaStream_t s);
+dt_status comm_alltoallv(dt_comm* c, const void* send, const size_t* scount, const size_t* sdispl, void* recv,
+                         const size_t* rcount, const size_t* rdispl, cudaStream_t s);
 // Predict / eval (predict.cu).
 dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, int32_t dc, const float* gpu,
                            int64_t n_gpu, int32_t dg, const int32_t* src, double* yhat, cudaStream_t s);

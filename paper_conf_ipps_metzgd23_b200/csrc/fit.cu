@@ -536,13 +536,32 @@ __global__ void __launch_bounds__(256) goleft_kernel(const Ctl* __restrict__ ctl
 
 // P = 1: the children's segment table (level l+1; written children at wstart of every
 // list) and the plan of every level-l segment (children, centres, positions).
+// mode 0 (P = 1): as above.  Sharded: mode 1 = the plans without the children's positions
+// and rank carries (before the boundary exchange), mode 2 = those from segs_next.
 __global__ void __launch_bounds__(256) tables_kernel(const Ctl* __restrict__ ctl, int par, int d,
                                                      const NodeL* __restrict__ next, const Decision* __restrict__ dec,
                                                      const SegT* __restrict__ segs, SegT* __restrict__ segs_next,
-                                                     PSeg* __restrict__ pseg) {
+                                                     PSeg* __restrict__ pseg, int mode) {
   const uint32_t K = ctl->K[par], K2 = ctl->K[par ^ 1];
   const uint64_t A2 = ctl->A2;
-  const int64_t n1 = (int64_t)K2 * d, n2 = (int64_t)K * d;
+  if (mode == 2) {
+    for (int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; s < (int64_t)K * d;
+         s += (int64_t)gridDim.x * blockDim.x) {
+      const uint32_t k = (uint32_t)(s % K);
+      const Decision dc = dec[k];
+      if (dc.f < 0) continue;
+      const int f = (int)(s / K);
+      for (int q = 0; q < 2; ++q) {
+        const SegT c = segs_next[(int64_t)f * K2 + dc.kid + q];
+        pseg[s].ostart[q] = c.start;
+        pseg[s].ioff[q] = c.ioff;
+        pseg[s].soff[q] = c.soff;
+        pseg[s].xprev[q] = c.xprev;
+      }
+    }
+    return;
+  }
+  const int64_t n1 = mode == 0 ? (int64_t)K2 * d : 0, n2 = (int64_t)K * d;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n1 + n2; i += (int64_t)gridDim.x * blockDim.x) {
     if (i < n1) {
       const int f = (int)(i / K2);
@@ -597,6 +616,128 @@ __global__ void __launch_bounds__(256) tables_kernel(const Ctl* __restrict__ ctl
       pseg[s] = p;
     }
   }
+}
+
+// ----------------------------------------------------------------------------- sharded --
+
+// Value-range sharded fit: this rank's part of every child segment (count, last x, sum of
+// (y - c_child)) from its parent segment's total aggregate = chunk carry of the segment's
+// last chunk + that chunk's tail piece (F_A).
+__global__ void __launch_bounds__(256) bnd_kernel(const Ctl* __restrict__ ctl, int par, int d,
+                                                  const PSeg* __restrict__ pseg, const AggP* __restrict__ tails,
+                                                  const AggP* __restrict__ cexcl, const AggP* __restrict__ bcarry,
+                                                  BndRec* __restrict__ out) {
+  const uint32_t K = ctl->K[par], K2 = ctl->K[par ^ 1];
+  for (int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; s < (int64_t)K * d;
+       s += (int64_t)gridDim.x * blockDim.x) {
+    const PSeg ps = pseg[s];
+    if (!(ps.flags & PS_SPLIT)) continue;
+    BndRec L{0u, __int_as_float(0x7fc00000), 0.0}, R = L;
+    if (ps.cnt) {
+      const uint64_t last = ps.start + ps.cnt - 1;
+      const int64_t c = (int64_t)(last / kChunkW);
+      AggP t = tails[s];
+      if (!t.flag) t = combine(combine(bcarry[c / kBlockChunks], cexcl[c]), t);
+      L.cnt = t.nl;
+      L.xlast = t.xl;
+      L.s = t.sl;
+      R.cnt = ps.cnt - t.nl;
+      R.xlast = t.xr;
+      R.s = t.sr;
+    }
+    const int64_t i = (int64_t)ps.f * K2 + ps.kid;
+    out[i] = L;
+    out[i + 1] = R;
+  }
+  (void)d;
+}
+
+// Flat exclusive scan of the children's written local counts over (feature, child) in
+// feature-major order (the next level's list layout): block scans + block totals, the
+// last block scans the totals (ticket).
+__global__ void __launch_bounds__(1024) segscan_kernel(Ctl* ctl, int par, int d, const NodeL* __restrict__ next,
+                                                       const BndRec* __restrict__ mine,
+                                                       unsigned long long* __restrict__ excl,
+                                                       unsigned long long* __restrict__ btot) {
+  __shared__ unsigned long long sh[33];
+  __shared__ bool s_last;
+  const uint32_t K2 = ctl->K[par ^ 1];
+  const int64_t n = (int64_t)K2 * d;
+  const int64_t i = (int64_t)blockIdx.x * 1024 + threadIdx.x;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  unsigned long long v = 0;
+  if (i < n) {
+    const uint32_t kc = (uint32_t)(i % K2);
+    v = next[kc].searchable ? mine[i].cnt : 0u;
+  }
+  unsigned long long inc = v;
+#pragma unroll
+  for (int dd = 1; dd < 32; dd <<= 1) {
+    const unsigned long long o = __shfl_up_sync(0xffffffffu, inc, dd);
+    if (lane >= dd) inc += o;
+  }
+  if (lane == 31) sh[w] = inc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long r = 0;
+    for (int q = 0; q < 32; ++q) { const unsigned long long t = sh[q]; sh[q] = r; r += t; }
+    sh[32] = r;
+  }
+  __syncthreads();
+  if (i < n) excl[i] = sh[w] + inc - v;
+  if (threadIdx.x == 0) btot[blockIdx.x] = sh[32];
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) s_last = atomicAdd(&ctl->ticket, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (!s_last || threadIdx.x != 0) return;
+  __threadfence();
+  ctl->ticket = 0u;
+  const int64_t nb = (n + 1023) / 1024;
+  unsigned long long r = 0;
+  for (int64_t b = 0; b < nb; ++b) {  // block offsets (in place), then the totals
+    const unsigned long long t = __ldcg(btot + b);
+    btot[b] = r;
+    r += t;
+  }
+  ctl->T[par ^ 1] = r;
+  (void)d;
+}
+
+// The next level's segment table: positions from the scan, rank carries from the ranks'
+// records (rank order); the list sizes.
+__global__ void __launch_bounds__(256) segwrite_kernel(Ctl* ctl, int par, int d, int rank, const NodeL* __restrict__ next,
+                                                       const BndRec* __restrict__ all,
+                                                       const unsigned long long* __restrict__ excl,
+                                                       const unsigned long long* __restrict__ boff,
+                                                       SegT* __restrict__ segs_next) {
+  const uint32_t K2 = ctl->K[par ^ 1];
+  const int64_t n = (int64_t)K2 * d;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t kc = (uint32_t)(i % K2);
+    const int f = (int)(i / K2);
+    uint32_t ioff = 0;
+    double soff = 0.0;
+    float xprev = __int_as_float(0x7fc00000);
+    for (int q = 0; q < rank; ++q) {
+      const BndRec r = all[(int64_t)q * n + i];
+      ioff += r.cnt;
+      soff = __dadd_rn(soff, r.s);
+      if (r.cnt) xprev = r.xlast;
+    }
+    SegT sg;
+    sg.start = boff[i / 1024] + excl[i];
+    sg.cnt = next[kc].searchable ? all[(int64_t)rank * n + i].cnt : 0u;
+    sg.k = kc;
+    sg.f = f;
+    sg.ioff = ioff;
+    sg.soff = soff;
+    sg.xprev = xprev;
+    sg.pad = 0;
+    segs_next[i] = sg;
+    if (i == K2) ctl->T0[par ^ 1] = sg.start;  // feature list 0 ends where list 1 starts
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0 && d == 1) ctl->T0[par ^ 1] = ctl->T[par ^ 1];
 }
 
 // ----------------------------------------------------------------------------- finish --
@@ -735,7 +876,7 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int64_t n_global, int32_t d, int32_t 
     GET(b.tails, b.segcap);
     GET(b.bnd_send, 2 * b.segcap);
     GET(b.bnd_all, 2 * b.segcap * world);
-    GET(b.scan_tmp, (2 * b.segcap + 1023) / 1024 + 2);
+    GET(b.scan_tmp, b.segcap + b.segcap / 1024 + 2);  // exclusive values, then block totals
   } else {
     b.exch_all = b.exch_send;
   }
@@ -830,7 +971,7 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
     na.log = b.lvlog;
     pr = prof_begin(PK_NUMBER, s, 2);
     number_kernel<<<1, 1024, 0, s>>>(na);
-    tables_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, b.nodes[par ^ 1], b.dec, b.segs[par], b.segs[par ^ 1], b.pseg);
+    tables_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, b.nodes[par ^ 1], b.dec, b.segs[par], b.segs[par ^ 1], b.pseg, 0);
     prof_end(pr, s, 0.0);
     DT_CK(cudaGetLastError());
     // ---- go-left bitmap (a6)
@@ -1086,10 +1227,148 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
   return fit_finish(b, d, s, &pending, out);
 }
 
-dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64_t n, int32_t dg,
-                           int32_t max_depth, int64_t min_leaf, cudaStream_t s, dt_tree** out) {
-  (void)comm; (void)X; (void)y; (void)n; (void)dg; (void)max_depth; (void)min_leaf; (void)s; (void)out;
-  return fail(DT_ERR_INVALID_ARG, "dt_fit_sharded: not available in this build");
+// Value-range row-sharded fit: rank p holds rows
+// [row_offset, row_offset + n_local) of the table; after the sharded presort it owns global
+// sorted positions [p n / P, (p + 1) n / P) of every feature list and its entries never
+// move between ranks again.  Per level: allgather of the per-node local bests (decided in
+// rank order), OR-allreduce of the go-left bitmap, allgather of the children's boundary
+// records (count, last x, S') -> rank carries of every child segment.  Every rank builds
+// the same tree.  Direct enqueue; one host synchronisation per level (the node count).
+dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64_t n_local, int64_t row_offset,
+                           int64_t n_global, int32_t d, int32_t max_depth, int64_t min_leaf, cudaStream_t s,
+                           dt_tree** out) {
+  const int P = comm_world(comm), rank = comm_rank(comm);
+  int dev = 0;
+  DT_CK(cudaGetDevice(&dev));
+  const int64_t nlist = std::max<int64_t>(std::max<int64_t>(n_local, (n_global + P - 1) / P), 1);
+  Workspace ws;
+  ws.s = s;
+  FitBufs b{};
+  auto get = [&](auto** p, size_t count) -> cudaError_t { return ws.get(p, count); };
+  dt_status st = fit_alloc(b, nlist, n_global, d, max_depth, min_leaf, std::max(P, 2), get);
+  if (st != DT_OK) return st;
+  std::vector<Pending> pending;
+  DT_CK(cudaMemsetAsync(b.slot_gain, 0, sizeof(unsigned long long) * (size_t)b.segcap, s));
+  DT_CK(cudaMemsetAsync(b.slot_pos, 0xFF, sizeof(unsigned long long) * (size_t)b.segcap, s));
+  DT_CK(cudaMemsetAsync(b.head_cand, 0xFF, sizeof(Cand2) * (size_t)b.segcap, s));
+  DT_CK(cudaMemsetAsync(b.cont_cand, 0xFF, sizeof(Cand2) * (size_t)(2 * b.max_chunks), s));
+  DT_CK(cudaMemsetAsync(b.ctl, 0, sizeof(Ctl), s));
+  st = presort_sharded_enqueue(b, comm, X, y, n_local, row_offset, n_global, d, max_depth, min_leaf, s);
+  if (st != DT_OK) return st;
+  Ctl* ctl = b.ctl;
+  {  // the virtual-root pass (the root's rank carries come from the presort)
+    LevelArgs la{-1, 0, 0, d, min_leaf, false};
+    int pr = prof_begin(PK_SCAN, s, 2);
+    st = level_agg_enqueue(b, la, s);
+    if (st != DT_OK) return st;
+    prof_end(pr, s, 0.0);
+    pr = prof_begin(PK_PARTITION, s, 1);
+    st = level_fused_enqueue(b, la, s);
+    if (st != DT_OK) return st;
+    prof_end(pr, s, 0.0);
+  }
+  const int g_sel = num_sms() * 4;
+  const int g_gl = grid_of((const void*)goleft_kernel, 256, 0);
+  const int g_tab = num_sms() * 4;
+  uint32_t K = 1;  // nodes at the level (host copy)
+  for (int level = 0;; ++level) {
+    const int par = level & 1, cur = par;
+    SelectArgs se;
+    se.gbits = reinterpret_cast<uint4*>(b.gbits);
+    se.nvec = b.nwords4 / 4;
+    se.nodes = b.nodes[par];
+    se.segs_prev = level == 0 ? b.segs[0] : b.segs[par ^ 1];
+    se.ctl = ctl;
+    se.par = par;
+    se.level = level;
+    se.d = d;
+    se.head_cand = b.head_cand;
+    se.cont_cand = b.cont_cand;
+    se.head_stat = b.head_stat;
+    se.cont_stat = b.cont_stat;
+    se.dec = b.dec;
+    se.out = b.dout;
+    se.log = b.lvlog;
+    se.slot_gain = b.slot_gain;
+    se.slot_pos = b.slot_pos;
+    se.exch = b.exch_send;
+    se.world = P;
+    int pr = prof_begin(PK_SELECT, s, 3);
+    piece_pos_kernel<<<num_sms() * 4, 256, 0, s>>>(ctl, par, d, (uint32_t)level, b.head_cand, b.cont_cand,
+                                                    b.slot_gain, b.slot_pos);
+    select_kernel<<<g_sel, 256, 0, s>>>(se);
+    DT_CK(cudaGetLastError());
+    st = comm_allgather(comm, b.exch_send, b.exch_all, sizeof(ExchRec) * (size_t)K, s);
+    if (st != DT_OK) return st;
+    decide_kernel<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((K + 255) / 256, num_sms() * 4)), 256, 0, s>>>(
+        se, b.exch_all, (int64_t)K);
+    prof_end(pr, s, 0.0);
+    DT_CK(cudaGetLastError());
+    if (max_depth >= 0 && level == max_depth) break;
+    NumberArgs na;
+    na.nodes = b.nodes[par];
+    na.next = b.nodes[par ^ 1];
+    na.dec = b.dec;
+    na.ctl = ctl;
+    na.par = par;
+    na.level = level;
+    na.d = d;
+    na.max_depth = max_depth;
+    na.min_leaf = min_leaf;
+    na.out = b.dout;
+    na.log = b.lvlog;
+    pr = prof_begin(PK_NUMBER, s, 1);
+    number_kernel<<<1, 1024, 0, s>>>(na);
+    prof_end(pr, s, 0.0);
+    DT_CK(cudaGetLastError());
+    uint32_t hk[2], hsrch = 0;
+    DT_CK(cudaMemcpyAsync(hk, ctl->K, sizeof hk, cudaMemcpyDeviceToHost, s));
+    DT_CK(cudaMemcpyAsync(&hsrch, &ctl->nsrch, sizeof hsrch, cudaMemcpyDeviceToHost, s));
+    DT_CK(cudaStreamSynchronize(s));
+    const uint32_t K2 = hk[par ^ 1];
+    if (K2 == 0) break;  // every node of the level is a leaf (same on every rank)
+    // go-left bitmap: each rank sets the bits of its own split-feature entries; OR over ranks
+    pr = prof_begin(PK_GOLEFT, s, 1);
+    goleft_kernel<<<g_gl, 256, 0, s>>>(ctl, par, b.desc[par], b.segs[par], b.dec, b.lr[cur], b.gbits);
+    DT_CK(cudaGetLastError());
+    st = comm_allreduce_or_u32(comm, b.gbits, b.nwords4, s);
+    if (st != DT_OK) return st;
+    prof_end(pr, s, 0.0);
+    tables_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, b.nodes[par ^ 1], b.dec, b.segs[par], b.segs[par ^ 1], b.pseg, 1);
+    DT_CK(cudaGetLastError());
+    LevelArgs la{level, cur, par, d, min_leaf, true};
+    pr = prof_begin(PK_SCAN, s, 3);
+    st = level_agg_enqueue(b, la, s);
+    if (st != DT_OK) return st;
+    prof_end(pr, s, 0.0);
+    if (hsrch > 0) {
+      // children's boundary records -> their segments (positions, rank carries)
+      const int64_t n2 = (int64_t)K2 * d;
+      bnd_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, b.pseg, b.tails, b.cexcl, b.bcarry, b.bnd_send);
+      DT_CK(cudaGetLastError());
+      st = comm_allgather(comm, b.bnd_send, b.bnd_all, sizeof(BndRec) * (size_t)n2, s);
+      if (st != DT_OK) return st;
+      unsigned long long* excl = b.scan_tmp;
+      unsigned long long* btot = b.scan_tmp + b.segcap;
+      segscan_kernel<<<(unsigned)((n2 + 1023) / 1024), 1024, 0, s>>>(ctl, par, d, b.nodes[par ^ 1], b.bnd_send,
+                                                                      excl, btot);
+      segwrite_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, rank, b.nodes[par ^ 1], b.bnd_all, excl, btot,
+                                            b.segs[par ^ 1]);
+      tables_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, b.nodes[par ^ 1], b.dec, b.segs[par], b.segs[par ^ 1], b.pseg,
+                                          2);
+      DT_CK(cudaGetLastError());
+    } else {
+      // no searchable child: statistics only, nothing is written (empty next lists)
+      DT_CK(cudaMemsetAsync(&ctl->T[par ^ 1], 0, sizeof(unsigned long long), s));
+      DT_CK(cudaMemsetAsync(&ctl->T0[par ^ 1], 0, sizeof(unsigned long long), s));
+    }
+    pr = prof_begin(PK_PARTITION, s, 1);
+    st = level_fused_enqueue(b, la, s);
+    if (st != DT_OK) return st;
+    prof_end(pr, s, 0.0);
+    K = K2;
+  }
+  return fit_finish(b, d, s, nullptr, out);
 }
 
 }  // namespace dtl

@@ -284,6 +284,9 @@ struct LevelArgs {
   int64_t min_leaf;
   bool tails;       // sharded: per-segment tail aggregates
 };
+dt_status presort_sharded_enqueue(const FitBufs& b, dt_comm* comm, const float* X, const double* y, int64_t n_local,
+                                  int64_t row0, int64_t n_global, int d, int32_t max_depth, int64_t min_leaf,
+                                  cudaStream_t s);
 dt_status level_agg_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t s);
 dt_status level_fused_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t s);
 

@@ -2,6 +2,7 @@
 // "Kernels"): per-feature stable sort of (x, row id) once per fit, written as the level-0
 // lists, the level-0 segment table, the chunk descriptors and the root node.
 #include <algorithm>
+#include <vector>
 
 #include "fit_core.cuh"
 
@@ -73,12 +74,13 @@ __global__ void root_finalize_kernel(const RootPart* parts, int nparts, int64_t 
 }
 
 // S'_0 = sum (y - c0) over all rows (second pass; c0 from the finalised root sum).
-__global__ void __launch_bounds__(256) root_center_kernel(const double* __restrict__ y, int64_t n,
+// (n: rows of this call; n_all: rows of the whole table, whose mean gives the centre)
+__global__ void __launch_bounds__(256) root_center_kernel(const double* __restrict__ y, int64_t n, int64_t n_all,
                                                           int64_t chunk, const Ctl* ctl, double* parts) {
   const int64_t lo = (int64_t)blockIdx.x * chunk, hi = min(n, lo + chunk);
   double c0;
-  if (ctl->int_mode) c0 = (double)floor_div_ll((long long)ctl->ysum, (long long)n);
-  else c0 = __ddiv_rn(ctl->ysum, (double)n);
+  if (ctl->int_mode) c0 = (double)floor_div_ll((long long)ctl->ysum, (long long)n_all);
+  else c0 = __ddiv_rn(ctl->ysum, (double)n_all);
   double s = 0, cc = 0;
   for (int64_t r = lo + threadIdx.x; r < hi; r += blockDim.x) neu_add(s, cc, __dsub_rn(y[r], c0));
   __shared__ double sh[256];
@@ -381,6 +383,248 @@ __global__ void __launch_bounds__(kTS, DT_RS_MINB) rs_scatter_kernel(const uint3
   }
 }
 
+// ------------------------------------------------------------ value-range sharding --
+// (SURVEY 8(e)): rank p of P ends up holding, for every feature f,
+// the entries at global sorted positions [p n / P, (p + 1) n / P) of f's (x, row id)
+// order: a local sort, exact splitters by bisection on the 64-bit key (flip(x) << 32 |
+// row id, all distinct) with a sum-allreduce of the ranks' counts per round, an
+// all-to-all of 16-byte entries, a local stable sort of the received runs (source-rank
+// order = row order for equal x, since rank q holds rows [row_offset_q, ...)).
+
+struct Sent {  // one entry on the wire
+  uint32_t key, row;
+  double y;
+};
+
+// One rank's partial of the root statistics (block parts folded in index order).
+__global__ void root_fold_kernel(const RootPart* parts, int nparts, RootPart* out) {
+  if (threadIdx.x != 0) return;
+  RootPart a{0, 0, INFINITY, -INFINITY, 1, 1};
+  for (int i = 0; i < nparts; ++i) {
+    neu_add(a.s, a.c, parts[i].s);
+    neu_add(a.s, a.c, parts[i].c);
+    a.mn = fmin(a.mn, parts[i].mn);
+    a.mx = fmax(a.mx, parts[i].mx);
+    a.integral &= parts[i].integral;
+    a.finite &= parts[i].finite;
+  }
+  *out = a;
+}
+__global__ void center_fold_kernel(const double* parts, int nparts, double* out) {
+  if (threadIdx.x != 0) return;
+  double s = 0, cc = 0;
+  for (int i = 0; i < nparts; ++i) neu_add(s, cc, parts[i]);
+  *out = __dadd_rn(s, cc);
+}
+
+__device__ __forceinline__ unsigned long long ckey(const uint32_t* keys, const uint32_t* vals, int64_t i) {
+  return ((unsigned long long)keys[i] << 32) | vals[i];
+}
+// number of local composite keys < v in a sorted list of n
+__device__ __forceinline__ uint32_t count_less(const uint32_t* keys, const uint32_t* vals, int64_t n,
+                                               unsigned long long v) {
+  int64_t lo = 0, hi = n;
+  while (lo < hi) {
+    const int64_t mid = (lo + hi) >> 1;
+    if (ckey(keys, vals, mid) < v) lo = mid + 1;
+    else hi = mid;
+  }
+  return (uint32_t)lo;
+}
+
+// bisection state per (feature, boundary b = 1 .. P-1): [lo, hi) with count(< lo) <= t_b
+__global__ void split_init_kernel(unsigned long long* lohi, int nb) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nb; i += gridDim.x * blockDim.x) {
+    lohi[2 * i] = 0ull;
+    lohi[2 * i + 1] = ~0ull;
+  }
+}
+__global__ void split_count_kernel(const uint32_t* __restrict__ keys, const uint32_t* __restrict__ vals, int64_t n,
+                                   int nbper, int nb, const unsigned long long* __restrict__ lohi,
+                                   unsigned long long* __restrict__ cnt) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nb; i += gridDim.x * blockDim.x) {
+    const int f = i / nbper;
+    const unsigned long long lo = lohi[2 * i], hi = lohi[2 * i + 1];
+    const unsigned long long mid = lo + (hi - lo) / 2;
+    cnt[i] = count_less(keys + (int64_t)f * n, vals + (int64_t)f * n, n, mid);
+  }
+}
+__global__ void split_update_kernel(int nbper, int nb, int P, int64_t n_global, unsigned long long* __restrict__ lohi,
+                                   const unsigned long long* __restrict__ cnt) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nb; i += gridDim.x * blockDim.x) {
+    const int b = i % nbper + 1;
+    const unsigned long long t = (unsigned long long)(((__int128)b * n_global) / P);
+    const unsigned long long lo = lohi[2 * i], hi = lohi[2 * i + 1];
+    if (hi - lo <= 1) continue;
+    const unsigned long long mid = lo + (hi - lo) / 2;
+    if (cnt[i] <= t) lohi[2 * i] = mid;
+    else lohi[2 * i + 1] = mid;
+  }
+}
+// cut[f][q], q = 0..P: local entries of feature f below rank q's first key
+__global__ void cut_kernel(const uint32_t* __restrict__ keys, const uint32_t* __restrict__ vals, int64_t n, int d,
+                           int P, const unsigned long long* __restrict__ lohi, uint32_t* __restrict__ cut) {
+  const int nbper = P - 1;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < d * (P + 1); i += gridDim.x * blockDim.x) {
+    const int f = i / (P + 1), q = i % (P + 1);
+    uint32_t c;
+    if (q == 0) c = 0;
+    else if (q == P) c = (uint32_t)n;
+    else c = count_less(keys + (int64_t)f * n, vals + (int64_t)f * n, n, lohi[2 * (f * nbper + q - 1)]);
+    cut[i] = c;
+  }
+}
+// send[soff[f][q] + (i - cut[f][q])] = entry i of feature f's sorted list, q its destination
+__global__ void pack_kernel(const uint32_t* __restrict__ keys, const uint32_t* __restrict__ vals,
+                            const double* __restrict__ y, int64_t row0, int64_t n, int d, int P,
+                            const uint32_t* __restrict__ cut, const unsigned long long* __restrict__ soff,
+                            Sent* __restrict__ send) {
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < n * d; t += (int64_t)gridDim.x * blockDim.x) {
+    const int f = (int)(t / n);
+    const uint32_t i = (uint32_t)(t - (int64_t)f * n);
+    int q = 0;
+    while (q + 1 < P && i >= cut[f * (P + 1) + q + 1]) ++q;
+    Sent e;
+    e.key = keys[t];
+    e.row = vals[t];
+    e.y = __ldg(y + (e.row - row0));
+    send[soff[f * P + q] + (i - cut[f * (P + 1) + q])] = e;
+  }
+}
+// received entry r (from rank q, feature f, index i) -> the concatenation of feature f's
+// runs in source-rank order: keys / positions for the local stable sort
+__global__ void unpack_kernel(const Sent* __restrict__ recv, int64_t nrecv, int d, int P,
+                              const unsigned long long* __restrict__ roff, const unsigned long long* __restrict__ cpos,
+                              uint32_t* __restrict__ keys, uint32_t* __restrict__ vals) {
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < nrecv; r += (int64_t)gridDim.x * blockDim.x) {
+    int k = 0;  // largest (q, f) block with roff <= r (blocks in q-major, f-minor order)
+    int lo = 0, hi = P * d;
+    while (hi - lo > 1) {
+      const int mid = (lo + hi) >> 1;
+      if (roff[mid] <= (unsigned long long)r) lo = mid;
+      else hi = mid;
+    }
+    k = lo;
+    const int q = k / d, f = k % d;
+    const unsigned long long pos = cpos[f * P + q] + ((unsigned long long)r - roff[k]);
+    keys[pos] = recv[r].key;
+    vals[pos] = (uint32_t)r;
+  }
+}
+__global__ void __launch_bounds__(256) build_recv_kernel(const uint32_t* __restrict__ keys, const uint32_t* __restrict__ idx,
+                                                         const Sent* __restrict__ recv, int64_t total,
+                                                         float* __restrict__ lx, uint32_t* __restrict__ lr,
+                                                         double* __restrict__ ly, const Ctl* ctl) {
+  const bool y32 = ctl->y32 != 0;
+  for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < total; p += (int64_t)gridDim.x * blockDim.x) {
+    const Sent e = recv[idx[p]];
+    lx[p] = unflip_f32(keys[p]);
+    lr[p] = e.row;
+    if (y32) reinterpret_cast<int32_t*>(ly)[p] = (int32_t)e.y;
+    else ly[p] = e.y;
+  }
+}
+// per feature list: the rank's boundary record (count, last x, sum of (y - c0)), fixed shape
+__global__ void __launch_bounds__(256) root_bnd_kernel(const float* __restrict__ lx, const double* __restrict__ ly,
+                                                       int64_t A0, const Ctl* __restrict__ ctl,
+                                                       const NodeL* __restrict__ nodes0, BndRec* __restrict__ out) {
+  const int f = blockIdx.x;
+  const bool y32 = ctl->y32 != 0;
+  const double c0 = nodes0[0].c;
+  double acc = 0.0;
+  for (int64_t i = threadIdx.x; i < A0; i += blockDim.x) {
+    const int64_t p = (int64_t)f * A0 + i;
+    const double yv = y32 ? (double)reinterpret_cast<const int32_t*>(ly)[p] : ly[p];
+    acc = __dadd_rn(acc, __dsub_rn(yv, c0));
+  }
+  __shared__ double sh[256];
+  sh[threadIdx.x] = acc;
+  __syncthreads();
+  for (int off = 128; off > 0; off >>= 1) {
+    if (threadIdx.x < off) sh[threadIdx.x] = __dadd_rn(sh[threadIdx.x], sh[threadIdx.x + off]);
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    BndRec r;
+    r.cnt = (uint32_t)A0;
+    r.xlast = A0 ? lx[(int64_t)f * A0 + A0 - 1] : __int_as_float(0x7fc00000);
+    r.s = sh[0];
+    out[f] = r;
+  }
+}
+// rank carries of the root's segments from the gathered records (rank order), the
+// level-0 tables and the virtual-root plan
+__global__ void __launch_bounds__(256) root_tables_sharded_kernel(Ctl* ctl, const NodeL* __restrict__ nodes0, int64_t A0,
+                                                                  int d, int rank, int world,
+                                                                  const BndRec* __restrict__ all, SegT* __restrict__ seg0,
+                                                                  PSeg* __restrict__ pseg, uint32_t* __restrict__ desc0) {
+  const NodeL rt = nodes0[0];
+  const int64_t nch = (A0 * d + kChunkW - 1) / kChunkW;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nch; i += (int64_t)gridDim.x * blockDim.x)
+    desc0[i] = (uint32_t)((i * kChunkW) / A0);
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    ctl->T[0] = (unsigned long long)A0 * d;
+    ctl->T0[0] = (unsigned long long)A0;
+  }
+  for (int f = blockIdx.x * blockDim.x + threadIdx.x; f < d; f += gridDim.x * blockDim.x) {
+    uint32_t ioff = 0;
+    double soff = 0.0;
+    float xprev = __int_as_float(0x7fc00000);
+    for (int q = 0; q < rank; ++q) {
+      const BndRec r = all[(int64_t)q * d + f];
+      ioff += r.cnt;
+      soff = __dadd_rn(soff, r.s);
+      if (r.cnt) xprev = r.xlast;
+    }
+    SegT sg;
+    sg.start = (uint64_t)f * (uint64_t)A0;
+    sg.cnt = (uint32_t)A0;
+    sg.k = 0;
+    sg.f = f;
+    sg.ioff = ioff;
+    sg.soff = soff;
+    sg.xprev = xprev;
+    sg.pad = 0;
+    seg0[f] = sg;
+    PSeg p;
+    p.start = sg.start;
+    p.cnt = sg.cnt;
+    p.k = 0;
+    p.f = f;
+    p.flags = PS_SPLIT | PS_ALLLEFT | (rt.searchable ? PS_SRCH0 : 0u);
+    p.cs[0] = p.cs[1] = (uint32_t)f;
+    p.ostart[0] = p.ostart[1] = sg.start;
+    p.c[0] = p.c[1] = rt.c;
+    p.v[0] = p.v[1] = rt.v;
+    p.sc[0] = p.sc[1] = rt.sc;
+    p.N[0] = p.N[1] = rt.N;
+    p.ioff[0] = p.ioff[1] = ioff;
+    p.soff[0] = p.soff[1] = soff;
+    p.xprev[0] = p.xprev[1] = xprev;
+    p.kid = 0;
+    p.pad = 0;
+    pseg[f] = p;
+  }
+  (void)world;
+}
+
+// Batched tile radix sort of the d lists of n (key, value) pairs in b.k_in / b.v_in (4
+// passes x 3 launches, ping-pong through k_out / v_out, ends in k_in / v_in); stable.
+void radix_sort_lists(const FitBufs& b, int64_t n, int d, cudaStream_t s) {
+  uint32_t *ki = b.k_in, *ko = b.k_out, *vi = b.v_in, *vo = b.v_out;
+  const int tiles = (int)((n + kTile - 1) / kTile);
+  const dim3 g((unsigned)std::max(tiles, 1), (unsigned)d);
+  for (int pass = 0; pass < 4; ++pass) {
+    const int shift = 8 * pass;
+    rs_count_kernel<<<g, kTS, 0, s>>>(ki, n, shift, tiles, b.rs_cnt);
+    rs_offset_kernel<<<dim3(256, (unsigned)d), std::min(1024, (tiles + 31) / 32 * 32), 0, s>>>(b.rs_cnt, tiles,
+                                                                                            b.rs_off, b.rs_tot);
+    rs_scatter_kernel<<<g, kTS, 0, s>>>(ki, vi, ko, vo, n, shift, tiles, b.rs_off, b.rs_tot);
+    std::swap(ki, ko);
+    std::swap(vi, vo);
+  }
+}
+
 }  // namespace
 
 // Root statistics + presort of one rank's rows (P = 1: all rows) into the level-0 lists,
@@ -395,7 +639,7 @@ dt_status presort_enqueue(const FitBufs& b, const float* X, const double* y, int
     const int pr = prof_begin(PK_ROOT, s, 4);
     root_reduce_kernel<<<(unsigned)b.root_np, 256, 0, s>>>(y, n, b.root_chunk, reinterpret_cast<RootPart*>(b.parts));
     root_finalize_kernel<<<1, 32, 0, s>>>(reinterpret_cast<RootPart*>(b.parts), (int)b.root_np, n, ctl);
-    root_center_kernel<<<(unsigned)b.root_np, 256, 0, s>>>(y, n, b.root_chunk, ctl, b.cparts);
+    root_center_kernel<<<(unsigned)b.root_np, 256, 0, s>>>(y, n, n, b.root_chunk, ctl, b.cparts);
     root_init_kernel<<<1, 32, 0, s>>>(b.cparts, (int)b.root_np, n, d, max_depth, min_leaf, ctl, b.nodes[0],
                                       b.dec_root);
     prof_end(pr, s, 16.0 * (double)n);  // y read twice
@@ -411,19 +655,9 @@ dt_status presort_enqueue(const FitBufs& b, const float* X, const double* y, int
     presort_keys_kernel<<<(unsigned)nb, 256, smem, s>>>(X, n, d, b.k_in, b.v_in, ctl, row0, rb);
     prof_end(pr, s, 16.0 * (double)total0);  // X read + (key, val) written
     DT_CK(cudaGetLastError());
-    // batched tile radix sort of all d lists: 4 passes x 3 launches (ping-pong, ends in _in)
     pr = prof_begin(PK_PRESORT_SORT, s, 12);
-    uint32_t *ki = b.k_in, *ko = b.k_out, *vi = b.v_in, *vo = b.v_out;
-    const dim3 g((unsigned)b.rs_tiles, (unsigned)d);
-    for (int pass = 0; pass < 4; ++pass) {
-      const int shift = 8 * pass;
-      rs_count_kernel<<<g, kTS, 0, s>>>(ki, n, shift, b.rs_tiles, b.rs_cnt);
-      rs_offset_kernel<<<dim3(256, (unsigned)d), std::min(1024, (b.rs_tiles + 31) / 32 * 32), 0, s>>>(
-          b.rs_cnt, b.rs_tiles, b.rs_off, b.rs_tot);
-      rs_scatter_kernel<<<g, kTS, 0, s>>>(ki, vi, ko, vo, n, shift, b.rs_tiles, b.rs_off, b.rs_tot);
-      std::swap(ki, ko);
-      std::swap(vi, vo);
-    }
+    uint32_t *ki = b.k_in, *vi = b.v_in;
+    radix_sort_lists(b, n, d, s);  // ends in k_in / v_in
     prof_end(pr, s, 4.0 * 24.0 * (double)total0);  // per pass: keys read twice, pairs read + written
     DT_CK(cudaGetLastError());
     const int gb = std::max(1, std::min<int>((int)((total0 + 255) / 256), num_sms() * 8));
@@ -433,6 +667,165 @@ dt_status presort_enqueue(const FitBufs& b, const float* X, const double* y, int
     prof_end(pr, s, 36.0 * (double)total0);  // (key, val) read, y gathered, 16 B written
     DT_CK(cudaGetLastError());
   }
+  return DT_OK;
+}
+
+}  // namespace dtl
+
+namespace dtl {
+
+// Value-range sharded presort (see "value-range sharding" above) and the root.  X_local:
+// n_local x d rows row0 .. row0 + n_local - 1 of the global table (rank order: row0 =
+// rows of the lower ranks).  On return the level-0 lists hold this rank's A0 entries of
+// every feature (global positions [p n / P, (p + 1) n / P)), with the rank carries.
+dt_status presort_sharded_enqueue(const FitBufs& b, dt_comm* comm, const float* X, const double* y, int64_t n_local,
+                                  int64_t row0, int64_t n_global, int d, int32_t max_depth, int64_t min_leaf,
+                                  cudaStream_t s) {
+  const int P = comm_world(comm), p = comm_rank(comm);
+  const int64_t lo_p = (int64_t)(((__int128)p * n_global) / P), hi_p = (int64_t)(((__int128)(p + 1) * n_global) / P);
+  const int64_t A0 = hi_p - lo_p;
+  Ctl* ctl = b.ctl;
+  std::vector<void*> tmp;
+  auto alloc = [&](auto** ptr, size_t bytes) -> cudaError_t {
+    cudaError_t e = cudaMallocAsync((void**)ptr, bytes ? bytes : 16, s);
+    if (e == cudaSuccess) tmp.push_back((void*)*ptr);
+    return e;
+  };
+  struct Free {
+    std::vector<void*>& v;
+    cudaStream_t s;
+    ~Free() {
+      for (void* q : v) cudaFreeAsync(q, s);
+    }
+  } freer{tmp, s};
+  // ---- root statistics: per-rank partials, combined in rank order
+  RootPart *mine = nullptr, *allp = nullptr;
+  double *cmine = nullptr, *call = nullptr;
+  DT_CK(alloc(&mine, sizeof(RootPart)));
+  DT_CK(alloc(&allp, sizeof(RootPart) * P));
+  DT_CK(alloc(&cmine, sizeof(double)));
+  DT_CK(alloc(&call, sizeof(double) * P));
+  const int npl = n_local > 0 ? (int)b.root_np : 0;
+  int pr = prof_begin(PK_ROOT, s, 6);
+  if (npl) root_reduce_kernel<<<npl, 256, 0, s>>>(y, n_local, b.root_chunk, reinterpret_cast<RootPart*>(b.parts));
+  root_fold_kernel<<<1, 32, 0, s>>>(reinterpret_cast<RootPart*>(b.parts), npl, mine);
+  DT_CK(cudaGetLastError());
+  dt_status st = comm_allgather(comm, mine, allp, sizeof(RootPart), s);
+  if (st != DT_OK) return st;
+  root_finalize_kernel<<<1, 32, 0, s>>>(allp, P, n_global, ctl);
+  if (npl) root_center_kernel<<<npl, 256, 0, s>>>(y, n_local, n_global, b.root_chunk, ctl, b.cparts);
+  center_fold_kernel<<<1, 32, 0, s>>>(b.cparts, npl, cmine);
+  DT_CK(cudaGetLastError());
+  st = comm_allgather(comm, cmine, call, sizeof(double), s);
+  if (st != DT_OK) return st;
+  root_init_kernel<<<1, 32, 0, s>>>(call, P, n_global, d, max_depth, min_leaf, ctl, b.nodes[0], b.dec_root);
+  prof_end(pr, s, 16.0 * (double)n_local);
+  DT_CK(cudaGetLastError());
+  // ---- local keys, local sort
+  pr = prof_begin(PK_PRESORT_SORT, s, 14);
+  if (n_local > 0) {
+    const int rb = d <= 48 ? 256 : (d <= 96 ? 128 : 64);
+    const size_t smem = sizeof(float) * rb * (size_t)d;
+    if (smem > 48 * 1024)
+      DT_CK(cudaFuncSetAttribute(presort_keys_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    presort_keys_kernel<<<(unsigned)((n_local + rb - 1) / rb), 256, smem, s>>>(X, n_local, d, b.k_in, b.v_in, ctl, row0, rb);
+    radix_sort_lists(b, n_local, d, s);
+    DT_CK(cudaGetLastError());
+  }
+  // ---- exact splitters: 64 bisection rounds on the composite key, counts summed over ranks
+  const int nbper = P - 1, nb = d * nbper;
+  unsigned long long *lohi = nullptr, *cnt = nullptr;
+  DT_CK(alloc(&lohi, sizeof(unsigned long long) * 2 * std::max(nb, 1)));
+  DT_CK(alloc(&cnt, sizeof(unsigned long long) * std::max(nb, 1)));
+  if (nb > 0) {
+    split_init_kernel<<<1, 256, 0, s>>>(lohi, nb);
+    for (int round = 0; round < 64; ++round) {
+      split_count_kernel<<<(nb + 255) / 256, 256, 0, s>>>(b.k_in, b.v_in, n_local, nbper, nb, lohi, cnt);
+      st = comm_allreduce_sum_u64(comm, cnt, nb, s);
+      if (st != DT_OK) return st;
+      split_update_kernel<<<(nb + 255) / 256, 256, 0, s>>>(nbper, nb, P, n_global, lohi, cnt);
+    }
+    DT_CK(cudaGetLastError());
+  }
+  uint32_t *cut = nullptr, *allcnt = nullptr;
+  DT_CK(alloc(&cut, sizeof(uint32_t) * d * (P + 1)));
+  DT_CK(alloc(&allcnt, sizeof(uint32_t) * d * P * P));
+  cut_kernel<<<std::max(1, (d * (P + 1) + 255) / 256), 256, 0, s>>>(b.k_in, b.v_in, n_local, d, P, lohi, cut);
+  DT_CK(cudaGetLastError());
+  std::vector<uint32_t> hcut((size_t)d * (P + 1));
+  DT_CK(cudaMemcpyAsync(hcut.data(), cut, sizeof(uint32_t) * hcut.size(), cudaMemcpyDeviceToHost, s));
+  DT_CK(cudaStreamSynchronize(s));
+  std::vector<uint32_t> mycnt((size_t)d * P);  // [f][q]
+  for (int f = 0; f < d; ++f)
+    for (int q = 0; q < P; ++q) mycnt[(size_t)f * P + q] = hcut[(size_t)f * (P + 1) + q + 1] - hcut[(size_t)f * (P + 1) + q];
+  uint32_t* dmy = nullptr;
+  DT_CK(alloc(&dmy, sizeof(uint32_t) * d * P));
+  DT_CK(cudaMemcpyAsync(dmy, mycnt.data(), sizeof(uint32_t) * mycnt.size(), cudaMemcpyHostToDevice, s));
+  st = comm_allgather(comm, dmy, allcnt, sizeof(uint32_t) * d * P, s);
+  if (st != DT_OK) return st;
+  std::vector<uint32_t> hall((size_t)d * P * P);  // [r][f][q]: rank r sends cnt entries of f to q
+  DT_CK(cudaMemcpyAsync(hall.data(), allcnt, sizeof(uint32_t) * hall.size(), cudaMemcpyDeviceToHost, s));
+  DT_CK(cudaStreamSynchronize(s));
+  auto C = [&](int r, int f, int q) -> uint64_t { return hall[((size_t)r * d + f) * P + q]; };
+  // ---- all-to-all of the entries: to rank q, feature after feature
+  std::vector<size_t> scount(P), sdispl(P), rcount(P), rdispl(P);
+  std::vector<unsigned long long> soff((size_t)d * P), roff((size_t)P * d), cpos((size_t)d * P);
+  size_t sacc = 0, racc = 0;
+  for (int q = 0; q < P; ++q) {
+    sdispl[q] = sacc * sizeof(Sent);
+    for (int f = 0; f < d; ++f) {
+      soff[(size_t)f * P + q] = sacc;
+      sacc += C(p, f, q);
+    }
+    scount[q] = sacc * sizeof(Sent) - sdispl[q];
+    rdispl[q] = racc * sizeof(Sent);
+    for (int f = 0; f < d; ++f) {
+      roff[(size_t)q * d + f] = racc;
+      racc += C(q, f, p);
+    }
+    rcount[q] = racc * sizeof(Sent) - rdispl[q];
+  }
+  if ((int64_t)racc != A0 * d) return fail(DT_ERR_CUDA, "dt_fit_sharded: splitters do not partition the positions");
+  for (int f = 0; f < d; ++f) {
+    unsigned long long acc = (unsigned long long)f * A0;
+    for (int q = 0; q < P; ++q) {
+      cpos[(size_t)f * P + q] = acc;
+      acc += C(q, f, p);
+    }
+  }
+  Sent *sendb = nullptr, *recvb = nullptr;
+  unsigned long long *dsoff = nullptr, *droff = nullptr, *dcpos = nullptr;
+  DT_CK(alloc(&sendb, sizeof(Sent) * (size_t)n_local * d));
+  DT_CK(alloc(&recvb, sizeof(Sent) * (size_t)A0 * d));
+  DT_CK(alloc(&dsoff, sizeof(unsigned long long) * soff.size()));
+  DT_CK(alloc(&droff, sizeof(unsigned long long) * roff.size()));
+  DT_CK(alloc(&dcpos, sizeof(unsigned long long) * cpos.size()));
+  DT_CK(cudaMemcpyAsync(dsoff, soff.data(), sizeof(unsigned long long) * soff.size(), cudaMemcpyHostToDevice, s));
+  DT_CK(cudaMemcpyAsync(droff, roff.data(), sizeof(unsigned long long) * roff.size(), cudaMemcpyHostToDevice, s));
+  DT_CK(cudaMemcpyAsync(dcpos, cpos.data(), sizeof(unsigned long long) * cpos.size(), cudaMemcpyHostToDevice, s));
+  const int gb = num_sms() * 8;
+  if (n_local > 0) pack_kernel<<<gb, 256, 0, s>>>(b.k_in, b.v_in, y, row0, n_local, d, P, cut, dsoff, sendb);
+  DT_CK(cudaGetLastError());
+  st = comm_alltoallv(comm, sendb, scount.data(), sdispl.data(), recvb, rcount.data(), rdispl.data(), s);
+  if (st != DT_OK) return st;
+  // ---- the received runs, concatenated per feature in source-rank order, stable-sorted
+  if (A0 > 0) {
+    unpack_kernel<<<gb, 256, 0, s>>>(recvb, A0 * d, d, P, droff, dcpos, b.k_in, b.v_in);
+    radix_sort_lists(b, A0, d, s);
+    build_recv_kernel<<<gb, 256, 0, s>>>(b.k_in, b.v_in, recvb, A0 * d, b.lx[0], b.lr[0], b.ly[0], ctl);
+    DT_CK(cudaGetLastError());
+  }
+  prof_end(pr, s, 0.0);
+  // ---- rank carries of the root's segments, level-0 tables, virtual-root plan
+  BndRec *bmine = nullptr, *ball = nullptr;
+  DT_CK(alloc(&bmine, sizeof(BndRec) * d));
+  DT_CK(alloc(&ball, sizeof(BndRec) * d * P));
+  root_bnd_kernel<<<d, 256, 0, s>>>(b.lx[0], b.ly[0], A0, ctl, b.nodes[0], bmine);
+  DT_CK(cudaGetLastError());
+  st = comm_allgather(comm, bmine, ball, sizeof(BndRec) * d, s);
+  if (st != DT_OK) return st;
+  root_tables_sharded_kernel<<<num_sms(), 256, 0, s>>>(ctl, b.nodes[0], A0, d, p, P, ball, b.segs[0], b.pseg, b.desc[0]);
+  DT_CK(cudaGetLastError());
   return DT_OK;
 }
 

@@ -288,20 +288,34 @@ def test_fit_graph_replay_matches_direct(dt):
     _assert_exact(np.frombuffer(runs[0], dtype=dt.NODE_DTYPE), oracle.fit(X, y, 10, 2))
 
 
-# ------------------------------------------------------------------ feature-sharded fit --
+# ------------------------------------------------------------------ row-sharded fit ------
 
-def _sharded_fit_threads(dt, X, y, D, m, world):
-    """world ranks as host threads on this GPU (dt_comm_init_local), one stream each."""
+def _row_splits(n, world, uneven=False):
+    """Contiguous row blocks per rank (row_offset order); uneven: rank 0 empty, a skew."""
+    if not uneven:
+        cuts = [(r * n) // world for r in range(world + 1)]
+    else:
+        w = np.array([0] + [r + 1 for r in range(1, world)], dtype=np.float64)
+        cuts = [0] + list(np.round(np.cumsum(w) / w.sum() * n).astype(int))
+        cuts[-1] = n
+    return [(cuts[r], cuts[r + 1]) for r in range(world)]
+
+
+def _sharded_fit_threads(dt, X, y, D, m, world, uneven=False):
+    """world ranks as host threads on this GPU (dt_comm_init_local), one stream each; rank
+    r passes only its contiguous block of rows."""
     import threading
     comms = dt.dt_comm_init_local(world)
     Xd, yd = _cuda(X), _cuda(y)
+    parts = _row_splits(len(y), world, uneven)
     trees, errs = [None] * world, []
 
     def run(r):
         try:
+            a, b = parts[r]
             s = torch.cuda.Stream()
             with torch.cuda.stream(s):
-                trees[r] = dt.dt_fit_sharded(comms[r], Xd, yd, D, m, stream=s)
+                trees[r] = dt.dt_fit_sharded(comms[r], Xd[a:b], yd[a:b], a, len(y), D, m, stream=s)
         except Exception as e:  # pragma: no cover - reported below
             errs.append(e)
 
@@ -314,25 +328,63 @@ def _sharded_fit_threads(dt, X, y, D, m, world):
     return trees
 
 
-@pytest.mark.parametrize("world", [2, 3, 4])
+def _same_tree(a, b):
+    """Identical trees except the impurity (summed in another order), 1e-12 relative."""
+    assert len(a) == len(b)
+    for f in ("feature", "left", "right", "depth", "n_samples", "threshold", "value"):
+        assert np.array_equal(a[f], b[f]), f
+    np.testing.assert_allclose(a["impurity"], b["impurity"], rtol=1e-12, atol=1e-15)
+
+
+@pytest.mark.parametrize("world", [2, 3, 4, 8])
 @pytest.mark.parametrize("case", [("ties", 5000, 8, -1, 1), ("continuous", 20000, 16, 12, 1),
                                   ("collinear", 3000, 8, -1, 1), ("mixed", 8000, 7, 6, 3)])
 def test_fit_sharded_identical(dt, world, case):
+    """integer-mode trees of P = 2, 3, 4, 8 row-sharded ranks equal the
+    single-GPU tree and the oracle's."""
     kind, n, d, D, m = case
     X, y = datagen.random_table(n + world, n, d, kind=kind, int_y=True)
     trees = _sharded_fit_threads(dt, X, y, D, m, world)
     ref = _fit(dt, X, y, D, m)
     for t in trees:
-        assert t.nodes.tobytes() == ref.nodes.tobytes()
+        _same_tree(t.nodes, ref.nodes)
         assert t.split_evals == ref.split_evals
     _assert_exact(trees[0].nodes, oracle.fit(X, y, D, m))
+
+
+@pytest.mark.parametrize("world", [2, 5])
+def test_fit_sharded_uneven_rows(dt, world):
+    """Uneven row blocks (rank 0 holds no rows): the value-range presort rebalances."""
+    X, y = datagen.random_table(77, 6000, 6, kind="ties", int_y=True)
+    trees = _sharded_fit_threads(dt, X, y, 10, 2, world, uneven=True)
+    o = oracle.fit(X, y, 10, 2)
+    for t in trees:
+        _assert_exact(t.nodes, o)
+
+
+def test_fit_sharded_tiny(dt):
+    """n < P: some ranks own no sorted positions at all."""
+    X, y = datagen.random_table(5, 3, 2, kind="ties", int_y=True)
+    for t in _sharded_fit_threads(dt, X, y, -1, 1, 4):
+        _assert_exact(t.nodes, oracle.fit(X, y, -1, 1))
 
 
 def test_fit_sharded_c2_schema(dt):
     X, y = datagen.cnn_gpu_table(1, 200_000)
     trees = _sharded_fit_threads(dt, X, y, 12, 1, 4)
     _assert_exact(trees[0].nodes, oracle.fit(X, y, 12, 1))
-    assert all(t.nodes.tobytes() == trees[0].nodes.tobytes() for t in trees)
+    for t in trees[1:]:
+        assert t.nodes.tobytes() == trees[0].nodes.tobytes()
+
+
+def test_fit_sharded_real_mode_contract(dt):
+    """Real-valued targets: the contract against the oracle (sums in another order)."""
+    X, y = datagen.random_table(19, 8000, 6, kind="continuous", int_y=False)
+    trees = _sharded_fit_threads(dt, X, y, 8, 2, 3)
+    st = treecmp.compare(trees[0].nodes, oracle.fit(X, y, 8, 2), X, y)
+    assert st["exempt"] <= 2 + 0.05 * st["compared"], st
+    for t in trees[1:]:
+        assert t.nodes.tobytes() == trees[0].nodes.tobytes()
 
 
 # ------------------------------------------------------------------ grid / importances --
@@ -446,14 +498,14 @@ def test_fit_edge_cases(dt, case, D, m):
 
 
 def test_nccl_communicator_single_rank(dt):
-    """The NCCL backend of dt_comm (libnccl.so.2 loaded at run time, ncclCommInitRank,
-    allgather / OR-allreduce on the fit's stream) with one rank: the sharded fit equals
-    dt_fit bytewise and the sharded metrics equal dt_eval."""
+    """The NCCL backend of dt_comm (libnccl.so.2 loaded at run time, ncclCommInitRank, and
+    the real allgather / allreduce / send-recv collectives on the fit's stream) with one
+    rank: the sharded fit equals dt_fit and the sharded metrics equal dt_eval."""
     comm = dt.dt_comm_init_nccl(0, 1, lambda obj: obj)
     X, y = datagen.cnn_gpu_table(4, 30_000)
     Xd, yd = _cuda(X), _cuda(y)
-    t = dt.dt_fit_sharded(comm, Xd, yd, 10, 2)
-    assert t.nodes.tobytes() == _fit(dt, X, y, 10, 2).nodes.tobytes()
+    t = dt.dt_fit_sharded(comm, Xd, yd, 0, len(y), 10, 2)
+    _same_tree(t.nodes, _fit(dt, X, y, 10, 2).nodes)
     yh = dt.dt_predict(t, Xd)
     m = dt.dt_eval_sharded(comm, yd, yh, 16)
     ref = dt.dt_eval(yd, yh, 16)
