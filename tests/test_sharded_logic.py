@@ -1,14 +1,20 @@
-"""Feature-sharded CART decomposition across REAL process boundaries (gloo, world 2, CPU).
+"""Value-range row-sharded CART across REAL process boundaries (gloo, world 2, CPU): the
+host-side logic of dt_fit_sharded without a GPU.
 
-Each rank searches only its features (global feature j*world + rank) with exact
-rationals (oracle/exact.py), the ranks all_gather their per-node bests, and every rank
-reduces them in the fixed order of the library's decide step (highest gain, then lowest
-global feature; positions within a feature are already lowest-first).  The resulting
-tree must equal the exact greedy tree on every rank -- the host-side logic of
-dt_fit_sharded (Multi-GPU), without a GPU.
+Each rank holds a contiguous block of rows.  The presort: a local sort by the 64-bit key
+(flip(x) << 32 | row id), exact splitters by 64 bisection rounds on the ranks' summed
+counts, an all-to-all of the entries; rank p must then hold exactly the global sorted
+positions [p n / P, (p + 1) n / P) of every feature list.  The levels: per (node, feature)
+each rank all_gathers its boundary record (count, sum of y, last x) and forms its rank
+carries (entries, S' and neighbour x of the lower ranks), scores its own positions with
+exact rationals (oracle/exact.py definitions), the ranks all_gather their per-node bests
+and reduce them in the library's fixed order (highest gain, then lowest feature, then
+lowest position), OR together the go-left rows of their split-feature parts and partition
+their lists stably.  The resulting tree must equal the exact greedy tree on every rank.
 """
 import os
 import socket
+from fractions import Fraction
 
 import numpy as np
 import pytest
@@ -26,45 +32,105 @@ def _free_port():
     return p
 
 
-def _sharded_tree(X, y, rank, world, max_depth, min_leaf):
-    from fractions import Fraction
+def _flip(x):
+    u = int(np.float32(x).view(np.uint32))
+    if (u << 1) & 0xFFFFFFFF == 0:
+        u = 0  # -0.0 == +0.0
+    return (~u) & 0xFFFFFFFF if u & 0x80000000 else u | 0x80000000
 
-    from oracle import exact
-    yy = [Fraction(int(v)) for v in y]
+
+def _gather(obj, world):
+    lst = [None] * world
+    dist.all_gather_object(lst, obj)
+    return lst
+
+
+def _value_range_presort(X, rank, world):
+    """Per feature: this rank's sorted (key, row) entries after the exchange."""
     n, d = X.shape
-    mine = [f for f in range(d) if f % world == rank]
-    nodes, queue, head = [None], [(list(range(n)), 0, 0)], 0
+    lo, hi = rank * n // world, (rank + 1) * n // world
+    local = [sorted((_flip(X[r, f]) << 32 | r) for r in range(lo, hi)) for f in range(d)]
+    # splitters: max composite K with global count(< K) <= t_b, t_b = b n / world
+    bounds = [[0, (1 << 64) - 1] for _ in range(d * (world - 1))]
+    for _ in range(64):
+        mids = [(a + (b - a) // 2) for a, b in bounds]
+        cnt = [sum(1 for v in local[i // (world - 1)] if v < mids[i]) for i in range(len(mids))]
+        tot = [sum(c) for c in zip(*_gather(cnt, world))]
+        for i, (a, b) in enumerate(bounds):
+            if b - a > 1:
+                t = (i % (world - 1) + 1) * n // world
+                bounds[i] = [mids[i], b] if tot[i] <= t else [a, mids[i]]
+    cuts = [[0] + [bounds[f * (world - 1) + q][0] for q in range(world - 1)] + [1 << 64] for f in range(d)]
+    send = [[[v for v in local[f] if cuts[f][q] <= v < cuts[f][q + 1]] for f in range(d)] for q in range(world)]
+    got = _gather(send, world)  # got[src][dst][f]
+    mine = [sorted(v for src in range(world) for v in got[src][rank][f]) for f in range(d)]
+    return [[(v >> 32, v & 0xFFFFFFFF) for v in lst] for lst in mine]
+
+
+def _sharded_tree(X, y, rank, world, max_depth, min_leaf):
+    n, d = X.shape
+    yy = [Fraction(int(v)) for v in y]
+    lists = _value_range_presort(X, rank, world)
+    # the exchange must leave rank p with global sorted positions [p n / P, (p+1) n / P)
+    for f in range(d):
+        glob = sorted(range(n), key=lambda r: (_flip(X[r, f]), r))
+        assert [r for _, r in lists[f]] == glob[rank * n // world:(rank + 1) * n // world]
+    segs = {0: [[r for _, r in lists[f]] for f in range(d)]}  # node -> per-feature local rows (sorted)
+    nodes, queue, head = [None], [(0, 0, n)], 0
     while head < len(queue):
-        rows, depth, idx = queue[head]
+        idx, depth, N = queue[head]
         head += 1
-        ys = [yy[r] for r in rows]
-        nd = dict(feature=-1, left=-1, threshold=0.0, n=len(rows), depth=depth)
+        nd = dict(feature=-1, left=-1, threshold=0.0, n=N)
         nodes[idx] = nd
-        searchable = (max_depth < 0 or depth < max_depth) and len(rows) >= 2 * min_leaf and min(ys) != max(ys)
+        seg = segs.pop(idx)
+        ys0 = [yy[r] for r in seg[0]]
+        mm = _gather((min(ys0) if ys0 else None, max(ys0) if ys0 else None), world)
+        lo_y = min(a for a, _ in mm if a is not None)
+        hi_y = max(b for _, b in mm if b is not None)
+        searchable = (max_depth < 0 or depth < max_depth) and N >= 2 * min_leaf and lo_y != hi_y
         best = None
         if searchable:
-            for f, i, gain, thr, L, R in exact.candidates(X[:, mine], yy, rows, min_leaf):
-                if best is None or gain > best[0]:
-                    best = (gain, mine[f], thr, L, R)
-        recs = [None] * world
-        dist.all_gather_object(recs, None if best is None else (str(best[0]), best[1], best[2]))
+            recs = _gather([(len(seg[f]), sum((yy[r] for r in seg[f]), Fraction(0)),
+                             float(X[seg[f][-1], f]) if seg[f] else None) for f in range(d)], world)
+            tot = [sum((recs[q][f][1] for q in range(world)), Fraction(0)) for f in range(d)]
+            for f in range(d):
+                ioff = sum(recs[q][f][0] for q in range(rank))
+                soff = sum((recs[q][f][1] for q in range(rank)), Fraction(0))
+                xprev = None
+                for q in range(rank):
+                    if recs[q][f][0]:
+                        xprev = recs[q][f][2]
+                S = soff
+                for t, r in enumerate(seg[f]):
+                    i, x = ioff + t, float(X[r, f])
+                    if i >= max(min_leaf, 1) and N - i >= min_leaf and xprev is not None and np.float32(xprev) < np.float32(x):
+                        nl, nr = i, N - i
+                        gain = (S * nr - (tot[f] - S) * nl) ** 2 / (N * nl * nr)  # = SSE_P - SSE_L - SSE_R
+                        if best is None or gain > best[0]:  # strict >: lowest position per feature
+                            best = (gain, f, i, float(xprev) / 2.0 + x / 2.0)
+                    S += yy[r]
+                    xprev = x
+        bests = _gather(None if best is None else (str(best[0]), best[1], best[2], best[3]), world)
         win = None
-        for r in recs:  # fixed order: highest gain, then lowest global feature
-            if r is None:
+        for b in bests:  # rank order: highest gain, then lowest feature, then lowest position
+            if b is None:
                 continue
-            g = Fraction(r[0])
-            if win is None or g > win[0] or (g == win[0] and r[1] < win[1]):
-                win = (g, r[1], r[2])
+            g = Fraction(b[0])
+            if win is None or g > win[0] or (g == win[0] and (b[1] < win[1] or (b[1] == win[1] and b[2] < win[2]))):
+                win = (g, b[1], b[2], b[3])
         if not searchable or win is None:
             continue
-        f, thr = win[1], win[2]
-        L = [r for r in rows if float(X[r, f]) <= thr]
-        R = [r for r in rows if float(X[r, f]) > thr]
+        f, i, thr = win[1], win[2], win[3]
+        ioff = sum(c for c in _gather(len(seg[f]), world)[:rank])
+        left_mine = {r for t, r in enumerate(seg[f]) if ioff + t < i}
+        left = set().union(*_gather(left_mine, world))  # the OR-allreduce of the go-left bitmap
         li = len(nodes)
         nodes.extend([None, None])
         nd.update(feature=f, left=li, threshold=thr)
-        queue.append((L, depth + 1, li))
-        queue.append((R, depth + 1, li + 1))
+        segs[li] = [[r for r in seg[g] if r in left] for g in range(d)]
+        segs[li + 1] = [[r for r in seg[g] if r not in left] for g in range(d)]
+        queue.append((li, depth + 1, i))
+        queue.append((li + 1, depth + 1, N - i))
     return [(nd["feature"], nd["left"], nd["threshold"], nd["n"]) for nd in nodes]
 
 
@@ -76,7 +142,7 @@ def _worker(rank, world, port, q):
     from oracle import exact
     ok = True
     for seed in range(6):
-        X, y = datagen.random_table(seed, 24, 5, kind=("ties", "collinear", "mixed")[seed % 3],
+        X, y = datagen.random_table(seed, 24, 3, kind=("ties", "collinear", "mixed")[seed % 3],
                                     int_y=True, y_range=6)
         for D, m in ((-1, 1), (2, 2)):
             got = _sharded_tree(X, y, rank, world, D, m)
@@ -87,7 +153,7 @@ def _worker(rank, world, port, q):
     dist.destroy_process_group()
 
 
-def test_feature_sharded_decomposition_gloo():
+def test_value_range_sharded_decomposition_gloo():
     world = 2
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -95,7 +161,7 @@ def test_feature_sharded_decomposition_gloo():
     procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
     for p in procs:
         p.start()
-    res = [q.get(timeout=300) for _ in range(world)]
+    res = [q.get(timeout=600) for _ in range(world)]
     for p in procs:
         p.join(timeout=60)
     assert sorted(r for r, _ in res) == [0, 1]
