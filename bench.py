@@ -7,8 +7,11 @@ max_depth 12, min_samples_leaf 1; one step = dt_fit on the training table + fuse
 dt_predict_eval on a 1M-row held-out table (seed 2).  value = split evals / step time
 (split evals = sum over searched nodes of N*d).  Inputs are resident in HBM; L2 is
 flushed (256 MB write) between timed steps, outside the per-step CUDA events.
-N>1 (torchrun): every rank fits its own replica table (seed 1 + rank): "replicas only",
-weak scaling, no data-path collective (Multi-GPU); max over ranks.
+N>1 (torchrun, or --gpus N, which re-launches itself through torch.distributed.run): the
+headline is BASELINE configs[2] -- ONE 100M x 32 (S32, seed 3), depth-16 fit row-sharded
+over the N ranks (dt_fit_sharded over NCCL: value-range presort, per-level allgathers of
+node bests and boundary records, OR-allreduce of the go-left bitmap), strong scaling,
+device-timed, max over ranks; independent configs[1] replicas are an extra key.
 
 Also reported: e2e (same metric through the C-ABI with host buffers, H2D/D2H inside the
 timed region), DSE predictions/s (BASELINE configs[3] shape on one GPU: 2^28 materialised
@@ -29,6 +32,8 @@ import statistics
 import sys
 import threading
 import time
+
+import numpy as np
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
@@ -62,6 +67,8 @@ def parse():
     p.add_argument("--grid-rows", type=int, default=10_000_000, help="configs[4] rows (0 = skip)")
     p.add_argument("--c3-rows", type=int, default=100_000_000,
                    help="configs[2] rows (x 32 features, depth 16; 0 = skip)")
+    p.add_argument("--force-sharded", action="store_true",
+                   help="run the N>1 headline (row-sharded configs[2] over NCCL) even with one rank")
     p.add_argument("--sharded-local", type=int, default=0,
                    help="N=1 only: also time a feature-sharded fit with this many thread ranks on the GPU")
     return p.parse_args()
@@ -136,6 +143,11 @@ def dist_init():
         import torch.distributed as dist
         torch.cuda.set_device(local)
         dist.init_process_group("nccl")
+    elif "--force-sharded" in sys.argv:  # one-rank process group for the NCCL id broadcast
+        import torch.distributed as dist
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29511")
+        dist.init_process_group("gloo", rank=0, world_size=1)
     return world, rank, local
 
 
@@ -254,59 +266,48 @@ def run_reference(args, world, rank):
 
 # ---------------------------------------------------------------------- ours (GPU) ----
 
-def sharded_fit_measure(args, world, rank, dev, X, y, stream):
-    """dt_fit_sharded of the configs[1] table (the same table on every rank) split by
-    features over the ranks: strong scaling of ONE fit.  With --sharded-local P on a single
-    process, P host-thread ranks share this GPU (functional check of the sharded path)."""
+def sharded_fit_measure(args, rank, dev, X, y, stream):
+    """--sharded-local P (N=1): the configs[1] table row-sharded over P host-thread ranks
+    sharing this GPU (dt_comm_init_local): a functional check of the sharded path, timed
+    by the host clock (the ranks share one GPU, so this is no scaling number)."""
     import threading
 
     import torch
 
     import paper_conf_ipps_metzgd23_b200 as dt
-    # the SAME table on every rank (the replicas of the headline use seed 1 + rank)
-    Xs, ys = dt.dt_gen_table(1, N_TRAIN, d=D, device=dev) if world > 1 else (X, y)
-    if world > 1:
-        import torch.distributed as dist
-
-        def bcast(obj):
-            lst = [obj]
-            dist.broadcast_object_list(lst, src=0)
-            return lst[0]
-        comms = [dt.dt_comm_init_nccl(rank, world, bcast)]
-    else:
-        comms = dt.dt_comm_init_local(args.sharded_local)
+    P = args.sharded_local
+    comms = dt.dt_comm_init_local(P)
+    n = X.shape[0]
+    cuts = [(r * n) // P for r in range(P + 1)]
     steps = max(3, min(args.steps, 10))
 
     def one_round():
-        trees = [None] * len(comms)
+        trees = [None] * P
 
         def run(i):
-            s = torch.cuda.Stream() if len(comms) > 1 else stream
+            s = torch.cuda.Stream()
             with torch.cuda.stream(s):
-                trees[i] = dt.dt_fit_sharded(comms[i], Xs, ys, MAX_DEPTH, MIN_LEAF, stream=s)
-        th = [threading.Thread(target=run, args=(i,)) for i in range(len(comms))]
+                a, b = cuts[i], cuts[i + 1]
+                trees[i] = dt.dt_fit_sharded(comms[i], X[a:b], y[a:b], a, n, MAX_DEPTH, MIN_LEAF, stream=s)
+        th = [threading.Thread(target=run, args=(i,)) for i in range(P)]
         for t in th:
             t.start()
         for t in th:
             t.join()
         return trees
 
-    for _ in range(2):
-        one_round()
-    barrier(world)
+    one_round()
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     for _ in range(steps):
         trees = one_round()
     torch.cuda.synchronize()
-    dt_s = max_over_ranks(time.perf_counter() - t0, world)
-    ref = dt.dt_fit(Xs, ys, MAX_DEPTH, MIN_LEAF)
-    same = all(t.nodes.tobytes() == ref.nodes.tobytes() for t in trees)
-    evals = trees[0].split_evals
-    return {"ranks": world if world > 1 else args.sharded_local,
-            "backend": "nccl" if world > 1 else "local-threads (one GPU)",
-            "split_evals_per_s": evals * steps / dt_s, "ms_per_fit": dt_s / steps * 1e3,
-            "identical_to_dt_fit": bool(same), "timing": "host wall clock around synchronised fits, max over ranks"}
+    dt_s = time.perf_counter() - t0
+    ref = dt.dt_fit(X, y, MAX_DEPTH, MIN_LEAF).nodes
+    same = all(np.array_equal(t.nodes[k], ref[k]) for t in trees
+               for k in ("feature", "left", "threshold", "value", "n_samples"))
+    return {"ranks": P, "backend": "local-threads (one GPU)", "ms_per_fit": dt_s / steps * 1e3,
+            "identical_to_dt_fit": bool(same), "timing": "host wall clock around synchronised fits"}
 
 
 def extra_configs(args, dev, stream, rank=0, world=1):
@@ -378,9 +379,8 @@ def extra_configs(args, dev, stream, rank=0, world=1):
 def c3_measure(args, world, rank, dev, stream):
     """BASELINE configs[2]: 100M x 32 (S32, seed 3), max_depth 16, min_samples_leaf 1.
     N=1: dt_fit on one B200 (~110 GB of HBM: the level lists, double-buffered, hold the
-    presort buffers).  N>1: dt_fit_sharded over NCCL, features split over the ranks (every
-    rank holds the whole table; strong scaling of one fit).  Device-timed with CUDA events
-    on the fit's stream, max over ranks; the first fit (planning + graph capture) is
+    presort buffers) -- the strong-scaling reference of the N>1 headline.  Device-timed
+    with CUDA events on the fit's stream; the first fit (planning + graph capture) is
     untimed.  One extra profiled fit splits presort / levels."""
     import torch
 
@@ -389,20 +389,8 @@ def c3_measure(args, world, rank, dev, stream):
     dt.dt_release_workspace()
     torch.cuda.empty_cache()
     X, y = dt.dt_gen_table(3, n, d=d, cnn_pool_bits=22, gpu_pool_bits=12, device=dev)
-    comm = None
-    if world > 1:
-        import torch.distributed as dist
-
-        def bcast(obj):
-            lst = [obj]
-            dist.broadcast_object_list(lst, src=0)
-            return lst[0]
-        comm = dt.dt_comm_init_nccl(rank, world, bcast)
-
     def fit():
-        if comm is None:
-            return dt.dt_fit(X, y, depth, 1)
-        return dt.dt_fit_sharded(comm, X, y, depth, 1, stream=stream)
+        return dt.dt_fit(X, y, depth, 1)
     tree = fit()
     reps = 3
     a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -428,7 +416,7 @@ def c3_measure(args, world, rank, dev, stream):
     presort = sum(v["ms"] for k, v in prof.items() if k.startswith("presort"))
     levels = sum(v["ms"] for k, v in prof.items() if not k.startswith("presort"))
     return {"workload": f"configs[2]: {n} x {d} (S32, seed 3, pools 2^22 x 2^12), max_depth {depth}, min_samples_leaf 1",
-            "mode": "dt_fit (1 GPU)" if world == 1 else f"dt_fit_sharded over NCCL ({world} ranks, features split)",
+            "mode": "dt_fit (1 GPU)",
             "ms_per_fit": t * 1e3, "split_evals_per_fit": tree.split_evals,
             "split_evals_per_s": tree.split_evals / t, "tree_nodes": tree.size, "tree_depth": tree.depth,
             "profiled_fit_ms": {"presort": presort, "levels": levels},
@@ -635,9 +623,9 @@ def run_ours(args, world, rank, local):
 
     # ---- feature-sharded fit across the N ranks (NCCL): one C2 fit split by features
     sharded = None
-    if world > 1 or args.sharded_local > 1:
+    if world == 1 and args.sharded_local > 1:
         try:
-            sharded = sharded_fit_measure(args, world, rank, dev, X, y, stream)
+            sharded = sharded_fit_measure(args, rank, dev, X, y, stream)
         except Exception as e:  # never let the extra measurement kill the headline
             sharded = {"error": f"{type(e).__name__}: {e}"}
 
@@ -754,11 +742,122 @@ def run_ours(args, world, rank, local):
         print(json.dumps(line), flush=True)
 
 
+def run_sharded(args, world, rank, local):
+    """N>1 headline: BASELINE configs[2] (100M x 32, S32 seed 3, depth 16, m 1) as ONE fit
+    row-sharded over the ranks (dt_fit_sharded over NCCL); rank r generates and holds rows
+    [r n / N, (r + 1) n / N).  Strong scaling: value = the fit's split evals / the max over
+    ranks of the device time per fit.  e2e: the same fit with the rank's rows copied from
+    pinned host memory every step (H2D inside the timed region) and the tree read back."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_metzgd23_b200 as dt
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    stream = torch.cuda.current_stream()
+    n, d, depth = args.c3_rows if args.c3_rows > 0 else 100_000_000, 32, 16
+    lo, hi = rank * n // world, (rank + 1) * n // world
+    X, y = dt.dt_gen_table(3, hi - lo, d=d, row0=lo, cnn_pool_bits=22, gpu_pool_bits=12, device=dev)
+
+    def bcast(obj):
+        lst = [obj]
+        dist.broadcast_object_list(lst, src=0)
+        return lst[0]
+    comm = dt.dt_comm_init_nccl(rank, world, bcast)
+
+    def fit(Xl, yl):
+        return dt.dt_fit_sharded(comm, Xl, yl, lo, n, depth, 1, stream=stream)
+
+    for _ in range(max(1, args.warmup)):
+        tree = fit(X, y)
+    steps = max(1, args.steps)
+    ev0 = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+    ev1 = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+    launches0 = dt.dt_launch_count()
+    with ClockSampler(local) as clk:
+        barrier(world)
+        torch.cuda.synchronize()
+        for i in range(steps):
+            ev0[i].record(stream)
+            tree = fit(X, y)
+            ev1[i].record(stream)
+        torch.cuda.synchronize()
+        barrier(world)
+    launches = dt.dt_launch_count() - launches0
+    t_total = sum(a.elapsed_time(b) for a, b in zip(ev0, ev1)) / 1e3
+    t_max = max_over_ranks(t_total, world)
+    evals = tree.split_evals  # the global tree's split evals (same on every rank)
+    value = evals * steps / t_max
+    # e2e: host rows -> device every step, the tree back to the host
+    Xh, yh = X.cpu().pin_memory(), y.cpu().pin_memory()
+    Xd, yd = torch.empty_like(X), torch.empty_like(y)
+    e_steps = max(1, min(args.e2e_steps, steps))
+    barrier(world)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(e_steps):
+        Xd.copy_(Xh, non_blocking=True)
+        yd.copy_(yh, non_blocking=True)
+        tr = fit(Xd, yd)
+    torch.cuda.synchronize()
+    e2e_t = max_over_ranks(time.perf_counter() - t0, world)
+    # per-kernel roofline of this rank's fused pass (one profiled fit)
+    peak, peak_src = peaks()
+    dt.dt_profile_reset()
+    dt.dt_profile_enable(True)
+    fit(X, y)
+    dt.dt_profile_enable(False)
+    prof = dt.dt_profile()
+    roof = None
+    fk = {k: v for k, v in prof.items() if v["alg_bytes"] > 0}
+    if fk:
+        dom = max(fk, key=lambda k: fk[k]["ms"])
+        ach = fk[dom]["alg_bytes"] / (fk[dom]["ms"] / 1e3) / 1e9
+        roof = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
+                "peak_source": peak_src, "alg_bytes_per_launch": fk[dom]["alg_bytes"] / fk[dom]["launches"],
+                "avg_launch_ms": fk[dom]["ms"] / fk[dom]["launches"], "traffic": None,
+                "measured": "rank 0, one profiled sharded fit, per-launch CUDA events",
+                "by_kernel_ms_per_fit": {k: round(v["ms"], 3) for k, v in prof.items()}}
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "split evals/s", "n_gpus": world, "steps": steps,
+                "warmup": args.warmup, "ms_per_step": t_max / steps * 1e3, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": f"configs[2]: {n} x {d} (S32, seed 3, pools 2^22 x 2^12), max_depth {depth}, "
+                                       "min_samples_leaf 1; one fit row-sharded over the ranks",
+                           "n_train": n, "d": d, "max_depth": depth, "min_samples_leaf": 1,
+                           "parallelism": f"rowshard{world}", "ranks": world,
+                           "l2": "inputs (12.8 GB of X) larger than L2"},
+                "e2e": {"value": evals * e_steps / e2e_t, "unit": "split evals/s",
+                        "h2d_bytes_per_step": (hi - lo) * (4 * d + 8) * world, "d2h_bytes_per_step": tr.size * 48,
+                        "steps": e_steps},
+                "gpu_launches": launches, "roofline": roof, "cpu_baseline": None,
+                "fit": {"split_evals_per_fit": evals, "tree_nodes": tree.size, "tree_depth": tree.depth},
+                "clocks": clk.summary()}
+        print(json.dumps(line), flush=True)
+
+
+def relaunch(args):
+    """--gpus N without a torchrun environment: re-run this script under
+    torch.distributed.run with N processes on this node (127.0.0.1 rendezvous)."""
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    os.execv(sys.executable, cmd)
+
+
 def main():
     args = parse()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        relaunch(args)
     world, rank, local = dist_init()
     if args.impl == "reference":
         run_reference(args, world, rank)
+    elif world > 1 or args.force_sharded:
+        run_sharded(args, world, rank, local)
     else:
         run_ours(args, world, rank, local)
     if world > 1:
