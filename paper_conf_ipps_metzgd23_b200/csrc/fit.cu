@@ -26,9 +26,19 @@
 #include <mutex>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "fit_core.cuh"
 
 namespace dtl {
+
+namespace {
+// NVTX ranges (presort, every level) for nsys / ncu --nvtx; no-ops without a tool attached
+struct Nvtx {
+  explicit Nvtx(const char* name) { nvtxRangePushA(name); }
+  ~Nvtx() { nvtxRangePop(); }
+};
+}  // namespace
 
 namespace {
 
@@ -905,7 +915,11 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
   DT_CK(cudaMemsetAsync(b.head_cand, 0xFF, sizeof(Cand2) * (size_t)b.segcap, s));
   DT_CK(cudaMemsetAsync(b.cont_cand, 0xFF, sizeof(Cand2) * (size_t)(2 * b.max_chunks), s));
   DT_CK(cudaMemsetAsync(b.ctl, 0, sizeof(Ctl), s));
-  dt_status st = presort_enqueue(b, X, y, n, d, d, 0, max_depth, min_leaf, s);
+  dt_status st;
+  {
+    Nvtx range("dt presort");
+    st = presort_enqueue(b, X, y, n, d, d, 0, max_depth, min_leaf, s);
+  }
   if (st != DT_OK) return st;
   Ctl* ctl = b.ctl;
   // the virtual-root pass: the root's candidates and statistics
@@ -926,6 +940,9 @@ dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t
   const int g_gl = grid_of((const void*)goleft_kernel, 256, 0);
   const int g_tab = num_sms() * 4;
   for (int level = 0;; ++level) {
+    char nv[32];
+    snprintf(nv, sizeof nv, "dt level %d", level);
+    Nvtx range(nv);
     const int par = level & 1;
     const int cur = par;  // level l lists: buffer l & 1 (the virtual-root pass writes nothing)
     // ---- piece positions + select (a5, a8)
@@ -1117,16 +1134,23 @@ dt_status release_workspace_impl() {
   return DT_OK;
 }
 
+// Keep freed stream-ordered workspace in the device's default pool for the next call (no
+// cudaMalloc on the hot path); dt_release_workspace trims it.
+dt_status keep_pool(int dev) {
+  cudaMemPool_t pool;
+  DT_CK(cudaDeviceGetDefaultMemPool(&pool, dev));
+  uint64_t thr = UINT64_MAX;
+  DT_CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+  return DT_OK;
+}
+
 dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
                    int64_t min_leaf, cudaStream_t s, dt_tree** out) {
-  // Pool: keep freed workspace for the next fit (no cudaMalloc on the hot path).
   int dev = 0;
   DT_CK(cudaGetDevice(&dev));
   {
-    cudaMemPool_t pool;
-    DT_CK(cudaDeviceGetDefaultMemPool(&pool, dev));
-    uint64_t thr = UINT64_MAX;
-    DT_CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+    dt_status ps = keep_pool(dev);
+    if (ps != DT_OK) return ps;
   }
   static int graph_env = -1;
   if (graph_env < 0) {
@@ -1240,6 +1264,10 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
   const int P = comm_world(comm), rank = comm_rank(comm);
   int dev = 0;
   DT_CK(cudaGetDevice(&dev));
+  {
+    dt_status ps = keep_pool(dev);
+    if (ps != DT_OK) return ps;
+  }
   const int64_t nlist = std::max<int64_t>(std::max<int64_t>(n_local, (n_global + P - 1) / P), 1);
   Workspace ws;
   ws.s = s;
@@ -1253,7 +1281,10 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
   DT_CK(cudaMemsetAsync(b.head_cand, 0xFF, sizeof(Cand2) * (size_t)b.segcap, s));
   DT_CK(cudaMemsetAsync(b.cont_cand, 0xFF, sizeof(Cand2) * (size_t)(2 * b.max_chunks), s));
   DT_CK(cudaMemsetAsync(b.ctl, 0, sizeof(Ctl), s));
-  st = presort_sharded_enqueue(b, comm, X, y, n_local, row_offset, n_global, d, max_depth, min_leaf, s);
+  {
+    Nvtx range("dt sharded presort");
+    st = presort_sharded_enqueue(b, comm, X, y, n_local, row_offset, n_global, d, max_depth, min_leaf, s);
+  }
   if (st != DT_OK) return st;
   Ctl* ctl = b.ctl;
   {  // the virtual-root pass (the root's rank carries come from the presort)
@@ -1272,6 +1303,9 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
   const int g_tab = num_sms() * 4;
   uint32_t K = 1;  // nodes at the level (host copy)
   for (int level = 0;; ++level) {
+    char nv[32];
+    snprintf(nv, sizeof nv, "dt sharded level %d", level);
+    Nvtx range(nv);
     const int par = level & 1, cur = par;
     SelectArgs se;
     se.gbits = reinterpret_cast<uint4*>(b.gbits);
