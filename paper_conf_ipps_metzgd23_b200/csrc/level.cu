@@ -715,8 +715,8 @@ struct Side {
   double S, sc, Nd, jd;         // prefix (rank carry included), S' of the child, N, position (f64)
   uint32_t jl, lo, hi;          // local position, valid local range [lo, hi)
   float xp;                     // x of the previous entry of this child
-  double bg, bs;                // best gain (approximate pass: approximate), its S'_L
-  uint32_t bj;                  // best global position
+  double bg, bs, bjd;           // best gain (approximate pass: approximate), its S'_L, position
+  uint32_t bj;                  // best global position (after finish / the exact pass)
   float bxp, bx;
   __device__ __forceinline__ void init(const PSeg& ps, int side, uint32_t ilo, uint32_t m, bool srch, double S0,
                                        float x0, uint32_t j0) {
@@ -730,6 +730,7 @@ struct Side {
     xp = x0;
     bg = -1.0;
     bs = 0.0;
+    bjd = 0.0;
     bj = 0xffffffffu;
     bxp = bx = 0.f;
   }
@@ -745,7 +746,7 @@ struct Side {
         amb = bg >= __dmul_rn(ga, 1.0 - kTol);
         bg = ga;
         bs = S;
-        bj = (uint32_t)jd;
+        bjd = jd;
         bxp = xp;
         bx = x;
       } else {
@@ -764,7 +765,7 @@ struct Side {
       if (g > bg) {  // strict >: the lowest position wins exact ties
         bg = g;
         bs = S;
-        bj = (uint32_t)jd;
+        bjd = jd;
         bxp = xp;
         bx = x;
       }
@@ -775,7 +776,8 @@ struct Side {
     xp = x;
   }
   __device__ __forceinline__ void finish() {  // the exact gain of the approximate winner
-    if (bg >= 0.0) bg = split_gain_d(bs, sc, (double)bj, Nd);
+    if (bg >= 0.0) bg = split_gain_d(bs, sc, bjd, Nd);
+    bj = (uint32_t)bjd;
   }
 };
 
@@ -986,32 +988,29 @@ __global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArg
     if (full && (flags & (PS_SRCH0 | PS_SRCH1))) {
       // right position of my first in-range item: its segment-local index - lefts before
       const uint32_t jr0 = ib + (uint32_t)max(lane * kItems, e_lo) - nl;
-      Side sd[2];
-      sd[0].init(ps, 0, ilo, m, (flags & PS_SRCH0) != 0, SL, xl, nl);
-      sd[1].init(ps, 1, ilo, m, (flags & PS_SRCH1) != 0, SR, xr, jr0);
-      bool amb = false;
-#pragma unroll
-      for (int j = 0; j < kItems; ++j) {
-        if ((lbyte >> j) & 1u) amb |= sd[0].step(xv[j], dv[j]);
-        if ((rbyte >> j) & 1u) amb |= sd[1].step(xv[j], dv[j]);
-      }
-      if (__any_sync(0xffffffffu, amb)) {
-        // a near tie of approximate gains in some lane: exact gains at every position
-        sd[0].init(ps, 0, ilo, m, (flags & PS_SRCH0) != 0, SL, xl, nl);
-        sd[1].init(ps, 1, ilo, m, (flags & PS_SRCH1) != 0, SR, xr, jr0);
-#pragma unroll
-        for (int j = 0; j < kItems; ++j) {
-          if ((lbyte >> j) & 1u) sd[0].step_exact(xv[j], dv[j]);
-          if ((rbyte >> j) & 1u) sd[1].step_exact(xv[j], dv[j]);
-        }
-      } else {
-        sd[0].finish();
-        sd[1].finish();
-      }
-#pragma unroll
+      // the two children one after the other (one running state live: registers)
+#pragma unroll 1
       for (int side = 0; side < 2; ++side) {
-        const double bg = sd[side].bg;
-        const uint32_t bj = sd[side].bj;
+        if (!(flags & (side ? PS_SRCH1 : PS_SRCH0))) continue;  // warp-uniform
+        const uint32_t sb = side ? rbyte : lbyte;
+        Side sd;
+        sd.init(ps, side, ilo, m, true, side ? SR : SL, side ? xr : xl, side ? jr0 : nl);
+        bool amb = false;
+#pragma unroll
+        for (int j = 0; j < kItems; ++j)
+          if ((sb >> j) & 1u) amb |= sd.step(xv[j], dv[j]);
+        if (__any_sync(0xffffffffu, amb)) {
+          // a near tie of approximate gains in some lane: exact gains at every position
+          sd.init(ps, side, ilo, m, true, side ? SR : SL, side ? xr : xl, side ? jr0 : nl);
+#pragma unroll
+          for (int j = 0; j < kItems; ++j)
+            if ((sb >> j) & 1u) sd.step_exact(xv[j], dv[j]);
+          sd.bj = (uint32_t)sd.bjd;
+        } else {
+          sd.finish();
+        }
+        const double bg = sd.bg;
+        const uint32_t bj = sd.bj;
         // warp max of the exact gains (>= 0: the f64 bit patterns order like the values;
         // key 0 = no candidate), then the lowest position holding it
         const unsigned long long key = bg >= 0.0 ? (unsigned long long)__double_as_longlong(bg) + 1ull : 0ull;
@@ -1021,7 +1020,7 @@ __global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArg
         if (kmax != 0ull) {
           const uint32_t jmin = __reduce_min_sync(0xffffffffu, key == kmax ? bj : 0xffffffffu);
           if (key == kmax && bj == jmin)  // exactly one lane holds the winner
-            put_cand(a, headc, ch, side, ps.cs[side], bg, sd[side].bs, mid_threshold(sd[side].bxp, sd[side].bx), jmin);
+            put_cand(a, headc, ch, side, ps.cs[side], bg, sd.bs, mid_threshold(sd.bxp, sd.bx), jmin);
         }
       }
     }
