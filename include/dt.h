@@ -93,6 +93,16 @@ typedef struct {
 dt_status dt_fit(const float* X_dev, const double* y_dev, int64_t n, int32_t d,
                  int32_t max_depth, int64_t min_samples_leaf, void* stream, dt_tree** out);
 
+/* dt_fit_grid -- the trees of dt_fit(X, y, n, d, max_depth, m) for every m in
+ * min_samples_leafs[0 .. count) (BASELINE configs[4]'s (max_depth x min_samples_leaf)
+ * grid; the depths come from dt_tree_truncate / dt_predict_eval_depths): ONE presort of the
+ * table, then one level loop per m from a snapshot of the presorted lists (a greedy tree
+ * depends on m only through its leaf rules).  outs[i] receives tree i (owned by the
+ * caller; all NULL on error).  Needs ~16 B per (row, feature) beyond dt_fit's workspace.
+ * Sync.  Errors as dt_fit. */
+dt_status dt_fit_grid(const float* X_dev, const double* y_dev, int64_t n, int32_t d, int32_t max_depth,
+                      const int64_t* min_samples_leafs, int32_t count, void* stream, dt_tree** outs);
+
 /* Number of nodes; host view of the node array (valid until dt_tree_free). */
 int64_t dt_tree_size(const dt_tree* tree);
 const dt_node* dt_tree_nodes(const dt_tree* tree);

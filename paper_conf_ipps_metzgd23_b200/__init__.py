@@ -28,7 +28,7 @@ NODE_DTYPE = np.dtype([
 STATUS = {0: "DT_OK", 1: "DT_ERR_INVALID_ARG", 2: "DT_ERR_NONFINITE", 3: "DT_ERR_OOM",
           4: "DT_ERR_CUDA", 5: "DT_ERR_NCCL", 6: "DT_ERR_TOO_LARGE"}
 
-SYMBOLS = ("dt_fit", "dt_tree_size", "dt_tree_nodes", "dt_tree_depth", "dt_tree_num_features",
+SYMBOLS = ("dt_fit", "dt_fit_grid", "dt_tree_size", "dt_tree_nodes", "dt_tree_depth", "dt_tree_num_features",
            "dt_tree_split_evals", "dt_tree_from_nodes", "dt_tree_free", "dt_predict", "dt_eval",
            "dt_predict_eval", "dt_loo", "dt_gen_table", "dt_gen_dse", "dt_last_error",
            "dt_version", "dt_profile_enable", "dt_profile_reset", "dt_launch_count",
@@ -59,6 +59,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     P, I64, I32, U64, D = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, ctypes.c_double
     sig = {
         "dt_fit": ([P, P, I64, I32, I32, I64, P, ctypes.POINTER(P)], ctypes.c_int),
+        "dt_fit_grid": ([P, P, I64, I32, I32, P, I32, P, P], ctypes.c_int),
         "dt_tree_size": ([P], I64),
         "dt_tree_nodes": ([P], P),
         "dt_tree_depth": ([P], I32),
@@ -198,6 +199,19 @@ def dt_fit(X, y, max_depth: int = -1, min_samples_leaf: int = 1, stream=None) ->
     h = ctypes.c_void_p()
     _check(_lib.dt_fit(xp, yp, n, d, max_depth, min_samples_leaf, _stream(stream), ctypes.byref(h)))
     return Tree(h)
+
+
+def dt_fit_grid(X, y, max_depth: int, min_samples_leafs, stream=None):
+    """[dt_fit(X, y, max_depth, m) for m in min_samples_leafs] from ONE presort (include/dt.h)."""
+    import torch
+    xp = _dev(X, torch.float32, 2, "X")
+    yp = _dev(y, torch.float64, 1, "y")
+    n, d = X.shape
+    _same((X, y), ("y", y.shape[0], n))
+    ms = (ctypes.c_int64 * len(min_samples_leafs))(*[int(m) for m in min_samples_leafs])
+    hs = (ctypes.c_void_p * len(min_samples_leafs))()
+    _check(_lib.dt_fit_grid(xp, yp, n, d, max_depth, ms, len(min_samples_leafs), _stream(stream), hs))
+    return [Tree(ctypes.c_void_p(h)) for h in hs]
 
 
 def dt_tree_from_nodes(nodes: np.ndarray, d: int) -> Tree:
@@ -353,8 +367,8 @@ def dt_importances(tree: Tree, stream=None) -> np.ndarray:
 
 def grid_search(X, y, Xv, yv, depths, min_leafs, p=None, stream=None, rank=0, world=1, gather=None):
     """(max_depth x min_samples_leaf) grid with held-out evaluation (BASELINE configs[4]):
-    one dt_fit at max(depths) per m, then dt_predict_eval_depths -- every (D, m) tree is a
-    truncation of the deep one.  Returns {(D, m): (mape, r2, adj_r2)} and the split evals
+    dt_fit_grid (one presort, one deep fit at max(depths) per m), then
+    dt_predict_eval_depths -- every (D, m) tree is a truncation of the deep one.  Returns {(D, m): (mape, r2, adj_r2)} and the split evals
     actually performed.
 
     Multi-GPU ("LOO / grid"): with ``world`` ranks each fits the m values
@@ -364,8 +378,9 @@ def grid_search(X, y, Xv, yv, depths, min_leafs, p=None, stream=None, rank=0, wo
     p = X.shape[1] if p is None else p
     dmax = max(depths)
     out, evals = {}, 0
-    for m in list(min_leafs)[rank::world]:
-        t = dt_fit(X, y, dmax, m, stream=stream)
+    mine = list(min_leafs)[rank::world]
+    trees = dt_fit_grid(X, y, dmax, mine, stream=stream) if mine else []
+    for m, t in zip(mine, trees):
         evals += t.split_evals
         per = dt_predict_eval_depths(t, Xv, yv, p, stream=stream)
         for D in depths:

@@ -124,6 +124,27 @@ dt_status dt_fit_sharded(dt_comm* comm, const float* X_local_dev, const double* 
                           min_samples_leaf, S(stream), out);
 }
 
+dt_status dt_fit_grid(const float* X_dev, const double* y_dev, int64_t n, int32_t d, int32_t max_depth,
+                      const int64_t* min_samples_leafs, int32_t count, void* stream, dt_tree** outs) {
+  if (!outs || !min_samples_leafs || count < 1) return fail(DT_ERR_INVALID_ARG, "dt_fit_grid: need count >= 1 and arrays");
+  for (int32_t i = 0; i < count; ++i) outs[i] = nullptr;
+  if (!X_dev || !y_dev) return fail(DT_ERR_INVALID_ARG, "dt_fit_grid: NULL X or y");
+  if (n < 1) return fail(DT_ERR_INVALID_ARG, "dt_fit_grid: n must be >= 1");
+  if (n >= (int64_t)1 << 32) return fail(DT_ERR_TOO_LARGE, "dt_fit_grid: n must be < 2^32");
+  if (d < 1 || d > 255) return fail(DT_ERR_INVALID_ARG, "dt_fit_grid: d must be in [1, 255]");
+  if (max_depth < -1) return fail(DT_ERR_INVALID_ARG, "dt_fit_grid: max_depth must be >= -1");
+  for (int32_t i = 0; i < count; ++i)
+    if (min_samples_leafs[i] < 1) return fail(DT_ERR_INVALID_ARG, "dt_fit_grid: min_samples_leaf must be >= 1");
+  dt_status st = fit_grid_impl(X_dev, y_dev, n, d, max_depth, min_samples_leafs, count, S(stream), outs);
+  if (st != DT_OK) {
+    for (int32_t i = 0; i < count; ++i) {
+      dt_tree_free(outs[i]);
+      outs[i] = nullptr;
+    }
+  }
+  return st;
+}
+
 int64_t dt_tree_size(const dt_tree* t) { return t ? t->count : 0; }
 const dt_node* dt_tree_nodes(const dt_tree* t) { return t ? t->host : nullptr; }
 int32_t dt_tree_depth(const dt_tree* t) { return t ? t->depth : 0; }

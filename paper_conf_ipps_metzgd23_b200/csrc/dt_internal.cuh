@@ -50,6 +50,8 @@ dt_status release_workspace_impl();
 void forest_release_scratch();
 dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
                    int64_t min_leaf, cudaStream_t s, dt_tree** out);
+dt_status fit_grid_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
+                        const int64_t* min_leafs, int32_t count, cudaStream_t s, dt_tree** outs);
 dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64_t n_local, int64_t row_offset,
                            int64_t n_global, int32_t d, int32_t max_depth, int64_t min_leaf, cudaStream_t s,
                            dt_tree** out);

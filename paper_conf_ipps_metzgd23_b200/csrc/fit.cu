@@ -907,20 +907,35 @@ int grid_of(const void* kern, int threads, size_t smem) {
 }
 
 // Enqueues the whole fit on stream s (no host synchronisation unless `poll`).
-dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
-                      int64_t min_leaf, cudaStream_t s, bool poll, std::vector<Pending>* pending) {
+dt_status fit_levels(const FitBufs& b, int32_t d, int32_t max_depth, int64_t min_leaf, cudaStream_t s, bool poll,
+                     std::vector<Pending>* pending);
+
+dt_status clear_pieces(const FitBufs& b, cudaStream_t s) {
   DT_CK(cudaMemsetAsync(b.slot_gain, 0, sizeof(unsigned long long) * (size_t)b.segcap, s));
   DT_CK(cudaMemsetAsync(b.slot_pos, 0xFF, sizeof(unsigned long long) * (size_t)b.segcap, s));
   // candidate pieces carry the level that wrote them; none may match before it is written
   DT_CK(cudaMemsetAsync(b.head_cand, 0xFF, sizeof(Cand2) * (size_t)b.segcap, s));
   DT_CK(cudaMemsetAsync(b.cont_cand, 0xFF, sizeof(Cand2) * (size_t)(2 * b.max_chunks), s));
+  return DT_OK;
+}
+
+dt_status fit_enqueue(const FitBufs& b, const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
+                      int64_t min_leaf, cudaStream_t s, bool poll, std::vector<Pending>* pending) {
+  dt_status st = clear_pieces(b, s);
+  if (st != DT_OK) return st;
   DT_CK(cudaMemsetAsync(b.ctl, 0, sizeof(Ctl), s));
-  dt_status st;
   {
     Nvtx range("dt presort");
     st = presort_enqueue(b, X, y, n, d, d, 0, max_depth, min_leaf, s);
   }
   if (st != DT_OK) return st;
+  return fit_levels(b, d, max_depth, min_leaf, s, poll, pending);
+}
+
+// The virtual-root pass and the level loop, from the level-0 lists, root and tables.
+dt_status fit_levels(const FitBufs& b, int32_t d, int32_t max_depth, int64_t min_leaf, cudaStream_t s, bool poll,
+                     std::vector<Pending>* pending) {
+  dt_status st;
   Ctl* ctl = b.ctl;
   // the virtual-root pass: the root's candidates and statistics
   {
@@ -1258,6 +1273,98 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
 // rank order), OR-allreduce of the go-left bitmap, allgather of the children's boundary
 // records (count, last x, S') -> rank carries of every child segment.  Every rank builds
 // the same tree.  Direct enqueue; one host synchronisation per level (the node count).
+namespace {
+// The root's leaf rules and the virtual-root plan for another min_samples_leaf (the rest of
+// the presorted state is independent of it).
+__global__ void regrid_root_kernel(Ctl* ctl, NodeL* nodes0, PSeg* pseg, int d, int32_t max_depth, int64_t min_leaf) {
+  const int64_t n = nodes0[0].N;
+  const int srch = (max_depth != 0 && n >= 2 * min_leaf) ? 1 : 0;
+  for (int f = threadIdx.x; f < d; f += blockDim.x)
+    pseg[f].flags = PS_SPLIT | PS_ALLLEFT | (srch ? PS_SRCH0 : 0u);
+  if (threadIdx.x == 0) {
+    nodes0[0].searchable = srch;
+    ctl->nsrch = (uint32_t)srch;
+  }
+}
+}  // namespace
+
+// (max_depth x min_samples_leaf) grid, BASELINE configs[4]: ONE presort of the table, then
+// one level loop per min_samples_leaf from a snapshot of the level-0 lists and the root
+// (a greedy tree depends on m only through its leaf rules; the depths
+// come from truncation, dt_tree_truncate / dt_predict_eval_depths).
+dt_status fit_grid_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
+                        const int64_t* min_leafs, int32_t count, cudaStream_t s, dt_tree** outs) {
+  int dev = 0;
+  DT_CK(cudaGetDevice(&dev));
+  {
+    dt_status ps = keep_pool(dev);
+    if (ps != DT_OK) return ps;
+  }
+  int64_t mmin = min_leafs[0];
+  for (int i = 1; i < count; ++i) mmin = std::min(mmin, min_leafs[i]);
+  Workspace ws;
+  ws.s = s;
+  FitBufs b{};
+  auto get = [&](auto** p, size_t c) -> cudaError_t { return ws.get(p, c); };
+  dt_status st = fit_alloc(b, n, n, d, max_depth, mmin, 1, get);
+  if (st != DT_OK) return st;
+  const size_t tot = (size_t)n * d;
+  float* snx = nullptr;
+  uint32_t* snr = nullptr;
+  double* sny = nullptr;
+  Ctl* snc = nullptr;
+  NodeL* snn = nullptr;
+  SegT* sns = nullptr;
+  PSeg* snp = nullptr;
+  uint32_t* snd = nullptr;
+  const size_t nch0 = (tot + kChunkW - 1) / kChunkW;
+  st = alloc_status(ws.get(&sns, (size_t)d));
+  if (st == DT_OK) st = alloc_status(ws.get(&snp, (size_t)d));
+  if (st == DT_OK) st = alloc_status(ws.get(&snd, nch0));
+  if (st == DT_OK) st = alloc_status(ws.get(&snx, tot));
+  if (st == DT_OK) st = alloc_status(ws.get(&snr, tot));
+  if (st == DT_OK) st = alloc_status(ws.get(&sny, tot));
+  if (st == DT_OK) st = alloc_status(ws.get(&snc, 1));
+  if (st == DT_OK) st = alloc_status(ws.get(&snn, 1));
+  if (st != DT_OK) return st;
+  DT_CK(cudaMemsetAsync(b.ctl, 0, sizeof(Ctl), s));
+  {
+    Nvtx range("dt grid presort");
+    st = presort_enqueue(b, X, y, n, d, d, 0, max_depth, min_leafs[0], s);
+  }
+  if (st != DT_OK) return st;
+  DT_CK(cudaMemcpyAsync(snx, b.lx[0], sizeof(float) * tot, cudaMemcpyDeviceToDevice, s));
+  DT_CK(cudaMemcpyAsync(snr, b.lr[0], sizeof(uint32_t) * tot, cudaMemcpyDeviceToDevice, s));
+  DT_CK(cudaMemcpyAsync(sny, b.ly[0], sizeof(double) * tot, cudaMemcpyDeviceToDevice, s));
+  DT_CK(cudaMemcpyAsync(snc, b.ctl, sizeof(Ctl), cudaMemcpyDeviceToDevice, s));
+  DT_CK(cudaMemcpyAsync(snn, b.nodes[0], sizeof(NodeL), cudaMemcpyDeviceToDevice, s));
+  DT_CK(cudaMemcpyAsync(sns, b.segs[0], sizeof(SegT) * (size_t)d, cudaMemcpyDeviceToDevice, s));
+  DT_CK(cudaMemcpyAsync(snp, b.pseg, sizeof(PSeg) * (size_t)d, cudaMemcpyDeviceToDevice, s));
+  DT_CK(cudaMemcpyAsync(snd, b.desc[0], sizeof(uint32_t) * nch0, cudaMemcpyDeviceToDevice, s));
+  for (int i = 0; i < count; ++i) {
+    if (i > 0) {  // the presorted state again (the level loop consumed it)
+      DT_CK(cudaMemcpyAsync(b.lx[0], snx, sizeof(float) * tot, cudaMemcpyDeviceToDevice, s));
+      DT_CK(cudaMemcpyAsync(b.lr[0], snr, sizeof(uint32_t) * tot, cudaMemcpyDeviceToDevice, s));
+      DT_CK(cudaMemcpyAsync(b.ly[0], sny, sizeof(double) * tot, cudaMemcpyDeviceToDevice, s));
+      DT_CK(cudaMemcpyAsync(b.ctl, snc, sizeof(Ctl), cudaMemcpyDeviceToDevice, s));
+      DT_CK(cudaMemcpyAsync(b.nodes[0], snn, sizeof(NodeL), cudaMemcpyDeviceToDevice, s));
+      DT_CK(cudaMemcpyAsync(b.segs[0], sns, sizeof(SegT) * (size_t)d, cudaMemcpyDeviceToDevice, s));
+      DT_CK(cudaMemcpyAsync(b.pseg, snp, sizeof(PSeg) * (size_t)d, cudaMemcpyDeviceToDevice, s));
+      DT_CK(cudaMemcpyAsync(b.desc[0], snd, sizeof(uint32_t) * nch0, cudaMemcpyDeviceToDevice, s));
+      regrid_root_kernel<<<1, 256, 0, s>>>(b.ctl, b.nodes[0], b.pseg, d, max_depth, min_leafs[i]);
+      prof_add_launches(1);
+      DT_CK(cudaGetLastError());
+    }
+    st = clear_pieces(b, s);
+    if (st != DT_OK) return st;
+    st = fit_levels(b, d, max_depth, min_leafs[i], s, true, nullptr);
+    if (st != DT_OK) return st;
+    st = fit_finish(b, d, s, nullptr, &outs[i]);
+    if (st != DT_OK) return st;
+  }
+  return DT_OK;
+}
+
 dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64_t n_local, int64_t row_offset,
                            int64_t n_global, int32_t d, int32_t max_depth, int64_t min_leaf, cudaStream_t s,
                            dt_tree** out) {

@@ -417,6 +417,20 @@ def test_grid_search_matches_oracle(dt):
                 assert _close(a, b), (D, m, got, want)
 
 
+@pytest.mark.parametrize("real", [False, True])
+def test_fit_grid_equals_fits(dt, real):
+    """dt_fit_grid (one presort, one level loop per m from the presorted snapshot) returns
+    exactly dt_fit's tree for every min_samples_leaf, in any order of m."""
+    X, y = datagen.cnn_gpu_table(9, 30_000, real=real)
+    Xd, yd = _cuda(X), _cuda(y)
+    ms = [4, 1, 64, 2, 1024, 16]
+    trees = dt.dt_fit_grid(Xd, yd, 9, ms)
+    for m, t in zip(ms, trees):
+        assert t.nodes.tobytes() == dt.dt_fit(Xd, yd, 9, m).nodes.tobytes(), m
+    if not real:
+        _assert_exact(trees[1].nodes, oracle.fit(X, y, 9, 1))
+
+
 def test_importances_match_oracle(dt):
     X, y = datagen.cnn_gpu_table(6, 50000)
     t = _fit(dt, X, y, 12, 1)

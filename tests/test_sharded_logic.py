@@ -237,6 +237,7 @@ def _grid_worker(rank, world, port, q):
             self.split_evals, self.depth = 1000 + m, 5
 
     ns["dt_fit"] = lambda X, y, D, m, stream=None: FakeTree(m)
+    ns["dt_fit_grid"] = lambda X, y, D, ms, stream=None: [FakeTree(m) for m in ms]
     ns["dt_predict_eval_depths"] = lambda t, Xv, yv, p, stream=None: [
         (t.split_evals * 1e-3 + d, float(d), -float(d)) for d in range(t.depth + 1)]
     exec(body, ns)
