@@ -683,9 +683,10 @@ def run_ours(args, world, rank, local):
     knn = None
     if not args.no_extra:
         try:
-            ntr, nqk = 1 << 16, 1 << 20
+            ntr = 1 << 16
             Xtr, ytr = X[:ntr].contiguous(), y[:ntr].contiguous()
-            Xq = Xv[:nqk].contiguous()
+            Xq = Xv[:1 << 20].contiguous()
+            nqk = Xq.shape[0]  # the held-out rows (1M)
             outk = torch.empty(nqk, dtype=torch.float64, device=dev)
             dt.dt_knn_predict(Xtr, ytr, Xq[:4096], 5, out=outk[:4096])  # warm-up
             torch.cuda.synchronize()

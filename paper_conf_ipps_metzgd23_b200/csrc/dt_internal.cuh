@@ -4,6 +4,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <vector>
 
 #include "../../include/dt.h"
 
@@ -46,10 +47,10 @@ dt_status tree_upload(dt_tree* t, cudaStream_t s);
 
 // Fit driver (fit.cu).
 dt_status release_workspace_impl();
-// frees the forest's cached bootstrap scratch table (forest.cu); called by release_workspace_impl
-void forest_release_scratch();
 dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
                    int64_t min_leaf, cudaStream_t s, dt_tree** out);
+dt_status forest_trees_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t n_trees, int32_t max_depth,
+                            int64_t min_leaf, uint64_t seed, cudaStream_t s, std::vector<dt_tree*>& trees);
 dt_status fit_grid_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t max_depth,
                         const int64_t* min_leafs, int32_t count, cudaStream_t s, dt_tree** outs);
 dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64_t n_local, int64_t row_offset,

@@ -1139,7 +1139,6 @@ dt_status release_workspace_impl() {
     std::lock_guard<std::mutex> lk(g_plan_mu);
     for (auto& p : g_plans) p.reset();
   }
-  forest_release_scratch();
   DT_CK(cudaDeviceSynchronize());
   int dev = 0;
   DT_CK(cudaGetDevice(&dev));
@@ -1361,6 +1360,61 @@ dt_status fit_grid_impl(const float* X, const double* y, int64_t n, int32_t d, i
     if (st != DT_OK) return st;
     st = fit_finish(b, d, s, nullptr, &outs[i]);
     if (st != DT_OK) return st;
+  }
+  return DT_OK;
+}
+
+// Random Forest: ONE presort of the table; tree t = the exact CART of
+// its bootstrap sample, whose level-0 lists are the presorted lists expanded by the draw
+// counts (presort.cu, forest_tree_enqueue) -- no gather, no sort per tree.
+dt_status forest_trees_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t n_trees, int32_t max_depth,
+                            int64_t min_leaf, uint64_t seed, cudaStream_t s, std::vector<dt_tree*>& trees) {
+  int dev = 0;
+  DT_CK(cudaGetDevice(&dev));
+  {
+    dt_status ps = keep_pool(dev);
+    if (ps != DT_OK) return ps;
+  }
+  Workspace ws;
+  ws.s = s;
+  FitBufs b{};
+  auto get = [&](auto** p, size_t c) -> cudaError_t { return ws.get(p, c); };
+  dt_status st = fit_alloc(b, n, n, d, max_depth, min_leaf, 1, get);
+  if (st != DT_OK) return st;
+  const size_t tot = (size_t)n * d;
+  float* sx = nullptr;
+  uint32_t *sr = nullptr, *w = nullptr;
+  double *sy = nullptr, *ys = nullptr;
+  unsigned long long* tsum = nullptr;
+  st = alloc_status(ws.get(&sx, tot));
+  if (st == DT_OK) st = alloc_status(ws.get(&sr, tot));
+  if (st == DT_OK) st = alloc_status(ws.get(&sy, tot));
+  if (st == DT_OK) st = alloc_status(ws.get(&w, (size_t)n));
+  if (st == DT_OK) st = alloc_status(ws.get(&ys, (size_t)n));
+  if (st == DT_OK) st = alloc_status(ws.get(&tsum, tot / 2048 + 2));
+  if (st != DT_OK) return st;
+  DT_CK(cudaMemsetAsync(b.ctl, 0, sizeof(Ctl), s));
+  {
+    Nvtx range("dt forest presort");
+    st = presort_enqueue(b, X, y, n, d, d, 0, max_depth, min_leaf, s);
+  }
+  if (st != DT_OK) return st;
+  Ctl hc;
+  DT_CK(cudaMemcpyAsync(&hc, b.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+  DT_CK(cudaMemcpyAsync(sx, b.lx[0], sizeof(float) * tot, cudaMemcpyDeviceToDevice, s));
+  DT_CK(cudaMemcpyAsync(sr, b.lr[0], sizeof(uint32_t) * tot, cudaMemcpyDeviceToDevice, s));
+  DT_CK(cudaMemcpyAsync(sy, b.ly[0], sizeof(double) * tot, cudaMemcpyDeviceToDevice, s));
+  DT_CK(cudaStreamSynchronize(s));
+  if (hc.nonfinite) return fail(DT_ERR_NONFINITE, "dt_forest_fit: non-finite value in X or y");
+  for (int32_t t = 0; t < n_trees; ++t) {
+    st = clear_pieces(b, s);
+    if (st == DT_OK)
+      st = forest_tree_enqueue(b, sx, sr, sy, y, n, d, max_depth, min_leaf, seed, (uint32_t)t, hc.y32, w, ys, tsum, s);
+    if (st == DT_OK) st = fit_levels(b, d, max_depth, min_leaf, s, true, nullptr);
+    dt_tree* tr = nullptr;
+    if (st == DT_OK) st = fit_finish(b, d, s, nullptr, &tr);
+    if (st != DT_OK) return st;
+    trees.push_back(tr);
   }
   return DT_OK;
 }

@@ -2,6 +2,7 @@
 // "Kernels"): per-feature stable sort of (x, row id) once per fit, written as the level-0
 // lists, the level-0 segment table, the chunk descriptors and the root node.
 #include <algorithm>
+#include <type_traits>
 #include <vector>
 
 #include "fit_core.cuh"
@@ -825,6 +826,167 @@ dt_status presort_sharded_enqueue(const FitBufs& b, dt_comm* comm, const float* 
   st = comm_allgather(comm, bmine, ball, sizeof(BndRec) * d, s);
   if (st != DT_OK) return st;
   root_tables_sharded_kernel<<<num_sms(), 256, 0, s>>>(ctl, b.nodes[0], A0, d, p, P, ball, b.segs[0], b.pseg, b.desc[0]);
+  DT_CK(cudaGetLastError());
+  return DT_OK;
+}
+
+}  // namespace dtl
+
+namespace dtl {
+
+namespace {
+
+// Random Forest by expansion of the table's presorted lists: tree t's
+// bootstrap sample has row r w_r times (w = the draw counts); its level-0 lists are the
+// table's presorted lists with entry (x, r, y) repeated w_r times in place.  Equal x keep
+// any order -- no split falls between equal x -- so integer-mode trees equal the exact
+// CART of the sample in draw order (Reading R20); the copies keep row id r (they always go
+// the same way).
+__global__ void __launch_bounds__(256) boot_count_kernel(uint64_t seed, uint32_t t, int64_t n, uint32_t* __restrict__ w,
+                                                         const double* __restrict__ y, double* __restrict__ ys) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    uint64_t z = seed + 0x9E3779B97F4A7C15ull * ((((uint64_t)t) << 32) + (uint64_t)i + 1ull);  // Reading R21
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    z ^= z >> 31;
+    const uint32_t r = (uint32_t)(z % (uint64_t)n);
+    atomicAdd(w + r, 1u);
+    ys[i] = __ldg(y + r);  // the sample's targets in draw order (root statistics)
+  }
+}
+
+constexpr int kXT = 2048;  // entries per expansion tile
+__global__ void __launch_bounds__(256) expand_sum_kernel(const uint32_t* __restrict__ lr, const uint32_t* __restrict__ w,
+                                                         int64_t total, unsigned long long* __restrict__ tsum) {
+  __shared__ unsigned long long sh[8];
+  const int64_t base = (int64_t)blockIdx.x * kXT;
+  unsigned long long acc = 0;
+  for (int i = threadIdx.x; i < kXT; i += 256)
+    if (base + i < total) acc += __ldg(w + __ldg(lr + base + i));
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = acc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long t = 0;
+    for (int q = 0; q < 8; ++q) t += sh[q];
+    tsum[blockIdx.x] = t;
+  }
+}
+__global__ void __launch_bounds__(1024) expand_scan_kernel(unsigned long long* __restrict__ tsum, int64_t ntiles) {
+  __shared__ unsigned long long sh[33];
+  __shared__ unsigned long long run;
+  if (threadIdx.x == 0) run = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  for (int64_t b0 = 0; b0 < ntiles; b0 += 1024) {
+    const int64_t i = b0 + threadIdx.x;
+    const unsigned long long v = i < ntiles ? tsum[i] : 0ull;
+    unsigned long long inc = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const unsigned long long o = __shfl_up_sync(0xffffffffu, inc, d);
+      if (lane >= d) inc += o;
+    }
+    if (lane == 31) sh[w] = inc;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned long long r = 0;
+      for (int q = 0; q < 32; ++q) { const unsigned long long t = sh[q]; sh[q] = r; r += t; }
+      sh[32] = r;
+    }
+    __syncthreads();
+    if (i < ntiles) tsum[i] = run + sh[w] + inc - v;
+    __syncthreads();
+    if (threadIdx.x == 0) run += sh[32];
+    __syncthreads();
+  }
+}
+template <bool kY32>
+__global__ void __launch_bounds__(256) expand_write_kernel(const float* __restrict__ sx, const uint32_t* __restrict__ sr,
+                                                           const double* __restrict__ sy, const uint32_t* __restrict__ w,
+                                                           int64_t total, const unsigned long long* __restrict__ toff,
+                                                           float* __restrict__ ox, uint32_t* __restrict__ orow,
+                                                           double* __restrict__ oy) {
+  using YT = typename std::conditional<kY32, uint32_t, unsigned long long>::type;
+  __shared__ unsigned long long sh[9];
+  const int64_t base = (int64_t)blockIdx.x * kXT;
+  const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5;
+  // thread t owns entries base + 8 t .. base + 8 t + 7 (in order)
+  uint32_t cnt[8];
+  unsigned long long tot = 0;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    const int64_t p = base + 8 * threadIdx.x + j;
+    cnt[j] = p < total ? __ldg(w + __ldg(sr + p)) : 0u;
+    tot += cnt[j];
+  }
+  unsigned long long inc = tot;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const unsigned long long o = __shfl_up_sync(0xffffffffu, inc, d);
+    if (lane >= d) inc += o;
+  }
+  if (lane == 31) sh[wp] = inc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long r = 0;
+    for (int q = 0; q < 8; ++q) { const unsigned long long t = sh[q]; sh[q] = r; r += t; }
+  }
+  __syncthreads();
+  unsigned long long pos = toff[blockIdx.x] + sh[wp] + inc - tot;
+  const YT* ys = reinterpret_cast<const YT*>(sy);
+  YT* yo = reinterpret_cast<YT*>(oy);
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    const int64_t p = base + 8 * threadIdx.x + j;
+    if (cnt[j]) {
+      const float x = sx[p];
+      const uint32_t r = sr[p];
+      const YT yv = ys[p];
+      for (uint32_t c = 0; c < cnt[j]; ++c) {
+        ox[pos + c] = x;
+        orow[pos + c] = r;
+        yo[pos + c] = yv;
+      }
+      pos += cnt[j];
+    }
+  }
+}
+
+__global__ void set_storage_kernel(Ctl* ctl, int y32) { ctl->y32 = y32; }
+
+}  // namespace
+
+// Bootstrap tree t of a forest: draw counts, the sample's level-0 lists by expansion of the
+// table's presorted lists (sx, sr, sy: n entries per feature), the root of the sample (its
+// statistics in draw order) and the level-0 tables.  scratch: w (n u32), ys (n f64),
+// tsum (n d / kXT + 1 u64).  y32: the lists' y storage (the table's, Reading R24).
+dt_status forest_tree_enqueue(const FitBufs& b, const float* sx, const uint32_t* sr, const double* sy,
+                              const double* y, int64_t n, int d, int32_t max_depth, int64_t min_leaf, uint64_t seed,
+                              uint32_t t, int y32, uint32_t* w, double* ys, unsigned long long* tsum,
+                              cudaStream_t s) {
+  const int64_t total = n * (int64_t)d;
+  const int64_t ntiles = (total + kXT - 1) / kXT;
+  DT_CK(cudaMemsetAsync(w, 0, sizeof(uint32_t) * (size_t)n, s));
+  DT_CK(cudaMemsetAsync(b.ctl, 0, sizeof(Ctl), s));
+  const int gb = std::max(1, std::min<int>((int)((n + 255) / 256), num_sms() * 8));
+  int pr = prof_begin(PK_PRESORT_BUILD, s, 4);
+  boot_count_kernel<<<gb, 256, 0, s>>>(seed, t, n, w, y, ys);
+  expand_sum_kernel<<<(unsigned)ntiles, 256, 0, s>>>(sr, w, total, tsum);
+  expand_scan_kernel<<<1, 1024, 0, s>>>(tsum, ntiles);
+  if (y32) expand_write_kernel<true><<<(unsigned)ntiles, 256, 0, s>>>(sx, sr, sy, w, total, tsum, b.lx[0], b.lr[0], b.ly[0]);
+  else expand_write_kernel<false><<<(unsigned)ntiles, 256, 0, s>>>(sx, sr, sy, w, total, tsum, b.lx[0], b.lr[0], b.ly[0]);
+  prof_end(pr, s, (16.0 + 4.0) * (double)total * 2.0);
+  DT_CK(cudaGetLastError());
+  pr = prof_begin(PK_ROOT, s, 6);
+  root_reduce_kernel<<<(unsigned)b.root_np, 256, 0, s>>>(ys, n, b.root_chunk, reinterpret_cast<RootPart*>(b.parts));
+  root_finalize_kernel<<<1, 32, 0, s>>>(reinterpret_cast<RootPart*>(b.parts), (int)b.root_np, n, b.ctl);
+  root_center_kernel<<<(unsigned)b.root_np, 256, 0, s>>>(ys, n, n, b.root_chunk, b.ctl, b.cparts);
+  root_init_kernel<<<1, 32, 0, s>>>(b.cparts, (int)b.root_np, n, d, max_depth, min_leaf, b.ctl, b.nodes[0], b.dec_root);
+  set_storage_kernel<<<1, 1, 0, s>>>(b.ctl, y32);  // the lists keep the table's y storage
+  root_tables_kernel<<<num_sms(), 256, 0, s>>>(b.ctl, b.nodes[0], n, d, b.segs[0], b.pseg, b.desc[0]);
+  prof_end(pr, s, 16.0 * (double)n);
   DT_CK(cudaGetLastError());
   return DT_OK;
 }
