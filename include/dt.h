@@ -192,9 +192,12 @@ dt_status dt_importances(const dt_tree* tree, double* importances_host, void* st
  * z = (z ^ z >> 30) * 0xBF58476D1CE4E5B9, z = (z ^ z >> 27) * 0x94D049BB133111EB,
  * z ^= z >> 31, idx = z mod n (all mod 2^64).  Prediction: the mean of the trees'
  * predictions, summed in fp64 in tree order, then divided by n_trees.
- * dt_forest_fit: X_dev n x d f32 row-major, y_dev n f64 (as dt_fit); n_trees >= 1; the
- * library allocates one n x d bootstrap sample for the duration of the call; returns
- * when every tree is complete.  The forest owns its trees: dt_forest_tree returns a
+ * dt_forest_fit: X_dev n x d f32 row-major, y_dev n f64 (as dt_fit); n_trees >= 1.  The
+ * table is presorted ONCE; tree t's sorted lists are the presorted lists with every
+ * entry repeated by its row's draw count (equal x may then sit in another order than the
+ * draw order -- no split falls between equal x, so integer-mode trees are identical).
+ * Workspace (stream-ordered, pooled, for the duration of the call): dt_fit's plus
+ * ~16 B per (row, feature) for the presorted copy.  Returns when every tree is complete.  The forest owns its trees: dt_forest_tree returns a
  * borrowed pointer valid until dt_forest_free.  Errors as dt_fit. */
 typedef struct dt_forest dt_forest;
 dt_status dt_forest_fit(const float* X_dev, const double* y_dev, int64_t n, int32_t d,
@@ -318,9 +321,11 @@ dt_status dt_profile_get(int32_t kind, const char** name, int64_t* launches, dou
 
 /* Workspace is kept between calls so that repeated fits allocate nothing: the cached
  * CUDA-graph plans of the last two bounded-depth dt_fit inputs (least recently used
- * replaced; buffers ~32 B per training entry, i.e. 32 * n * d bytes each; a plan that
- * does not fit beside the other evicts it) and the freed blocks of the device's default
- * memory pool (stream-ordered workspace of the other calls).  dt_release_workspace
+ * replaced; buffers ~34 B per training entry, i.e. ~34 * n * d bytes each, plus per-node
+ * tables of ~290 B * min(n / m, 2^max_depth) * d; a plan that does not fit beside the
+ * other evicts it) and the freed blocks of the device's default memory pool
+ * (stream-ordered workspace of dt_fit_grid, dt_forest_fit, dt_fit_sharded, predict and
+ * eval calls; nothing else is cached across calls).  dt_release_workspace
  * synchronises the device, frees the cached plans and trims the pool of the CURRENT
  * device to zero, so that a following large allocation (e.g. the 100M x 32 fit of
  * BASELINE configs[2], ~110 GB) can use the whole HBM.  Always safe to call; the next fit
