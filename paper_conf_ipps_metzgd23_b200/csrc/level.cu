@@ -697,26 +697,15 @@ __device__ __forceinline__ uint32_t store_rows(const FusedArgs& a, const PSeg& p
   return pre;
 }
 
-// rcp with two Newton steps: relative error ~3e-16 (a filter only; the winner's gain is
-// exact)
-__device__ __forceinline__ double rcp_nr(double x) {
-  double r;
-  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
-  double e = __fma_rn(-x, r, 1.0);
-  r = __fma_rn(r, e, r);
-  e = __fma_rn(-x, r, 1.0);
-  return __fma_rn(r, e, r);
-}
-
-// One child's candidate search over a lane's items: running prefix S (child-centred), the
-// child position, the neighbour x; best candidate by a Newton-reciprocal gain with a
-// near-tie flag (then the exact pass decides), exact gain of the winner.
+// One child's candidate search over a lane's items: running prefix S'_L (child-centred,
+// rank carry included), the child position, the neighbour x; the exact gain (Reading
+// R19) at every valid position, strict > (the lowest position wins exact ties).
 struct Side {
   double S, sc, Nd, jd;         // prefix (rank carry included), S' of the child, N, position (f64)
   uint32_t jl, lo, hi;          // local position, valid local range [lo, hi)
   float xp;                     // x of the previous entry of this child
-  double bg, bs, bjd;           // best gain (approximate pass: approximate), its S'_L, position
-  uint32_t bj;                  // best global position (after finish / the exact pass)
+  double bg, bs, bjd;           // best gain, its S'_L and position
+  uint32_t bj;                  // best global position
   float bxp, bx;
   __device__ __forceinline__ void init(const PSeg& ps, int side, uint32_t ilo, uint32_t m, bool srch, double S0,
                                        float x0, uint32_t j0) {
@@ -734,31 +723,6 @@ struct Side {
     bj = 0xffffffffu;
     bxp = bx = 0.f;
   }
-  // approximate pass; returns true on a near tie with the current best
-  __device__ __forceinline__ bool step(float x, double d) {
-    bool amb = false;
-    if (jl >= lo && jl < hi && xp < x) {
-      const double nr = __dsub_rn(Nd, jd);
-      const double D = __dsub_rn(__dmul_rn(S, nr), __dmul_rn(__dsub_rn(sc, S), jd));
-      const double ga = __dmul_rn(__dmul_rn(D, D), rcp_nr(__dmul_rn(__dmul_rn(Nd, jd), nr)));
-      constexpr double kTol = 1e-13;  // >> |approx - exact| / exact (~3e-16)
-      if (ga > bg) {
-        amb = bg >= __dmul_rn(ga, 1.0 - kTol);
-        bg = ga;
-        bs = S;
-        bjd = jd;
-        bxp = xp;
-        bx = x;
-      } else {
-        amb = ga >= __dmul_rn(bg, 1.0 - kTol);
-      }
-    }
-    S = __dadd_rn(S, d);
-    ++jl;
-    jd = __dadd_rn(jd, 1.0);
-    xp = x;
-    return amb;
-  }
   __device__ __forceinline__ void step_exact(float x, double d) {
     if (jl >= lo && jl < hi && xp < x) {
       const double g = split_gain_d(S, sc, jd, Nd);
@@ -774,10 +738,6 @@ struct Side {
     ++jl;
     jd = __dadd_rn(jd, 1.0);
     xp = x;
-  }
-  __device__ __forceinline__ void finish() {  // the exact gain of the approximate winner
-    if (bg >= 0.0) bg = split_gain_d(bs, sc, bjd, Nd);
-    bj = (uint32_t)bjd;
   }
 };
 
@@ -995,20 +955,11 @@ __global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArg
         const uint32_t sb = side ? rbyte : lbyte;
         Side sd;
         sd.init(ps, side, ilo, m, true, side ? SR : SL, side ? xr : xl, side ? jr0 : nl);
-        bool amb = false;
+        // exact gain (Reading R19) at every valid position; strict >: lowest position
 #pragma unroll
         for (int j = 0; j < kItems; ++j)
-          if ((sb >> j) & 1u) amb |= sd.step(xv[j], dv[j]);
-        if (__any_sync(0xffffffffu, amb)) {
-          // a near tie of approximate gains in some lane: exact gains at every position
-          sd.init(ps, side, ilo, m, true, side ? SR : SL, side ? xr : xl, side ? jr0 : nl);
-#pragma unroll
-          for (int j = 0; j < kItems; ++j)
-            if ((sb >> j) & 1u) sd.step_exact(xv[j], dv[j]);
-          sd.bj = (uint32_t)sd.bjd;
-        } else {
-          sd.finish();
-        }
+          if ((sb >> j) & 1u) sd.step_exact(xv[j], dv[j]);
+        sd.bj = (uint32_t)sd.bjd;
         const double bg = sd.bg;
         const uint32_t bj = sd.bj;
         // warp max of the exact gains (>= 0: the f64 bit patterns order like the values;
