@@ -220,7 +220,7 @@ __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
   // nothing reads the bitmap between the previous level's F_A and this level's goleft
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + tid; i < a.nvec; i += (int64_t)gridDim.x * blockDim.x)
     a.gbits[i] = make_uint4(0u, 0u, 0u, 0u);
-  if (blockIdx.x == 0 && tid == 0) a.ctl->nfast = a.ctl->ngen = a.ctl->nunit = a.ctl->nbig = 0u;  // next chunk plan
+  if (blockIdx.x == 0 && tid == 0) a.ctl->nfast = a.ctl->ngen = a.ctl->nunit = a.ctl->nsmall = 0u;  // next chunk plan
   if (blockIdx.x == 0 && tid == 0 && a.level < kMaxLogLevels) {
     a.log[a.level].T = a.ctl->T[a.par];
     a.log[a.level].K = K;
@@ -469,10 +469,11 @@ __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
 // it hold left entries of a split feature?); the warp then sets the bits of the
 // qualifying chunks together.
 __global__ void __launch_bounds__(256) goleft_kernel(const Ctl* __restrict__ ctl, int par, const uint32_t* __restrict__ desc,
-                                                     const SegT* __restrict__ segs, const Decision* __restrict__ dec,
-                                                     const uint32_t* __restrict__ lr, uint32_t* __restrict__ gbits) {
+                                                     const PSeg* __restrict__ pseg, const uint32_t* __restrict__ lr,
+                                                     uint32_t* __restrict__ gbits, int d) {
   const uint64_t T = ctl->T[par];
   if (ctl->K[par ^ 1] == 0) return;  // nothing splits
+  const uint32_t nseg = ctl->K[par] * (uint32_t)d;
   const int64_t nch = (int64_t)((T + kChunkW - 1) / kChunkW);
   const int lane = threadIdx.x & 31;
   // warp gw tests chunks gw + (32 it + lane) nw: qualifying chunks (contiguous runs of a
@@ -485,14 +486,9 @@ __global__ void __launch_bounds__(256) goleft_kernel(const Ctl* __restrict__ ctl
     if (mych < nch) {
       const uint64_t cbase = (uint64_t)mych * kChunkW;
       const uint32_t s = __ldg(desc + mych);
-      const uint64_t st = __ldg(&segs[s].start), en = st + __ldg(&segs[s].cnt);
-      if (st <= cbase && en >= cbase + kChunkW) {
-        const uint32_t k = __ldg(&segs[s].k);
-        const uint32_t ioff = __ldg(&segs[s].ioff);
-        q = __ldg(&dec[k].f) == __ldg(&segs[s].f) && cbase < st + (uint64_t)(__ldg(&dec[k].nl) - min(ioff, __ldg(&dec[k].nl)));
-      } else {
-        q = true;  // segment heads inside: walk it
-      }
+      const uint64_t st = __ldg(&pseg[s].start), en = st + __ldg(&pseg[s].cnt);
+      // one segment: does it hold left entries here?  Else segment heads inside: walk it
+      q = (st <= cbase && en >= cbase + kChunkW) ? cbase < st + __ldg(&pseg[s].glim) : true;
     }
     uint32_t qm = __ballot_sync(0xffffffffu, q);
     while (qm) {
@@ -501,14 +497,10 @@ __global__ void __launch_bounds__(256) goleft_kernel(const Ctl* __restrict__ ctl
       const int64_t ch = gw + (it * 32 + c) * nw;
       const uint64_t cbase = (uint64_t)ch * kChunkW;
       uint32_t s = __ldg(desc + ch);
-      uint64_t st = __ldg(&segs[s].start), en = st + __ldg(&segs[s].cnt);
-      uint32_t k = __ldg(&segs[s].k);
-      int f = __ldg(&segs[s].f);
-      uint32_t ioff = __ldg(&segs[s].ioff);
+      uint64_t st = __ldg(&pseg[s].start), en = st + __ldg(&pseg[s].cnt);
+      uint64_t lim = st + __ldg(&pseg[s].glim);  // the segment's left entries: [st, lim)
       if (st <= cbase && en >= cbase + kChunkW) {
-        // one segment: its local positions i < nl - ioff go left (rows read coalesced)
-        const uint32_t nl = __ldg(&dec[k].nl);
-        const uint64_t lim = (nl > ioff) ? st + (nl - ioff) : st;
+        // one segment (rows read coalesced)
 #pragma unroll
         for (int j = 0; j < kItems; ++j) {
           const uint64_t p = cbase + (uint64_t)(j * 32 + lane);
@@ -519,21 +511,19 @@ __global__ void __launch_bounds__(256) goleft_kernel(const Ctl* __restrict__ ctl
         }
         continue;
       }
-      // segment heads inside: lane owns entries 8 lane .. 8 lane + 7, walks their segments
+      // segment heads inside: lane owns entries 8 lane .. 8 lane + 7, finds their segments
       const uint64_t p0 = cbase + (uint64_t)(lane * kItems);
 #pragma unroll
       for (int j = 0; j < kItems; ++j) {
         const uint64_t p = p0 + j;
         if (p >= T) break;
-        while (p >= en) {
-          ++s;
-          st = __ldg(&segs[s].start);
-          en = st + __ldg(&segs[s].cnt);
-          k = __ldg(&segs[s].k);
-          f = __ldg(&segs[s].f);
-          ioff = __ldg(&segs[s].ioff);
+        if (p >= en) {
+          s = seg_gallop(pseg, s + 1u, nseg - 1u, p);
+          st = __ldg(&pseg[s].start);
+          en = st + __ldg(&pseg[s].cnt);
+          lim = st + __ldg(&pseg[s].glim);
         }
-        if (__ldg(&dec[k].f) == f && ioff + (uint32_t)(p - st) < __ldg(&dec[k].nl)) {
+        if (p < lim) {
           const uint32_t r = __ldg(lr + p);
           atomicOr(gbits + (r >> 5), 1u << (r & 31));
         }
@@ -548,10 +538,26 @@ __global__ void __launch_bounds__(256) goleft_kernel(const Ctl* __restrict__ ctl
 // list) and the plan of every level-l segment (children, centres, positions).
 // mode 0 (P = 1): as above.  Sharded: mode 1 = the plans without the children's positions
 // and rank carries (before the boundary exchange), mode 2 = those from segs_next.
-__global__ void __launch_bounds__(256) tables_kernel(const Ctl* __restrict__ ctl, int par, int d,
+// The fused pass's work on split segment [start, start + cnt) (levels >= 0; listed from
+// the segment side): a segment of at most kSmallSeg entries -> the small list
+// (fused_small_kernel); else the chunks it meets without covering them -- its first and
+// last at most, the ones it covers are fast chunks (chunk_plan_kernel) -> unit-list pieces.
+__device__ __forceinline__ void piece_chunks(uint64_t start, uint32_t cnt, uint32_t& u0, uint32_t& u1, uint32_t& sm) {
+  if (cnt <= kSmallSeg) {
+    sm = 0u;
+    return;
+  }
+  const uint64_t end = start + cnt;
+  const uint64_t c0 = start / kChunkW, c1 = (end - 1) / kChunkW;
+  if (!(start == c0 * kChunkW && end >= c0 * kChunkW + kChunkW)) u0 = (uint32_t)c0;
+  if (c1 > c0 && end < c1 * kChunkW + kChunkW) u1 = (uint32_t)c1;
+}
+
+__global__ void __launch_bounds__(256) tables_kernel(Ctl* __restrict__ ctl, int par, int d,
                                                      const NodeL* __restrict__ next, const Decision* __restrict__ dec,
                                                      const SegT* __restrict__ segs, SegT* __restrict__ segs_next,
-                                                     PSeg* __restrict__ pseg, int mode) {
+                                                     PSeg* __restrict__ pseg, int mode, uint2* __restrict__ unit_list,
+                                                     uint32_t* __restrict__ small_list) {
   const uint32_t K = ctl->K[par], K2 = ctl->K[par ^ 1];
   const uint64_t A2 = ctl->A2;
   if (mode == 2) {
@@ -572,7 +578,11 @@ __global__ void __launch_bounds__(256) tables_kernel(const Ctl* __restrict__ ctl
     return;
   }
   const int64_t n1 = mode == 0 ? (int64_t)K2 * d : 0, n2 = (int64_t)K * d;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n1 + n2; i += (int64_t)gridDim.x * blockDim.x) {
+  const bool full = ctl->nsrch > 0;  // children searched: every list; else feature 0 (statistics)
+  const int lane = threadIdx.x & 31;
+  for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n1 + n2; base += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = base + threadIdx.x;  // warp-uniform trip count (the appends below)
+    uint32_t u0 = 0xffffffffu, u1 = 0xffffffffu, sm = 0xffffffffu;  // this segment's pieces
     if (i < n1) {
       const int f = (int)(i / K2);
       const uint32_t kc = (uint32_t)(i - (int64_t)f * K2);
@@ -587,7 +597,7 @@ __global__ void __launch_bounds__(256) tables_kernel(const Ctl* __restrict__ ctl
       sg.xprev = __int_as_float(0x7fc00000);
       sg.pad = 0;
       segs_next[i] = sg;
-    } else {
+    } else if (i < n1 + n2) {
       const int64_t s = i - n1;
       const int f = (int)(s / K);
       const uint32_t k = (uint32_t)(s - (int64_t)f * K);
@@ -600,7 +610,7 @@ __global__ void __launch_bounds__(256) tables_kernel(const Ctl* __restrict__ ctl
       p.f = f;
       p.flags = 0;
       p.kid = 0;
-      p.pad = 0;
+      p.glim = 0;
       for (int q = 0; q < 2; ++q) {
         p.cs[q] = 0;
         p.ostart[q] = 0;
@@ -611,6 +621,7 @@ __global__ void __launch_bounds__(256) tables_kernel(const Ctl* __restrict__ ctl
       if (dc.f >= 0) {
         p.flags = PS_SPLIT;
         p.kid = dc.kid;
+        if (dc.f == f) p.glim = min(sg.cnt, dc.nl > sg.ioff ? dc.nl - sg.ioff : 0u);
         for (int q = 0; q < 2; ++q) {
           const uint32_t kc = dc.kid + q;
           const NodeL c = next[kc];
@@ -624,7 +635,23 @@ __global__ void __launch_bounds__(256) tables_kernel(const Ctl* __restrict__ ctl
         }
       }
       pseg[s] = p;
+      if ((p.flags & PS_SPLIT) && p.cnt && (full || f == 0)) piece_chunks(p.start, p.cnt, u0, u1, sm);
     }
+    // warp-aggregated appends: pieces -> unit list, small segments -> small list
+    const uint32_t lt = (1u << lane) - 1u;
+    const uint32_t b0 = __ballot_sync(0xffffffffu, u0 != 0xffffffffu), b1 = __ballot_sync(0xffffffffu, u1 != 0xffffffffu);
+    const uint32_t bs = __ballot_sync(0xffffffffu, sm != 0xffffffffu);
+    uint32_t pu = 0, ps = 0;
+    if (lane == 0) {
+      if (b0 | b1) pu = atomicAdd(&ctl->nunit, (uint32_t)(__popc(b0) + __popc(b1)));
+      if (bs) ps = atomicAdd(&ctl->nsmall, (uint32_t)__popc(bs));
+    }
+    pu = __shfl_sync(0xffffffffu, pu, 0) + __popc(b0 & lt) + __popc(b1 & lt);
+    ps = __shfl_sync(0xffffffffu, ps, 0) + __popc(bs & lt);
+    const uint32_t sid = (uint32_t)(i - n1);
+    if (u0 != 0xffffffffu) unit_list[pu++] = make_uint2(u0, sid);
+    if (u1 != 0xffffffffu) unit_list[pu] = make_uint2(u1, sid);
+    if (sm != 0xffffffffu) small_list[ps] = sid;
   }
 }
 
@@ -847,8 +874,8 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int64_t n_global, int32_t d, int32_t 
   GET(b.gm, b.max_chunks * 32);
   GET(b.gen_list, b.max_chunks);
   GET(b.fast_list, b.max_chunks);
-  GET(b.unit_list, b.max_chunks * 9);  // <= 8 pieces per listed chunk (kMaxPieces)
-  GET(b.big_list, b.max_chunks);
+  GET(b.unit_list, b.max_chunks * 9);  // <= 9 pieces per listed chunk (kMaxPieces, level.cu)
+  GET(b.small_list, b.segcap);
   GET(b.head_cand, b.segcap);
   GET(b.cont_cand, 2 * b.max_chunks);
   GET(b.slot_gain, b.segcap);
@@ -1003,12 +1030,13 @@ dt_status fit_levels(const FitBufs& b, int32_t d, int32_t max_depth, int64_t min
     na.log = b.lvlog;
     pr = prof_begin(PK_NUMBER, s, 2);
     number_kernel<<<1, 1024, 0, s>>>(na);
-    tables_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, b.nodes[par ^ 1], b.dec, b.segs[par], b.segs[par ^ 1], b.pseg, 0);
+    tables_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, b.nodes[par ^ 1], b.dec, b.segs[par], b.segs[par ^ 1], b.pseg, 0,
+                                        b.unit_list, b.small_list);
     prof_end(pr, s, 0.0);
     DT_CK(cudaGetLastError());
     // ---- go-left bitmap (a6)
     pr = prof_begin(PK_GOLEFT, s, 1);
-    goleft_kernel<<<g_gl, 256, 0, s>>>(ctl, par, b.desc[par], b.segs[par], b.dec, b.lr[cur], b.gbits);
+    goleft_kernel<<<g_gl, 256, 0, s>>>(ctl, par, b.desc[par], b.pseg, b.lr[cur], b.gbits, d);
     prof_end(pr, s, 0.0);
     if (pending) pending->push_back({pr, level, PK_GOLEFT});
     DT_CK(cudaGetLastError());
@@ -1522,15 +1550,17 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
     DT_CK(cudaStreamSynchronize(s));
     const uint32_t K2 = hk[par ^ 1];
     if (K2 == 0) break;  // every node of the level is a leaf (same on every rank)
+    // plans of the level's segments (their go-left counts feed the bitmap)
+    tables_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, b.nodes[par ^ 1], b.dec, b.segs[par], b.segs[par ^ 1], b.pseg, 1,
+                                        b.unit_list, b.small_list);
+    DT_CK(cudaGetLastError());
     // go-left bitmap: each rank sets the bits of its own split-feature entries; OR over ranks
     pr = prof_begin(PK_GOLEFT, s, 1);
-    goleft_kernel<<<g_gl, 256, 0, s>>>(ctl, par, b.desc[par], b.segs[par], b.dec, b.lr[cur], b.gbits);
+    goleft_kernel<<<g_gl, 256, 0, s>>>(ctl, par, b.desc[par], b.pseg, b.lr[cur], b.gbits, d);
     DT_CK(cudaGetLastError());
     st = comm_allreduce_or_u32(comm, b.gbits, b.nwords4, s);
     if (st != DT_OK) return st;
     prof_end(pr, s, 0.0);
-    tables_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, b.nodes[par ^ 1], b.dec, b.segs[par], b.segs[par ^ 1], b.pseg, 1);
-    DT_CK(cudaGetLastError());
     LevelArgs la{level, cur, par, d, min_leaf, true};
     pr = prof_begin(PK_SCAN, s, 3);
     st = level_agg_enqueue(b, la, s);
@@ -1550,7 +1580,7 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
       segwrite_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, rank, b.nodes[par ^ 1], b.bnd_all, excl, btot,
                                             b.segs[par ^ 1]);
       tables_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, b.nodes[par ^ 1], b.dec, b.segs[par], b.segs[par ^ 1], b.pseg,
-                                          2);
+                                          2, b.unit_list, b.small_list);
       DT_CK(cudaGetLastError());
     } else {
       // no searchable child: statistics only, nothing is written (empty next lists)

@@ -26,6 +26,7 @@ namespace dtl {
 
 constexpr int kItems = 8;                 // entries per lane
 constexpr int kChunkW = 32 * kItems;      // entries per warp chunk
+constexpr uint32_t kSmallSeg = 32;         // split segments of <= 32 entries: the small pass (warp per segment)
 constexpr int kBlockChunks = 1024;        // chunks per block of the chunk-carry scan (F_B)
 constexpr int kMaxLogLevels = 4096;
 
@@ -80,7 +81,8 @@ struct __align__(16) PSeg {
   uint32_t ioff[2];    // children: rank carries (see SegT)
   double soff[2];
   float xprev[2];
-  uint32_t kid, pad;
+  uint32_t kid;
+  uint32_t glim;       // go-left bitmap: this rank's first glim entries of the segment go left
 };
 static_assert(sizeof(PSeg) == 144, "PSeg is copied with one bulk copy");
 
@@ -185,7 +187,7 @@ struct Ctl {
   uint32_t nfast;            // chunk plan of the pass: chunks inside one split segment,
   uint32_t ngen;             //   chunks with segment heads inside,
   uint32_t nunit;            //   split segment pieces of chunks (the fused pass),
-  uint32_t nbig;             //   chunks with too many pieces
+  uint32_t nsmall;           //   split segments of at most 32 entries (the small pass)
   unsigned long long split_evals;
   double ysum, ymin, ymax, ysc;
 };
@@ -226,6 +228,32 @@ __device__ __forceinline__ double split_gain_d(double sl, double sc, double nl, 
   return __ddiv_rn(__dmul_rn(D, D), __dmul_rn(__dmul_rn(Nd, nl), nr));
 }
 
+// The segment holding list position p: the largest t in [lo, hi] with segs[t].start <= p,
+// given segs[lo].start <= p.  Segments tile the level's lists in index order and an empty
+// segment shares its successor's start, so t is the non-empty segment containing p.
+// Galloping from lo (the next few segments are the usual answer), then bisection: a walk
+// over long runs of small or empty segments costs O(log distance) loads instead of O(distance).
+template <class Seg>
+__device__ __forceinline__ uint32_t seg_gallop(const Seg* __restrict__ segs, uint32_t lo, uint32_t hi, uint64_t p) {
+  uint32_t step = 1u;
+  while (lo < hi) {
+    const uint32_t t = (hi - lo > step) ? lo + step : hi;
+    if (__ldg(&segs[t].start) <= p) {
+      lo = t;
+      step <<= 1;
+    } else {
+      hi = t - 1u;
+      break;
+    }
+  }
+  while (lo < hi) {
+    const uint32_t mid = lo + ((hi - lo + 1u) >> 1);
+    if (__ldg(&segs[mid].start) <= p) lo = mid;
+    else hi = mid - 1u;
+  }
+  return lo;
+}
+
 __device__ __forceinline__ double mid_threshold(float xlo, float xhi) {  // Reading R5
   return __dadd_rn(__ddiv_rn((double)xlo, 2.0), __ddiv_rn((double)xhi, 2.0));
 }
@@ -248,7 +276,7 @@ struct FitBufs {
   uint2* fast_list;    // chunk plan of the pass: {chunk, segment} inside one split segment
   uint32_t* gen_list;  // chunks with segment heads inside
   uint2* unit_list;    // {chunk, segment}: split segment pieces of chunks (fused pass)
-  uint32_t* big_list;  // chunks with more than kMaxPieces pieces
+  uint32_t* small_list;  // split segments of at most 32 entries (their ids)
   Cand2 *head_cand, *cont_cand;
   unsigned long long *slot_gain, *slot_pos;
   Stat *head_stat, *cont_stat;

@@ -57,6 +57,7 @@ struct AggArgs {
   const uint32_t* gen_list;
   const Ctl* ctl;
   int par;
+  uint32_t d;  // lists per level (segments of the parent level: K * d)
   int64_t nwords;
 };
 
@@ -141,43 +142,69 @@ __device__ __forceinline__ SegLite seg_lite(const PSeg* __restrict__ ps, uint32_
 // Chunk plan of a pass (thread per chunk).  A chunk inside ONE segment: of a split node
 // -> fast list {chunk, segment} (F_A fast path) and unit list (F_C); of a node that does
 // not split -> nothing to do (its aggregate is written here).  A chunk with segment heads
-// inside -> gen list (F_A general path) and, per split segment piece, the unit list when
-// it has at most kMaxPieces such pieces (F_C processes the chunk once per piece, masked to
-// the piece's entries), else the big list (fused_general_kernel).  Warp-aggregated appends.
-constexpr int kMaxPieces = 8;
+// inside -> gen list (F_A general path) and, per split segment piece of more than
+// kSmallSeg entries, the unit list (F_C processes the chunk once per piece, masked to the
+// piece's entries).  Split segments of at most kSmallSeg entries go to the small list
+// (fused_small_kernel: a warp per segment, lane = entry), from the chunk holding their
+// head.  (Levels >= 0: tables_kernel lists the pieces and small segments from the segment
+// side, emit_pieces; this walk serves the virtual-root pass.)  So a chunk has at most kMaxPieces pieces: k segments of >= 33 entries meeting
+// 256 consecutive entries have their k - 2 middle ones inside, (k - 2) * 33 <= 254, k <= 9.
+// Block-aggregated appends.
+constexpr int kMaxPieces = 9;
 
-__device__ __forceinline__ uint32_t warp_append(uint32_t cnt, uint32_t* counter) {
-  const int lane = threadIdx.x & 31;
-  uint32_t inc = cnt;
+// Block-aggregated appends to four list counters (one atomic per counter per block;
+// block-uniform call: contains barriers).  pos[i] = this thread's first slot.
+__device__ __forceinline__ void block_append4(const uint32_t (&cnt)[4], uint32_t* const (&ctr)[4],
+                                              uint32_t (&pos)[4]) {
+  __shared__ uint32_t sw[32][4];
+  __shared__ uint32_t sb[4];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t inc[4];
 #pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    const uint32_t o = __shfl_up_sync(0xffffffffu, inc, d);
-    if (lane >= d) inc += o;
+  for (int i = 0; i < 4; ++i) {
+    inc[i] = cnt[i];
+#pragma unroll
+    for (int dd = 1; dd < 32; dd <<= 1) {
+      const uint32_t o = __shfl_up_sync(0xffffffffu, inc[i], dd);
+      if (lane >= dd) inc[i] += o;
+    }
+    if (lane == 31) sw[w][i] = inc[i];
   }
-  const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
-  uint32_t base = 0;
-  if (lane == 31 && tot) base = atomicAdd(counter, tot);
-  base = __shfl_sync(0xffffffffu, base, 31);
-  return base + inc - cnt;
+  __syncthreads();
+  if (threadIdx.x < 4) {
+    const int i = threadIdx.x;
+    uint32_t run = 0u;
+    for (int q = 0; q < (int)(blockDim.x >> 5); ++q) {
+      const uint32_t t = sw[q][i];
+      sw[q][i] = run;
+      run += t;
+    }
+    sb[i] = run ? atomicAdd(ctr[i], run) : 0u;
+  }
+  __syncthreads();
+#pragma unroll
+  for (int i = 0; i < 4; ++i) pos[i] = sb[i] + sw[w][i] + inc[i] - cnt[i];
+  __syncthreads();  // sw / sb are reused by the next call
 }
 
 __global__ void __launch_bounds__(256) chunk_plan_kernel(Ctl* ctl, int par, int d, const uint32_t* __restrict__ desc,
                                                          const PSeg* __restrict__ pseg, AggP* __restrict__ agg,
                                                          uint2* __restrict__ fast_list, uint32_t* __restrict__ gen_list,
-                                                         uint2* __restrict__ unit_list, uint32_t* __restrict__ big_list) {
+                                                         uint2* __restrict__ unit_list, uint32_t* __restrict__ small_list,
+                                                         bool walk) {
   const uint64_t T = ctl->T[par];
   const bool full = ctl->nsrch > 0;  // children searched: every list; else feature 0 (statistics)
   const uint64_t Tw = full ? T : ctl->T0[par];
   const int64_t nch = (int64_t)((Tw + kChunkW - 1) / kChunkW);
   const uint32_t nseg = ctl->K[par] * (uint32_t)d;  // segments of the parent level
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < nch; base += stride) {  // warp-uniform trip count
+  for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < nch; base += stride) {  // block-uniform trip count
     const int64_t ch = base + threadIdx.x;
-    bool fast = false, gen = false, big = false;
-    uint32_t npieces = 0;
+    bool fast = false, gen = false;
+    uint32_t npieces = 0, nsmall = 0;
     uint32_t s = 0;
+    const uint64_t cbase = (uint64_t)ch * kChunkW, cend = min(cbase + kChunkW, T);
     if (ch < nch) {
-      const uint64_t cbase = (uint64_t)ch * kChunkW, cend = min(cbase + kChunkW, T);
       s = __ldg(desc + ch);
       const uint64_t st = __ldg(&pseg[s].start), en = st + __ldg(&pseg[s].cnt);
       const bool split = (__ldg(&pseg[s].flags) & PS_SPLIT) != 0;
@@ -190,33 +217,39 @@ __global__ void __launch_bounds__(256) chunk_plan_kernel(Ctl* ctl, int par, int 
         }
       } else {
         gen = true;
-        for (uint32_t t = s; t < nseg; ++t) {  // split segment pieces of this chunk
+        // split segments meeting this chunk (non-empty segments; empty runs skipped)
+        for (uint32_t t = s; walk;) {
           const uint64_t ts = __ldg(&pseg[t].start);
-          if (ts >= cend) break;
-          if (__ldg(&pseg[t].cnt) && (__ldg(&pseg[t].flags) & PS_SPLIT)) ++npieces;
-          if (npieces > (uint32_t)kMaxPieces) break;
-        }
-        if (npieces > (uint32_t)kMaxPieces) {
-          big = true;
-          npieces = 0;
+          const uint32_t tc = __ldg(&pseg[t].cnt);
+          if (tc && (__ldg(&pseg[t].flags) & PS_SPLIT)) {
+            if (tc > kSmallSeg) ++npieces;
+            else if (ts >= cbase) ++nsmall;
+          }
+          if (ts + tc >= cend || t + 1u >= nseg) break;
+          t = seg_gallop(pseg, t + 1u, nseg - 1u, ts + tc);
         }
       }
     }
-    const uint32_t pf = warp_append(fast ? 1u : 0u, &ctl->nfast);
-    const uint32_t pg = warp_append(gen ? 1u : 0u, &ctl->ngen);
-    const uint32_t pb = warp_append(big ? 1u : 0u, &ctl->nbig);
-    uint32_t pu = warp_append(fast ? 1u : npieces, &ctl->nunit);
+    const uint32_t cnt[4] = {fast ? 1u : 0u, gen ? 1u : 0u, nsmall, fast ? 1u : npieces};
+    uint32_t* const ctr[4] = {&ctl->nfast, &ctl->ngen, &ctl->nsmall, &ctl->nunit};
+    uint32_t pos[4];
+    block_append4(cnt, ctr, pos);
     if (fast) {
-      fast_list[pf] = make_uint2((uint32_t)ch, s);
-      unit_list[pu] = make_uint2((uint32_t)ch, s);
+      fast_list[pos[0]] = make_uint2((uint32_t)ch, s);
+      unit_list[pos[3]] = make_uint2((uint32_t)ch, s);
     }
-    if (gen) gen_list[pg] = (uint32_t)ch;
-    if (big) big_list[pb] = (uint32_t)ch;
-    if (npieces) {
-      const uint64_t cend = min((uint64_t)ch * kChunkW + kChunkW, T);
-      for (uint32_t t = s; t < nseg; ++t) {
-        if (__ldg(&pseg[t].start) >= cend) break;
-        if (__ldg(&pseg[t].cnt) && (__ldg(&pseg[t].flags) & PS_SPLIT)) unit_list[pu++] = make_uint2((uint32_t)ch, t);
+    if (gen) gen_list[pos[1]] = (uint32_t)ch;
+    if (npieces || nsmall) {
+      uint32_t pu = pos[3], psm = pos[2];
+      for (uint32_t t = s;;) {
+        const uint64_t ts = __ldg(&pseg[t].start);
+        const uint32_t tc = __ldg(&pseg[t].cnt);
+        if (tc && (__ldg(&pseg[t].flags) & PS_SPLIT)) {
+          if (tc > kSmallSeg) unit_list[pu++] = make_uint2((uint32_t)ch, t);
+          else if (ts >= cbase) small_list[psm++] = t;
+        }
+        if (ts + tc >= cend || t + 1u >= nseg) break;
+        t = seg_gallop(pseg, t + 1u, nseg - 1u, ts + tc);
       }
     }
   }
@@ -329,6 +362,7 @@ __global__ void __launch_bounds__(kSmemBits ? 1024 : kThreads) level_agg_kernel(
     }
   }
   // ---- general chunks: segment heads inside; per item walk
+  const uint32_t nseg = a.ctl->K[a.par] * a.d;
   for (int64_t gi = gw; gi < ngen; gi += nw) {
     const int64_t ch = (int64_t)a.gen_list[gi];
     const uint64_t cbase = (uint64_t)ch * kChunkW;
@@ -348,7 +382,10 @@ __global__ void __launch_bounds__(kSmemBits ? 1024 : kThreads) level_agg_kernel(
       for (int j = 0; j < kItems; ++j) {
         const uint64_t p = (uint64_t)p0 + j;
         if (p < T) {
-          while (p >= g2.end) g2 = seg_lite(a.pseg, ++sc);
+          if (p >= g2.end) {
+            sc = seg_gallop(a.pseg, sc + 1u, nseg - 1u, p);
+            g2 = seg_lite(a.pseg, sc);
+          }
           if (p == g2.start) {
             run = agg_ident();
             run.flag = 1u;
@@ -386,7 +423,10 @@ __global__ void __launch_bounds__(kSmemBits ? 1024 : kThreads) level_agg_kernel(
       for (int j = 0; j < kItems; ++j) {
         const uint64_t p = (uint64_t)p0 + j;
         if (p < T) {
-          while (p >= g2.end) g2 = seg_lite(a.pseg, ++sc);
+          if (p >= g2.end) {
+            sc = seg_gallop(a.pseg, sc + 1u, nseg - 1u, p);
+            g2 = seg_lite(a.pseg, sc);
+          }
           if (p == g2.start) {
             r = agg_ident();
             r.flag = 1u;
@@ -527,10 +567,11 @@ struct FusedArgs {
   Stat* head_stat;
   Stat* cont_stat;
   const uint2* unit_list;    // {chunk, segment}: a split segment's piece of a chunk
-  const uint32_t* big_list;  // chunks with more than kMaxPieces pieces (fused_general_kernel)
+  const uint32_t* small_list;  // split segments of at most kSmallSeg entries (fused_small_kernel)
   Ctl* ctl;
   int par;
   uint32_t level;   // level of the children (written into the pieces)
+  uint32_t d;       // lists per level (segments of the parent level: K * d)
   uint32_t m;       // min_samples_leaf (clamped)
   uint32_t ystride; // bytes of one y entry (4 or 8)
   uint32_t stage_bytes;
@@ -551,46 +592,11 @@ struct Meta {
   uint32_t skip, pad;
 };
 
-struct ArgQ {  // segmented argmax: ties keep the earlier position
-  uint32_t flag, j;
-  double gain, sl, thr;
-};
-__device__ __forceinline__ ArgQ argq_ident() { return ArgQ{0u, 0u, -1.0, 0.0, 0.0}; }
-__device__ __forceinline__ ArgQ combine(const ArgQ& a, const ArgQ& b) {
-  if (b.flag) return b;
-  ArgQ r = (b.gain > a.gain) ? b : a;
-  r.flag = a.flag;
-  return r;
-}
-__device__ __forceinline__ ArgQ shfl_up(const ArgQ& v, int d) {
-  return ArgQ{__shfl_up_sync(0xffffffffu, v.flag, d), __shfl_up_sync(0xffffffffu, v.j, d),
-              __shfl_up_sync(0xffffffffu, v.gain, d), __shfl_up_sync(0xffffffffu, v.sl, d),
-              __shfl_up_sync(0xffffffffu, v.thr, d)};
-}
-__device__ __forceinline__ ArgQ shfl_idx(const ArgQ& v, int s) {
-  return ArgQ{__shfl_sync(0xffffffffu, v.flag, s), __shfl_sync(0xffffffffu, v.j, s),
-              __shfl_sync(0xffffffffu, v.gain, s), __shfl_sync(0xffffffffu, v.sl, s),
-              __shfl_sync(0xffffffffu, v.thr, s)};
-}
 struct StatQ {
   uint32_t flag;
   double sse, ymin, ymax, s1;
 };
 __device__ __forceinline__ StatQ statq_ident() { return StatQ{0u, 0.0, INFINITY, -INFINITY, 0.0}; }
-__device__ __forceinline__ StatQ combine(const StatQ& a, const StatQ& b) {
-  if (b.flag) return b;
-  return StatQ{a.flag, __dadd_rn(a.sse, b.sse), fmin(a.ymin, b.ymin), fmax(a.ymax, b.ymax), __dadd_rn(a.s1, b.s1)};
-}
-__device__ __forceinline__ StatQ shfl_up(const StatQ& v, int d) {
-  return StatQ{__shfl_up_sync(0xffffffffu, v.flag, d), __shfl_up_sync(0xffffffffu, v.sse, d),
-               __shfl_up_sync(0xffffffffu, v.ymin, d), __shfl_up_sync(0xffffffffu, v.ymax, d),
-               __shfl_up_sync(0xffffffffu, v.s1, d)};
-}
-__device__ __forceinline__ StatQ shfl_idx(const StatQ& v, int s) {
-  return StatQ{__shfl_sync(0xffffffffu, v.flag, s), __shfl_sync(0xffffffffu, v.sse, s),
-               __shfl_sync(0xffffffffu, v.ymin, s), __shfl_sync(0xffffffffu, v.ymax, s),
-               __shfl_sync(0xffffffffu, v.s1, s)};
-}
 __device__ __forceinline__ void stat_add(StatQ& st, double y, double v, double c) {
   const double e = __dsub_rn(y, v);
   st.sse = __dadd_rn(st.sse, __dmul_rn(e, e));
@@ -697,49 +703,6 @@ __device__ __forceinline__ uint32_t store_rows(const FusedArgs& a, const PSeg& p
   return pre;
 }
 
-// One child's candidate search over a lane's items: running prefix S'_L (child-centred,
-// rank carry included), the child position, the neighbour x; the exact gain (Reading
-// R19) at every valid position, strict > (the lowest position wins exact ties).
-struct Side {
-  double S, sc, Nd, jd;         // prefix (rank carry included), S' of the child, N, position (f64)
-  uint32_t jl, lo, hi;          // local position, valid local range [lo, hi)
-  float xp;                     // x of the previous entry of this child
-  double bg, bs, bjd;           // best gain, its S'_L and position
-  uint32_t bj;                  // best global position
-  float bxp, bx;
-  __device__ __forceinline__ void init(const PSeg& ps, int side, uint32_t ilo, uint32_t m, bool srch, double S0,
-                                       float x0, uint32_t j0) {
-    S = __dadd_rn(ps.soff[side], S0);
-    sc = ps.sc[side];
-    Nd = (double)ps.N[side];
-    jl = j0;
-    jd = (double)(ps.ioff[side] + j0);
-    lo = ilo > ps.ioff[side] ? ilo - ps.ioff[side] : 0u;
-    hi = (srch && ps.N[side] >= m + ps.ioff[side]) ? ps.N[side] - m - ps.ioff[side] + 1u : 0u;
-    xp = x0;
-    bg = -1.0;
-    bs = 0.0;
-    bjd = 0.0;
-    bj = 0xffffffffu;
-    bxp = bx = 0.f;
-  }
-  __device__ __forceinline__ void step_exact(float x, double d) {
-    if (jl >= lo && jl < hi && xp < x) {
-      const double g = split_gain_d(S, sc, jd, Nd);
-      if (g > bg) {  // strict >: the lowest position wins exact ties
-        bg = g;
-        bs = S;
-        bjd = jd;
-        bxp = xp;
-        bx = x;
-      }
-    }
-    S = __dadd_rn(S, d);
-    ++jl;
-    jd = __dadd_rn(jd, 1.0);
-    xp = x;
-  }
-};
 
 // y storage (int32 or f64, Reading R24) is decided on the device (root statistics): the
 // stage always has room for f64 entries; int32 lists copy and read half of it.
@@ -948,20 +911,42 @@ __global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArg
     if (full && (flags & (PS_SRCH0 | PS_SRCH1))) {
       // right position of my first in-range item: its segment-local index - lefts before
       const uint32_t jr0 = ib + (uint32_t)max(lane * kItems, e_lo) - nl;
-      // the two children one after the other (one running state live: registers)
+      // both children in one pass over my items (each item belongs to one child; the
+      // child's running state is selected per item: no divergence between the lanes)
+      const uint32_t io0 = ps.ioff[0], io1 = ps.ioff[1];
+      const uint32_t lo0 = ilo > io0 ? ilo - io0 : 0u, lo1 = ilo > io1 ? ilo - io1 : 0u;
+      const uint32_t hi0 = ((flags & PS_SRCH0) && ps.N[0] >= m + io0) ? ps.N[0] - m - io0 + 1u : 0u;
+      const uint32_t hi1 = ((flags & PS_SRCH1) && ps.N[1] >= m + io1) ? ps.N[1] - m - io1 + 1u : 0u;
+      double S0 = __dadd_rn(ps.soff[0], SL), S1 = __dadd_rn(ps.soff[1], SR);
+      uint32_t j0 = nl, j1 = jr0;
+      float xp0 = xl, xp1 = xr;
+      double bg0 = -1.0, bg1 = -1.0, bs0 = 0.0, bs1 = 0.0;
+      uint32_t bj0 = 0xffffffffu, bj1 = 0xffffffffu;
+      float bxp0 = 0.f, bx0 = 0.f, bxp1 = 0.f, bx1 = 0.f;
+      // exact gain (Reading R19) at every valid position; strict >: lowest position
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        const bool g = (lbyte >> j) & 1u, r = (rbyte >> j) & 1u;
+        const uint32_t jl = g ? j0 : j1;
+        const float xp = g ? xp0 : xp1;
+        if ((g || r) && jl >= (g ? lo0 : lo1) && jl < (g ? hi0 : hi1) && xp < xv[j]) {
+          const double S = g ? S0 : S1;
+          const double gn = split_gain_d(S, g ? ps.sc[0] : ps.sc[1], (double)((g ? io0 : io1) + jl),
+                                         (double)(g ? ps.N[0] : ps.N[1]));
+          if (g) {
+            if (gn > bg0) { bg0 = gn; bs0 = S; bj0 = io0 + jl; bxp0 = xp; bx0 = xv[j]; }
+          } else {
+            if (gn > bg1) { bg1 = gn; bs1 = S; bj1 = io1 + jl; bxp1 = xp; bx1 = xv[j]; }
+          }
+        }
+        if (g) { S0 = __dadd_rn(S0, dv[j]); ++j0; xp0 = xv[j]; }
+        if (r) { S1 = __dadd_rn(S1, dv[j]); ++j1; xp1 = xv[j]; }
+      }
 #pragma unroll 1
       for (int side = 0; side < 2; ++side) {
         if (!(flags & (side ? PS_SRCH1 : PS_SRCH0))) continue;  // warp-uniform
-        const uint32_t sb = side ? rbyte : lbyte;
-        Side sd;
-        sd.init(ps, side, ilo, m, true, side ? SR : SL, side ? xr : xl, side ? jr0 : nl);
-        // exact gain (Reading R19) at every valid position; strict >: lowest position
-#pragma unroll
-        for (int j = 0; j < kItems; ++j)
-          if ((sb >> j) & 1u) sd.step_exact(xv[j], dv[j]);
-        sd.bj = (uint32_t)sd.bjd;
-        const double bg = sd.bg;
-        const uint32_t bj = sd.bj;
+        const double bg = side ? bg1 : bg0;
+        const uint32_t bj = side ? bj1 : bj0;
         // warp max of the exact gains (>= 0: the f64 bit patterns order like the values;
         // key 0 = no candidate), then the lowest position holding it
         const unsigned long long key = bg >= 0.0 ? (unsigned long long)__double_as_longlong(bg) + 1ull : 0ull;
@@ -971,7 +956,8 @@ __global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArg
         if (kmax != 0ull) {
           const uint32_t jmin = __reduce_min_sync(0xffffffffu, key == kmax ? bj : 0xffffffffu);
           if (key == kmax && bj == jmin)  // exactly one lane holds the winner
-            put_cand(a, headc, ch, side, ps.cs[side], bg, sd.bs, mid_threshold(sd.bxp, sd.bx), jmin);
+            put_cand(a, headc, ch, side, ps.cs[side], bg, side ? bs1 : bs0,
+                     side ? mid_threshold(bxp1, bx1) : mid_threshold(bxp0, bx0), jmin);
         }
       }
     }
@@ -979,255 +965,123 @@ __global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArg
   }
 }
 
-// F_C for the chunks with segment heads inside (listed by fused_kernel): one warp per
-// chunk, the entries read directly (these chunks appear at deep levels, where nodes are
-// small); per lane a walk over its 8 entries' segments, segmented warp scans of the lanes'
-// runs for the candidate / statistics pieces of every segment in the chunk.
-__global__ void __launch_bounds__(kThreads) fused_general_kernel(FusedArgs a) {
+// F_C for the split segments of at most kSmallSeg entries (small list of chunk_plan_kernel):
+// a warp per segment, lane i = entry start + i.  The segment is one (head) piece: its
+// children's ranks are ballots, their prefix sums Kogge-Stone scans of the lanes, every
+// valid position is evaluated with the exact gain (Reading R19) and the lowest position of
+// the highest gain per child is recorded.  When the segment straddles a chunk boundary
+// the continuation statistics slot of its second chunk gets the identity.
+__global__ void __launch_bounds__(kThreads) fused_small_kernel(FusedArgs a) {
   const int lane = threadIdx.x & 31;
-  const int64_t ngen = a.ctl->nbig;
+  const int64_t ns = a.ctl->nsmall;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const uint64_t T = a.ctl->T[a.par];
   const bool full = a.ctl->nsrch > 0;
   const bool y32 = a.ctl->y32 != 0;
-  const uint32_t yb = y32 ? 4u : 8u;
   const uint32_t m = a.m;
   const uint32_t ilo = m > 1u ? m : 1u;
-  for (int64_t idx = gw; idx < ngen; idx += nw) {
-    const int64_t ch = (int64_t)a.big_list[idx];
-    const uint64_t cbase = (uint64_t)ch * kChunkW;
-    const float* sx = a.lx + cbase;
-    const uint32_t* sr = a.lr + cbase;
-    const unsigned char* sy = reinterpret_cast<const unsigned char*>(a.ly) + cbase * yb;
-    const uint32_t sid0 = __ldg(a.desc + ch);
-    const uint64_t ps_start = __ldg(&a.pseg[sid0].start);
-    const int32_t ps_f = __ldg(&a.pseg[sid0].f);
-    const bool headc = ps_start == cbase;
-    AggP carry = agg_ident();
-    if (full && !headc) carry = combine(a.bcarry[ch / kBlockChunks], a.cexcl[ch]);
-    float xv[kItems];
-    double yv[kItems];
-    const uint64_t pl = cbase + (uint64_t)(lane * kItems);
-#pragma unroll
-    for (int j = 0; j < kItems; ++j) {
-      const bool ok = pl + j < T;
-      xv[j] = ok ? sx[lane * kItems + j] : 0.f;
-      yv[j] = ok ? y_at(a.ly, (int64_t)(pl + j), y32) : 0.0;
+  const uint32_t lt = (1u << lane) - 1u;
+  for (int64_t idx = gw; idx < ns; idx += nw) {
+    SegCtx cx;
+    load_ctx(cx, a.pseg + a.small_list[idx]);
+    const uint32_t cnt = (uint32_t)(cx.end - cx.start);
+    const bool in = (uint32_t)lane < cnt;
+    const uint64_t p = cx.start + (uint64_t)lane;
+    float x = 0.f;
+    uint32_t row = 0u;
+    unsigned long long yraw = 0ull;
+    double y = 0.0;
+    bool g = false;
+    if (in) {
+      x = a.lx[p];
+      row = a.lr[p];
+      if (y32) {
+        const int32_t yi = reinterpret_cast<const int32_t*>(a.ly)[p];
+        yraw = (uint32_t)yi;
+        y = (double)yi;
+      } else {
+        yraw = reinterpret_cast<const unsigned long long*>(a.ly)[p];
+        y = __longlong_as_double((long long)yraw);
+      }
+      g = ((a.gm[p >> 3] >> (p & 7u)) & 1u) != 0u;
     }
-    const uint32_t gbyte = a.gm[cbase / 8 + lane];
-      // =================== general chunk: segment heads inside =======================
-      const uint64_t p0 = cbase + (uint64_t)(lane * kItems);
-      // pass 1: my trailing run's aggregate (segments walked from the chunk's first)
-      uint32_t sid = __ldg(a.desc + ch);
-      SegCtx cx;
-      load_ctx(cx, a.pseg + sid);
-      AggP run = agg_ident();
-      int lastL = -1, lastR = -1;
-      {
-        uint32_t s2 = sid;
-        uint64_t e2 = cx.end, st2 = cx.start;
-        uint32_t fl2 = cx.flags;
-        double c20 = cx.c[0], c21 = cx.c[1];
+    const int side = g ? 0 : 1;
+    const uint32_t Lb = __ballot_sync(0xffffffffu, in && g), Rb = __ballot_sync(0xffffffffu, in && !g);
+    const uint32_t mine = g ? Lb : Rb;
+    const uint32_t jl = __popc(mine & lt);  // my child's entries before mine (this rank)
+    // ---- partition: my child's run, in order
+    if (full && in && (cx.flags & (side ? PS_WR1 : PS_WR0))) {
+      const uint64_t dst = (side ? cx.os[1] : cx.os[0]) + jl;
+      a.ox[dst] = x;
+      a.orow[dst] = row;
+      if (y32) reinterpret_cast<uint32_t*>(a.oy)[dst] = (uint32_t)yraw;
+      else reinterpret_cast<unsigned long long*>(a.oy)[dst] = yraw;
+      if ((dst & (kChunkW - 1)) == 0) a.desc_next[dst / kChunkW] = (side ? cx.cs[1] : cx.cs[0]);
+    }
+    // ---- children's statistics from feature 0
+    if (cx.f == 0) {
+      StatQ q0 = statq_ident(), q1 = statq_ident();
+      if (in) {
+        if (g) stat_add(q0, y, cx.v[0], cx.c[0]);
+        else stat_add(q1, y, cx.v[1], cx.c[1]);
+      }
 #pragma unroll
-        for (int j = 0; j < kItems; ++j) {
-          const uint64_t p = p0 + j;
-          if (p < T) {
-            while (p >= e2) {
-              ++s2;
-              st2 = __ldg(&a.pseg[s2].start);
-              e2 = st2 + __ldg(&a.pseg[s2].cnt);
-              fl2 = __ldg(&a.pseg[s2].flags);
-              c20 = __ldg(&a.pseg[s2].c[0]);
-              c21 = __ldg(&a.pseg[s2].c[1]);
-            }
-            if (p == st2) {
-              run = agg_ident();
-              run.flag = 1u;
-              lastL = lastR = -1;
-            }
-            if (fl2 & PS_SPLIT) {
-              if ((gbyte >> j) & 1u) {
-                run.nl += 1u;
-                run.sl = __dadd_rn(run.sl, __dsub_rn(yv[j], c20));
-                lastL = j;
-              } else {
-                run.sr = __dadd_rn(run.sr, __dsub_rn(yv[j], c21));
-                lastR = j;
-              }
-            }
-          }
+      for (int off = 16; off > 0; off >>= 1) {
+        q0.sse = __dadd_rn(q0.sse, __shfl_xor_sync(0xffffffffu, q0.sse, off));
+        q0.ymin = fmin(q0.ymin, __shfl_xor_sync(0xffffffffu, q0.ymin, off));
+        q0.ymax = fmax(q0.ymax, __shfl_xor_sync(0xffffffffu, q0.ymax, off));
+        q0.s1 = __dadd_rn(q0.s1, __shfl_xor_sync(0xffffffffu, q0.s1, off));
+        q1.sse = __dadd_rn(q1.sse, __shfl_xor_sync(0xffffffffu, q1.sse, off));
+        q1.ymin = fmin(q1.ymin, __shfl_xor_sync(0xffffffffu, q1.ymin, off));
+        q1.ymax = fmax(q1.ymax, __shfl_xor_sync(0xffffffffu, q1.ymax, off));
+        q1.s1 = __dadd_rn(q1.s1, __shfl_xor_sync(0xffffffffu, q1.s1, off));
+      }
+      if (lane == 0) {
+        put_stat(a, true, 0, 0, cx.kid, q0);
+        if (!(cx.flags & PS_ALLLEFT)) put_stat(a, true, 0, 1, cx.kid + 1, q1);
+        const int64_t c0 = (int64_t)(cx.start / kChunkW), c1 = (int64_t)((cx.end - 1) / kChunkW);
+        if (c1 > c0) {
+          const Stat z{0.0, INFINITY, -INFINITY, 0.0};
+          a.cont_stat[2 * c1] = z;
+          a.cont_stat[2 * c1 + 1] = z;
         }
       }
-      if (lastL >= 0) run.xl = sx[lane * kItems + lastL];
-      if (lastR >= 0) run.xr = sx[lane * kItems + lastR];
-      AggP wagg;
-      const AggP ex = warp_excl_seg(run, agg_ident(), wagg);
-      const AggP E = combine(carry, ex);  // the open segment's state at my first item
-      // pass 2: positions, candidates, statistics, stores
-      const bool stats_chunk = ps_f == 0;
-      // walk to the segment of my first item
-      {
-        uint64_t q = p0 < T ? p0 : T - 1;
-        while (q >= cx.end) load_ctx(cx, a.pseg + (++sid));
-      }
-      uint32_t nl = E.nl;
-      double SL = E.sl, SR = E.sr;
-      float xl = isnan(E.xl) ? cx.xp[0] : E.xl, xr = isnan(E.xr) ? cx.xp[1] : E.xr;
-      // runs: the one open at my first item (its part before my first head: "first")
-      // and the current one
-      ArgQ fa0 = argq_ident(), fa1 = argq_ident(), ca0 = argq_ident(), ca1 = argq_ident();
-      StatQ fs0 = statq_ident(), fs1 = statq_ident(), cs0 = statq_ident(), cs1 = statq_ident();
-      bool seen = false;
-      // ids of the run's segment
-      uint32_t rcs0 = cx.cs[0], rcs1 = cx.cs[1], rkid = cx.kid, rfl = cx.flags;
-      int rf = cx.f;
-      const uint32_t fcs0 = cx.cs[0], fcs1 = cx.cs[1], fkid = cx.kid, ffl = cx.flags;
-      const int ff = cx.f;
-      bool item0_head = false;
-#pragma unroll
-      for (int j = 0; j < kItems; ++j) {
-        const uint64_t p = p0 + j;
-        if (p < T) {
-          while (p >= cx.end) load_ctx(cx, a.pseg + (++sid));
-          if (p == cx.start) {
-            if (j == 0) item0_head = true;
-            if (!seen) {
-              fa0 = ca0; fa1 = ca1; fs0 = cs0; fs1 = cs1;
-            } else {
-              // a run that started at a head inside this lane ends here: complete piece
-              if (full && (rfl & PS_SPLIT)) {
-                if ((rfl & PS_SRCH0) && ca0.gain >= 0.0) put_cand(a, true, ch, 0, rcs0, ca0.gain, ca0.sl, ca0.thr, ca0.j);
-                if ((rfl & PS_SRCH1) && ca1.gain >= 0.0) put_cand(a, true, ch, 1, rcs1, ca1.gain, ca1.sl, ca1.thr, ca1.j);
-              }
-              if (rf == 0 && (rfl & PS_SPLIT)) {
-                put_stat(a, true, ch, 0, rkid, cs0);
-                if (!(rfl & PS_ALLLEFT)) put_stat(a, true, ch, 1, rkid + 1, cs1);
-              }
-            }
-            seen = true;
-            ca0 = argq_ident(); ca1 = argq_ident(); ca0.flag = ca1.flag = 1u;
-            cs0 = statq_ident(); cs1 = statq_ident(); cs0.flag = cs1.flag = 1u;
-            nl = 0u;
-            SL = 0.0;
-            SR = 0.0;
-            xl = cx.xp[0];
-            xr = cx.xp[1];
-            rcs0 = cx.cs[0]; rcs1 = cx.cs[1]; rkid = cx.kid; rfl = cx.flags; rf = cx.f;
-          }
-          if (cx.flags & PS_SPLIT) {
-            const float x = xv[j];
-            const double y = yv[j];
-            const uint32_t i = (uint32_t)(p - cx.start);
-            if ((gbyte >> j) & 1u) {
-              if (full) {
-                const uint32_t jg = cx.ioff[0] + nl;
-                if ((cx.flags & PS_SRCH0) && jg >= ilo && cx.N[0] - jg >= m && xl < x) {
-                  const double S = __dadd_rn(cx.soff[0], SL);
-                  const double g = split_gain_d(S, cx.sc[0], (double)jg, (double)cx.N[0]);
-                  if (g > ca0.gain) { ca0.gain = g; ca0.j = jg; ca0.sl = S; ca0.thr = mid_threshold(xl, x); }
-                }
-                if (cx.flags & PS_WR0)
-                  store_entry(a, y32, cx.os[0] + nl, x, sr[lane * kItems + j], sy + (size_t)(lane * kItems + j) * yb, cx.cs[0]);
-              }
-              if (cx.f == 0) stat_add(cs0, y, cx.v[0], cx.c[0]);
-              SL = __dadd_rn(SL, __dsub_rn(y, cx.c[0]));
-              ++nl;
-              xl = x;
-            } else {
-              if (full) {
-                const uint32_t jr = i - nl;
-                const uint32_t jg = cx.ioff[1] + jr;
-                if ((cx.flags & PS_SRCH1) && jg >= ilo && cx.N[1] - jg >= m && xr < x) {
-                  const double S = __dadd_rn(cx.soff[1], SR);
-                  const double g = split_gain_d(S, cx.sc[1], (double)jg, (double)cx.N[1]);
-                  if (g > ca1.gain) { ca1.gain = g; ca1.j = jg; ca1.sl = S; ca1.thr = mid_threshold(xr, x); }
-                }
-                if (cx.flags & PS_WR1)
-                  store_entry(a, y32, cx.os[1] + jr, x, sr[lane * kItems + j], sy + (size_t)(lane * kItems + j) * yb, cx.cs[1]);
-              }
-              if (cx.f == 0) stat_add(cs1, y, cx.v[1], cx.c[1]);
-              SR = __dadd_rn(SR, __dsub_rn(y, cx.c[1]));
-              xr = x;
-            }
-          }
-        }
-      }
-      if (!seen) { fa0 = ca0; fa1 = ca1; fs0 = cs0; fs1 = cs1; }
-      // segmented scans of the lane trails (the last run, flagged when it began at a head)
-      ArgQ ta0 = ca0, ta1 = ca1;
-      ta0.flag = ta1.flag = seen ? 1u : 0u;
-      ArgQ w0, w1;
-      const ArgQ ax0 = warp_excl_seg(ta0, argq_ident(), w0);
-      const ArgQ ax1 = warp_excl_seg(ta1, argq_ident(), w1);
-      StatQ sx0 = statq_ident(), sx1 = statq_ident();
-      if (stats_chunk) {
-        StatQ ts0 = cs0, ts1 = cs1, v0, v1;
-        ts0.flag = ts1.flag = seen ? 1u : 0u;
-        sx0 = warp_excl_seg(ts0, statq_ident(), v0);
-        sx1 = warp_excl_seg(ts1, statq_ident(), v1);
-      }
-      // the segment open at my first item ends in this lane: its piece = earlier lanes + "first"
-      if (seen && !(lane == 0 && item0_head) && !item0_head) {
-        const bool h = ax0.flag != 0;  // its head lies in an earlier lane of this chunk
-        if (full && (ffl & PS_SPLIT)) {
-          const ArgQ d0 = combine(ax0, fa0), d1 = combine(ax1, fa1);
-          if ((ffl & PS_SRCH0) && d0.gain >= 0.0) put_cand(a, h, ch, 0, fcs0, d0.gain, d0.sl, d0.thr, d0.j);
-          if ((ffl & PS_SRCH1) && d1.gain >= 0.0) put_cand(a, h, ch, 1, fcs1, d1.gain, d1.sl, d1.thr, d1.j);
-        }
-        if (ff == 0 && (ffl & PS_SPLIT)) {
-          put_stat(a, h, ch, 0, fkid, combine(sx0, fs0));
-          if (!(ffl & PS_ALLLEFT)) put_stat(a, h, ch, 1, fkid + 1, combine(sx1, fs1));
-        }
-      } else if (seen && item0_head && lane > 0) {
-        // my first item is a head: the segment open before me ended in an earlier lane;
-        // its piece (earlier lanes only) is closed here
-        // the previous non-empty segment: the one holding position p0 - 1
-        SegCtx pc;
-        {
-          uint32_t t2 = __ldg(a.desc + ch);
-          load_ctx(pc, a.pseg + t2);
-          while (p0 - 1 >= pc.end) load_ctx(pc, a.pseg + (++t2));
-        }
-        const bool h = ax0.flag != 0;
-        if (full && (pc.flags & PS_SPLIT)) {
-          if ((pc.flags & PS_SRCH0) && ax0.gain >= 0.0) put_cand(a, h, ch, 0, pc.cs[0], ax0.gain, ax0.sl, ax0.thr, ax0.j);
-          if ((pc.flags & PS_SRCH1) && ax1.gain >= 0.0) put_cand(a, h, ch, 1, pc.cs[1], ax1.gain, ax1.sl, ax1.thr, ax1.j);
-        }
-        if (pc.f == 0 && (pc.flags & PS_SPLIT)) {
-          put_stat(a, h, ch, 0, pc.kid, sx0);
-          if (!(pc.flags & PS_ALLLEFT)) put_stat(a, h, ch, 1, pc.kid + 1, sx1);
-        }
-      }
-      // the last lane closes the segment open at the chunk's end
-      if (lane == 31) {
-        SegCtx lc;
-        bool lh;
-        ArgQ d0, d1;
-        StatQ e0, e1;
-        if (p0 < T && seen) {
-          lc = cx;  // my last run began at a head in my items
-          lh = true;
-          d0 = ca0; d1 = ca1; e0 = cs0; e1 = cs1;
-        } else {
-          // no head in my items (or no items): earlier lanes + my run
-          const uint64_t last = (cbase + kChunkW <= T ? cbase + kChunkW : T) - 1;
-          uint32_t t2 = __ldg(a.desc + ch);
-          load_ctx(lc, a.pseg + t2);
-          while (last >= lc.end) load_ctx(lc, a.pseg + (++t2));
-          lh = ax0.flag != 0;
-          d0 = combine(ax0, ca0); d1 = combine(ax1, ca1);
-          e0 = combine(sx0, cs0); e1 = combine(sx1, cs1);
-        }
-        if (full && (lc.flags & PS_SPLIT)) {
-          if ((lc.flags & PS_SRCH0) && d0.gain >= 0.0) put_cand(a, lh, ch, 0, lc.cs[0], d0.gain, d0.sl, d0.thr, d0.j);
-          if ((lc.flags & PS_SRCH1) && d1.gain >= 0.0) put_cand(a, lh, ch, 1, lc.cs[1], d1.gain, d1.sl, d1.thr, d1.j);
-        }
-        if (lc.f == 0 && (lc.flags & PS_SPLIT)) {
-          put_stat(a, lh, ch, 0, lc.kid, e0);
-          if (!(lc.flags & PS_ALLLEFT)) put_stat(a, lh, ch, 1, lc.kid + 1, e1);
-        }
-      }
+    }
+    if (!full || !(cx.flags & (PS_SRCH0 | PS_SRCH1))) continue;  // warp-uniform
+    // ---- prefix sums of (y - c_child) over my child's earlier entries (exclusive: the
+    // inclusive scan of the lane below; non-members add +0.0, exact)
+    const double dv = in ? __dsub_rn(y, side ? cx.c[1] : cx.c[0]) : 0.0;
+    double il = (in && g) ? dv : 0.0, ir = (in && !g) ? dv : 0.0;
+    warp_incl2(il, ir);
+    double el = __shfl_up_sync(0xffffffffu, il, 1), er = __shfl_up_sync(0xffffffffu, ir, 1);
+    if (lane == 0) el = er = 0.0;
+    // x of my child's previous entry (this rank), else the rank carry (NaN: none)
+    const uint32_t below = mine & lt;
+    const float xo = __shfl_sync(0xffffffffu, x, below ? 31 - __clz(below) : 0);
+    const float xp = below ? xo : (side ? cx.xp[1] : cx.xp[0]);
+    // ---- my position's candidate (as fused_kernel: valid local range [lo, hi), x_prev < x)
+    double gain = -1.0, S = 0.0;
+    const uint32_t io = (side ? cx.ioff[1] : cx.ioff[0]), Nc = (side ? cx.N[1] : cx.N[0]);
+    if (in && (cx.flags & (side ? PS_SRCH1 : PS_SRCH0))) {
+      const uint32_t lo = ilo > io ? ilo - io : 0u;
+      const uint32_t hi = Nc >= m + io ? Nc - m - io + 1u : 0u;
+      S = __dadd_rn((side ? cx.soff[1] : cx.soff[0]), side ? er : el);
+      if (jl >= lo && jl < hi && xp < x) gain = split_gain_d(S, (side ? cx.sc[1] : cx.sc[0]), (double)(io + jl), (double)Nc);
+    }
+    const uint32_t jg = io + jl;
+#pragma unroll 1
+    for (int sd = 0; sd < 2; ++sd) {
+      if (!(cx.flags & (sd ? PS_SRCH1 : PS_SRCH0))) continue;  // warp-uniform
+      const unsigned long long key =
+          (side == sd && gain >= 0.0) ? (unsigned long long)__double_as_longlong(gain) + 1ull : 0ull;
+      const uint32_t khi = __reduce_max_sync(0xffffffffu, (uint32_t)(key >> 32));
+      const uint32_t klo = __reduce_max_sync(0xffffffffu, (uint32_t)(key >> 32) == khi ? (uint32_t)key : 0u);
+      const unsigned long long kmax = ((unsigned long long)khi << 32) | klo;
+      if (kmax == 0ull) continue;
+      const uint32_t jmin = __reduce_min_sync(0xffffffffu, key == kmax ? jg : 0xffffffffu);
+      if (key == kmax && jg == jmin)
+        put_cand(a, true, 0, sd, (sd ? cx.cs[1] : cx.cs[0]), gain, S, mid_threshold(xp, x), jg);
+    }
   }
 }
 
@@ -1261,9 +1115,10 @@ dt_status level_agg_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t 
   a.gen_list = b.gen_list;
   a.ctl = b.ctl;
   a.par = la.par;
+  a.d = (uint32_t)la.d;
   a.nwords = b.nwords4;
   chunk_plan_kernel<<<num_sms() * 8, 256, 0, s>>>(b.ctl, la.par, la.d, b.desc[la.par], b.pseg, b.agg, b.fast_list,
-                                                  b.gen_list, b.unit_list, b.big_list);
+                                                  b.gen_list, b.unit_list, b.small_list, la.level < 0);
   DT_CK(cudaGetLastError());
   const size_t bytes = sizeof(uint32_t) * (size_t)b.nwords4;
   if ((int64_t)bytes <= kMaxSmemBits) {
@@ -1309,17 +1164,18 @@ dt_status level_fused_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_
   a.ctl = b.ctl;
   a.par = la.par;
   a.level = (uint32_t)(la.level + 1);
+  a.d = (uint32_t)la.d;
   a.m = (uint32_t)std::min<int64_t>(la.min_leaf, 0x7fffffff);
   a.ystride = 0;
   a.stage_bytes = 0;
   const size_t sm = fused_smem();
   a.unit_list = b.unit_list;
-  a.big_list = b.big_list;
+  a.small_list = b.small_list;
   auto k = fused_kernel;
   DT_CK(cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
   k<<<grid_for((const void*)k, kThreads, sm), kThreads, sm, s>>>(a);
   DT_CK(cudaGetLastError());
-  fused_general_kernel<<<grid_for((const void*)fused_general_kernel, kThreads, 0), kThreads, 0, s>>>(a);
+  fused_small_kernel<<<grid_for((const void*)fused_small_kernel, kThreads, 0), kThreads, 0, s>>>(a);
   DT_CK(cudaGetLastError());
   return DT_OK;
 }

@@ -173,7 +173,7 @@ __global__ void __launch_bounds__(256) root_tables_kernel(const Ctl* __restrict_
     p.soff[0] = p.soff[1] = 0.0;
     p.xprev[0] = p.xprev[1] = __int_as_float(0x7fc00000);
     p.kid = 0;
-    p.pad = 0;
+    p.glim = 0;
     pseg[f] = p;
   }
   (void)ctl;
@@ -603,7 +603,7 @@ __global__ void __launch_bounds__(256) root_tables_sharded_kernel(Ctl* ctl, cons
     p.soff[0] = p.soff[1] = soff;
     p.xprev[0] = p.xprev[1] = xprev;
     p.kid = 0;
-    p.pad = 0;
+    p.glim = 0;
     pseg[f] = p;
   }
   (void)world;
