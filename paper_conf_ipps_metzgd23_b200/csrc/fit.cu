@@ -227,7 +227,7 @@ __global__ void __launch_bounds__(256) select_kernel(SelectArgs a) {
     a.log[a.level].T_next = 0;
     a.log[a.level].K_next = 0;
   }
-  if (K > gridDim.x) {
+  if (K > gridDim.x / 4) {
     // many (small) nodes: one warp per node, no block barriers
     const int nwarps = blockDim.x >> 5;
     for (uint32_t k = blockIdx.x * nwarps + w; k < K; k += gridDim.x * nwarps) {
@@ -347,18 +347,19 @@ struct NumberArgs {
   int64_t min_leaf;
   dt_node* out;
   LevelLog* log;
+  uint32_t* wst;  // per split node: its written children's first position (scan -> children_kernel)
 };
 
-// Single block: BFS numbering (children appended left, right in node order), the
-// children's exact statistics, and (P = 1) their positions in the next level's lists
-// (written children = searchable children, in node order).
+// Single block: BFS numbering (children appended left, right in node order) and (P = 1)
+// the children's positions in the next level's lists (written children = searchable
+// children, in node order): three block scans over the nodes.  children_kernel then
+// builds the children (exact statistics) on the whole grid.
 __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
   __shared__ unsigned long long sh_a[33], sh_b[33], sh_c[33];
   __shared__ unsigned long long base_split, base_rows, base_srch;
   const uint32_t K = a.ctl->K[a.par];
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   const int next_id0 = a.ctl->next_id;
-  const int int_mode = a.ctl->int_mode;
   const int child_depth = a.level + 1;
   const bool depth_ok = (a.max_depth < 0) || (child_depth < a.max_depth);
   if (tid == 0) { base_split = 0; base_rows = 0; base_srch = 0; }
@@ -368,8 +369,7 @@ __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
     const bool in = k < K;
     const Decision dc = in ? a.dec[k] : Decision{-1, 0, 0, 0, 0.0, 0.0};
     const bool sp = in && dc.f >= 0;
-    const NodeL nd = in ? a.nodes[k] : NodeL{};
-    const uint32_t nl = sp ? dc.nl : 0u, nr = sp ? nd.N - dc.nl : 0u;
+    const uint32_t nl = sp ? dc.nl : 0u, nr = sp ? a.nodes[k].N - dc.nl : 0u;
     const bool sl_ok = sp && depth_ok && (int64_t)nl >= 2 * a.min_leaf;
     const bool sr_ok = sp && depth_ok && (int64_t)nr >= 2 * a.min_leaf;
     // three exclusive scans over the block: splits, written rows, searchable children
@@ -385,63 +385,27 @@ __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
     }
     if (lane == 31) { sh_a[w] = ia; sh_b[w] = ib; sh_c[w] = ic; }
     __syncthreads();
-    if (tid == 0) {
-      unsigned long long ra = 0, rb = 0, rc = 0;
-      for (int i = 0; i < (int)(blockDim.x >> 5); ++i) {
-        const unsigned long long ta = sh_a[i], tb = sh_b[i], tc = sh_c[i];
-        sh_a[i] = ra; sh_b[i] = rb; sh_c[i] = rc;
-        ra += ta; rb += tb; rc += tc;
+    if (w == 0) {  // the 32 warp totals: exclusive prefixes (and the tile totals in [32])
+      const unsigned long long ta = sh_a[lane], tb = sh_b[lane], tc = sh_c[lane];
+      unsigned long long xa = ta, xb = tb, xc = tc;
+#pragma unroll
+      for (int dd = 1; dd < 32; dd <<= 1) {
+        const unsigned long long oa = __shfl_up_sync(0xffffffffu, xa, dd);
+        const unsigned long long ob = __shfl_up_sync(0xffffffffu, xb, dd);
+        const unsigned long long oc = __shfl_up_sync(0xffffffffu, xc, dd);
+        if (lane >= dd) { xa += oa; xb += ob; xc += oc; }
       }
-      sh_a[32] = ra; sh_b[32] = rb; sh_c[32] = rc;
+      sh_a[lane] = xa - ta; sh_b[lane] = xb - tb; sh_c[lane] = xc - tc;
+      if (lane == 31) { sh_a[32] = xa; sh_b[32] = xb; sh_c[32] = xc; }
     }
     __syncthreads();
     const uint32_t rank = (uint32_t)(base_split + sh_a[w] + (ia - va));
     const unsigned long long rows_ex = base_rows + sh_b[w] + (ib - vb);
     if (sp) {
-      const int lid = next_id0 + 2 * (int)rank;
-      a.out[nd.id].left = lid;
-      a.out[nd.id].right = lid + 1;
       Decision d2 = dc;
       d2.kid = 2 * rank;
       a.dec[k] = d2;
-      NodeL L, R;
-      L.N = nl;
-      R.N = nr;
-      L.id = lid;
-      R.id = lid + 1;
-      L.searchable = sl_ok ? 1 : 0;
-      R.searchable = sr_ok ? 1 : 0;
-      L.parent = R.parent = k;
-      L.side = 0;
-      R.side = 1;
-      L.wstart = (uint32_t)rows_ex;
-      R.wstart = (uint32_t)(rows_ex + (sl_ok ? nl : 0u));
-      L.pad[0] = L.pad[1] = L.pad[2] = L.pad[3] = 0;
-      R.pad[0] = R.pad[1] = R.pad[2] = R.pad[3] = 0;
-      const double slp = dc.sl;                  // parent-centred S'_L
-      const double srp = __dsub_rn(nd.sc, slp);  // parent-centred S'_R
-      if (int_mode) {
-        const long long cp = (long long)nd.c;
-        const long long SL = (long long)nl * cp + (long long)slp;
-        const long long SR = (long long)nr * cp + (long long)srp;
-        const long long cl = floor_div_ll(SL, nl), cr = floor_div_ll(SR, nr);
-        L.c = (double)cl;
-        R.c = (double)cr;
-        L.v = __ddiv_rn((double)SL, (double)nl);
-        R.v = __ddiv_rn((double)SR, (double)nr);
-        L.sc = (double)(SL - (long long)nl * cl);
-        R.sc = (double)(SR - (long long)nr * cr);
-      } else {
-        L.v = __dadd_rn(nd.c, __ddiv_rn(slp, (double)nl));
-        R.v = __dadd_rn(nd.c, __ddiv_rn(srp, (double)nr));
-        L.c = L.v;
-        R.c = R.v;
-        // re-centre: S'_child = S'_(parent-centred) - n * (c_child - c_parent)
-        L.sc = __dsub_rn(slp, __dmul_rn((double)nl, __dsub_rn(L.c, nd.c)));
-        R.sc = __dsub_rn(srp, __dmul_rn((double)nr, __dsub_rn(R.c, nd.c)));
-      }
-      a.next[2 * rank] = L;
-      a.next[2 * rank + 1] = R;
+      a.wst[k] = (uint32_t)rows_ex;
     }
     __syncthreads();
     if (tid == 0) { base_split += sh_a[32]; base_rows += sh_b[32]; base_srch += sh_c[32]; }
@@ -449,6 +413,7 @@ __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
   }
   if (tid == 0) {
     const int np = a.par ^ 1;
+    a.ctl->next_id_prev = next_id0;
     a.ctl->K[np] = (uint32_t)(2 * base_split);
     a.ctl->A2 = (uint32_t)base_rows;
     a.ctl->T[np] = base_rows * (unsigned long long)a.d;
@@ -459,6 +424,67 @@ __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
       a.log[a.level].T_next = base_rows * (unsigned long long)a.d;
       a.log[a.level].K_next = (uint32_t)(2 * base_split);
     }
+  }
+}
+
+// The children of every split node (grid-stride): ids, exact statistics (Reading R17 /
+// real mode), searchability, list positions; the parent's child links.
+__global__ void __launch_bounds__(256) children_kernel(NumberArgs a) {
+  const uint32_t K = a.ctl->K[a.par];
+  const int next_id0 = a.ctl->next_id_prev;
+  const int int_mode = a.ctl->int_mode;
+  const int child_depth = a.level + 1;
+  const bool depth_ok = (a.max_depth < 0) || (child_depth < a.max_depth);
+  for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < K; k += gridDim.x * blockDim.x) {
+    const Decision dc = a.dec[k];
+    if (dc.f < 0) continue;
+    const NodeL nd = a.nodes[k];
+    const uint32_t rank = dc.kid >> 1;
+    const uint32_t nl = dc.nl, nr = nd.N - dc.nl;
+    const bool sl_ok = depth_ok && (int64_t)nl >= 2 * a.min_leaf;
+    const bool sr_ok = depth_ok && (int64_t)nr >= 2 * a.min_leaf;
+    const unsigned long long rows_ex = a.wst[k];
+    const int lid = next_id0 + 2 * (int)rank;
+    a.out[nd.id].left = lid;
+    a.out[nd.id].right = lid + 1;
+    NodeL L, R;
+    L.N = nl;
+    R.N = nr;
+    L.id = lid;
+    R.id = lid + 1;
+    L.searchable = sl_ok ? 1 : 0;
+    R.searchable = sr_ok ? 1 : 0;
+    L.parent = R.parent = k;
+    L.side = 0;
+    R.side = 1;
+    L.wstart = (uint32_t)rows_ex;
+    R.wstart = (uint32_t)(rows_ex + (sl_ok ? nl : 0u));
+    L.pad[0] = L.pad[1] = L.pad[2] = L.pad[3] = 0;
+    R.pad[0] = R.pad[1] = R.pad[2] = R.pad[3] = 0;
+    const double slp = dc.sl;                  // parent-centred S'_L
+    const double srp = __dsub_rn(nd.sc, slp);  // parent-centred S'_R
+    if (int_mode) {
+      const long long cp = (long long)nd.c;
+      const long long SL = (long long)nl * cp + (long long)slp;
+      const long long SR = (long long)nr * cp + (long long)srp;
+      const long long cl = floor_div_ll(SL, nl), cr = floor_div_ll(SR, nr);
+      L.c = (double)cl;
+      R.c = (double)cr;
+      L.v = __ddiv_rn((double)SL, (double)nl);
+      R.v = __ddiv_rn((double)SR, (double)nr);
+      L.sc = (double)(SL - (long long)nl * cl);
+      R.sc = (double)(SR - (long long)nr * cr);
+    } else {
+      L.v = __dadd_rn(nd.c, __ddiv_rn(slp, (double)nl));
+      R.v = __dadd_rn(nd.c, __ddiv_rn(srp, (double)nr));
+      L.c = L.v;
+      R.c = R.v;
+      // re-centre: S'_child = S'_(parent-centred) - n * (c_child - c_parent)
+      L.sc = __dsub_rn(slp, __dmul_rn((double)nl, __dsub_rn(L.c, nd.c)));
+      R.sc = __dsub_rn(srp, __dmul_rn((double)nr, __dsub_rn(R.c, nd.c)));
+    }
+    a.next[2 * rank] = L;
+    a.next[2 * rank + 1] = R;
   }
 }
 
@@ -866,6 +892,7 @@ dt_status fit_alloc(FitBufs& b, int64_t n, int64_t n_global, int32_t d, int32_t 
   }
   GET(b.pseg, b.segcap);
   GET(b.dec, b.kcap);
+  GET(b.wst, b.kcap);
   GET(b.dec_root, 1);
   GET(b.agg, b.max_chunks);
   GET(b.cexcl, b.max_chunks);
@@ -1029,7 +1056,9 @@ dt_status fit_levels(const FitBufs& b, int32_t d, int32_t max_depth, int64_t min
     na.out = b.dout;
     na.log = b.lvlog;
     pr = prof_begin(PK_NUMBER, s, 2);
+    na.wst = b.wst;
     number_kernel<<<1, 1024, 0, s>>>(na);
+    children_kernel<<<g_tab, 256, 0, s>>>(na);
     tables_kernel<<<g_tab, 256, 0, s>>>(ctl, par, d, b.nodes[par ^ 1], b.dec, b.segs[par], b.segs[par ^ 1], b.pseg, 0,
                                         b.unit_list, b.small_list);
     prof_end(pr, s, 0.0);
@@ -1541,7 +1570,9 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
     na.out = b.dout;
     na.log = b.lvlog;
     pr = prof_begin(PK_NUMBER, s, 1);
+    na.wst = b.wst;
     number_kernel<<<1, 1024, 0, s>>>(na);
+    children_kernel<<<g_tab, 256, 0, s>>>(na);
     prof_end(pr, s, 0.0);
     DT_CK(cudaGetLastError());
     uint32_t hk[2], hsrch = 0;

@@ -176,6 +176,7 @@ struct Ctl {
   uint32_t K[2];             // nodes at the level, by level parity
   uint32_t A2;               // P = 1: rows per list of the next level (written children)
   int32_t next_id;           // output nodes allocated so far
+  int32_t next_id_prev;      // next_id before the current level's children (number -> children_kernel)
   int32_t int_mode;
   int32_t y32;               // the level lists hold y as int32 (Reading R24)
   int32_t max_depth_seen;
@@ -268,6 +269,7 @@ struct FitBufs {
   SegT* segs[2];
   PSeg* pseg;
   Decision* dec;
+  uint32_t* wst;  // number -> children_kernel: written-children offset per split node
   Decision* dec_root;  // the virtual-root decision (all rows to node 0)
   uint32_t* desc[2];
   AggP *agg, *cexcl, *bagg, *bcarry;

@@ -49,18 +49,28 @@ __global__ void __launch_bounds__(256) root_reduce_kernel(const double* __restri
   if (threadIdx.x == 0) parts[blockIdx.x] = sh[0];
 }
 
-__global__ void root_finalize_kernel(const RootPart* parts, int nparts, int64_t n, Ctl* ctl) {
-  if (threadIdx.x != 0) return;
+// Folds of the block parts in index order (one thread; the parts are staged in shared
+// memory by the whole block, 256 at a time, so the fold does not wait on each load).
+__global__ void __launch_bounds__(256) root_finalize_kernel(const RootPart* parts, int nparts, int64_t n, Ctl* ctl) {
+  __shared__ RootPart sp[256];
   double s = 0, c = 0, mn = INFINITY, mx = -INFINITY;
   int integral = 1, finite = 1;
-  for (int i = 0; i < nparts; ++i) {
-    neu_add(s, c, parts[i].s);
-    neu_add(s, c, parts[i].c);
-    mn = fmin(mn, parts[i].mn);
-    mx = fmax(mx, parts[i].mx);
-    integral &= parts[i].integral;
-    finite &= parts[i].finite;
+  for (int i0 = 0; i0 < nparts; i0 += 256) {
+    __syncthreads();
+    if (i0 + (int)threadIdx.x < nparts) sp[threadIdx.x] = parts[i0 + threadIdx.x];
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      for (int i = 0; i < min(256, nparts - i0); ++i) {
+        neu_add(s, c, sp[i].s);
+        neu_add(s, c, sp[i].c);
+        mn = fmin(mn, sp[i].mn);
+        mx = fmax(mx, sp[i].mx);
+        integral &= sp[i].integral;
+        finite &= sp[i].finite;
+      }
+    }
   }
+  if (threadIdx.x != 0) return;
   ctl->ysum = __dadd_rn(s, c);
   ctl->ymin = mn;
   ctl->ymax = mx;
@@ -94,11 +104,19 @@ __global__ void __launch_bounds__(256) root_center_kernel(const double* __restri
   if (threadIdx.x == 0) parts[blockIdx.x] = sh[0];
 }
 
-__global__ void root_init_kernel(const double* parts, int nparts, int64_t n, int d, int32_t max_depth,
-                                 int64_t min_leaf, Ctl* ctl, NodeL* nodes0, Decision* dec_root) {
-  if (threadIdx.x != 0) return;
+__global__ void __launch_bounds__(256) root_init_kernel(const double* parts, int nparts, int64_t n, int d,
+                                                        int32_t max_depth, int64_t min_leaf, Ctl* ctl, NodeL* nodes0,
+                                                        Decision* dec_root) {
+  __shared__ double sp[256];
   double s = 0, cc = 0;
-  for (int i = 0; i < nparts; ++i) neu_add(s, cc, parts[i]);
+  for (int i0 = 0; i0 < nparts; i0 += 256) {
+    __syncthreads();
+    if (i0 + (int)threadIdx.x < nparts) sp[threadIdx.x] = parts[i0 + threadIdx.x];
+    __syncthreads();
+    if (threadIdx.x == 0)
+      for (int i = 0; i < min(256, nparts - i0); ++i) neu_add(s, cc, sp[i]);
+  }
+  if (threadIdx.x != 0) return;
   NodeL nd;
   nd.N = (uint32_t)n;
   nd.id = 0;
@@ -180,50 +198,6 @@ __global__ void __launch_bounds__(256) root_tables_kernel(const Ctl* __restrict_
 }
 
 
-// keys[f*n + r] = flip(x[r][f]); vals = row0 + r.  X row-major -> feature-major via smem.
-__global__ void __launch_bounds__(256) presort_keys_kernel(const float* __restrict__ X, int64_t n, int d,
-                                                           uint32_t* __restrict__ keys,
-                                                           uint32_t* __restrict__ vals, Ctl* ctl, int64_t row0,
-                                                           int rb) {
-  extern __shared__ float tileX[];  // rb rows x d
-  const int64_t r0 = (int64_t)blockIdx.x * rb;
-  const int rows = (int)min((int64_t)rb, n - r0);
-  const int64_t base = r0 * d;
-  const int tot = rows * d;
-  bool bad = false;
-  for (int i = threadIdx.x; i < tot; i += blockDim.x) {
-    float v = X[base + i];
-    if (!isfinite(v)) bad = true;
-    tileX[i] = v;
-  }
-  if (__syncthreads_or(bad) && threadIdx.x == 0) ctl->nonfinite = 1;
-  for (int f = 0; f < d; ++f) {
-    if (threadIdx.x < rows) {
-      const int64_t r = r0 + threadIdx.x;
-      keys[(int64_t)f * n + r] = flip_f32(tileX[threadIdx.x * d + f]);
-      vals[(int64_t)f * n + r] = (uint32_t)(row0 + r);
-    }
-  }
-}
-
-// SoA level-0 lists from the sorted pairs: x = unflip(key), row = val, y = y[row].
-__global__ void __launch_bounds__(256) presort_build_kernel(const uint32_t* __restrict__ keys,
-                                                            const uint32_t* __restrict__ vals,
-                                                            const double* __restrict__ y, int64_t total,
-                                                            float* __restrict__ lx, uint32_t* __restrict__ lr,
-                                                            double* __restrict__ ly, const Ctl* ctl, int64_t row0) {
-  const bool y32 = ctl->y32 != 0;
-  for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < total;
-       p += (int64_t)gridDim.x * blockDim.x) {
-    const uint32_t r = vals[p];
-    lx[p] = unflip_f32(keys[p]);
-    lr[p] = r;
-    const double v = __ldg(y + (r - row0));
-    if (y32) reinterpret_cast<int32_t*>(ly)[p] = (int32_t)v;
-    else ly[p] = v;
-  }
-}
-
 // Batched LSD radix sort of the d per-feature key lists (any n < 2^32): 4 passes
 // of 8-bit digits; per pass three launches, each over all d features (grid.y = feature):
 //   rs_count:   per-tile digit counts;
@@ -235,15 +209,34 @@ __global__ void __launch_bounds__(256) presort_build_kernel(const uint32_t* __re
 // Stable within a feature, so equal keys keep the row order: (x, row id) order (R6).
 constexpr int kTS = 256, kTI = 8, kTile = kTS * kTI;
 
-__global__ void __launch_bounds__(kTS) rs_count_kernel(const uint32_t* __restrict__ keys, int64_t n, int shift,
-                                                       int tiles, uint32_t* __restrict__ cnt) {
+// Source of a pass's keys: the key lists, or (first pass, kFromX) X itself: key =
+// flip(X[r][f]), value = row0 + r (the table's columns read in place; the d blocks of a
+// tile run side by side, so X's rows are read from L2 once per tile).
+template <bool kFromX>
+__device__ __forceinline__ uint32_t rs_key(const uint32_t* __restrict__ keys, const float* __restrict__ X, int64_t n,
+                                           int d, int f, int64_t i) {
+  if (kFromX) return flip_f32(__ldg(X + i * d + f));
+  return __ldg(keys + (int64_t)f * n + i);
+}
+
+// grid: d x tiles blocks, block b = (feature b % d, tile b / d)
+template <bool kFromX>
+__global__ void __launch_bounds__(kTS) rs_count_kernel(const uint32_t* __restrict__ keys, const float* __restrict__ X,
+                                                       int64_t n, int d, int shift, int tiles,
+                                                       uint32_t* __restrict__ cnt, Ctl* ctl) {
   __shared__ uint32_t h[256];
-  const int f = blockIdx.y, tile = blockIdx.x;
+  const int f = (int)(blockIdx.x % (unsigned)d), tile = (int)(blockIdx.x / (unsigned)d);
   h[threadIdx.x] = 0u;
   __syncthreads();
-  const int64_t base = (int64_t)f * n + (int64_t)tile * kTile;
-  const int m = (int)min((int64_t)kTile, n - (int64_t)tile * kTile);
-  for (int i = threadIdx.x; i < m; i += kTS) atomicAdd(&h[(__ldg(keys + base + i) >> shift) & 255u], 1u);
+  const int64_t base = (int64_t)tile * kTile;
+  const int m = (int)min((int64_t)kTile, n - base);
+  bool bad = false;
+  for (int i = threadIdx.x; i < m; i += kTS) {
+    const uint32_t key = rs_key<kFromX>(keys, X, n, d, f, base + i);
+    if (kFromX && !isfinite(unflip_f32(key))) bad = true;  // a6: non-finite X (flip keeps NaN / inf patterns)
+    atomicAdd(&h[(key >> shift) & 255u], 1u);
+  }
+  if (kFromX && __syncthreads_or(bad) && threadIdx.x == 0) ctl->nonfinite = 1;
   __syncthreads();
   cnt[((int64_t)f * 256 + threadIdx.x) * tiles + tile] = h[threadIdx.x];
 }
@@ -292,8 +285,21 @@ __global__ void __launch_bounds__(1024) rs_offset_kernel(const uint32_t* __restr
 #ifndef DT_RS_MINB
 #define DT_RS_MINB 4  // 4 CTAs/SM (64 registers): more tiles in flight (measured 4.04 -> 3.95 ms/step)
 #endif
+// kToLists (last pass): the sorted pairs go straight into the level-0 lists: x =
+// unflip(key), row = value, y = y[row - row0] (int32 when the fit stores y so, R24).
+struct RsOut {
+  uint32_t* kout;
+  uint32_t* vout;
+  float* lx;
+  uint32_t* lr;
+  double* ly;
+  const double* y;
+  int64_t row0;
+  const Ctl* ctl;
+};
+template <bool kFromX, bool kToLists>
 __global__ void __launch_bounds__(kTS, DT_RS_MINB) rs_scatter_kernel(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ vin,
-                                                         uint32_t* __restrict__ kout, uint32_t* __restrict__ vout,
+                                                         const float* __restrict__ X, int d, RsOut o,
                                                          int64_t n, int shift, int tiles, const uint32_t* __restrict__ off,
                                                          const uint32_t* __restrict__ tot) {
   __shared__ uint32_t wc[kTS / 32][256];  // per-warp digit counters -> per-warp prefixes
@@ -301,18 +307,18 @@ __global__ void __launch_bounds__(kTS, DT_RS_MINB) rs_scatter_kernel(const uint3
   __shared__ uint32_t s_start[256];       // digit starts inside the tile
   __shared__ uint32_t skey[kTile], sval[kTile];
   __shared__ uint32_t sw[kTS / 32], sw2[kTS / 32];
-  const int f = blockIdx.y, tile = blockIdx.x;
+  const int f = (int)(blockIdx.x % (unsigned)d), tile = (int)(blockIdx.x / (unsigned)d);
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int64_t base = (int64_t)f * n + (int64_t)tile * kTile;
-  const int m = (int)min((int64_t)kTile, n - (int64_t)tile * kTile);
+  const int64_t tbase = (int64_t)tile * kTile;
+  const int m = (int)min((int64_t)kTile, n - tbase);
   for (int q = lane; q < 256; q += 32) wc[w][q] = 0u;
   // keys of warp w: tile positions w * 256 + j * 32 + lane (coalesced, in tile order)
   uint32_t keys[kTI], vals[kTI], rk[kTI];
 #pragma unroll
   for (int j = 0; j < kTI; ++j) {
     const int i = w * 256 + j * 32 + lane;
-    keys[j] = (i < m) ? __ldg(kin + base + i) : 0u;
-    vals[j] = (i < m) ? __ldg(vin + base + i) : 0u;
+    keys[j] = (i < m) ? rs_key<kFromX>(kin, X, n, d, f, tbase + i) : 0u;
+    vals[j] = (i < m) ? (kFromX ? (uint32_t)(o.row0 + tbase + i) : __ldg(vin + (int64_t)f * n + tbase + i)) : 0u;
   }
   __syncwarp();
   const uint32_t lt = (1u << lane) - 1u;
@@ -375,12 +381,22 @@ __global__ void __launch_bounds__(kTS, DT_RS_MINB) rs_scatter_kernel(const uint3
     }
   }
   __syncthreads();
+  const bool y32 = kToLists && o.ctl->y32 != 0;
   for (int i = threadIdx.x; i < m; i += kTS) {
     const uint32_t key = skey[i];
     const uint32_t dg = (key >> shift) & 255u;
     const int64_t dst = (int64_t)f * n + s_base[dg] + ((uint32_t)i - s_start[dg]);
-    kout[dst] = key;
-    vout[dst] = sval[i];
+    if (kToLists) {
+      const uint32_t r = sval[i];
+      o.lx[dst] = unflip_f32(key);
+      o.lr[dst] = r;
+      const double v = __ldg(o.y + (r - o.row0));
+      if (y32) reinterpret_cast<int32_t*>(o.ly)[dst] = (int32_t)v;
+      else o.ly[dst] = v;
+    } else {
+      o.kout[dst] = key;
+      o.vout[dst] = sval[i];
+    }
   }
 }
 
@@ -397,25 +413,39 @@ struct Sent {  // one entry on the wire
   double y;
 };
 
-// One rank's partial of the root statistics (block parts folded in index order).
-__global__ void root_fold_kernel(const RootPart* parts, int nparts, RootPart* out) {
-  if (threadIdx.x != 0) return;
+// One rank's partial of the root statistics (block parts folded in index order; staged
+// in shared memory as in root_finalize_kernel).
+__global__ void __launch_bounds__(256) root_fold_kernel(const RootPart* parts, int nparts, RootPart* out) {
+  __shared__ RootPart sp[256];
   RootPart a{0, 0, INFINITY, -INFINITY, 1, 1};
-  for (int i = 0; i < nparts; ++i) {
-    neu_add(a.s, a.c, parts[i].s);
-    neu_add(a.s, a.c, parts[i].c);
-    a.mn = fmin(a.mn, parts[i].mn);
-    a.mx = fmax(a.mx, parts[i].mx);
-    a.integral &= parts[i].integral;
-    a.finite &= parts[i].finite;
+  for (int i0 = 0; i0 < nparts; i0 += 256) {
+    __syncthreads();
+    if (i0 + (int)threadIdx.x < nparts) sp[threadIdx.x] = parts[i0 + threadIdx.x];
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      for (int i = 0; i < min(256, nparts - i0); ++i) {
+        neu_add(a.s, a.c, sp[i].s);
+        neu_add(a.s, a.c, sp[i].c);
+        a.mn = fmin(a.mn, sp[i].mn);
+        a.mx = fmax(a.mx, sp[i].mx);
+        a.integral &= sp[i].integral;
+        a.finite &= sp[i].finite;
+      }
+    }
   }
-  *out = a;
+  if (threadIdx.x == 0) *out = a;
 }
-__global__ void center_fold_kernel(const double* parts, int nparts, double* out) {
-  if (threadIdx.x != 0) return;
+__global__ void __launch_bounds__(256) center_fold_kernel(const double* parts, int nparts, double* out) {
+  __shared__ double sp[256];
   double s = 0, cc = 0;
-  for (int i = 0; i < nparts; ++i) neu_add(s, cc, parts[i]);
-  *out = __dadd_rn(s, cc);
+  for (int i0 = 0; i0 < nparts; i0 += 256) {
+    __syncthreads();
+    if (i0 + (int)threadIdx.x < nparts) sp[threadIdx.x] = parts[i0 + threadIdx.x];
+    __syncthreads();
+    if (threadIdx.x == 0)
+      for (int i = 0; i < min(256, nparts - i0); ++i) neu_add(s, cc, sp[i]);
+  }
+  if (threadIdx.x == 0) *out = __dadd_rn(s, cc);
 }
 
 __device__ __forceinline__ unsigned long long ckey(const uint32_t* keys, const uint32_t* vals, int64_t i) {
@@ -609,18 +639,26 @@ __global__ void __launch_bounds__(256) root_tables_sharded_kernel(Ctl* ctl, cons
   (void)world;
 }
 
-// Batched tile radix sort of the d lists of n (key, value) pairs in b.k_in / b.v_in (4
-// passes x 3 launches, ping-pong through k_out / v_out, ends in k_in / v_in); stable.
-void radix_sort_lists(const FitBufs& b, int64_t n, int d, cudaStream_t s) {
+// Batched tile radix sort of the d lists of n (key, value) pairs (4 passes x 3 launches,
+// stable).  Keys from b.k_in / b.v_in, or with X from the table itself (first pass,
+// rows row0 + r).  Result in b.k_in / b.v_in, or with y straight in the level-0 lists
+// (last pass).
+void radix_sort_lists(const FitBufs& b, int64_t n, int d, cudaStream_t s, const float* X = nullptr,
+                      int64_t row0 = 0, const double* y = nullptr) {
   uint32_t *ki = b.k_in, *ko = b.k_out, *vi = b.v_in, *vo = b.v_out;
   const int tiles = (int)((n + kTile - 1) / kTile);
-  const dim3 g((unsigned)std::max(tiles, 1), (unsigned)d);
+  const unsigned g = (unsigned)(std::max(tiles, 1) * d);
   for (int pass = 0; pass < 4; ++pass) {
     const int shift = 8 * pass;
-    rs_count_kernel<<<g, kTS, 0, s>>>(ki, n, shift, tiles, b.rs_cnt);
+    const bool fx = X != nullptr && pass == 0, tl = y != nullptr && pass == 3;
+    if (fx) rs_count_kernel<true><<<g, kTS, 0, s>>>(ki, X, n, d, shift, tiles, b.rs_cnt, b.ctl);
+    else rs_count_kernel<false><<<g, kTS, 0, s>>>(ki, X, n, d, shift, tiles, b.rs_cnt, b.ctl);
     rs_offset_kernel<<<dim3(256, (unsigned)d), std::min(1024, (tiles + 31) / 32 * 32), 0, s>>>(b.rs_cnt, tiles,
                                                                                             b.rs_off, b.rs_tot);
-    rs_scatter_kernel<<<g, kTS, 0, s>>>(ki, vi, ko, vo, n, shift, tiles, b.rs_off, b.rs_tot);
+    RsOut o{ko, vo, b.lx[0], b.lr[0], b.ly[0], y, row0, b.ctl};
+    if (fx) rs_scatter_kernel<true, false><<<g, kTS, 0, s>>>(ki, vi, X, d, o, n, shift, tiles, b.rs_off, b.rs_tot);
+    else if (tl) rs_scatter_kernel<false, true><<<g, kTS, 0, s>>>(ki, vi, X, d, o, n, shift, tiles, b.rs_off, b.rs_tot);
+    else rs_scatter_kernel<false, false><<<g, kTS, 0, s>>>(ki, vi, X, d, o, n, shift, tiles, b.rs_off, b.rs_tot);
     std::swap(ki, ko);
     std::swap(vi, vo);
   }
@@ -639,33 +677,23 @@ dt_status presort_enqueue(const FitBufs& b, const float* X, const double* y, int
   {
     const int pr = prof_begin(PK_ROOT, s, 4);
     root_reduce_kernel<<<(unsigned)b.root_np, 256, 0, s>>>(y, n, b.root_chunk, reinterpret_cast<RootPart*>(b.parts));
-    root_finalize_kernel<<<1, 32, 0, s>>>(reinterpret_cast<RootPart*>(b.parts), (int)b.root_np, n, ctl);
+    root_finalize_kernel<<<1, 256, 0, s>>>(reinterpret_cast<RootPart*>(b.parts), (int)b.root_np, n, ctl);
     root_center_kernel<<<(unsigned)b.root_np, 256, 0, s>>>(y, n, n, b.root_chunk, ctl, b.cparts);
-    root_init_kernel<<<1, 32, 0, s>>>(b.cparts, (int)b.root_np, n, d, max_depth, min_leaf, ctl, b.nodes[0],
+    root_init_kernel<<<1, 256, 0, s>>>(b.cparts, (int)b.root_np, n, d, max_depth, min_leaf, ctl, b.nodes[0],
                                       b.dec_root);
     prof_end(pr, s, 16.0 * (double)n);  // y read twice
     DT_CK(cudaGetLastError());
   }
   {
-    const int rb = d <= 48 ? 256 : (d <= 96 ? 128 : 64);  // rows per block (smem)
-    const int64_t nb = (n + rb - 1) / rb;
-    const size_t smem = sizeof(float) * rb * (size_t)d;
-    if (smem > 48 * 1024)
-      DT_CK(cudaFuncSetAttribute(presort_keys_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    int pr = prof_begin(PK_PRESORT_KEYS, s, 1);
-    presort_keys_kernel<<<(unsigned)nb, 256, smem, s>>>(X, n, d, b.k_in, b.v_in, ctl, row0, rb);
-    prof_end(pr, s, 16.0 * (double)total0);  // X read + (key, val) written
-    DT_CK(cudaGetLastError());
-    pr = prof_begin(PK_PRESORT_SORT, s, 12);
-    uint32_t *ki = b.k_in, *vi = b.v_in;
-    radix_sort_lists(b, n, d, s);  // ends in k_in / v_in
+    // the sort reads X in its first pass (keys, non-finite check) and writes the level-0
+    // lists (x, row, y gathered) in its last
+    int pr = prof_begin(PK_PRESORT_SORT, s, 12);
+    radix_sort_lists(b, n, d, s, X, row0, y);
     prof_end(pr, s, 4.0 * 24.0 * (double)total0);  // per pass: keys read twice, pairs read + written
     DT_CK(cudaGetLastError());
-    const int gb = std::max(1, std::min<int>((int)((total0 + 255) / 256), num_sms() * 8));
-    pr = prof_begin(PK_PRESORT_BUILD, s, 2);
-    presort_build_kernel<<<gb, 256, 0, s>>>(ki, vi, y, total0, b.lx[0], b.lr[0], b.ly[0], ctl, row0);
+    pr = prof_begin(PK_PRESORT_BUILD, s, 1);
     root_tables_kernel<<<num_sms(), 256, 0, s>>>(ctl, b.nodes[0], n, d, b.segs[0], b.pseg, b.desc[0]);
-    prof_end(pr, s, 36.0 * (double)total0);  // (key, val) read, y gathered, 16 B written
+    prof_end(pr, s, 0.0);
     DT_CK(cudaGetLastError());
   }
   return DT_OK;
@@ -709,28 +737,23 @@ dt_status presort_sharded_enqueue(const FitBufs& b, dt_comm* comm, const float* 
   const int npl = n_local > 0 ? (int)b.root_np : 0;
   int pr = prof_begin(PK_ROOT, s, 6);
   if (npl) root_reduce_kernel<<<npl, 256, 0, s>>>(y, n_local, b.root_chunk, reinterpret_cast<RootPart*>(b.parts));
-  root_fold_kernel<<<1, 32, 0, s>>>(reinterpret_cast<RootPart*>(b.parts), npl, mine);
+  root_fold_kernel<<<1, 256, 0, s>>>(reinterpret_cast<RootPart*>(b.parts), npl, mine);
   DT_CK(cudaGetLastError());
   dt_status st = comm_allgather(comm, mine, allp, sizeof(RootPart), s);
   if (st != DT_OK) return st;
-  root_finalize_kernel<<<1, 32, 0, s>>>(allp, P, n_global, ctl);
+  root_finalize_kernel<<<1, 256, 0, s>>>(allp, P, n_global, ctl);
   if (npl) root_center_kernel<<<npl, 256, 0, s>>>(y, n_local, n_global, b.root_chunk, ctl, b.cparts);
-  center_fold_kernel<<<1, 32, 0, s>>>(b.cparts, npl, cmine);
+  center_fold_kernel<<<1, 256, 0, s>>>(b.cparts, npl, cmine);
   DT_CK(cudaGetLastError());
   st = comm_allgather(comm, cmine, call, sizeof(double), s);
   if (st != DT_OK) return st;
-  root_init_kernel<<<1, 32, 0, s>>>(call, P, n_global, d, max_depth, min_leaf, ctl, b.nodes[0], b.dec_root);
+  root_init_kernel<<<1, 256, 0, s>>>(call, P, n_global, d, max_depth, min_leaf, ctl, b.nodes[0], b.dec_root);
   prof_end(pr, s, 16.0 * (double)n_local);
   DT_CK(cudaGetLastError());
   // ---- local keys, local sort
   pr = prof_begin(PK_PRESORT_SORT, s, 14);
   if (n_local > 0) {
-    const int rb = d <= 48 ? 256 : (d <= 96 ? 128 : 64);
-    const size_t smem = sizeof(float) * rb * (size_t)d;
-    if (smem > 48 * 1024)
-      DT_CK(cudaFuncSetAttribute(presort_keys_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    presort_keys_kernel<<<(unsigned)((n_local + rb - 1) / rb), 256, smem, s>>>(X, n_local, d, b.k_in, b.v_in, ctl, row0, rb);
-    radix_sort_lists(b, n_local, d, s);
+    radix_sort_lists(b, n_local, d, s, X, row0);
     DT_CK(cudaGetLastError());
   }
   // ---- exact splitters: 64 bisection rounds on the composite key, counts summed over ranks
@@ -981,9 +1004,9 @@ dt_status forest_tree_enqueue(const FitBufs& b, const float* sx, const uint32_t*
   DT_CK(cudaGetLastError());
   pr = prof_begin(PK_ROOT, s, 6);
   root_reduce_kernel<<<(unsigned)b.root_np, 256, 0, s>>>(ys, n, b.root_chunk, reinterpret_cast<RootPart*>(b.parts));
-  root_finalize_kernel<<<1, 32, 0, s>>>(reinterpret_cast<RootPart*>(b.parts), (int)b.root_np, n, b.ctl);
+  root_finalize_kernel<<<1, 256, 0, s>>>(reinterpret_cast<RootPart*>(b.parts), (int)b.root_np, n, b.ctl);
   root_center_kernel<<<(unsigned)b.root_np, 256, 0, s>>>(ys, n, n, b.root_chunk, b.ctl, b.cparts);
-  root_init_kernel<<<1, 32, 0, s>>>(b.cparts, (int)b.root_np, n, d, max_depth, min_leaf, b.ctl, b.nodes[0], b.dec_root);
+  root_init_kernel<<<1, 256, 0, s>>>(b.cparts, (int)b.root_np, n, d, max_depth, min_leaf, b.ctl, b.nodes[0], b.dec_root);
   set_storage_kernel<<<1, 1, 0, s>>>(b.ctl, y32);  // the lists keep the table's y storage
   root_tables_kernel<<<num_sms(), 256, 0, s>>>(b.ctl, b.nodes[0], n, d, b.segs[0], b.pseg, b.desc[0]);
   prof_end(pr, s, 16.0 * (double)n);

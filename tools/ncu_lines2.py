@@ -1,9 +1,10 @@
 """Per-CUDA-source-line instruction counts and stall samples from an ncu report
-(`ncu -i rep --page source --csv --print-source cuda,sass`).  Usage: ncu_lines2.py rep [top]"""
+(`ncu -i rep --page source --csv --print-source cuda,sass`).  Usage: ncu_lines2.py rep [top] [kernel-regex]"""
 import csv, subprocess, sys, collections
 rep = sys.argv[1]
 top = int(sys.argv[2]) if len(sys.argv) > 2 else 40
-out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
+kf = ["-k", "regex:" + sys.argv[3]] if len(sys.argv) > 3 else []  # optional kernel-name filter
+out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"] + kf,
                      capture_output=True, text=True).stdout.splitlines()
 rows = list(csv.reader(out))
 agg = collections.defaultdict(lambda: [0.0, 0.0, ""])
