@@ -1508,10 +1508,12 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
   {  // the virtual-root pass (the root's rank carries come from the presort)
     LevelArgs la{-1, 0, 0, d, min_leaf, false};
     int pr = prof_begin(PK_SCAN, s, 2);
+    pending.push_back({pr, -1, PK_SCAN});
     st = level_agg_enqueue(b, la, s);
     if (st != DT_OK) return st;
     prof_end(pr, s, 0.0);
     pr = prof_begin(PK_PARTITION, s, 1);
+    pending.push_back({pr, -1, PK_PARTITION});
     st = level_fused_enqueue(b, la, s);
     if (st != DT_OK) return st;
     prof_end(pr, s, 0.0);
@@ -1587,6 +1589,7 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
     DT_CK(cudaGetLastError());
     // go-left bitmap: each rank sets the bits of its own split-feature entries; OR over ranks
     pr = prof_begin(PK_GOLEFT, s, 1);
+    pending.push_back({pr, level, PK_GOLEFT});
     goleft_kernel<<<g_gl, 256, 0, s>>>(ctl, par, b.desc[par], b.pseg, b.lr[cur], b.gbits, d);
     DT_CK(cudaGetLastError());
     st = comm_allreduce_or_u32(comm, b.gbits, b.nwords4, s);
@@ -1594,6 +1597,7 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
     prof_end(pr, s, 0.0);
     LevelArgs la{level, cur, par, d, min_leaf, true};
     pr = prof_begin(PK_SCAN, s, 3);
+    pending.push_back({pr, level, PK_SCAN});
     st = level_agg_enqueue(b, la, s);
     if (st != DT_OK) return st;
     prof_end(pr, s, 0.0);
@@ -1619,12 +1623,13 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
       DT_CK(cudaMemsetAsync(&ctl->T0[par ^ 1], 0, sizeof(unsigned long long), s));
     }
     pr = prof_begin(PK_PARTITION, s, 1);
+    pending.push_back({pr, level, PK_PARTITION});
     st = level_fused_enqueue(b, la, s);
     if (st != DT_OK) return st;
     prof_end(pr, s, 0.0);
     K = K2;
   }
-  return fit_finish(b, d, s, nullptr, out);
+  return fit_finish(b, d, s, &pending, out);
 }
 
 }  // namespace dtl

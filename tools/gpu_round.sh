@@ -3,7 +3,7 @@
 #   GPU tests, smoke, the default bench line, an ncu launch list of one bench step and an
 #   ncu --set full capture of the fit's streaming kernels + predict.  Outputs in gpurun_out/.
 # usage: gpurun --timeout 2400 -- 'bash tools/gpu_round.sh [tag] [tests=1]'
-TAG=${1:-r01}
+TAG=${1:-r02}
 TESTS=${2:-1}
 mkdir -p gpurun_out
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,memory.total --format=csv > gpurun_out/${TAG}_smi.txt 2>&1
@@ -20,8 +20,8 @@ timeout 600 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__byte
   python bench.py --steps 1 --warmup 0 --no-cpu --no-extra --e2e-steps 0 --no-dse --c3-rows 0 > gpurun_out/${TAG}_ncu_launch.log 2>&1
 echo "ncu launch exit $?" >> gpurun_out/${TAG}_ncu_launch.log
 timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base function \
-  -k regex:'^(scan_kernel|scan_single_kernel|partition_kernel|part_agg_kernel|scan_agg_kernel|rs_scatter_kernel|select_kernel|prep_kernel)$' \
-  --launch-count 12 -o /tmp/${TAG}_full -f \
+  -k regex:'fused_kernel|level_agg_kernel|rs_scatter_kernel|goleft_kernel|select_kernel' \
+  --launch-count 14 -o /tmp/${TAG}_full -f \
   python bench.py --steps 1 --warmup 0 --no-cpu --no-extra --e2e-steps 0 --no-dse --c3-rows 0 > gpurun_out/${TAG}_ncu_full.log 2>&1
 echo "ncu full exit $?" >> gpurun_out/${TAG}_ncu_full.log
 ncu -i /tmp/${TAG}_full.ncu-rep --page raw --csv > gpurun_out/${TAG}_full_raw.csv 2>/dev/null

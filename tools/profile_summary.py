@@ -17,17 +17,15 @@ import sys
 
 # kernel name -> library profiling kind (dt_profile_* kinds, csrc/prof.cu)
 KIND = {
-    "scan_desc_kernel": "scan", "scan_agg_kernel": "scan", "scan_kernel": "scan",
-    "part_desc_kernel": "partition", "decide_kernel": "select",
-    "chunk_scan_kernel<SumP>": "scan", "block_carry_kernel<SumP>": "scan",
-    "part_agg_kernel": "partition", "partition_kernel": "partition",
-    "chunk_scan_kernel<CntP>": "partition", "block_carry_kernel<CntP>": "partition",
-    "piece_pos_kernel": "select", "select_kernel": "select", "number_kernel": "number",
-    "goleft_kernel": "goleft", "presort_keys_kernel": "presort_keys",
-    "presort_build_kernel": "presort_build", "predict_kernel<true>": "predict",
-    "predict_kernel<false>": "predict", "scan_single_kernel": "scan", "prep_kernel": "goleft",
-    "rs_count_kernel": "presort_sort", "rs_offset_kernel": "presort_sort",
-    "rs_scatter_kernel": "presort_sort", "predict_col_kernel": "predict",
+    "fused_kernel": "fused", "fused_small_kernel": "fused",
+    "level_agg_kernel": "agg", "chunk_plan_kernel": "agg", "agg_scan_kernel": "agg",
+    "piece_pos_kernel": "select", "select_kernel": "select",
+    "number_kernel": "number", "children_kernel": "number", "tables_kernel": "number",
+    "goleft_kernel": "goleft",
+    "rs_count_kernel": "presort_sort", "rs_offset_kernel": "presort_sort", "rs_scatter_kernel": "presort_sort",
+    "root_reduce_kernel": "root_stats", "root_finalize_kernel": "root_stats", "root_center_kernel": "root_stats",
+    "root_init_kernel": "root_stats", "root_tables_kernel": "presort_build",
+    "predict_col_kernel": "predict", "eval_partial_kernel": "eval", "eval_final_kernel": "eval",
 }
 
 
@@ -38,10 +36,7 @@ def short(name):
         return "cub_radix_sort"
     if base.startswith("void "):
         base = base[5:]
-    for key in ("chunk_scan_kernel", "block_carry_kernel"):
-        if base.startswith(key):
-            return key + ("<SumP>" if "SumP" in name else "<CntP>")
-    return base
+    return base.split("<")[0]  # template arguments folded
 
 
 def main():
@@ -84,13 +79,14 @@ def main():
         k = KIND.get(n)
         if k:
             per_kind[k][0] += b
-    region_launches = {"scan": agg.get("scan_kernel", [1])[0],
-                       "partition": agg.get("partition_kernel", [1])[0],
+    region_launches = {"fused": agg.get("fused_kernel", [1])[0],
+                       "agg": agg.get("level_agg_kernel", [1])[0],
                        "select": agg.get("select_kernel", [1])[0],
-                       "goleft": agg.get("prep_kernel", [1])[0],
+                       "number": agg.get("number_kernel", [1])[0],
+                       "goleft": agg.get("goleft_kernel", [1])[0],
                        "presort_sort": 1}
     tpath = os.path.join(os.path.dirname(os.path.abspath(__file__)), "..", "profiles", "traffic.json")
-    traffic = json.load(open(tpath)) if os.path.exists(tpath) else {}
+    traffic = {}  # this capture's kinds only
     for k, (b, _) in per_kind.items():
         launches = region_launches.get(k) or sum(c for n, (c, t, bb) in agg.items() if KIND.get(n) == k)
         traffic[k] = b / max(1, launches)
