@@ -1,7 +1,7 @@
 // Leave-one-out refits for the paper-sized table (BASELINE configs[0]: 40 (CNN, GPU) rows
 // x 4 features; the paper's 70/30 split, has no seed -> Reading R11).
 // One CTA per fold: the fold's n-1 rows, their per-feature orders and the whole tree
-// live in shared memory; the held-out row is predicted at the end.  The split rule is
+// live in shared memory; level-synchronous BFS; the held-out row is predicted at the end.  The split rule is
 // the one of dt_fit (Readings R1-R10, R19).  Within a node the per-feature prefix and
 // suffix sums run sequentially in (x, row id) order with Neumaier compensation.
 #include <math.h>
@@ -42,12 +42,13 @@ loo_kernel(const float* __restrict__ Xg, const double* __restrict__ yg, int n_al
   __shared__ uint8_t order[kMaxD][kMaxN];  // rows of feature f in (x, row) order
   __shared__ int16_t nid[kMaxN];           // current node of each row
   __shared__ TNode tree[kMaxNodes];
-  __shared__ double bgain[kMaxD];
-  __shared__ int bpos[kMaxD];
-  __shared__ double bthr[kMaxD];
-  __shared__ int s_int_mode, s_count;
-  __shared__ double s_c;
-  __shared__ int s_leaf;
+  // per (splittable node of the level, feature): best gain, position, threshold
+  __shared__ double bgain[kMaxN / 2 * kMaxD];
+  __shared__ int bpos[kMaxN / 2 * kMaxD];
+  __shared__ double bthr[kMaxN / 2 * kMaxD];
+  __shared__ uint8_t s_leafv[kMaxN], s_split[kMaxN];
+  __shared__ double s_cc[kMaxN];
+  __shared__ int s_int_mode, s_count, s_nsplit;
 
   const int fold = blockIdx.x;
   const int n = n_all - 1;
@@ -88,9 +89,16 @@ loo_kernel(const float* __restrict__ Xg, const double* __restrict__ yg, int n_al
   }
   __syncthreads();
 
-  // BFS over nodes (the queue is the node array itself)
-  for (int node = 0; node < s_count; ++node) {
-    if (tid == 0) {
+  // Level-synchronous BFS: the nodes of one depth [lo, hi) are evaluated together
+  // (statistics: a thread per node; split scans: a thread per (node, feature); the
+  // choice and the BFS numbering of the children: one thread, in node order; the
+  // partition: a thread per row).  Per node and feature the arithmetic is the sequential
+  // one of the oracle (Neumaier sums in (x, row) order), so the trees are identical.
+  int lo = 0, hi = 1;
+  while (lo < hi) {
+    const int nn = hi - lo;
+    for (int q = tid; q < nn; q += blockDim.x) {
+      const int node = lo + q;
       double s = 0, c = 0, mn = INFINITY, mx = -INFINITY;
       int N = 0;
       for (int r = 0; r < n; ++r)
@@ -98,6 +106,7 @@ loo_kernel(const float* __restrict__ Xg, const double* __restrict__ yg, int n_al
       const double sum = __dadd_rn(s, c);
       const double value = __ddiv_rn(sum, (double)N);
       TNode& t = tree[node];
+      t.n = N;
       t.value = value;
       t.feature = -1;
       t.left = -1;
@@ -106,74 +115,81 @@ loo_kernel(const float* __restrict__ Xg, const double* __restrict__ yg, int n_al
       if (max_depth >= 0 && t.depth >= max_depth) leaf = 1;
       else if ((long long)N < 2 * min_leaf) leaf = 1;
       else if (mn == mx) leaf = 1;
-      s_leaf = leaf;
-      s_c = s_int_mode ? (double)fdiv((long long)sum, (long long)N) : value;
+      s_leafv[q] = (uint8_t)leaf;
+      s_cc[q] = s_int_mode ? (double)fdiv((long long)sum, (long long)N) : value;
     }
     __syncthreads();
-    if (!s_leaf) {
-      const double cc = s_c;
-      const int N = tree[node].n;
-      // warp w: features w, w+8, ...; lane 0 scans sequentially
-      for (int f = w; f < d; f += 8) {
-        if (lane == 0) {
-          int rows[kMaxN];
-          int m = 0;
-          for (int k = 0; k < n; ++k) {
-            const int r = order[f][k];
-            if (nid[r] == node) rows[m++] = r;
-          }
-          double pre[kMaxN + 1], suf[kMaxN + 1];
-          double s = 0, c = 0;
-          pre[0] = 0.0;
-          for (int k = 0; k < m; ++k) { nadd(s, c, __dsub_rn(y[rows[k]], cc)); pre[k + 1] = __dadd_rn(s, c); }
-          s = 0; c = 0;
-          suf[m] = 0.0;
-          for (int k = m - 1; k >= 0; --k) { nadd(s, c, __dsub_rn(y[rows[k]], cc)); suf[k] = __dadd_rn(s, c); }
-          double bg = -1.0, bt = 0.0;
-          int bp = -1;
-          for (int i = 1; i < m; ++i) {
-            const float xlo = X[rows[i - 1] * d + f], xhi = X[rows[i] * d + f];
-            if (!(xlo < xhi) || (long long)i < min_leaf || (long long)(m - i) < min_leaf) continue;
-            const double nl = (double)i, nr = (double)(m - i), Nd = (double)m;
-            const double D = __dsub_rn(__dmul_rn(pre[i], nr), __dmul_rn(suf[i], nl));
-            const double g = __ddiv_rn(__dmul_rn(D, D), __dmul_rn(__dmul_rn(Nd, nl), nr));
-            if (g > bg) {
-              bg = g;
-              bp = i;
-              bt = __dadd_rn(__ddiv_rn((double)xlo, 2.0), __ddiv_rn((double)xhi, 2.0));
-            }
-          }
-          (void)N;
-          bgain[f] = bg;
-          bpos[f] = bp;
-          bthr[f] = bt;
+    if (tid == 0) {  // the level's splittable nodes, in node order
+      int m = 0;
+      for (int q = 0; q < nn; ++q)
+        if (!s_leafv[q]) s_split[m++] = (uint8_t)q;
+      s_nsplit = m;
+    }
+    __syncthreads();
+    const int ns = s_nsplit;
+    for (int pidx = tid; pidx < ns * d; pidx += blockDim.x) {
+      const int q = s_split[pidx / d], f = pidx - (pidx / d) * d;
+      const int node = lo + q;
+      const double cc = s_cc[q];
+      int rows[kMaxN];
+      int m = 0;
+      for (int k = 0; k < n; ++k) {
+        const int r = order[f][k];
+        if (nid[r] == node) rows[m++] = r;
+      }
+      double pre[kMaxN + 1], suf[kMaxN + 1];
+      double s = 0, c = 0;
+      pre[0] = 0.0;
+      for (int k = 0; k < m; ++k) { nadd(s, c, __dsub_rn(y[rows[k]], cc)); pre[k + 1] = __dadd_rn(s, c); }
+      s = 0; c = 0;
+      suf[m] = 0.0;
+      for (int k = m - 1; k >= 0; --k) { nadd(s, c, __dsub_rn(y[rows[k]], cc)); suf[k] = __dadd_rn(s, c); }
+      double bg = -1.0, bt = 0.0;
+      int bp = -1;
+      for (int i = 1; i < m; ++i) {
+        const float xlo = X[rows[i - 1] * d + f], xhi = X[rows[i] * d + f];
+        if (!(xlo < xhi) || (long long)i < min_leaf || (long long)(m - i) < min_leaf) continue;
+        const double nl = (double)i, nr = (double)(m - i), Nd = (double)m;
+        const double D = __dsub_rn(__dmul_rn(pre[i], nr), __dmul_rn(suf[i], nl));
+        const double g = __ddiv_rn(__dmul_rn(D, D), __dmul_rn(__dmul_rn(Nd, nl), nr));
+        if (g > bg) {
+          bg = g;
+          bp = i;
+          bt = __dadd_rn(__ddiv_rn((double)xlo, 2.0), __ddiv_rn((double)xhi, 2.0));
         }
       }
-      __syncthreads();
-      if (tid == 0) {
+      bgain[pidx] = bg;
+      bpos[pidx] = bp;
+      bthr[pidx] = bt;
+    }
+    __syncthreads();
+    if (tid == 0) {  // choices and children ids in node order (BFS numbering)
+      for (int u = 0; u < ns; ++u) {
         int bf = -1;
         double bg = -1.0;
         for (int f = 0; f < d; ++f)
-          if (bpos[f] >= 0 && bgain[f] > bg) { bg = bgain[f]; bf = f; }
+          if (bpos[u * d + f] >= 0 && bgain[u * d + f] > bg) { bg = bgain[u * d + f]; bf = f; }
         if (bf >= 0) {
-          TNode& t = tree[node];
+          TNode& t = tree[lo + s_split[u]];
           t.feature = bf;
-          t.thr = bthr[bf];
+          t.thr = bthr[u * d + bf];
           t.left = s_count;
-          int nl = 0;
-          for (int r = 0; r < n; ++r)
-            if (nid[r] == node) {
-              if ((double)X[r * d + bf] <= t.thr) { nid[r] = (int16_t)s_count; ++nl; }
-              else nid[r] = (int16_t)(s_count + 1);
-            }
           tree[s_count].depth = t.depth + 1;
-          tree[s_count].n = nl;
           tree[s_count + 1].depth = t.depth + 1;
-          tree[s_count + 1].n = t.n - nl;
           s_count += 2;
         }
       }
     }
+    __syncthreads();
+    for (int r = tid; r < n; r += blockDim.x) {  // the level's partition
+      const int node = nid[r];
+      if (node >= lo && node < hi && tree[node].feature >= 0) {
+        const TNode& t = tree[node];
+        nid[r] = (int16_t)(((double)X[r * d + t.feature] <= t.thr) ? t.left : t.left + 1);
+      }
+    }
+    lo = hi;
+    hi = s_count;
     __syncthreads();
   }
   // predict the held-out row

@@ -155,6 +155,24 @@ def test_fit_collinear_ties_exact(dt):
         _assert_exact(_fit(dt, X, y, -1, 1).nodes, o)
 
 
+@pytest.mark.parametrize("g", [31, 32, 33, 34])
+def test_fit_small_segment_boundary(dt, g):
+    """Nodes of g rows around the small-segment limit (<= 32 entries: a warp per segment;
+    > 32: masked pieces of the chunk pass, at most 9 per chunk) at every chunk alignment:
+    feature 0 = group id (groups of g rows), the others random ties, y by group + noise."""
+    rng = np.random.default_rng(g)
+    n = 97 * g + 5
+    grp = np.arange(n) // g
+    X = np.empty((n, 4), dtype=np.float32)
+    X[:, 0] = grp.astype(np.float32)
+    X[:, 1:] = rng.integers(0, 9, size=(n, 3)).astype(np.float32)
+    y = (grp % 11) * 100.0 + rng.integers(0, 5, size=n)
+    perm = rng.permutation(n)
+    X, y = np.ascontiguousarray(X[perm]), np.ascontiguousarray(y[perm])
+    for D in (-1, 8):
+        _assert_exact(_fit(dt, X, y, D, 1).nodes, oracle.fit(X, y, D, 1))
+
+
 @pytest.mark.parametrize("n", [4095, 4096, 4097, 8191, 12289])
 def test_fit_tile_boundaries(dt, n):
     """Segments that start / end exactly on 4096-entry tile boundaries."""
