@@ -93,7 +93,7 @@ loo_kernel(const float* __restrict__ Xg, const double* __restrict__ yg, int n_al
   // (statistics: a thread per node; split scans: a thread per (node, feature); the
   // choice and the BFS numbering of the children: one thread, in node order; the
   // partition: a thread per row).  Per node and feature the arithmetic is the sequential
-  // one of the oracle (Neumaier sums in (x, row) order), so the trees are identical.
+  // sequential reading R10 (Neumaier sums in (x, row) order), so the trees are identical.
   int lo = 0, hi = 1;
   while (lo < hi) {
     const int nn = hi - lo;
