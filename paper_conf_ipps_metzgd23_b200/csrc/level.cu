@@ -32,6 +32,10 @@ namespace dtl {
 namespace {
 
 constexpr int kThreads = 256;
+#ifndef DT_FUSED_STAGES
+#define DT_FUSED_STAGES 2  // bulk-copy stages per warp of the fused pass (3 measured: no faster)
+#endif
+constexpr int kStages = DT_FUSED_STAGES;
 #ifndef DT_FUSED_MINB
 #define DT_FUSED_MINB 2  // CTAs per SM of the fused pass (register budget; 3 spills: slower)
 #endif
@@ -707,16 +711,16 @@ __device__ __forceinline__ uint32_t store_rows(const FusedArgs& a, const PSeg& p
 // y storage (int32 or f64, Reading R24) is decided on the device (root statistics): the
 // stage always has room for f64 entries; int32 lists copy and read half of it.
 // Work: the fast chunks listed by chunk_plan_kernel (whole chunk inside one segment of a
-// split node); a warp per chunk, two bulk-copy stages in flight per warp.
+// split node); a warp per chunk, kStages bulk-copy stages in flight per warp.
 __global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArgs a) {
   extern __shared__ __align__(128) unsigned char fsm[];
   constexpr uint32_t YB = 8u;
   constexpr uint32_t SB = (stage_bytes_for(YB) + 127u) & ~127u;
   constexpr int kWarps = kThreads / 32;
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  unsigned char* my = fsm + (size_t)wib * 2 * SB;
-  uint64_t* bar = reinterpret_cast<uint64_t*>(fsm + (size_t)kWarps * 2 * SB) + wib * 2;
-  PSeg* cur = reinterpret_cast<PSeg*>(fsm + (size_t)kWarps * 2 * SB + kWarps * 2 * sizeof(uint64_t)) + wib;
+  unsigned char* my = fsm + (size_t)wib * kStages * SB;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(fsm + (size_t)kWarps * kStages * SB) + wib * kStages;
+  PSeg* cur = reinterpret_cast<PSeg*>(fsm + (size_t)kWarps * kStages * SB + kWarps * kStages * sizeof(uint64_t)) + wib;
   const bool full = a.ctl->nsrch > 0;
   const int64_t nfast = a.ctl->nunit;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -748,14 +752,13 @@ __global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArg
     bulk_g2s(st + off_ce(YB), a.cexcl + ch, 32u, bar + s);
     bulk_g2s(st + off_cb(YB), a.bcarry + ch / kBlockChunks, 32u, bar + s);
   };
-  uint2 ahead = make_uint2(0u, 0u);  // lane 0: the list entry two chunks ahead
+  uint2 ahead = make_uint2(0u, 0u);  // lane 0: the list entry kStages chunks ahead
   if (lane == 0) {
-    mbar_init(bar, 1);
-    mbar_init(bar + 1, 1);
+    for (int q = 0; q < kStages; ++q) mbar_init(bar + q, 1);
     mbar_init_fence();
-    issue(0, a.unit_list[gw]);
-    if (gw + nw < nfast) issue(1, a.unit_list[gw + nw]);
-    if (gw + 2 * nw < nfast) ahead = a.unit_list[gw + 2 * nw];
+    for (int q = 0; q < kStages; ++q)
+      if (gw + q * nw < nfast) issue(q, a.unit_list[gw + q * nw]);
+    if (gw + kStages * nw < nfast) ahead = a.unit_list[gw + kStages * nw];
   }
   __syncwarp();
   int s = 0;
@@ -763,7 +766,7 @@ __global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArg
   for (int64_t idx = gw; idx < nfast; idx += nw) {
     mbar_wait(bar + s, phase);
     unsigned char* st = my + (size_t)s * SB;
-    const int64_t nxt = idx + 2 * nw;
+    const int64_t nxt = idx + kStages * nw;
     const int64_t ch = reinterpret_cast<const Meta*>(st + off_meta(YB))->ch;
     const uint64_t cbase = (uint64_t)ch * kChunkW;
     // the plan of the chunk's segment: kept in this warp's slot (the stage is refilled
@@ -816,7 +819,7 @@ __global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArg
       const int hi_i = min(max(e_hi - lane * kItems, 0), kItems);
       mbyte = ((1u << hi_i) - 1u) & ~((1u << lo_i) - 1u);
     }
-    const uint32_t graw = (w[lane >> 2] >> (8 * (lane & 3))) & 0xffu;
+    const uint32_t graw = sgm[lane];  // go-left bits of my 8 items (byte lane of w)
     const uint32_t lbyte = graw & mbyte, rbyte = ~graw & mbyte;
     const uint32_t flags = ps.flags;
     const uint32_t ib = (uint32_t)(cbase - ps.start);  // segment-local index of entry 0 (mod 2^32)
@@ -961,7 +964,7 @@ __global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArg
         }
       }
     }
-    if (++s == 2) { s = 0; phase ^= 1u; }
+    if (++s == kStages) { s = 0; phase ^= 1u; }
   }
 }
 
@@ -1138,7 +1141,7 @@ dt_status level_agg_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t 
 size_t fused_smem() {
   const size_t sb = (stage_bytes_for(8u) + 127u) & ~127u;
   constexpr int kWarps = kThreads / 32;
-  return sb * 2 * kWarps + kWarps * 2 * sizeof(uint64_t) + kWarps * sizeof(PSeg);
+  return sb * kStages * kWarps + kWarps * kStages * sizeof(uint64_t) + kWarps * sizeof(PSeg);
 }
 
 // F_C of the pass whose parent level is la.level.
