@@ -421,114 +421,174 @@ __global__ void __launch_bounds__(256) importances_kernel(const dt_node* __restr
 
 // The paper's design-space exploration estimates one CNN on n GPU configurations
 // (T_est = t_dca + n * t_pm): candidate (i, j) = CNN row i composed with
-// GPU row j, never materialised.  A CTA keeps the tree (features re-encoded: 0x80 | g =
-// GPU column g, c = CNN column c), the transposed GPU table (thread j reads column
-// entries j: conflict-free) and kR CNN rows in shared memory; thread j walks kR
-// candidates (i0 + r, j) at once (independent chains) and writes yhat[(i0 + r) * n_gpu + j]
-// (coalesced).  Output-write bound: 8 B per prediction (the inputs are O(n_cnn + n_gpu)).
+// GPU row j, never materialised.  Tree features are re-encoded (0x80 | g = GPU column g,
+// c = CNN column c).  Output-write bound at best: 8 B per prediction (the inputs are
+// O(n_cnn + n_gpu)).
 struct DseMap {
   uint8_t code[256];  // tree feature f -> 0x80 | GPU column, or CNN column
 };
 
-template <bool kSmemTree, bool kSorted, int kR>
+// GPU-specialised trees (the per-candidate cost of the factored DSE): for GPU row j the
+// GPU-side decisions are fixed, so tree T_j = the tree with every GPU-feature node
+// replaced by the child row j takes.  T_j keeps only CNN-feature nodes and leaves (C2
+// tree, depth 20: ~220 of 11487 nodes, depth <= 13), and candidate (i, j) is a walk of
+// T_j on CNN row i -- the same comparisons x > RD32(t) as the full walk, in the same
+// order, so the reached leaf (hence yhat) is identical.  The 32 trees of a group of 32
+// consecutive GPU rows are stored interleaved (node k of lane j at word k * 32 + j), so a
+// warp's node reads are conflict-free whatever nodes its lanes sit on.  T_j node: {f32
+// threshold bits, CNN column << 24 | local left child (right = left + 1)}; T_j leaves
+// self-loop with threshold NaN (x > NaN is false) whose payload is the leaf's id in the
+// full tree (value index).
+constexpr int kSpecCap = 800;        // nodes per T_j slot: 32 * 800 * 8 B = 200 KB of shared memory
+constexpr int kSpecStack = 64;
+struct SpecMeta {
+  int32_t P;      // padded T_j size of the group (max over its lanes), or -1: does not fit
+  int32_t D;      // steps: max leaf depth of the group's T_j
+};
+
+__device__ __forceinline__ uint32_t dse_resolve(const uint2* __restrict__ gnodes, const DseMap& map,
+                                                const float* __restrict__ grow, uint32_t k) {
+  // follow GPU-feature nodes with row j's features (the full walk's comparison)
+  for (;;) {
+    const uint2 nd = __ldg(gnodes + k);
+    const uint32_t left = nd.y & 0xFFFFFFu;
+    if (left == k) return k;  // leaf
+    const uint32_t code = map.code[nd.y >> 24];
+    if (!(code & 0x80u)) return k;  // CNN node
+    k = (__ldg(grow + (code & 0x7Fu)) > __uint_as_float(nd.x)) ? left + 1 : left;
+  }
+}
+
+// One thread per GPU row: pass 1 sizes / depths, pass 2 the interleaved nodes of T_j.
+__global__ void __launch_bounds__(32) dse_spec_kernel(const uint2* __restrict__ gnodes, DseMap map,
+                                                      const float* __restrict__ gpu, int64_t n_gpu, int dg,
+                                                      uint2* __restrict__ spec, SpecMeta* __restrict__ meta) {
+  const int lane = threadIdx.x;
+  const int64_t j = (int64_t)blockIdx.x * 32 + lane;
+  const bool live = j < n_gpu;
+  const float* grow = gpu + (live ? j : 0) * dg;
+  uint32_t stk[kSpecStack];  // (node, depth) packed: node < 2^24, depth < 2^8
+  int sp = 0;
+  uint32_t cnt = 1, dmax = 0;
+  bool ok = true;
+  if (live) {
+    stk[sp++] = dse_resolve(gnodes, map, grow, 0u) << 8;
+    while (sp > 0) {
+      const uint32_t e = stk[--sp];
+      const uint32_t k = e >> 8, dep = e & 0xFFu;
+      const uint2 nd = __ldg(gnodes + k);
+      const uint32_t left = nd.y & 0xFFFFFFu;
+      if (left == k) { dmax = max(dmax, dep); continue; }
+      cnt += 2;
+      if (sp + 2 > kSpecStack || dep + 1 > 255u) { ok = false; break; }
+      stk[sp++] = (dse_resolve(gnodes, map, grow, left + 1) << 8) | (dep + 1);
+      stk[sp++] = (dse_resolve(gnodes, map, grow, left) << 8) | (dep + 1);
+    }
+  }
+  const uint32_t P = __reduce_max_sync(0xffffffffu, cnt);
+  const uint32_t D = __reduce_max_sync(0xffffffffu, dmax);
+  const bool all_ok = __all_sync(0xffffffffu, ok) && P <= (uint32_t)kSpecCap;
+  if (lane == 0) meta[blockIdx.x] = SpecMeta{all_ok ? (int32_t)P : -1, (int32_t)D};
+  if (!all_ok) return;
+  uint2* out = spec + (size_t)blockIdx.x * kSpecCap * 32 + lane;
+  if (!live) {  // padding lane: one leaf (never written out)
+    out[0] = make_uint2(0x7fc00000u, 0u);
+    return;
+  }
+  // pass 2: slot s of node k; an internal node gets two consecutive slots for its children
+  sp = 0;
+  uint32_t nfree = 1;
+  stk[sp++] = dse_resolve(gnodes, map, grow, 0u) << 8;  // (node << 8) with slot in a parallel stack
+  uint32_t sslot[kSpecStack];
+  sslot[0] = 0;
+  while (sp > 0) {
+    --sp;
+    const uint32_t k = stk[sp] >> 8, slot = sslot[sp];
+    const uint2 nd = __ldg(gnodes + k);
+    const uint32_t left = nd.y & 0xFFFFFFu;
+    if (left == k) {
+      out[(size_t)slot * 32] = make_uint2(0x7fc00000u | k, slot);  // NaN(k): self-loop
+      continue;
+    }
+    const uint32_t a = nfree;
+    nfree += 2;
+    out[(size_t)slot * 32] = make_uint2(nd.x, ((uint32_t)map.code[nd.y >> 24] << 24) | a);
+    stk[sp] = dse_resolve(gnodes, map, grow, left + 1) << 8;
+    sslot[sp++] = a + 1;
+    stk[sp] = dse_resolve(gnodes, map, grow, left) << 8;
+    sslot[sp++] = a;
+  }
+}
+
+// Candidates (i, j): block = one group of 32 GPU rows (lane = j) x a range of CNN rows;
+// each warp walks kR CNN rows at once (independent chains) on the group's trees in
+// shared memory and writes yhat[i * n_gpu + j] for its 32 consecutive j (256 B per row).
+// A group whose trees do not fit (meta P = -1) walks the full tree from global memory.
+template <int kR>
 __global__ void __launch_bounds__(1024, 1)
-predict_dse_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ value, int count, int depth,
-                   const float* __restrict__ cnn, int64_t n_cnn, int dc, const float* __restrict__ gpu,
-                   int n_gpu, int dg, int p2, DseMap map, double* __restrict__ yhat) {
+predict_dse_spec_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ value, int depth, DseMap map,
+                        const uint2* __restrict__ spec, const SpecMeta* __restrict__ meta, int ngroups,
+                        const float* __restrict__ cnn, int64_t n_cnn, int dc, const float* __restrict__ gpu,
+                        int64_t n_gpu, int dg, double* __restrict__ yhat) {
   extern __shared__ __align__(16) unsigned char dse_smem[];
-  uint2* snodes = reinterpret_cast<uint2*>(dse_smem);
-  float* gpu_t = reinterpret_cast<float*>(dse_smem + (kSmemTree ? sizeof(uint2) * (size_t)count : 0));
-  float* cnn_s = gpu_t + (size_t)dg * n_gpu;
-  // kSorted: sort keys (p2 >= n_gpu, a power of two), the GPU order, output staging
-  unsigned long long* skey = reinterpret_cast<unsigned long long*>(
-      reinterpret_cast<unsigned char*>(cnn_s) + ((sizeof(float) * kR * dc + 15) & ~(size_t)15));
-  uint32_t* perm = reinterpret_cast<uint32_t*>(skey + (kSorted ? p2 : 0));
-  double* out_s = reinterpret_cast<double*>(perm + (kSorted ? ((n_gpu + 3) & ~3) : 0));
-  const int tid = threadIdx.x;
-  auto recode = [&](uint2 nd) {
-    nd.y = ((uint32_t)map.code[nd.y >> 24] << 24) | (nd.y & 0xFFFFFFu);
-    return nd;
-  };
-  if (kSmemTree) {
-    for (int k = tid; k < count; k += blockDim.x) snodes[k] = recode(gnodes[k]);
-    __syncthreads();
+  const int dcp = dc | 1;  // odd row pitch: the lanes' reads of one row hit distinct banks
+  uint2* tn = reinterpret_cast<uint2*>(dse_smem);
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+  float* cs = reinterpret_cast<float*>(dse_smem + (size_t)kSpecCap * 32 * sizeof(uint2)) + (size_t)w * kR * dcp;
+  const int g = (int)(blockIdx.x % (unsigned)ngroups);
+  const int64_t part = blockIdx.x / (unsigned)ngroups, nparts = gridDim.x / (unsigned)ngroups;
+  const SpecMeta mt = meta[g];
+  const int64_t j = (int64_t)g * 32 + lane;
+  const bool live = j < n_gpu;
+  if (mt.P > 0) {
+    const uint4* src = reinterpret_cast<const uint4*>(spec + (size_t)g * kSpecCap * 32);
+    uint4* dst = reinterpret_cast<uint4*>(tn);
+    for (int e = threadIdx.x; e < mt.P * 16; e += blockDim.x) dst[e] = __ldg(src + e);
   }
-  if (kSorted) {
-    // GPU rows grouped by the leaf they reach with CNN row 0: neighbouring threads then
-    // share most of their GPU-side decisions for any CNN, so a warp's node reads hit
-    // fewer distinct shared-memory words (broadcasts instead of bank conflicts).
-    for (int j = tid; j < p2; j += blockDim.x) {
-      unsigned long long key = ~0ull;
-      if (j < n_gpu) {
-        uint32_t k = 0;
-        for (int l = 0; l < depth; ++l) {
-          const uint2 nd = kSmemTree ? snodes[k] : recode(__ldg(gnodes + k));
-          const uint32_t code = nd.y >> 24, left = nd.y & 0xFFFFFFu;
-          const float x = (code & 0x80u) ? __ldg(gpu + (int64_t)j * dg + (code & 0x7Fu)) : __ldg(cnn + code);
-          k = (x > __uint_as_float(nd.x)) ? left + 1 : left;
-        }
-        key = ((unsigned long long)k << 32) | (uint32_t)j;
-      }
-      skey[j] = key;
+  __syncthreads();
+  // this block's CNN rows: [r0, r1), in warp tiles of kR rows
+  const int64_t per = (n_cnn + nparts - 1) / nparts;
+  const int64_t r0 = part * per, r1 = min(n_cnn, r0 + per);
+  const float* grow = gpu + (live ? j : 0) * dg;
+  for (int64_t i0 = r0 + (int64_t)w * kR; i0 < r1; i0 += (int64_t)nwarps * kR) {
+    __syncwarp();
+    for (int e = lane; e < kR * dc; e += 32) {
+      const int r = e / dc, c = e - r * dc;
+      cs[r * dcp + c] = (i0 + r < r1) ? __ldg(cnn + (i0 + r) * dc + c) : 0.f;
     }
-    __syncthreads();
-    for (int kk = 2; kk <= p2; kk <<= 1) {  // bitonic sort of (leaf, row)
-      for (int jj = kk >> 1; jj > 0; jj >>= 1) {
-        for (int i = tid; i < p2; i += blockDim.x) {
-          const int ixj = i ^ jj;
-          if (ixj > i) {
-            const unsigned long long u = skey[i], v = skey[ixj];
-            const bool up = (i & kk) == 0;
-            if ((u > v) == up) { skey[i] = v; skey[ixj] = u; }
-          }
-        }
-        __syncthreads();
-      }
-    }
-    for (int j = tid; j < n_gpu; j += blockDim.x) perm[j] = (uint32_t)skey[j];
-    __syncthreads();
-  }
-  for (int e = tid; e < dg * n_gpu; e += blockDim.x) {
-    const int g = e / n_gpu, j = e - g * n_gpu;
-    const int src = kSorted ? (int)perm[j] : j;
-    gpu_t[e] = __ldg(gpu + (int64_t)src * dg + g);
-  }
-  const int64_t nblk = (n_cnn + kR - 1) / kR;
-  for (int64_t b = blockIdx.x; b < nblk; b += gridDim.x) {
-    const int64_t i0 = b * kR;
-    __syncthreads();  // previous CNN rows consumed (and the tables above written)
-    for (int e = tid; e < kR * dc; e += blockDim.x) {
-      const int r = e / dc;
-      cnn_s[e] = (i0 + r < n_cnn) ? __ldg(cnn + (i0 + r) * dc + (e - r * dc)) : 0.f;
-    }
-    __syncthreads();
-    for (int j = tid; j < n_gpu; j += blockDim.x) {
-      uint32_t k[kR];
+    __syncwarp();
+    uint32_t k[kR];
 #pragma unroll
-      for (int r = 0; r < kR; ++r) k[r] = 0;
+    for (int r = 0; r < kR; ++r) k[r] = 0;
+    double v[kR];
+    if (mt.P > 0) {
+      for (int l = 0; l < mt.D; ++l) {
+#pragma unroll
+        for (int r = 0; r < kR; ++r) {
+          const uint2 nd = tn[k[r] * 32 + lane];
+          const float x = cs[r * dcp + (nd.y >> 24)];
+          k[r] = (nd.y & 0xFFFFFFu) + (x > __uint_as_float(nd.x) ? 1u : 0u);
+        }
+      }
+#pragma unroll
+      for (int r = 0; r < kR; ++r) v[r] = __ldg(value + (tn[k[r] * 32 + lane].x & 0x3FFFFFu));
+    } else {  // full tree, both tables from global memory
       for (int l = 0; l < depth; ++l) {
 #pragma unroll
         for (int r = 0; r < kR; ++r) {
-          const uint2 nd = kSmemTree ? snodes[k[r]] : recode(__ldg(gnodes + k[r]));
-          const uint32_t code = nd.y >> 24, left = nd.y & 0xFFFFFFu;
-          const float* src = (code & 0x80u) ? gpu_t + (code & 0x7Fu) * (uint32_t)n_gpu + j
-                                            : cnn_s + r * dc + code;
-          // go left iff !(x > RD32(t)) (Reading R5); leaves self-loop
-          k[r] = (*src > __uint_as_float(nd.x)) ? left + 1 : left;
+          const uint2 nd = __ldg(gnodes + k[r]);
+          const uint32_t code = map.code[nd.y >> 24], left = nd.y & 0xFFFFFFu;
+          const float x = (code & 0x80u) ? __ldg(grow + (code & 0x7Fu)) : cs[r * dcp + code];
+          k[r] = (x > __uint_as_float(nd.x)) ? left + 1 : left;
         }
       }
 #pragma unroll
-      for (int r = 0; r < kR; ++r) {
-        if (kSorted) out_s[r * n_gpu + perm[j]] = __ldg(value + k[r]);
-        else if (i0 + r < n_cnn) yhat[(i0 + r) * (int64_t)n_gpu + j] = __ldg(value + k[r]);
-      }
+      for (int r = 0; r < kR; ++r) v[r] = __ldg(value + k[r]);
     }
-    if (kSorted) {  // the staged rows, in GPU order, coalesced
-      __syncthreads();
-      for (int e = tid; e < kR * n_gpu; e += blockDim.x) {
-        const int r = e / n_gpu;
-        if (i0 + r < n_cnn) yhat[i0 * (int64_t)n_gpu + e] = out_s[e];
-      }
+    if (live) {
+#pragma unroll
+      for (int r = 0; r < kR; ++r)
+        if (i0 + r < r1) yhat[(i0 + r) * n_gpu + j] = v[r];
     }
   }
 }
@@ -549,31 +609,37 @@ dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, in
       map.code[f] = (uint8_t)(0x80 | g);
     }
   }
-  // kR CNN rows per thread: independent tree walks in flight (measured 2 / 4 / 6 / 8 / 12 /
-  // 16: 70 / 72 / 87 / 87 / 87 / 71 G predictions/s at 2^20 x 2^10)
+  if (n_cnn == 0 || n_gpu == 0) return DT_OK;
+  // the GPU-specialised trees of every group of 32 GPU rows (scratch from the stream's
+  // pool, freed in stream order), then the candidates
+  const int64_t ngroups = (n_gpu + 31) / 32;
+  uint2* spec = nullptr;
+  SpecMeta* meta = nullptr;
+  DT_CK(cudaMallocAsync((void**)&spec, sizeof(uint2) * (size_t)kSpecCap * 32 * (size_t)ngroups, s));
+  DT_CK(cudaMallocAsync((void**)&meta, sizeof(SpecMeta) * (size_t)ngroups, s));
+  const int pr = prof_begin(PK_PREDICT, s, 2);
+  if (t->count < ((int64_t)1 << 22)) {  // leaf ids fit the NaN payload of T_j leaves
+    dse_spec_kernel<<<(unsigned)ngroups, 32, 0, s>>>(t->dev_packed, map, gpu, n_gpu, dg, spec, meta);
+  } else {
+    DT_CK(cudaMemsetAsync(meta, 0xff, sizeof(SpecMeta) * (size_t)ngroups, s));  // P = -1: full walks
+  }
+  DT_CK(cudaGetLastError());
+  // kR CNN rows per warp: independent walks in flight
   constexpr int kR = 8, kThr = 1024;
-  const size_t cnn_bytes = (sizeof(float) * kR * (size_t)dc + 15) & ~(size_t)15;
-  const size_t tables = sizeof(float) * (size_t)dg * (size_t)n_gpu + cnn_bytes;
-  int p2 = 1;
-  while (p2 < n_gpu) p2 <<= 1;
-  const size_t sort_bytes = sizeof(unsigned long long) * (size_t)p2 + sizeof(uint32_t) * (size_t)((n_gpu + 3) & ~3) +
-                            sizeof(double) * kR * (size_t)n_gpu;
-  const size_t tree = sizeof(uint2) * (size_t)t->count;
-  const size_t cap = 227 * 1024;
-  if (tables > cap) return fail(DT_ERR_TOO_LARGE, "dt_predict_dse: GPU table too large for shared memory");
-  const bool smem_tree = tree + tables <= cap;
-  const bool sorted = (smem_tree ? tree : 0) + tables + sort_bytes <= cap;
-  const size_t sm = (smem_tree ? tree : 0) + tables + (sorted ? sort_bytes : 0);
-  auto kern = smem_tree ? (sorted ? predict_dse_kernel<true, true, kR> : predict_dse_kernel<true, false, kR>)
-                        : (sorted ? predict_dse_kernel<false, true, kR> : predict_dse_kernel<false, false, kR>);
+  const size_t sm = sizeof(uint2) * (size_t)kSpecCap * 32 + sizeof(float) * (size_t)(kThr / 32) * kR * (size_t)(dc | 1);
+  if (sm > 227 * 1024) return fail(DT_ERR_TOO_LARGE, "dt_predict_dse: dc too large");
+  auto kern = predict_dse_spec_kernel<kR>;
   DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
-  const int64_t nblk = (n_cnn + kR - 1) / kR;
-  const int64_t g = std::min<int64_t>((int64_t)num_sms(), nblk);
-  const int pr = prof_begin(PK_PREDICT, s, 1);
-  kern<<<(unsigned)g, kThr, sm, s>>>(t->dev_packed, t->dev_value, (int)t->count, t->depth, cnn, n_cnn, dc, gpu,
-                                     (int)n_gpu, dg, p2, map, yhat);
+  // blocks: every group x nparts row ranges, about 8 waves of the SMs
+  int64_t nparts = std::max<int64_t>(1, (8 * (int64_t)num_sms() + ngroups - 1) / ngroups);
+  nparts = std::min<int64_t>(nparts, std::max<int64_t>(1, (n_cnn + kR - 1) / kR));
+  nparts = std::min<int64_t>(nparts, (int64_t)0x7fffffff / ngroups);
+  kern<<<(unsigned)(ngroups * nparts), kThr, sm, s>>>(t->dev_packed, t->dev_value, t->depth, map, spec, meta,
+                                                     (int)ngroups, cnn, n_cnn, dc, gpu, n_gpu, dg, yhat);
   prof_end(pr, s, 8.0 * (double)n_cnn * (double)n_gpu);  // the yhat write (inputs are O(n_cnn + n_gpu))
   DT_CK(cudaGetLastError());
+  DT_CK(cudaFreeAsync(spec, s));
+  DT_CK(cudaFreeAsync(meta, s));
   return DT_OK;
 }
 

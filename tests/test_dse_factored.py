@@ -99,6 +99,52 @@ def test_predict_dse_rejects_bad_args(dt):
     bad[0] = 10  # CNN column out of range
     with pytest.raises(dt.DTError):
         dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), torch.from_numpy(gpu).cuda(), bad)
-    big = torch.zeros((1 << 16, 6), dtype=torch.float32, device="cuda")  # 1.5 MB table
-    with pytest.raises(dt.DTError):
-        dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), big, src)
+
+
+@pytest.mark.gpu
+def test_predict_dse_large_gpu_table(dt):
+    """2^16 GPU rows (2048 groups of GPU-specialised trees, no shared-memory table limit)
+    and a ragged last group: bit-exact against the composed rows."""
+    X, y = datagen.cnn_gpu_table(1, 50_000)
+    nodes = oracle.fit(X, y, 14, 8)
+    tree = dt.dt_tree_from_nodes(nodes, 16)
+    cnn, gpu, src = datagen.dse_tables(3, 0, 3, (1 << 16) - 5)
+    out = dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), torch.from_numpy(gpu).cuda(), src)
+    assert np.array_equal(out.cpu().numpy(), oracle.predict(nodes, _compose(cnn, gpu, src)))
+
+
+def _chain_tree(depth, src, rng):
+    """A caterpillar tree: internal node 2k (depth k) splits feature f_k, its left child
+    2k+1 is a leaf, its right child 2k+2 the next internal node; deeper than the
+    specialiser's stack for depth > 62 (the full-tree path)."""
+    import oracle as o
+    n = 2 * depth + 1
+    nodes = np.zeros(n, dtype=o.NODE_DTYPE)
+    nodes["feature"] = -1
+    nodes["left"] = -1
+    nodes["right"] = -1
+    for k in range(depth):
+        i = 2 * k
+        nodes[i]["feature"] = k % len(src)
+        nodes[i]["left"], nodes[i]["right"] = i + 1, i + 2
+        nodes[i]["threshold"] = float(rng.integers(0, 60))
+        nodes[i + 1]["depth"] = k + 1
+        nodes[i + 2]["depth"] = k + 1
+    nodes["value"] = np.arange(n, dtype=np.float64) * 1.5
+    nodes["n_samples"] = 1
+    return nodes
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("depth", [5, 61, 100])
+def test_predict_dse_deep_chain(dt, depth):
+    """Trees whose specialised walk needs every step (and, at depth 100, the full-tree
+    fallback): bit-exact."""
+    rng = np.random.default_rng(depth)
+    src = [0, -1, 1, -2, 2, -3]
+    nodes = _chain_tree(depth, src, rng)
+    tree = dt.dt_tree_from_nodes(nodes, len(src))
+    cnn = rng.integers(0, 64, size=(40, 3)).astype(np.float32)
+    gpu = rng.integers(0, 64, size=(70, 3)).astype(np.float32)
+    out = dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), torch.from_numpy(gpu).cuda(), src)
+    assert np.array_equal(out.cpu().numpy(), oracle.predict(nodes, _compose(cnn, gpu, src)))
