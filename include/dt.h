@@ -141,9 +141,12 @@ dt_status dt_predict(const dt_tree* tree, const float* X_dev, int64_t n, int32_t
  * from: c >= 0 -> CNN column c, -1 - g -> GPU column g.  Candidate (i, j) is the row
  * x[f] = feature_src[f] >= 0 ? cnn[i][feature_src[f]] : gpu[j][-1 - feature_src[f]], and
  * yhat_dev[i * n_gpu + j] (f64, n_cnn * n_gpu entries, CNN-major) is exactly what
- * dt_predict returns for that row.  1 <= dc, dg <= 128; the GPU table must fit shared
- * memory (dg * n_gpu * 4 B <= ~220 KB, e.g. 6 x 1024 GPUs); n_gpu < 2^24.  The tree sits
- * in shared memory when it fits beside the GPU table, else it is read through L1/L2.
+ * dt_predict returns for that row.  1 <= dc, dg <= 128; n_gpu < 2^24.  Method: per group
+ * of 32 GPU rows the tree is specialised (GPU-feature nodes resolved, CNN thresholds in
+ * rank form) into shared memory and each candidate walks only CNN-side decisions; groups
+ * whose specialised trees exceed 720 nodes, trees with > 4095 thresholds on one CNN
+ * column or of >= 2^22 nodes, and dc > 32 fall back to full-tree walks (same results).
+ * Scratch: ~184 KB per GPU group + 2 B per CNN table entry, from the stream-ordered pool.
  * Errors: INVALID_ARG (NULL pointers, bad feature_src), TOO_LARGE.  Async on stream. */
 dt_status dt_predict_dse(const dt_tree* tree, const float* cnn_dev, int64_t n_cnn, int32_t dc,
                          const float* gpu_dev, int64_t n_gpu, int32_t dg,

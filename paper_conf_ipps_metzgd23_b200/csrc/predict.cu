@@ -432,92 +432,208 @@ struct DseMap {
 // GPU-side decisions are fixed, so tree T_j = the tree with every GPU-feature node
 // replaced by the child row j takes.  T_j keeps only CNN-feature nodes and leaves (C2
 // tree, depth 20: ~220 of 11487 nodes, depth <= 13), and candidate (i, j) is a walk of
-// T_j on CNN row i -- the same comparisons x > RD32(t) as the full walk, in the same
-// order, so the reached leaf (hence yhat) is identical.  The 32 trees of a group of 32
-// consecutive GPU rows are stored interleaved (node k of lane j at word k * 32 + j), so a
-// warp's node reads are conflict-free whatever nodes its lanes sit on.  T_j node: {f32
-// threshold bits, CNN column << 24 | local left child (right = left + 1)}; T_j leaves
-// self-loop with threshold NaN (x > NaN is false) whose payload is the leaf's id in the
-// full tree (value index).
-constexpr int kSpecCap = 800;        // nodes per T_j slot: 32 * 800 * 8 B = 200 KB of shared memory
+// T_j on CNN row i making the full walk's CNN-side comparisons in the same order, so the
+// reached leaf (hence yhat) is identical.
+//
+// Rank form of the comparisons (4-byte nodes): per CNN column c, T_c = the thresholds
+// RD32(t) of the tree's nodes on column c, sorted (duplicates kept); rank(t) = #{t' in
+// T_c : t' < t} and r(x) = #{t' in T_c : t' < x}.  Then x > t <=> r(x) > rank(t) (if t < x
+// every t' <= t is below x, so r(x) >= rank(t) + 1; if t >= x, r(x) <= rank(t)), NaN x
+// has r = 0 (goes left, as x > t is false).  A T_j node is one word: rank << 20 | local
+// left child a << 7 (right = a + 1; a * 128 is the child's byte offset in the interleaved
+// layout) | CNN column * 4 (its byte offset in a rank row); leaves self-loop with rank 0xFFF
+// (never exceeded: r(x) <= |T_c| <= kRankCap) and keep their full-tree id in a parallel
+// word.  The 32 trees of a group of 32 consecutive GPU rows are interleaved (node k of
+// lane j at word k * 32 + j), so a warp's node reads hit 32 distinct banks whatever nodes
+// its lanes sit on: one shared-memory wavefront per node read, one per CNN rank read (the
+// lanes read one row, pitch kRowPitch words).
+constexpr int kSpecCap = 720;      // slots per T_j: 32 x 720 x (4 + 4) B = 180 KB of shared memory
 constexpr int kSpecStack = 64;
+constexpr int kRankCap = 4095;     // thresholds per CNN column in rank form (12-bit ranks)
+constexpr int kSpecMaxCols = 32;   // CNN columns of the rank form
+constexpr int kRowPitch = 33;      // words per staged CNN rank row (odd: conflict-free)
 struct SpecMeta {
-  int32_t P;      // padded T_j size of the group (max over its lanes), or -1: does not fit
+  int32_t P;      // padded T_j size of the group (max over its lanes), or -1: full-tree walks
   int32_t D;      // steps: max leaf depth of the group's T_j
 };
 
-__device__ __forceinline__ uint32_t dse_resolve(const uint2* __restrict__ gnodes, const DseMap& map,
+// Block c: T_c (bitonic sort in shared memory, duplicates kept) and rank(t) of every tree
+// node on column c (lower bound in T_c).
+__global__ void __launch_bounds__(512) dse_rank_kernel(const uint2* __restrict__ gnodes, int count, DseMap map,
+                                                       float* __restrict__ rt, uint32_t* __restrict__ rn,
+                                                       uint16_t* __restrict__ nrank, int* __restrict__ bad) {
+  __shared__ float th[4096];
+  __shared__ uint32_t nk[kRankCap];
+  __shared__ uint32_t s_n;
+  const uint32_t c = blockIdx.x;
+  if (threadIdx.x == 0) s_n = 0u;
+  __syncthreads();
+  for (int k = threadIdx.x; k < count; k += blockDim.x) {
+    const uint2 nd = __ldg(gnodes + k);
+    if ((nd.y & 0xFFFFFFu) == (uint32_t)k) continue;  // leaf
+    if (map.code[nd.y >> 24] != c) continue;          // another column (or a GPU column)
+    const uint32_t q = atomicAdd(&s_n, 1u);
+    if (q < (uint32_t)kRankCap) {
+      th[q] = __uint_as_float(nd.x);
+      nk[q] = (uint32_t)k;
+    }
+  }
+  __syncthreads();
+  const uint32_t n = s_n;
+  if (n > (uint32_t)kRankCap) {
+    if (threadIdx.x == 0) *bad = 1;
+    return;
+  }
+  uint32_t p2 = 1u;
+  while (p2 < n) p2 <<= 1;
+  for (uint32_t q = n + threadIdx.x; q < p2; q += blockDim.x) th[q] = INFINITY;  // thresholds are finite
+  __syncthreads();
+  for (uint32_t kk = 2; kk <= p2; kk <<= 1) {
+    for (uint32_t jj = kk >> 1; jj > 0; jj >>= 1) {
+      for (uint32_t i = threadIdx.x; i < p2; i += blockDim.x) {
+        const uint32_t ixj = i ^ jj;
+        if (ixj > i) {
+          const float u = th[i], v = th[ixj];
+          if ((u > v) == ((i & kk) == 0)) { th[i] = v; th[ixj] = u; }
+        }
+      }
+      __syncthreads();
+    }
+  }
+  for (uint32_t q = threadIdx.x; q < n; q += blockDim.x) rt[(size_t)c * kRankCap + q] = th[q];
+  // rank of each collected node: lower bound of its threshold
+  for (uint32_t q = threadIdx.x; q < n; q += blockDim.x) {
+    const float t = __uint_as_float(__ldg(gnodes + nk[q]).x);
+    uint32_t lo = 0u, hi = n;
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (th[mid] < t) lo = mid + 1u;
+      else hi = mid;
+    }
+    nrank[nk[q]] = (uint16_t)lo;
+  }
+  if (threadIdx.x == 0) rn[c] = n;
+}
+
+// r(x) of every CNN table entry (binary search in T_c).
+__global__ void __launch_bounds__(256) dse_cnn_rank_kernel(const float* __restrict__ cnn, int64_t total, int dc,
+                                                           const float* __restrict__ rt, const uint32_t* __restrict__ rn,
+                                                           uint16_t* __restrict__ crank) {
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+    const int c = (int)(e % dc);
+    const float x = __ldg(cnn + e);
+    const float* T = rt + (size_t)c * kRankCap;
+    uint32_t lo = 0u, hi = c < kSpecMaxCols ? __ldg(rn + c) : 0u;  // first index with !(T < x)
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (__ldg(T + mid) < x) lo = mid + 1u;
+      else hi = mid;
+    }
+    crank[e] = (uint16_t)lo;
+  }
+}
+
+// The specialiser reads the packed tree and the node ranks from shared memory when they
+// fit (every DFS step is a dependent load), else from global memory.
+template <bool kSmem>
+struct SpecTree {
+  const uint2* nodes;
+  const uint16_t* rank;
+  __device__ __forceinline__ uint2 node(uint32_t k) const { return kSmem ? nodes[k] : __ldg(nodes + k); }
+  __device__ __forceinline__ uint32_t rk(uint32_t k) const { return kSmem ? rank[k] : __ldg(rank + k); }
+};
+
+template <bool kSmem>
+__device__ __forceinline__ uint32_t dse_resolve(const SpecTree<kSmem>& tr, const DseMap& map,
                                                 const float* __restrict__ grow, uint32_t k) {
   // follow GPU-feature nodes with row j's features (the full walk's comparison)
   for (;;) {
-    const uint2 nd = __ldg(gnodes + k);
+    const uint2 nd = tr.node(k);
     const uint32_t left = nd.y & 0xFFFFFFu;
     if (left == k) return k;  // leaf
     const uint32_t code = map.code[nd.y >> 24];
     if (!(code & 0x80u)) return k;  // CNN node
-    k = (__ldg(grow + (code & 0x7Fu)) > __uint_as_float(nd.x)) ? left + 1 : left;
+    k = (grow[code & 0x7Fu] > __uint_as_float(nd.x)) ? left + 1 : left;
   }
 }
 
-// One thread per GPU row: pass 1 sizes / depths, pass 2 the interleaved nodes of T_j.
-__global__ void __launch_bounds__(32) dse_spec_kernel(const uint2* __restrict__ gnodes, DseMap map,
-                                                      const float* __restrict__ gpu, int64_t n_gpu, int dg,
-                                                      uint2* __restrict__ spec, SpecMeta* __restrict__ meta) {
-  const int lane = threadIdx.x;
-  const int64_t j = (int64_t)blockIdx.x * 32 + lane;
-  const bool live = j < n_gpu;
-  const float* grow = gpu + (live ? j : 0) * dg;
-  uint32_t stk[kSpecStack];  // (node, depth) packed: node < 2^24, depth < 2^8
+// Lane j of block g: T_j in one depth-first pass (an internal node gets two consecutive
+// slots for its children), written straight to the group's interleaved slots; a lane
+// whose tree outgrows kSpecCap (or the stack, or the rank form) fails the whole group.
+template <bool kSmem>
+__device__ void dse_spec_build(const SpecTree<kSmem>& tr, const DseMap& map, const float* __restrict__ grow,
+                               bool live, bool ok, uint32_t* __restrict__ spec, SpecMeta* __restrict__ meta) {
+  const int lane = threadIdx.x & 31;
+  uint32_t* out = spec + (size_t)blockIdx.x * kSpecCap * 64 + lane;  // nodes, then leaf ids
+  uint32_t* lid = out + (size_t)kSpecCap * 32;
+  uint32_t stk[kSpecStack], sslot[kSpecStack];  // pending (node << 8 | depth, slot)
   int sp = 0;
-  uint32_t cnt = 1, dmax = 0;
-  bool ok = true;
-  if (live) {
-    stk[sp++] = dse_resolve(gnodes, map, grow, 0u) << 8;
+  uint32_t nfree = 1, dmax = 0;
+  if (!live) {  // padding lane: one leaf (its outputs are never written)
+    out[0] = 0xFFF00000u;
+    lid[0] = 0u;
+  } else if (ok) {
+    stk[sp] = dse_resolve(tr, map, grow, 0u) << 8;
+    sslot[sp++] = 0u;
     while (sp > 0) {
-      const uint32_t e = stk[--sp];
-      const uint32_t k = e >> 8, dep = e & 0xFFu;
-      const uint2 nd = __ldg(gnodes + k);
+      --sp;
+      const uint32_t k = stk[sp] >> 8, dep = stk[sp] & 0xFFu, slot = sslot[sp];
+      const uint2 nd = tr.node(k);
       const uint32_t left = nd.y & 0xFFFFFFu;
-      if (left == k) { dmax = max(dmax, dep); continue; }
-      cnt += 2;
-      if (sp + 2 > kSpecStack || dep + 1 > 255u) { ok = false; break; }
-      stk[sp++] = (dse_resolve(gnodes, map, grow, left + 1) << 8) | (dep + 1);
-      stk[sp++] = (dse_resolve(gnodes, map, grow, left) << 8) | (dep + 1);
+      if (left == k) {
+        out[(size_t)slot * 32] = 0xFFF00000u | (slot << 7);  // self-loop, rank never exceeded
+        lid[(size_t)slot * 32] = k;
+        dmax = max(dmax, dep);
+        continue;
+      }
+      const uint32_t code = map.code[nd.y >> 24];
+      const uint32_t a = nfree;
+      nfree += 2;
+      if (sp + 2 > kSpecStack || dep + 1 > 255u || nfree > (uint32_t)kSpecCap || code >= (uint32_t)kSpecMaxCols) {
+        ok = false;
+        break;
+      }
+      out[(size_t)slot * 32] = (tr.rk(k) << 20) | (a << 7) | (code << 2);
+      stk[sp] = (dse_resolve(tr, map, grow, left + 1) << 8) | (dep + 1);
+      sslot[sp++] = a + 1;
+      stk[sp] = (dse_resolve(tr, map, grow, left) << 8) | (dep + 1);
+      sslot[sp++] = a;
     }
   }
-  const uint32_t P = __reduce_max_sync(0xffffffffu, cnt);
+  const uint32_t P = __reduce_max_sync(0xffffffffu, nfree);
   const uint32_t D = __reduce_max_sync(0xffffffffu, dmax);
-  const bool all_ok = __all_sync(0xffffffffu, ok) && P <= (uint32_t)kSpecCap;
+  const bool all_ok = __all_sync(0xffffffffu, ok);
   if (lane == 0) meta[blockIdx.x] = SpecMeta{all_ok ? (int32_t)P : -1, (int32_t)D};
-  if (!all_ok) return;
-  uint2* out = spec + (size_t)blockIdx.x * kSpecCap * 32 + lane;
-  if (!live) {  // padding lane: one leaf (never written out)
-    out[0] = make_uint2(0x7fc00000u, 0u);
-    return;
+}
+
+// Block g (256 threads): the packed tree, the node ranks and the group's GPU rows staged
+// in shared memory (the tree when it fits), then warp 0 builds the group's 32 trees.
+__global__ void __launch_bounds__(256) dse_spec_kernel(const uint2* __restrict__ gnodes, int count, DseMap map,
+                                                       const float* __restrict__ gpu, int64_t n_gpu, int dg,
+                                                       const uint16_t* __restrict__ nrank, const int* __restrict__ bad,
+                                                       bool smem_tree, uint32_t* __restrict__ spec,
+                                                       SpecMeta* __restrict__ meta) {
+  extern __shared__ __align__(16) unsigned char spec_smem[];
+  const bool ok = *bad == 0;
+  float* sg = reinterpret_cast<float*>(spec_smem);  // 32 x dg
+  for (int e = threadIdx.x; e < 32 * dg; e += blockDim.x) {
+    const int64_t jj = (int64_t)blockIdx.x * 32 + e / dg;
+    sg[e] = jj < n_gpu ? __ldg(gpu + jj * dg + e % dg) : 0.f;
   }
-  // pass 2: slot s of node k; an internal node gets two consecutive slots for its children
-  sp = 0;
-  uint32_t nfree = 1;
-  stk[sp++] = dse_resolve(gnodes, map, grow, 0u) << 8;  // (node << 8) with slot in a parallel stack
-  uint32_t sslot[kSpecStack];
-  sslot[0] = 0;
-  while (sp > 0) {
-    --sp;
-    const uint32_t k = stk[sp] >> 8, slot = sslot[sp];
-    const uint2 nd = __ldg(gnodes + k);
-    const uint32_t left = nd.y & 0xFFFFFFu;
-    if (left == k) {
-      out[(size_t)slot * 32] = make_uint2(0x7fc00000u | k, slot);  // NaN(k): self-loop
-      continue;
+  uint2* sn = reinterpret_cast<uint2*>(spec_smem + ((sizeof(float) * 32 * (size_t)dg + 15) & ~(size_t)15));
+  uint16_t* sr = reinterpret_cast<uint16_t*>(sn + count);
+  if (smem_tree) {
+    for (int k = threadIdx.x; k < count; k += blockDim.x) {
+      sn[k] = __ldg(gnodes + k);
+      sr[k] = ok ? __ldg(nrank + k) : (uint16_t)0;
     }
-    const uint32_t a = nfree;
-    nfree += 2;
-    out[(size_t)slot * 32] = make_uint2(nd.x, ((uint32_t)map.code[nd.y >> 24] << 24) | a);
-    stk[sp] = dse_resolve(gnodes, map, grow, left + 1) << 8;
-    sslot[sp++] = a + 1;
-    stk[sp] = dse_resolve(gnodes, map, grow, left) << 8;
-    sslot[sp++] = a;
   }
+  __syncthreads();
+  if (threadIdx.x >= 32) return;
+  const bool live = (int64_t)blockIdx.x * 32 + threadIdx.x < n_gpu;
+  const float* grow = sg + threadIdx.x * dg;
+  if (smem_tree) dse_spec_build(SpecTree<true>{sn, sr}, map, grow, live, ok, spec, meta);
+  else dse_spec_build(SpecTree<false>{gnodes, nrank}, map, grow, live, ok, spec, meta);
 }
 
 // Candidates (i, j): block = one group of 32 GPU rows (lane = j) x a range of CNN rows;
@@ -527,58 +643,78 @@ __global__ void __launch_bounds__(32) dse_spec_kernel(const uint2* __restrict__ 
 template <int kR>
 __global__ void __launch_bounds__(1024, 1)
 predict_dse_spec_kernel(const uint2* __restrict__ gnodes, const double* __restrict__ value, int depth, DseMap map,
-                        const uint2* __restrict__ spec, const SpecMeta* __restrict__ meta, int ngroups,
-                        const float* __restrict__ cnn, int64_t n_cnn, int dc, const float* __restrict__ gpu,
-                        int64_t n_gpu, int dg, double* __restrict__ yhat) {
+                        const uint32_t* __restrict__ spec, const SpecMeta* __restrict__ meta, int ngroups,
+                        const float* __restrict__ cnn, const uint16_t* __restrict__ crank, int64_t n_cnn, int dc,
+                        const float* __restrict__ gpu, int64_t n_gpu, int dg, double* __restrict__ yhat) {
   extern __shared__ __align__(16) unsigned char dse_smem[];
-  const int dcp = dc | 1;  // odd row pitch: the lanes' reads of one row hit distinct banks
-  uint2* tn = reinterpret_cast<uint2*>(dse_smem);
+  uint32_t* tn = reinterpret_cast<uint32_t*>(dse_smem);
+  uint32_t* tl = tn + (size_t)kSpecCap * 32;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
-  float* cs = reinterpret_cast<float*>(dse_smem + (size_t)kSpecCap * 32 * sizeof(uint2)) + (size_t)w * kR * dcp;
+  uint32_t* cs = tl + (size_t)kSpecCap * 32 + (size_t)w * kR * kRowPitch;
   const int g = (int)(blockIdx.x % (unsigned)ngroups);
   const int64_t part = blockIdx.x / (unsigned)ngroups, nparts = gridDim.x / (unsigned)ngroups;
   const SpecMeta mt = meta[g];
   const int64_t j = (int64_t)g * 32 + lane;
   const bool live = j < n_gpu;
   if (mt.P > 0) {
-    const uint4* src = reinterpret_cast<const uint4*>(spec + (size_t)g * kSpecCap * 32);
+    const uint4* src = reinterpret_cast<const uint4*>(spec + (size_t)g * kSpecCap * 64);
     uint4* dst = reinterpret_cast<uint4*>(tn);
-    for (int e = threadIdx.x; e < mt.P * 16; e += blockDim.x) dst[e] = __ldg(src + e);
+    const int n4 = mt.P * 8;  // P slots x 32 lanes x 4 B / 16 B
+    for (int e = threadIdx.x; e < n4; e += blockDim.x) {
+      dst[e] = __ldg(src + e);
+      dst[kSpecCap * 8 + e] = __ldg(src + kSpecCap * 8 + e);
+    }
   }
   __syncthreads();
   // this block's CNN rows: [r0, r1), in warp tiles of kR rows
   const int64_t per = (n_cnn + nparts - 1) / nparts;
   const int64_t r0 = part * per, r1 = min(n_cnn, r0 + per);
   const float* grow = gpu + (live ? j : 0) * dg;
+  // shared byte addresses: my slot-0 word of the trees, my warp's rank rows.  The walk
+  // loads are plain (schedulable) asm; these addresses pass through volatile movs placed
+  // after the barriers that publish the data, so no load can be hoisted above them.
+  uint32_t tn0, cs0;
+  asm volatile("mov.u32 %0, %1;" : "=r"(tn0) : "r"((uint32_t)__cvta_generic_to_shared(tn) + 4u * lane));
   for (int64_t i0 = r0 + (int64_t)w * kR; i0 < r1; i0 += (int64_t)nwarps * kR) {
-    __syncwarp();
-    for (int e = lane; e < kR * dc; e += 32) {
-      const int r = e / dc, c = e - r * dc;
-      cs[r * dcp + c] = (i0 + r < r1) ? __ldg(cnn + (i0 + r) * dc + c) : 0.f;
-    }
-    __syncwarp();
-    uint32_t k[kR];
-#pragma unroll
-    for (int r = 0; r < kR; ++r) k[r] = 0;
     double v[kR];
     if (mt.P > 0) {
+      __syncwarp();
+      for (int e = lane; e < kR * dc; e += 32) {
+        const int r = e / dc, c = e - r * dc;
+        cs[r * kRowPitch + c] = (i0 + r < r1) ? (uint32_t)__ldg(crank + (i0 + r) * dc + c) : 0u;
+      }
+      __syncwarp();
+      asm volatile("mov.u32 %0, %1;" : "=r"(cs0) : "r"((uint32_t)__cvta_generic_to_shared(cs)));
+      uint32_t ka[kR];  // shared byte address of my current node, per row
+#pragma unroll
+      for (int r = 0; r < kR; ++r) ka[r] = tn0;
       for (int l = 0; l < mt.D; ++l) {
 #pragma unroll
         for (int r = 0; r < kR; ++r) {
-          const uint2 nd = tn[k[r] * 32 + lane];
-          const float x = cs[r * dcp + (nd.y >> 24)];
-          k[r] = (nd.y & 0xFFFFFFu) + (x > __uint_as_float(nd.x) ? 1u : 0u);
+          uint32_t nd, xr;
+          asm("ld.shared.u32 %0, [%1];" : "=r"(nd) : "r"(ka[r]));
+          asm("ld.shared.u32 %0, [%1];" : "=r"(xr) : "r"(cs0 + (uint32_t)(r * kRowPitch * 4) + (nd & 0x7Cu)));
+          // child word: my slot-0 word + (a + go) * 128 B
+          ka[r] = tn0 + (nd & 0xFFF80u) + (xr > (nd >> 20) ? 128u : 0u);
         }
       }
 #pragma unroll
-      for (int r = 0; r < kR; ++r) v[r] = __ldg(value + (tn[k[r] * 32 + lane].x & 0x3FFFFFu));
+      for (int r = 0; r < kR; ++r) {
+        uint32_t id;
+        asm("ld.shared.u32 %0, [%1];" : "=r"(id) : "r"(ka[r] + (uint32_t)(kSpecCap * 32 * 4)));
+        v[r] = __ldg(value + id);
+      }
     } else {  // full tree, both tables from global memory
+      uint32_t k[kR];
+#pragma unroll
+      for (int r = 0; r < kR; ++r) k[r] = 0;
       for (int l = 0; l < depth; ++l) {
 #pragma unroll
         for (int r = 0; r < kR; ++r) {
           const uint2 nd = __ldg(gnodes + k[r]);
           const uint32_t code = map.code[nd.y >> 24], left = nd.y & 0xFFFFFFu;
-          const float x = (code & 0x80u) ? __ldg(grow + (code & 0x7Fu)) : cs[r * dcp + code];
+          const int64_t ir = min(i0 + r, n_cnn - 1);
+          const float x = (code & 0x80u) ? __ldg(grow + (code & 0x7Fu)) : __ldg(cnn + ir * dc + code);
           k[r] = (x > __uint_as_float(nd.x)) ? left + 1 : left;
         }
       }
@@ -610,24 +746,46 @@ dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, in
     }
   }
   if (n_cnn == 0 || n_gpu == 0) return DT_OK;
-  // the GPU-specialised trees of every group of 32 GPU rows (scratch from the stream's
-  // pool, freed in stream order), then the candidates
+  // rank tables, the GPU-specialised trees of every group of 32 GPU rows (scratch from
+  // the stream's pool, freed in stream order), then the candidates
   const int64_t ngroups = (n_gpu + 31) / 32;
-  uint2* spec = nullptr;
-  SpecMeta* meta = nullptr;
-  DT_CK(cudaMallocAsync((void**)&spec, sizeof(uint2) * (size_t)kSpecCap * 32 * (size_t)ngroups, s));
-  DT_CK(cudaMallocAsync((void**)&meta, sizeof(SpecMeta) * (size_t)ngroups, s));
-  const int pr = prof_begin(PK_PREDICT, s, 2);
-  if (t->count < ((int64_t)1 << 22)) {  // leaf ids fit the NaN payload of T_j leaves
-    dse_spec_kernel<<<(unsigned)ngroups, 32, 0, s>>>(t->dev_packed, map, gpu, n_gpu, dg, spec, meta);
-  } else {
-    DT_CK(cudaMemsetAsync(meta, 0xff, sizeof(SpecMeta) * (size_t)ngroups, s));  // P = -1: full walks
-  }
+  const int ncols = std::min<int>(dc, kSpecMaxCols);
+  unsigned char* scratch = nullptr;
+  const size_t b_spec = sizeof(uint32_t) * (size_t)kSpecCap * 64 * (size_t)ngroups;
+  const size_t b_meta = sizeof(SpecMeta) * (size_t)ngroups;
+  const size_t b_rt = sizeof(float) * (size_t)kRankCap * kSpecMaxCols;
+  const size_t b_rn = sizeof(uint32_t) * kSpecMaxCols + 16;  // + the bad flag
+  const size_t b_nr = ((sizeof(uint16_t) * (size_t)t->count) + 15) & ~(size_t)15;
+  const size_t b_cr = sizeof(uint16_t) * (size_t)n_cnn * (size_t)dc;
+  DT_CK(cudaMallocAsync((void**)&scratch, b_spec + b_meta + b_rt + b_rn + b_nr + b_cr, s));
+  uint32_t* spec = reinterpret_cast<uint32_t*>(scratch);
+  SpecMeta* meta = reinterpret_cast<SpecMeta*>(scratch + b_spec);
+  float* rt = reinterpret_cast<float*>(scratch + b_spec + b_meta);
+  uint32_t* rn = reinterpret_cast<uint32_t*>(scratch + b_spec + b_meta + b_rt);
+  int* bad = reinterpret_cast<int*>(rn + kSpecMaxCols);
+  uint16_t* nrank = reinterpret_cast<uint16_t*>(scratch + b_spec + b_meta + b_rt + b_rn);
+  uint16_t* crank = reinterpret_cast<uint16_t*>(scratch + b_spec + b_meta + b_rt + b_rn + b_nr);
+  const int pr = prof_begin(PK_PREDICT, s, 4);
+  DT_CK(cudaMemsetAsync(rn, 0, b_rn, s));
+  if (dc > kSpecMaxCols) DT_CK(cudaMemsetAsync(bad, 0xff, sizeof(int), s));  // rank rows hold <= 32 columns
+  if (ncols > 0)
+    dse_rank_kernel<<<(unsigned)ncols, 512, 0, s>>>(t->dev_packed, (int)t->count, map, rt, rn, nrank, bad);
+  DT_CK(cudaGetLastError());
+  const int64_t total = n_cnn * (int64_t)dc;
+  dse_cnn_rank_kernel<<<(unsigned)std::min<int64_t>((total + 255) / 256, (int64_t)num_sms() * 16), 256, 0, s>>>(
+      cnn, total, dc, rt, rn, crank);
+  DT_CK(cudaGetLastError());
+  const size_t g_sm = (sizeof(float) * 32 * (size_t)dg + 15) & ~(size_t)15;
+  const size_t tree_sm = (sizeof(uint2) + sizeof(uint16_t)) * (size_t)t->count;
+  const bool smem_tree = g_sm + tree_sm <= 200 * 1024;
+  const size_t spec_sm = g_sm + (smem_tree ? tree_sm : 0);
+  DT_CK(cudaFuncSetAttribute(dse_spec_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)spec_sm));
+  dse_spec_kernel<<<(unsigned)ngroups, 256, spec_sm, s>>>(t->dev_packed, (int)t->count, map, gpu, n_gpu, dg, nrank,
+                                                         bad, smem_tree, spec, meta);
   DT_CK(cudaGetLastError());
   // kR CNN rows per warp: independent walks in flight
   constexpr int kR = 8, kThr = 1024;
-  const size_t sm = sizeof(uint2) * (size_t)kSpecCap * 32 + sizeof(float) * (size_t)(kThr / 32) * kR * (size_t)(dc | 1);
-  if (sm > 227 * 1024) return fail(DT_ERR_TOO_LARGE, "dt_predict_dse: dc too large");
+  const size_t sm = sizeof(uint32_t) * (size_t)kSpecCap * 64 + sizeof(uint32_t) * (size_t)(kThr / 32) * kR * kRowPitch;
   auto kern = predict_dse_spec_kernel<kR>;
   DT_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
   // blocks: every group x nparts row ranges, about 8 waves of the SMs
@@ -635,11 +793,10 @@ dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, in
   nparts = std::min<int64_t>(nparts, std::max<int64_t>(1, (n_cnn + kR - 1) / kR));
   nparts = std::min<int64_t>(nparts, (int64_t)0x7fffffff / ngroups);
   kern<<<(unsigned)(ngroups * nparts), kThr, sm, s>>>(t->dev_packed, t->dev_value, t->depth, map, spec, meta,
-                                                     (int)ngroups, cnn, n_cnn, dc, gpu, n_gpu, dg, yhat);
+                                                     (int)ngroups, cnn, crank, n_cnn, dc, gpu, n_gpu, dg, yhat);
   prof_end(pr, s, 8.0 * (double)n_cnn * (double)n_gpu);  // the yhat write (inputs are O(n_cnn + n_gpu))
   DT_CK(cudaGetLastError());
-  DT_CK(cudaFreeAsync(spec, s));
-  DT_CK(cudaFreeAsync(meta, s));
+  DT_CK(cudaFreeAsync(scratch, s));
   return DT_OK;
 }
 
