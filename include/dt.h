@@ -145,7 +145,7 @@ dt_status dt_predict(const dt_tree* tree, const float* X_dev, int64_t n, int32_t
  * of 32 GPU rows the tree is specialised (GPU-feature nodes resolved, CNN thresholds in
  * rank form) into shared memory and each candidate walks only CNN-side decisions; groups
  * whose specialised trees exceed 720 nodes, trees with > 4095 thresholds on one CNN
- * column or of >= 2^22 nodes, and dc > 32 fall back to full-tree walks (same results).
+ * column, and dc > 32 fall back to full-tree walks (same results).
  * Scratch: ~184 KB per GPU group + 2 B per CNN table entry, from the stream-ordered pool.
  * Errors: INVALID_ARG (NULL pointers, bad feature_src), TOO_LARGE.  Async on stream. */
 dt_status dt_predict_dse(const dt_tree* tree, const float* cnn_dev, int64_t n_cnn, int32_t dc,

@@ -840,6 +840,38 @@ __global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArg
         if ((g ? w0 : w1) && b0 < hi) a.desc_next[b0 / kChunkW] = ps.cs[g ? 0 : 1];
       }
     }
+    // ---- a chunk (piece) of one x value (few-valued columns: GPU descriptors): no prefix
+    // sums are needed -- a child's only possible split position in it is its first item
+    // (x there differs from the child's previous x iff the carried x is smaller), whose
+    // S'_L is the chunk carry, and the statistics come from feature 0 only (ps.f != 0)
+    if (full && ps.f != 0 && sx[e_lo] == sx[e_hi - 1]) {
+      const bool anyL = __ballot_sync(0xffffffffu, lbyte != 0u) != 0u;
+      const bool anyR = __ballot_sync(0xffffffffu, rbyte != 0u) != 0u;
+      const float xc = sx[e_lo];
+      __syncwarp();  // the stage is read completely: refill it
+      if (lane == 0) {
+        if (nxt < nfast) issue(s, ahead);
+        if (nxt + nw < nfast) ahead = a.unit_list[nxt + nw];
+      }
+      const int sd = lane;
+      if (lane < 2 && (flags & (sd ? PS_SRCH1 : PS_SRCH0)) && (sd ? anyR : anyL)) {
+        float xp = sd ? carry.xr : carry.xl;
+        if (isnan(xp)) xp = ps.xprev[sd];
+        // the child's items before this one: lefts before the chunk, or rights before it
+        const uint32_t jl = sd ? ib + (uint32_t)e_lo - carry.nl : carry.nl;
+        const uint32_t io = ps.ioff[sd];
+        const uint32_t lo = ilo > io ? ilo - io : 0u;
+        const uint32_t hi = ps.N[sd] >= m + io ? ps.N[sd] - m - io + 1u : 0u;
+        if (jl >= lo && jl < hi && xp < xc) {
+          // S'_L exactly as the item scan forms it: carry + (+0.0 lane prefix)
+          const double S = __dadd_rn(ps.soff[sd], __dadd_rn(sd ? carry.sr : carry.sl, 0.0));
+          const double gn = split_gain_d(S, ps.sc[sd], (double)(io + jl), (double)ps.N[sd]);
+          put_cand(a, headc, ch, sd, ps.cs[sd], gn, S, mid_threshold(xp, xc), io + jl);
+        }
+      }
+      if (++s == kStages) { s = 0; phase ^= 1u; }
+      continue;
+    }
     // ---- left count before my items, neighbour x across lanes
     uint32_t nl = carry.nl;
     {
