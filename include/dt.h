@@ -312,7 +312,11 @@ dt_status dt_eval_sharded(dt_comm* comm, const double* y_dev, const double* yhat
  * launches, tagged with the kernel kind and the launch's ALGORITHMIC bytes (DESIGN.md,
  * "Roofline"); dt_profile_get synchronises those events and returns, for one kind, the
  * number of launches, the summed device time (ms) and the summed algorithmic bytes.
- * dt_launch_count counts this library's own kernel launches since the last reset. */
+ * dt_launch_count counts this library's own kernel launches since the last reset.
+ * on = 1: events on the stream (a bounded-depth dt_fit then enqueues directly instead of
+ * replaying its graph); on = 2: dt_fit keeps its cached CUDA graph, captured once more
+ * with event-record nodes around the same kernel groups, and each replay's times are
+ * collected when the call returns; on = 0: off. */
 void dt_profile_enable(int on);
 void dt_profile_reset(void);
 int64_t dt_launch_count(void);

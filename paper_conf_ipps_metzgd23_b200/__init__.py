@@ -313,8 +313,10 @@ def dt_gen_dse(seed: int, row0: int, n: int, gpu_bits: int = 10, out=None, devic
     return out
 
 
-def dt_profile_enable(on: bool = True):
-    _lib.dt_profile_enable(1 if on else 0)
+def dt_profile_enable(on: bool = True, graph: bool = False):
+    """Measurement hooks (include/dt.h): graph=True keeps dt_fit's CUDA-graph replay and
+    times its kernel groups with event-record nodes inside the graph."""
+    _lib.dt_profile_enable((2 if graph else 1) if on else 0)
 
 
 def dt_profile_reset():

@@ -108,6 +108,16 @@ int prof_begin(int kind, cudaStream_t s, int nlaunch);
 void prof_end(int idx, cudaStream_t s, double alg_bytes);
 void prof_set_bytes(int idx, double alg_bytes);
 bool prof_enabled();
+// graph-captured profiling (dt_profile_enable(2)): event-record nodes of one fit graph
+struct GRec {
+  int kind;
+  cudaEvent_t a, b;
+  double bytes;
+};
+bool prof_graph_mode();
+void prof_capture_target(std::vector<GRec>* v);  // prof_begin/end/set_bytes go to v (nullptr: off)
+void prof_collect_graph(const std::vector<GRec>& v);  // after a replay completed
+void prof_destroy_graph_recs(std::vector<GRec>& v);
 void prof_add_launches(long long n);
 
 }  // namespace dtl

@@ -1174,8 +1174,12 @@ struct FitPlan {
   cudaStream_t cap = nullptr;
   int64_t launches = 0;
   uint64_t last_use = 0;
+  bool prof = false;               // captured with profiling event-record nodes
+  std::vector<GRec> grecs;         // their events
+  std::vector<Pending> pending;    // their byte counts (from the level log)
   ~FitPlan() {
     if (exec) cudaGraphExecDestroy(exec);
+    prof_destroy_graph_recs(grecs);
     if (cap) cudaStreamDestroy(cap);
     for (void* p : mem) cudaFree(p);
   }
@@ -1228,13 +1232,14 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     const char* e = getenv("DT_FIT_GRAPH");
     graph_env = (e && e[0] == '0') ? 0 : 1;
   }
-  const bool use_graph = graph_env && !prof_enabled() && max_depth >= 0 && max_depth <= 24;
+  const bool gprof = prof_graph_mode();
+  const bool use_graph = graph_env && (!prof_enabled() || gprof) && max_depth >= 0 && max_depth <= 24;
   if (use_graph) {
     std::lock_guard<std::mutex> lk(g_plan_mu);
     FitPlan* pl = nullptr;
     for (auto& p : g_plans)
       if (p && p->X == X && p->y == y && p->n == n && p->d == d && p->max_depth == max_depth &&
-          p->min_leaf == min_leaf && p->device == dev)
+          p->min_leaf == min_leaf && p->device == dev && p->prof == gprof)
         pl = p.get();
     if (!pl) {
       // victim slot: an empty one, else the least recently used
@@ -1265,6 +1270,7 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
       np->max_depth = max_depth;
       np->min_leaf = min_leaf;
       np->device = dev;
+      np->prof = gprof;
       if (!same_shape) {
         auto get = [&](auto** p, size_t count) -> cudaError_t {
           cudaError_t e = cudaMalloc((void**)p, sizeof(**p) * (count ? count : 1));
@@ -1288,7 +1294,9 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
       }
       const int64_t l0 = dt_launch_count();
       DT_CK(cudaStreamBeginCapture(np->cap, cudaStreamCaptureModeThreadLocal));
-      dt_status st = fit_enqueue(np->b, X, y, n, d, max_depth, min_leaf, np->cap, false, nullptr);
+      if (gprof) prof_capture_target(&np->grecs);
+      dt_status st = fit_enqueue(np->b, X, y, n, d, max_depth, min_leaf, np->cap, false, gprof ? &np->pending : nullptr);
+      prof_capture_target(nullptr);
       cudaGraph_t graph = nullptr;
       cudaError_t ce = cudaStreamEndCapture(np->cap, &graph);
       if (st != DT_OK) {
@@ -1307,7 +1315,13 @@ dt_status fit_impl(const float* X, const double* y, int64_t n, int32_t d, int32_
     pl->last_use = ++g_plan_tick;
     DT_CK(cudaGraphLaunch(pl->exec, s));
     prof_add_launches(pl->launches);
-    return fit_finish(pl->b, d, s, nullptr, out);
+    if (!pl->prof) return fit_finish(pl->b, d, s, nullptr, out);
+    // profiled replay: the byte counts from this replay's level log, then its event times
+    prof_capture_target(&pl->grecs);
+    dt_status fs = fit_finish(pl->b, d, s, &pl->pending, out);
+    prof_capture_target(nullptr);
+    if (fs == DT_OK) prof_collect_graph(pl->grecs);
+    return fs;
   }
   // Direct path: stream-ordered workspace, kernels enqueued one by one.
   Workspace ws;

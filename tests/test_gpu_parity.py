@@ -306,6 +306,27 @@ def test_fit_graph_replay_matches_direct(dt):
     _assert_exact(np.frombuffer(runs[0], dtype=dt.NODE_DTYPE), oracle.fit(X, y, 10, 2))
 
 
+def test_fit_graph_profiled_replay(dt):
+    """dt_profile_enable(graph=True): the fit graph is captured with event-record nodes and
+    replayed; the trees are bytewise those of the plain graph, and every replay reports the
+    fused pass with its algorithmic bytes (32 B per split eval of the children)."""
+    X, y = datagen.cnn_gpu_table(5, 60_000)
+    Xd, yd = _cuda(X), _cuda(y)
+    plain = dt.dt_fit(Xd, yd, 9, 1).nodes.tobytes()
+    dt.dt_profile_reset()
+    dt.dt_profile_enable(True, graph=True)
+    try:
+        runs = [dt.dt_fit(Xd, yd, 9, 1).nodes.tobytes() for _ in range(3)]
+    finally:
+        dt.dt_profile_enable(False)
+    assert all(r == plain for r in runs)
+    prof = dt.dt_profile()
+    assert prof["fused"]["launches"] == 3 * 10  # virtual root + 9 levels, per replay
+    assert prof["fused"]["ms"] > 0 and prof["fused"]["alg_bytes"] > 0
+    assert prof["agg"]["launches"] == 3 * 10
+    dt.dt_profile_reset()
+
+
 # ------------------------------------------------------------------ row-sharded fit ------
 
 def _row_splits(n, world, uneven=False):

@@ -29,7 +29,7 @@ ncu -i /tmp/${TAG}_full.ncu-rep --page details --csv > gpurun_out/${TAG}_full_de
 ls -la /tmp/${TAG}_full.ncu-rep >> gpurun_out/${TAG}_ncu_full.log
 # predict kernels (materialised rows and the factored DSE), one launch each
 timeout 600 ncu --set full --clock-control none --import-source on --kernel-name-base function \
-  -k regex:'^(predict_col_kernel|predict_dse_kernel|forest_predict_kernel)$' --launch-count 3 -o /tmp/${TAG}_pred -f \
+  -k regex:'^(predict_col_kernel|predict_dse_spec_kernel|dse_spec_kernel|forest_predict_kernel)$' --launch-count 4 -o /tmp/${TAG}_pred -f \
   python bench.py --steps 1 --warmup 0 --no-cpu --e2e-steps 0 --dse-log2 24 --c3-rows 0 --grid-rows 0 > gpurun_out/${TAG}_ncu_pred.log 2>&1
 echo "ncu pred exit $?" >> gpurun_out/${TAG}_ncu_pred.log
 ncu -i /tmp/${TAG}_pred.ncu-rep --page raw --csv > gpurun_out/${TAG}_pred_raw.csv 2>/dev/null
