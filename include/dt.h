@@ -279,8 +279,10 @@ dt_status dt_gen_dse(uint64_t seed, int64_t row0, int64_t n, int32_t gpu_bits,
  * impurity (summed in another order; within 1e-12 relative), within the parity contract
  * otherwise.  Sync (one host synchronisation per level).
  *   dt_comm_unique_id: 128-byte NCCL id, created by rank 0 and broadcast by the caller
- *     (e.g. torch.distributed); dt_comm_init: NCCL communicator on the current device
- *     (libnccl.so.2 is loaded at run time; DT_ERR_NCCL if absent); a 1-rank communicator
+ *     (e.g. torch.distributed); dt_comm_init: NCCL communicator of rank `rank` bound to
+ *     CUDA device `device` (made current for the calling thread; INVALID_ARG if out of
+ *     range); the caller's dt_fit_sharded / dt_eval_sharded run on that device.
+ *     libnccl.so.2 is loaded at run time (DT_ERR_NCCL if absent); a 1-rank communicator
  *     runs the real NCCL collectives.
  *   dt_comm_init_local: `world` communicators for host THREADS of one process (device
  *     copies behind a host barrier), e.g. to run the sharded path on a single GPU.
@@ -288,7 +290,7 @@ dt_status dt_gen_dse(uint64_t seed, int64_t row0, int64_t n, int32_t gpu_bits,
 typedef struct dt_comm dt_comm;
 int32_t dt_comm_unique_id_bytes(void);
 dt_status dt_comm_unique_id(void* id_out);
-dt_status dt_comm_init(const void* id, int32_t rank, int32_t world, dt_comm** out);
+dt_status dt_comm_init(const void* id, int32_t rank, int32_t world, int32_t device, dt_comm** out);
 dt_status dt_comm_init_local(int32_t world, dt_comm** comms_out);
 void dt_comm_free(dt_comm* comm);
 int32_t dt_comm_rank(const dt_comm* comm);

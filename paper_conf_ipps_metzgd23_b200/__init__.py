@@ -83,7 +83,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
                             ctypes.POINTER(D), ctypes.POINTER(D)], ctypes.c_int),
         "dt_comm_unique_id_bytes": ([], I32),
         "dt_comm_unique_id": ([P], ctypes.c_int),
-        "dt_comm_init": ([P, I32, I32, ctypes.POINTER(P)], ctypes.c_int),
+        "dt_comm_init": ([P, I32, I32, I32, ctypes.POINTER(P)], ctypes.c_int),
         "dt_comm_init_local": ([I32, P], ctypes.c_int),
         "dt_comm_free": ([P], None),
         "dt_comm_rank": ([P], I32),
@@ -421,9 +421,13 @@ class Comm:
             self._h = None
 
 
-def dt_comm_init_nccl(rank: int, world: int, broadcast) -> Comm:
-    """NCCL communicator; ``broadcast(obj)`` must return rank 0's object on every rank
-    (e.g. a torch.distributed broadcast_object_list wrapper)."""
+def dt_comm_init_nccl(rank: int, world: int, broadcast, device: int = None) -> Comm:
+    """NCCL communicator on CUDA device ``device`` (default: the current one);
+    ``broadcast(obj)`` must return rank 0's object on every rank (e.g. a
+    torch.distributed broadcast_object_list wrapper)."""
+    if device is None:
+        import torch
+        device = torch.cuda.current_device()
     nb = int(_lib.dt_comm_unique_id_bytes())
     uid = (ctypes.c_char * nb)()
     if rank == 0:
@@ -431,7 +435,7 @@ def dt_comm_init_nccl(rank: int, world: int, broadcast) -> Comm:
     raw = broadcast(bytes(uid) if rank == 0 else None)
     uid = (ctypes.c_char * nb).from_buffer_copy(raw)
     h = ctypes.c_void_p()
-    _check(_lib.dt_comm_init(uid, rank, world, ctypes.byref(h)))
+    _check(_lib.dt_comm_init(uid, rank, world, int(device), ctypes.byref(h)))
     return Comm(h)
 
 

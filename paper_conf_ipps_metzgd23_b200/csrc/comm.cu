@@ -120,6 +120,7 @@ __global__ void or_u32_kernel(const uint32_t* const* __restrict__ src, int nsrc,
 struct CommImpl {
   int rank = 0, world = 1;
   int backend = 0;  // 0 = NCCL, 1 = local
+  int device = -1;  // NCCL: the device the communicator is bound to
   ncclComm_t nccl = nullptr;
   std::shared_ptr<LocalGroup> group;
   uint32_t** dev_ptrs = nullptr;  // local backend: device array of peer pointers
@@ -267,15 +268,22 @@ dt_status dt_comm_unique_id(void* id_out) {
 
 int32_t dt_comm_unique_id_bytes(void) { return (int32_t)sizeof(ncclUniqueId); }
 
-dt_status dt_comm_init(const void* id, int32_t rank, int32_t world, dt_comm** out) {
+dt_status dt_comm_init(const void* id, int32_t rank, int32_t world, int32_t device, dt_comm** out) {
   if (!out) return fail(DT_ERR_INVALID_ARG, "dt_comm_init: out is NULL");
   *out = nullptr;
   if (!id || world < 1 || rank < 0 || rank >= world)
     return fail(DT_ERR_INVALID_ARG, "dt_comm_init: need id, 0 <= rank < world");
+  int ndev = 0;
+  DT_CK(cudaGetDeviceCount(&ndev));
+  if (device < 0 || device >= ndev) return fail(DT_ERR_INVALID_ARG, "dt_comm_init: bad device");
+  // the communicator is bound to `device`: made current for this thread (NCCL binds the
+  // communicator to the current device at init)
+  DT_CK(cudaSetDevice(device));
   std::unique_ptr<dt_comm> c(new dt_comm());
   c->impl.rank = rank;
   c->impl.world = world;
   c->impl.backend = 0;
+  c->impl.device = device;
   if (!load_nccl()) return fail(DT_ERR_NCCL, "dt_comm_init: libnccl.so.2 not loadable");
   ncclUniqueId uid;
   memcpy(&uid, id, sizeof(uid));

@@ -565,6 +565,22 @@ def test_nccl_communicator_single_rank(dt):
     assert (m["mape"], m["r2"], m["adj_r2"], m["n"]) == (ref["mape"], ref["r2"], ref["adj_r2"], ref["n"])
 
 
+def test_nccl_communicator_device_argument(dt):
+    """dt_comm_init binds the communicator to an explicit device; a device
+    out of range is INVALID_ARG."""
+    import ctypes
+    nb = int(dt._lib.dt_comm_unique_id_bytes())
+    uid = (ctypes.c_char * nb)()
+    assert dt._lib.dt_comm_unique_id(uid) == 0
+    h = ctypes.c_void_p()
+    assert dt._lib.dt_comm_init(uid, 0, 1, torch.cuda.device_count(), ctypes.byref(h)) == 1  # INVALID_ARG
+    assert dt._lib.dt_comm_init(uid, 0, 1, -1, ctypes.byref(h)) == 1
+    comm = dt.dt_comm_init_nccl(0, 1, lambda obj: obj, device=0)
+    X, y = datagen.cnn_gpu_table(6, 20_000)
+    t = dt.dt_fit_sharded(comm, _cuda(X), _cuda(y), 0, len(y), 8, 1)
+    _same_tree(t.nodes, _fit(dt, X, y, 8, 1).nodes)
+
+
 def test_concurrent_fits_from_threads(dt):
     """Two host threads fitting different tables of the same shape at once (the cached
     graph plan is shared under a lock and re-planned per input): both trees exact."""
