@@ -32,6 +32,10 @@ namespace dtl {
 namespace {
 
 constexpr int kThreads = 256;
+#ifndef DT_FUSED_THREADS
+#define DT_FUSED_THREADS 256  // threads per CTA of the fused pass (per-warp work: no block barriers)
+#endif
+constexpr int kFusedThreads = DT_FUSED_THREADS;
 #ifndef DT_FUSED_STAGES
 #define DT_FUSED_STAGES 2  // bulk-copy stages per warp of the fused pass (3 measured: no faster)
 #endif
@@ -712,11 +716,11 @@ __device__ __forceinline__ uint32_t store_rows(const FusedArgs& a, const PSeg& p
 // stage always has room for f64 entries; int32 lists copy and read half of it.
 // Work: the fast chunks listed by chunk_plan_kernel (whole chunk inside one segment of a
 // split node); a warp per chunk, kStages bulk-copy stages in flight per warp.
-__global__ void __launch_bounds__(kThreads, DT_FUSED_MINB) fused_kernel(FusedArgs a) {
+__global__ void __launch_bounds__(kFusedThreads, DT_FUSED_MINB) fused_kernel(FusedArgs a) {
   extern __shared__ __align__(128) unsigned char fsm[];
   constexpr uint32_t YB = 8u;
   constexpr uint32_t SB = (stage_bytes_for(YB) + 127u) & ~127u;
-  constexpr int kWarps = kThreads / 32;
+  constexpr int kWarps = kFusedThreads / 32;
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   unsigned char* my = fsm + (size_t)wib * kStages * SB;
   uint64_t* bar = reinterpret_cast<uint64_t*>(fsm + (size_t)kWarps * kStages * SB) + wib * kStages;
@@ -1172,7 +1176,7 @@ dt_status level_agg_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t 
 
 size_t fused_smem() {
   const size_t sb = (stage_bytes_for(8u) + 127u) & ~127u;
-  constexpr int kWarps = kThreads / 32;
+  constexpr int kWarps = kFusedThreads / 32;
   return sb * kStages * kWarps + kWarps * kStages * sizeof(uint64_t) + kWarps * sizeof(PSeg);
 }
 
@@ -1208,7 +1212,7 @@ dt_status level_fused_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_
   a.small_list = b.small_list;
   auto k = fused_kernel;
   DT_CK(cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
-  k<<<grid_for((const void*)k, kThreads, sm), kThreads, sm, s>>>(a);
+  k<<<grid_for((const void*)k, kFusedThreads, sm), kFusedThreads, sm, s>>>(a);
   DT_CK(cudaGetLastError());
   fused_small_kernel<<<grid_for((const void*)fused_small_kernel, kThreads, 0), kThreads, 0, s>>>(a);
   DT_CK(cudaGetLastError());

@@ -448,7 +448,6 @@ struct DseMap {
 // its lanes sit on: one shared-memory wavefront per node read, one per CNN rank read (the
 // lanes read one row, pitch kRowPitch words).
 constexpr int kSpecCap = 720;      // slots per T_j: 32 x 720 x (4 + 4) B = 180 KB of shared memory
-constexpr int kSpecStack = 64;
 constexpr int kRankCap = 4095;     // thresholds per CNN column in rank form (12-bit ranks)
 constexpr int kSpecMaxCols = 32;   // CNN columns of the rank form
 constexpr int kRowPitch = 33;      // words per staged CNN rank row (odd: conflict-free)
@@ -468,6 +467,7 @@ __global__ void __launch_bounds__(512) dse_rank_kernel(const uint2* __restrict__
   const uint32_t c = blockIdx.x;
   if (threadIdx.x == 0) s_n = 0u;
   __syncthreads();
+#pragma unroll 4
   for (int k = threadIdx.x; k < count; k += blockDim.x) {
     const uint2 nd = __ldg(gnodes + k);
     if ((nd.y & 0xFFFFFFu) == (uint32_t)k) continue;  // leaf
@@ -515,21 +515,58 @@ __global__ void __launch_bounds__(512) dse_rank_kernel(const uint2* __restrict__
   if (threadIdx.x == 0) rn[c] = n;
 }
 
-// r(x) of every CNN table entry (binary search in T_c).
-__global__ void __launch_bounds__(256) dse_cnn_rank_kernel(const float* __restrict__ cnn, int64_t total, int dc,
-                                                           const float* __restrict__ rt, const uint32_t* __restrict__ rn,
-                                                           uint16_t* __restrict__ crank) {
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
-    const int c = (int)(e % dc);
-    const float x = __ldg(cnn + e);
-    const float* T = rt + (size_t)c * kRankCap;
-    uint32_t lo = 0u, hi = c < kSpecMaxCols ? __ldg(rn + c) : 0u;  // first index with !(T < x)
-    while (lo < hi) {
-      const uint32_t mid = (lo + hi) >> 1;
-      if (__ldg(T + mid) < x) lo = mid + 1u;
-      else hi = mid;
+// r(x) of every CNN table entry (binary search in T_c); the tables are staged in shared
+// memory, packed by column, when they fit (kSmemRanks floats), else searched in place.
+constexpr int kSmemRanks = 12000;
+__global__ void __launch_bounds__(1024) dse_cnn_rank_kernel(const float* __restrict__ cnn, int64_t total, int dc,
+                                                            const float* __restrict__ rt,
+                                                            const uint32_t* __restrict__ rn,
+                                                            uint16_t* __restrict__ crank) {
+  __shared__ float st[kSmemRanks];
+  __shared__ uint32_t s_off[kSpecMaxCols + 1];
+  const int ncols = min(dc, kSpecMaxCols);
+  if (threadIdx.x == 0) {
+    uint32_t o = 0;
+    for (int c = 0; c < ncols; ++c) {
+      s_off[c] = o;
+      o += __ldg(rn + c);
     }
-    crank[e] = (uint16_t)lo;
+    s_off[ncols] = o;
+  }
+  __syncthreads();
+  const bool smem = s_off[ncols] <= (uint32_t)kSmemRanks;
+  if (smem) {
+    for (int c = 0; c < ncols; ++c)
+      for (uint32_t q = threadIdx.x; q < s_off[c + 1] - s_off[c]; q += blockDim.x)
+        st[s_off[c] + q] = __ldg(rt + (size_t)c * kRankCap + q);
+  }
+  __syncthreads();
+  const int64_t nrow = total / dc;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nrow; i += (int64_t)gridDim.x * blockDim.x) {
+    for (int c = 0; c < dc; ++c) {  // a thread per row: no 64-bit division per entry
+      const int64_t e = i * dc + c;
+      const float x = __ldg(cnn + e);
+      uint32_t lo = 0u, hi = 0u;  // first index with !(T < x)
+      if (c < ncols) {
+        hi = s_off[c + 1] - s_off[c];
+        if (smem) {
+          const float* T = st + s_off[c];
+          while (lo < hi) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (T[mid] < x) lo = mid + 1u;
+            else hi = mid;
+          }
+        } else {
+          const float* T = rt + (size_t)c * kRankCap;
+          while (lo < hi) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (__ldg(T + mid) < x) lo = mid + 1u;
+            else hi = mid;
+          }
+        }
+      }
+      crank[e] = (uint16_t)lo;
+    }
   }
 }
 
@@ -557,63 +594,76 @@ __device__ __forceinline__ uint32_t dse_resolve(const SpecTree<kSmem>& tr, const
   }
 }
 
-// Lane j of block g: T_j in one depth-first pass (an internal node gets two consecutive
-// slots for its children), written straight to the group's interleaved slots; a lane
-// whose tree outgrows kSpecCap (or the stack, or the rank form) fails the whole group.
+// Warp w of block g builds T_j (j = 32 g + w) breadth-first: the frontier of a level is
+// the contiguous slot range [lo, hi) whose full-tree nodes sit in the slots' id words;
+// each lane expands one frontier slot per round (an internal node's two children get
+// consecutive slots, placed by a warp prefix sum; each child is resolved through the
+// GPU-feature nodes with row j's features).  Returns the slots used (P), the deepest
+// leaf (D) and whether the tree fits (slots, rank form).
 template <bool kSmem>
 __device__ void dse_spec_build(const SpecTree<kSmem>& tr, const DseMap& map, const float* __restrict__ grow,
-                               bool live, bool ok, uint32_t* __restrict__ spec, SpecMeta* __restrict__ meta) {
+                               bool live, bool ok, uint32_t* __restrict__ out, uint32_t& P, uint32_t& D) {
   const int lane = threadIdx.x & 31;
-  uint32_t* out = spec + (size_t)blockIdx.x * kSpecCap * 64 + lane;  // nodes, then leaf ids
-  uint32_t* lid = out + (size_t)kSpecCap * 32;
-  uint32_t stk[kSpecStack], sslot[kSpecStack];  // pending (node << 8 | depth, slot)
-  int sp = 0;
-  uint32_t nfree = 1, dmax = 0;
-  if (!live) {  // padding lane: one leaf (its outputs are never written)
-    out[0] = 0xFFF00000u;
-    lid[0] = 0u;
-  } else if (ok) {
-    stk[sp] = dse_resolve(tr, map, grow, 0u) << 8;
-    sslot[sp++] = 0u;
-    while (sp > 0) {
-      --sp;
-      const uint32_t k = stk[sp] >> 8, dep = stk[sp] & 0xFFu, slot = sslot[sp];
+  const uint32_t lt = (1u << lane) - 1u;
+  uint32_t* lid = out + (size_t)kSpecCap * 32;  // slot k of this tree: out[32 k], lid[32 k]
+  P = 1u;
+  D = 0u;
+  if (!live || !ok) {  // padding row (its outputs are never written) or no rank form
+    if (lane == 0) {
+      out[0] = 0xFFF00000u;
+      lid[0] = 0u;
+    }
+    return;
+  }
+  if (lane == 0) lid[0] = dse_resolve(tr, map, grow, 0u);
+  __syncwarp();
+  uint32_t lo = 0u, hi = 1u, depth = 0u;
+  while (lo < hi) {
+    uint32_t nfree = hi;  // the next level's slots follow this level's
+    for (uint32_t base = lo; base < hi; base += 32u) {
+      const uint32_t slot = base + (uint32_t)lane;
+      const bool act = slot < hi;
+      const uint32_t k = act ? lid[(size_t)slot * 32] : 0u;
       const uint2 nd = tr.node(k);
       const uint32_t left = nd.y & 0xFFFFFFu;
-      if (left == k) {
-        out[(size_t)slot * 32] = 0xFFF00000u | (slot << 7);  // self-loop, rank never exceeded
-        lid[(size_t)slot * 32] = k;
-        dmax = max(dmax, dep);
-        continue;
-      }
+      const bool internal = act && left != k;
       const uint32_t code = map.code[nd.y >> 24];
-      const uint32_t a = nfree;
-      nfree += 2;
-      if (sp + 2 > kSpecStack || dep + 1 > 255u || nfree > (uint32_t)kSpecCap || code >= (uint32_t)kSpecMaxCols) {
-        ok = false;
-        break;
+      const uint32_t bal = __ballot_sync(0xffffffffu, internal);
+      const bool bad = __any_sync(0xffffffffu, internal && code >= (uint32_t)kSpecMaxCols);
+      if (bad || nfree + 2u * __popc(bal) > (uint32_t)kSpecCap) {
+        P = 0xFFFFFFFFu;  // does not fit
+        return;
       }
-      out[(size_t)slot * 32] = (tr.rk(k) << 20) | (a << 7) | (code << 2);
-      stk[sp] = (dse_resolve(tr, map, grow, left + 1) << 8) | (dep + 1);
-      sslot[sp++] = a + 1;
-      stk[sp] = (dse_resolve(tr, map, grow, left) << 8) | (dep + 1);
-      sslot[sp++] = a;
+      if (internal) {
+        const uint32_t ac = nfree + 2u * __popc(bal & lt);
+        out[(size_t)slot * 32] = (tr.rk(k) << 20) | (ac << 7) | (code << 2);
+        lid[(size_t)ac * 32] = dse_resolve(tr, map, grow, left);
+        lid[(size_t)(ac + 1u) * 32] = dse_resolve(tr, map, grow, left + 1u);
+      } else if (act) {
+        out[(size_t)slot * 32] = 0xFFF00000u | (slot << 7);  // leaf: self-loop, rank never exceeded
+        D = depth;
+      }
+      nfree += 2u * __popc(bal);
     }
+    __syncwarp();  // the next level's id words are visible to the whole warp
+    lo = hi;
+    hi = nfree;
+    ++depth;
   }
-  const uint32_t P = __reduce_max_sync(0xffffffffu, nfree);
-  const uint32_t D = __reduce_max_sync(0xffffffffu, dmax);
-  const bool all_ok = __all_sync(0xffffffffu, ok);
-  if (lane == 0) meta[blockIdx.x] = SpecMeta{all_ok ? (int32_t)P : -1, (int32_t)D};
+  P = hi;
+  D = __reduce_max_sync(0xffffffffu, D);
 }
 
-// Block g (256 threads): the packed tree, the node ranks and the group's GPU rows staged
-// in shared memory (the tree when it fits), then warp 0 builds the group's 32 trees.
-__global__ void __launch_bounds__(256) dse_spec_kernel(const uint2* __restrict__ gnodes, int count, DseMap map,
-                                                       const float* __restrict__ gpu, int64_t n_gpu, int dg,
-                                                       const uint16_t* __restrict__ nrank, const int* __restrict__ bad,
-                                                       bool smem_tree, uint32_t* __restrict__ spec,
-                                                       SpecMeta* __restrict__ meta) {
+// Block g (one warp per GPU row of the group): the packed tree, the node ranks and the
+// group's GPU rows staged in shared memory (the tree when it fits), the 32 trees built,
+// then the group's padded size and depth.
+__global__ void __launch_bounds__(1024) dse_spec_kernel(const uint2* __restrict__ gnodes, int count, DseMap map,
+                                                        const float* __restrict__ gpu, int64_t n_gpu, int dg,
+                                                        const uint16_t* __restrict__ nrank, const int* __restrict__ bad,
+                                                        bool smem_tree, uint32_t* __restrict__ spec,
+                                                        SpecMeta* __restrict__ meta) {
   extern __shared__ __align__(16) unsigned char spec_smem[];
+  __shared__ uint32_t s_p[32], s_d[32];
   const bool ok = *bad == 0;
   float* sg = reinterpret_cast<float*>(spec_smem);  // 32 x dg
   for (int e = threadIdx.x; e < 32 * dg; e += blockDim.x) {
@@ -629,11 +679,22 @@ __global__ void __launch_bounds__(256) dse_spec_kernel(const uint2* __restrict__
     }
   }
   __syncthreads();
-  if (threadIdx.x >= 32) return;
-  const bool live = (int64_t)blockIdx.x * 32 + threadIdx.x < n_gpu;
-  const float* grow = sg + threadIdx.x * dg;
-  if (smem_tree) dse_spec_build(SpecTree<true>{sn, sr}, map, grow, live, ok, spec, meta);
-  else dse_spec_build(SpecTree<false>{gnodes, nrank}, map, grow, live, ok, spec, meta);
+  const int w = threadIdx.x >> 5;
+  const bool live = (int64_t)blockIdx.x * 32 + w < n_gpu;
+  uint32_t* out = spec + (size_t)blockIdx.x * kSpecCap * 64 + w;
+  uint32_t P, D;
+  if (smem_tree) dse_spec_build(SpecTree<true>{sn, sr}, map, sg + w * dg, live, ok, out, P, D);
+  else dse_spec_build(SpecTree<false>{gnodes, nrank}, map, sg + w * dg, live, ok, out, P, D);
+  if ((threadIdx.x & 31) == 0) {
+    s_p[w] = ok ? P : 0xFFFFFFFFu;
+    s_d[w] = D;
+  }
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    const uint32_t p = __reduce_max_sync(0xffffffffu, s_p[threadIdx.x]);
+    const uint32_t dd = __reduce_max_sync(0xffffffffu, s_d[threadIdx.x]);
+    if (threadIdx.x == 0) meta[blockIdx.x] = SpecMeta{p <= (uint32_t)kSpecCap ? (int32_t)p : -1, (int32_t)dd};
+  }
 }
 
 // Candidates (i, j): block = one group of 32 GPU rows (lane = j) x a range of CNN rows;
@@ -772,7 +833,7 @@ dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, in
     dse_rank_kernel<<<(unsigned)ncols, 512, 0, s>>>(t->dev_packed, (int)t->count, map, rt, rn, nrank, bad);
   DT_CK(cudaGetLastError());
   const int64_t total = n_cnn * (int64_t)dc;
-  dse_cnn_rank_kernel<<<(unsigned)std::min<int64_t>((total + 255) / 256, (int64_t)num_sms() * 16), 256, 0, s>>>(
+  dse_cnn_rank_kernel<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((n_cnn + 1023) / 1024, (int64_t)num_sms() * 2)), 1024, 0, s>>>(
       cnn, total, dc, rt, rn, crank);
   DT_CK(cudaGetLastError());
   const size_t g_sm = (sizeof(float) * 32 * (size_t)dg + 15) & ~(size_t)15;
@@ -780,7 +841,7 @@ dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, in
   const bool smem_tree = g_sm + tree_sm <= 200 * 1024;
   const size_t spec_sm = g_sm + (smem_tree ? tree_sm : 0);
   DT_CK(cudaFuncSetAttribute(dse_spec_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)spec_sm));
-  dse_spec_kernel<<<(unsigned)ngroups, 256, spec_sm, s>>>(t->dev_packed, (int)t->count, map, gpu, n_gpu, dg, nrank,
+  dse_spec_kernel<<<(unsigned)ngroups, 1024, spec_sm, s>>>(t->dev_packed, (int)t->count, map, gpu, n_gpu, dg, nrank,
                                                          bad, smem_tree, spec, meta);
   DT_CK(cudaGetLastError());
   // kR CNN rows per warp: independent walks in flight
