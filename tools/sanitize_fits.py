@@ -56,5 +56,13 @@ Xc, yc = datagen.cnn_gpu_table(3, 20000)
 tc = dt.dt_fit(cuda(Xc), cuda(yc), 8, 4)
 cnn, gpu, src = datagen.dse_tables(3, 0, 64, 32)
 dt.dt_predict_dse(tc, cuda(cnn), cuda(gpu), src)
+cnn, gpu, src = datagen.dse_tables(3, 5, 50, 37)  # ragged last GPU group
+dt.dt_predict_dse(tc, cuda(cnn), cuda(gpu), src)
+big = dt.dt_fit(cuda(Xc), cuda(yc), -1, 1)       # large specialised trees: full-tree fallback groups
+dt.dt_predict_dse(big, cuda(cnn), cuda(gpu), src)
+dt.dt_profile_enable(True, graph=True)           # the fit graph with event-record nodes
+for _ in range(2):
+    dt.dt_fit(cuda(Xc), cuda(yc), 6, 2)
+dt.dt_profile_enable(False)
 torch.cuda.synchronize()
 print("SANITIZE_DONE", flush=True)
