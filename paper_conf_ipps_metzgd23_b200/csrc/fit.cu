@@ -994,12 +994,12 @@ dt_status fit_levels(const FitBufs& b, int32_t d, int32_t max_depth, int64_t min
   // the virtual-root pass: the root's candidates and statistics
   {
     LevelArgs la{-1, 0, 0, d, min_leaf, false};
-    int pr = prof_begin(PK_SCAN, s, 2);
+    int pr = prof_begin(PK_SCAN, s, 3);
     st = level_agg_enqueue(b, la, s);
     if (st != DT_OK) return st;
     prof_end(pr, s, 0.0);
     if (pending) pending->push_back({pr, -1, PK_SCAN});
-    pr = prof_begin(PK_PARTITION, s, 1);
+    pr = prof_begin(PK_PARTITION, s, 2);
     st = level_fused_enqueue(b, la, s);
     if (st != DT_OK) return st;
     prof_end(pr, s, 0.0);
@@ -1055,7 +1055,7 @@ dt_status fit_levels(const FitBufs& b, int32_t d, int32_t max_depth, int64_t min
     na.min_leaf = min_leaf;
     na.out = b.dout;
     na.log = b.lvlog;
-    pr = prof_begin(PK_NUMBER, s, 2);
+    pr = prof_begin(PK_NUMBER, s, 3);
     na.wst = b.wst;
     number_kernel<<<1, 1024, 0, s>>>(na);
     children_kernel<<<g_tab, 256, 0, s>>>(na);
@@ -1071,12 +1071,12 @@ dt_status fit_levels(const FitBufs& b, int32_t d, int32_t max_depth, int64_t min
     DT_CK(cudaGetLastError());
     // ---- fused partition + children's split search (a4, a7)
     LevelArgs la{level, cur, par, d, min_leaf, false};
-    pr = prof_begin(PK_SCAN, s, 2);
+    pr = prof_begin(PK_SCAN, s, 3);
     st = level_agg_enqueue(b, la, s);
     if (st != DT_OK) return st;
     prof_end(pr, s, 0.0);
     if (pending) pending->push_back({pr, level, PK_SCAN});
-    pr = prof_begin(PK_PARTITION, s, 1);
+    pr = prof_begin(PK_PARTITION, s, 2);
     st = level_fused_enqueue(b, la, s);
     if (st != DT_OK) return st;
     prof_end(pr, s, 0.0);
@@ -1521,12 +1521,12 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
   Ctl* ctl = b.ctl;
   {  // the virtual-root pass (the root's rank carries come from the presort)
     LevelArgs la{-1, 0, 0, d, min_leaf, false};
-    int pr = prof_begin(PK_SCAN, s, 2);
+    int pr = prof_begin(PK_SCAN, s, 3);
     pending.push_back({pr, -1, PK_SCAN});
     st = level_agg_enqueue(b, la, s);
     if (st != DT_OK) return st;
     prof_end(pr, s, 0.0);
-    pr = prof_begin(PK_PARTITION, s, 1);
+    pr = prof_begin(PK_PARTITION, s, 2);
     pending.push_back({pr, -1, PK_PARTITION});
     st = level_fused_enqueue(b, la, s);
     if (st != DT_OK) return st;
@@ -1585,7 +1585,7 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
     na.min_leaf = min_leaf;
     na.out = b.dout;
     na.log = b.lvlog;
-    pr = prof_begin(PK_NUMBER, s, 1);
+    pr = prof_begin(PK_NUMBER, s, 2);
     na.wst = b.wst;
     number_kernel<<<1, 1024, 0, s>>>(na);
     children_kernel<<<g_tab, 256, 0, s>>>(na);
@@ -1636,7 +1636,7 @@ dt_status fit_sharded_impl(dt_comm* comm, const float* X, const double* y, int64
       DT_CK(cudaMemsetAsync(&ctl->T[par ^ 1], 0, sizeof(unsigned long long), s));
       DT_CK(cudaMemsetAsync(&ctl->T0[par ^ 1], 0, sizeof(unsigned long long), s));
     }
-    pr = prof_begin(PK_PARTITION, s, 1);
+    pr = prof_begin(PK_PARTITION, s, 2);
     pending.push_back({pr, level, PK_PARTITION});
     st = level_fused_enqueue(b, la, s);
     if (st != DT_OK) return st;
