@@ -44,6 +44,9 @@ constexpr int kStages = DT_FUSED_STAGES;
 #define DT_FUSED_MINB 2  // CTAs per SM of the fused pass (register budget; 3 spills: slower)
 #endif
 constexpr float kNaN = __builtin_nanf("");
+// chunk aggregate x fields: a NaN with this payload | item index = "x of entry index of
+// this chunk" (resolved by agg_scan_kernel); the plain NaN means "none" (x is finite)
+constexpr uint32_t kXMark = 0x7FE00000u;
 
 __device__ __forceinline__ double y_at(const double* __restrict__ ly, int64_t p, bool y32) {
   return y32 ? (double)reinterpret_cast<const int32_t*>(ly)[p] : ly[p];
@@ -301,17 +304,32 @@ __device__ __forceinline__ void agg_fast_chunk(const AggArgs& a, const uint32_t*
   out.sr = __shfl_sync(0xffffffffu, sr, 31);
   out.xl = kNaN;
   out.xr = kNaN;
-  if (Lm) {
-    const int h = 31 - __clz(Lm);
-    float v = 0.f;
-    if (lane == h) v = a.lx[p0 + 31 - __clz(gbyte)];
-    out.xl = __shfl_sync(0xffffffffu, v, h);
-  }
-  if (Rm) {
-    const int h = 31 - __clz(Rm);
-    float v = 0.f;
-    if (lane == h) v = a.lx[p0 + 31 - __clz(~gbyte & 0xffu)];
-    out.xr = __shfl_sync(0xffffffffu, v, h);
+  if (kTails) {  // sharded: the tails need the x values here
+    if (Lm) {
+      const int h = 31 - __clz(Lm);
+      float v = 0.f;
+      if (lane == h) v = a.lx[p0 + 31 - __clz(gbyte)];
+      out.xl = __shfl_sync(0xffffffffu, v, h);
+    }
+    if (Rm) {
+      const int h = 31 - __clz(Rm);
+      float v = 0.f;
+      if (lane == h) v = a.lx[p0 + 31 - __clz(~gbyte & 0xffu)];
+      out.xr = __shfl_sync(0xffffffffu, v, h);
+    }
+  } else {
+    // the last left / right entry's index in the chunk, as a marker NaN that agg_scan
+    // resolves to its x when it loads the aggregate (no dependent x load here)
+    if (Lm) {
+      const int h = 31 - __clz(Lm);
+      const uint32_t gh = __shfl_sync(0xffffffffu, gbyte, h);
+      out.xl = __uint_as_float(kXMark | (uint32_t)(8 * h + 31 - __clz(gh)));
+    }
+    if (Rm) {
+      const int h = 31 - __clz(Rm);
+      const uint32_t gh = __shfl_sync(0xffffffffu, gbyte, h);
+      out.xr = __uint_as_float(kXMark | (uint32_t)(8 * h + 31 - __clz(~gh & 0xffu)));
+    }
   }
   a.gm[cbase / 8 + lane] = (uint8_t)gbyte;
   if (lane == 0) {
@@ -512,8 +530,14 @@ __device__ __forceinline__ AggP ld_cg_agg(const AggP* p) {
   return r;
 }
 
+__device__ __forceinline__ float resolve_x(float v, const float* __restrict__ lx, int64_t c) {
+  const uint32_t u = __float_as_uint(v);
+  return (u & 0xFFFFFF00u) == kXMark ? __ldg(lx + c * kChunkW + (u & 0xFFu)) : v;
+}
+
 __global__ void __launch_bounds__(1024) agg_scan_kernel(Ctl* ctl, int par, const AggP* __restrict__ agg,
-                                                       AggP* __restrict__ cexcl, AggP* bagg, AggP* __restrict__ bcarry) {
+                                                       AggP* __restrict__ cexcl, AggP* bagg, AggP* __restrict__ bcarry,
+                                                       const float* __restrict__ lx) {
   __shared__ AggP sh[33];
   __shared__ AggP sh_run;
   __shared__ bool s_last;
@@ -523,7 +547,11 @@ __global__ void __launch_bounds__(1024) agg_scan_kernel(Ctl* ctl, int par, const
   const int64_t b0 = (int64_t)blockIdx.x * kBlockChunks;
   if (b0 < nch) {  // block-uniform
     const int64_t c = b0 + threadIdx.x;
-    const AggP v = (c < nch) ? agg[c] : agg_ident();
+    AggP v = (c < nch) ? agg[c] : agg_ident();
+    if (c < nch) {
+      v.xl = resolve_x(v.xl, lx, c);
+      v.xr = resolve_x(v.xr, lx, c);
+    }
     AggP ba;
     const AggP ex = block_excl_agg(v, ba, sh);
     if (c < nch) cexcl[c] = ex;
@@ -1169,7 +1197,8 @@ dt_status level_agg_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t 
     k<<<grid_for((const void*)k, kThreads, 0), kThreads, 0, s>>>(a);
   }
   DT_CK(cudaGetLastError());
-  agg_scan_kernel<<<(unsigned)b.max_cblocks, 1024, 0, s>>>(b.ctl, la.par, b.agg, b.cexcl, b.bagg, b.bcarry);
+  agg_scan_kernel<<<(unsigned)b.max_cblocks, 1024, 0, s>>>(b.ctl, la.par, b.agg, b.cexcl, b.bagg, b.bcarry,
+                                                          b.lx[la.cur]);
   DT_CK(cudaGetLastError());
   return DT_OK;
 }
