@@ -345,11 +345,21 @@ __global__ void __launch_bounds__(kSmemBits ? 1024 : kThreads) level_agg_kernel(
   const uint64_t T = a.ctl->T[a.par];
   const bool y32 = a.ctl->y32 != 0;
   const int64_t nfast = a.ctl->nfast, ngen = a.ctl->ngen;
+  // the go-left bitmap into shared memory by bulk copies (TMA), completed on an mbarrier:
+  // the first chunk's rows and y are fetched while it lands
+  __shared__ uint64_t sbar;
   if (kSmemBits) {
-    const int64_t n4 = a.nwords / 4;
-    const uint4* g4 = reinterpret_cast<const uint4*>(a.gbits);
-    for (int64_t i = threadIdx.x; i < n4; i += blockDim.x) smem_bits4[i] = __ldg(g4 + i);
-    __syncthreads();
+    if (threadIdx.x == 0) {
+      mbar_init(&sbar, 1);
+      mbar_init_fence();
+      const uint32_t bytes = (uint32_t)(a.nwords * 4);
+      mbar_arrive_expect_tx(&sbar, bytes);
+      constexpr uint32_t kPiece = 32768u;
+      for (uint32_t o = 0; o < bytes; o += kPiece)
+        bulk_g2s(reinterpret_cast<unsigned char*>(smem_bits4) + o, reinterpret_cast<const unsigned char*>(a.gbits) + o,
+                 min(kPiece, bytes - o), &sbar);
+    }
+    __syncthreads();  // the barrier is initialised before anyone waits on it
   }
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -367,6 +377,7 @@ __global__ void __launch_bounds__(kSmemBits ? 1024 : kThreads) level_agg_kernel(
       q0 = __ldcs(y4); q1 = __ldcs(y4 + 1);
     };
     if (gw < nfast) fetch(e);
+    if (kSmemBits) mbar_wait(&sbar, 0);
     for (int64_t i = gw; i < nfast; i += nw) {
       const uint2 cur = e;
       const uint32_t rv[kItems] = {r0.x, r0.y, r0.z, r0.w, r1.x, r1.y, r1.z, r1.w};
@@ -379,6 +390,7 @@ __global__ void __launch_bounds__(kSmemBits ? 1024 : kThreads) level_agg_kernel(
       agg_fast_chunk<kSmemBits, kTails>(a, bits, (int64_t)cur.x, cur.y, rv, yv);
     }
   } else {
+    if (kSmemBits) mbar_wait(&sbar, 0);
     for (int64_t i = gw; i < nfast; i += nw) {
       const uint2 cur = a.fast_list[i];
       uint32_t rv[kItems];
@@ -388,6 +400,7 @@ __global__ void __launch_bounds__(kSmemBits ? 1024 : kThreads) level_agg_kernel(
     }
   }
   // ---- general chunks: segment heads inside; per item walk
+  if (kSmemBits) mbar_wait(&sbar, 0);
   const uint32_t nseg = a.ctl->K[a.par] * a.d;
   for (int64_t gi = gw; gi < ngen; gi += nw) {
     const int64_t ch = (int64_t)a.gen_list[gi];
