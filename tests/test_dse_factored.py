@@ -148,3 +148,42 @@ def test_predict_dse_deep_chain(dt, depth):
     gpu = rng.integers(0, 64, size=(70, 3)).astype(np.float32)
     out = dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), torch.from_numpy(gpu).cuda(), src)
     assert np.array_equal(out.cpu().numpy(), oracle.predict(nodes, _compose(cnn, gpu, src)))
+
+
+@pytest.mark.gpu
+def test_predict_dse_edge_cases(dt):
+    """A single-leaf tree; NaN / inf CNN and GPU features (x > t is false: left, as in
+    dt_predict); more than 32 CNN columns (the rank form's limit: full-tree walks); one
+    GPU row; every case against dt_predict on the composed rows and the oracle."""
+    rng = np.random.default_rng(11)
+    # single leaf
+    X, y = datagen.cnn_gpu_table(1, 1000)
+    nodes = oracle.fit(X, y, 0, 1)
+    tree = dt.dt_tree_from_nodes(nodes, 16)
+    cnn, gpu, src = datagen.dse_tables(3, 0, 5, 7)
+    out = dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), torch.from_numpy(gpu).cuda(), src)
+    assert np.array_equal(out.cpu().numpy(), np.full(35, nodes["value"][0]))
+    # non-finite features
+    X, y = datagen.cnn_gpu_table(1, 20_000)
+    nodes = oracle.fit(X, y, 10, 4)
+    tree = dt.dt_tree_from_nodes(nodes, 16)
+    cnn, gpu, src = datagen.dse_tables(3, 0, 40, 33)
+    cnn[::3, 0] = np.nan
+    cnn[1::5, 4] = np.inf
+    gpu[::4, 1] = -np.inf
+    gpu[2::7, 0] = np.nan
+    out = dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), torch.from_numpy(gpu).cuda(), src)
+    Xc = _compose(cnn, gpu, src)
+    ref = dt.dt_predict(tree, torch.from_numpy(Xc).cuda())
+    assert torch.equal(out, ref)
+    # > 32 CNN columns (tree features reach column 40), one GPU row
+    n = 30_000
+    Xw = rng.integers(0, 50, size=(n, 42)).astype(np.float32)
+    yw = np.floor(rng.random(n) * 1e4)
+    nodes = oracle.fit(Xw, yw, 8, 2)
+    tree = dt.dt_tree_from_nodes(nodes, 42)
+    src = list(range(41)) + [-1]
+    cnn = rng.integers(0, 50, size=(64, 41)).astype(np.float32)
+    gpu = rng.integers(0, 50, size=(1, 1)).astype(np.float32)
+    out = dt.dt_predict_dse(tree, torch.from_numpy(cnn).cuda(), torch.from_numpy(gpu).cuda(), src)
+    assert np.array_equal(out.cpu().numpy(), oracle.predict(nodes, _compose(cnn, gpu, src)))
