@@ -1,4 +1,4 @@
-// Communicators for the feature-sharded fit (dt_fit_sharded).
+// Communicators for the value-range row-sharded fit (dt_fit_sharded).
 //
 // Two backends behind one interface, both stream-ordered from the caller's view:
 //   * NCCL (one process per GPU; NVLink / NVSwitch): ncclAllGather / ncclAllReduce on the
