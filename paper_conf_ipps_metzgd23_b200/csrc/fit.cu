@@ -527,18 +527,23 @@ __global__ void __launch_bounds__(256) goleft_kernel(const Ctl* __restrict__ ctl
       uint64_t lim = st + __ldg(&pseg[s].glim);  // the segment's left entries: [st, lim)
       if (st <= cbase && en >= cbase + kChunkW) {
         // one segment (rows read coalesced)
+        // every row id in flight first, then the bit updates (no load -> atomic chain)
+        uint32_t rr[kItems];
 #pragma unroll
         for (int j = 0; j < kItems; ++j) {
           const uint64_t p = cbase + (uint64_t)(j * 32 + lane);
-          if (p < lim) {
-            const uint32_t r = __ldg(lr + p);
-            atomicOr(gbits + (r >> 5), 1u << (r & 31));
-          }
+          rr[j] = p < lim ? __ldg(lr + p) : 0xffffffffu;
         }
+#pragma unroll
+        for (int j = 0; j < kItems; ++j)
+          if (rr[j] != 0xffffffffu) atomicOr(gbits + (rr[j] >> 5), 1u << (rr[j] & 31));
         continue;
       }
       // segment heads inside: lane owns entries 8 lane .. 8 lane + 7, finds their segments
       const uint64_t p0 = cbase + (uint64_t)(lane * kItems);
+      uint32_t rr[kItems];
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) rr[j] = 0xffffffffu;
 #pragma unroll
       for (int j = 0; j < kItems; ++j) {
         const uint64_t p = p0 + j;
@@ -549,11 +554,11 @@ __global__ void __launch_bounds__(256) goleft_kernel(const Ctl* __restrict__ ctl
           en = st + __ldg(&pseg[s].cnt);
           lim = st + __ldg(&pseg[s].glim);
         }
-        if (p < lim) {
-          const uint32_t r = __ldg(lr + p);
-          atomicOr(gbits + (r >> 5), 1u << (r & 31));
-        }
+        if (p < lim) rr[j] = __ldg(lr + p);
       }
+#pragma unroll
+      for (int j = 0; j < kItems; ++j)
+        if (rr[j] != 0xffffffffu) atomicOr(gbits + (rr[j] >> 5), 1u << (rr[j] & 31));
     }
   }
 }
