@@ -735,6 +735,13 @@ def run_ours(args, world, rank, local):
                "pinned": "one core (sched_setaffinity)", "sklearn": sk}
 
     if rank == 0:
+        if dse is not None:  # the prediction kernels' rooflines beside the fit's (north star:
+            # split search AND prediction against HBM)
+            roofline["predict"] = dict(dse["roofline"], workload="2^%d materialised DSE candidates" % args.dse_log2,
+                                       predictions_per_s=dse["predictions_per_s"])
+            if "factored" in dse:
+                roofline["predict_dse_factored"] = dict(dse["factored"]["roofline"],
+                                                        predictions_per_s=dse["factored"]["predictions_per_s"])
         line = {"metric": METRIC, "value": value, "unit": "split evals/s", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": step_ms,
                 "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
