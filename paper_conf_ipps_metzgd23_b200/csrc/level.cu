@@ -1210,7 +1210,7 @@ dt_status level_agg_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t 
     k<<<grid_for((const void*)k, kThreads, 0), kThreads, 0, s>>>(a);
   }
   DT_CK(cudaGetLastError());
-  agg_scan_kernel<<<(unsigned)b.max_cblocks, 1024, 0, s>>>(b.ctl, la.par, b.agg, b.cexcl, b.bagg, b.bcarry,
+  agg_scan_kernel<<<(unsigned)b.max_cblocks, kBlockChunks, 0, s>>>(b.ctl, la.par, b.agg, b.cexcl, b.bagg, b.bcarry,
                                                           b.lx[la.cur]);
   DT_CK(cudaGetLastError());
   return DT_OK;
