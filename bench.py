@@ -62,7 +62,8 @@ def parse():
     p.add_argument("--dse-log2", type=int, default=28, help="log2 of DSE candidates (30 = full C4)")
     p.add_argument("--no-dse", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
-    p.add_argument("--e2e-steps", type=int, default=10)
+    p.add_argument("--e2e-steps", type=int, default=30,
+                   help="e2e steps (double-buffered: the first upload is a pipeline fill inside the region)")
     p.add_argument("--no-extra", action="store_true", help="skip configs[0] LOO and configs[4] grid")
     p.add_argument("--grid-rows", type=int, default=10_000_000, help="configs[4] rows (0 = skip)")
     p.add_argument("--c3-rows", type=int, default=100_000_000,
