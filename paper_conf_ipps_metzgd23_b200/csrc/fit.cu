@@ -833,6 +833,8 @@ __global__ void __launch_bounds__(256) pack_tree_kernel(const dt_node* __restric
   }
 }
 
+__global__ void set_u32_kernel(uint32_t* p, uint32_t v) { *p = v; }
+
 // ----------------------------------------------------------------------------- buffers --
 
 struct Workspace {
@@ -1482,13 +1484,61 @@ dt_status forest_trees_impl(const float* X, const double* y, int64_t n, int32_t 
   DT_CK(cudaMemcpyAsync(sy, b.ly[0], sizeof(double) * tot, cudaMemcpyDeviceToDevice, s));
   DT_CK(cudaStreamSynchronize(s));
   if (hc.nonfinite) return fail(DT_ERR_NONFINITE, "dt_forest_fit: non-finite value in X or y");
-  for (int32_t t = 0; t < n_trees; ++t) {
-    st = clear_pieces(b, s);
+  uint32_t* tdev = nullptr;
+  st = alloc_status(ws.get(&tdev, 1));
+  if (st != DT_OK) return st;
+  // Bounded depth: one tree's sequence (pieces cleared, bootstrap expansion, level loop) is
+  // captured once as a CUDA graph and replayed per tree with the tree index set on the device.
+  const bool use_graph = !prof_enabled() && max_depth >= 0 && max_depth <= 24;
+  cudaGraphExec_t exec = nullptr;
+  cudaStream_t cap = nullptr;
+  struct Drop {
+    cudaGraphExec_t& e;
+    cudaStream_t& c;
+    ~Drop() {
+      if (e) cudaGraphExecDestroy(e);
+      if (c) cudaStreamDestroy(c);
+    }
+  } drop{exec, cap};
+  int64_t per_tree_launches = 0;
+  if (use_graph) {
+    DT_CK(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
+    DT_CK(cudaStreamSynchronize(s));  // the workspace and copies above are complete
+    const int64_t l0 = dt_launch_count();
+    DT_CK(cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal));
+    st = clear_pieces(b, cap);
     if (st == DT_OK)
-      st = forest_tree_enqueue(b, sx, sr, sy, y, n, d, max_depth, min_leaf, seed, (uint32_t)t, hc.y32, w, ys, tsum, s);
-    if (st == DT_OK) st = fit_levels(b, d, max_depth, min_leaf, s, true, nullptr);
+      st = forest_tree_enqueue(b, sx, sr, sy, y, n, d, max_depth, min_leaf, seed, tdev, hc.y32, w, ys, tsum, cap);
+    if (st == DT_OK) st = fit_levels(b, d, max_depth, min_leaf, cap, false, nullptr);
+    cudaGraph_t graph = nullptr;
+    const cudaError_t ce = cudaStreamEndCapture(cap, &graph);
+    if (st != DT_OK) {
+      if (graph) cudaGraphDestroy(graph);
+      return st;
+    }
+    if (ce != cudaSuccess) return cuda_fail(ce, "cudaStreamEndCapture", __FILE__, __LINE__);
+    per_tree_launches = dt_launch_count() - l0;
+    prof_add_launches(-per_tree_launches);  // counted per replay
+    const cudaError_t ie = cudaGraphInstantiate(&exec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (ie != cudaSuccess) return cuda_fail(ie, "cudaGraphInstantiate", __FILE__, __LINE__);
+  }
+  for (int32_t t = 0; t < n_trees; ++t) {
+    set_u32_kernel<<<1, 1, 0, s>>>(tdev, (uint32_t)t);
+    prof_add_launches(1);
+    DT_CK(cudaGetLastError());
+    if (use_graph) {
+      DT_CK(cudaGraphLaunch(exec, s));
+      prof_add_launches(per_tree_launches);
+    } else {
+      st = clear_pieces(b, s);
+      if (st == DT_OK)
+        st = forest_tree_enqueue(b, sx, sr, sy, y, n, d, max_depth, min_leaf, seed, tdev, hc.y32, w, ys, tsum, s);
+      if (st == DT_OK) st = fit_levels(b, d, max_depth, min_leaf, s, true, nullptr);
+      if (st != DT_OK) return st;
+    }
     dt_tree* tr = nullptr;
-    if (st == DT_OK) st = fit_finish(b, d, s, nullptr, &tr);
+    st = fit_finish(b, d, s, nullptr, &tr);
     if (st != DT_OK) return st;
     trees.push_back(tr);
   }

@@ -322,7 +322,7 @@ dt_status presort_sharded_enqueue(const FitBufs& b, dt_comm* comm, const float* 
                                   cudaStream_t s);
 dt_status forest_tree_enqueue(const FitBufs& b, const float* sx, const uint32_t* sr, const double* sy,
                               const double* y, int64_t n, int d, int32_t max_depth, int64_t min_leaf, uint64_t seed,
-                              uint32_t t, int y32, uint32_t* w, double* ys, unsigned long long* tsum,
+                              const uint32_t* tdev, int y32, uint32_t* w, double* ys, unsigned long long* tsum,
                               cudaStream_t s);
 dt_status level_agg_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t s);
 dt_status level_fused_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t s);

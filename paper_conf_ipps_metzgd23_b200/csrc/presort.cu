@@ -865,8 +865,10 @@ namespace {
 // any order -- no split falls between equal x -- so integer-mode trees equal the exact
 // CART of the sample in draw order (Reading R20); the copies keep row id r (they always go
 // the same way).
-__global__ void __launch_bounds__(256) boot_count_kernel(uint64_t seed, uint32_t t, int64_t n, uint32_t* __restrict__ w,
-                                                         const double* __restrict__ y, double* __restrict__ ys) {
+__global__ void __launch_bounds__(256) boot_count_kernel(uint64_t seed, const uint32_t* __restrict__ tdev, int64_t n,
+                                                         uint32_t* __restrict__ w, const double* __restrict__ y,
+                                                         double* __restrict__ ys) {
+  const uint32_t t = *tdev;  // the tree index lives on the device: one captured graph serves every tree
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     uint64_t z = seed + 0x9E3779B97F4A7C15ull * ((((uint64_t)t) << 32) + (uint64_t)i + 1ull);  // Reading R21
     z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
@@ -987,7 +989,7 @@ __global__ void set_storage_kernel(Ctl* ctl, int y32) { ctl->y32 = y32; }
 // tsum (n d / kXT + 1 u64).  y32: the lists' y storage (the table's, Reading R24).
 dt_status forest_tree_enqueue(const FitBufs& b, const float* sx, const uint32_t* sr, const double* sy,
                               const double* y, int64_t n, int d, int32_t max_depth, int64_t min_leaf, uint64_t seed,
-                              uint32_t t, int y32, uint32_t* w, double* ys, unsigned long long* tsum,
+                              const uint32_t* tdev, int y32, uint32_t* w, double* ys, unsigned long long* tsum,
                               cudaStream_t s) {
   const int64_t total = n * (int64_t)d;
   const int64_t ntiles = (total + kXT - 1) / kXT;
@@ -995,7 +997,7 @@ dt_status forest_tree_enqueue(const FitBufs& b, const float* sx, const uint32_t*
   DT_CK(cudaMemsetAsync(b.ctl, 0, sizeof(Ctl), s));
   const int gb = std::max(1, std::min<int>((int)((n + 255) / 256), num_sms() * 8));
   int pr = prof_begin(PK_PRESORT_BUILD, s, 4);
-  boot_count_kernel<<<gb, 256, 0, s>>>(seed, t, n, w, y, ys);
+  boot_count_kernel<<<gb, 256, 0, s>>>(seed, tdev, n, w, y, ys);
   expand_sum_kernel<<<(unsigned)ntiles, 256, 0, s>>>(sr, w, total, tsum);
   expand_scan_kernel<<<1, 1024, 0, s>>>(tsum, ntiles);
   if (y32) expand_write_kernel<true><<<(unsigned)ntiles, 256, 0, s>>>(sx, sr, sy, w, total, tsum, b.lx[0], b.lr[0], b.ly[0]);
