@@ -71,7 +71,7 @@ def parse():
     p.add_argument("--force-sharded", action="store_true",
                    help="run the N>1 headline (row-sharded configs[2] over NCCL) even with one rank")
     p.add_argument("--sharded-local", type=int, default=0,
-                   help="N=1 only: also time a feature-sharded fit with this many thread ranks on the GPU")
+                   help="N=1 only: also time a row-sharded fit with this many thread ranks on the GPU")
     return p.parse_args()
 
 

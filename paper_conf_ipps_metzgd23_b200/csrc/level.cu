@@ -8,7 +8,7 @@
 //                           (left count, child-centred sums of both sides, last x of
 //                           both sides) since the chunk's last segment head;
 //   F_B  agg_scan_kernel    fixed-shape exclusive scan of the chunk aggregates -> the
-//                           carry of every chunk (blocks of 1024 chunks + block carries);
+//                           carry of every chunk (blocks of kBlockChunks chunks + block carries);
 //   F_C  fused_kernel       per warp chunk, a TMA bulk-copy pipeline (x, row, y, bits,
 //                           segment plan, carries): the chunk's entries are written to
 //                           their child lists (stable: left entries in order, then right
