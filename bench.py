@@ -18,7 +18,7 @@ timed region), DSE predictions/s (BASELINE configs[3] shape on one GPU: 2^28 mat
 candidates by default, depth-20 / min_samples_leaf-128 tree; and the full 2^30 cross
 product through the factored predictor), the dominant kernel's roofline, the oracle timed
 on the host as cpu_baseline, configs[0] LOO, configs[4] grid, configs[2] (100M x 32,
-depth 16) on one GPU (feature-sharded over NCCL at N>1), a 16-tree Random Forest and
+depth 16) on one GPU (row-sharded over NCCL at N>1: the N>1 headline), a 16-tree Random Forest and
 KNN regression.
 
 --impl reference: the oracle (the slow CPU reference of this tier) timed on the host.
@@ -631,7 +631,7 @@ def run_ours(args, world, rank, local):
                          "note": "8 B yhat write per prediction; the traversal is issue-bound"}}
         del out, cnn_d, gpu_d
 
-    # ---- feature-sharded fit across the N ranks (NCCL): one C2 fit split by features
+    # ---- optional (--sharded-local P): the C2 table row-sharded over P host-thread ranks on this GPU
     sharded = None
     if world == 1 and args.sharded_local > 1:
         try:
