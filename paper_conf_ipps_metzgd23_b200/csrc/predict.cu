@@ -819,6 +819,11 @@ dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, in
   const size_t b_nr = ((sizeof(uint16_t) * (size_t)t->count) + 15) & ~(size_t)15;
   const size_t b_cr = sizeof(uint16_t) * (size_t)n_cnn * (size_t)dc;
   DT_CK(cudaMallocAsync((void**)&scratch, b_spec + b_meta + b_rt + b_rn + b_nr + b_cr, s));
+  struct FreeScratch {  // stream-ordered release on every return path
+    unsigned char* p;
+    cudaStream_t s;
+    ~FreeScratch() { cudaFreeAsync(p, s); }
+  } free_scratch{scratch, s};
   uint32_t* spec = reinterpret_cast<uint32_t*>(scratch);
   SpecMeta* meta = reinterpret_cast<SpecMeta*>(scratch + b_spec);
   float* rt = reinterpret_cast<float*>(scratch + b_spec + b_meta);
@@ -857,7 +862,6 @@ dt_status predict_dse_impl(const dt_tree* t, const float* cnn, int64_t n_cnn, in
                                                      (int)ngroups, cnn, crank, n_cnn, dc, gpu, n_gpu, dg, yhat);
   prof_end(pr, s, 8.0 * (double)n_cnn * (double)n_gpu);  // the yhat write (inputs are O(n_cnn + n_gpu))
   DT_CK(cudaGetLastError());
-  DT_CK(cudaFreeAsync(scratch, s));
   return DT_OK;
 }
 
