@@ -55,6 +55,7 @@ __device__ __forceinline__ double y_at(const double* __restrict__ ly, int64_t p,
 // ----------------------------------------------------------------------------- F_A --
 
 struct AggArgs {
+  bool walk_gen;  // general chunks by the per-item segment walk (virtual root, sharded tails)
   const uint32_t* lr;
   const double* ly;
   const float* lx;
@@ -402,6 +403,68 @@ __global__ void __launch_bounds__(kSmemBits ? 1024 : kThreads) level_agg_kernel(
   // ---- general chunks: segment heads inside; per item walk
   if (kSmemBits) mbar_wait(&sbar, 0);
   const uint32_t nseg = a.ctl->K[a.par] * a.d;
+  if (!kTails && !a.walk_gen) {
+    // The chunk's aggregate only needs its LAST segment's entries (the scan restarts at
+    // that segment's head): one segment lookup per chunk, no per-item walk.  The go-left
+    // bits of every entry (F_C's pieces of the other segments read them) are looked up
+    // regardless of the segment (levels >= 0 have no all-left segments).
+    for (int64_t gi = gw; gi < ngen; gi += nw) {
+      const int64_t ch = (int64_t)a.gen_list[gi];
+      const uint64_t cbase = (uint64_t)ch * kChunkW;
+      const int64_t p0 = (int64_t)cbase + lane * kItems;
+      const uint64_t plast = min(cbase + (uint64_t)kChunkW, T) - 1u;
+      uint32_t sidx = __ldg(a.desc + ch);
+      SegLite g = seg_lite(a.pseg, sidx);
+      if (plast >= g.end) {
+        sidx = seg_gallop(a.pseg, sidx + 1u, nseg - 1u, plast);
+        g = seg_lite(a.pseg, sidx);
+      }
+      uint32_t rv[kItems];
+      double yv[kItems];
+      load_rows_y(a, p0, (int64_t)T, y32, true, rv, yv);
+      uint32_t gbyte = 0u, inl = 0u;  // go-left bits; my items in the last segment (and split)
+      const bool split = (g.flags & PS_SPLIT) != 0;
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        const uint64_t p = (uint64_t)p0 + j;
+        if (p < T) {
+          gbyte |= ((bits[rv[j] >> 5] >> (rv[j] & 31)) & 1u) << j;
+          if (split && p >= g.start) inl |= 1u << j;
+        }
+      }
+      double sl = 0.0, sr = 0.0;
+#pragma unroll
+      for (int j = 0; j < kItems; ++j) {
+        const bool in = (inl >> j) & 1u, gl = (gbyte >> j) & 1u;
+        const double dd = __dsub_rn(yv[j], gl ? g.c0 : g.c1);
+        // adding +0.0 is exact: a sum of (y - c) terms is never -0.0
+        sl = __dadd_rn(sl, in && gl ? dd : 0.0);
+        sr = __dadd_rn(sr, in && !gl ? dd : 0.0);
+      }
+      warp_incl2(sl, sr);
+      const uint32_t lb = gbyte & inl, rb = ~gbyte & inl;
+      const uint32_t Lm = __ballot_sync(0xffffffffu, lb != 0u);
+      const uint32_t Rm = __ballot_sync(0xffffffffu, rb != 0u);
+      AggP out = agg_ident();
+      out.flag = g.start >= cbase ? 1u : 0u;
+      out.nl = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(lb));
+      out.sl = __shfl_sync(0xffffffffu, sl, 31);
+      out.sr = __shfl_sync(0xffffffffu, sr, 31);
+      if (Lm) {
+        const int h = 31 - __clz(Lm);
+        const uint32_t gh = __shfl_sync(0xffffffffu, lb, h);
+        out.xl = __uint_as_float(kXMark | (uint32_t)(8 * h + 31 - __clz(gh)));
+      }
+      if (Rm) {
+        const int h = 31 - __clz(Rm);
+        const uint32_t gh = __shfl_sync(0xffffffffu, rb, h);
+        out.xr = __uint_as_float(kXMark | (uint32_t)(8 * h + 31 - __clz(gh)));
+      }
+      a.gm[cbase / 8 + lane] = (uint8_t)gbyte;
+      if (lane == 0) a.agg[ch] = out;
+    }
+    return;
+  }
   for (int64_t gi = gw; gi < ngen; gi += nw) {
     const int64_t ch = (int64_t)a.gen_list[gi];
     const uint64_t cbase = (uint64_t)ch * kChunkW;
@@ -1182,6 +1245,7 @@ constexpr int64_t kMaxSmemBits = 227 * 1024;
 // F_A + F_B of the pass whose parent level is la.level (la.level = -1: the virtual root).
 dt_status level_agg_enqueue(const FitBufs& b, const LevelArgs& la, cudaStream_t s) {
   AggArgs a;
+  a.walk_gen = la.level < 0 || la.tails;
   a.lr = b.lr[la.cur];
   a.ly = b.ly[la.cur];
   a.lx = b.lx[la.cur];
