@@ -1202,11 +1202,13 @@ uint64_t g_plan_tick = 0;
 
 }  // namespace
 
+void forest_graph_release();
 dt_status release_workspace_impl() {
   {
     std::lock_guard<std::mutex> lk(g_plan_mu);
     for (auto& p : g_plans) p.reset();
   }
+  forest_graph_release();
   DT_CK(cudaDeviceSynchronize());
   int dev = 0;
   DT_CK(cudaGetDevice(&dev));
@@ -1445,6 +1447,30 @@ dt_status fit_grid_impl(const float* X, const double* y, int64_t n, int32_t d, i
 // Random Forest: ONE presort of the table; tree t = the exact CART of
 // its bootstrap sample, whose level-0 lists are the presorted lists expanded by the draw
 // counts (presort.cu, forest_tree_enqueue) -- no gather, no sort per tree.
+// The per-tree forest graph of the last forest on this host thread, with what it captured.
+struct ForestGraph {
+  FitBufs b{};
+  const void* p[9] = {};
+  int64_t n = 0, min_leaf = 0;
+  int32_t d = 0, max_depth = 0;
+  uint64_t seed = 0;
+  int y32 = 0, device = -1;
+  cudaGraphExec_t exec = nullptr;
+  int64_t launches = 0;
+  bool same(const ForestGraph& o) const {
+    return memcmp(&b, &o.b, sizeof(FitBufs)) == 0 && memcmp(p, o.p, sizeof(p)) == 0 && n == o.n &&
+           min_leaf == o.min_leaf && d == o.d && max_depth == o.max_depth && seed == o.seed && y32 == o.y32 &&
+           device == o.device;
+  }
+  void reset() {
+    if (exec) cudaGraphExecDestroy(exec);
+    exec = nullptr;
+  }
+  ~ForestGraph() { reset(); }
+};
+thread_local ForestGraph t_forest_graph;
+void forest_graph_release() { t_forest_graph.reset(); }
+
 dt_status forest_trees_impl(const float* X, const double* y, int64_t n, int32_t d, int32_t n_trees, int32_t max_depth,
                             int64_t min_leaf, uint64_t seed, cudaStream_t s, std::vector<dt_tree*>& trees) {
   int dev = 0;
@@ -1488,22 +1514,25 @@ dt_status forest_trees_impl(const float* X, const double* y, int64_t n, int32_t 
   st = alloc_status(ws.get(&tdev, 1));
   if (st != DT_OK) return st;
   // Bounded depth: one tree's sequence (pieces cleared, bootstrap expansion, level loop) is
-  // captured once as a CUDA graph and replayed per tree with the tree index set on the device.
+  // captured once as a CUDA graph and replayed per tree with the tree index set on the
+  // device.  The instantiated graph is kept (per host thread) and reused by the next forest
+  // whose buffers (stream-ordered pool: usually the same addresses) and shape match.
   const bool use_graph = !prof_enabled() && max_depth >= 0 && max_depth <= 24;
-  cudaGraphExec_t exec = nullptr;
-  cudaStream_t cap = nullptr;
-  struct Drop {
-    cudaGraphExec_t& e;
-    cudaStream_t& c;
-    ~Drop() {
-      if (e) cudaGraphExecDestroy(e);
-      if (c) cudaStreamDestroy(c);
-    }
-  } drop{exec, cap};
-  int64_t per_tree_launches = 0;
-  if (use_graph) {
+  ForestGraph& fg = t_forest_graph;
+  ForestGraph key;
+  key.b = b;
+  key.p[0] = X; key.p[1] = y; key.p[2] = sx; key.p[3] = sr; key.p[4] = sy; key.p[5] = w; key.p[6] = ys;
+  key.p[7] = tsum; key.p[8] = tdev;
+  key.n = n; key.d = d; key.max_depth = max_depth; key.min_leaf = min_leaf; key.seed = seed; key.y32 = hc.y32;
+  DT_CK(cudaGetDevice(&key.device));
+  if (use_graph && !(fg.exec && fg.same(key))) {
+    fg.reset();
+    cudaStream_t cap = nullptr;
     DT_CK(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
-    DT_CK(cudaStreamSynchronize(s));  // the workspace and copies above are complete
+    struct DropStream {
+      cudaStream_t c;
+      ~DropStream() { cudaStreamDestroy(c); }
+    } drop_cap{cap};
     const int64_t l0 = dt_launch_count();
     DT_CK(cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal));
     st = clear_pieces(b, cap);
@@ -1517,19 +1546,24 @@ dt_status forest_trees_impl(const float* X, const double* y, int64_t n, int32_t 
       return st;
     }
     if (ce != cudaSuccess) return cuda_fail(ce, "cudaStreamEndCapture", __FILE__, __LINE__);
-    per_tree_launches = dt_launch_count() - l0;
-    prof_add_launches(-per_tree_launches);  // counted per replay
+    const int64_t per_tree = dt_launch_count() - l0;
+    prof_add_launches(-per_tree);  // counted per replay
+    cudaGraphExec_t exec = nullptr;
     const cudaError_t ie = cudaGraphInstantiate(&exec, graph, 0);
     cudaGraphDestroy(graph);
     if (ie != cudaSuccess) return cuda_fail(ie, "cudaGraphInstantiate", __FILE__, __LINE__);
+    key.exec = exec;
+    key.launches = per_tree;
+    fg = key;
+    key.exec = nullptr;  // owned by the cache now
   }
   for (int32_t t = 0; t < n_trees; ++t) {
     set_u32_kernel<<<1, 1, 0, s>>>(tdev, (uint32_t)t);
     prof_add_launches(1);
     DT_CK(cudaGetLastError());
     if (use_graph) {
-      DT_CK(cudaGraphLaunch(exec, s));
-      prof_add_launches(per_tree_launches);
+      DT_CK(cudaGraphLaunch(fg.exec, s));
+      prof_add_launches(fg.launches);
     } else {
       st = clear_pieces(b, s);
       if (st == DT_OK)
