@@ -201,8 +201,8 @@ __global__ void __launch_bounds__(256) root_tables_kernel(const Ctl* __restrict_
 // Batched LSD radix sort of the d per-feature key lists (any n < 2^32): 4 passes
 // of 8-bit digits; per pass three launches, each over all d features (grid.y = feature):
 //   rs_count:   per-tile digit counts;
-//   rs_offset:  per (feature, digit) exclusive scan of the counts over the tiles, and the
-//               digit totals;
+//   rs_offset_warp: per (feature, digit) exclusive scan of the counts over the tiles, and
+//               the digit totals (a warp per scan);
 //   rs_scatter: every key's stable rank inside its tile (warp match_any per step of 32
 //               keys + per-warp digit counters; keys in tile order), then its destination
 //               = (keys of smaller digits) + (same digit, earlier tiles) + rank.
@@ -241,45 +241,31 @@ __global__ void __launch_bounds__(kTS) rs_count_kernel(const uint32_t* __restric
   cnt[((int64_t)f * 256 + threadIdx.x) * tiles + tile] = h[threadIdx.x];
 }
 
-// grid (256 digits, d features): exclusive prefix of one digit's counts over the tiles
-// (fixed shape; integers), and the digit's total.
-__global__ void __launch_bounds__(1024) rs_offset_kernel(const uint32_t* __restrict__ cnt, int tiles,
-                                                         uint32_t* __restrict__ off, uint32_t* __restrict__ tot) {
-  __shared__ uint32_t sw[32];
-  __shared__ uint32_t s_run;
-  const int64_t base = ((int64_t)blockIdx.y * 256 + blockIdx.x) * tiles;
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  if (threadIdx.x == 0) s_run = 0u;
-  __syncthreads();
-  for (int t0 = 0; t0 < tiles; t0 += blockDim.x) {
-    const int t = t0 + threadIdx.x;
-    const uint32_t c = (t < tiles) ? __ldg(cnt + base + t) : 0u;
+// Exclusive prefix of one (feature, digit)'s counts over the tiles, and the digit's total:
+// a warp per scan, 32 tiles per step (lane = tile), a warp inclusive scan plus the running
+// carry; the next step's counts are loaded before this step's scan (fixed shape; integers).
+__global__ void __launch_bounds__(256) rs_offset_warp_kernel(const uint32_t* __restrict__ cnt, int tiles, int nscan,
+                                                             uint32_t* __restrict__ off, uint32_t* __restrict__ tot) {
+  const int lane = threadIdx.x & 31;
+  const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (wid >= nscan) return;
+  const int64_t base = wid * tiles;  // scan wid = feature * 256 + digit
+  uint32_t run = 0u;
+  uint32_t c = lane < tiles ? __ldg(cnt + base + lane) : 0u;
+  for (int t0 = 0; t0 < tiles; t0 += 32) {
+    const int t = t0 + lane, tn = t + 32;
+    const uint32_t cn = tn < tiles ? __ldg(cnt + base + tn) : 0u;  // next step in flight
     uint32_t inc = c;
 #pragma unroll
     for (int dd = 1; dd < 32; dd <<= 1) {
       const uint32_t o = __shfl_up_sync(0xffffffffu, inc, dd);
       if (lane >= dd) inc += o;
     }
-    if (lane == 31) sw[w] = inc;
-    __syncthreads();
-    if (w == 0) {
-      const uint32_t v = (lane < (int)(blockDim.x >> 5)) ? sw[lane] : 0u;
-      uint32_t vi = v;
-#pragma unroll
-      for (int dd = 1; dd < 32; dd <<= 1) {
-        const uint32_t o = __shfl_up_sync(0xffffffffu, vi, dd);
-        if (lane >= dd) vi += o;
-      }
-      sw[lane] = vi - v;  // exclusive prefix of the warp totals
-    }
-    __syncthreads();
-    const uint32_t run = s_run;
-    if (t < tiles) off[base + t] = run + sw[w] + inc - c;
-    __syncthreads();
-    if (threadIdx.x == blockDim.x - 1) s_run = run + sw[w] + inc;
-    __syncthreads();
+    if (t < tiles) off[base + t] = run + inc - c;
+    run += __shfl_sync(0xffffffffu, inc, 31);
+    c = cn;
   }
-  if (threadIdx.x == 0) tot[(int64_t)blockIdx.y * 256 + blockIdx.x] = s_run;
+  if (lane == 0) tot[wid] = run;
 }
 
 #ifndef DT_RS_MINB
@@ -653,8 +639,8 @@ void radix_sort_lists(const FitBufs& b, int64_t n, int d, cudaStream_t s, const 
     const bool fx = X != nullptr && pass == 0, tl = y != nullptr && pass == 3;
     if (fx) rs_count_kernel<true><<<g, kTS, 0, s>>>(ki, X, n, d, shift, tiles, b.rs_cnt, b.ctl);
     else rs_count_kernel<false><<<g, kTS, 0, s>>>(ki, X, n, d, shift, tiles, b.rs_cnt, b.ctl);
-    rs_offset_kernel<<<dim3(256, (unsigned)d), std::min(1024, (tiles + 31) / 32 * 32), 0, s>>>(b.rs_cnt, tiles,
-                                                                                            b.rs_off, b.rs_tot);
+    rs_offset_warp_kernel<<<(unsigned)((256 * d + 7) / 8), 256, 0, s>>>(b.rs_cnt, tiles, 256 * d, b.rs_off,
+                                                                         b.rs_tot);
     RsOut o{ko, vo, b.lx[0], b.lr[0], b.ly[0], y, row0, b.ctl};
     if (fx) rs_scatter_kernel<true, false><<<g, kTS, 0, s>>>(ki, vi, X, d, o, n, shift, tiles, b.rs_off, b.rs_tot);
     else if (tl) rs_scatter_kernel<false, true><<<g, kTS, 0, s>>>(ki, vi, X, d, o, n, shift, tiles, b.rs_off, b.rs_tot);

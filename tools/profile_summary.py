@@ -22,7 +22,7 @@ KIND = {
     "piece_pos_kernel": "select", "select_kernel": "select",
     "number_kernel": "number", "children_kernel": "number", "tables_kernel": "number",
     "goleft_kernel": "goleft",
-    "rs_count_kernel": "presort_sort", "rs_offset_kernel": "presort_sort", "rs_scatter_kernel": "presort_sort",
+    "rs_count_kernel": "presort_sort", "rs_offset_kernel": "presort_sort", "rs_offset_warp_kernel": "presort_sort", "rs_scatter_kernel": "presort_sort",
     "root_reduce_kernel": "root_stats", "root_finalize_kernel": "root_stats", "root_center_kernel": "root_stats",
     "root_init_kernel": "root_stats", "root_tables_kernel": "presort_build",
     "predict_col_kernel": "predict", "eval_partial_kernel": "eval", "eval_final_kernel": "eval",
