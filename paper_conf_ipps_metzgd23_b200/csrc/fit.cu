@@ -368,8 +368,9 @@ __global__ void __launch_bounds__(1024) number_kernel(NumberArgs a) {
     const uint32_t k = k0 + tid;
     const bool in = k < K;
     const Decision dc = in ? a.dec[k] : Decision{-1, 0, 0, 0, 0.0, 0.0};
+    const uint32_t nN = in ? a.nodes[k].N : 0u;  // loaded beside the decision (no dependent load)
     const bool sp = in && dc.f >= 0;
-    const uint32_t nl = sp ? dc.nl : 0u, nr = sp ? a.nodes[k].N - dc.nl : 0u;
+    const uint32_t nl = sp ? dc.nl : 0u, nr = sp ? nN - dc.nl : 0u;
     const bool sl_ok = sp && depth_ok && (int64_t)nl >= 2 * a.min_leaf;
     const bool sr_ok = sp && depth_ok && (int64_t)nr >= 2 * a.min_leaf;
     // three exclusive scans over the block: splits, written rows, searchable children
@@ -436,14 +437,15 @@ __global__ void __launch_bounds__(256) children_kernel(NumberArgs a) {
   const int child_depth = a.level + 1;
   const bool depth_ok = (a.max_depth < 0) || (child_depth < a.max_depth);
   for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < K; k += gridDim.x * blockDim.x) {
+    // the decision, the node and its row offset loaded together (no dependent loads)
     const Decision dc = a.dec[k];
-    if (dc.f < 0) continue;
     const NodeL nd = a.nodes[k];
+    const unsigned long long rows_ex = a.wst[k];
+    if (dc.f < 0) continue;
     const uint32_t rank = dc.kid >> 1;
     const uint32_t nl = dc.nl, nr = nd.N - dc.nl;
     const bool sl_ok = depth_ok && (int64_t)nl >= 2 * a.min_leaf;
     const bool sr_ok = depth_ok && (int64_t)nr >= 2 * a.min_leaf;
-    const unsigned long long rows_ex = a.wst[k];
     const int lid = next_id0 + 2 * (int)rank;
     a.out[nd.id].left = lid;
     a.out[nd.id].right = lid + 1;
