@@ -207,7 +207,12 @@ __global__ void __launch_bounds__(256) root_tables_kernel(const Ctl* __restrict_
 //               keys + per-warp digit counters; keys in tile order), then its destination
 //               = (keys of smaller digits) + (same digit, earlier tiles) + rank.
 // Stable within a feature, so equal keys keep the row order: (x, row id) order (R6).
-constexpr int kTS = 256, kTI = 8, kTile = kTS * kTI;
+#ifndef DT_RS_WARPS
+#define DT_RS_WARPS 12  // warps per scatter tile (256 keys each): 3072-key tiles (8 warps: 2% slower presort)
+#endif
+constexpr int kTS = 256, kTI = 8;                    // count: threads per block; keys per scatter thread
+constexpr int kSTS = 32 * DT_RS_WARPS;               // scatter: threads per block
+constexpr int kTile = kSTS * kTI;                    // keys per tile (count and scatter)
 
 // Source of a pass's keys: the key lists, or (first pass, kFromX) X itself: key =
 // flip(X[r][f]), value = row0 + r (the table's columns read in place; the d blocks of a
@@ -269,7 +274,7 @@ __global__ void __launch_bounds__(256) rs_offset_warp_kernel(const uint32_t* __r
 }
 
 #ifndef DT_RS_MINB
-#define DT_RS_MINB 4  // 4 CTAs/SM (64 registers): more tiles in flight (measured 4.04 -> 3.95 ms/step)
+#define DT_RS_MINB 3  // CTAs/SM of the scatter: 3 x 384 threads (2: 14% slower presort)
 #endif
 // kToLists (last pass): the sorted pairs go straight into the level-0 lists: x =
 // unflip(key), row = value, y = y[row - row0] (int32 when the fit stores y so, R24).
@@ -284,15 +289,15 @@ struct RsOut {
   const Ctl* ctl;
 };
 template <bool kFromX, bool kToLists>
-__global__ void __launch_bounds__(kTS, DT_RS_MINB) rs_scatter_kernel(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ vin,
+__global__ void __launch_bounds__(kSTS, DT_RS_MINB) rs_scatter_kernel(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ vin,
                                                          const float* __restrict__ X, int d, RsOut o,
                                                          int64_t n, int shift, int tiles, const uint32_t* __restrict__ off,
                                                          const uint32_t* __restrict__ tot) {
-  __shared__ uint32_t wc[kTS / 32][256];  // per-warp digit counters -> per-warp prefixes
+  __shared__ uint32_t wc[kSTS / 32][256];  // per-warp digit counters -> per-warp prefixes
   __shared__ uint32_t s_base[256];        // digit base of this tile: smaller digits + earlier tiles
   __shared__ uint32_t s_start[256];       // digit starts inside the tile
   __shared__ uint32_t skey[kTile], sval[kTile];
-  __shared__ uint32_t sw[kTS / 32], sw2[kTS / 32];
+  __shared__ uint32_t sw[8], sw2[8];       // digit scans: 256 digits = 8 warps
   const int f = (int)(blockIdx.x % (unsigned)d), tile = (int)(blockIdx.x / (unsigned)d);
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int64_t tbase = (int64_t)tile * kTile;
@@ -324,35 +329,39 @@ __global__ void __launch_bounds__(kTS, DT_RS_MINB) rs_scatter_kernel(const uint3
   // thread = digit: exclusive prefix over the warps, the tile's digit starts (exclusive
   // scan of its digit counts) and the digit's global base for this tile
   {
-    const int dgt = threadIdx.x;
-    uint32_t run = 0u;
+    const int dgt = threadIdx.x;  // threads 0..255: one digit each
+    uint32_t run = 0u, inc = 0u, t = 0u, tinc = 0u;
+    if (dgt < 256) {
 #pragma unroll
-    for (int q = 0; q < kTS / 32; ++q) {
-      const uint32_t c = wc[q][dgt];
-      wc[q][dgt] = run;
-      run += c;
-    }
-    uint32_t inc = run;  // tile count of this digit
+      for (int q = 0; q < kSTS / 32; ++q) {
+        const uint32_t c = wc[q][dgt];
+        wc[q][dgt] = run;
+        run += c;
+      }
+      inc = run;  // tile count of this digit
 #pragma unroll
-    for (int dd = 1; dd < 32; dd <<= 1) {
-      const uint32_t o = __shfl_up_sync(0xffffffffu, inc, dd);
-      if (lane >= dd) inc += o;
-    }
-    if (lane == 31) sw[w] = inc;
-    // exclusive prefix of the digit totals of this feature
-    const uint32_t t = __ldg(tot + (int64_t)f * 256 + dgt);
-    uint32_t tinc = t;
+      for (int dd = 1; dd < 32; dd <<= 1) {
+        const uint32_t o = __shfl_up_sync(0xffffffffu, inc, dd);
+        if (lane >= dd) inc += o;
+      }
+      if (lane == 31) sw[w] = inc;
+      // exclusive prefix of the digit totals of this feature
+      t = __ldg(tot + (int64_t)f * 256 + dgt);
+      tinc = t;
 #pragma unroll
-    for (int dd = 1; dd < 32; dd <<= 1) {
-      const uint32_t o = __shfl_up_sync(0xffffffffu, tinc, dd);
-      if (lane >= dd) tinc += o;
+      for (int dd = 1; dd < 32; dd <<= 1) {
+        const uint32_t o = __shfl_up_sync(0xffffffffu, tinc, dd);
+        if (lane >= dd) tinc += o;
+      }
+      if (lane == 31) sw2[w] = tinc;
     }
-    if (lane == 31) sw2[w] = tinc;
     __syncthreads();
-    uint32_t wp = 0u, wp2 = 0u;
-    for (int q = 0; q < w; ++q) { wp += sw[q]; wp2 += sw2[q]; }
-    s_start[dgt] = wp + inc - run;
-    s_base[dgt] = wp2 + tinc - t + __ldg(off + ((int64_t)f * 256 + dgt) * tiles + tile);
+    if (dgt < 256) {
+      uint32_t wp = 0u, wp2 = 0u;
+      for (int q = 0; q < w; ++q) { wp += sw[q]; wp2 += sw2[q]; }
+      s_start[dgt] = wp + inc - run;
+      s_base[dgt] = wp2 + tinc - t + __ldg(off + ((int64_t)f * 256 + dgt) * tiles + tile);
+    }
   }
   __syncthreads();
   // local (tile-sorted) order in shared memory, then coalesced runs to global memory
@@ -368,7 +377,7 @@ __global__ void __launch_bounds__(kTS, DT_RS_MINB) rs_scatter_kernel(const uint3
   }
   __syncthreads();
   const bool y32 = kToLists && o.ctl->y32 != 0;
-  for (int i = threadIdx.x; i < m; i += kTS) {
+  for (int i = threadIdx.x; i < m; i += kSTS) {
     const uint32_t key = skey[i];
     const uint32_t dg = (key >> shift) & 255u;
     const int64_t dst = (int64_t)f * n + s_base[dg] + ((uint32_t)i - s_start[dg]);
@@ -642,9 +651,9 @@ void radix_sort_lists(const FitBufs& b, int64_t n, int d, cudaStream_t s, const 
     rs_offset_warp_kernel<<<(unsigned)((256 * d + 7) / 8), 256, 0, s>>>(b.rs_cnt, tiles, 256 * d, b.rs_off,
                                                                          b.rs_tot);
     RsOut o{ko, vo, b.lx[0], b.lr[0], b.ly[0], y, row0, b.ctl};
-    if (fx) rs_scatter_kernel<true, false><<<g, kTS, 0, s>>>(ki, vi, X, d, o, n, shift, tiles, b.rs_off, b.rs_tot);
-    else if (tl) rs_scatter_kernel<false, true><<<g, kTS, 0, s>>>(ki, vi, X, d, o, n, shift, tiles, b.rs_off, b.rs_tot);
-    else rs_scatter_kernel<false, false><<<g, kTS, 0, s>>>(ki, vi, X, d, o, n, shift, tiles, b.rs_off, b.rs_tot);
+    if (fx) rs_scatter_kernel<true, false><<<g, kSTS, 0, s>>>(ki, vi, X, d, o, n, shift, tiles, b.rs_off, b.rs_tot);
+    else if (tl) rs_scatter_kernel<false, true><<<g, kSTS, 0, s>>>(ki, vi, X, d, o, n, shift, tiles, b.rs_off, b.rs_tot);
+    else rs_scatter_kernel<false, false><<<g, kSTS, 0, s>>>(ki, vi, X, d, o, n, shift, tiles, b.rs_off, b.rs_tot);
     std::swap(ki, ko);
     std::swap(vi, vo);
   }
