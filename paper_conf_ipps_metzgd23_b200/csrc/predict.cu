@@ -978,8 +978,9 @@ dt_status eval_impl(const double* y, const double* yhat, const float* X, const d
     cudaFreeAsync(tmp, s);
     return st;
   }
-  // Fixed partition of [0, n) into nparts chunks (deterministic for a given n).
-  int64_t chunk = 4096;
+  // Fixed partition of [0, n) into nparts chunks (deterministic for a given n); 1024 rows
+  // per 256-thread block: 4 rows per thread, enough blocks to fill the SMs at 1M rows
+  int64_t chunk = 1024;
   int64_t nparts = (n + chunk - 1) / chunk;
   if (nparts > 4096) {
     nparts = 4096;
