@@ -1021,7 +1021,7 @@ dt_status eval_impl(const double* y, const double* yhat, const float* X, const d
 dt_status eval_sharded_impl(dt_comm* comm, const double* y, const double* yhat, int64_t n, int32_t p,
                             cudaStream_t s, dt_metrics* out) {
   const int world = comm_world(comm);
-  int64_t chunk = 4096;
+  int64_t chunk = 1024;  // the partition of eval_impl: one rank reproduces dt_eval bitwise
   int64_t nparts = n > 0 ? (n + chunk - 1) / chunk : 0;
   if (nparts > 4096) {
     nparts = 4096;
